@@ -1,0 +1,182 @@
+"""ctypes wrapper of liboracle.so -- TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference legs may import
+this module.  It shares nothing with the CUDA path except the seeded input generators
+(paper_conf_ipps_adamsbkw22_b200/inputs.py, which hold no method arithmetic).
+See oracle.h for what each call computes and which passage of the paper it follows.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB = None
+
+_d = np.ctypeslib.ndpointer(dtype=np.float64, flags="C_CONTIGUOUS")
+_i64 = np.ctypeslib.ndpointer(dtype=np.int64, flags="C_CONTIGUOUS")
+_i32 = np.ctypeslib.ndpointer(dtype=np.int32, flags="C_CONTIGUOUS")
+_u8 = np.ctypeslib.ndpointer(dtype=np.uint8, flags="C_CONTIGUOUS")
+
+
+def build():
+    subprocess.run(["make", "-s", "-C", _HERE], check=True)
+
+
+def lib():
+    global _LIB
+    if _LIB is None:
+        path = os.path.join(_HERE, "liboracle.so")
+        if not os.path.exists(path):
+            build()
+        L = C.CDLL(path)
+        vp = C.c_void_p
+        L.oracle_create.restype = vp
+        L.oracle_create.argtypes = [C.c_int, _i64, _d, _d, C.c_int, C.c_int, C.c_int, _d, _d, _i32,
+                                    C.c_double, C.c_char_p, C.c_int]
+        L.oracle_destroy.argtypes = [vp]
+        P64 = C.POINTER(C.c_longlong)
+        L.oracle_sizes.argtypes = [vp, P64, P64, P64, P64]
+        L.oracle_grid_ndof.restype = C.c_longlong
+        L.oracle_grid_ndof.argtypes = [vp, C.c_int]
+        L.oracle_grid_npoints.restype = C.c_longlong
+        L.oracle_grid_npoints.argtypes = [vp, C.c_int]
+        L.oracle_grid_nodes.argtypes = [vp, C.c_int, _d, _d]
+        L.oracle_points.argtypes = [vp, _d, _d, _d]
+        L.oracle_pattern.argtypes = [vp, _i64, _i32]
+        L.oracle_coo_pattern.argtypes = [vp, _i32, _i32]
+        L.oracle_tensor.argtypes = [C.c_double, C.c_double, C.c_double, C.c_double, _d]
+        L.oracle_inner.argtypes = [C.c_longlong, _d, _d, _d, _d, _d, _d, C.c_longlong, vp, vp, vp]
+        L.oracle_point_fields.argtypes = [vp, _d, _d, _d, _d]
+        L.oracle_point_coeffs.argtypes = [vp, _d, C.c_longlong, vp, vp, vp]
+        L.oracle_jacobian.argtypes = [vp, _d, _d, _d]
+        L.oracle_jacobian_coo.argtypes = [vp, _d, vp, _d, _d]
+        L.oracle_mass.argtypes = [vp, C.c_double, _d]
+        L.oracle_mass_coo.argtypes = [vp, C.c_double, _d]
+        L.oracle_set_threads.argtypes = [C.c_int]
+        L.oracle_get_threads.restype = C.c_int
+        _LIB = L
+    return _LIB
+
+
+def _ptr(a):
+    return None if a is None else a.ctypes.data_as(C.c_void_p)
+
+
+def tensor(r, z, rb, zb):
+    out = np.zeros(5)
+    lib().oracle_tensor(float(r), float(z), float(rb), float(zb), out)
+    return out
+
+
+def inner(r, z, w, TD, TKr, TKz, targets=None, with_abs=False):
+    r, z, w, TD, TKr, TKz = (np.ascontiguousarray(a, dtype=np.float64) for a in (r, z, w, TD, TKr, TKz))
+    n = r.size
+    tg = None if targets is None else np.ascontiguousarray(targets, dtype=np.int64)
+    nt = n if tg is None else tg.size
+    G = np.zeros((5, nt))
+    Ga = np.zeros((5, nt)) if with_abs else None
+    lib().oracle_inner(n, r, z, w, TD, TKr, TKz, nt, _ptr(tg), _ptr(G), _ptr(Ga))
+    return (G, Ga) if with_abs else G
+
+
+def set_threads(n):
+    lib().oracle_set_threads(int(n))
+
+
+def get_threads():
+    return int(lib().oracle_get_threads())
+
+
+class Oracle:
+    """The whole O0-O10 pipeline for one Problem (paper_conf_ipps_adamsbkw22_b200.inputs.Problem)."""
+
+    def __init__(self, prob, nq1d: int = 0):
+        L = lib()
+        err = C.create_string_buffer(256)
+        self.prob = prob
+        self._h = L.oracle_create(len(prob.grids), prob.ncells, prob.cells, prob.radius, prob.order, nq1d,
+                                  len(prob.species), prob.mass, prob.charge, prob.grid_of, prob.nu, err, 256)
+        if not self._h:
+            raise ValueError("oracle_create: " + err.value.decode())
+        a, b, c, d = (C.c_longlong() for _ in range(4))
+        L.oracle_sizes(self._h, C.byref(a), C.byref(b), C.byref(c), C.byref(d))
+        self.ndof, self.npoints, self.nnz, self.ncoo = a.value, b.value, c.value, d.value
+
+    def __del__(self):
+        if getattr(self, "_h", None) and _LIB is not None:
+            _LIB.oracle_destroy(self._h)
+            self._h = None
+
+    def grid_ndof(self, g):
+        return int(lib().oracle_grid_ndof(self._h, g))
+
+    def nodes(self, g):
+        n = self.grid_ndof(g)
+        r, z = np.zeros(n), np.zeros(n)
+        lib().oracle_grid_nodes(self._h, g, r, z)
+        return r, z
+
+    def all_nodes(self):
+        return [self.nodes(g) for g in range(len(self.prob.grids))]
+
+    def points(self):
+        r, z, w = (np.zeros(self.npoints) for _ in range(3))
+        lib().oracle_points(self._h, r, z, w)
+        return r, z, w
+
+    def pattern(self):
+        rp = np.zeros(self.ndof + 1, dtype=np.int64)
+        col = np.zeros(max(self.nnz, 1), dtype=np.int32)
+        lib().oracle_pattern(self._h, rp, col)
+        return rp, col[: self.nnz]
+
+    def coo_pattern(self):
+        row = np.zeros(max(self.ncoo, 1), dtype=np.int32)
+        col = np.zeros(max(self.ncoo, 1), dtype=np.int32)
+        lib().oracle_coo_pattern(self._h, row, col)
+        return row[: self.ncoo], col[: self.ncoo]
+
+    def point_fields(self, f):
+        f = np.ascontiguousarray(f, dtype=np.float64)
+        TD, TKr, TKz = (np.zeros(self.npoints) for _ in range(3))
+        lib().oracle_point_fields(self._h, f, TD, TKr, TKz)
+        return TD, TKr, TKz
+
+    def point_coeffs(self, f, targets=None):
+        f = np.ascontiguousarray(f, dtype=np.float64)
+        tg = None if targets is None else np.ascontiguousarray(targets, dtype=np.int64)
+        nt = self.npoints if tg is None else tg.size
+        G, Ga = np.zeros((5, nt)), np.zeros((5, nt))
+        lib().oracle_point_coeffs(self._h, f, nt, _ptr(tg), _ptr(G), _ptr(Ga))
+        return G, Ga
+
+    def jacobian(self, f):
+        f = np.ascontiguousarray(f, dtype=np.float64)
+        v, va = np.zeros(max(self.nnz, 1)), np.zeros(max(self.nnz, 1))
+        lib().oracle_jacobian(self._h, f, v, va)
+        return v[: self.nnz], va[: self.nnz]
+
+    def jacobian_coo(self, f, elem_mask=None):
+        f = np.ascontiguousarray(f, dtype=np.float64)
+        m = None if elem_mask is None else np.ascontiguousarray(elem_mask, dtype=np.uint8)
+        v, va = np.full(max(self.ncoo, 1), np.nan), np.full(max(self.ncoo, 1), np.nan)
+        lib().oracle_jacobian_coo(self._h, f, _ptr(m), v, va)
+        return v[: self.ncoo], va[: self.ncoo]
+
+    def mass(self, shift=1.0):
+        v = np.zeros(max(self.nnz, 1))
+        lib().oracle_mass(self._h, float(shift), v)
+        return v[: self.nnz]
+
+    def mass_coo(self, shift=1.0):
+        v = np.zeros(max(self.ncoo, 1))
+        lib().oracle_mass_coo(self._h, float(shift), v)
+        return v[: self.ncoo]
+
+    def coefficients(self, with_noise=True):
+        from paper_conf_ipps_adamsbkw22_b200 import inputs
+        return inputs.coefficients(self.prob, self.all_nodes(), with_noise)

@@ -1,0 +1,206 @@
+"""Pins P3, P4, P5, P9 and the paper's Maxwellian-energy statement for the oracle.
+
+P3: C(f_M, f_M) = 0 at every quadrature point for Maxwellians of a common T and drift, any masses
+    (continuum statement behind PAPER.md:1@2223 'conserves ... exactly'; discrete via P2).
+P4: density, parallel momentum and energy conservation of the assembled Jacobian (@2223, [3],[4]),
+    with the negative control that per-species momentum is NOT conserved.
+P5: normalisation (2 pi, r weights, U scale): the inner integral of a Maxwellian converges at O(h^2)
+    to the closed-form Rosenbluth potentials D = grad grad g, K = 2 grad h.
+P9: the whole O3-O5 pipeline on C1 against an independent azimuthal quadrature of Eq. 3 for every pair.
+Energy: 'resolves the total energy of the Maxwellian with about five digits' (@27330, mesh A, Q3).
+"""
+import json
+import math
+import os
+
+import mpmath as mp
+import numpy as np
+import pytest
+
+from oracle.oracle import Oracle, inner
+from paper_conf_ipps_adamsbkw22_b200 import inputs
+from tests._brute import tensors_quadrature
+
+GOLD = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "paper_counts.json")))
+
+
+def test_p3_maxwellian_null_pointwise():
+    prob = inputs.config2()
+    o = Oracle(prob)
+    r, z, w = o.points()
+    T, u = 0.3, 0.17
+    sp = prob.species
+    f = [inputs.maxwellian(r, z, 1.0 + a, T, s.mass, u) for a, s in enumerate(sp)]
+    g = [inputs.maxwellian_grad(r, z, 1.0 + a, T, s.mass, u) for a, s in enumerate(sp)]
+    TD = sum(s.charge ** 2 * f[a] for a, s in enumerate(sp))
+    TKr = sum(s.charge ** 2 / s.mass * g[a][0] for a, s in enumerate(sp))
+    TKz = sum(s.charge ** 2 / s.mass * g[a][1] for a, s in enumerate(sp))
+    G, Ga = inner(r, z, w, TD, TKr, TKz, with_abs=True)
+    for a, s in enumerate(sp):
+        fr, fz = g[a]
+        # bracket of Eqs. 5-6 up to nu e_a^2 (m0/m_a): -(m0/m_a) G_D.grad f_a + G_K f_a
+        flux_r = -(G[0] * fr + G[1] * fz) / s.mass + G[3] * f[a]
+        flux_z = -(G[1] * fr + G[2] * fz) / s.mass + G[4] * f[a]
+        scale_r = (Ga[0] * abs(fr) + Ga[1] * abs(fz)) / s.mass + Ga[3] * f[a]
+        scale_z = (Ga[1] * abs(fr) + Ga[2] * abs(fz)) / s.mass + Ga[4] * f[a]
+        m = scale_r > 0
+        assert np.max(np.abs(flux_r[m]) / scale_r[m]) < 1e-13
+        m = scale_z > 0
+        assert np.max(np.abs(flux_z[m]) / scale_z[m]) < 1e-13
+    # negative control: different temperatures do not give a null
+    f2 = inputs.maxwellian(r, z, 1.0, 2 * T, sp[1].mass, u)
+    flux = -(G[1] * inputs.maxwellian_grad(r, z, 1.0, 2 * T, sp[1].mass, u)[0]) / sp[1].mass + G[4] * f2
+    assert np.max(np.abs(flux)) > 1e-6 * np.max(np.abs(G[4] * f2))
+
+
+def _csr_dense_rows(o):
+    rp, col = o.pattern()
+    return np.repeat(np.arange(o.ndof), np.diff(rp)), col
+
+
+def _moments(prob, o, J, Ja, f):
+    """(density per species, momentum total, energy total, per-species momentum) residuals, normalised."""
+    row, col = _csr_dense_rows(o)
+    nodes = o.all_nodes()
+    out = {"density": [], "mom_species": []}
+    tot = {"mom": 0.0, "mom_s": 0.0, "en": 0.0, "en_s": 0.0}
+    start = 0
+    for a, s in enumerate(prob.species):
+        nd = o.grid_ndof(s.grid)
+        sel = (row >= start) & (row < start + nd)
+        rr, cc = row[sel] - start, col[sel] - start
+        Jv, Jav = J[sel], Ja[sel]
+        fa = f[start:start + nd]
+        Jf = np.bincount(rr, Jv * fa[cc], minlength=nd)
+        Jaf = np.bincount(rr, Jav * np.abs(fa[cc]), minlength=nd)
+        nr, nz = nodes[s.grid]
+        one = np.ones(nd)
+        out["density"].append(abs(one @ Jf) / (one @ Jaf))
+        mom, moms = s.mass * (nz @ Jf), s.mass * (np.abs(nz) @ Jaf)
+        en, ens = s.mass * ((nr ** 2 + nz ** 2) @ Jf), s.mass * ((nr ** 2 + nz ** 2) @ Jaf)
+        out["mom_species"].append(abs(mom) / moms)
+        tot["mom"] += mom
+        tot["mom_s"] += moms
+        tot["en"] += en
+        tot["en_s"] += ens
+        start += nd
+    out["momentum"] = abs(tot["mom"]) / tot["mom_s"]
+    out["energy"] = abs(tot["en"]) / tot["en_s"]
+    return out
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3"])
+def test_p4_conservation(cfg):
+    prob = inputs.CONFIGS[cfg]()
+    o = Oracle(prob)
+    f = o.coefficients()
+    J, Ja = o.jacobian(f)
+    m = _moments(prob, o, J, Ja, f)
+    assert max(m["density"]) < 1e-13, m
+    assert m["momentum"] < 1e-13, m
+    assert m["energy"] < 1e-13, m
+    if cfg == "C2":
+        # negative control: e-D momentum exchange is real, only the total is conserved
+        assert min(m["mom_species"]) > 1e-6, m
+
+
+def test_p4_coo_assembles_to_csr():
+    prob = inputs.config2()
+    o = Oracle(prob)
+    f = o.coefficients()
+    J, _ = o.jacobian(f)
+    Jc, _ = o.jacobian_coo(f)
+    row, col = o.coo_pattern()
+    rp, ccol = o.pattern()
+    import scipy.sparse as sps
+    A = sps.coo_matrix((Jc, (row, col)), shape=(o.ndof, o.ndof)).tocsr()
+    A.sort_indices()
+    B = sps.csr_matrix((J, ccol, rp), shape=(o.ndof, o.ndof))
+    assert abs(A - B).max() <= 1e-14 * abs(B).max()
+
+
+def _rosenbluth(r, z, T, m):
+    """Exact D = grad grad g, K = 2 grad h of f = (pi th)^-3/2 exp(-v^2/th), via mpmath derivatives."""
+    vt = mp.sqrt(mp.mpf(inputs.theta(T, m)))
+
+    def g(x, y):
+        v = mp.sqrt(x * x + y * y)
+        s = v / vt
+        return vt * ((s + 1 / (2 * s)) * mp.erf(s) + mp.exp(-s * s) / mp.sqrt(mp.pi))
+
+    def h(x, y):
+        v = mp.sqrt(x * x + y * y)
+        return mp.erf(v / vt) / v
+
+    mp.mp.dps = 25
+    out = []
+    for x, y in zip(r, z):
+        out.append([float(mp.diff(g, (x, y), (2, 0))), float(mp.diff(g, (x, y), (1, 1))),
+                    float(mp.diff(g, (x, y), (0, 2))), float(2 * mp.diff(h, (x, y), (1, 0))),
+                    float(2 * mp.diff(h, (x, y), (0, 1)))])
+    return np.array(out).T
+
+
+def test_p5_rosenbluth_normalisation_converges_h2():
+    T, m = 1.0, 1.0
+    R = inputs.R_E
+    rng = np.random.default_rng(3)
+    tr = rng.uniform(0.2, 2.5, 24)
+    tz = rng.uniform(-2.5, 2.5, 24)
+    exact = _rosenbluth(tr, tz, T, m)
+    errs = []
+    for ref in range(3):
+        cells = inputs.refine_uniform(inputs.origin_chain(R, 3), ref)
+        o = Oracle(inputs.Problem("p5", 3, [(R, cells)], [inputs.Species("e", 1.0, 1.0, 0)],
+                                  fmix=[[(1.0, T, 0.0)]]))
+        r, z, w = o.points()
+        f = inputs.maxwellian(r, z, 1.0, T, m)
+        fr, fz = inputs.maxwellian_grad(r, z, 1.0, T, m)
+        # targets appended with zero weight (they are not sources)
+        R_ = np.concatenate([r, tr])
+        Z_ = np.concatenate([z, tz])
+        W_ = np.concatenate([w, np.zeros_like(tr)])
+        G = inner(R_, Z_, W_, np.concatenate([f, 0 * tr]), np.concatenate([fr, 0 * tr]),
+                  np.concatenate([fz, 0 * tr]), targets=np.arange(r.size, r.size + tr.size))
+        errs.append(np.abs(G - exact).max() / np.abs(exact).max())
+    # a 2 pi or r-weight slip would leave an O(1) error; O(h^2) over two halvings gives ~16x
+    # (the log-singular kernel near targets that fall close to a source point makes single steps noisy)
+    assert errs[2] < 2e-3, errs
+    assert errs[0] > errs[1] > errs[2] and errs[0] / errs[2] > 10.0, errs
+
+
+def test_p9_pipeline_vs_bruteforce_quadrature_C1():
+    prob = inputs.config1()
+    o = Oracle(prob)
+    f = o.coefficients()
+    TD, TKr, TKz = o.point_fields(f)
+    r, z, w = o.points()
+    N = r.size
+    ii, jj = np.meshgrid(np.arange(N), np.arange(N), indexing="ij")
+    ii, jj = ii.ravel(), jj.ravel()
+    keep = ~((r[ii] == r[jj]) & (z[ii] == z[jj]))
+    ii, jj = ii[keep], jj[keep]
+    U = tensors_quadrature(r[ii], z[ii], r[jj], z[jj])
+    wd, wkr, wkz = w[jj] * TD[jj], w[jj] * TKr[jj], w[jj] * TKz[jj]
+    comps = [wd * U[0], wd * U[1], wd * U[2], U[3] * wkr + U[1] * wkz, U[4] * wkr + U[2] * wkz]
+    Gb = np.stack([np.array([math.fsum(c[ii == i]) for i in range(N)]) for c in comps])
+    G, Ga = o.point_coeffs(f)
+    assert np.max(np.abs(G - Gb) / Ga) < 1e-13
+
+
+def test_maxwellian_energy_five_digits_mesh_A():
+    """Mesh A + Q3 Gauss points resolve the Maxwellian's total energy to about five digits (@27330,
+    Fig. 3: 20 cells, domain 5 v_th).  2 pi sum_q w_q f(q) v_q^2 against the exact 3 theta / 2 pins
+    the point placement, the r-weighted quadrature and the 2 pi of Eq. 4 (Amb-2)."""
+    R = inputs.R_E
+    prob = inputs.Problem("A", 3, [(R, inputs.origin_chain(R, 3))], [inputs.Species("e", 1.0, 1.0, 0)],
+                          fmix=[[(1.0, 1.0, 0.0)]], noise=0.0)
+    o = Oracle(prob)
+    r, z, w = o.points()
+    f = inputs.maxwellian(r, z, 1.0, 1.0, 1.0)
+    energy = 2 * np.pi * np.sum(w * f * (r ** 2 + z ** 2))
+    exact = 1.5 * inputs.theta(1.0, 1.0)
+    digits = -math.log10(abs(energy / exact - 1))
+    assert abs(digits - GOLD["maxwellian_energy_digits"]["value"]) <= 0.5, digits
+    density = 2 * np.pi * np.sum(w * f)
+    assert abs(density - 1) < 1e-4
