@@ -1,0 +1,313 @@
+#!/usr/bin/env python3
+"""Benchmark of the Landau Jacobian hot path on B200 (contract: see DESIGN.md §Measurement).
+
+Workload (default, BASELINE.json configs[3] built on configs[1]): a batch of 1024 independent
+spatial-vertex velocity grids, each the e + D Q3 AMR C2 grid (68 cells, N = 1,088 points, 601 DOFs
+per species) with its own thermal-quench-shaped f; the batch is split evenly over the ranks with no
+communication (1024 / world vertices per GPU: strong scaling of a fixed job).
+
+One step = the whole hot path (SURVEY.md §8(a) a-1 .. a-6) for the local batch:
+    landau_set_state_batched -> landau_jacobian_batched (CSR) -> landau_mass (CSR)
+with the inputs already resident in HBM.  L2 (126 MB) is flushed between timed steps by writing a
+256 MiB buffer outside the timed events.  e2e repeats the step through landau_jacobian_host with
+pinned host buffers (H2D of f and D2H of every Jacobian value inside the timed region).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl landau|reference] [--workload C4|C2|C3|C5]
+"""
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "Landau Jacobian builds/sec + pair-interactions/sec; FP64 % of peak, 1/2/4/8 B200"
+UNIT = "builds/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="landau", choices=["landau", "reference"])
+    ap.add_argument("--workload", default="C4", choices=["C4", "C2", "C3", "C5"])
+    ap.add_argument("--batch", type=int, default=1024, help="C4 vertices in the whole job")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample", type=int, default=0, help="oracle vertices for cpu_baseline (0 = auto)")
+    return ap.parse_args()
+
+
+def workload(args, world, rank):
+    """(name, problem for the mesh, list of per-item problems of this rank, pairs per build)."""
+    from paper_conf_ipps_adamsbkw22_b200 import inputs
+    if args.workload == "C4":
+        B = args.batch
+        lo, hi = rank * B // world, (rank + 1) * B // world
+        items = [inputs.config4_vertex(b, B) for b in range(lo, hi)]
+        desc = {"workload": f"C4: {B} x C2 vertex grids (e+D, Q3 AMR 68 cells, N=1088, thermal-quench f), "
+                            f"{B // world} per GPU, no communication",
+                "vertices": B, "points_per_vertex": 1088, "order": 3, "species": 2,
+                "l2": "flushed between timed steps (256 MiB write)"}
+        return desc, items[0] if items else inputs.config4_vertex(0, B), items
+    p = inputs.CONFIGS[args.workload]()
+    desc = {"workload": f"{args.workload} single build", "points": p.npoints, "order": p.order,
+            "species": len(p.species), "l2": "flushed between timed steps (256 MiB write)"}
+    return desc, p, [p] if rank == 0 or world == 1 else []
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5).stdout
+                for line in out.strip().splitlines():
+                    self.rows.append([x.strip() for x in line.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows for k in range(4) if len(r) > 5 + k and r[5 + k] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def fp64_peak_tflops(props, sm_max_mhz):
+    """Derived FP64 (DFMA) peak: SMs x 64 FP64 lanes per SM per clock (4 SMSPs x 16) x 2 FLOP x clock.
+    See DESIGN.md 'Roofline'; tools/fp64_peak.cu measures the DFMA rate on the box."""
+    return props.multi_processor_count * 64 * 2 * sm_max_mhz * 1e6 / 1e12
+
+
+def load_profile_traffic(workload):
+    path = os.path.join(ROOT, "profiles", "inner_traffic.json")
+    try:
+        d = json.load(open(path))
+        return d.get(workload)
+    except Exception:
+        return None
+
+
+# FP64 FLOP per ordered pair, executed on the fast path of landau_pair (2*DFMA + DMUL + DADD), counted
+# once from ncu sm__sass_thread_inst_executed_op_{dfma,dmul,dadd}_pred_on / pairs.
+FLOP_PER_PAIR = float(os.environ.get("LANDAU_FLOP_PER_PAIR", "228"))
+
+
+def cpu_baseline(args, desc, nsample):
+    from oracle.oracle import Oracle, get_threads
+    from paper_conf_ipps_adamsbkw22_b200 import inputs
+    B = args.batch
+    if args.workload == "C4":
+        verts = [int(round(k * (B - 1) / max(nsample - 1, 1))) for k in range(nsample)]
+        probs = [inputs.config4_vertex(b, B) for b in verts]
+        sample = f"full oracle Jacobian (incl. |.| scale) of {nsample} of the {B} C4 vertices (b = {verts})"
+    else:
+        probs = [inputs.CONFIGS[args.workload]()]
+        sample = f"full oracle Jacobian of one {args.workload} build"
+    t = 0.0
+    for p in probs:
+        o = Oracle(p)
+        f = o.coefficients()
+        t0 = time.perf_counter()
+        o.jacobian(f)
+        t += time.perf_counter() - t0
+    return {"value": len(probs) / t, "unit": UNIT, "cores": get_threads(), "kind": "oracle", "sample": sample,
+            "seconds": t}
+
+
+def run_reference(args, world, rank):
+    """--impl reference: the oracle arm (the CPU program the paper's equations define), timed on host cores."""
+    if rank != 0:
+        return 0
+    from oracle.oracle import Oracle, get_threads
+    from paper_conf_ipps_adamsbkw22_b200 import inputs
+    desc, prob0, _ = workload(args, 1, 0)
+    B = args.batch
+    times = []
+    n_per_step = 1
+    for k in range(args.warmup + args.steps):
+        if args.workload == "C4":
+            p = inputs.config4_vertex((k * 97) % B, B)
+        else:
+            p = inputs.CONFIGS[args.workload]()
+        o = Oracle(p)
+        f = o.coefficients()
+        t0 = time.perf_counter()
+        o.jacobian(f)
+        dt = time.perf_counter() - t0
+        if k >= args.warmup:
+            times.append(dt)
+    T = sum(times)
+    value = n_per_step * len(times) / T
+    N = 1088 if args.workload == "C4" else prob0.npoints
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / len(times),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": desc, "pairs_per_s": value * N * N,
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": get_threads(), "kind": "oracle",
+                             "sample": f"1 vertex Jacobian per step ({args.workload}), full oracle"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, world, rank)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_adamsbkw22_b200 import inputs
+    from paper_conf_ipps_adamsbkw22_b200 import landau as L
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    stream = torch.cuda.current_stream()
+    desc, prob0, items = workload(args, world, rank)
+    h = L.Landau.from_problem(prob0, device=local, stream=stream)
+    nodes = h.all_nodes()
+    nloc = len(items)
+    N = h.npoints
+    F_host = np.stack([inputs.coefficients(p, nodes) for p in items]) if nloc else np.zeros((1, h.ndof))
+    F = torch.tensor(F_host, device="cuda")
+    vals = torch.empty((max(nloc, 1), h.nnz), dtype=torch.float64, device="cuda")
+    mvals = torch.empty(h.nnz, dtype=torch.float64, device="cuda")
+    flush = torch.empty(256 * 1024 * 1024 // 8, dtype=torch.float64, device="cuda")
+    shift = 1.0e3
+
+    def step():
+        if nloc:
+            h.set_state_batched(F)
+            h.jacobian_batched(vals)
+            h.mass(shift, mvals)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    h.set_timing(True)
+    n0 = h.launch_count()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    with Clocks(local) as clk:
+        torch.cuda.synchronize()
+        for k in range(args.steps):
+            flush.fill_(float(k))
+            evs[k][0].record(stream)
+            step()
+            evs[k][1].record(stream)
+        torch.cuda.synchronize()
+    launches = h.launch_count() - n0
+    tim = h.get_timing()
+    h.set_timing(False)
+    local_ms = sum(a.elapsed_time(b) for a, b in evs)
+    t = torch.tensor([local_ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.barrier()
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_ms = float(t.item())
+    total_builds = args.batch if args.workload == "C4" else 1
+    ms_per_step = total_ms / args.steps
+    value = total_builds / (ms_per_step / 1e3)
+    pairs_per_build = N * N
+
+    # ---- e2e through the host-pointer C-ABI entry point --------------------------------------
+    f_pin = torch.tensor(F_host).pin_memory()
+    v_pin = torch.empty((max(nloc, 1), h.nnz), dtype=torch.float64).pin_memory()
+    for _ in range(min(args.warmup, 2)):
+        if nloc:
+            h.jacobian_host(f_pin, v_pin)
+    e_ms = 0.0
+    for k in range(args.steps):
+        flush.fill_(float(k))
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        if nloc:
+            h.jacobian_host(f_pin, v_pin)
+        b.record(stream)
+        torch.cuda.synchronize()
+        e_ms += a.elapsed_time(b)
+    et = torch.tensor([e_ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(et, op=dist.ReduceOp.MAX)
+    e2e_value = total_builds / (float(et.item()) / args.steps / 1e3)
+
+    # ---- roofline of the dominant kernel (inner integral, FP64 pipe) --------------------------
+    inner_ms, inner_n = tim["inner"]
+    inner_avg_s = inner_ms / max(inner_n, 1) / 1e3
+    flops_per_launch = FLOP_PER_PAIR * pairs_per_build * max(nloc, 1)
+    achieved = flops_per_launch / inner_avg_s / 1e12 if inner_n else None
+    clocks = clk.summary()
+    props = torch.cuda.get_device_properties(local)
+    sm_max = clocks["sm_max_mhz"] or 1965.0
+    peak = fp64_peak_tflops(props, sm_max)
+    step_ms_lib = sum(v[0] for v in tim.values()) / args.steps
+    roof = {"bound": "alu", "kernel": "inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
+            "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None,
+            "traffic": load_profile_traffic(args.workload),
+            "peak_note": f"derived FP64 DFMA peak: {props.multi_processor_count} SMs x 64 lanes x 2 FLOP x {sm_max:.0f} MHz",
+            "flop_per_pair": FLOP_PER_PAIR, "inner_ms_per_launch": inner_avg_s * 1e3,
+            "inner_share_of_step": (inner_ms / args.steps) / ms_per_step if ms_per_step else None,
+            "pairs_per_s_inner": pairs_per_build * max(nloc, 1) / inner_avg_s * world if inner_n else None}
+    stage_ms = {k: v[0] / args.steps for k, v in tim.items()}
+
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": dict(desc, parallelism=f"batch-shard x{world}" if world > 1 else "1 GPU"),
+            "pairs_per_s": value * pairs_per_build, "roofline": roof, "stage_ms_per_step": stage_ms,
+            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(F_host.nbytes) * world,
+                    "d2h_bytes_per_step": int(v_pin.numel() * 8) * world, "api": "landau_jacobian_host"},
+            "gpu_launches": int(launches), "clocks": clocks}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        ns = args.cpu_sample or (8 if args.workload == "C4" else 1)
+        line["cpu_baseline"] = cpu_baseline(args, desc, ns)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

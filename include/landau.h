@@ -1,0 +1,169 @@
+/* landau.h -- C ABI of liblandau.so: the FP64 conservative finite-element Landau Jacobian on B200.
+ *
+ * Reference: M. F. Adams, D. P. Brennan, M. G. Knepley, P. Wang, "Landau collision operator in the
+ * CUDA programming model applied to thermal quench plasmas", IPDPS 2022.  Citations "@N" are
+ * character offsets into the single-line paper text PAPER.md; "Amb-k" are the
+ * readings of ambiguous passages listed in DESIGN.md.
+ *
+ * What a build computes; all arithmetic is FP64 on the device:
+ *   a-1  f, grad f of every species at the quadrature points from the FE coefficients (Alg. 1
+ *        lines 5-8 @15260-15570; Eqs. 10-11 @12313-13111), summed into
+ *        T_D(j) = sum_b e_b^2 f_b(j),  T_K(j) = sum_b e_b^2 (m0/m_b) grad f_b(j)  (b on j's grid);
+ *   a-2  the inner integral (Eqs. 7-8 @9251-9509; Alg. 1 lines 3-11 @14935-15669)
+ *        G_D(i) = sum_{j: (r_j,z_j) != (r_i,z_i)} w_j T_D(j) U^D(i,j),
+ *        G_K(i) = sum_j w_j U^K(i,j) . T_K(j), with U^D, U^K the azimuthal integrals of Eq. 3
+ *        (@7593) written with complete elliptic integrals (Amb-1, Amb-6);
+ *   a-3  species factors  D~_a = -nu e_a^2 (m0/m_a)^2 G_D,  K~_a = nu e_a^2 (m0/m_a) G_K
+ *        (Alg. 1 lines 13-16 @15729-16012);
+ *   a-4  element matrices C_a[k,l] = sum_q w_q [grad phi_k . D~_a . grad phi_l + (grad phi_k . K~_a) phi_l]
+ *        (Eqs. 5-6 @8833-9206; rows = test functions);
+ *   a-5  assembly J_a = sum_e P_e^T C_a,e P_e with hanging-node interpolation P_e (@14112, @42262),
+ *        species-block-diagonal (@11094-11357), deterministic (no atomics; Amb-15);
+ *   a-6  mass  shift * sum_e P_e^T (sum_q w_q phi_k phi_l) P_e (@39757-39999).
+ * J is the Picard ("approximate linearization", @10657-10914) matrix with C(f) ~= J f (Amb-4); the
+ * caller forms shift*M - J.
+ *
+ * Units: App. A (@58269): velocities in v0 = (8 k T_e / (pi m_e))^(1/2), masses in m_e (m0 = m_e),
+ * charges in e, nu_ab = nu e_a^2 e_b^2 with nu = 1 for lnLambda = 10 (Amb-13).
+ *
+ * Discretisation conventions (fixed by this ABI):
+ *   - grid g is a 2:1-balanced quadtree of square leaf cells {r0, z0, h} (lower-left corner, side h)
+ *     tiling [0, R_g] x [-R_g, R_g]; cells are given leaves-only, in any order;
+ *   - Q_p Lagrange elements, p in {2,3,4}, equispaced nodes (Amb-8); a node on the interior of a
+ *     coarser neighbour's edge is constrained to that edge's degree-p interpolant (Amb-10);
+ *   - (p+1)^2 Gauss-Legendre points per cell, weight w = w_a w_b (h/2)^2 r, no 2 pi (Amb-2, Amb-9);
+ *   - points are numbered grid-major, cells in input order, q = qz*(p+1) + qr inside a cell;
+ *   - DOFs of a grid: the non-constrained node positions, ordered by z ascending then r ascending
+ *     (Amb-12); the state vector is species-major: [f_0 on grid(0)][f_1 on grid(1)]...;
+ *   - CSR: block a holds rows/columns offset by sum_{b<a} ndof(grid(b)); columns sorted;
+ *   - COO: per species a, per cell e of grid(a) (input order), the n_e x n_e block P_e^T C P_e over
+ *     the cell's sorted distinct DOFs, row-major; duplicates across cells are to be summed.
+ *
+ * Conventions of the calls:
+ *   - every call returns 0 (LANDAU_OK) or a negative code; nothing throws or aborts;
+ *   - device pointers (suffix _dev) are owned by the caller; the library owns its workspace;
+ *   - all device work is enqueued on the stream given to landau_create; outputs are valid once that
+ *     stream has synchronised; set_state copies its input (the caller may reuse it immediately);
+ *   - one handle per host thread; a handle is tied to one device.
+ */
+#ifndef LANDAU_H
+#define LANDAU_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct landau_s *landau_t;
+
+enum {
+  LANDAU_OK = 0,
+  LANDAU_EINVAL = -1,       /* invalid argument (bad mesh, order, species, format, size)        */
+  LANDAU_ENOMEM = -2,       /* host or device allocation failed                                  */
+  LANDAU_ECUDA = -3,        /* a CUDA runtime call or kernel launch failed                       */
+  LANDAU_ENCCL = -4,        /* NCCL could not be loaded or a collective failed                   */
+  LANDAU_ESTATE = -5,       /* jacobian/point_coeffs before set_state (or batch size mismatch)   */
+  LANDAU_EUNSUPPORTED = -6  /* valid request this build does not implement                       */
+};
+enum { LANDAU_CSR = 0, LANDAU_COO = 1 };
+enum { LANDAU_DIST_REPLICATE = 0, LANDAU_DIST_BATCH = 1, LANDAU_DIST_ELEMENTS = 2 };
+
+typedef struct {
+  int32_t ngrids;
+  const int64_t *ncells;   /* [ngrids] leaf cells per grid                                       */
+  const double *cells;     /* [sum ncells][3] = {r0, z0, h}, grids concatenated                  */
+  const double *radius;    /* [ngrids] R_g                                                       */
+} landau_mesh_t;
+
+typedef struct {
+  int32_t order;           /* p in {2, 3, 4}                                                     */
+  int32_t nq1d;            /* Gauss points per direction; 0 -> p + 1 (the only supported value)   */
+  int32_t nspecies;        /* S in [1, 16]                                                       */
+  const double *mass;      /* [S] m_a / m_e > 0                                                  */
+  const double *charge;    /* [S] e_a / e (only e_a^2 enters)                                    */
+  const int32_t *grid;     /* [S] grid index of each species                                     */
+  double nu;               /* nu_ab = nu e_a^2 e_b^2                                             */
+} landau_params_t;
+
+typedef struct {
+  int32_t rank, world;         /* this process and the number of processes (one GPU each)        */
+  const void *nccl_unique_id;  /* 128 bytes from landau_nccl_unique_id on rank 0, broadcast by the
+                                  caller (torch.distributed); only read for LANDAU_DIST_ELEMENTS   */
+  int32_t mode;                /* LANDAU_DIST_*: REPLICATE and BATCH need no communicator (the
+                                  caller splits batches); ELEMENTS splits target cells into world
+                                  contiguous equal ranges and all-gathers G over NCCL              */
+} landau_dist_t;
+
+/* cuda_device = LANDAU_HOST_ONLY builds only the host-side plan (sizes, nodes, points, patterns can
+ * be queried without a GPU); every device call on such a handle returns LANDAU_EUNSUPPORTED. */
+#define LANDAU_HOST_ONLY (-1)
+
+/* Create a handle: validates the mesh (EINVAL if cells overlap, do not tile [0,R]x[-R,R], are not
+ * on a quadtree lattice, r0 < 0, h <= 0, or violate 2:1 edge balance), builds the FE space, the
+ * CSR/COO patterns and the assembly gather map on the host, uploads them and computes the mass
+ * matrix on the device.  cuda_stream is a cudaStream_t (NULL = legacy default stream).
+ * dist may be NULL (single process). */
+int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_t *prm, int32_t cuda_device,
+                  void *cuda_stream, const landau_dist_t *dist);
+void landau_destroy(landau_t h);
+
+/* Sizes: ndof = sum over species of ndof(grid(a)); npoints = N; nnz_csr and ncoo of the whole
+ * block-diagonal matrix.  Any output pointer may be NULL. */
+int landau_get_sizes(landau_t h, int64_t *ndof, int64_t *npoints, int64_t *nnz_csr, int64_t *ncoo);
+int landau_get_grid_ndof(landau_t h, int32_t grid, int64_t *ndof);
+/* host, caller-allocated [ndof(grid)]: coordinates of the DOF nodes of one grid, in DOF order */
+int landau_get_nodes(landau_t h, int32_t grid, double *r, double *z);
+/* host, caller-allocated [npoints]: quadrature points and weights */
+int landau_get_points(landau_t h, double *r, double *z, double *w);
+/* host, caller-allocated; any pointer may be NULL: csr_rowptr [ndof+1], csr_col [nnz_csr],
+ * coo_row/coo_col [ncoo] */
+int landau_get_pattern(landau_t h, int64_t *csr_rowptr, int32_t *csr_col, int32_t *coo_row, int32_t *coo_col);
+
+/* State: f_dev = [ndof] species-major FE coefficients (device).  Batched: [nbatch][ndof]; the
+ * batch shares the mesh (independent spatial vertices). */
+int landau_set_state(landau_t h, const double *f_dev);
+int landau_set_state_batched(landau_t h, int64_t nbatch, const double *f_dev);
+
+/* Jacobian of the current state: values_dev = [nnz_csr] (LANDAU_CSR) or [ncoo] (LANDAU_COO);
+ * batched: [nbatch][nnz] with nbatch equal to the last set_state_batched. */
+int landau_jacobian(landau_t h, double *values_dev, int32_t format);
+int landau_jacobian_batched(landau_t h, int64_t nbatch, double *values_dev, int32_t format);
+
+/* Convenience for host data (end-to-end path): copies f_host [nbatch][ndof] to the device, builds,
+ * copies the values back to values_host [nbatch][nnz] and synchronises the stream.  Pinned host
+ * memory gives asynchronous copies. */
+int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, double *values_host, int32_t format);
+
+/* Mass matrix values shift * M for every species block: [nnz_csr] or [ncoo]. */
+int landau_mass(landau_t h, double shift, double *values_dev, int32_t format);
+
+/* Debug/parity hook for step a-2: G_dev = [5][npoints] (G_D rr, rz, zz, G_K r, z) of the current
+ * state (batched: [nbatch][5][npoints]). */
+int landau_point_coeffs(landau_t h, double *G_dev);
+int landau_point_coeffs_batched(landau_t h, int64_t nbatch, double *G_dev);
+
+/* Element split (LANDAU_DIST_ELEMENTS): contiguous cell range [e0, e1) owned by a rank for a mesh
+ * of nelem cells; pure host arithmetic, usable without a GPU. */
+int landau_partition(int64_t nelem, int32_t world, int32_t rank, int64_t *e0, int64_t *e1);
+/* 128-byte NCCL unique id (rank 0 only; loads libnccl.so.2 on demand). */
+int landau_nccl_unique_id(void *out128);
+
+/* Per-stage device timers (CUDA events on the handle's stream): stage = 0 field, 1 inner,
+ * 2 reduce, 3 element, 4 assemble, 5 mass, 6 allgather.  enable resets the accumulators. */
+enum { LANDAU_T_FIELD = 0, LANDAU_T_INNER, LANDAU_T_REDUCE, LANDAU_T_ELEMENT, LANDAU_T_ASSEMBLE,
+       LANDAU_T_MASS, LANDAU_T_ALLGATHER, LANDAU_NTIMERS };
+int landau_set_timing(landau_t h, int32_t enable);
+/* ms[LANDAU_NTIMERS] total milliseconds, launches[LANDAU_NTIMERS] kernel launches (synchronises) */
+int landau_get_timing(landau_t h, double *ms, int64_t *launches);
+/* kernels launched by this handle since creation (all stages) */
+int landau_get_launch_count(landau_t h, int64_t *count);
+
+const char *landau_strerror(int code);
+/* last detailed error message of a handle (or of the last failed create when h == NULL) */
+const char *landau_last_error(landau_t h);
+const char *landau_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,406 @@
+// host_setup.cpp -- step a-0 (see host_setup.h).  Host-only C++17; no CUDA.
+#include "host_setup.h"
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <climits>
+#include <functional>
+#include <map>
+#include <unordered_map>
+#include <unordered_set>
+
+namespace landau {
+namespace {
+
+// ---------------------------------------------------------------------------------------------
+// 1D building blocks
+// ---------------------------------------------------------------------------------------------
+void gauss_legendre(int n, std::vector<double> &x, std::vector<double> &w) {
+  x.assign(n, 0.0);
+  w.assign(n, 0.0);
+  const double pi = 3.14159265358979323846;
+  for (int i = 0; i < (n + 1) / 2; i++) {
+    double t = std::cos(pi * (i + 0.75) / (n + 0.5)), dp = 1.0;
+    for (int it = 0; it < 100; it++) {
+      double p0 = 1.0, p1 = t;
+      for (int k = 2; k <= n; k++) {
+        double p2 = ((2.0 * k - 1.0) * t * p1 - (k - 1.0) * p0) / k;
+        p0 = p1;
+        p1 = p2;
+      }
+      if (n == 1) p0 = 1.0, p1 = t;
+      dp = n * (t * p1 - p0) / (t * t - 1.0);
+      double dt = p1 / dp;
+      t -= dt;
+      if (std::fabs(dt) < 1e-17) break;
+    }
+    double p0 = 1.0, p1 = t;
+    for (int k = 2; k <= n; k++) {
+      double p2 = ((2.0 * k - 1.0) * t * p1 - (k - 1.0) * p0) / k;
+      p0 = p1;
+      p1 = p2;
+    }
+    dp = n * (t * p1 - p0) / (t * t - 1.0);
+    double wt = 2.0 / ((1.0 - t * t) * dp * dp);
+    x[i] = -t;
+    x[n - 1 - i] = t;
+    w[i] = w[n - 1 - i] = wt;
+  }
+  if (n % 2 == 1) x[n / 2] = 0.0;
+}
+
+// equispaced Lagrange basis on [-1, 1] (nodes -1 + 2k/p): value and derivative
+double lagrange(int p, int a, double x) {
+  double v = 1.0;
+  for (int k = 0; k <= p; k++)
+    if (k != a) v *= (x - (-1.0 + 2.0 * k / p)) / (2.0 * (a - k) / p);
+  return v;
+}
+double lagrange_d(int p, int a, double x) {
+  double s = 0.0;
+  for (int m = 0; m <= p; m++) {
+    if (m == a) continue;
+    double v = 1.0 / (2.0 * (a - m) / p);
+    for (int k = 0; k <= p; k++)
+      if (k != a && k != m) v *= (x - (-1.0 + 2.0 * k / p)) / (2.0 * (a - k) / p);
+    s += v;
+  }
+  return s;
+}
+
+inline uint64_t key2(int64_t ir, int64_t iz) { return (uint64_t(iz) << 32) | uint64_t(ir); }
+
+struct ICell {
+  int64_t R0, Z0, H;   // in units of the grid's smallest cell size; Z0 measured from z = -R
+  int level;           // H = 2^(L - level)
+};
+
+}  // namespace
+
+std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, const double *radius, int order,
+                       Plan &plan) {
+  char msg[256];
+  const int p = order, nq = order + 1, nb = (p + 1) * (p + 1), nqp = nq * nq;
+  plan = Plan();
+  plan.p = p;
+  plan.nq = nq;
+  plan.nb = nb;
+  plan.nqp = nqp;
+  plan.ngrids = ngrids;
+  // reference tables
+  std::vector<double> xg, wg;
+  gauss_legendre(nq, xg, wg);
+  plan.tab_phi.resize(nqp * nb);
+  plan.tab_dxi.resize(nqp * nb);
+  plan.tab_deta.resize(nqp * nb);
+  for (int qz = 0; qz < nq; qz++)
+    for (int qr = 0; qr < nq; qr++)
+      for (int b = 0; b <= p; b++)
+        for (int a = 0; a <= p; a++) {
+          int q = qz * nq + qr, n = b * (p + 1) + a;
+          plan.tab_phi[q * nb + n] = lagrange(p, a, xg[qr]) * lagrange(p, b, xg[qz]);
+          plan.tab_dxi[q * nb + n] = lagrange_d(p, a, xg[qr]) * lagrange(p, b, xg[qz]);
+          plan.tab_deta[q * nb + n] = lagrange(p, a, xg[qr]) * lagrange_d(p, b, xg[qz]);
+        }
+
+  int64_t c0 = 0, pt0 = 0;
+  plan.grids.resize(ngrids);
+  for (int g = 0; g < ngrids; g++) {
+    GridPlan &G = plan.grids[g];
+    const double R = radius[g];
+    const int64_t n = ncells[g];
+    if (!(R > 0) || n < 2) {
+      snprintf(msg, sizeof msg, "grid %d: radius must be > 0 and the grid needs >= 2 cells", g);
+      return msg;
+    }
+    G.R = R;
+    G.cell0 = c0;
+    G.ncell = n;
+    G.pt0 = pt0;
+    const double *cc = cells + 3 * c0;
+    // ---- integer quadtree coordinates -------------------------------------------------------
+    double hmin = 1e300;
+    for (int64_t c = 0; c < n; c++) {
+      if (!(cc[3 * c + 2] > 0) || cc[3 * c] < 0) {
+        snprintf(msg, sizeof msg, "grid %d cell %lld: h must be > 0 and r0 >= 0", g, (long long)c);
+        return msg;
+      }
+      hmin = std::min(hmin, cc[3 * c + 2]);
+    }
+    const double rootH = R / hmin;
+    const int L = (int)std::llround(std::log2(rootH));
+    if (L < 0 || L > 26 || std::fabs(std::ldexp(1.0, L) - rootH) > 1e-9 * rootH) {
+      snprintf(msg, sizeof msg, "grid %d: cell sizes are not R / 2^k", g);
+      return msg;
+    }
+    std::vector<ICell> ic(n);
+    std::unordered_set<uint64_t> present;   // (level, R0/H, Z0/H)
+    auto qkey = [](int level, int64_t i, int64_t j) { return (uint64_t(level) << 58) | (uint64_t(j) << 29) | uint64_t(i); };
+    int64_t area = 0;
+    const int64_t Rl = int64_t(1) << L;
+    for (int64_t c = 0; c < n; c++) {
+      double a = cc[3 * c] / hmin, b = (cc[3 * c + 1] + R) / hmin, h = cc[3 * c + 2] / hmin;
+      ICell &x = ic[c];
+      x.R0 = std::llround(a);
+      x.Z0 = std::llround(b);
+      x.H = std::llround(h);
+      int lv = L - (int)std::llround(std::log2((double)x.H));
+      x.level = lv;
+      bool ok = std::fabs(a - x.R0) < 1e-6 && std::fabs(b - x.Z0) < 1e-6 && std::fabs(h - x.H) < 1e-6 && x.H >= 1 &&
+                (x.H & (x.H - 1)) == 0 && lv >= 0 && x.R0 % x.H == 0 && x.Z0 % x.H == 0 && x.R0 + x.H <= Rl &&
+                x.Z0 + x.H <= 2 * Rl && x.Z0 >= 0;
+      if (!ok) {
+        snprintf(msg, sizeof msg, "grid %d cell %lld is not a quadtree cell of [0,R]x[-R,R]", g, (long long)c);
+        return msg;
+      }
+      if (!present.insert(qkey(lv, x.R0 / x.H, x.Z0 / x.H)).second) {
+        snprintf(msg, sizeof msg, "grid %d: duplicate cell %lld", g, (long long)c);
+        return msg;
+      }
+      area += x.H * x.H;
+    }
+    for (int64_t c = 0; c < n; c++) {   // no ancestor of a leaf may itself be a leaf
+      const ICell &x = ic[c];
+      for (int lv = x.level - 1; lv >= 0; lv--) {
+        int64_t H = int64_t(1) << (L - lv);
+        if (present.count(qkey(lv, x.R0 / H, x.Z0 / H))) {
+          snprintf(msg, sizeof msg, "grid %d: overlapping cells", g);
+          return msg;
+        }
+      }
+    }
+    if (area != 2 * Rl * Rl) {
+      snprintf(msg, sizeof msg, "grid %d: cells do not tile [0,R]x[-R,R]", g);
+      return msg;
+    }
+    // 2:1 edge balance: the leaf across each edge of a cell is at most twice its size
+    auto leaf_size = [&](int64_t x2, int64_t z2) -> int64_t {   // doubled coords of an interior point
+      if (x2 < 0 || z2 < 0 || x2 >= 2 * Rl || z2 >= 4 * Rl) return 0;
+      for (int lv = L; lv >= 0; lv--) {
+        int64_t H = int64_t(1) << (L - lv);
+        if (present.count(qkey(lv, (x2 / 2) / H, (z2 / 2) / H))) return H;
+      }
+      return -1;
+    };
+    for (int64_t c = 0; c < n; c++) {
+      const ICell &x = ic[c];
+      int64_t pts[4][2] = {{2 * (x.R0 + x.H) + 1, 2 * x.Z0 + 1}, {2 * x.R0 - 1, 2 * x.Z0 + 1},
+                           {2 * x.R0 + 1, 2 * (x.Z0 + x.H) + 1}, {2 * x.R0 + 1, 2 * x.Z0 - 1}};
+      for (auto &q : pts) {
+        int64_t s = leaf_size(q[0], q[1]);
+        if (s > 2 * x.H) {
+          snprintf(msg, sizeof msg, "grid %d: quadtree not 2:1 balanced at cell %lld", g, (long long)c);
+          return msg;
+        }
+      }
+    }
+    // ---- node positions (lattice unit hmin / p) ------------------------------------------------
+    std::unordered_map<uint64_t, int> pos_id;   // candidate positions
+    std::vector<std::pair<int64_t, int64_t>> pos;   // (ir, iz)
+    pos_id.reserve(n * nb);
+    std::vector<int> cell_node(n * nb);
+    for (int64_t c = 0; c < n; c++)
+      for (int b = 0; b <= p; b++)
+        for (int a = 0; a <= p; a++) {
+          int64_t ir = ic[c].R0 * p + a * ic[c].H, iz = ic[c].Z0 * p + b * ic[c].H;
+          auto it = pos_id.emplace(key2(ir, iz), (int)pos.size());
+          if (it.second) pos.emplace_back(ir, iz);
+          cell_node[c * nb + b * (p + 1) + a] = it.first->second;
+        }
+    // hanging positions: odd multiples of H/2 on a cell edge that some finer neighbour has as node
+    struct Hang {
+      int64_t mr[8], mz[8];
+      double mw[8];
+    };
+    std::unordered_map<int, Hang> hang;
+    for (int64_t c = 0; c < n; c++) {
+      const ICell &x = ic[c];
+      if (x.H < 2) continue;
+      const int64_t h2 = x.H / 2, r0 = x.R0 * p, z0 = x.Z0 * p, Lp = x.H * p;
+      // edges: (start point, direction)
+      const int64_t E[4][4] = {{r0, z0, 1, 0}, {r0, z0 + Lp, 1, 0}, {r0, z0, 0, 1}, {r0 + Lp, z0, 0, 1}};
+      for (auto &e : E) {
+        for (int k = 1; k < 2 * p; k += 2) {
+          int64_t ir = e[0] + e[2] * k * h2, iz = e[1] + e[3] * k * h2;
+          auto it = pos_id.find(key2(ir, iz));
+          if (it == pos_id.end()) continue;
+          Hang hg;
+          for (int j = 0; j <= p; j++) {
+            hg.mr[j] = e[0] + e[2] * j * x.H;
+            hg.mz[j] = e[1] + e[3] * j * x.H;
+            // L_j(t), t = k / (2p), nodes i/p: prod_{i != j} (k - 2i) / (2 (j - i)) -- exact integers
+            double num = 1.0, den = 1.0;
+            for (int i = 0; i <= p; i++)
+              if (i != j) num *= double(k - 2 * i), den *= double(2 * (j - i));
+            hg.mw[j] = num / den;
+          }
+          hang[it->second] = hg;
+        }
+      }
+    }
+    // DOFs: non-hanging positions sorted by (iz, ir)
+    std::vector<int> order_;
+    for (int i = 0; i < (int)pos.size(); i++)
+      if (!hang.count(i)) order_.push_back(i);
+    std::sort(order_.begin(), order_.end(), [&](int a, int b) {
+      return pos[a].second != pos[b].second ? pos[a].second < pos[b].second : pos[a].first < pos[b].first;
+    });
+    std::vector<int> dof_of(pos.size(), -1);
+    G.ndof = (int)order_.size();
+    G.node_r.resize(G.ndof);
+    G.node_z.resize(G.ndof);
+    const double unit = hmin / p;
+    for (int d = 0; d < G.ndof; d++) {
+      dof_of[order_[d]] = d;
+      G.node_r[d] = pos[order_[d]].first * unit;
+      G.node_z[d] = pos[order_[d]].second * unit - R;
+    }
+    // resolve a position into (dof, weight) terms (recursive through constraints)
+    std::function<void(int, double, std::vector<std::pair<int, double>> &, int)> resolve =
+        [&](int pid, double s, std::vector<std::pair<int, double>> &out, int depth) {
+          if (dof_of[pid] >= 0) {
+            for (auto &t : out)
+              if (t.first == dof_of[pid]) {
+                t.second += s;
+                return;
+              }
+            out.emplace_back(dof_of[pid], s);
+            return;
+          }
+          if (depth > 8) return;
+          const Hang &hg = hang.at(pid);
+          for (int j = 0; j <= p; j++) {
+            if (hg.mw[j] == 0.0) continue;
+            auto it = pos_id.find(key2(hg.mr[j], hg.mz[j]));
+            if (it == pos_id.end()) continue;   // cannot happen for a tiled, balanced tree
+            resolve(it->second, s * hg.mw[j], out, depth + 1);
+          }
+        };
+    // ---- per-cell extraction ----------------------------------------------------------------
+    G.ne.resize(n);
+    G.edof_off.assign(n + 1, 0);
+    G.P_off.assign(n + 1, 0);
+    std::vector<std::vector<std::pair<int, double>>> loc(nb);
+    for (int64_t c = 0; c < n; c++) {
+      std::vector<int> d;
+      for (int a = 0; a < nb; a++) {
+        loc[a].clear();
+        resolve(cell_node[c * nb + a], 1.0, loc[a], 0);
+        if (loc[a].empty()) {
+          snprintf(msg, sizeof msg, "grid %d: unresolvable node in cell %lld", g, (long long)c);
+          return msg;
+        }
+        for (auto &t : loc[a]) d.push_back(t.first);
+        // field extraction list (global over grids)
+        plan.ext_ptr.push_back((int32_t)plan.ext_dof.size());
+        for (auto &t : loc[a]) {
+          plan.ext_dof.push_back(t.first);
+          plan.ext_w.push_back(t.second);
+        }
+      }
+      std::sort(d.begin(), d.end());
+      d.erase(std::unique(d.begin(), d.end()), d.end());
+      int ne = (int)d.size();
+      G.ne[c] = ne;
+      G.edof_off[c + 1] = G.edof_off[c] + ne;
+      G.edof.insert(G.edof.end(), d.begin(), d.end());
+      G.P_off[c + 1] = G.P_off[c] + (int64_t)nb * ne;
+      size_t base = G.P.size();
+      G.P.resize(base + (size_t)nb * ne, 0.0);
+      for (int a = 0; a < nb; a++)
+        for (auto &t : loc[a]) {
+          int j = int(std::lower_bound(d.begin(), d.end(), t.first) - d.begin());
+          G.P[base + (size_t)a * ne + j] += t.second;
+        }
+      G.ncoo += (int64_t)ne * ne;
+    }
+    // ---- CSR pattern ------------------------------------------------------------------------
+    std::vector<std::vector<int>> rows(G.ndof);
+    for (int64_t c = 0; c < n; c++) {
+      const int *d = &G.edof[G.edof_off[c]];
+      for (int i = 0; i < G.ne[c]; i++)
+        for (int j = 0; j < G.ne[c]; j++) rows[d[i]].push_back(d[j]);
+    }
+    G.rowptr.assign(G.ndof + 1, 0);
+    for (int i = 0; i < G.ndof; i++) {
+      auto &r = rows[i];
+      std::sort(r.begin(), r.end());
+      r.erase(std::unique(r.begin(), r.end()), r.end());
+      G.rowptr[i + 1] = G.rowptr[i] + (int64_t)r.size();
+      G.col.insert(G.col.end(), r.begin(), r.end());
+    }
+    // ---- gather maps --------------------------------------------------------------------------
+    // slot contributions: (cell, a, b) with P[a][i] P[b][j] != 0, in (cell, a, b) order
+    GatherMap csr, coo;
+    std::vector<std::vector<std::pair<int32_t, double>>> csr_slots(G.col.size());
+    coo.ptr.push_back(0);
+    for (int64_t c = 0; c < n; c++) {
+      const int ne = G.ne[c];
+      const int *d = &G.edof[G.edof_off[c]];
+      const double *Pc = &G.P[G.P_off[c]];
+      const int64_t ge = c0 + c;
+      std::vector<int64_t> slot(ne * ne);
+      for (int i = 0; i < ne; i++)
+        for (int j = 0; j < ne; j++) {
+          auto b = G.col.begin() + G.rowptr[d[i]], e = G.col.begin() + G.rowptr[d[i] + 1];
+          slot[i * ne + j] = std::lower_bound(b, e, d[j]) - G.col.begin();
+        }
+      std::vector<std::vector<std::pair<int32_t, double>>> cslot(ne * ne);
+      for (int a = 0; a < nb; a++)
+        for (int bb = 0; bb < nb; bb++) {
+          const int32_t idx = (int32_t)(ge * 2 * nb * nb + a * nb + bb);
+          for (int i = 0; i < ne; i++) {
+            double pa = Pc[a * ne + i];
+            if (pa == 0.0) continue;
+            for (int j = 0; j < ne; j++) {
+              double pb = Pc[bb * ne + j];
+              if (pb == 0.0) continue;
+              csr_slots[slot[i * ne + j]].emplace_back(idx, pa * pb);
+              cslot[i * ne + j].emplace_back(idx, pa * pb);
+            }
+          }
+        }
+      for (auto &s : cslot) {
+        for (auto &t : s) {
+          coo.idx.push_back(t.first);
+          coo.w.push_back(t.second);
+        }
+        coo.ptr.push_back((int64_t)coo.idx.size());
+      }
+    }
+    csr.ptr.push_back(0);
+    for (auto &s : csr_slots) {
+      for (auto &t : s) {
+        csr.idx.push_back(t.first);
+        csr.w.push_back(t.second);
+      }
+      csr.ptr.push_back((int64_t)csr.idx.size());
+    }
+    plan.csr_map.push_back(std::move(csr));
+    plan.coo_map.push_back(std::move(coo));
+    // ---- points and per-cell data ---------------------------------------------------------------
+    for (int64_t c = 0; c < n; c++) {
+      const double r0 = cc[3 * c], z0 = cc[3 * c + 1], h = cc[3 * c + 2];
+      plan.cell_h.push_back(h);
+      plan.cell_grid.push_back(g);
+      for (int qz = 0; qz < nq; qz++)
+        for (int qr = 0; qr < nq; qr++) {
+          double r = r0 + 0.5 * h * (xg[qr] + 1.0);
+          double z = z0 + 0.5 * h * (xg[qz] + 1.0);
+          plan.pr.push_back(r);
+          plan.pz.push_back(z);
+          plan.pw.push_back(wg[qr] * wg[qz] * (0.25 * h * h) * r);
+        }
+    }
+    c0 += n;
+    pt0 += n * nqp;
+  }
+  plan.ext_ptr.push_back((int32_t)plan.ext_dof.size());
+  plan.ncell = c0;
+  plan.npts = pt0;
+  if (plan.ncell * 2 * nb * nb > INT32_MAX) return "mesh too large for 32-bit gather indices";
+  return "";
+}
+
+}  // namespace landau

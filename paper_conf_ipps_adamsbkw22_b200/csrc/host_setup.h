@@ -1,0 +1,68 @@
+// host_setup.h -- step a-0 of SURVEY.md §8(a): everything the device kernels need that depends only
+// on the mesh, the order and the species (built once per handle, on the host, in C++17).
+//
+//   * quadtree validation (lattice alignment, no overlap, full tiling, 2:1 edge balance; Amb-10)
+//   * Gauss-Legendre points/weights and Q_p tables at the reference points (Amb-8, Amb-9)
+//   * DOF numbering: non-hanging node positions ordered by (z, r) (Amb-12)
+//   * hanging-node extraction P_e: a node inside a coarser neighbour's edge takes that edge's
+//     degree-p Lagrange interpolant ("interpolate ... to four DOFs" for Q3, PAPER.md:1@42262)
+//   * CSR pattern (species-block-diagonal, @11277), COO layout, and the deterministic gather maps
+//     that replace the paper's atomic MatSetValues (@23291-24297, Amb-15).
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace landau {
+
+struct GridPlan {
+  double R = 0;
+  int64_t cell0 = 0;        // first global cell index
+  int64_t ncell = 0;
+  int64_t pt0 = 0;          // first global point index
+  int ndof = 0;
+  std::vector<double> node_r, node_z;   // [ndof]
+  // per cell: sorted distinct DOFs and dense extraction P[Nb][n_e]
+  std::vector<int> ne;                   // [ncell]
+  std::vector<int64_t> edof_off;         // [ncell+1]
+  std::vector<int> edof;                 // distinct DOFs
+  std::vector<int64_t> P_off;            // [ncell+1]
+  std::vector<double> P;                 // Nb * n_e per cell
+  // CSR pattern of one species block
+  std::vector<int64_t> rowptr;           // [ndof+1]
+  std::vector<int> col;
+  int64_t ncoo = 0;                      // sum_e n_e^2
+};
+
+// A gather map: output slot s = sum over its contributions (idx, w) of w * Celem[idx], in a fixed
+// order (cell, a, b).  idx = e * 2 Nb^2 + a * Nb + b indexes the [cell][2][Nb][Nb] element buffer.
+struct GatherMap {
+  std::vector<int64_t> ptr;   // [nslots+1]
+  std::vector<int32_t> idx;
+  std::vector<double> w;
+};
+
+struct Plan {
+  int p = 0, nq = 0, nb = 0, nqp = 0;
+  int ngrids = 0, nspecies = 0;
+  int64_t ncell = 0, npts = 0;
+  std::vector<GridPlan> grids;
+  // global per cell
+  std::vector<double> cell_h;            // [ncell]
+  std::vector<int> cell_grid;            // [ncell]
+  // global per point
+  std::vector<double> pr, pz, pw;        // [npts]
+  // reference tables at the Gauss points: [nqp][nb]
+  std::vector<double> tab_phi, tab_dxi, tab_deta;
+  // field extraction per cell-local node: ext_ptr[ncell*nb+1] -> (dof in its grid, weight)
+  std::vector<int32_t> ext_ptr, ext_dof;
+  std::vector<double> ext_w;
+  // gather maps per grid (CSR slots, COO slots)
+  std::vector<GatherMap> csr_map, coo_map;
+};
+
+// Build the plan.  Returns "" on success or an error message (the mesh is invalid).
+std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, const double *radius, int order,
+                       Plan &plan);
+
+}  // namespace landau

@@ -1,0 +1,994 @@
+// landau.cu -- liblandau.so: the C ABI of include/landau.h and the sm_100a kernels of one build.
+//
+//   N1 field_kernel     a-1  f, grad f at the quadrature points -> w T_D, w T_K      (HBM/latency)
+//   N2 inner_kernel     a-2  pairwise U^D, U^K sums (split-j partials)               (FP64 pipe)
+//   N2r reduce_kernel   a-2  fixed-order sum of the split-j partials                 (HBM)
+//   N3 element_kernel   a-4  species-independent element matrices C^D_e, C^K_e       (FP64/L1)
+//   N4 assemble_kernel  a-3+a-5  species factors + deterministic gather into CSR/COO (HBM)
+//   N5 mass             a-6  element mass at create (cached), shift-scaled copy       (HBM)
+// Citations: see include/landau.h and DESIGN.md.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/landau.h"
+#include "host_setup.h"
+#include "kernels.cuh"
+
+using namespace landau;
+
+namespace {
+
+__constant__ SpeciesConst c_sp;
+__constant__ double c_phi[kMaxNb * kMaxNb];
+__constant__ double c_dxi[kMaxNb * kMaxNb];
+__constant__ double c_deta[kMaxNb * kMaxNb];
+
+// ------------------------------------------------------------------------------------------------
+// N1: point fields.  One block handles EPB cells; thread (cell, q) evaluates its point.
+// The per-grid species sums T_D = sum e^2 f, T_K = sum e^2/m grad f are linear in f, so the
+// combined element coefficients gD_a = sum_b e_b^2 f_b,a and gK_a = sum_b e_b^2/m_b f_b,a are formed
+// first (one pass over the extraction list), then interpolated once.
+// ------------------------------------------------------------------------------------------------
+template <int NB, int EPB>
+__global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int64_t ndof_total, const double *__restrict__ f,
+                                                         const int32_t *__restrict__ ext_ptr,
+                                                         const int32_t *__restrict__ ext_dof,
+                                                         const double *__restrict__ ext_w,
+                                                         const int *__restrict__ cell_grid,
+                                                         const double *__restrict__ cell_h, const double *__restrict__ pw,
+                                                         double *__restrict__ wT, int64_t npts) {
+  __shared__ double gD[EPB][NB], gK[EPB][NB];
+  const int b = blockIdx.y;
+  const int el = threadIdx.x / NB, a = threadIdx.x % NB;
+  const int64_t e = (int64_t)blockIdx.x * EPB + el;
+  const double *fb = f + (int64_t)b * ndof_total;
+  if (e < ncell) {
+    const int g = cell_grid[e];
+    const int32_t k0 = ext_ptr[e * NB + a], k1 = ext_ptr[e * NB + a + 1];
+    double sD = 0.0, sK = 0.0;
+    for (int s = 0; s < c_sp.grid_nsp[g]; s++) {
+      const int sp = c_sp.grid_sp[g][s];
+      const double *fs = fb + c_sp.soff[sp];
+      double v = 0.0;
+      for (int32_t k = k0; k < k1; k++) v = fma(ext_w[k], __ldg(fs + ext_dof[k]), v);
+      sD = fma(c_sp.e2[sp], v, sD);
+      sK = fma(c_sp.e2m[sp], v, sK);
+    }
+    gD[el][a] = sD;
+    gK[el][a] = sK;
+  }
+  __syncthreads();
+  if (e < ncell) {
+    const int q = a;   // NQP == NB for (p+1)^2 Gauss points
+    const int64_t pt = e * NB + q;
+    double td = 0.0, tr = 0.0, tz = 0.0;
+#pragma unroll
+    for (int k = 0; k < NB; k++) {
+      td = fma(c_phi[q * NB + k], gD[el][k], td);
+      tr = fma(c_dxi[q * NB + k], gK[el][k], tr);
+      tz = fma(c_deta[q * NB + k], gK[el][k], tz);
+    }
+    const double s = 2.0 / cell_h[e];
+    const double w = pw[pt];
+    double *o = wT + (int64_t)b * 3 * npts;
+    o[pt] = w * td;
+    o[npts + pt] = w * s * tr;
+    o[2 * npts + pt] = w * s * tz;
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// N2: inner integral.  Block = TB threads x TPT targets each; sources streamed through shared
+// memory in tiles of TB (all lanes read the same source: broadcast).  blockIdx.y = split of the
+// source range (split-j), blockIdx.z = batch item.  out = [batch][nsplit][5][nt] partials.
+// ------------------------------------------------------------------------------------------------
+constexpr int kInnerTB = 128;
+
+template <int TPT>
+__global__ void __launch_bounds__(kInnerTB) inner_kernel(int64_t N, int64_t t0, int64_t nt, int64_t split_len,
+                                                          const double *__restrict__ pr, const double *__restrict__ pz,
+                                                          const double *__restrict__ wT, double *__restrict__ out,
+                                                          int64_t out_bstride) {
+  __shared__ double sr[kInnerTB], sz[kInnerTB], sd[kInnerTB], skr[kInnerTB], skz[kInnerTB];
+  const int b = blockIdx.z, split = blockIdx.y, nsplit = gridDim.y;
+  const double *wb = wT + (int64_t)b * 3 * N;
+  int64_t ti[TPT];
+  double tr[TPT], tz[TPT];
+  Acc5 acc[TPT];
+#pragma unroll
+  for (int t = 0; t < TPT; t++) {
+    ti[t] = (int64_t)blockIdx.x * kInnerTB * TPT + t * kInnerTB + threadIdx.x;
+    const int64_t gi = t0 + (ti[t] < nt ? ti[t] : nt - 1);
+    tr[t] = pr[gi];
+    tz[t] = pz[gi];
+    acc[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+  }
+  const int64_t j0 = (int64_t)split * split_len;
+  const int64_t j1 = min(N, j0 + split_len);
+  for (int64_t jt = j0; jt < j1; jt += kInnerTB) {
+    const int64_t j = jt + threadIdx.x;
+    if (j < j1) {
+      sr[threadIdx.x] = pr[j];
+      sz[threadIdx.x] = pz[j];
+      sd[threadIdx.x] = wb[j];
+      skr[threadIdx.x] = wb[N + j];
+      skz[threadIdx.x] = wb[2 * N + j];
+    }
+    __syncthreads();
+    const int n = (int)min((int64_t)kInnerTB, j1 - jt);
+    for (int k = 0; k < n; k++) {
+      const double rb = sr[k], zb = sz[k], wd = sd[k], wkr = skr[k], wkz = skz[k];
+#pragma unroll
+      for (int t = 0; t < TPT; t++) landau_pair(tr[t], tz[t], rb, zb, wd, wkr, wkz, acc[t]);
+    }
+    __syncthreads();
+  }
+  double *o = out + (int64_t)b * out_bstride + (int64_t)split * 5 * nt;
+#pragma unroll
+  for (int t = 0; t < TPT; t++) {
+    if (ti[t] < nt) {
+      o[ti[t]] = acc[t].drr;
+      o[nt + ti[t]] = acc[t].drz;
+      o[2 * nt + ti[t]] = acc[t].dzz;
+      o[3 * nt + ti[t]] = acc[t].kr;
+      o[4 * nt + ti[t]] = acc[t].kz;
+    }
+  }
+  (void)nsplit;
+}
+
+// N2r: G[b][c][i] = sum_{s = 0..nsplit-1} part[b][s][c][i] in fixed order (deterministic).
+__global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__ part, double *__restrict__ G,
+                              int64_t G_bstride, int nbatch) {
+  const int64_t total = (int64_t)nbatch * 5 * nt;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = k / (5 * nt), ci = k % (5 * nt);
+    const double *p = part + b * (int64_t)nsplit * 5 * nt + ci;
+    double s = 0.0;
+    for (int q = 0; q < nsplit; q++) s += p[(int64_t)q * 5 * nt];
+    G[b * G_bstride + ci] = s;
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// N3: element matrices (species independent).  One block per (cell, batch); thread (k, l).
+//   C^D[k,l] = (2/h)^2 sum_q w_q (gk . G_D(q) . gl),  C^K[k,l] = (2/h) sum_q w_q (gk . G_K(q)) phi_l(q)
+// with gk the reference gradients.  G is read in the chunked layout
+//   G[((i / Nc) * nbatch + b) * 5 + c][i % Nc]     (Nc = N when not distributed).
+// ------------------------------------------------------------------------------------------------
+template <int NB>
+__global__ void __launch_bounds__(NB * NB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
+                                                            int nbatch, const double *__restrict__ pw,
+                                                            const double *__restrict__ cell_h, double *__restrict__ Cbuf) {
+  __shared__ double sG[5][NB], sw[NB];
+  const int64_t e = blockIdx.x;
+  const int b = blockIdx.y;
+  const int tid = threadIdx.x;
+  if (tid < NB) {
+    const int64_t i = e * NB + tid;
+    const int64_t chunk = i / Nc, off = i % Nc;
+    const double *Gb = G + ((chunk * nbatch + b) * 5) * Nc + off;
+#pragma unroll
+    for (int c = 0; c < 5; c++) sG[c][tid] = Gb[c * Nc];
+    sw[tid] = pw[i];
+  }
+  __syncthreads();
+  const int k = tid / NB, l = tid % NB;
+  double cd = 0.0, ck = 0.0;
+#pragma unroll 4
+  for (int q = 0; q < NB; q++) {
+    const double gkr = c_dxi[q * NB + k], gkz = c_deta[q * NB + k];
+    const double glr = c_dxi[q * NB + l], glz = c_deta[q * NB + l], pl = c_phi[q * NB + l];
+    const double Grr = sG[0][q], Grz = sG[1][q], Gzz = sG[2][q], Kr = sG[3][q], Kz = sG[4][q];
+    const double w = sw[q];
+    const double vd = gkr * fma(Grr, glr, Grz * glz) + gkz * fma(Grz, glr, Gzz * glz);
+    cd = fma(w, vd, cd);
+    ck = fma(w * fma(gkr, Kr, gkz * Kz), pl, ck);
+  }
+  const double s = 2.0 / cell_h[e];
+  double *o = Cbuf + ((int64_t)b * ncell + e) * 2 * NB * NB;
+  o[tid] = cd * s * s;
+  o[NB * NB + tid] = ck * s;
+}
+
+// Mass element matrices (create time): M[k,l] = sum_q w_q phi_k phi_l, stored in the [cell][2][NB^2]
+// layout (second half zero) so the same gather maps apply.
+template <int NB>
+__global__ void __launch_bounds__(NB * NB) mass_element_kernel(int64_t ncell, const double *__restrict__ pw,
+                                                                 double *__restrict__ Mbuf) {
+  const int64_t e = blockIdx.x;
+  const int tid = threadIdx.x, k = tid / NB, l = tid % NB;
+  double m = 0.0;
+  for (int q = 0; q < NB; q++) m = fma(pw[e * NB + q] * c_phi[q * NB + k], c_phi[q * NB + l], m);
+  Mbuf[e * 2 * NB * NB + tid] = m;
+  Mbuf[e * 2 * NB * NB + NB * NB + tid] = 0.0;
+}
+
+// ------------------------------------------------------------------------------------------------
+// N4: deterministic gather.  For grid slot s (CSR nonzero or COO entry):
+//   sD = sum_k w_k C^D[idx_k], sK = sum_k w_k C^K[idx_k]   (fixed (cell, a, b) order)
+//   out[b][out_off(a) + s] = fD_a sD + fK_a sK   for every species a on the grid   (a-3 + a-5)
+// ------------------------------------------------------------------------------------------------
+struct GatherDev {
+  const int64_t *ptr;
+  const int32_t *idx;
+  const double *w;
+  int64_t nslots;
+  int64_t out_off[kMaxSpecies];   // output offset per species slot on this grid
+};
+
+template <int NB>
+__global__ void assemble_kernel(GatherDev gm, int grid, const double *__restrict__ Cbuf, int64_t cbuf_bstride,
+                                double *__restrict__ out, int64_t out_bstride) {
+  const int b = blockIdx.y;
+  const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= gm.nslots) return;
+  const double *C = Cbuf + (int64_t)b * cbuf_bstride;
+  const int64_t k0 = gm.ptr[s], k1 = gm.ptr[s + 1];
+  double sD = 0.0, sK = 0.0;
+  for (int64_t k = k0; k < k1; k++) {
+    const int64_t i = gm.idx[k];
+    const double w = gm.w[k];
+    sD = fma(w, C[i], sD);
+    sK = fma(w, C[i + NB * NB], sK);
+  }
+  double *o = out + (int64_t)b * out_bstride;
+  const int ns = c_sp.grid_nsp[grid];
+  for (int q = 0; q < ns; q++) {
+    const int sp = c_sp.grid_sp[grid][q];
+    o[gm.out_off[q] + s] = fma(c_sp.fD[sp], sD, c_sp.fK[sp] * sK);
+  }
+}
+
+// mass gather (create time): out[s] = sum_k w_k M[idx_k]
+__global__ void mass_gather_kernel(const int64_t *__restrict__ ptr, const int32_t *__restrict__ idx,
+                                   const double *__restrict__ w, int64_t nslots, const double *__restrict__ M,
+                                   double *__restrict__ out) {
+  const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= nslots) return;
+  double v = 0.0;
+  for (int64_t k = ptr[s]; k < ptr[s + 1]; k++) v = fma(w[k], M[idx[k]], v);
+  out[s] = v;
+}
+
+// N5: out[o0 + i] = shift * M[i]
+__global__ void scale_copy_kernel(const double *__restrict__ M, double shift, int64_t n, double *__restrict__ out) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = shift * M[i];
+}
+
+// copy chunked G layout -> [b][5][N]
+__global__ void unchunk_kernel(const double *__restrict__ G, int64_t N, int64_t Nc, int nbatch, double *__restrict__ out) {
+  const int64_t total = (int64_t)nbatch * 5 * N;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = k / (5 * N), c = (k / N) % 5, i = k % N;
+    out[k] = G[(((i / Nc) * nbatch + b) * 5 + c) * Nc + (i % Nc)];
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// NCCL, loaded on demand (only LANDAU_DIST_ELEMENTS needs it)
+// ------------------------------------------------------------------------------------------------
+typedef struct {
+  char internal[128];
+} ncclUniqueId_;
+typedef void *ncclComm_;
+struct NcclApi {
+  void *so = nullptr;
+  int (*GetUniqueId)(ncclUniqueId_ *) = nullptr;
+  int (*CommInitRank)(ncclComm_ *, int, ncclUniqueId_, int) = nullptr;
+  int (*AllGather)(const void *, void *, size_t, int, ncclComm_, cudaStream_t) = nullptr;
+  int (*CommDestroy)(ncclComm_) = nullptr;
+  const char *(*GetErrorString)(int) = nullptr;
+};
+NcclApi g_nccl;
+std::mutex g_nccl_mu;
+bool load_nccl() {
+  std::lock_guard<std::mutex> lk(g_nccl_mu);
+  if (g_nccl.so) return true;
+  const char *names[] = {"libnccl.so.2", "libnccl.so"};
+  void *so = nullptr;
+  for (const char *n : names)
+    if ((so = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
+  if (!so) return false;
+  g_nccl.GetUniqueId = (int (*)(ncclUniqueId_ *))dlsym(so, "ncclGetUniqueId");
+  g_nccl.CommInitRank = (int (*)(ncclComm_ *, int, ncclUniqueId_, int))dlsym(so, "ncclCommInitRank");
+  g_nccl.AllGather = (int (*)(const void *, void *, size_t, int, ncclComm_, cudaStream_t))dlsym(so, "ncclAllGather");
+  g_nccl.CommDestroy = (int (*)(ncclComm_))dlsym(so, "ncclCommDestroy");
+  g_nccl.GetErrorString = (const char *(*)(int))dlsym(so, "ncclGetErrorString");
+  if (!g_nccl.GetUniqueId || !g_nccl.CommInitRank || !g_nccl.AllGather || !g_nccl.CommDestroy) return false;
+  g_nccl.so = so;
+  return true;
+}
+constexpr int kNcclFloat64 = 8;
+
+thread_local std::string g_create_error;
+
+}  // namespace
+
+// ==================================================================================================
+// handle
+// ==================================================================================================
+struct landau_s {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  Plan plan;
+  int S = 0;
+  std::vector<double> mass, charge;
+  std::vector<int> sgrid;
+  double nu = 1.0;
+  SpeciesConst spc{};
+  int64_t ndof = 0, nnz = 0, ncoo = 0;
+  std::vector<int64_t> soff, snnz_off, scoo_off;
+  // distribution
+  int rank = 0, world = 1, mode = 0;
+  int64_t e0 = 0, e1 = 0, chunk_cells = 0, Nc = 0;
+  ncclComm_ comm = nullptr;
+  // device: static
+  double *d_r = nullptr, *d_z = nullptr, *d_w = nullptr, *d_h = nullptr;
+  int *d_cell_grid = nullptr;
+  int32_t *d_ext_ptr = nullptr, *d_ext_dof = nullptr;
+  double *d_ext_w = nullptr;
+  struct DevMap {
+    int64_t *ptr = nullptr;
+    int32_t *idx = nullptr;
+    double *w = nullptr;
+    int64_t nslots = 0;
+  };
+  std::vector<DevMap> d_csr, d_coo;
+  std::vector<double *> d_mass_csr, d_mass_coo;   // per grid
+  // device: state + workspace
+  int64_t cap = 0, nbatch = 0;
+  bool have_state = false;
+  double *d_f = nullptr, *d_wT = nullptr, *d_part = nullptr, *d_G = nullptr, *d_C = nullptr;
+  int64_t part_cap = 0;
+  // host staging for landau_jacobian_host
+  double *d_vals_tmp = nullptr;
+  int64_t vals_tmp_cap = 0;
+  // timing
+  bool timing = false;
+  std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> ev_used;
+  std::vector<cudaEvent_t> ev_pool;
+  int64_t tlaunch[LANDAU_NTIMERS] = {0};
+  int64_t launches = 0;
+  bool host_only = false;
+  std::string err;
+};
+
+namespace {
+
+int fail(landau_t h, int code, const std::string &msg) {
+  if (h) h->err = msg;
+  else g_create_error = msg;
+  return code;
+}
+
+#define CU(call)                                                                                   \
+  do {                                                                                             \
+    cudaError_t e_ = (call);                                                                       \
+    if (e_ != cudaSuccess) return fail(h, LANDAU_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+#define KCHECK()                                                                                   \
+  do {                                                                                             \
+    cudaError_t e_ = cudaGetLastError();                                                           \
+    if (e_ != cudaSuccess) return fail(h, LANDAU_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(e_)); \
+  } while (0)
+
+template <class T>
+int upload(landau_t h, T **dst, const std::vector<T> &src) {
+  size_t bytes = std::max<size_t>(src.size(), 1) * sizeof(T);
+  CU(cudaMalloc((void **)dst, bytes));
+  if (!src.empty()) CU(cudaMemcpyAsync(*dst, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice, h->stream));
+  return LANDAU_OK;
+}
+
+cudaEvent_t get_event(landau_t h) {
+  if (!h->ev_pool.empty()) {
+    cudaEvent_t e = h->ev_pool.back();
+    h->ev_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e;
+  cudaEventCreate(&e);
+  return e;
+}
+
+struct Timer {
+  landau_t h;
+  int stage;
+  cudaEvent_t a = nullptr, b = nullptr;
+  Timer(landau_t h_, int s) : h(h_), stage(s) {
+    if (h->timing) {
+      a = get_event(h);
+      b = get_event(h);
+      cudaEventRecord(a, h->stream);
+    }
+  }
+  ~Timer() {
+    if (h->timing) {
+      cudaEventRecord(b, h->stream);
+      h->ev_used.push_back({stage, {a, b}});
+    }
+  }
+};
+
+int ensure_workspace(landau_t h, int64_t nbatch) {
+  const int64_t N = h->plan.npts, Ne = h->plan.ncell, nb = h->plan.nb;
+  if (nbatch <= h->cap) return LANDAU_OK;
+  cudaFree(h->d_f);
+  cudaFree(h->d_wT);
+  cudaFree(h->d_G);
+  cudaFree(h->d_C);
+  h->d_f = h->d_wT = h->d_G = h->d_C = nullptr;
+  CU(cudaMalloc(&h->d_f, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
+  CU(cudaMalloc(&h->d_wT, sizeof(double) * nbatch * 3 * N));
+  CU(cudaMalloc(&h->d_G, sizeof(double) * nbatch * 5 * h->Nc * h->world));
+  CU(cudaMalloc(&h->d_C, sizeof(double) * nbatch * Ne * 2 * nb * nb));
+  h->cap = nbatch;
+  return LANDAU_OK;
+}
+
+int set_constants(landau_t h) {
+  const Plan &P = h->plan;
+  CU(cudaMemcpyToSymbolAsync(c_sp, &h->spc, sizeof(SpeciesConst), 0, cudaMemcpyHostToDevice, h->stream));
+  CU(cudaMemcpyToSymbolAsync(c_phi, P.tab_phi.data(), sizeof(double) * P.tab_phi.size(), 0, cudaMemcpyHostToDevice, h->stream));
+  CU(cudaMemcpyToSymbolAsync(c_dxi, P.tab_dxi.data(), sizeof(double) * P.tab_dxi.size(), 0, cudaMemcpyHostToDevice, h->stream));
+  CU(cudaMemcpyToSymbolAsync(c_deta, P.tab_deta.data(), sizeof(double) * P.tab_deta.size(), 0, cudaMemcpyHostToDevice, h->stream));
+  return LANDAU_OK;
+}
+
+// Constant memory is per device & module, not per handle: re-upload when another handle (different
+// mesh/order/species) was the last one to set it on this device.
+const landau_s *g_const_owner[64] = {nullptr};
+std::mutex g_const_mu;
+int bind_constants(landau_t h) {
+  std::lock_guard<std::mutex> lk(g_const_mu);
+  if (g_const_owner[h->device & 63] == h) return LANDAU_OK;
+  int rc = set_constants(h);
+  if (rc == LANDAU_OK) g_const_owner[h->device & 63] = h;
+  return rc;
+}
+
+// ---------------------------------------------------------------------------------------------
+// launch helpers
+// ---------------------------------------------------------------------------------------------
+template <int NB>
+int launch_field(landau_t h, int64_t nbatch) {
+  constexpr int EPB = NB == 9 ? 8 : (NB == 16 ? 8 : 4);
+  const Plan &P = h->plan;
+  dim3 grid((unsigned)((P.ncell + EPB - 1) / EPB), (unsigned)nbatch);
+  Timer t(h, LANDAU_T_FIELD);
+  field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, h->ndof, h->d_f, h->d_ext_ptr, h->d_ext_dof, h->d_ext_w,
+                                                          h->d_cell_grid, h->d_h, h->d_w, h->d_wT, P.npts);
+  h->launches++;
+  h->tlaunch[LANDAU_T_FIELD]++;
+  KCHECK();
+  return LANDAU_OK;
+}
+
+int num_sms(landau_t h) {
+  static int sms[64] = {0};
+  int &s = sms[h->device & 63];
+  if (!s) cudaDeviceGetAttribute(&s, cudaDevAttrMultiProcessorCount, h->device);
+  return s ? s : 148;
+}
+
+int launch_inner(landau_t h, int64_t nbatch) {
+  const Plan &P = h->plan;
+  const int64_t N = P.npts;
+  const int64_t t0 = h->e0 * P.nqp, nt = (h->e1 - h->e0) * P.nqp;
+  constexpr int TPT = 1;
+  const int64_t tblocks = (nt + kInnerTB * TPT - 1) / (kInnerTB * TPT);
+  // split-j so that small problems still fill the machine: aim for >= 8 blocks per SM
+  const int64_t want = 8LL * num_sms(h);
+  int64_t nsplit = std::max<int64_t>(1, (want + tblocks * nbatch - 1) / (tblocks * nbatch));
+  nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, N / 32));
+  const int64_t split_len = (N + nsplit - 1) / nsplit;
+  nsplit = (N + split_len - 1) / split_len;
+  double *G_own = h->d_G + (int64_t)h->rank * nbatch * 5 * h->Nc;   // [world][batch][5][Nc]
+  double *out;
+  int64_t out_bstride;
+  if (nsplit == 1) {
+    out = G_own;
+    out_bstride = 5 * h->Nc;
+  } else {
+    const int64_t need = nbatch * nsplit * 5 * nt;
+    if (need > h->part_cap) {
+      cudaFree(h->d_part);
+      h->d_part = nullptr;
+      CU(cudaMalloc(&h->d_part, sizeof(double) * need));
+      h->part_cap = need;
+    }
+    out = h->d_part;
+    out_bstride = nsplit * 5 * nt;
+  }
+  {
+    Timer t(h, LANDAU_T_INNER);
+    dim3 grid((unsigned)tblocks, (unsigned)nsplit, (unsigned)nbatch);
+    inner_kernel<TPT><<<grid, kInnerTB, 0, h->stream>>>(N, t0, nt, split_len, h->d_r, h->d_z, h->d_wT, out, out_bstride);
+    h->launches++;
+    h->tlaunch[LANDAU_T_INNER]++;
+    KCHECK();
+  }
+  if (nsplit > 1) {
+    Timer t(h, LANDAU_T_REDUCE);
+    const int64_t total = nbatch * 5 * nt;
+    const int blocks = (int)std::min<int64_t>((total + 255) / 256, 16LL * num_sms(h));
+    // G_own is [batch][5][Nc] with Nc >= nt
+    reduce_kernel<<<blocks, 256, 0, h->stream>>>(nt, (int)nsplit, h->d_part, G_own, 5 * h->Nc, (int)nbatch);
+    h->launches++;
+    h->tlaunch[LANDAU_T_REDUCE]++;
+    KCHECK();
+  }
+  if (h->world > 1 && h->mode == LANDAU_DIST_ELEMENTS) {
+    Timer t(h, LANDAU_T_ALLGATHER);
+    int rc = g_nccl.AllGather(G_own, h->d_G, (size_t)(nbatch * 5 * h->Nc), kNcclFloat64, h->comm, h->stream);
+    if (rc != 0) return fail(h, LANDAU_ENCCL, std::string("ncclAllGather: ") + (g_nccl.GetErrorString ? g_nccl.GetErrorString(rc) : "error"));
+  }
+  return LANDAU_OK;
+}
+
+template <int NB>
+int launch_element(landau_t h, int64_t nbatch) {
+  const Plan &P = h->plan;
+  Timer t(h, LANDAU_T_ELEMENT);
+  dim3 grid((unsigned)P.ncell, (unsigned)nbatch);
+  element_kernel<NB><<<grid, NB * NB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, h->d_w, h->d_h, h->d_C);
+  h->launches++;
+  h->tlaunch[LANDAU_T_ELEMENT]++;
+  KCHECK();
+  return LANDAU_OK;
+}
+
+template <int NB>
+int launch_assemble(landau_t h, int64_t nbatch, double *out, int format) {
+  const Plan &P = h->plan;
+  Timer t(h, LANDAU_T_ASSEMBLE);
+  const int64_t out_bstride = format == LANDAU_CSR ? h->nnz : h->ncoo;
+  for (int g = 0; g < P.ngrids; g++) {
+    const auto &m = format == LANDAU_CSR ? h->d_csr[g] : h->d_coo[g];
+    GatherDev gd;
+    gd.ptr = m.ptr;
+    gd.idx = m.idx;
+    gd.w = m.w;
+    gd.nslots = m.nslots;
+    for (int q = 0; q < h->spc.grid_nsp[g]; q++) {
+      int sp = h->spc.grid_sp[g][q];
+      gd.out_off[q] = format == LANDAU_CSR ? h->snnz_off[sp] : h->scoo_off[sp];
+    }
+    if (h->spc.grid_nsp[g] == 0 || m.nslots == 0) continue;
+    dim3 grid((unsigned)((m.nslots + 255) / 256), (unsigned)nbatch);
+    assemble_kernel<NB><<<grid, 256, 0, h->stream>>>(gd, g, h->d_C, P.ncell * 2 * NB * NB, out, out_bstride);
+    h->launches++;
+    h->tlaunch[LANDAU_T_ASSEMBLE]++;
+    KCHECK();
+  }
+  return LANDAU_OK;
+}
+
+template <int NB>
+int build_jacobian(landau_t h, int64_t nbatch, double *out, int format) {
+  int rc;
+  if ((rc = bind_constants(h))) return rc;
+  if ((rc = launch_field<NB>(h, nbatch))) return rc;
+  if ((rc = launch_inner(h, nbatch))) return rc;
+  if ((rc = launch_element<NB>(h, nbatch))) return rc;
+  if (out && (rc = launch_assemble<NB>(h, nbatch, out, format))) return rc;
+  return LANDAU_OK;
+}
+
+int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
+  switch (h->plan.nb) {
+    case 9: return build_jacobian<9>(h, nbatch, out, format);
+    case 16: return build_jacobian<16>(h, nbatch, out, format);
+    case 25: return build_jacobian<25>(h, nbatch, out, format);
+  }
+  return fail(h, LANDAU_EUNSUPPORTED, "order");
+}
+
+template <int NB>
+int build_mass(landau_t h) {
+  const Plan &P = h->plan;
+  double *Mbuf = nullptr;
+  CU(cudaMalloc(&Mbuf, sizeof(double) * P.ncell * 2 * NB * NB));
+  mass_element_kernel<NB><<<(unsigned)P.ncell, NB * NB, 0, h->stream>>>(P.ncell, h->d_w, Mbuf);
+  h->launches++;
+  KCHECK();
+  for (int g = 0; g < P.ngrids; g++) {
+    for (int f = 0; f < 2; f++) {
+      const auto &m = f == 0 ? h->d_csr[g] : h->d_coo[g];
+      double *&dst = f == 0 ? h->d_mass_csr[g] : h->d_mass_coo[g];
+      CU(cudaMalloc(&dst, sizeof(double) * std::max<int64_t>(m.nslots, 1)));
+      if (m.nslots == 0) continue;
+      mass_gather_kernel<<<(unsigned)((m.nslots + 255) / 256), 256, 0, h->stream>>>(m.ptr, m.idx, m.w, m.nslots, Mbuf, dst);
+      h->launches++;
+      KCHECK();
+    }
+  }
+  CU(cudaStreamSynchronize(h->stream));
+  cudaFree(Mbuf);
+  return LANDAU_OK;
+}
+
+}  // namespace
+
+// ==================================================================================================
+// C ABI
+// ==================================================================================================
+extern "C" {
+
+const char *landau_version(void) { return "landau-b200 0.1 (sm_100a, FP64)"; }
+
+const char *landau_strerror(int code) {
+  switch (code) {
+    case LANDAU_OK: return "ok";
+    case LANDAU_EINVAL: return "invalid argument";
+    case LANDAU_ENOMEM: return "out of memory";
+    case LANDAU_ECUDA: return "CUDA error";
+    case LANDAU_ENCCL: return "NCCL error";
+    case LANDAU_ESTATE: return "no state set (or batch size mismatch)";
+    case LANDAU_EUNSUPPORTED: return "unsupported";
+  }
+  return "unknown error";
+}
+
+const char *landau_last_error(landau_t h) { return h ? h->err.c_str() : g_create_error.c_str(); }
+
+int landau_partition(int64_t nelem, int32_t world, int32_t rank, int64_t *e0, int64_t *e1) {
+  if (nelem < 0 || world < 1 || rank < 0 || rank >= world || !e0 || !e1) return LANDAU_EINVAL;
+  const int64_t chunk = (nelem + world - 1) / world;
+  *e0 = std::min<int64_t>(nelem, (int64_t)rank * chunk);
+  *e1 = std::min<int64_t>(nelem, (int64_t)(rank + 1) * chunk);
+  return LANDAU_OK;
+}
+
+int landau_nccl_unique_id(void *out128) {
+  if (!out128) return LANDAU_EINVAL;
+  if (!load_nccl()) return LANDAU_ENCCL;
+  ncclUniqueId_ id;
+  if (g_nccl.GetUniqueId(&id) != 0) return LANDAU_ENCCL;
+  memcpy(out128, &id, 128);
+  return LANDAU_OK;
+}
+
+int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_t *prm, int32_t cuda_device,
+                  void *cuda_stream, const landau_dist_t *dist) {
+  landau_t h = nullptr;
+  if (!out || !mesh || !prm) return fail(h, LANDAU_EINVAL, "null argument");
+  *out = nullptr;
+  if (mesh->ngrids < 1 || mesh->ngrids > kMaxSpecies || !mesh->ncells || !mesh->cells || !mesh->radius)
+    return fail(h, LANDAU_EINVAL, "bad mesh descriptor");
+  if (prm->order < 2 || prm->order > 4) return fail(h, LANDAU_EINVAL, "order must be 2, 3 or 4");
+  if (prm->nq1d != 0 && prm->nq1d != prm->order + 1) return fail(h, LANDAU_EUNSUPPORTED, "nq1d must be 0 or order+1");
+  if (prm->nspecies < 1 || prm->nspecies > kMaxSpecies || !prm->mass || !prm->charge || !prm->grid)
+    return fail(h, LANDAU_EINVAL, "bad species descriptor");
+  for (int a = 0; a < prm->nspecies; a++)
+    if (!(prm->mass[a] > 0) || prm->grid[a] < 0 || prm->grid[a] >= mesh->ngrids || !std::isfinite(prm->charge[a]))
+      return fail(h, LANDAU_EINVAL, "bad species " + std::to_string(a));
+  int rank = 0, world = 1, mode = LANDAU_DIST_REPLICATE;
+  if (dist) {
+    rank = dist->rank;
+    world = dist->world;
+    mode = dist->mode;
+    if (world < 1 || rank < 0 || rank >= world || mode < 0 || mode > 2) return fail(h, LANDAU_EINVAL, "bad dist descriptor");
+    if (mode != LANDAU_DIST_ELEMENTS) world = 1, rank = 0;   // replicas / caller-split batches: independent handles
+  }
+  h = new landau_s();
+  h->device = cuda_device;
+  h->stream = (cudaStream_t)cuda_stream;
+  h->rank = rank;
+  h->world = world;
+  h->mode = mode;
+  std::string msg = build_plan(mesh->ngrids, mesh->ncells, mesh->cells, mesh->radius, prm->order, h->plan);
+  if (!msg.empty()) {
+    delete h;
+    return fail(nullptr, LANDAU_EINVAL, msg);
+  }
+  const Plan &P = h->plan;
+  h->S = prm->nspecies;
+  h->nu = prm->nu;
+  h->spc = SpeciesConst{};
+  h->spc.nspecies = h->S;
+  h->spc.ngrids = P.ngrids;
+  h->soff.assign(h->S + 1, 0);
+  h->snnz_off.assign(h->S + 1, 0);
+  h->scoo_off.assign(h->S + 1, 0);
+  for (int a = 0; a < h->S; a++) {
+    const int g = prm->grid[a];
+    h->mass.push_back(prm->mass[a]);
+    h->charge.push_back(prm->charge[a]);
+    h->sgrid.push_back(g);
+    const double e2 = prm->charge[a] * prm->charge[a], im = 1.0 / prm->mass[a];
+    h->spc.e2[a] = e2;
+    h->spc.e2m[a] = e2 * im;
+    h->spc.fD[a] = -prm->nu * e2 * im * im;
+    h->spc.fK[a] = prm->nu * e2 * im;
+    h->spc.grid_sp[g][h->spc.grid_nsp[g]++] = a;
+    h->soff[a + 1] = h->soff[a] + P.grids[g].ndof;
+    h->snnz_off[a + 1] = h->snnz_off[a] + (int64_t)P.grids[g].col.size();
+    h->scoo_off[a + 1] = h->scoo_off[a] + P.grids[g].ncoo;
+    h->spc.soff[a] = h->soff[a];
+  }
+  h->ndof = h->soff[h->S];
+  h->nnz = h->snnz_off[h->S];
+  h->ncoo = h->scoo_off[h->S];
+  // element partition
+  landau_partition(P.ncell, world, rank, &h->e0, &h->e1);
+  h->chunk_cells = (P.ncell + world - 1) / world;
+  h->Nc = world > 1 ? h->chunk_cells * P.nqp : P.npts;
+  int rc;
+  if (cuda_device == LANDAU_HOST_ONLY) {
+    h->host_only = true;
+    *out = h;
+    return LANDAU_OK;
+  }
+  cudaError_t ce = cudaSetDevice(cuda_device);
+  if (ce != cudaSuccess) {
+    std::string m = std::string("cudaSetDevice: ") + cudaGetErrorString(ce);
+    delete h;
+    return fail(nullptr, LANDAU_ECUDA, m);
+  }
+  auto bail = [&](int code) {
+    std::string m = h->err;
+    landau_destroy(h);
+    return fail(nullptr, code, m);
+  };
+  if ((rc = upload(h, &h->d_r, P.pr)) || (rc = upload(h, &h->d_z, P.pz)) || (rc = upload(h, &h->d_w, P.pw)) ||
+      (rc = upload(h, &h->d_h, P.cell_h)) || (rc = upload(h, &h->d_cell_grid, P.cell_grid)) ||
+      (rc = upload(h, &h->d_ext_ptr, P.ext_ptr)) || (rc = upload(h, &h->d_ext_dof, P.ext_dof)) ||
+      (rc = upload(h, &h->d_ext_w, P.ext_w)))
+    return bail(rc);
+  h->d_csr.resize(P.ngrids);
+  h->d_coo.resize(P.ngrids);
+  h->d_mass_csr.assign(P.ngrids, nullptr);
+  h->d_mass_coo.assign(P.ngrids, nullptr);
+  for (int g = 0; g < P.ngrids; g++) {
+    for (int f = 0; f < 2; f++) {
+      const GatherMap &m = f == 0 ? P.csr_map[g] : P.coo_map[g];
+      auto &d = f == 0 ? h->d_csr[g] : h->d_coo[g];
+      if ((rc = upload(h, &d.ptr, m.ptr)) || (rc = upload(h, &d.idx, m.idx)) || (rc = upload(h, &d.w, m.w))) return bail(rc);
+      d.nslots = (int64_t)m.ptr.size() - 1;
+    }
+  }
+  if ((rc = bind_constants(h))) return bail(rc);
+  switch (P.nb) {
+    case 9: rc = build_mass<9>(h); break;
+    case 16: rc = build_mass<16>(h); break;
+    case 25: rc = build_mass<25>(h); break;
+  }
+  if (rc) return bail(rc);
+  if (world > 1) {
+    if (!dist->nccl_unique_id) return bail(fail(h, LANDAU_EINVAL, "nccl_unique_id required for element split"));
+    if (!load_nccl()) return bail(fail(h, LANDAU_ENCCL, "cannot load libnccl.so.2"));
+    ncclUniqueId_ id;
+    memcpy(&id, dist->nccl_unique_id, 128);
+    int nr = g_nccl.CommInitRank(&h->comm, world, id, rank);
+    if (nr != 0) return bail(fail(h, LANDAU_ENCCL, std::string("ncclCommInitRank: ") + g_nccl.GetErrorString(nr)));
+  }
+  *out = h;
+  return LANDAU_OK;
+}
+
+void landau_destroy(landau_t h) {
+  if (!h) return;
+  if (h->host_only) {
+    delete h;
+    return;
+  }
+  cudaSetDevice(h->device);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
+  for (double *p : {h->d_r, h->d_z, h->d_w, h->d_h, h->d_ext_w, h->d_f, h->d_wT, h->d_part, h->d_G, h->d_C, h->d_vals_tmp})
+    cudaFree(p);
+  cudaFree(h->d_cell_grid);
+  cudaFree(h->d_ext_ptr);
+  cudaFree(h->d_ext_dof);
+  for (auto *v : {&h->d_csr, &h->d_coo})
+    for (auto &m : *v) {
+      cudaFree(m.ptr);
+      cudaFree(m.idx);
+      cudaFree(m.w);
+    }
+  for (double *p : h->d_mass_csr) cudaFree(p);
+  for (double *p : h->d_mass_coo) cudaFree(p);
+  for (auto &u : h->ev_used) {
+    cudaEventDestroy(u.second.first);
+    cudaEventDestroy(u.second.second);
+  }
+  for (auto e : h->ev_pool) cudaEventDestroy(e);
+  {
+    std::lock_guard<std::mutex> lk(g_const_mu);
+    if (g_const_owner[h->device & 63] == h) g_const_owner[h->device & 63] = nullptr;
+  }
+  delete h;
+}
+
+int landau_get_sizes(landau_t h, int64_t *ndof, int64_t *npoints, int64_t *nnz_csr, int64_t *ncoo) {
+  if (!h) return LANDAU_EINVAL;
+  if (ndof) *ndof = h->ndof;
+  if (npoints) *npoints = h->plan.npts;
+  if (nnz_csr) *nnz_csr = h->nnz;
+  if (ncoo) *ncoo = h->ncoo;
+  return LANDAU_OK;
+}
+
+int landau_get_grid_ndof(landau_t h, int32_t grid, int64_t *ndof) {
+  if (!h || !ndof || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
+  *ndof = h->plan.grids[grid].ndof;
+  return LANDAU_OK;
+}
+
+int landau_get_nodes(landau_t h, int32_t grid, double *r, double *z) {
+  if (!h || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
+  const auto &G = h->plan.grids[grid];
+  if (r) memcpy(r, G.node_r.data(), sizeof(double) * G.ndof);
+  if (z) memcpy(z, G.node_z.data(), sizeof(double) * G.ndof);
+  return LANDAU_OK;
+}
+
+int landau_get_points(landau_t h, double *r, double *z, double *w) {
+  if (!h) return LANDAU_EINVAL;
+  const Plan &P = h->plan;
+  if (r) memcpy(r, P.pr.data(), sizeof(double) * P.npts);
+  if (z) memcpy(z, P.pz.data(), sizeof(double) * P.npts);
+  if (w) memcpy(w, P.pw.data(), sizeof(double) * P.npts);
+  return LANDAU_OK;
+}
+
+int landau_get_pattern(landau_t h, int64_t *csr_rowptr, int32_t *csr_col, int32_t *coo_row, int32_t *coo_col) {
+  if (!h) return LANDAU_EINVAL;
+  const Plan &P = h->plan;
+  int64_t row = 0, k = 0, kc = 0;
+  if (csr_rowptr) csr_rowptr[0] = 0;
+  for (int a = 0; a < h->S; a++) {
+    const GridPlan &G = P.grids[h->sgrid[a]];
+    const int64_t off = h->soff[a];
+    for (int i = 0; i < G.ndof; i++, row++) {
+      for (int64_t q = G.rowptr[i]; q < G.rowptr[i + 1]; q++, k++)
+        if (csr_col) csr_col[k] = (int32_t)(off + G.col[q]);
+      if (csr_rowptr) csr_rowptr[row + 1] = k;
+    }
+    for (int64_t c = 0; c < G.ncell; c++) {
+      const int ne = G.ne[c];
+      const int *d = &G.edof[G.edof_off[c]];
+      for (int i = 0; i < ne; i++)
+        for (int j = 0; j < ne; j++, kc++) {
+          if (coo_row) coo_row[kc] = (int32_t)(off + d[i]);
+          if (coo_col) coo_col[kc] = (int32_t)(off + d[j]);
+        }
+    }
+  }
+  return LANDAU_OK;
+}
+
+int landau_set_state_batched(landau_t h, int64_t nbatch, const double *f_dev) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !f_dev) return fail(h, LANDAU_EINVAL, "set_state: bad argument");
+  int rc = ensure_workspace(h, nbatch);
+  if (rc) return rc;
+  CU(cudaMemcpyAsync(h->d_f, f_dev, sizeof(double) * nbatch * h->ndof, cudaMemcpyDeviceToDevice, h->stream));
+  h->nbatch = nbatch;
+  h->have_state = true;
+  return LANDAU_OK;
+}
+
+int landau_set_state(landau_t h, const double *f_dev) { return landau_set_state_batched(h, 1, f_dev); }
+
+int landau_jacobian_batched(landau_t h, int64_t nbatch, double *values_dev, int32_t format) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "jacobian: bad argument");
+  if (!h->have_state || nbatch != h->nbatch) return fail(h, LANDAU_ESTATE, "jacobian: set_state first (batch size must match)");
+  return dispatch_build(h, nbatch, values_dev, format);
+}
+
+int landau_jacobian(landau_t h, double *values_dev, int32_t format) {
+  if (h && h->have_state && h->nbatch != 1) return fail(h, LANDAU_ESTATE, "jacobian: state is batched");
+  return landau_jacobian_batched(h, 1, values_dev, format);
+}
+
+int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, double *values_host, int32_t format) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !f_host || !values_host || (format != LANDAU_CSR && format != LANDAU_COO))
+    return fail(h, LANDAU_EINVAL, "jacobian_host: bad argument");
+  int rc = ensure_workspace(h, nbatch);
+  if (rc) return rc;
+  const int64_t nv = format == LANDAU_CSR ? h->nnz : h->ncoo;
+  if (nbatch * nv > h->vals_tmp_cap) {
+    cudaFree(h->d_vals_tmp);
+    h->d_vals_tmp = nullptr;
+    CU(cudaMalloc(&h->d_vals_tmp, sizeof(double) * nbatch * nv));
+    h->vals_tmp_cap = nbatch * nv;
+  }
+  CU(cudaMemcpyAsync(h->d_f, f_host, sizeof(double) * nbatch * h->ndof, cudaMemcpyHostToDevice, h->stream));
+  h->nbatch = nbatch;
+  h->have_state = true;
+  if ((rc = dispatch_build(h, nbatch, h->d_vals_tmp, format))) return rc;
+  CU(cudaMemcpyAsync(values_host, h->d_vals_tmp, sizeof(double) * nbatch * nv, cudaMemcpyDeviceToHost, h->stream));
+  CU(cudaStreamSynchronize(h->stream));
+  return LANDAU_OK;
+}
+
+int landau_mass(landau_t h, double shift, double *values_dev, int32_t format) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "mass: bad argument");
+  Timer t(h, LANDAU_T_MASS);
+  for (int a = 0; a < h->S; a++) {
+    const int g = h->sgrid[a];
+    const double *M = format == LANDAU_CSR ? h->d_mass_csr[g] : h->d_mass_coo[g];
+    const int64_t n = format == LANDAU_CSR ? (int64_t)h->plan.grids[g].col.size() : h->plan.grids[g].ncoo;
+    const int64_t off = format == LANDAU_CSR ? h->snnz_off[a] : h->scoo_off[a];
+    if (n == 0) continue;
+    const int blocks = (int)std::min<int64_t>((n + 255) / 256, 8LL * num_sms(h));
+    scale_copy_kernel<<<blocks, 256, 0, h->stream>>>(M, shift, n, values_dev + off);
+    h->launches++;
+    h->tlaunch[LANDAU_T_MASS]++;
+    KCHECK();
+  }
+  return LANDAU_OK;
+}
+
+int landau_point_coeffs_batched(landau_t h, int64_t nbatch, double *G_dev) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || !G_dev) return fail(h, LANDAU_EINVAL, "point_coeffs: bad argument");
+  if (!h->have_state || nbatch != h->nbatch) return fail(h, LANDAU_ESTATE, "point_coeffs: set_state first");
+  int rc = dispatch_build(h, nbatch, nullptr, LANDAU_CSR);
+  if (rc) return rc;
+  const int64_t N = h->plan.npts;
+  if (h->world == 1) {
+    CU(cudaMemcpyAsync(G_dev, h->d_G, sizeof(double) * nbatch * 5 * N, cudaMemcpyDeviceToDevice, h->stream));
+  } else {
+    const int64_t total = nbatch * 5 * N;
+    unchunk_kernel<<<(int)std::min<int64_t>((total + 255) / 256, 4096), 256, 0, h->stream>>>(h->d_G, N, h->Nc, (int)nbatch, G_dev);
+    h->launches++;
+    KCHECK();
+  }
+  return LANDAU_OK;
+}
+
+int landau_point_coeffs(landau_t h, double *G_dev) { return landau_point_coeffs_batched(h, 1, G_dev); }
+
+int landau_set_timing(landau_t h, int32_t enable) {
+  if (!h) return LANDAU_EINVAL;
+  for (auto &u : h->ev_used) {
+    h->ev_pool.push_back(u.second.first);
+    h->ev_pool.push_back(u.second.second);
+  }
+  h->ev_used.clear();
+  for (auto &x : h->tlaunch) x = 0;
+  h->timing = enable != 0;
+  return LANDAU_OK;
+}
+
+int landau_get_timing(landau_t h, double *ms, int64_t *launches) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h) return LANDAU_EINVAL;
+  CU(cudaStreamSynchronize(h->stream));
+  double acc[LANDAU_NTIMERS] = {0};
+  for (auto &u : h->ev_used) {
+    float t = 0;
+    CU(cudaEventElapsedTime(&t, u.second.first, u.second.second));
+    acc[u.first] += t;
+  }
+  for (int i = 0; i < LANDAU_NTIMERS; i++) {
+    if (ms) ms[i] = acc[i];
+    if (launches) launches[i] = h->tlaunch[i];
+  }
+  return LANDAU_OK;
+}
+
+int landau_get_launch_count(landau_t h, int64_t *count) {
+  if (!h || !count) return LANDAU_EINVAL;
+  *count = h->launches;
+  return LANDAU_OK;
+}
+
+}  // extern "C"

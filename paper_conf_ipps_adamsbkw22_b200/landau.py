@@ -1,0 +1,272 @@
+"""Thin ctypes binding of liblandau.so (include/landau.h).  Argument marshalling only: every step
+of a Jacobian build runs in the library's CUDA kernels.  PyTorch supplies device memory, the stream
+and (for the element split) the process group that broadcasts the NCCL id.
+
+There is no CPU fallback: if liblandau.so is missing or a call fails, this module raises.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liblandau.so")
+
+LANDAU_OK, LANDAU_EINVAL, LANDAU_ENOMEM, LANDAU_ECUDA, LANDAU_ENCCL, LANDAU_ESTATE, LANDAU_EUNSUPPORTED = \
+    0, -1, -2, -3, -4, -5, -6
+LANDAU_CSR, LANDAU_COO = 0, 1
+LANDAU_DIST_REPLICATE, LANDAU_DIST_BATCH, LANDAU_DIST_ELEMENTS = 0, 1, 2
+LANDAU_HOST_ONLY = -1
+TIMERS = ("field", "inner", "reduce", "element", "assemble", "mass", "allgather")
+
+_lib = None
+
+
+class LandauError(RuntimeError):
+    def __init__(self, code, where, detail=""):
+        self.code = code
+        super().__init__(f"{where}: {landau_strerror(code)} ({code}) {detail}".strip())
+
+
+class _Mesh(C.Structure):
+    _fields_ = [("ngrids", C.c_int32), ("ncells", C.POINTER(C.c_int64)), ("cells", C.POINTER(C.c_double)),
+                ("radius", C.POINTER(C.c_double))]
+
+
+class _Params(C.Structure):
+    _fields_ = [("order", C.c_int32), ("nq1d", C.c_int32), ("nspecies", C.c_int32),
+                ("mass", C.POINTER(C.c_double)), ("charge", C.POINTER(C.c_double)),
+                ("grid", C.POINTER(C.c_int32)), ("nu", C.c_double)]
+
+
+class _Dist(C.Structure):
+    _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("nccl_unique_id", C.c_void_p), ("mode", C.c_int32)]
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+                              "(no CPU fallback exists)")
+        L = C.CDLL(LIB_PATH)
+        vp, i32, i64, d = C.c_void_p, C.c_int32, C.c_int64, C.c_double
+        P64, Pd, P32 = C.POINTER(C.c_int64), C.POINTER(C.c_double), C.POINTER(C.c_int32)
+        sig = {
+            "landau_create": (C.c_int, [C.POINTER(vp), C.POINTER(_Mesh), C.POINTER(_Params), i32, vp, C.POINTER(_Dist)]),
+            "landau_destroy": (None, [vp]),
+            "landau_get_sizes": (C.c_int, [vp, P64, P64, P64, P64]),
+            "landau_get_grid_ndof": (C.c_int, [vp, i32, P64]),
+            "landau_get_nodes": (C.c_int, [vp, i32, Pd, Pd]),
+            "landau_get_points": (C.c_int, [vp, Pd, Pd, Pd]),
+            "landau_get_pattern": (C.c_int, [vp, P64, P32, P32, P32]),
+            "landau_set_state": (C.c_int, [vp, vp]),
+            "landau_set_state_batched": (C.c_int, [vp, i64, vp]),
+            "landau_jacobian": (C.c_int, [vp, vp, i32]),
+            "landau_jacobian_batched": (C.c_int, [vp, i64, vp, i32]),
+            "landau_jacobian_host": (C.c_int, [vp, i64, vp, vp, i32]),
+            "landau_mass": (C.c_int, [vp, d, vp, i32]),
+            "landau_point_coeffs": (C.c_int, [vp, vp]),
+            "landau_point_coeffs_batched": (C.c_int, [vp, i64, vp]),
+            "landau_partition": (C.c_int, [i64, i32, i32, P64, P64]),
+            "landau_nccl_unique_id": (C.c_int, [vp]),
+            "landau_set_timing": (C.c_int, [vp, i32]),
+            "landau_get_timing": (C.c_int, [vp, Pd, P64]),
+            "landau_get_launch_count": (C.c_int, [vp, P64]),
+            "landau_strerror": (C.c_char_p, [C.c_int]),
+            "landau_last_error": (C.c_char_p, [vp]),
+            "landau_version": (C.c_char_p, []),
+        }
+        for name, (res, args) in sig.items():
+            fn = getattr(L, name)
+            fn.restype = res
+            fn.argtypes = args
+        _lib = L
+    return _lib
+
+
+def landau_strerror(code):
+    return lib().landau_strerror(int(code)).decode()
+
+
+def landau_version():
+    return lib().landau_version().decode()
+
+
+def landau_partition(nelem, world, rank):
+    e0, e1 = C.c_int64(), C.c_int64()
+    rc = lib().landau_partition(int(nelem), int(world), int(rank), C.byref(e0), C.byref(e1))
+    if rc:
+        raise LandauError(rc, "landau_partition")
+    return e0.value, e1.value
+
+
+def landau_nccl_unique_id():
+    buf = (C.c_ubyte * 128)()
+    rc = lib().landau_nccl_unique_id(buf)
+    if rc:
+        raise LandauError(rc, "landau_nccl_unique_id")
+    return bytes(buf)
+
+
+def _dptr(a):
+    return a.ctypes.data_as(C.POINTER(C.c_double))
+
+
+def _tptr(t, dtype=None):
+    """device pointer of a torch tensor (contiguous, float64 unless stated)."""
+    import torch
+    if not t.is_contiguous():
+        raise ValueError("tensor must be contiguous")
+    if t.dtype != (dtype or torch.float64):
+        raise TypeError(f"expected {dtype or torch.float64}, got {t.dtype}")
+    return C.c_void_p(t.data_ptr())
+
+
+class Landau:
+    """One handle (one mesh, FE order and species set; optional batch of states)."""
+
+    def __init__(self, grids, order, mass, charge, grid_of, nu=1.0, device=0, stream=None, dist=None):
+        """grids: list of (R, cells[n][3]); mass/charge/grid_of: per species.  device =
+        LANDAU_HOST_ONLY builds only the host plan.  stream: torch.cuda.Stream or raw handle (int)."""
+        L = lib()
+        ncells = np.array([len(c) for _, c in grids], dtype=np.int64)
+        cells = np.ascontiguousarray(np.concatenate([np.asarray(c, dtype=np.float64).reshape(-1, 3) for _, c in grids]))
+        radius = np.array([R for R, _ in grids], dtype=np.float64)
+        self._keep = [ncells, cells, radius]
+        mesh = _Mesh(len(grids), ncells.ctypes.data_as(C.POINTER(C.c_int64)), _dptr(cells), _dptr(radius))
+        m = np.ascontiguousarray(mass, dtype=np.float64)
+        q = np.ascontiguousarray(charge, dtype=np.float64)
+        g = np.ascontiguousarray(grid_of, dtype=np.int32)
+        self._keep += [m, q, g]
+        prm = _Params(int(order), 0, len(m), _dptr(m), _dptr(q), g.ctypes.data_as(C.POINTER(C.c_int32)), float(nu))
+        if stream is None and device != LANDAU_HOST_ONLY:
+            import torch
+            stream = torch.cuda.current_stream(device)
+        if stream is not None and not isinstance(stream, int):
+            stream = stream.cuda_stream
+        dptr = None
+        if dist is not None:
+            uid = dist.get("nccl_unique_id")
+            self._uid = C.create_string_buffer(uid, 128) if uid else None
+            dptr = C.byref(_Dist(int(dist["rank"]), int(dist["world"]),
+                                 C.cast(self._uid, C.c_void_p) if self._uid else None, int(dist["mode"])))
+        h = C.c_void_p()
+        rc = L.landau_create(C.byref(h), C.byref(mesh), C.byref(prm), int(device), C.c_void_p(stream or 0), dptr)
+        if rc:
+            raise LandauError(rc, "landau_create", L.landau_last_error(None).decode())
+        self._h = h
+        self.device = device
+        a, b, c, d = (C.c_int64() for _ in range(4))
+        L.landau_get_sizes(h, C.byref(a), C.byref(b), C.byref(c), C.byref(d))
+        self.ndof, self.npoints, self.nnz, self.ncoo = a.value, b.value, c.value, d.value
+        self.ngrids = len(grids)
+        self.nspecies = len(m)
+        self.nbatch = 0
+
+    @classmethod
+    def from_problem(cls, prob, device=0, stream=None, dist=None):
+        return cls(prob.grids, prob.order, prob.mass, prob.charge, prob.grid_of, prob.nu, device, stream, dist)
+
+    def _check(self, rc, where):
+        if rc:
+            raise LandauError(rc, where, lib().landau_last_error(self._h).decode())
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().landau_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---- host-side queries ---------------------------------------------------------------------
+    def grid_ndof(self, g):
+        n = C.c_int64()
+        self._check(lib().landau_get_grid_ndof(self._h, g, C.byref(n)), "landau_get_grid_ndof")
+        return n.value
+
+    def nodes(self, g):
+        n = self.grid_ndof(g)
+        r, z = np.zeros(n), np.zeros(n)
+        self._check(lib().landau_get_nodes(self._h, g, _dptr(r), _dptr(z)), "landau_get_nodes")
+        return r, z
+
+    def all_nodes(self):
+        return [self.nodes(g) for g in range(self.ngrids)]
+
+    def points(self):
+        r, z, w = (np.zeros(self.npoints) for _ in range(3))
+        self._check(lib().landau_get_points(self._h, _dptr(r), _dptr(z), _dptr(w)), "landau_get_points")
+        return r, z, w
+
+    def pattern(self, coo=False):
+        if coo:
+            row = np.zeros(max(self.ncoo, 1), dtype=np.int32)
+            col = np.zeros(max(self.ncoo, 1), dtype=np.int32)
+            self._check(lib().landau_get_pattern(self._h, None, None, row.ctypes.data_as(C.POINTER(C.c_int32)),
+                                                 col.ctypes.data_as(C.POINTER(C.c_int32))), "landau_get_pattern")
+            return row[: self.ncoo], col[: self.ncoo]
+        rp = np.zeros(self.ndof + 1, dtype=np.int64)
+        col = np.zeros(max(self.nnz, 1), dtype=np.int32)
+        self._check(lib().landau_get_pattern(self._h, rp.ctypes.data_as(C.POINTER(C.c_int64)),
+                                             col.ctypes.data_as(C.POINTER(C.c_int32)), None, None), "landau_get_pattern")
+        return rp, col[: self.nnz]
+
+    # ---- device calls (torch tensors, float64, on this handle's device) --------------------------
+    def set_state(self, f):
+        self._check(lib().landau_set_state(self._h, _tptr(f)), "landau_set_state")
+        self.nbatch = 1
+
+    def set_state_batched(self, f):
+        nb = f.shape[0]
+        self._check(lib().landau_set_state_batched(self._h, nb, _tptr(f)), "landau_set_state_batched")
+        self.nbatch = nb
+
+    def jacobian(self, values, format=LANDAU_CSR):
+        self._check(lib().landau_jacobian(self._h, _tptr(values), format), "landau_jacobian")
+        return values
+
+    def jacobian_batched(self, values, format=LANDAU_CSR):
+        self._check(lib().landau_jacobian_batched(self._h, values.shape[0], _tptr(values), format),
+                    "landau_jacobian_batched")
+        return values
+
+    def jacobian_host(self, f_host, values_host, format=LANDAU_CSR):
+        """f_host: torch CPU tensor [nbatch, ndof] (pinned for async copies); values_host [nbatch, nnz]."""
+        nb = f_host.shape[0] if f_host.dim() == 2 else 1
+        self._check(lib().landau_jacobian_host(self._h, nb, C.c_void_p(f_host.data_ptr()),
+                                               C.c_void_p(values_host.data_ptr()), format), "landau_jacobian_host")
+        return values_host
+
+    def mass(self, shift, values, format=LANDAU_CSR):
+        self._check(lib().landau_mass(self._h, float(shift), _tptr(values), format), "landau_mass")
+        return values
+
+    def point_coeffs(self, G):
+        self._check(lib().landau_point_coeffs(self._h, _tptr(G)), "landau_point_coeffs")
+        return G
+
+    def point_coeffs_batched(self, G):
+        self._check(lib().landau_point_coeffs_batched(self._h, G.shape[0], _tptr(G)), "landau_point_coeffs_batched")
+        return G
+
+    def set_timing(self, enable=True):
+        self._check(lib().landau_set_timing(self._h, int(bool(enable))), "landau_set_timing")
+
+    def get_timing(self):
+        ms = np.zeros(len(TIMERS))
+        n = np.zeros(len(TIMERS), dtype=np.int64)
+        self._check(lib().landau_get_timing(self._h, _dptr(ms), n.ctypes.data_as(C.POINTER(C.c_int64))),
+                    "landau_get_timing")
+        return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(TIMERS)}
+
+    def launch_count(self):
+        n = C.c_int64()
+        self._check(lib().landau_get_launch_count(self._h, C.byref(n)), "landau_get_launch_count")
+        return n.value

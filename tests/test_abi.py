@@ -1,0 +1,127 @@
+"""CPU tests of the C ABI (no GPU): the library loads and exports every symbol include/landau.h
+declares; the host-side plan (step a-0: nodes, DOF numbering, points, CSR/COO patterns) agrees with
+the independent oracle; invalid meshes are rejected; the element partition is a partition."""
+import ctypes
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+from paper_conf_ipps_adamsbkw22_b200 import inputs
+from paper_conf_ipps_adamsbkw22_b200 import landau as L
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    txt = open(os.path.join(ROOT, "include", "landau.h")).read()
+    return sorted(set(re.findall(r"^\s*(?:int|void|const char \*)\s*(landau_\w+)\s*\(", txt, re.M)))
+
+
+def test_library_exports_every_declared_symbol():
+    syms = header_symbols()
+    assert len(syms) >= 20
+    out = subprocess.run(["nm", "-D", "--defined-only", L.LIB_PATH], capture_output=True, text=True, check=True).stdout
+    exported = set(re.findall(r"\bT (landau_\w+)", out))
+    missing = [s for s in syms if s not in exported]
+    assert not missing, missing
+    lib = ctypes.CDLL(L.LIB_PATH)
+    for s in syms:
+        getattr(lib, s)
+
+
+def test_strerror_and_version():
+    assert "invalid" in L.landau_strerror(L.LANDAU_EINVAL)
+    assert "sm_100a" in L.landau_version()
+
+
+@pytest.mark.parametrize("nelem,world", [(68, 1), (68, 2), (4352, 8), (7, 3), (3, 8)])
+def test_partition_covers_cells_once(nelem, world):
+    seen = np.zeros(nelem, dtype=int)
+    for r in range(world):
+        e0, e1 = L.landau_partition(nelem, world, r)
+        assert 0 <= e0 <= e1 <= nelem
+        seen[e0:e1] += 1
+    assert np.all(seen == 1)
+    with pytest.raises(L.LandauError):
+        L.landau_partition(nelem, world, world)
+
+
+def _host(prob):
+    return L.Landau.from_problem(prob, device=L.LANDAU_HOST_ONLY)
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3"])
+def test_host_plan_matches_oracle(cfg):
+    from oracle.oracle import Oracle
+    prob = inputs.CONFIGS[cfg]()
+    h = _host(prob)
+    o = Oracle(prob)
+    assert (h.ndof, h.npoints, h.nnz, h.ncoo) == (o.ndof, o.npoints, o.nnz, o.ncoo)
+    for g in range(len(prob.grids)):
+        hr, hz = h.nodes(g)
+        orr, oz = o.nodes(g)
+        np.testing.assert_allclose(hr, orr, rtol=0, atol=1e-14 * prob.grids[g][0])
+        np.testing.assert_allclose(hz, oz, rtol=0, atol=1e-14 * prob.grids[g][0])
+    hr, hz, hw = h.points()
+    orr, oz, ow = o.points()
+    np.testing.assert_allclose(hr, orr, rtol=1e-15, atol=0)
+    np.testing.assert_allclose(hz, oz, rtol=1e-15, atol=1e-16)
+    np.testing.assert_allclose(hw, ow, rtol=4e-15)
+    rp, col = h.pattern()
+    orp, ocol = o.pattern()
+    np.testing.assert_array_equal(rp, orp)
+    np.testing.assert_array_equal(col, ocol)
+    row, col = h.pattern(coo=True)
+    orow, ocol = o.coo_pattern()
+    np.testing.assert_array_equal(row, orow)
+    np.testing.assert_array_equal(col, ocol)
+
+
+def test_host_plan_C5_sizes():
+    prob = inputs.config5()
+    h = _host(prob)
+    assert h.npoints == 108800 and len(prob.grids[0][1]) == 4352
+
+
+def test_invalid_meshes_rejected():
+    R = 1.0
+    base = inputs.origin_chain(R, 2)
+    c0 = [c for c in base if c[0] == 0.0 and c[1] == 0.0][0]
+    unbalanced = [c for c in base if c != c0] + inputs.refine_uniform([c0], 2)
+    bad = {
+        "unbalanced": unbalanced,
+        "overlap": base + [(0.0, 0.0, R / 8)],
+        "hole": base[1:],
+        "off-lattice": [(0.0, -R, R), (0.0, 0.0, R / 2), (R / 2, 0.0, R / 2), (0.1, R / 2, R / 2), (R / 2, R / 2, R / 2)],
+        "negative r": [(-R, -R, R), (0.0, 0.0, R)],
+    }
+    for name, cells in bad.items():
+        prob = inputs.Problem("bad", 3, [(R, cells)], [inputs.Species("e", 1.0, -1.0, 0)], fmix=[[(1, 1, 0)]])
+        with pytest.raises(L.LandauError) as ei:
+            _host(prob)
+        assert ei.value.code == L.LANDAU_EINVAL, name
+    prob = inputs.Problem("ok", 5, [(R, base)], [inputs.Species("e", 1.0, -1.0, 0)], fmix=[[(1, 1, 0)]])
+    with pytest.raises(L.LandauError):
+        _host(prob)                       # order 5 unsupported
+    prob = inputs.Problem("ok", 3, [(R, base)], [inputs.Species("e", -1.0, -1.0, 0)], fmix=[[(1, 1, 0)]])
+    with pytest.raises(L.LandauError):
+        _host(prob)                       # negative mass
+
+
+def test_host_only_handle_refuses_device_calls():
+    h = _host(inputs.config1())
+    lib = L.lib()
+    rc = lib.landau_mass(h._h, 1.0, ctypes.c_void_p(16), L.LANDAU_CSR)
+    assert rc == L.LANDAU_EUNSUPPORTED
+
+
+def test_create_without_gpu_fails_loudly():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(L.LandauError) as ei:
+        L.Landau.from_problem(inputs.config1(), device=0, stream=0)
+    assert ei.value.code == L.LANDAU_ECUDA
