@@ -13,6 +13,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -32,80 +33,115 @@ __constant__ double c_dxi[kMaxNb * kMaxNb];
 __constant__ double c_deta[kMaxNb * kMaxNb];
 
 // ------------------------------------------------------------------------------------------------
-// N1: point fields.  One block handles EPB cells; thread (cell, q) evaluates its point.
-// The per-grid species sums T_D = sum e^2 f, T_K = sum e^2/m grad f are linear in f, so the
-// combined element coefficients gD_a = sum_b e_b^2 f_b,a and gK_a = sum_b e_b^2/m_b f_b,a are formed
-// first (one pass over the extraction list), then interpolated once.
+// Reference tables in shared memory: thread-varying indices into __constant__ memory serialise, so
+// kernels that index the tables by thread copy them to shared memory once per block.
+// ------------------------------------------------------------------------------------------------
+template <int NB>
+__device__ __forceinline__ void load_tables(double (*s_phi)[NB], double (*s_dxi)[NB], double (*s_deta)[NB]) {
+  for (int i = threadIdx.x; i < NB * NB; i += blockDim.x) {
+    s_phi[i / NB][i % NB] = c_phi[i];
+    s_dxi[i / NB][i % NB] = c_dxi[i];
+    s_deta[i / NB][i % NB] = c_deta[i];
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// N1: point fields.  A block handles EPB cells at a time (grid-stride over cells x batch); thread
+// (cell, a) first forms the combined element coefficients gD_a = sum_b e_b^2 f_b,a and
+// gK_a = sum_b e_b^2/m_b f_b,a through the extraction list (T_D, T_K are linear in f), then thread
+// (cell, q) interpolates: w T_D, w T_Kr, w T_Kz at its point.
 // ------------------------------------------------------------------------------------------------
 template <int NB, int EPB>
-__global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int64_t ndof_total, const double *__restrict__ f,
+__global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbatch, int64_t ndof_total,
+                                                         const double *__restrict__ f,
                                                          const int32_t *__restrict__ ext_ptr,
                                                          const int32_t *__restrict__ ext_dof,
                                                          const double *__restrict__ ext_w,
                                                          const int *__restrict__ cell_grid,
                                                          const double *__restrict__ cell_h, const double *__restrict__ pw,
                                                          double *__restrict__ wT, int64_t npts) {
+  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
   __shared__ double gD[EPB][NB], gK[EPB][NB];
-  const int b = blockIdx.y;
+  load_tables<NB>(s_phi, s_dxi, s_deta);
   const int el = threadIdx.x / NB, a = threadIdx.x % NB;
-  const int64_t e = (int64_t)blockIdx.x * EPB + el;
-  const double *fb = f + (int64_t)b * ndof_total;
-  if (e < ncell) {
-    const int g = cell_grid[e];
-    const int32_t k0 = ext_ptr[e * NB + a], k1 = ext_ptr[e * NB + a + 1];
-    double sD = 0.0, sK = 0.0;
-    for (int s = 0; s < c_sp.grid_nsp[g]; s++) {
-      const int sp = c_sp.grid_sp[g][s];
-      const double *fs = fb + c_sp.soff[sp];
-      double v = 0.0;
-      for (int32_t k = k0; k < k1; k++) v = fma(ext_w[k], __ldg(fs + ext_dof[k]), v);
-      sD = fma(c_sp.e2[sp], v, sD);
-      sK = fma(c_sp.e2m[sp], v, sK);
+  const int64_t nchunks = (ncell + EPB - 1) / EPB;
+  for (int64_t it = blockIdx.x; it < nchunks * nbatch; it += gridDim.x) {
+    const int b = (int)(it / nchunks);
+    const int64_t e = (it % nchunks) * EPB + el;
+    const double *fb = f + (int64_t)b * ndof_total;
+    __syncthreads();
+    if (e < ncell) {
+      const int g = cell_grid[e];
+      const int32_t k0 = ext_ptr[e * NB + a], k1 = ext_ptr[e * NB + a + 1];
+      double sD = 0.0, sK = 0.0;
+      for (int s = 0; s < c_sp.grid_nsp[g]; s++) {
+        const int sp = c_sp.grid_sp[g][s];
+        const double *fs = fb + c_sp.soff[sp];
+        double v = 0.0;
+        for (int32_t k = k0; k < k1; k++) v = fma(ext_w[k], __ldg(fs + ext_dof[k]), v);
+        sD = fma(c_sp.e2[sp], v, sD);
+        sK = fma(c_sp.e2m[sp], v, sK);
+      }
+      gD[el][a] = sD;
+      gK[el][a] = sK;
     }
-    gD[el][a] = sD;
-    gK[el][a] = sK;
-  }
-  __syncthreads();
-  if (e < ncell) {
-    const int q = a;   // NQP == NB for (p+1)^2 Gauss points
-    const int64_t pt = e * NB + q;
-    double td = 0.0, tr = 0.0, tz = 0.0;
+    __syncthreads();
+    if (e < ncell) {
+      const int q = a;   // NQP == NB for (p+1)^2 Gauss points
+      const int64_t pt = e * NB + q;
+      double td = 0.0, tr = 0.0, tz = 0.0;
 #pragma unroll
-    for (int k = 0; k < NB; k++) {
-      td = fma(c_phi[q * NB + k], gD[el][k], td);
-      tr = fma(c_dxi[q * NB + k], gK[el][k], tr);
-      tz = fma(c_deta[q * NB + k], gK[el][k], tz);
+      for (int k = 0; k < NB; k++) {
+        td = fma(s_phi[q][k], gD[el][k], td);
+        tr = fma(s_dxi[q][k], gK[el][k], tr);
+        tz = fma(s_deta[q][k], gK[el][k], tz);
+      }
+      const double w = pw[pt], ws = w * (2.0 / cell_h[e]);
+      double *o = wT + (int64_t)b * 3 * npts;
+      o[pt] = w * td;
+      o[npts + pt] = ws * tr;
+      o[2 * npts + pt] = ws * tz;
     }
-    const double s = 2.0 / cell_h[e];
-    const double w = pw[pt];
-    double *o = wT + (int64_t)b * 3 * npts;
-    o[pt] = w * td;
-    o[npts + pt] = w * s * tr;
-    o[2 * npts + pt] = w * s * tz;
   }
 }
 
 // ------------------------------------------------------------------------------------------------
-// N2: inner integral.  Block = TB threads x TPT targets each; sources streamed through shared
-// memory in tiles of TB (all lanes read the same source: broadcast).  blockIdx.y = split of the
-// source range (split-j), blockIdx.z = batch item.  out = [batch][nsplit][5][nt] partials.
+// N2: inner integral.  Work is warp-granular: a warp owns 32*TPT consecutive targets of one batch
+// item and one split of the source range (split-j), so the target tiling never pads across batch
+// items.  Sources are staged per warp through shared memory, 32 at a time (one per lane), and every
+// lane then reads the same source (broadcast LDS.128).  Coefficients of the elliptic fits live in
+// registers (see kernels.cuh).  out = [batch][nsplit][5][nt] partials (or G when nsplit == 1).
 // ------------------------------------------------------------------------------------------------
 constexpr int kInnerTB = 128;
+constexpr int kInnerWarps = kInnerTB / 32;
 
-template <int TPT>
-__global__ void __launch_bounds__(kInnerTB) inner_kernel(int64_t N, int64_t t0, int64_t nt, int64_t split_len,
-                                                          const double *__restrict__ pr, const double *__restrict__ pz,
-                                                          const double *__restrict__ wT, double *__restrict__ out,
-                                                          int64_t out_bstride) {
-  __shared__ double sr[kInnerTB], sz[kInnerTB], sd[kInnerTB], skr[kInnerTB], skz[kInnerTB];
-  const int b = blockIdx.z, split = blockIdx.y, nsplit = gridDim.y;
-  const double *wb = wT + (int64_t)b * 3 * N;
+template <int TPT, int MINB>
+__global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_t t0, int64_t nt, int64_t split_len,
+                                                             int nsplit, int64_t wtiles, int64_t nitems,
+                                                             const double *__restrict__ pr, const double *__restrict__ pz,
+                                                             const double *__restrict__ wT, double *__restrict__ out,
+                                                             int64_t out_bstride) {
+  __shared__ double2 s_rz[kInnerWarps][32], s_w[kInnerWarps][32];
+  __shared__ double s_wz[kInnerWarps][32];
+  __shared__ double s_coef[kNumPairCoef];
+  stage_pair_coef(s_coef);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, cf);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t item = (int64_t)blockIdx.x * kInnerWarps + wid;
+  if (item >= nitems) return;   // whole warp: no block-level barrier follows
+  const int64_t b = item / (nsplit * wtiles);
+  const int64_t rem = item % (nsplit * wtiles);
+  const int split = (int)(rem / wtiles);
+  const int64_t wt = rem % wtiles;
+  const double *wb = wT + b * 3 * N;
   int64_t ti[TPT];
   double tr[TPT], tz[TPT];
   Acc5 acc[TPT];
 #pragma unroll
   for (int t = 0; t < TPT; t++) {
-    ti[t] = (int64_t)blockIdx.x * kInnerTB * TPT + t * kInnerTB + threadIdx.x;
+    ti[t] = wt * 32 * TPT + t * 32 + lane;
     const int64_t gi = t0 + (ti[t] < nt ? ti[t] : nt - 1);
     tr[t] = pr[gi];
     tz[t] = pz[gi];
@@ -113,25 +149,25 @@ __global__ void __launch_bounds__(kInnerTB) inner_kernel(int64_t N, int64_t t0, 
   }
   const int64_t j0 = (int64_t)split * split_len;
   const int64_t j1 = min(N, j0 + split_len);
-  for (int64_t jt = j0; jt < j1; jt += kInnerTB) {
-    const int64_t j = jt + threadIdx.x;
+  for (int64_t jt = j0; jt < j1; jt += 32) {
+    const int64_t j = jt + lane;
+    __syncwarp();
     if (j < j1) {
-      sr[threadIdx.x] = pr[j];
-      sz[threadIdx.x] = pz[j];
-      sd[threadIdx.x] = wb[j];
-      skr[threadIdx.x] = wb[N + j];
-      skz[threadIdx.x] = wb[2 * N + j];
+      s_rz[wid][lane] = make_double2(pr[j], pz[j]);
+      s_w[wid][lane] = make_double2(wb[j], wb[N + j]);
+      s_wz[wid][lane] = wb[2 * N + j];
     }
-    __syncthreads();
-    const int n = (int)min((int64_t)kInnerTB, j1 - jt);
+    __syncwarp();
+    const int n = (int)min((int64_t)32, j1 - jt);
+#pragma unroll 2
     for (int k = 0; k < n; k++) {
-      const double rb = sr[k], zb = sz[k], wd = sd[k], wkr = skr[k], wkz = skz[k];
+      const double2 rz = s_rz[wid][k], w = s_w[wid][k];
+      const double wkz = s_wz[wid][k];
 #pragma unroll
-      for (int t = 0; t < TPT; t++) landau_pair(tr[t], tz[t], rb, zb, wd, wkr, wkz, acc[t]);
+      for (int t = 0; t < TPT; t++) landau_pair(tr[t], tz[t], rz.x, rz.y, w.x, w.y, wkz, cf, acc[t]);
     }
-    __syncthreads();
   }
-  double *o = out + (int64_t)b * out_bstride + (int64_t)split * 5 * nt;
+  double *o = out + b * out_bstride + (int64_t)split * 5 * nt;
 #pragma unroll
   for (int t = 0; t < TPT; t++) {
     if (ti[t] < nt) {
@@ -142,7 +178,6 @@ __global__ void __launch_bounds__(kInnerTB) inner_kernel(int64_t N, int64_t t0, 
       o[4 * nt + ti[t]] = acc[t].kz;
     }
   }
-  (void)nsplit;
 }
 
 // N2r: G[b][c][i] = sum_{s = 0..nsplit-1} part[b][s][c][i] in fixed order (deterministic).
@@ -159,8 +194,8 @@ __global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__
 }
 
 // ------------------------------------------------------------------------------------------------
-// N3: element matrices (species independent).  One block per (cell, batch); thread (k, l).
-//   C^D[k,l] = (2/h)^2 sum_q w_q (gk . G_D(q) . gl),  C^K[k,l] = (2/h) sum_q w_q (gk . G_K(q)) phi_l(q)
+// N3: element matrices (species independent).  Grid-stride over (cell, batch); thread (k, l).
+//   C^D[k,l] = (2/h)^2 sum_q (gk . w_q G_D(q) . gl),  C^K[k,l] = (2/h) sum_q (gk . w_q G_K(q)) phi_l(q)
 // with gk the reference gradients.  G is read in the chunked layout
 //   G[((i / Nc) * nbatch + b) * 5 + c][i % Nc]     (Nc = N when not distributed).
 // ------------------------------------------------------------------------------------------------
@@ -168,35 +203,39 @@ template <int NB>
 __global__ void __launch_bounds__(NB * NB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
                                                             int nbatch, const double *__restrict__ pw,
                                                             const double *__restrict__ cell_h, double *__restrict__ Cbuf) {
-  __shared__ double sG[5][NB], sw[NB];
-  const int64_t e = blockIdx.x;
-  const int b = blockIdx.y;
+  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
+  __shared__ double sA[5][NB];
+  load_tables<NB>(s_phi, s_dxi, s_deta);
   const int tid = threadIdx.x;
-  if (tid < NB) {
-    const int64_t i = e * NB + tid;
-    const int64_t chunk = i / Nc, off = i % Nc;
-    const double *Gb = G + ((chunk * nbatch + b) * 5) * Nc + off;
-#pragma unroll
-    for (int c = 0; c < 5; c++) sG[c][tid] = Gb[c * Nc];
-    sw[tid] = pw[i];
-  }
-  __syncthreads();
   const int k = tid / NB, l = tid % NB;
-  double cd = 0.0, ck = 0.0;
+  for (int64_t it = blockIdx.x; it < ncell * nbatch; it += gridDim.x) {
+    const int b = (int)(it / ncell);
+    const int64_t e = it % ncell;
+    __syncthreads();
+    if (tid < NB) {
+      const int64_t i = e * NB + tid;
+      const int64_t chunk = i / Nc, off = i % Nc;
+      const double *Gb = G + ((chunk * nbatch + b) * 5) * Nc + off;
+      const double w = pw[i];
+#pragma unroll
+      for (int c = 0; c < 5; c++) sA[c][tid] = w * Gb[c * Nc];
+    }
+    __syncthreads();
+    double cd = 0.0, ck = 0.0;
 #pragma unroll 4
-  for (int q = 0; q < NB; q++) {
-    const double gkr = c_dxi[q * NB + k], gkz = c_deta[q * NB + k];
-    const double glr = c_dxi[q * NB + l], glz = c_deta[q * NB + l], pl = c_phi[q * NB + l];
-    const double Grr = sG[0][q], Grz = sG[1][q], Gzz = sG[2][q], Kr = sG[3][q], Kz = sG[4][q];
-    const double w = sw[q];
-    const double vd = gkr * fma(Grr, glr, Grz * glz) + gkz * fma(Grz, glr, Gzz * glz);
-    cd = fma(w, vd, cd);
-    ck = fma(w * fma(gkr, Kr, gkz * Kz), pl, ck);
+    for (int q = 0; q < NB; q++) {
+      const double gkr = s_dxi[q][k], gkz = s_deta[q][k];
+      const double glr = s_dxi[q][l], glz = s_deta[q][l], pl = s_phi[q][l];
+      const double Arr = sA[0][q], Arz = sA[1][q], Azz = sA[2][q], Kr = sA[3][q], Kz = sA[4][q];
+      cd = fma(gkr, fma(Arr, glr, Arz * glz), cd);
+      cd = fma(gkz, fma(Arz, glr, Azz * glz), cd);
+      ck = fma(fma(gkr, Kr, gkz * Kz), pl, ck);
+    }
+    const double s = 2.0 / cell_h[e];
+    double *o = Cbuf + ((int64_t)b * ncell + e) * 2 * NB * NB;
+    o[tid] = cd * s * s;
+    o[NB * NB + tid] = ck * s;
   }
-  const double s = 2.0 / cell_h[e];
-  double *o = Cbuf + ((int64_t)b * ncell + e) * 2 * NB * NB;
-  o[tid] = cd * s * s;
-  o[NB * NB + tid] = ck * s;
 }
 
 // Mass element matrices (create time): M[k,l] = sum_q w_q phi_k phi_l, stored in the [cell][2][NB^2]
@@ -204,10 +243,13 @@ __global__ void __launch_bounds__(NB * NB) element_kernel(int64_t ncell, const d
 template <int NB>
 __global__ void __launch_bounds__(NB * NB) mass_element_kernel(int64_t ncell, const double *__restrict__ pw,
                                                                  double *__restrict__ Mbuf) {
+  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
+  load_tables<NB>(s_phi, s_dxi, s_deta);
+  __syncthreads();
   const int64_t e = blockIdx.x;
   const int tid = threadIdx.x, k = tid / NB, l = tid % NB;
   double m = 0.0;
-  for (int q = 0; q < NB; q++) m = fma(pw[e * NB + q] * c_phi[q * NB + k], c_phi[q * NB + l], m);
+  for (int q = 0; q < NB; q++) m = fma(pw[e * NB + q] * s_phi[q][k], s_phi[q][l], m);
   Mbuf[e * 2 * NB * NB + tid] = m;
   Mbuf[e * 2 * NB * NB + NB * NB + tid] = 0.0;
 }
@@ -461,20 +503,6 @@ int bind_constants(landau_t h) {
 // ---------------------------------------------------------------------------------------------
 // launch helpers
 // ---------------------------------------------------------------------------------------------
-template <int NB>
-int launch_field(landau_t h, int64_t nbatch) {
-  constexpr int EPB = NB == 9 ? 8 : (NB == 16 ? 8 : 4);
-  const Plan &P = h->plan;
-  dim3 grid((unsigned)((P.ncell + EPB - 1) / EPB), (unsigned)nbatch);
-  Timer t(h, LANDAU_T_FIELD);
-  field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, h->ndof, h->d_f, h->d_ext_ptr, h->d_ext_dof, h->d_ext_w,
-                                                          h->d_cell_grid, h->d_h, h->d_w, h->d_wT, P.npts);
-  h->launches++;
-  h->tlaunch[LANDAU_T_FIELD]++;
-  KCHECK();
-  return LANDAU_OK;
-}
-
 int num_sms(landau_t h) {
   static int sms[64] = {0};
   int &s = sms[h->device & 63];
@@ -482,15 +510,36 @@ int num_sms(landau_t h) {
   return s ? s : 148;
 }
 
+template <int NB>
+int launch_field(landau_t h, int64_t nbatch) {
+  constexpr int EPB = NB == 9 ? 8 : (NB == 16 ? 8 : 4);
+  const Plan &P = h->plan;
+  const int64_t items = (P.ncell + EPB - 1) / EPB * nbatch;
+  const unsigned grid = (unsigned)std::min<int64_t>(items, 8LL * num_sms(h));
+  Timer t(h, LANDAU_T_FIELD);
+  field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->d_f, h->d_ext_ptr, h->d_ext_dof,
+                                                          h->d_ext_w, h->d_cell_grid, h->d_h, h->d_w, h->d_wT, P.npts);
+  h->launches++;
+  h->tlaunch[LANDAU_T_FIELD]++;
+  KCHECK();
+  return LANDAU_OK;
+}
+
+
 int launch_inner(landau_t h, int64_t nbatch) {
   const Plan &P = h->plan;
   const int64_t N = P.npts;
   const int64_t t0 = h->e0 * P.nqp, nt = (h->e1 - h->e0) * P.nqp;
-  constexpr int TPT = 1;
-  const int64_t tblocks = (nt + kInnerTB * TPT - 1) / (kInnerTB * TPT);
-  // split-j so that small problems still fill the machine: aim for >= 8 blocks per SM
-  const int64_t want = 8LL * num_sms(h);
-  int64_t nsplit = std::max<int64_t>(1, (want + tblocks * nbatch - 1) / (tblocks * nbatch));
+  // inner-kernel variant (targets per thread, min blocks per SM); LANDAU_INNER_VARIANT overrides
+  static const int variant = [] {
+    const char *e = getenv("LANDAU_INNER_VARIANT");
+    return e ? atoi(e) : 1;
+  }();
+  const int TPT = variant == 0 ? 1 : (variant == 4 ? 4 : 2);
+  const int64_t wtiles = (nt + 32 * TPT - 1) / (32 * TPT);
+  // split-j so that small problems still fill the machine: aim for >= 12 warps per SM
+  const int64_t want = 12LL * num_sms(h);
+  int64_t nsplit = std::max<int64_t>(1, (want + wtiles * nbatch - 1) / (wtiles * nbatch));
   nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, N / 32));
   const int64_t split_len = (N + nsplit - 1) / nsplit;
   nsplit = (N + split_len - 1) / split_len;
@@ -513,8 +562,18 @@ int launch_inner(landau_t h, int64_t nbatch) {
   }
   {
     Timer t(h, LANDAU_T_INNER);
-    dim3 grid((unsigned)tblocks, (unsigned)nsplit, (unsigned)nbatch);
-    inner_kernel<TPT><<<grid, kInnerTB, 0, h->stream>>>(N, t0, nt, split_len, h->d_r, h->d_z, h->d_wT, out, out_bstride);
+    const int64_t nitems = nbatch * nsplit * wtiles;
+    const unsigned grid = (unsigned)((nitems + kInnerWarps - 1) / kInnerWarps);
+#define LAUNCH_INNER(T, M)                                                                              \
+  inner_kernel<T, M><<<grid, kInnerTB, 0, h->stream>>>(N, t0, nt, split_len, (int)nsplit, wtiles, nitems, h->d_r, h->d_z, \
+                                                      h->d_wT, out, out_bstride)
+    switch (variant) {
+      case 0: LAUNCH_INNER(1, 3); break;
+      case 1: LAUNCH_INNER(2, 2); break;
+      case 4: LAUNCH_INNER(4, 2); break;
+      default: LAUNCH_INNER(2, 3); break;
+    }
+#undef LAUNCH_INNER
     h->launches++;
     h->tlaunch[LANDAU_T_INNER]++;
     KCHECK();
@@ -541,7 +600,7 @@ template <int NB>
 int launch_element(landau_t h, int64_t nbatch) {
   const Plan &P = h->plan;
   Timer t(h, LANDAU_T_ELEMENT);
-  dim3 grid((unsigned)P.ncell, (unsigned)nbatch);
+  const unsigned grid = (unsigned)std::min<int64_t>(P.ncell * nbatch, (NB == 25 ? 3LL : 6LL) * num_sms(h));
   element_kernel<NB><<<grid, NB * NB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, h->d_w, h->d_h, h->d_C);
   h->launches++;
   h->tlaunch[LANDAU_T_ELEMENT]++;
