@@ -27,21 +27,21 @@ using namespace landau;
 
 namespace {
 
-__constant__ SpeciesConst c_sp;
-__constant__ double c_phi[kMaxNb * kMaxNb];
-__constant__ double c_dxi[kMaxNb * kMaxNb];
-__constant__ double c_deta[kMaxNb * kMaxNb];
+// Per-handle data reaches the kernels as arguments (species table by value, basis tables through
+// global memory) -- no per-handle __constant__ state, so several handles can share a device and a
+// captured CUDA graph stays valid.
 
 // ------------------------------------------------------------------------------------------------
 // Reference tables in shared memory: thread-varying indices into __constant__ memory serialise, so
 // kernels that index the tables by thread copy them to shared memory once per block.
 // ------------------------------------------------------------------------------------------------
 template <int NB>
-__device__ __forceinline__ void load_tables(double (*s_phi)[NB], double (*s_dxi)[NB], double (*s_deta)[NB]) {
+__device__ __forceinline__ void load_tables(const double *__restrict__ tab, double (*s_phi)[NB], double (*s_dxi)[NB],
+                                            double (*s_deta)[NB]) {
   for (int i = threadIdx.x; i < NB * NB; i += blockDim.x) {
-    s_phi[i / NB][i % NB] = c_phi[i];
-    s_dxi[i / NB][i % NB] = c_dxi[i];
-    s_deta[i / NB][i % NB] = c_deta[i];
+    s_phi[i / NB][i % NB] = tab[i];
+    s_dxi[i / NB][i % NB] = tab[NB * NB + i];
+    s_deta[i / NB][i % NB] = tab[2 * NB * NB + i];
   }
 }
 
@@ -59,10 +59,12 @@ __global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbat
                                                          const double *__restrict__ ext_w,
                                                          const int *__restrict__ cell_grid,
                                                          const double *__restrict__ cell_h, const double *__restrict__ pw,
+                                                         const double *__restrict__ tab, const SpeciesConst sp_,
                                                          double *__restrict__ wT, int64_t npts) {
   __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
   __shared__ double gD[EPB][NB], gK[EPB][NB];
-  load_tables<NB>(s_phi, s_dxi, s_deta);
+  load_tables<NB>(tab, s_phi, s_dxi, s_deta);
+  const SpeciesConst &c_sp = sp_;
   const int el = threadIdx.x / NB, a = threadIdx.x % NB;
   const int64_t nchunks = (ncell + EPB - 1) / EPB;
   for (int64_t it = blockIdx.x; it < nchunks * nbatch; it += gridDim.x) {
@@ -202,10 +204,11 @@ __global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__
 template <int NB>
 __global__ void __launch_bounds__(NB * NB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
                                                             int nbatch, const double *__restrict__ pw,
-                                                            const double *__restrict__ cell_h, double *__restrict__ Cbuf) {
+                                                            const double *__restrict__ cell_h, const double *__restrict__ tab,
+                                                            double *__restrict__ Cbuf) {
   __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
   __shared__ double sA[5][NB];
-  load_tables<NB>(s_phi, s_dxi, s_deta);
+  load_tables<NB>(tab, s_phi, s_dxi, s_deta);
   const int tid = threadIdx.x;
   const int k = tid / NB, l = tid % NB;
   for (int64_t it = blockIdx.x; it < ncell * nbatch; it += gridDim.x) {
@@ -242,9 +245,9 @@ __global__ void __launch_bounds__(NB * NB) element_kernel(int64_t ncell, const d
 // layout (second half zero) so the same gather maps apply.
 template <int NB>
 __global__ void __launch_bounds__(NB * NB) mass_element_kernel(int64_t ncell, const double *__restrict__ pw,
-                                                                 double *__restrict__ Mbuf) {
+                                                                 const double *__restrict__ tab, double *__restrict__ Mbuf) {
   __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
-  load_tables<NB>(s_phi, s_dxi, s_deta);
+  load_tables<NB>(tab, s_phi, s_dxi, s_deta);
   __syncthreads();
   const int64_t e = blockIdx.x;
   const int tid = threadIdx.x, k = tid / NB, l = tid % NB;
@@ -264,11 +267,13 @@ struct GatherDev {
   const int32_t *idx;
   const double *w;
   int64_t nslots;
-  int64_t out_off[kMaxSpecies];   // output offset per species slot on this grid
+  int nsp;                        // species on this grid
+  int64_t out_off[kMaxSpecies];   // output offset per species on this grid
+  double fD[kMaxSpecies], fK[kMaxSpecies];   // a-3 species factors
 };
 
 template <int NB>
-__global__ void assemble_kernel(GatherDev gm, int grid, const double *__restrict__ Cbuf, int64_t cbuf_bstride,
+__global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ Cbuf, int64_t cbuf_bstride,
                                 double *__restrict__ out, int64_t out_bstride) {
   const int b = blockIdx.y;
   const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -283,11 +288,7 @@ __global__ void assemble_kernel(GatherDev gm, int grid, const double *__restrict
     sK = fma(w, C[i + NB * NB], sK);
   }
   double *o = out + (int64_t)b * out_bstride;
-  const int ns = c_sp.grid_nsp[grid];
-  for (int q = 0; q < ns; q++) {
-    const int sp = c_sp.grid_sp[grid][q];
-    o[gm.out_off[q] + s] = fma(c_sp.fD[sp], sD, c_sp.fK[sp] * sK);
-  }
+  for (int q = 0; q < gm.nsp; q++) o[gm.out_off[q] + s] = fma(gm.fD[q], sD, gm.fK[q] * sK);
 }
 
 // mass gather (create time): out[s] = sum_k w_k M[idx_k]
@@ -375,7 +376,7 @@ struct landau_s {
   int64_t e0 = 0, e1 = 0, chunk_cells = 0, Nc = 0;
   ncclComm_ comm = nullptr;
   // device: static
-  double *d_r = nullptr, *d_z = nullptr, *d_w = nullptr, *d_h = nullptr;
+  double *d_r = nullptr, *d_z = nullptr, *d_w = nullptr, *d_h = nullptr, *d_tab = nullptr;
   int *d_cell_grid = nullptr;
   int32_t *d_ext_ptr = nullptr, *d_ext_dof = nullptr;
   double *d_ext_w = nullptr;
@@ -402,6 +403,16 @@ struct landau_s {
   int64_t tlaunch[LANDAU_NTIMERS] = {0};
   int64_t launches = 0;
   bool host_only = false;
+  // CUDA graphs of whole builds (no per-stage timers): key (nbatch, format, out) -> exec, kernels
+  struct GraphEntry {
+    int64_t nbatch;
+    int format;
+    double *out;
+    cudaGraphExec_t exec;
+    int64_t kernels;
+  };
+  std::vector<GraphEntry> graphs;
+  bool use_graphs = true;
   std::string err;
 };
 
@@ -463,9 +474,15 @@ struct Timer {
   }
 };
 
+void drop_graphs(landau_t h) {
+  for (auto &g : h->graphs) cudaGraphExecDestroy(g.exec);
+  h->graphs.clear();
+}
+
 int ensure_workspace(landau_t h, int64_t nbatch) {
   const int64_t N = h->plan.npts, Ne = h->plan.ncell, nb = h->plan.nb;
   if (nbatch <= h->cap) return LANDAU_OK;
+  drop_graphs(h);
   cudaFree(h->d_f);
   cudaFree(h->d_wT);
   cudaFree(h->d_G);
@@ -477,27 +494,6 @@ int ensure_workspace(landau_t h, int64_t nbatch) {
   CU(cudaMalloc(&h->d_C, sizeof(double) * nbatch * Ne * 2 * nb * nb));
   h->cap = nbatch;
   return LANDAU_OK;
-}
-
-int set_constants(landau_t h) {
-  const Plan &P = h->plan;
-  CU(cudaMemcpyToSymbolAsync(c_sp, &h->spc, sizeof(SpeciesConst), 0, cudaMemcpyHostToDevice, h->stream));
-  CU(cudaMemcpyToSymbolAsync(c_phi, P.tab_phi.data(), sizeof(double) * P.tab_phi.size(), 0, cudaMemcpyHostToDevice, h->stream));
-  CU(cudaMemcpyToSymbolAsync(c_dxi, P.tab_dxi.data(), sizeof(double) * P.tab_dxi.size(), 0, cudaMemcpyHostToDevice, h->stream));
-  CU(cudaMemcpyToSymbolAsync(c_deta, P.tab_deta.data(), sizeof(double) * P.tab_deta.size(), 0, cudaMemcpyHostToDevice, h->stream));
-  return LANDAU_OK;
-}
-
-// Constant memory is per device & module, not per handle: re-upload when another handle (different
-// mesh/order/species) was the last one to set it on this device.
-const landau_s *g_const_owner[64] = {nullptr};
-std::mutex g_const_mu;
-int bind_constants(landau_t h) {
-  std::lock_guard<std::mutex> lk(g_const_mu);
-  if (g_const_owner[h->device & 63] == h) return LANDAU_OK;
-  int rc = set_constants(h);
-  if (rc == LANDAU_OK) g_const_owner[h->device & 63] = h;
-  return rc;
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -518,7 +514,7 @@ int launch_field(landau_t h, int64_t nbatch) {
   const unsigned grid = (unsigned)std::min<int64_t>(items, 8LL * num_sms(h));
   Timer t(h, LANDAU_T_FIELD);
   field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->d_f, h->d_ext_ptr, h->d_ext_dof,
-                                                          h->d_ext_w, h->d_cell_grid, h->d_h, h->d_w, h->d_wT, P.npts);
+                                                          h->d_ext_w, h->d_cell_grid, h->d_h, h->d_w, h->d_tab, h->spc, h->d_wT, P.npts);
   h->launches++;
   h->tlaunch[LANDAU_T_FIELD]++;
   KCHECK();
@@ -526,23 +522,56 @@ int launch_field(landau_t h, int64_t nbatch) {
 }
 
 
+struct InnerPlan {
+  int tpt;
+  int64_t wtiles, nsplit, split_len;
+};
+
+// inner-kernel variant (targets per thread, min blocks per SM); LANDAU_INNER_VARIANT overrides
+int inner_variant() {
+  static const int v = [] {
+    const char *e = getenv("LANDAU_INNER_VARIANT");
+    return e ? atoi(e) : 1;
+  }();
+  return v;
+}
+
+// Work decomposition of N2 for a batch, and the split-j partial buffer (allocated here, outside any
+// graph capture).
+int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
+  const Plan &P = h->plan;
+  const int64_t N = P.npts, nt = (h->e1 - h->e0) * P.nqp;
+  const int variant = inner_variant();
+  ip.tpt = variant == 0 ? 1 : (variant == 4 ? 4 : 2);
+  ip.wtiles = (nt + 32 * ip.tpt - 1) / (32 * ip.tpt);
+  // split-j so that small problems still fill the machine: aim for >= 12 warps per SM
+  const int64_t want = 12LL * num_sms(h);
+  int64_t nsplit = std::max<int64_t>(1, (want + ip.wtiles * nbatch - 1) / (ip.wtiles * nbatch));
+  nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, N / 32));
+  ip.split_len = (N + nsplit - 1) / nsplit;
+  ip.nsplit = (N + ip.split_len - 1) / ip.split_len;
+  if (ip.nsplit > 1) {
+    const int64_t need = nbatch * ip.nsplit * 5 * nt;
+    if (need > h->part_cap) {
+      drop_graphs(h);
+      cudaFree(h->d_part);
+      h->d_part = nullptr;
+      CU(cudaMalloc(&h->d_part, sizeof(double) * need));
+      h->part_cap = need;
+    }
+  }
+  return LANDAU_OK;
+}
+
 int launch_inner(landau_t h, int64_t nbatch) {
   const Plan &P = h->plan;
   const int64_t N = P.npts;
   const int64_t t0 = h->e0 * P.nqp, nt = (h->e1 - h->e0) * P.nqp;
-  // inner-kernel variant (targets per thread, min blocks per SM); LANDAU_INNER_VARIANT overrides
-  static const int variant = [] {
-    const char *e = getenv("LANDAU_INNER_VARIANT");
-    return e ? atoi(e) : 1;
-  }();
-  const int TPT = variant == 0 ? 1 : (variant == 4 ? 4 : 2);
-  const int64_t wtiles = (nt + 32 * TPT - 1) / (32 * TPT);
-  // split-j so that small problems still fill the machine: aim for >= 12 warps per SM
-  const int64_t want = 12LL * num_sms(h);
-  int64_t nsplit = std::max<int64_t>(1, (want + wtiles * nbatch - 1) / (wtiles * nbatch));
-  nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, N / 32));
-  const int64_t split_len = (N + nsplit - 1) / nsplit;
-  nsplit = (N + split_len - 1) / split_len;
+  InnerPlan ip;
+  int rc = inner_plan(h, nbatch, ip);
+  if (rc) return rc;
+  const int variant = inner_variant();
+  const int64_t wtiles = ip.wtiles, nsplit = ip.nsplit, split_len = ip.split_len;
   double *G_own = h->d_G + (int64_t)h->rank * nbatch * 5 * h->Nc;   // [world][batch][5][Nc]
   double *out;
   int64_t out_bstride;
@@ -550,13 +579,6 @@ int launch_inner(landau_t h, int64_t nbatch) {
     out = G_own;
     out_bstride = 5 * h->Nc;
   } else {
-    const int64_t need = nbatch * nsplit * 5 * nt;
-    if (need > h->part_cap) {
-      cudaFree(h->d_part);
-      h->d_part = nullptr;
-      CU(cudaMalloc(&h->d_part, sizeof(double) * need));
-      h->part_cap = need;
-    }
     out = h->d_part;
     out_bstride = nsplit * 5 * nt;
   }
@@ -601,7 +623,7 @@ int launch_element(landau_t h, int64_t nbatch) {
   const Plan &P = h->plan;
   Timer t(h, LANDAU_T_ELEMENT);
   const unsigned grid = (unsigned)std::min<int64_t>(P.ncell * nbatch, (NB == 25 ? 3LL : 6LL) * num_sms(h));
-  element_kernel<NB><<<grid, NB * NB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, h->d_w, h->d_h, h->d_C);
+  element_kernel<NB><<<grid, NB * NB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, h->d_w, h->d_h, h->d_tab, h->d_C);
   h->launches++;
   h->tlaunch[LANDAU_T_ELEMENT]++;
   KCHECK();
@@ -620,13 +642,16 @@ int launch_assemble(landau_t h, int64_t nbatch, double *out, int format) {
     gd.idx = m.idx;
     gd.w = m.w;
     gd.nslots = m.nslots;
+    gd.nsp = h->spc.grid_nsp[g];
     for (int q = 0; q < h->spc.grid_nsp[g]; q++) {
       int sp = h->spc.grid_sp[g][q];
       gd.out_off[q] = format == LANDAU_CSR ? h->snnz_off[sp] : h->scoo_off[sp];
+      gd.fD[q] = h->spc.fD[sp];
+      gd.fK[q] = h->spc.fK[sp];
     }
     if (h->spc.grid_nsp[g] == 0 || m.nslots == 0) continue;
     dim3 grid((unsigned)((m.nslots + 255) / 256), (unsigned)nbatch);
-    assemble_kernel<NB><<<grid, 256, 0, h->stream>>>(gd, g, h->d_C, P.ncell * 2 * NB * NB, out, out_bstride);
+    assemble_kernel<NB><<<grid, 256, 0, h->stream>>>(gd, h->d_C, P.ncell * 2 * NB * NB, out, out_bstride);
     h->launches++;
     h->tlaunch[LANDAU_T_ASSEMBLE]++;
     KCHECK();
@@ -637,7 +662,6 @@ int launch_assemble(landau_t h, int64_t nbatch, double *out, int format) {
 template <int NB>
 int build_jacobian(landau_t h, int64_t nbatch, double *out, int format) {
   int rc;
-  if ((rc = bind_constants(h))) return rc;
   if ((rc = launch_field<NB>(h, nbatch))) return rc;
   if ((rc = launch_inner(h, nbatch))) return rc;
   if ((rc = launch_element<NB>(h, nbatch))) return rc;
@@ -645,7 +669,7 @@ int build_jacobian(landau_t h, int64_t nbatch, double *out, int format) {
   return LANDAU_OK;
 }
 
-int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
+int dispatch_build_direct(landau_t h, int64_t nbatch, double *out, int format) {
   switch (h->plan.nb) {
     case 9: return build_jacobian<9>(h, nbatch, out, format);
     case 16: return build_jacobian<16>(h, nbatch, out, format);
@@ -654,12 +678,55 @@ int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
   return fail(h, LANDAU_EUNSUPPORTED, "order");
 }
 
+// A whole build replays as one CUDA graph (launch-latency bound for small meshes) unless per-stage
+// timers are on, the legacy default stream is in use, or the build has a collective.
+int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
+  if (h->timing || !h->use_graphs || !h->stream || h->world > 1 || !out)
+    return dispatch_build_direct(h, nbatch, out, format);
+  for (auto &g : h->graphs)
+    if (g.nbatch == nbatch && g.format == format && g.out == out) {
+      CU(cudaGraphLaunch(g.exec, h->stream));
+      h->launches += g.kernels;
+      return LANDAU_OK;
+    }
+  InnerPlan ip;   // allocate everything before capturing
+  int rc = inner_plan(h, nbatch, ip);
+  if (rc) return rc;
+  const int64_t l0 = h->launches;
+  int64_t tl[LANDAU_NTIMERS];
+  memcpy(tl, h->tlaunch, sizeof tl);
+  CU(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
+  rc = dispatch_build_direct(h, nbatch, out, format);
+  cudaGraph_t graph = nullptr;
+  cudaError_t ce = cudaStreamEndCapture(h->stream, &graph);
+  const int64_t kernels = h->launches - l0;
+  h->launches = l0;
+  memcpy(h->tlaunch, tl, sizeof tl);
+  if (rc) {
+    if (graph) cudaGraphDestroy(graph);
+    return rc;
+  }
+  if (ce != cudaSuccess) return fail(h, LANDAU_ECUDA, std::string("graph capture: ") + cudaGetErrorString(ce));
+  cudaGraphExec_t exec = nullptr;
+  ce = cudaGraphInstantiate(&exec, graph, 0);
+  cudaGraphDestroy(graph);
+  if (ce != cudaSuccess) return fail(h, LANDAU_ECUDA, std::string("graph instantiate: ") + cudaGetErrorString(ce));
+  if (h->graphs.size() >= 8) {
+    cudaGraphExecDestroy(h->graphs.front().exec);
+    h->graphs.erase(h->graphs.begin());
+  }
+  h->graphs.push_back({nbatch, format, out, exec, kernels});
+  CU(cudaGraphLaunch(exec, h->stream));
+  h->launches += kernels;
+  return LANDAU_OK;
+}
+
 template <int NB>
 int build_mass(landau_t h) {
   const Plan &P = h->plan;
   double *Mbuf = nullptr;
   CU(cudaMalloc(&Mbuf, sizeof(double) * P.ncell * 2 * NB * NB));
-  mass_element_kernel<NB><<<(unsigned)P.ncell, NB * NB, 0, h->stream>>>(P.ncell, h->d_w, Mbuf);
+  mass_element_kernel<NB><<<(unsigned)P.ncell, NB * NB, 0, h->stream>>>(P.ncell, h->d_w, h->d_tab, Mbuf);
   h->launches++;
   KCHECK();
   for (int g = 0; g < P.ngrids; g++) {
@@ -744,6 +811,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
   h = new landau_s();
   h->device = cuda_device;
   h->stream = (cudaStream_t)cuda_stream;
+  if (const char *e = getenv("LANDAU_GRAPHS")) h->use_graphs = atoi(e) != 0;
   h->rank = rank;
   h->world = world;
   h->mode = mode;
@@ -806,6 +874,12 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
       (rc = upload(h, &h->d_ext_ptr, P.ext_ptr)) || (rc = upload(h, &h->d_ext_dof, P.ext_dof)) ||
       (rc = upload(h, &h->d_ext_w, P.ext_w)))
     return bail(rc);
+  {
+    std::vector<double> tab(P.tab_phi);
+    tab.insert(tab.end(), P.tab_dxi.begin(), P.tab_dxi.end());
+    tab.insert(tab.end(), P.tab_deta.begin(), P.tab_deta.end());
+    if ((rc = upload(h, &h->d_tab, tab))) return bail(rc);
+  }
   h->d_csr.resize(P.ngrids);
   h->d_coo.resize(P.ngrids);
   h->d_mass_csr.assign(P.ngrids, nullptr);
@@ -818,7 +892,6 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
       d.nslots = (int64_t)m.ptr.size() - 1;
     }
   }
-  if ((rc = bind_constants(h))) return bail(rc);
   switch (P.nb) {
     case 9: rc = build_mass<9>(h); break;
     case 16: rc = build_mass<16>(h); break;
@@ -845,8 +918,9 @@ void landau_destroy(landau_t h) {
   }
   cudaSetDevice(h->device);
   if (h->stream) cudaStreamSynchronize(h->stream);
+  drop_graphs(h);
   if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
-  for (double *p : {h->d_r, h->d_z, h->d_w, h->d_h, h->d_ext_w, h->d_f, h->d_wT, h->d_part, h->d_G, h->d_C, h->d_vals_tmp})
+  for (double *p : {h->d_r, h->d_z, h->d_w, h->d_h, h->d_tab, h->d_ext_w, h->d_f, h->d_wT, h->d_part, h->d_G, h->d_C, h->d_vals_tmp})
     cudaFree(p);
   cudaFree(h->d_cell_grid);
   cudaFree(h->d_ext_ptr);
@@ -864,10 +938,6 @@ void landau_destroy(landau_t h) {
     cudaEventDestroy(u.second.second);
   }
   for (auto e : h->ev_pool) cudaEventDestroy(e);
-  {
-    std::lock_guard<std::mutex> lk(g_const_mu);
-    if (g_const_owner[h->device & 63] == h) g_const_owner[h->device & 63] = nullptr;
-  }
   delete h;
 }
 
