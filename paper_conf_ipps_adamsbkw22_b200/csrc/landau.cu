@@ -610,7 +610,7 @@ int launch_inner(landau_t h, int64_t nbatch) {
     h->tlaunch[LANDAU_T_REDUCE]++;
     KCHECK();
   }
-  if (h->world > 1 && h->mode == LANDAU_DIST_ELEMENTS) {
+  if (h->comm) {   // LANDAU_DIST_ELEMENTS: the exchange step (also run at world == 1)
     Timer t(h, LANDAU_T_ALLGATHER);
     int rc = g_nccl.AllGather(G_own, h->d_G, (size_t)(nbatch * 5 * h->Nc), kNcclFloat64, h->comm, h->stream);
     if (rc != 0) return fail(h, LANDAU_ENCCL, std::string("ncclAllGather: ") + (g_nccl.GetErrorString ? g_nccl.GetErrorString(rc) : "error"));
@@ -681,7 +681,7 @@ int dispatch_build_direct(landau_t h, int64_t nbatch, double *out, int format) {
 // A whole build replays as one CUDA graph (launch-latency bound for small meshes) unless per-stage
 // timers are on, the legacy default stream is in use, or the build has a collective.
 int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
-  if (h->timing || !h->use_graphs || !h->stream || h->world > 1 || !out)
+  if (h->timing || !h->use_graphs || !h->stream || h->comm || !out)
     return dispatch_build_direct(h, nbatch, out, format);
   for (auto &g : h->graphs)
     if (g.nbatch == nbatch && g.format == format && g.out == out) {
@@ -851,7 +851,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
   // element partition
   landau_partition(P.ncell, world, rank, &h->e0, &h->e1);
   h->chunk_cells = (P.ncell + world - 1) / world;
-  h->Nc = world > 1 ? h->chunk_cells * P.nqp : P.npts;
+  h->Nc = mode == LANDAU_DIST_ELEMENTS ? h->chunk_cells * P.nqp : P.npts;
   int rc;
   if (cuda_device == LANDAU_HOST_ONLY) {
     h->host_only = true;
@@ -898,7 +898,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     case 25: rc = build_mass<25>(h); break;
   }
   if (rc) return bail(rc);
-  if (world > 1) {
+  if (mode == LANDAU_DIST_ELEMENTS) {
     if (!dist->nccl_unique_id) return bail(fail(h, LANDAU_EINVAL, "nccl_unique_id required for element split"));
     if (!load_nccl()) return bail(fail(h, LANDAU_ENCCL, "cannot load libnccl.so.2"));
     ncclUniqueId_ id;
@@ -1072,7 +1072,7 @@ int landau_point_coeffs_batched(landau_t h, int64_t nbatch, double *G_dev) {
   int rc = dispatch_build(h, nbatch, nullptr, LANDAU_CSR);
   if (rc) return rc;
   const int64_t N = h->plan.npts;
-  if (h->world == 1) {
+  if (h->Nc == N) {
     CU(cudaMemcpyAsync(G_dev, h->d_G, sizeof(double) * nbatch * 5 * N, cudaMemcpyDeviceToDevice, h->stream));
   } else {
     const int64_t total = nbatch * 5 * N;

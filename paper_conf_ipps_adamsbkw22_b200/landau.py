@@ -270,3 +270,30 @@ class Landau:
         n = C.c_int64()
         self._check(lib().landau_get_launch_count(self._h, C.byref(n)), "landau_get_launch_count")
         return n.value
+
+
+# ------------------------------------------------------------------------------------------------
+# multi-process helpers (host logic only; the data path never leaves the library)
+# ------------------------------------------------------------------------------------------------
+def batch_range(nbatch, world, rank):
+    """Contiguous share [lo, hi) of a batch of independent vertices for one rank (C4 sharding)."""
+    return rank * nbatch // world, (rank + 1) * nbatch // world
+
+
+def chunk_points(ncell, nqp, world):
+    """Points per rank chunk of the element split's G exchange (cells are split by landau_partition)."""
+    e0, e1 = landau_partition(ncell, world, 0)
+    return (e1 - e0) * nqp
+
+
+def make_dist(mode, group=None):
+    """dist descriptor for Landau(...): rank/world from torch.distributed; for the element split, rank 0
+    creates the NCCL id through the library and the process group broadcasts it."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    uid = None
+    if mode == LANDAU_DIST_ELEMENTS:
+        obj = [landau_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        uid = obj[0]
+    return {"rank": rank, "world": world, "mode": mode, "nccl_unique_id": uid}
