@@ -182,6 +182,157 @@ __global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_
   }
 }
 
+// ------------------------------------------------------------------------------------------------
+// N2 (symmetric): each unordered pair of points is evaluated once.  The points
+// are cut into T tiles of 32.  A warp item is one j-tile b (its 32 points and their reverse-sum
+// accumulators in warp-private shared memory) against one or two i-tiles a1 < a2 < b, or the
+// diagonal item (b, b).  Lane L holds target i = a*32 + L (forward sums in registers); at step k it
+// pairs with j = b*32 + ((L + k) mod 32), so the 32 lanes touch 32 distinct j each step
+// (conflict-free, no atomics).  Diagonal items run k = 1..16 (lanes < 16 only at k = 16) so every
+// unordered pair is visited exactly once.  Two i-tiles per item give two independent pair chains
+// per lane (the FP64 pipe needs the ILP) and share one accumulator update per step.
+// Every item writes 32-point partial "slots"; reduce_sym_kernel sums, for each tile, its slots in a
+// fixed host-built order -> bitwise reproducible.  part = [batch][nslots][5][32].
+// ------------------------------------------------------------------------------------------------
+constexpr int kSymWarps = 4;
+
+struct SymItem {   // host-built, see build_sym_items
+  int a1, a2, b;   // a2 < 0: one i-tile; a1 == b: diagonal
+  int slot;        // first of its 2 (diagonal, one i-tile) or 3 (two i-tiles) consecutive slots
+};
+
+__device__ __forceinline__ void sym_load_i(const double *pr, const double *pz, const double *wb, int64_t N, int64_t i,
+                                           int lane, double &r, double &z, double &wd, double &wkr, double &wkz) {
+  const bool v = i < N;   // padding: far away, zero weights -- contributes nothing, never read back
+  r = v ? pr[i] : 1.0;
+  z = v ? pz[i] : 1.0e6 + lane;
+  wd = v ? wb[i] : 0.0;
+  wkr = v ? wb[N + i] : 0.0;
+  wkz = v ? wb[2 * N + i] : 0.0;
+}
+
+__device__ __forceinline__ void sym_store(double *o, int lane, const Acc5 &a) {
+  o[lane] = a.drr;
+  o[32 + lane] = a.drz;
+  o[64 + lane] = a.dzz;
+  o[96 + lane] = a.kr;
+  o[128 + lane] = a.kz;
+}
+
+template <int MINB>
+__global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t N, int64_t nitems_b, int64_t nslots,
+                                                                         int64_t nitems,
+                                                                         const SymItem *__restrict__ items,
+                                                                         const double *__restrict__ pr,
+                                                                         const double *__restrict__ pz,
+                                                                         const double *__restrict__ wT,
+                                                                         double *__restrict__ part) {
+  __shared__ double2 s_rz[kSymWarps][32], s_w[kSymWarps][32];
+  __shared__ double s_wz[kSymWarps][32];
+  __shared__ double s_acc[kSymWarps][5][32];
+  __shared__ double s_coef[kNumPairCoef];
+  stage_pair_coef(s_coef);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, cf);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t item = (int64_t)blockIdx.x * kSymWarps + wid;
+  if (item >= nitems) return;   // whole warp: no block-level barrier follows
+  const int64_t bb = item / nitems_b;
+  const SymItem it = items[item % nitems_b];
+  const double *wb = wT + bb * 3 * N;
+  {
+    double r, z, wd, wkr, wkz;
+    sym_load_i(pr, pz, wb, N, (int64_t)it.b * 32 + lane, lane, r, z, wd, wkr, wkz);
+    s_rz[wid][lane] = make_double2(r, z + (((int64_t)it.b * 32 + lane) < N ? 0.0 : 1.0e6));
+    s_w[wid][lane] = make_double2(wd, wkr);
+    s_wz[wid][lane] = wkz;
+  }
+#pragma unroll
+  for (int c = 0; c < 5; c++) s_acc[wid][c][lane] = 0.0;
+  __syncwarp();
+  double *o = part + (bb * nslots + it.slot) * 160;
+  if (it.a1 == it.b) {   // diagonal
+    double r1, z1, wd1, wkr1, wkz1;
+    sym_load_i(pr, pz, wb, N, (int64_t)it.a1 * 32 + lane, lane, r1, z1, wd1, wkr1, wkz1);
+    Acc5 a1{0.0, 0.0, 0.0, 0.0, 0.0};
+    for (int k = 1; k <= 16; k++) {
+      const int jj = (lane + k) & 31;
+      const double2 rz = s_rz[wid][jj], w = s_w[wid][jj];
+      const double wkz = s_wz[wid][jj];
+      Acc5 aj{s_acc[wid][0][jj], s_acc[wid][1][jj], s_acc[wid][2][jj], s_acc[wid][3][jj], s_acc[wid][4][jj]};
+      landau_pair_sym(r1, z1, wd1, wkr1, wkz1, rz.x, rz.y, w.x, w.y, wkz, !(k == 16 && lane >= 16), cf, a1, aj);
+      s_acc[wid][0][jj] = aj.drr;
+      s_acc[wid][1][jj] = aj.drz;
+      s_acc[wid][2][jj] = aj.dzz;
+      s_acc[wid][3][jj] = aj.kr;
+      s_acc[wid][4][jj] = aj.kz;
+      __syncwarp();   // lane L next reads the slot lane L+1 just wrote
+    }
+    sym_store(o, lane, a1);
+    o += 160;
+  } else if (it.a2 < 0) {   // one i-tile
+    double r1, z1, wd1, wkr1, wkz1;
+    sym_load_i(pr, pz, wb, N, (int64_t)it.a1 * 32 + lane, lane, r1, z1, wd1, wkr1, wkz1);
+    Acc5 a1{0.0, 0.0, 0.0, 0.0, 0.0};
+    for (int k = 0; k < 32; k++) {
+      const int jj = (lane + k) & 31;
+      const double2 rz = s_rz[wid][jj], w = s_w[wid][jj];
+      const double wkz = s_wz[wid][jj];
+      Acc5 aj{s_acc[wid][0][jj], s_acc[wid][1][jj], s_acc[wid][2][jj], s_acc[wid][3][jj], s_acc[wid][4][jj]};
+      landau_pair_sym(r1, z1, wd1, wkr1, wkz1, rz.x, rz.y, w.x, w.y, wkz, true, cf, a1, aj);
+      s_acc[wid][0][jj] = aj.drr;
+      s_acc[wid][1][jj] = aj.drz;
+      s_acc[wid][2][jj] = aj.dzz;
+      s_acc[wid][3][jj] = aj.kr;
+      s_acc[wid][4][jj] = aj.kz;
+      __syncwarp();
+    }
+    sym_store(o, lane, a1);
+    o += 160;
+  } else {   // two i-tiles share the j-tile
+    double r1, z1, wd1, wkr1, wkz1, r2, z2, wd2, wkr2, wkz2;
+    sym_load_i(pr, pz, wb, N, (int64_t)it.a1 * 32 + lane, lane, r1, z1, wd1, wkr1, wkz1);
+    sym_load_i(pr, pz, wb, N, (int64_t)it.a2 * 32 + lane, lane, r2, z2, wd2, wkr2, wkz2);
+    Acc5 a1{0.0, 0.0, 0.0, 0.0, 0.0}, a2{0.0, 0.0, 0.0, 0.0, 0.0};
+    for (int k = 0; k < 32; k++) {
+      const int jj = (lane + k) & 31;
+      const double2 rz = s_rz[wid][jj], w = s_w[wid][jj];
+      const double wkz = s_wz[wid][jj];
+      Acc5 aj{s_acc[wid][0][jj], s_acc[wid][1][jj], s_acc[wid][2][jj], s_acc[wid][3][jj], s_acc[wid][4][jj]};
+      landau_pair_sym(r1, z1, wd1, wkr1, wkz1, rz.x, rz.y, w.x, w.y, wkz, true, cf, a1, aj);
+      landau_pair_sym(r2, z2, wd2, wkr2, wkz2, rz.x, rz.y, w.x, w.y, wkz, true, cf, a2, aj);
+      s_acc[wid][0][jj] = aj.drr;
+      s_acc[wid][1][jj] = aj.drz;
+      s_acc[wid][2][jj] = aj.dzz;
+      s_acc[wid][3][jj] = aj.kr;
+      s_acc[wid][4][jj] = aj.kz;
+      __syncwarp();
+    }
+    sym_store(o, lane, a1);
+    sym_store(o + 160, lane, a2);
+    o += 320;
+  }
+  __syncwarp();
+  Acc5 aj{s_acc[wid][0][lane], s_acc[wid][1][lane], s_acc[wid][2][lane], s_acc[wid][3][lane], s_acc[wid][4][lane]};
+  sym_store(o, lane, aj);
+}
+
+// G[b][c][i] = sum of the partial slots of tile t = i / 32 in the fixed order of tile_slots.
+__global__ void reduce_sym_kernel(int64_t N, int64_t nslots, const int32_t *__restrict__ tile_ptr,
+                                  const int32_t *__restrict__ tile_slots, const double *__restrict__ part,
+                                  double *__restrict__ G, int64_t G_bstride, int nbatch) {
+  const int64_t total = (int64_t)nbatch * 5 * N;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = k / (5 * N), c = (k / N) % 5, i = k % N;
+    const int t = (int)(i / 32), lane = (int)(i % 32);
+    const double *pb = part + b * nslots * 160 + c * 32 + lane;
+    double s = 0.0;
+    for (int q = tile_ptr[t]; q < tile_ptr[t + 1]; q++) s += pb[(int64_t)tile_slots[q] * 160];
+    G[b * G_bstride + c * N + i] = s;
+  }
+}
+
 // N2r: G[b][c][i] = sum_{s = 0..nsplit-1} part[b][s][c][i] in fixed order (deterministic).
 __global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__ part, double *__restrict__ G,
                               int64_t G_bstride, int nbatch) {
@@ -393,6 +544,10 @@ struct landau_s {
   bool have_state = false;
   double *d_f = nullptr, *d_wT = nullptr, *d_part = nullptr, *d_G = nullptr, *d_C = nullptr;
   int64_t part_cap = 0;
+  SymItem *d_sym_items = nullptr;   // work items of the symmetric inner kernel
+  int32_t *d_tile_ptr = nullptr, *d_tile_slots = nullptr;
+  int ntiles = 0;
+  int64_t nsym_items = 0, nsym_slots = 0;
   // host staging for landau_jacobian_host
   double *d_vals_tmp = nullptr;
   int64_t vals_tmp_cap = 0;
@@ -523,9 +678,18 @@ int launch_field(landau_t h, int64_t nbatch) {
 
 
 struct InnerPlan {
+  bool sym;   // symmetric pair evaluation (whole point set as targets, enough tile pairs to fill the GPU)
   int tpt;
   int64_t wtiles, nsplit, split_len;
 };
+
+bool sym_enabled() {
+  static const bool v = [] {
+    const char *e = getenv("LANDAU_SYM");
+    return !(e && atoi(e) == 0);
+  }();
+  return v;
+}
 
 // inner-kernel variant (targets per thread, min blocks per SM); LANDAU_INNER_VARIANT overrides
 int inner_variant() {
@@ -542,6 +706,23 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
   const Plan &P = h->plan;
   const int64_t N = P.npts, nt = (h->e1 - h->e0) * P.nqp;
   const int variant = inner_variant();
+  ip.sym = sym_enabled() && !h->comm && h->nsym_items > 0 && nbatch * h->nsym_items >= 8LL * kSymWarps * num_sms(h) &&
+           nbatch * h->nsym_slots * 160 * (int64_t)sizeof(double) <= (8LL << 30);
+  if (ip.sym) {
+    ip.tpt = 1;
+    ip.wtiles = h->ntiles;
+    ip.nsplit = 1;
+    ip.split_len = N;
+    const int64_t need = nbatch * h->nsym_slots * 160;
+    if (need > h->part_cap) {
+      drop_graphs(h);
+      cudaFree(h->d_part);
+      h->d_part = nullptr;
+      CU(cudaMalloc(&h->d_part, sizeof(double) * need));
+      h->part_cap = need;
+    }
+    return LANDAU_OK;
+  }
   ip.tpt = variant == 0 ? 1 : (variant == 4 ? 4 : 2);
   ip.wtiles = (nt + 32 * ip.tpt - 1) / (32 * ip.tpt);
   // split-j so that small problems still fill the machine: aim for >= 12 warps per SM
@@ -573,6 +754,27 @@ int launch_inner(landau_t h, int64_t nbatch) {
   const int variant = inner_variant();
   const int64_t wtiles = ip.wtiles, nsplit = ip.nsplit, split_len = ip.split_len;
   double *G_own = h->d_G + (int64_t)h->rank * nbatch * 5 * h->Nc;   // [world][batch][5][Nc]
+  if (ip.sym) {
+    {
+      Timer t(h, LANDAU_T_INNER);
+      const int64_t nitems = nbatch * h->nsym_items;
+      const unsigned grid = (unsigned)((nitems + kSymWarps - 1) / kSymWarps);
+      inner_sym_kernel<2><<<grid, 32 * kSymWarps, 0, h->stream>>>(N, h->nsym_items, h->nsym_slots, nitems,
+                                                                   h->d_sym_items, h->d_r, h->d_z, h->d_wT, h->d_part);
+      h->launches++;
+      h->tlaunch[LANDAU_T_INNER]++;
+      KCHECK();
+    }
+    Timer t(h, LANDAU_T_REDUCE);
+    const int64_t total = nbatch * 5 * N;
+    const int blocks = (int)std::min<int64_t>((total + 255) / 256, 16LL * num_sms(h));
+    reduce_sym_kernel<<<blocks, 256, 0, h->stream>>>(N, h->nsym_slots, h->d_tile_ptr, h->d_tile_slots, h->d_part, G_own,
+                                                     5 * h->Nc, (int)nbatch);
+    h->launches++;
+    h->tlaunch[LANDAU_T_REDUCE]++;
+    KCHECK();
+    return LANDAU_OK;
+  }
   double *out;
   int64_t out_bstride;
   if (nsplit == 1) {
@@ -880,6 +1082,43 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     tab.insert(tab.end(), P.tab_deta.begin(), P.tab_deta.end());
     if ((rc = upload(h, &h->d_tab, tab))) return bail(rc);
   }
+  if (mode != LANDAU_DIST_ELEMENTS) {   // work items + slot map of the symmetric inner kernel
+    const int T = (int)((P.npts + 31) / 32);
+    std::vector<SymItem> items;
+    std::vector<std::vector<int32_t>> slots_of(T);
+    int slot = 0;
+    for (int b = 0; b < T; b++) {          // column b: diagonal, then i-tiles a < b two at a time
+      items.push_back({b, -1, b, slot});
+      slots_of[b].push_back(slot);
+      slots_of[b].push_back(slot + 1);
+      slot += 2;
+      for (int a = 0; a < b; a += 2) {
+        if (a + 1 < b) {
+          items.push_back({a, a + 1, b, slot});
+          slots_of[a].push_back(slot);
+          slots_of[a + 1].push_back(slot + 1);
+          slots_of[b].push_back(slot + 2);
+          slot += 3;
+        } else {
+          items.push_back({a, -1, b, slot});
+          slots_of[a].push_back(slot);
+          slots_of[b].push_back(slot + 1);
+          slot += 2;
+        }
+      }
+    }
+    std::vector<int32_t> tptr(1, 0), tslots;
+    for (int t = 0; t < T; t++) {
+      tslots.insert(tslots.end(), slots_of[t].begin(), slots_of[t].end());
+      tptr.push_back((int32_t)tslots.size());
+    }
+    h->ntiles = T;
+    h->nsym_items = (int64_t)items.size();
+    h->nsym_slots = slot;
+    if ((rc = upload(h, &h->d_sym_items, items)) || (rc = upload(h, &h->d_tile_ptr, tptr)) ||
+        (rc = upload(h, &h->d_tile_slots, tslots)))
+      return bail(rc);
+  }
   h->d_csr.resize(P.ngrids);
   h->d_coo.resize(P.ngrids);
   h->d_mass_csr.assign(P.ngrids, nullptr);
@@ -923,6 +1162,9 @@ void landau_destroy(landau_t h) {
   for (double *p : {h->d_r, h->d_z, h->d_w, h->d_h, h->d_tab, h->d_ext_w, h->d_f, h->d_wT, h->d_part, h->d_G, h->d_C, h->d_vals_tmp})
     cudaFree(p);
   cudaFree(h->d_cell_grid);
+  cudaFree(h->d_sym_items);
+  cudaFree(h->d_tile_ptr);
+  cudaFree(h->d_tile_slots);
   cudaFree(h->d_ext_ptr);
   cudaFree(h->d_ext_dof);
   for (auto *v : {&h->d_csr, &h->d_coo})

@@ -259,3 +259,37 @@ def test_graph_replay_matches_direct_launches():
     c = gpu_jacobian(h, fg)
     assert np.array_equal(a.view(np.uint64), b.view(np.uint64))
     assert np.array_equal(b.view(np.uint64), c.view(np.uint64))
+
+
+def test_symmetric_kernel_batch_C4():
+    """A batch large enough for the symmetric inner kernel (each unordered pair evaluated once, both
+    targets updated): vertices against the oracle, conservation, and bitwise determinism."""
+    nb = 24
+    prob0 = inputs.config4_vertex(0)
+    h = L.Landau.from_problem(prob0, device=0)
+    verts = [int(round(k * 1023 / (nb - 1))) for k in range(nb)]
+    probs = [inputs.config4_vertex(b) for b in verts]
+    nodes = h.all_nodes()
+    F = torch.tensor(np.stack([inputs.coefficients(p, nodes) for p in probs]), device=DEV)
+    h.set_state_batched(F)
+    out = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
+    h.set_timing(True)
+    h.jacobian_batched(out)
+    t = h.get_timing()
+    h.set_timing(False)
+    assert t["reduce"][1] == 1    # the symmetric path always reduces its partial slots
+    Jb = out.cpu().numpy()
+    for k in (0, nb // 2, nb - 1):
+        o = Oracle(probs[k])
+        fo = o.coefficients()
+        Jo, Ja = o.jacobian(fo)
+        assert np.all(np.abs(Jb[k] - Jo) <= 1e-11 * Ja), verts[k]
+        d, m, e = _conservation(probs[k], h, Jb[k], inputs.coefficients(probs[k], nodes))
+        assert d < 1e-13 and m < 1e-13 and e < 1e-13, (d, m, e)
+    h.jacobian_batched(out)
+    assert np.array_equal(out.cpu().numpy().view(np.uint64), Jb.view(np.uint64))
+    G = torch.empty((nb, 5, h.npoints), dtype=torch.float64, device=DEV)
+    h.point_coeffs_batched(G)
+    o = Oracle(probs[5])
+    Go, Ga = o.point_coeffs(o.coefficients())
+    assert np.max(np.abs(G[5].cpu().numpy() - Go) / Ga) <= 1e-12
