@@ -195,17 +195,24 @@ __global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_
 // fixed host-built order -> bitwise reproducible.  part = [batch][nslots][5][32].
 // ------------------------------------------------------------------------------------------------
 constexpr int kSymWarps = 4;
+#ifndef LANDAU_SYM_NI
+#define LANDAU_SYM_NI 2
+#endif
+constexpr int kSymNI = LANDAU_SYM_NI;   // max i-tiles per item (independent pair chains per lane)
+static_assert(kSymNI >= 2 && kSymNI <= 3, "sym items carry 1..3 i-tiles");
 
-struct SymItem {   // host-built, see build_sym_items
-  int a1, a2, b;   // a2 < 0: one i-tile; a1 == b: diagonal
-  int slot;        // first of its 2 (diagonal, one i-tile) or 3 (two i-tiles) consecutive slots
+struct SymItem {   // host-built, see landau_create
+  int a[3];        // i-tiles (n of them, all < b); n == 0: the diagonal item (b, b)
+  int b, n;
+  int slot;        // first of the item's consecutive partial slots: one per i-tile (or the diagonal's
+                   // forward sums), then the j-tile's reverse sums
 };
 
 __device__ __forceinline__ void sym_load_i(const double *pr, const double *pz, const double *wb, int64_t N, int64_t i,
-                                           int lane, double &r, double &z, double &wd, double &wkr, double &wkz) {
+                                           double zpad, double &r, double &z, double &wd, double &wkr, double &wkz) {
   const bool v = i < N;   // padding: far away, zero weights -- contributes nothing, never read back
   r = v ? pr[i] : 1.0;
-  z = v ? pz[i] : 1.0e6 + lane;
+  z = v ? pz[i] : zpad;
   wd = v ? wb[i] : 0.0;
   wkr = v ? wb[N + i] : 0.0;
   wkz = v ? wb[2 * N + i] : 0.0;
@@ -219,6 +226,53 @@ __device__ __forceinline__ void sym_store(double *o, int lane, const Acc5 &a) {
   o[128 + lane] = a.kz;
 }
 
+// NI i-tiles against the warp's j-tile (NI independent pair chains per lane and step); DIAG: the
+// tile against itself, k = 1..16 (lanes < 16 only at k = 16) -- every unordered pair exactly once.
+// The reverse sums travel with their j: at step k lane L holds the accumulator of j = (L + k) mod 32
+// and hands it to lane L - 1 by a shuffle, so consecutive steps carry no memory fence and their
+// (long, independent) pair evaluations overlap; the j data itself is read-only shared memory.
+template <int NI, bool DIAG>
+__device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, const double *pz, const double *wb,
+                                        int64_t N, int lane, const double2 *s_rz, const double2 *s_w,
+                                        const double *s_wz, const PairCoef &cf, double *o) {
+  double r[NI], z[NI], wd[NI], wkr[NI], wkz[NI];
+  Acc5 ai[NI];
+#pragma unroll
+  for (int t = 0; t < NI; t++) {
+    sym_load_i(pr, pz, wb, N, (int64_t)(DIAG ? it.b : it.a[t]) * 32 + lane, 1.0e6 + 64.0 * t + lane, r[t], z[t], wd[t],
+               wkr[t], wkz[t]);
+    ai[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+  }
+  constexpr int k0 = DIAG ? 1 : 0, k1 = DIAG ? 17 : 32;
+  const int src = (lane + 1) & 31;
+  Acc5 aj{0.0, 0.0, 0.0, 0.0, 0.0};
+#pragma unroll 2
+  for (int k = k0; k < k1; k++) {
+    const int jj = (lane + k) & 31;
+    const double2 rz = s_rz[jj], w = s_w[jj];
+    const double wkz_j = s_wz[jj];
+    const bool on = !DIAG || !(k == 16 && lane >= 16);
+#pragma unroll
+    for (int t = 0; t < NI; t++)
+      landau_pair_sym(r[t], z[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, w.x, w.y, wkz_j, on, cf, ai[t], aj);
+    aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
+    aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
+    aj.dzz = __shfl_sync(0xffffffffu, aj.dzz, src);
+    aj.kr = __shfl_sync(0xffffffffu, aj.kr, src);
+    aj.kz = __shfl_sync(0xffffffffu, aj.kz, src);
+  }
+#pragma unroll
+  for (int t = 0; t < NI; t++) sym_store(o + t * 160, lane, ai[t]);
+  // after the last hand-over lane L holds the reverse sums of j = (L + k1) mod 32
+  const int jf = (lane + k1) & 31;
+  double *oj = o + (DIAG ? 1 : NI) * 160;
+  oj[jf] = aj.drr;
+  oj[32 + jf] = aj.drz;
+  oj[64 + jf] = aj.dzz;
+  oj[96 + jf] = aj.kr;
+  oj[128 + jf] = aj.kz;
+}
+
 template <int MINB>
 __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t N, int64_t nitems_b, int64_t nslots,
                                                                          int64_t nitems,
@@ -229,93 +283,36 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t
                                                                          double *__restrict__ part) {
   __shared__ double2 s_rz[kSymWarps][32], s_w[kSymWarps][32];
   __shared__ double s_wz[kSymWarps][32];
-  __shared__ double s_acc[kSymWarps][5][32];
   __shared__ double s_coef[kNumPairCoef];
   stage_pair_coef(s_coef);
   __syncthreads();
   PairCoef cf;
   load_pair_coef(s_coef, cf);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const int64_t item = (int64_t)blockIdx.x * kSymWarps + wid;
-  if (item >= nitems) return;   // whole warp: no block-level barrier follows
+  // persistent warps: grid-stride over the (batch item, work item) list
+  for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
   const int64_t bb = item / nitems_b;
   const SymItem it = items[item % nitems_b];
   const double *wb = wT + bb * 3 * N;
+  __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
   {
     double r, z, wd, wkr, wkz;
-    sym_load_i(pr, pz, wb, N, (int64_t)it.b * 32 + lane, lane, r, z, wd, wkr, wkz);
-    s_rz[wid][lane] = make_double2(r, z + (((int64_t)it.b * 32 + lane) < N ? 0.0 : 1.0e6));
+    sym_load_i(pr, pz, wb, N, (int64_t)it.b * 32 + lane, 2.0e6 + lane, r, z, wd, wkr, wkz);
+    s_rz[wid][lane] = make_double2(r, z);
     s_w[wid][lane] = make_double2(wd, wkr);
     s_wz[wid][lane] = wkz;
   }
-#pragma unroll
-  for (int c = 0; c < 5; c++) s_acc[wid][c][lane] = 0.0;
   __syncwarp();
   double *o = part + (bb * nslots + it.slot) * 160;
-  if (it.a1 == it.b) {   // diagonal
-    double r1, z1, wd1, wkr1, wkz1;
-    sym_load_i(pr, pz, wb, N, (int64_t)it.a1 * 32 + lane, lane, r1, z1, wd1, wkr1, wkz1);
-    Acc5 a1{0.0, 0.0, 0.0, 0.0, 0.0};
-    for (int k = 1; k <= 16; k++) {
-      const int jj = (lane + k) & 31;
-      const double2 rz = s_rz[wid][jj], w = s_w[wid][jj];
-      const double wkz = s_wz[wid][jj];
-      Acc5 aj{s_acc[wid][0][jj], s_acc[wid][1][jj], s_acc[wid][2][jj], s_acc[wid][3][jj], s_acc[wid][4][jj]};
-      landau_pair_sym(r1, z1, wd1, wkr1, wkz1, rz.x, rz.y, w.x, w.y, wkz, !(k == 16 && lane >= 16), cf, a1, aj);
-      s_acc[wid][0][jj] = aj.drr;
-      s_acc[wid][1][jj] = aj.drz;
-      s_acc[wid][2][jj] = aj.dzz;
-      s_acc[wid][3][jj] = aj.kr;
-      s_acc[wid][4][jj] = aj.kz;
-      __syncwarp();   // lane L next reads the slot lane L+1 just wrote
-    }
-    sym_store(o, lane, a1);
-    o += 160;
-  } else if (it.a2 < 0) {   // one i-tile
-    double r1, z1, wd1, wkr1, wkz1;
-    sym_load_i(pr, pz, wb, N, (int64_t)it.a1 * 32 + lane, lane, r1, z1, wd1, wkr1, wkz1);
-    Acc5 a1{0.0, 0.0, 0.0, 0.0, 0.0};
-    for (int k = 0; k < 32; k++) {
-      const int jj = (lane + k) & 31;
-      const double2 rz = s_rz[wid][jj], w = s_w[wid][jj];
-      const double wkz = s_wz[wid][jj];
-      Acc5 aj{s_acc[wid][0][jj], s_acc[wid][1][jj], s_acc[wid][2][jj], s_acc[wid][3][jj], s_acc[wid][4][jj]};
-      landau_pair_sym(r1, z1, wd1, wkr1, wkz1, rz.x, rz.y, w.x, w.y, wkz, true, cf, a1, aj);
-      s_acc[wid][0][jj] = aj.drr;
-      s_acc[wid][1][jj] = aj.drz;
-      s_acc[wid][2][jj] = aj.dzz;
-      s_acc[wid][3][jj] = aj.kr;
-      s_acc[wid][4][jj] = aj.kz;
-      __syncwarp();
-    }
-    sym_store(o, lane, a1);
-    o += 160;
-  } else {   // two i-tiles share the j-tile
-    double r1, z1, wd1, wkr1, wkz1, r2, z2, wd2, wkr2, wkz2;
-    sym_load_i(pr, pz, wb, N, (int64_t)it.a1 * 32 + lane, lane, r1, z1, wd1, wkr1, wkz1);
-    sym_load_i(pr, pz, wb, N, (int64_t)it.a2 * 32 + lane, lane, r2, z2, wd2, wkr2, wkz2);
-    Acc5 a1{0.0, 0.0, 0.0, 0.0, 0.0}, a2{0.0, 0.0, 0.0, 0.0, 0.0};
-    for (int k = 0; k < 32; k++) {
-      const int jj = (lane + k) & 31;
-      const double2 rz = s_rz[wid][jj], w = s_w[wid][jj];
-      const double wkz = s_wz[wid][jj];
-      Acc5 aj{s_acc[wid][0][jj], s_acc[wid][1][jj], s_acc[wid][2][jj], s_acc[wid][3][jj], s_acc[wid][4][jj]};
-      landau_pair_sym(r1, z1, wd1, wkr1, wkz1, rz.x, rz.y, w.x, w.y, wkz, true, cf, a1, aj);
-      landau_pair_sym(r2, z2, wd2, wkr2, wkz2, rz.x, rz.y, w.x, w.y, wkz, true, cf, a2, aj);
-      s_acc[wid][0][jj] = aj.drr;
-      s_acc[wid][1][jj] = aj.drz;
-      s_acc[wid][2][jj] = aj.dzz;
-      s_acc[wid][3][jj] = aj.kr;
-      s_acc[wid][4][jj] = aj.kz;
-      __syncwarp();
-    }
-    sym_store(o, lane, a1);
-    sym_store(o + 160, lane, a2);
-    o += 320;
+  switch (it.n) {
+    case 0: sym_run<1, true>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
+    case 1: sym_run<1, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
+    case 2: sym_run<2, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
+    default:
+      if constexpr (kSymNI >= 3) sym_run<kSymNI, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
+      break;
   }
-  __syncwarp();
-  Acc5 aj{s_acc[wid][0][lane], s_acc[wid][1][lane], s_acc[wid][2][lane], s_acc[wid][3][lane], s_acc[wid][4][lane]};
-  sym_store(o, lane, aj);
+  }
 }
 
 // G[b][c][i] = sum of the partial slots of tile t = i / 32 in the fixed order of tile_slots.
@@ -758,7 +755,7 @@ int launch_inner(landau_t h, int64_t nbatch) {
     {
       Timer t(h, LANDAU_T_INNER);
       const int64_t nitems = nbatch * h->nsym_items;
-      const unsigned grid = (unsigned)((nitems + kSymWarps - 1) / kSymWarps);
+      const unsigned grid = (unsigned)std::min<int64_t>((nitems + kSymWarps - 1) / kSymWarps, 2LL * num_sms(h));
       inner_sym_kernel<2><<<grid, 32 * kSymWarps, 0, h->stream>>>(N, h->nsym_items, h->nsym_slots, nitems,
                                                                    h->d_sym_items, h->d_r, h->d_z, h->d_wT, h->d_part);
       h->launches++;
@@ -1087,24 +1084,19 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     std::vector<SymItem> items;
     std::vector<std::vector<int32_t>> slots_of(T);
     int slot = 0;
-    for (int b = 0; b < T; b++) {          // column b: diagonal, then i-tiles a < b two at a time
-      items.push_back({b, -1, b, slot});
+    for (int b = 0; b < T; b++) {          // column b: the diagonal, then i-tiles a < b, kSymNI at a time
+      items.push_back({{b, -1, -1}, b, 0, slot});
       slots_of[b].push_back(slot);
       slots_of[b].push_back(slot + 1);
       slot += 2;
-      for (int a = 0; a < b; a += 2) {
-        if (a + 1 < b) {
-          items.push_back({a, a + 1, b, slot});
-          slots_of[a].push_back(slot);
-          slots_of[a + 1].push_back(slot + 1);
-          slots_of[b].push_back(slot + 2);
-          slot += 3;
-        } else {
-          items.push_back({a, -1, b, slot});
-          slots_of[a].push_back(slot);
-          slots_of[b].push_back(slot + 1);
-          slot += 2;
+      for (int a = 0; a < b; a += kSymNI) {
+        SymItem it{{-1, -1, -1}, b, std::min(kSymNI, b - a), slot};
+        for (int t = 0; t < it.n; t++) {
+          it.a[t] = a + t;
+          slots_of[a + t].push_back(slot++);
         }
+        slots_of[b].push_back(slot++);
+        items.push_back(it);
       }
     }
     std::vector<int32_t> tptr(1, 0), tslots;

@@ -12,7 +12,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "liblandau.so")
+LIB_PATH = os.environ.get("LANDAU_LIB") or os.path.join(_HERE, "liblandau.so")
 
 LANDAU_OK, LANDAU_EINVAL, LANDAU_ENOMEM, LANDAU_ECUDA, LANDAU_ENCCL, LANDAU_ESTATE, LANDAU_EUNSUPPORTED = \
     0, -1, -2, -3, -4, -5, -6
