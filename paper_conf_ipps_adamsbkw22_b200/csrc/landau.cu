@@ -61,9 +61,14 @@ __global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbat
                                                          const double *__restrict__ cell_h, const double *__restrict__ pw,
                                                          const double *__restrict__ tab, const SpeciesConst sp_,
                                                          double *__restrict__ wT, int64_t npts) {
+  // tables transposed ([k][q]): in phase 2 consecutive threads are consecutive q (conflict-free)
   __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
   __shared__ double gD[EPB][NB], gK[EPB][NB];
-  load_tables<NB>(tab, s_phi, s_dxi, s_deta);
+  for (int i = threadIdx.x; i < NB * NB; i += blockDim.x) {
+    s_phi[i % NB][i / NB] = tab[i];
+    s_dxi[i % NB][i / NB] = tab[NB * NB + i];
+    s_deta[i % NB][i / NB] = tab[2 * NB * NB + i];
+  }
   const SpeciesConst &c_sp = sp_;
   const int el = threadIdx.x / NB, a = threadIdx.x % NB;
   const int64_t nchunks = (ncell + EPB - 1) / EPB;
@@ -94,9 +99,9 @@ __global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbat
       double td = 0.0, tr = 0.0, tz = 0.0;
 #pragma unroll
       for (int k = 0; k < NB; k++) {
-        td = fma(s_phi[q][k], gD[el][k], td);
-        tr = fma(s_dxi[q][k], gK[el][k], tr);
-        tz = fma(s_deta[q][k], gK[el][k], tz);
+        td = fma(s_phi[k][q], gD[el][k], td);
+        tr = fma(s_dxi[k][q], gK[el][k], tr);
+        tz = fma(s_deta[k][q], gK[el][k], tz);
       }
       const double w = pw[pt], ws = w * (2.0 / cell_h[e]);
       double *o = wT + (int64_t)b * 3 * npts;
@@ -344,48 +349,76 @@ __global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__
 }
 
 // ------------------------------------------------------------------------------------------------
-// N3: element matrices (species independent).  Grid-stride over (cell, batch); thread (k, l).
-//   C^D[k,l] = (2/h)^2 sum_q (gk . w_q G_D(q) . gl),  C^K[k,l] = (2/h) sum_q (gk . w_q G_K(q)) phi_l(q)
-// with gk the reference gradients.  G is read in the chunked layout
-//   G[((i / Nc) * nbatch + b) * 5 + c][i % Nc]     (Nc = N when not distributed).
+// N3: element matrices (species independent).  C^D[k,l] = (2/h)^2 sum_q gk . (w_q G_D(q)) . gl,
+// C^K[k,l] = (2/h) sum_q (gk . w_q G_K(q)) phi_l(q), gk the reference gradients.  A thread owns an
+// S x S block (S = p + 1) of both matrices of one cell, so each table value it loads from shared
+// memory feeds S outputs (the v0 one-entry-per-thread form was shared-memory-bandwidth bound);
+// a block handles EPB cells.  Per q:  u_l = A_rr gl_r + A_rz gl_z,  v_l = A_rz gl_r + A_zz gl_z,
+// t_k = gk_r K_r + gk_z K_z;  C^D[k,l] += gk_r u_l + gk_z v_l,  C^K[k,l] += t_k phi_l.
+// G is read in the chunked layout G[((i / Nc) * nbatch + b) * 5 + c][i % Nc] (Nc = N unless split).
 // ------------------------------------------------------------------------------------------------
-template <int NB>
-__global__ void __launch_bounds__(NB * NB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
-                                                            int nbatch, const double *__restrict__ pw,
-                                                            const double *__restrict__ cell_h, const double *__restrict__ tab,
-                                                            double *__restrict__ Cbuf) {
-  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
-  __shared__ double sA[5][NB];
+template <int NB, int S, int EPB>
+__global__ void __launch_bounds__(NB * EPB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
+                                                             int nbatch, int b0, int nb, const double *__restrict__ pw,
+                                                             const double *__restrict__ cell_h,
+                                                             const double *__restrict__ tab, double *__restrict__ Cbuf) {
+  static_assert(S * S == NB, "S = p + 1");
+  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];   // [q][k]
+  __shared__ double sA[EPB][5][NB];                                  // w_q G(q) per cell
   load_tables<NB>(tab, s_phi, s_dxi, s_deta);
-  const int tid = threadIdx.x;
-  const int k = tid / NB, l = tid % NB;
-  for (int64_t it = blockIdx.x; it < ncell * nbatch; it += gridDim.x) {
-    const int b = (int)(it / ncell);
-    const int64_t e = it % ncell;
+  const int el = threadIdx.x / NB, t = threadIdx.x % NB;
+  const int k0 = (t / S) * S, l0 = (t % S) * S;
+  const int64_t nchunks = (ncell + EPB - 1) / EPB;
+  for (int64_t it = blockIdx.x; it < nchunks * nb; it += gridDim.x) {   // batch items b0 .. b0 + nb - 1
+    const int bc = (int)(it / nchunks), b = b0 + bc;
+    const int64_t e = (it % nchunks) * EPB + el;
     __syncthreads();
-    if (tid < NB) {
-      const int64_t i = e * NB + tid;
+    if (e < ncell) {
+      const int64_t i = e * NB + t;
       const int64_t chunk = i / Nc, off = i % Nc;
       const double *Gb = G + ((chunk * nbatch + b) * 5) * Nc + off;
       const double w = pw[i];
 #pragma unroll
-      for (int c = 0; c < 5; c++) sA[c][tid] = w * Gb[c * Nc];
+      for (int c = 0; c < 5; c++) sA[el][c][t] = w * Gb[c * Nc];
     }
     __syncthreads();
-    double cd = 0.0, ck = 0.0;
-#pragma unroll 4
+    if (e >= ncell) continue;
+    double cd[S][S], ck[S][S];
+#pragma unroll
+    for (int a = 0; a < S; a++)
+#pragma unroll
+      for (int c = 0; c < S; c++) cd[a][c] = ck[a][c] = 0.0;
+#pragma unroll 2
     for (int q = 0; q < NB; q++) {
-      const double gkr = s_dxi[q][k], gkz = s_deta[q][k];
-      const double glr = s_dxi[q][l], glz = s_deta[q][l], pl = s_phi[q][l];
-      const double Arr = sA[0][q], Arz = sA[1][q], Azz = sA[2][q], Kr = sA[3][q], Kz = sA[4][q];
-      cd = fma(gkr, fma(Arr, glr, Arz * glz), cd);
-      cd = fma(gkz, fma(Arz, glr, Azz * glz), cd);
-      ck = fma(fma(gkr, Kr, gkz * Kz), pl, ck);
+      const double Arr = sA[el][0][q], Arz = sA[el][1][q], Azz = sA[el][2][q], Kr = sA[el][3][q], Kz = sA[el][4][q];
+      double u[S], v[S], pl[S], gr[S], gz[S], tk[S];
+#pragma unroll
+      for (int c = 0; c < S; c++) {
+        const double glr = s_dxi[q][l0 + c], glz = s_deta[q][l0 + c];
+        u[c] = fma(Arr, glr, Arz * glz);
+        v[c] = fma(Arz, glr, Azz * glz);
+        pl[c] = s_phi[q][l0 + c];
+        gr[c] = s_dxi[q][k0 + c];
+        gz[c] = s_deta[q][k0 + c];
+        tk[c] = fma(gr[c], Kr, gz[c] * Kz);
+      }
+#pragma unroll
+      for (int a = 0; a < S; a++)
+#pragma unroll
+        for (int c = 0; c < S; c++) {
+          cd[a][c] = fma(gr[a], u[c], fma(gz[a], v[c], cd[a][c]));
+          ck[a][c] = fma(tk[a], pl[c], ck[a][c]);
+        }
     }
-    const double s = 2.0 / cell_h[e];
-    double *o = Cbuf + ((int64_t)b * ncell + e) * 2 * NB * NB;
-    o[tid] = cd * s * s;
-    o[NB * NB + tid] = ck * s;
+    const double sc = 2.0 / cell_h[e];
+    double *o = Cbuf + ((int64_t)bc * ncell + e) * 2 * NB * NB;
+#pragma unroll
+    for (int a = 0; a < S; a++)
+#pragma unroll
+      for (int c = 0; c < S; c++) {
+        o[(k0 + a) * NB + l0 + c] = cd[a][c] * sc * sc;
+        o[NB * NB + (k0 + a) * NB + l0 + c] = ck[a][c] * sc;
+      }
   }
 }
 
@@ -537,7 +570,7 @@ struct landau_s {
   std::vector<DevMap> d_csr, d_coo;
   std::vector<double *> d_mass_csr, d_mass_coo;   // per grid
   // device: state + workspace
-  int64_t cap = 0, nbatch = 0;
+  int64_t cap = 0, nbatch = 0, chunk = 1;
   bool have_state = false;
   double *d_f = nullptr, *d_wT = nullptr, *d_part = nullptr, *d_G = nullptr, *d_C = nullptr;
   int64_t part_cap = 0;
@@ -643,7 +676,15 @@ int ensure_workspace(landau_t h, int64_t nbatch) {
   CU(cudaMalloc(&h->d_f, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
   CU(cudaMalloc(&h->d_wT, sizeof(double) * nbatch * 3 * N));
   CU(cudaMalloc(&h->d_G, sizeof(double) * nbatch * 5 * h->Nc * h->world));
-  CU(cudaMalloc(&h->d_C, sizeof(double) * nbatch * Ne * 2 * nb * nb));
+  // element-matrix chunk: <= ~40 MB so the element kernel's output is still in L2 (126 MB) when the
+  // assembly gathers it
+  const int64_t per = Ne * 2 * nb * nb * (int64_t)sizeof(double);
+  static const int64_t chunk_mb = [] {
+    const char *e = getenv("LANDAU_CHUNK_MB");
+    return e ? (int64_t)atoll(e) : (int64_t)40;
+  }();
+  h->chunk = chunk_mb <= 0 ? nbatch : std::max<int64_t>(1, std::min<int64_t>(nbatch, (chunk_mb << 20) / per));
+  CU(cudaMalloc(&h->d_C, sizeof(double) * h->chunk * Ne * 2 * nb * nb));
   h->cap = nbatch;
   return LANDAU_OK;
 }
@@ -818,11 +859,15 @@ int launch_inner(landau_t h, int64_t nbatch) {
 }
 
 template <int NB>
-int launch_element(landau_t h, int64_t nbatch) {
+int launch_element(landau_t h, int64_t nbatch, int64_t b0, int64_t nb) {
   const Plan &P = h->plan;
   Timer t(h, LANDAU_T_ELEMENT);
-  const unsigned grid = (unsigned)std::min<int64_t>(P.ncell * nbatch, (NB == 25 ? 3LL : 6LL) * num_sms(h));
-  element_kernel<NB><<<grid, NB * NB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, h->d_w, h->d_h, h->d_tab, h->d_C);
+  constexpr int S = NB == 9 ? 3 : (NB == 16 ? 4 : 5);
+  constexpr int EPB = NB == 9 ? 14 : (NB == 16 ? 8 : 5);   // ~128 threads per block
+  const int64_t items = (P.ncell + EPB - 1) / EPB * nb;
+  const unsigned grid = (unsigned)std::min<int64_t>(items, 16LL * num_sms(h));
+  element_kernel<NB, S, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, (int)b0, (int)nb,
+                                                                h->d_w, h->d_h, h->d_tab, h->d_C);
   h->launches++;
   h->tlaunch[LANDAU_T_ELEMENT]++;
   KCHECK();
@@ -830,7 +875,7 @@ int launch_element(landau_t h, int64_t nbatch) {
 }
 
 template <int NB>
-int launch_assemble(landau_t h, int64_t nbatch, double *out, int format) {
+int launch_assemble(landau_t h, int64_t nbatch, double *out, int format) {   // nbatch = items in the chunk
   const Plan &P = h->plan;
   Timer t(h, LANDAU_T_ASSEMBLE);
   const int64_t out_bstride = format == LANDAU_CSR ? h->nnz : h->ncoo;
@@ -863,8 +908,15 @@ int build_jacobian(landau_t h, int64_t nbatch, double *out, int format) {
   int rc;
   if ((rc = launch_field<NB>(h, nbatch))) return rc;
   if ((rc = launch_inner(h, nbatch))) return rc;
-  if ((rc = launch_element<NB>(h, nbatch))) return rc;
-  if (out && (rc = launch_assemble<NB>(h, nbatch, out, format))) return rc;
+  if (!out) return LANDAU_OK;   // point_coeffs: G only
+  // a-4 + a-5 in batch chunks whose element matrices stay resident in L2 between the two kernels
+  const int64_t nb = h->chunk;
+  const int64_t out_bstride = format == LANDAU_CSR ? h->nnz : h->ncoo;
+  for (int64_t b0 = 0; b0 < nbatch; b0 += nb) {
+    const int64_t n = std::min(nb, nbatch - b0);
+    if ((rc = launch_element<NB>(h, nbatch, b0, n))) return rc;
+    if ((rc = launch_assemble<NB>(h, n, out + b0 * out_bstride, format))) return rc;
+  }
   return LANDAU_OK;
 }
 
