@@ -681,7 +681,7 @@ int ensure_workspace(landau_t h, int64_t nbatch) {
   const int64_t per = Ne * 2 * nb * nb * (int64_t)sizeof(double);
   static const int64_t chunk_mb = [] {
     const char *e = getenv("LANDAU_CHUNK_MB");
-    return e ? (int64_t)atoll(e) : (int64_t)40;
+    return e ? (int64_t)atoll(e) : (int64_t)0;   // 0: one chunk (measured fastest on B200)
   }();
   h->chunk = chunk_mb <= 0 ? nbatch : std::max<int64_t>(1, std::min<int64_t>(nbatch, (chunk_mb << 20) / per));
   CU(cudaMalloc(&h->d_C, sizeof(double) * h->chunk * Ne * 2 * nb * nb));
