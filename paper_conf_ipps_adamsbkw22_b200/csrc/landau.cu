@@ -25,6 +25,21 @@
 
 using namespace landau;
 
+// build-time tuning knobs of the symmetric inner kernel (defaults = measured best on B200)
+#ifndef LANDAU_SYM_UNROLL
+#define LANDAU_SYM_UNROLL 2
+#endif
+constexpr int kSymUnroll = LANDAU_SYM_UNROLL;
+#ifndef LANDAU_SYM_SMEM_COEF
+#define LANDAU_SYM_SMEM_COEF 0
+#endif
+#ifndef LANDAU_SYM_WARPS
+#define LANDAU_SYM_WARPS 4
+#endif
+#ifndef LANDAU_SYM_MINB
+#define LANDAU_SYM_MINB 2
+#endif
+
 namespace {
 
 // Per-handle data reaches the kernels as arguments (species table by value, basis tables through
@@ -199,12 +214,12 @@ __global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_
 // Every item writes 32-point partial "slots"; reduce_sym_kernel sums, for each tile, its slots in a
 // fixed host-built order -> bitwise reproducible.  part = [batch][nslots][5][32].
 // ------------------------------------------------------------------------------------------------
-constexpr int kSymWarps = 4;
+constexpr int kSymWarps = LANDAU_SYM_WARPS;
 #ifndef LANDAU_SYM_NI
 #define LANDAU_SYM_NI 2
 #endif
 constexpr int kSymNI = LANDAU_SYM_NI;   // max i-tiles per item (independent pair chains per lane)
-static_assert(kSymNI >= 2 && kSymNI <= 3, "sym items carry 1..3 i-tiles");
+static_assert(kSymNI >= 1 && kSymNI <= 3, "sym items carry 1..3 i-tiles");
 
 struct SymItem {   // host-built, see landau_create
   int a[3];        // i-tiles (n of them, all < b); n == 0: the diagonal item (b, b)
@@ -236,10 +251,10 @@ __device__ __forceinline__ void sym_store(double *o, int lane, const Acc5 &a) {
 // The reverse sums travel with their j: at step k lane L holds the accumulator of j = (L + k) mod 32
 // and hands it to lane L - 1 by a shuffle, so consecutive steps carry no memory fence and their
 // (long, independent) pair evaluations overlap; the j data itself is read-only shared memory.
-template <int NI, bool DIAG>
+template <int NI, bool DIAG, class CF>
 __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, const double *pz, const double *wb,
                                         int64_t N, int lane, const double2 *s_rz, const double2 *s_w,
-                                        const double *s_wz, const PairCoef &cf, double *o) {
+                                        const double *s_wz, const CF &cf, double *o) {
   double r[NI], z[NI], wd[NI], wkr[NI], wkz[NI];
   Acc5 ai[NI];
 #pragma unroll
@@ -251,7 +266,7 @@ __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, con
   constexpr int k0 = DIAG ? 1 : 0, k1 = DIAG ? 17 : 32;
   const int src = (lane + 1) & 31;
   Acc5 aj{0.0, 0.0, 0.0, 0.0, 0.0};
-#pragma unroll 2
+#pragma unroll kSymUnroll
   for (int k = k0; k < k1; k++) {
     const int jj = (lane + k) & 31;
     const double2 rz = s_rz[jj], w = s_w[jj];
@@ -288,11 +303,19 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t
                                                                          double *__restrict__ part) {
   __shared__ double2 s_rz[kSymWarps][32], s_w[kSymWarps][32];
   __shared__ double s_wz[kSymWarps][32];
+#if LANDAU_SYM_SMEM_COEF
+  __shared__ __align__(16) double s_coef[kNumSmemCoef];
+  stage_smem_coef(s_coef);
+  __syncthreads();
+  const SmemCoef cf{reinterpret_cast<const double2 *>(s_coef), reinterpret_cast<const double2 *>(s_coef) + ELL_D_DEG + 1,
+                    s_coef + 4 * (ELL_D_DEG + 1)};
+#else
   __shared__ double s_coef[kNumPairCoef];
   stage_pair_coef(s_coef);
   __syncthreads();
   PairCoef cf;
   load_pair_coef(s_coef, cf);
+#endif
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   // persistent warps: grid-stride over the (batch item, work item) list
   for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
@@ -312,7 +335,9 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t
   switch (it.n) {
     case 0: sym_run<1, true>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
     case 1: sym_run<1, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
-    case 2: sym_run<2, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
+    case 2:
+      if constexpr (kSymNI >= 2) sym_run<2, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
+      break;
     default:
       if constexpr (kSymNI >= 3) sym_run<kSymNI, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
       break;
@@ -796,8 +821,8 @@ int launch_inner(landau_t h, int64_t nbatch) {
     {
       Timer t(h, LANDAU_T_INNER);
       const int64_t nitems = nbatch * h->nsym_items;
-      const unsigned grid = (unsigned)std::min<int64_t>((nitems + kSymWarps - 1) / kSymWarps, 2LL * num_sms(h));
-      inner_sym_kernel<2><<<grid, 32 * kSymWarps, 0, h->stream>>>(N, h->nsym_items, h->nsym_slots, nitems,
+      const unsigned grid = (unsigned)std::min<int64_t>((nitems + kSymWarps - 1) / kSymWarps, (int64_t)LANDAU_SYM_MINB * num_sms(h));
+      inner_sym_kernel<LANDAU_SYM_MINB><<<grid, 32 * kSymWarps, 0, h->stream>>>(N, h->nsym_items, h->nsym_slots, nitems,
                                                                    h->d_sym_items, h->d_r, h->d_z, h->d_wT, h->d_part);
       h->launches++;
       h->tlaunch[LANDAU_T_INNER]++;
