@@ -130,8 +130,9 @@ int landau_jacobian(landau_t h, double *values_dev, int32_t format);
 int landau_jacobian_batched(landau_t h, int64_t nbatch, double *values_dev, int32_t format);
 
 /* Convenience for host data (end-to-end path): copies f_host [nbatch][ndof] to the device, builds,
- * copies the values back to values_host [nbatch][nnz] and synchronises the stream.  Pinned host
- * memory gives asynchronous copies. */
+ * copies the values back to values_host [nbatch][nnz] and synchronises.  Large batches are cut into
+ * up to 8 chunks whose uploads, builds and downloads overlap on two internal copy streams (pinned
+ * host memory required for the overlap).  Does not change the handle's set_state state. */
 int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, double *values_host, int32_t format);
 
 /* Mass matrix values shift * M for every species block: [nnz_csr] or [ncoo]. */

@@ -603,9 +603,12 @@ struct landau_s {
   int32_t *d_tile_ptr = nullptr, *d_tile_slots = nullptr;
   int ntiles = 0;
   int64_t nsym_items = 0, nsym_slots = 0;
-  // host staging for landau_jacobian_host
+  // host staging for landau_jacobian_host: full-batch device buffers, two copy streams
   double *d_vals_tmp = nullptr;
   int64_t vals_tmp_cap = 0;
+  cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+  std::vector<cudaEvent_t> ev_h2d, ev_built;
+  const double *fin = nullptr;   // state read by the field kernel (nullptr: d_f)
   // timing
   bool timing = false;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> ev_used;
@@ -618,6 +621,7 @@ struct landau_s {
     int64_t nbatch;
     int format;
     double *out;
+    const double *fin;
     cudaGraphExec_t exec;
     int64_t kernels;
   };
@@ -731,7 +735,8 @@ int launch_field(landau_t h, int64_t nbatch) {
   const int64_t items = (P.ncell + EPB - 1) / EPB * nbatch;
   const unsigned grid = (unsigned)std::min<int64_t>(items, 8LL * num_sms(h));
   Timer t(h, LANDAU_T_FIELD);
-  field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->d_f, h->d_ext_ptr, h->d_ext_dof,
+  field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->fin ? h->fin : h->d_f,
+                                                          h->d_ext_ptr, h->d_ext_dof,
                                                           h->d_ext_w, h->d_cell_grid, h->d_h, h->d_w, h->d_tab, h->spc, h->d_wT, P.npts);
   h->launches++;
   h->tlaunch[LANDAU_T_FIELD]++;
@@ -960,7 +965,7 @@ int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
   if (h->timing || !h->use_graphs || !h->stream || h->comm || !out)
     return dispatch_build_direct(h, nbatch, out, format);
   for (auto &g : h->graphs)
-    if (g.nbatch == nbatch && g.format == format && g.out == out) {
+    if (g.nbatch == nbatch && g.format == format && g.out == out && g.fin == h->fin) {
       CU(cudaGraphLaunch(g.exec, h->stream));
       h->launches += g.kernels;
       return LANDAU_OK;
@@ -987,11 +992,11 @@ int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
   ce = cudaGraphInstantiate(&exec, graph, 0);
   cudaGraphDestroy(graph);
   if (ce != cudaSuccess) return fail(h, LANDAU_ECUDA, std::string("graph instantiate: ") + cudaGetErrorString(ce));
-  if (h->graphs.size() >= 8) {
+  if (h->graphs.size() >= 16) {
     cudaGraphExecDestroy(h->graphs.front().exec);
     h->graphs.erase(h->graphs.begin());
   }
-  h->graphs.push_back({nbatch, format, out, exec, kernels});
+  h->graphs.push_back({nbatch, format, out, h->fin, exec, kernels});
   CU(cudaGraphLaunch(exec, h->stream));
   h->launches += kernels;
   return LANDAU_OK;
@@ -1227,6 +1232,10 @@ void landau_destroy(landau_t h) {
   cudaSetDevice(h->device);
   if (h->stream) cudaStreamSynchronize(h->stream);
   drop_graphs(h);
+  if (h->s_h2d) cudaStreamDestroy(h->s_h2d);
+  if (h->s_d2h) cudaStreamDestroy(h->s_d2h);
+  for (auto e : h->ev_h2d) cudaEventDestroy(e);
+  for (auto e : h->ev_built) cudaEventDestroy(e);
   if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
   for (double *p : {h->d_r, h->d_z, h->d_w, h->d_h, h->d_tab, h->d_ext_w, h->d_f, h->d_wT, h->d_part, h->d_G, h->d_C, h->d_vals_tmp})
     cudaFree(p);
@@ -1335,6 +1344,11 @@ int landau_jacobian(landau_t h, double *values_dev, int32_t format) {
   return landau_jacobian_batched(h, 1, values_dev, format);
 }
 
+// End-to-end entry: the batch is cut into K chunks; chunk c's upload (stream s_h2d), its build
+// (the handle's stream) and its download (stream s_d2h) are ordered by events, so downloads of
+// finished chunks overlap the builds of later ones.  Chunks are independent vertices, so the
+// values are identical to one whole-batch build up to the split-j / symmetric grouping (the same
+// for every chunk size at or above the symmetric threshold).
 int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, double *values_host, int32_t format) {
   if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
   if (!h || nbatch < 1 || !f_host || !values_host || (format != LANDAU_CSR && format != LANDAU_COO))
@@ -1343,16 +1357,48 @@ int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, doubl
   if (rc) return rc;
   const int64_t nv = format == LANDAU_CSR ? h->nnz : h->ncoo;
   if (nbatch * nv > h->vals_tmp_cap) {
+    drop_graphs(h);
     cudaFree(h->d_vals_tmp);
     h->d_vals_tmp = nullptr;
     CU(cudaMalloc(&h->d_vals_tmp, sizeof(double) * nbatch * nv));
     h->vals_tmp_cap = nbatch * nv;
   }
-  CU(cudaMemcpyAsync(h->d_f, f_host, sizeof(double) * nbatch * h->ndof, cudaMemcpyHostToDevice, h->stream));
-  h->nbatch = nbatch;
-  h->have_state = true;
-  if ((rc = dispatch_build(h, nbatch, h->d_vals_tmp, format))) return rc;
-  CU(cudaMemcpyAsync(values_host, h->d_vals_tmp, sizeof(double) * nbatch * nv, cudaMemcpyDeviceToHost, h->stream));
+  if (!h->s_h2d) {
+    CU(cudaStreamCreateWithFlags(&h->s_h2d, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&h->s_d2h, cudaStreamNonBlocking));
+  }
+  const int64_t K = std::max<int64_t>(1, std::min<int64_t>(8, nbatch / 64));
+  const int64_t cb = (nbatch + K - 1) / K;
+  while ((int64_t)h->ev_h2d.size() < K) {
+    cudaEvent_t a, b;
+    CU(cudaEventCreateWithFlags(&a, cudaEventDisableTiming));
+    CU(cudaEventCreateWithFlags(&b, cudaEventDisableTiming));
+    h->ev_h2d.push_back(a);
+    h->ev_built.push_back(b);
+  }
+  // the copies may only start once earlier work on the handle's stream is done with the buffers
+  CU(cudaEventRecord(h->ev_built[0], h->stream));
+  CU(cudaStreamWaitEvent(h->s_h2d, h->ev_built[0], 0));
+  CU(cudaStreamWaitEvent(h->s_d2h, h->ev_built[0], 0));
+  for (int64_t c = 0; c < K; c++) {
+    const int64_t b0 = c * cb, n = std::min(cb, nbatch - b0);
+    if (n <= 0) break;
+    CU(cudaMemcpyAsync(h->d_f + b0 * h->ndof, f_host + b0 * h->ndof, sizeof(double) * n * h->ndof,
+                       cudaMemcpyHostToDevice, h->s_h2d));
+    CU(cudaEventRecord(h->ev_h2d[c], h->s_h2d));
+    CU(cudaStreamWaitEvent(h->stream, h->ev_h2d[c], 0));
+    h->fin = h->d_f + b0 * h->ndof;
+    rc = dispatch_build(h, n, h->d_vals_tmp + b0 * nv, format);
+    h->fin = nullptr;
+    if (rc) return rc;
+    CU(cudaEventRecord(h->ev_built[c], h->stream));
+    CU(cudaStreamWaitEvent(h->s_d2h, h->ev_built[c], 0));
+    CU(cudaMemcpyAsync(values_host + b0 * nv, h->d_vals_tmp + b0 * nv, sizeof(double) * n * nv,
+                       cudaMemcpyDeviceToHost, h->s_d2h));
+  }
+  h->nbatch = cb;          // the device state now holds the last chunk's batch layout
+  h->have_state = false;   // (d_f holds the whole host batch, but not as one set_state)
+  CU(cudaStreamSynchronize(h->s_d2h));
   CU(cudaStreamSynchronize(h->stream));
   return LANDAU_OK;
 }
