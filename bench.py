@@ -36,7 +36,7 @@ UNIT = "builds/s"
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="landau", choices=["landau", "reference"])
     ap.add_argument("--workload", default="C4", choices=["C4", "C2", "C3", "C5"])
@@ -122,9 +122,13 @@ def load_profile_traffic(workload):
         return None
 
 
-# FP64 FLOP per ordered pair, executed on the fast path of landau_pair (2*DFMA + DMUL + DADD), counted
-# once from ncu sm__sass_thread_inst_executed_op_{dfma,dmul,dadd}_pred_on / pairs.
-FLOP_PER_PAIR = float(os.environ.get("LANDAU_FLOP_PER_PAIR", "193"))
+# FP64 FLOP (2*DFMA + DMUL + DADD) per pair evaluation, counted once from ncu
+# sm__sass_thread_inst_executed_op_{dfma,dmul,dadd}_pred_on of each inner kernel on the C4 workload
+# (profiles/r01_inner_ncu.txt):
+#   directed kernel:  193 FLOP per ordered (target, source) pair, N^2 per batch item
+#   symmetric kernel: 207 FLOP per unordered pair, N (N - 1) / 2 per batch item (both targets updated)
+FLOP_PER_PAIR_DIRECTED = 193.0
+FLOP_PER_PAIR_SYMMETRIC = 207.0
 
 
 def cpu_baseline(args, desc, nsample):
@@ -296,18 +300,26 @@ def main():
     # ---- roofline of the dominant kernel (inner integral, FP64 pipe) --------------------------
     inner_ms, inner_n = tim["inner"]
     inner_avg_s = inner_ms / max(inner_n, 1) / 1e3
-    flops_per_launch = FLOP_PER_PAIR * pairs_per_build * max(nloc, 1)
+    st = h.stats()
+    if st["inner_path"] == 1:
+        flop_per_pair = FLOP_PER_PAIR_SYMMETRIC
+        flops_per_launch = flop_per_pair * st["nbatch"] * N * (N - 1) / 2
+    else:
+        flop_per_pair = FLOP_PER_PAIR_DIRECTED
+        flops_per_launch = flop_per_pair * st["nbatch"] * st["targets"] * N
     achieved = flops_per_launch / inner_avg_s / 1e12 if inner_n else None
     clocks = clk.summary()
     props = torch.cuda.get_device_properties(local)
     sm_max = clocks["sm_max_mhz"] or 1965.0
     peak = fp64_peak_tflops(props, sm_max)
     step_ms_lib = sum(v[0] for v in tim.values()) / args.steps
-    roof = {"bound": "alu", "kernel": "inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
+    roof = {"bound": "alu", "kernel": "inner_sym_kernel / inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
             "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None,
             "traffic": load_profile_traffic(args.workload),
             "peak_note": f"derived FP64 DFMA peak: {props.multi_processor_count} SMs x 64 lanes x 2 FLOP x {sm_max:.0f} MHz",
-            "flop_per_pair": FLOP_PER_PAIR, "inner_ms_per_launch": inner_avg_s * 1e3,
+            "inner_path": "symmetric (unordered pairs)" if st["inner_path"] == 1 else "directed (ordered pairs)",
+            "flop_per_pair": flop_per_pair, "flops_per_launch": flops_per_launch,
+            "inner_ms_per_launch": inner_avg_s * 1e3,
             "inner_share_of_step": (inner_ms / args.steps) / ms_per_step if ms_per_step else None,
             "pairs_per_s_inner": pairs_per_build * max(nloc, 1) / inner_avg_s * world if inner_n else None}
     stage_ms = {k: v[0] / args.steps for k, v in tim.items()}

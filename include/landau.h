@@ -159,6 +159,19 @@ int landau_get_timing(landau_t h, double *ms, int64_t *launches);
 /* kernels launched by this handle since creation (all stages) */
 int landau_get_launch_count(landau_t h, int64_t *count);
 
+/* How the last build ran (for FLOP accounting and diagnostics). */
+typedef struct {
+  int32_t inner_path;        /* 0: directed pair kernel (every ordered pair, split-j when small);
+                                1: symmetric pair kernel (every unordered pair once, both targets)  */
+  int64_t nbatch;            /* batch items of the last build                                      */
+  int64_t targets;           /* target points per batch item (all N unless element-split)          */
+  int64_t sources;           /* source points per batch item (N)                                   */
+  int64_t pair_evaluations;  /* pair-body evaluations issued, per batch item, including padded and
+                                masked lanes: directed ~ targets x sources, symmetric ~ N^2 / 2    */
+  int64_t nsplit;            /* source splits (directed path)                                      */
+} landau_stats_t;
+int landau_get_stats(landau_t h, landau_stats_t *stats);
+
 const char *landau_strerror(int code);
 /* last detailed error message of a handle (or of the last failed create when h == NULL) */
 const char *landau_last_error(landau_t h);

@@ -609,6 +609,7 @@ struct landau_s {
   cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
   std::vector<cudaEvent_t> ev_h2d, ev_built;
   const double *fin = nullptr;   // state read by the field kernel (nullptr: d_f)
+  landau_stats_t stats{};        // how the last build ran
   // timing
   bool timing = false;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> ev_used;
@@ -822,6 +823,18 @@ int launch_inner(landau_t h, int64_t nbatch) {
   const int variant = inner_variant();
   const int64_t wtiles = ip.wtiles, nsplit = ip.nsplit, split_len = ip.split_len;
   double *G_own = h->d_G + (int64_t)h->rank * nbatch * 5 * h->Nc;   // [world][batch][5][Nc]
+  h->stats.nbatch = nbatch;
+  h->stats.targets = nt;
+  h->stats.sources = N;
+  h->stats.inner_path = ip.sym ? 1 : 0;
+  h->stats.nsplit = ip.sym ? 1 : ip.nsplit;
+  if (ip.sym) {
+    int64_t ev = 0;   // lane-steps per batch item: diagonal items 16 x 32, others 32 x 32 per i-tile
+    ev = (int64_t)h->ntiles * 16 * 32 + (int64_t)h->ntiles * (h->ntiles - 1) / 2 * 32 * 32;
+    h->stats.pair_evaluations = ev;
+  } else {
+    h->stats.pair_evaluations = ip.wtiles * 32 * ip.tpt * N;
+  }
   if (ip.sym) {
     {
       Timer t(h, LANDAU_T_INNER);
@@ -1468,6 +1481,12 @@ int landau_get_timing(landau_t h, double *ms, int64_t *launches) {
     if (ms) ms[i] = acc[i];
     if (launches) launches[i] = h->tlaunch[i];
   }
+  return LANDAU_OK;
+}
+
+int landau_get_stats(landau_t h, landau_stats_t *stats) {
+  if (!h || !stats) return LANDAU_EINVAL;
+  *stats = h->stats;
   return LANDAU_OK;
 }
 

@@ -41,6 +41,11 @@ class _Params(C.Structure):
                 ("grid", C.POINTER(C.c_int32)), ("nu", C.c_double)]
 
 
+class _Stats(C.Structure):
+    _fields_ = [("inner_path", C.c_int32), ("nbatch", C.c_int64), ("targets", C.c_int64), ("sources", C.c_int64),
+                ("pair_evaluations", C.c_int64), ("nsplit", C.c_int64)]
+
+
 class _Dist(C.Structure):
     _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("nccl_unique_id", C.c_void_p), ("mode", C.c_int32)]
 
@@ -75,6 +80,7 @@ def lib():
             "landau_set_timing": (C.c_int, [vp, i32]),
             "landau_get_timing": (C.c_int, [vp, Pd, P64]),
             "landau_get_launch_count": (C.c_int, [vp, P64]),
+            "landau_get_stats": (C.c_int, [vp, C.POINTER(_Stats)]),
             "landau_strerror": (C.c_char_p, [C.c_int]),
             "landau_last_error": (C.c_char_p, [vp]),
             "landau_version": (C.c_char_p, []),
@@ -265,6 +271,11 @@ class Landau:
         self._check(lib().landau_get_timing(self._h, _dptr(ms), n.ctypes.data_as(C.POINTER(C.c_int64))),
                     "landau_get_timing")
         return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(TIMERS)}
+
+    def stats(self):
+        st = _Stats()
+        self._check(lib().landau_get_stats(self._h, C.byref(st)), "landau_get_stats")
+        return {k: getattr(st, k) for k, _ in _Stats._fields_}
 
     def launch_count(self):
         n = C.c_int64()
