@@ -775,8 +775,10 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
   const Plan &P = h->plan;
   const int64_t N = P.npts, nt = (h->e1 - h->e0) * P.nqp;
   const int variant = inner_variant();
-  ip.sym = sym_enabled() && !h->comm && h->nsym_items > 0 && nbatch * h->nsym_items >= 8LL * kSymWarps * num_sms(h) &&
-           nbatch * h->nsym_slots * 160 * (int64_t)sizeof(double) <= (8LL << 30);
+  // symmetric path: all targets on this rank (no element split across ranks), enough work items to
+  // fill the GPU, and partial slots within 24 GiB (C5: ~11 GiB of the 180 GB HBM)
+  ip.sym = sym_enabled() && h->world == 1 && h->nsym_items > 0 && nbatch * h->nsym_items >= 8LL * kSymWarps * num_sms(h) &&
+           nbatch * h->nsym_slots * 160 * (int64_t)sizeof(double) <= (24LL << 30);
   if (ip.sym) {
     ip.tpt = 1;
     ip.wtiles = h->ntiles;
@@ -1174,7 +1176,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     tab.insert(tab.end(), P.tab_deta.begin(), P.tab_deta.end());
     if ((rc = upload(h, &h->d_tab, tab))) return bail(rc);
   }
-  if (mode != LANDAU_DIST_ELEMENTS) {   // work items + slot map of the symmetric inner kernel
+  if (world == 1) {   // work items + slot map of the symmetric inner kernel
     const int T = (int)((P.npts + 31) / 32);
     std::vector<SymItem> items;
     std::vector<std::vector<int32_t>> slots_of(T);
