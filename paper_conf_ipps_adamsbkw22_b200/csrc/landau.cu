@@ -143,8 +143,7 @@ __global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_
                                                              const double *__restrict__ pr, const double *__restrict__ pz,
                                                              const double *__restrict__ wT, double *__restrict__ out,
                                                              int64_t out_bstride) {
-  __shared__ double2 s_rz[kInnerWarps][32], s_w[kInnerWarps][32];
-  __shared__ double s_wz[kInnerWarps][32];
+  __shared__ double2 s_rz[kInnerWarps][32], s_w[kInnerWarps][32], s_wz[kInnerWarps][32];   // (wkz, rb^2)
   __shared__ double s_coef[kNumPairCoef];
   stage_pair_coef(s_coef);
   __syncthreads();
@@ -159,7 +158,7 @@ __global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_
   const int64_t wt = rem % wtiles;
   const double *wb = wT + b * 3 * N;
   int64_t ti[TPT];
-  double tr[TPT], tz[TPT];
+  double tr[TPT], tz[TPT], tr2[TPT];
   Acc5 acc[TPT];
 #pragma unroll
   for (int t = 0; t < TPT; t++) {
@@ -167,6 +166,7 @@ __global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_
     const int64_t gi = t0 + (ti[t] < nt ? ti[t] : nt - 1);
     tr[t] = pr[gi];
     tz[t] = pz[gi];
+    tr2[t] = tr[t] * tr[t];
     acc[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
   }
   const int64_t j0 = (int64_t)split * split_len;
@@ -175,18 +175,18 @@ __global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_
     const int64_t j = jt + lane;
     __syncwarp();
     if (j < j1) {
-      s_rz[wid][lane] = make_double2(pr[j], pz[j]);
+      const double rj = pr[j];
+      s_rz[wid][lane] = make_double2(rj, pz[j]);
       s_w[wid][lane] = make_double2(wb[j], wb[N + j]);
-      s_wz[wid][lane] = wb[2 * N + j];
+      s_wz[wid][lane] = make_double2(wb[2 * N + j], rj * rj);
     }
     __syncwarp();
     const int n = (int)min((int64_t)32, j1 - jt);
 #pragma unroll 2
     for (int k = 0; k < n; k++) {
-      const double2 rz = s_rz[wid][k], w = s_w[wid][k];
-      const double wkz = s_wz[wid][k];
+      const double2 rz = s_rz[wid][k], w = s_w[wid][k], wz = s_wz[wid][k];
 #pragma unroll
-      for (int t = 0; t < TPT; t++) landau_pair(tr[t], tz[t], rz.x, rz.y, w.x, w.y, wkz, cf, acc[t]);
+      for (int t = 0; t < TPT; t++) landau_pair(tr[t], tz[t], tr2[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, cf, acc[t]);
     }
   }
   double *o = out + b * out_bstride + (int64_t)split * 5 * nt;
@@ -254,13 +254,14 @@ __device__ __forceinline__ void sym_store(double *o, int lane, const Acc5 &a) {
 template <int NI, bool DIAG, class CF>
 __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, const double *pz, const double *wb,
                                         int64_t N, int lane, const double2 *s_rz, const double2 *s_w,
-                                        const double *s_wz, const CF &cf, double *o) {
-  double r[NI], z[NI], wd[NI], wkr[NI], wkz[NI];
+                                        const double2 *s_wz, const CF &cf, double *o) {
+  double r[NI], z[NI], r2[NI], wd[NI], wkr[NI], wkz[NI];
   Acc5 ai[NI];
 #pragma unroll
   for (int t = 0; t < NI; t++) {
     sym_load_i(pr, pz, wb, N, (int64_t)(DIAG ? it.b : it.a[t]) * 32 + lane, 1.0e6 + 64.0 * t + lane, r[t], z[t], wd[t],
                wkr[t], wkz[t]);
+    r2[t] = r[t] * r[t];
     ai[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
   }
   constexpr int k0 = DIAG ? 1 : 0, k1 = DIAG ? 17 : 32;
@@ -269,12 +270,11 @@ __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, con
 #pragma unroll kSymUnroll
   for (int k = k0; k < k1; k++) {
     const int jj = (lane + k) & 31;
-    const double2 rz = s_rz[jj], w = s_w[jj];
-    const double wkz_j = s_wz[jj];
+    const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
     const bool on = !DIAG || !(k == 16 && lane >= 16);
 #pragma unroll
     for (int t = 0; t < NI; t++)
-      landau_pair_sym(r[t], z[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, w.x, w.y, wkz_j, on, cf, ai[t], aj);
+      landau_pair_sym(r[t], z[t], r2[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, on, cf, ai[t], aj);
     aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
     aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
     aj.dzz = __shfl_sync(0xffffffffu, aj.dzz, src);
@@ -301,8 +301,7 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t
                                                                          const double *__restrict__ pz,
                                                                          const double *__restrict__ wT,
                                                                          double *__restrict__ part) {
-  __shared__ double2 s_rz[kSymWarps][32], s_w[kSymWarps][32];
-  __shared__ double s_wz[kSymWarps][32];
+  __shared__ double2 s_rz[kSymWarps][32], s_w[kSymWarps][32], s_wz[kSymWarps][32];   // (wkz, rb^2)
 #if LANDAU_SYM_SMEM_COEF
   __shared__ __align__(16) double s_coef[kNumSmemCoef];
   stage_smem_coef(s_coef);
@@ -328,7 +327,7 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t
     sym_load_i(pr, pz, wb, N, (int64_t)it.b * 32 + lane, 2.0e6 + lane, r, z, wd, wkr, wkz);
     s_rz[wid][lane] = make_double2(r, z);
     s_w[wid][lane] = make_double2(wd, wkr);
-    s_wz[wid][lane] = wkz;
+    s_wz[wid][lane] = make_double2(wkz, r * r);
   }
   __syncwarp();
   double *o = part + (bb * nslots + it.slot) * 160;
