@@ -251,7 +251,7 @@ __device__ __forceinline__ void sym_store(double *o, int lane, const Acc5 &a) {
 // The reverse sums travel with their j: at step k lane L holds the accumulator of j = (L + k) mod 32
 // and hands it to lane L - 1 by a shuffle, so consecutive steps carry no memory fence and their
 // (long, independent) pair evaluations overlap; the j data itself is read-only shared memory.
-template <int NI, bool DIAG, class CF>
+template <int NI, bool DIAG, bool MASK, class CF>
 __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, const double *pz, const double *wb,
                                         int64_t N, int lane, const double2 *s_rz, const double2 *s_w,
                                         const double2 *s_wz, const CF &cf, double *o) {
@@ -267,14 +267,27 @@ __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, con
   constexpr int k0 = DIAG ? 1 : 0, k1 = DIAG ? 17 : 32;
   const int src = (lane + 1) & 31;
   Acc5 aj{0.0, 0.0, 0.0, 0.0, 0.0};
+  // diagonal items: steps 1..15 are unmasked, step 16 (lanes >= 16 would double-count) is peeled
+  constexpr int kmain = DIAG ? 16 : 32;
 #pragma unroll kSymUnroll
-  for (int k = k0; k < k1; k++) {
+  for (int k = k0; k < kmain; k++) {
     const int jj = (lane + k) & 31;
     const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
-    const bool on = !DIAG || !(k == 16 && lane >= 16);
 #pragma unroll
     for (int t = 0; t < NI; t++)
-      landau_pair_sym(r[t], z[t], r2[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, on, cf, ai[t], aj);
+      landau_pair_sym<CF, MASK>(r[t], z[t], r2[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, true, cf,
+                                ai[t], aj);
+    aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
+    aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
+    aj.dzz = __shfl_sync(0xffffffffu, aj.dzz, src);
+    aj.kr = __shfl_sync(0xffffffffu, aj.kr, src);
+    aj.kz = __shfl_sync(0xffffffffu, aj.kz, src);
+  }
+  if constexpr (DIAG) {
+    const int jj = (lane + 16) & 31;
+    const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
+    landau_pair_sym<CF, true>(r[0], z[0], r2[0], wd[0], wkr[0], wkz[0], rz.x, rz.y, wz.y, w.x, w.y, wz.x, lane < 16, cf,
+                              ai[0], aj);
     aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
     aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
     aj.dzz = __shfl_sync(0xffffffffu, aj.dzz, src);
@@ -293,7 +306,7 @@ __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, con
   oj[128 + jf] = aj.kz;
 }
 
-template <int MINB>
+template <int MINB, bool MASK>
 __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t N, int64_t nitems_b, int64_t nslots,
                                                                          int64_t nitems,
                                                                          const SymItem *__restrict__ items,
@@ -332,13 +345,14 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t
   __syncwarp();
   double *o = part + (bb * nslots + it.slot) * 160;
   switch (it.n) {
-    case 0: sym_run<1, true>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
-    case 1: sym_run<1, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
+    case 0: sym_run<1, true, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
+    case 1: sym_run<1, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
     case 2:
-      if constexpr (kSymNI >= 2) sym_run<2, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
+      if constexpr (kSymNI >= 2) sym_run<2, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
       break;
     default:
-      if constexpr (kSymNI >= 3) sym_run<kSymNI, false>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
+      if constexpr (kSymNI >= 3)
+        sym_run<kSymNI, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
       break;
   }
   }
@@ -602,6 +616,7 @@ struct landau_s {
   int32_t *d_tile_ptr = nullptr, *d_tile_slots = nullptr;
   int ntiles = 0;
   int64_t nsym_items = 0, nsym_slots = 0;
+  bool coincident = false;   // two distinct quadrature points with identical (r, z) (never for one grid)
   // host staging for landau_jacobian_host: full-batch device buffers, two copy streams
   double *d_vals_tmp = nullptr;
   int64_t vals_tmp_cap = 0;
@@ -841,8 +856,12 @@ int launch_inner(landau_t h, int64_t nbatch) {
       Timer t(h, LANDAU_T_INNER);
       const int64_t nitems = nbatch * h->nsym_items;
       const unsigned grid = (unsigned)std::min<int64_t>((nitems + kSymWarps - 1) / kSymWarps, (int64_t)LANDAU_SYM_MINB * num_sms(h));
-      inner_sym_kernel<LANDAU_SYM_MINB><<<grid, 32 * kSymWarps, 0, h->stream>>>(N, h->nsym_items, h->nsym_slots, nitems,
-                                                                   h->d_sym_items, h->d_r, h->d_z, h->d_wT, h->d_part);
+      if (h->coincident)   // distinct points share coordinates somewhere: mask every pair (Amb-3)
+        inner_sym_kernel<LANDAU_SYM_MINB, true><<<grid, 32 * kSymWarps, 0, h->stream>>>(
+            N, h->nsym_items, h->nsym_slots, nitems, h->d_sym_items, h->d_r, h->d_z, h->d_wT, h->d_part);
+      else
+        inner_sym_kernel<LANDAU_SYM_MINB, false><<<grid, 32 * kSymWarps, 0, h->stream>>>(
+            N, h->nsym_items, h->nsym_slots, nitems, h->d_sym_items, h->d_r, h->d_z, h->d_wT, h->d_part);
       h->launches++;
       h->tlaunch[LANDAU_T_INNER]++;
       KCHECK();
@@ -1174,6 +1193,13 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     tab.insert(tab.end(), P.tab_dxi.begin(), P.tab_dxi.end());
     tab.insert(tab.end(), P.tab_deta.begin(), P.tab_deta.end());
     if ((rc = upload(h, &h->d_tab, tab))) return bail(rc);
+  }
+  {   // do two distinct points share their coordinates (only possible across grids)?
+    std::vector<std::pair<double, double>> rz(P.npts);
+    for (int64_t i = 0; i < P.npts; i++) rz[i] = {P.pr[i], P.pz[i]};
+    std::sort(rz.begin(), rz.end());
+    for (int64_t i = 1; i < P.npts; i++)
+      if (rz[i] == rz[i - 1]) h->coincident = true;
   }
   if (world == 1) {   // work items + slot map of the symmetric inner kernel
     const int T = (int)((P.npts + 31) / 32);

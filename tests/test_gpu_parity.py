@@ -312,3 +312,33 @@ def test_host_entry_pipelined_chunks_match_device_batch():
     vh = torch.full((nb, h.nnz), float("nan"), dtype=torch.float64).pin_memory()
     h.jacobian_host(fh, vh)
     assert np.array_equal(vh.numpy().view(np.uint64), ref.view(np.uint64))
+
+
+def test_symmetric_kernel_with_coincident_points():
+    """Two species on two identical grids: every point has a distinct twin with identical (r, z), so
+    the library must take the masked symmetric kernel (Amb-3: coincident pairs contribute nothing)."""
+    R = inputs.R_E
+    mesh = inputs.origin_chain(R, 3)
+    prob = inputs.Problem("twin", 3, [(R, mesh), (R, mesh)],
+                          [inputs.Species("e", 1.0, -1.0, 0), inputs.Species("D", inputs.M_D, 1.0, 1)],
+                          fmix=[[(1.0, 1.0, 0.0)], [(1.0, 0.5, 0.0)]], seed=99)
+    h = L.Landau.from_problem(prob, device=0)
+    nodes = h.all_nodes()
+    nb = 48
+    fs = []
+    for b in range(nb):
+        p = inputs.Problem("twin", 3, prob.grids, prob.species, fmix=[[(1.0 + 0.01 * b, 1.0, 0.0)], [(1.0, 0.5, 0.0)]],
+                           seed=99 + b)
+        fs.append(inputs.coefficients(p, nodes))
+    h.set_state_batched(torch.tensor(np.stack(fs), device=DEV))
+    out = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
+    h.jacobian_batched(out)
+    torch.cuda.synchronize()
+    assert h.stats()["inner_path"] == 1
+    Jb = out.cpu().numpy()
+    for b in (0, nb - 1):
+        p = inputs.Problem("twin", 3, prob.grids, prob.species, fmix=[[(1.0 + 0.01 * b, 1.0, 0.0)], [(1.0, 0.5, 0.0)]],
+                           seed=99 + b)
+        o = Oracle(p)
+        Jo, Ja = o.jacobian(o.coefficients())
+        assert np.all(np.abs(Jb[b] - Jo) <= 1e-11 * Ja)
