@@ -39,7 +39,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="landau", choices=["landau", "reference"])
-    ap.add_argument("--workload", default="C4", choices=["C4", "C2", "C3", "C5"])
+    ap.add_argument("--workload", default="C4", choices=["C4", "C1", "C2", "C3", "C5"])
     ap.add_argument("--batch", type=int, default=1024, help="C4 vertices in the whole job")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle vertices for cpu_baseline (0 = auto)")

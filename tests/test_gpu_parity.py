@@ -342,3 +342,30 @@ def test_symmetric_kernel_with_coincident_points():
         o = Oracle(p)
         Jo, Ja = o.jacobian(o.coefficients())
         assert np.all(np.abs(Jb[b] - Jo) <= 1e-11 * Ja)
+
+
+def _adhoc(order, mesh, species_grid=(0, 0)):
+    R = inputs.R_E
+    sp = [inputs.Species("e", 1.0, -1.0, species_grid[0]), inputs.Species("D", inputs.M_D, 1.0, species_grid[1])]
+    grids = [(R, mesh)] * (max(species_grid) + 1)
+    return inputs.Problem(f"Q{order}", order, grids, sp, fmix=[[(1.0, 1.0, 0.0), (0.3, 0.2, 0.4)], [(1.3, 0.5, 0.0)]],
+                          seed=4242 + order)
+
+
+@pytest.mark.parametrize("order,mesh", [(4, "A"), (2, "C2"), (4, "chain6")])
+def test_full_parity_other_orders(order, mesh):
+    """Full-Jacobian parity (every CSR entry, every G) for Q2 and Q4 AMR meshes with hanging nodes."""
+    R = inputs.R_E
+    cells = {"A": inputs.origin_chain(R, 3), "C2": inputs.c2_mesh(), "chain6": inputs.origin_chain(R, 6)}[mesh]
+    prob = _adhoc(order, cells)
+    h = L.Landau.from_problem(prob, device=0)
+    o = Oracle(prob)
+    fg, fo = inputs.coefficients(prob, h.all_nodes()), o.coefficients()
+    G = gpu_G(h, fg)
+    Go, Ga = o.point_coeffs(fo)
+    assert np.max(np.abs(G - Go) / Ga) <= 1e-12
+    J = gpu_jacobian(h, fg)
+    Jo, Ja = o.jacobian(fo)
+    assert np.all(np.abs(J - Jo) <= 1e-11 * Ja)
+    d, m, e = _conservation(prob, h, J, fg)
+    assert max(d, m, e) < 1e-13, (d, m, e)

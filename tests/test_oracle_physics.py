@@ -204,3 +204,27 @@ def test_maxwellian_energy_five_digits_mesh_A():
     assert abs(digits - GOLD["maxwellian_energy_digits"]["value"]) <= 0.5, digits
     density = 2 * np.pi * np.sum(w * f)
     assert abs(density - 1) < 1e-4
+
+
+def _maxwellian_residual(cells, R, p):
+    prob = inputs.Problem("p10", p, [(R, cells)], [inputs.Species("e", 1.0, -1.0, 0)], fmix=[[(1.0, 1.0, 0.0)]],
+                          noise=0.0)
+    o = Oracle(prob)
+    f = o.coefficients(with_noise=False)
+    J, _ = o.jacobian(f)
+    rp, col = o.pattern()
+    row = np.repeat(np.arange(o.ndof), np.diff(rp))
+    Jf = np.bincount(row, J * f[col], minlength=o.ndof)
+    Jaf = np.bincount(row, np.abs(J) * np.abs(f[col]), minlength=o.ndof)
+    return np.abs(Jf).max() / Jaf.max()
+
+
+def test_p10_maxwellian_discretisation_error_shrinks():
+    """P10 (discretisation, not parity): C(f_M, f_M) = 0 in the continuum, so ||J(f_M) f_M|| relative
+    to ||J| |f_M|| measures the discretisation error; it must fall under refinement (SURVEY S5:
+    7.7e-2 on Q2 2x4 -> 8.3e-4 on Q3 4x8)."""
+    R = inputs.R_E
+    coarse = _maxwellian_residual(inputs.uniform_mesh(R, 2), R, 2)
+    fine = _maxwellian_residual(inputs.uniform_mesh(R, 4), R, 3)
+    assert coarse > 1e-3
+    assert fine < coarse / 10, (coarse, fine)
