@@ -43,6 +43,8 @@ def parse():
     ap.add_argument("--batch", type=int, default=1024, help="C4 vertices in the whole job")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle vertices for cpu_baseline (0 = auto)")
+    ap.add_argument("--tensor-cache", action="store_true",
+                    help="NEXT-4 variant: cached mesh tensors + FP64 GEMM inner integral (not the headline path)")
     return ap.parse_args()
 
 
@@ -232,6 +234,9 @@ def main():
         desc = dict(desc, workload="C5: one e+D Q4 mesh (4352 cells, N=108800), target cells split over the GPUs, "
                                    "NCCL all-gather of G")
     h = L.Landau.from_problem(prob0, device=local, stream=stream, dist=dist_desc)
+    if args.tensor_cache:
+        h.set_tensor_cache(True)
+        desc = dict(desc, variant="NEXT-4 tensor cache: inner integral as FP64 GEMMs over cached tensors")
     nodes = h.all_nodes()
     nloc = len(items)
     N = h.npoints
@@ -313,7 +318,10 @@ def main():
     # ---- roofline of the dominant kernel (inner integral, FP64 pipe) --------------------------
     inner_ms, inner_n = tim["inner"]
     inner_avg_s = inner_ms / max(inner_n, 1) / 1e3
-    if st["inner_path"] == 1:
+    if st["inner_path"] == 2:   # GEMMs: 2 FLOP per multiply-add, 7 N^2 per batch item (three DGEMMs)
+        flop_per_pair = 14.0
+        flops_per_launch = 14.0 * st["nbatch"] * N * N
+    elif st["inner_path"] == 1:
         flop_per_pair = FLOP_PER_PAIR_SYMMETRIC
         flops_per_launch = flop_per_pair * st["nbatch"] * N * (N - 1) / 2
     else:
@@ -329,7 +337,8 @@ def main():
             "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None,
             "traffic": load_profile_traffic(args.workload),
             "peak_note": f"derived FP64 DFMA peak: {props.multi_processor_count} SMs x 64 lanes x 2 FLOP x {sm_max:.0f} MHz",
-            "inner_path": "symmetric (unordered pairs)" if st["inner_path"] == 1 else "directed (ordered pairs)",
+            "inner_path": ["directed (ordered pairs)", "symmetric (unordered pairs)",
+                           "tensor cache + FP64 DGEMM (cuBLAS)"][st["inner_path"]],
             "flop_per_pair": flop_per_pair, "flops_per_launch": flops_per_launch,
             "inner_ms_per_launch": inner_avg_s * 1e3,
             "inner_share_of_step": (inner_ms / args.steps) / ms_per_step if ms_per_step else None,
@@ -346,6 +355,36 @@ def main():
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(F_host.nbytes) * world,
                     "d2h_bytes_per_step": int(v_pin.numel() * 8) * world, "api": "landau_jacobian_host"},
             "gpu_launches": int(launches), "clocks": clocks}
+    # NEXT-4 variant on the same job (informational; the headline above is the pairwise path)
+    if args.workload == "C4" and not args.tensor_cache and nloc:
+        try:
+            h.set_tensor_cache(True)
+            step()
+            torch.cuda.synchronize()
+            h.set_timing(True)
+            vev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+            for k in range(args.steps):
+                flush.fill_(float(k))
+                vev[k][0].record(stream)
+                step()
+                vev[k][1].record(stream)
+            torch.cuda.synchronize()
+            vt = h.get_timing()
+            h.set_timing(False)
+            h.set_tensor_cache(False)
+            vms = torch.tensor([sum(a.elapsed_time(b) for a, b in vev)], dtype=torch.float64, device="cuda")
+            if world > 1:
+                dist.all_reduce(vms, op=dist.ReduceOp.MAX)
+            vstep = float(vms.item()) / args.steps
+            gemm_s = vt["inner"][0] / max(vt["inner"][1], 1) / 1e3
+            line["variants"] = {"tensor_cache_gemm": {
+                "value": total_builds / (vstep / 1e3), "unit": UNIT, "ms_per_step": vstep,
+                "inner_ms_per_launch": gemm_s * 1e3,
+                "inner_tflops": 14.0 * nloc * N * N / gemm_s / 1e12,
+                "note": "SURVEY NEXT-4: mesh tensors cached once (7 N^2 doubles), inner integral as three FP64 "
+                        "DGEMMs (cuBLAS, FP64 tensor cores); same sums up to order, parity-tested"}}
+        except Exception as e:   # the variant is optional: report why it did not run
+            line["variants"] = {"tensor_cache_gemm": {"unavailable": str(e)[:200]}}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         ns = args.cpu_sample or (8 if args.workload == "C4" else 1)
         line["cpu_baseline"] = cpu_baseline(args, desc, ns)

@@ -159,10 +159,22 @@ int landau_get_timing(landau_t h, double *ms, int64_t *launches);
 /* kernels launched by this handle since creation (all stages) */
 int landau_get_launch_count(landau_t h, int64_t *count);
 
+/* Tensor cache (SURVEY §8(f) NEXT-4, U-caching variant): the axisymmetric tensors depend only on the
+ * mesh, so for a handle whose builds share it (batched vertices, repeated Newton iterations) the
+ * library can evaluate the five N x N tensor matrices U^D_rr, U^D_rz, U^D_zz, U^K_rr, U^K_zr once
+ * (7 N^2 doubles, stacked for GEMM) and then form the inner integral of a batch as three FP64 GEMMs
+ * (cuBLAS DGEMM on the FP64 tensor cores, libcublas.so.12 loaded on demand):
+ *   [G_Drr; G_Drz; G_Dzz] = [U^D_rr; U^D_rz; U^D_zz] (3N x N) . W_D (N x batch)
+ *   G_Kr = [U^K_rr  U^D_rz] (N x 2N) . [W_Kr; W_Kz],   G_Kz = [U^K_zr  U^D_zz] . [W_Kr; W_Kz].
+ * The same sums as the pairwise kernels up to summation order.  EUNSUPPORTED for element-split
+ * handles or when 7 N^2 doubles exceed 16 GiB; enable = 0 frees the cache. */
+int landau_set_tensor_cache(landau_t h, int32_t enable);
+
 /* How the last build ran (for FLOP accounting and diagnostics). */
 typedef struct {
   int32_t inner_path;        /* 0: directed pair kernel (every ordered pair, split-j when small);
-                                1: symmetric pair kernel (every unordered pair once, both targets)  */
+                                1: symmetric pair kernel (every unordered pair once, both targets);
+                                2: tensor cache + FP64 GEMM (landau_set_tensor_cache)              */
   int64_t nbatch;            /* batch items of the last build                                      */
   int64_t targets;           /* target points per batch item (all N unless element-split)          */
   int64_t sources;           /* source points per batch item (N)                                   */

@@ -373,6 +373,37 @@ __global__ void reduce_sym_kernel(int64_t N, int64_t nslots, const int32_t *__re
   }
 }
 
+// ------------------------------------------------------------------------------------------------
+// Tensor cache fill (NEXT-4): every ordered pair (i, j) once, written column-major for the GEMMs:
+//   A1 (3N x N): rows c N + i, c = 0,1,2 -> U^D_rr, U^D_rz, U^D_zz
+//   A2 (N x 2N): [U^K_rr | U^D_rz],  A3 (N x 2N): [U^K_zr | U^D_zz]
+// Coincident points (the diagonal and any twins) get zeros (Amb-3).
+// ------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(128) tensor_fill_kernel(int64_t N, const double *__restrict__ pr,
+                                                          const double *__restrict__ pz, double *__restrict__ A1,
+                                                          double *__restrict__ A2, double *__restrict__ A3) {
+  __shared__ double s_coef[kNumPairCoef];
+  stage_pair_coef(s_coef);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, cf);
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t j = blockIdx.y;
+  if (i >= N) return;
+  const double r = pr[i], z = pz[i], rb = pr[j], zb = pz[j];
+  bool ok;
+  double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
+  pair_tensors<PairCoef, true>(r, z, r * r, rb, zb, rb * rb, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
+  if (!ok) Udrr = Udrz = Udzz = Ukrr = Ukzr = 0.0;
+  A1[i + j * 3 * N] = Udrr;
+  A1[N + i + j * 3 * N] = Udrz;
+  A1[2 * N + i + j * 3 * N] = Udzz;
+  A2[i + j * N] = Ukrr;
+  A2[i + (N + j) * N] = Udrz;
+  A3[i + j * N] = Ukzr;
+  A3[i + (N + j) * N] = Udzz;
+}
+
 // N2r: G[b][c][i] = sum_{s = 0..nsplit-1} part[b][s][c][i] in fixed order (deterministic).
 __global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__ part, double *__restrict__ G,
                               int64_t G_bstride, int nbatch) {
@@ -572,6 +603,35 @@ bool load_nccl() {
 }
 constexpr int kNcclFloat64 = 8;
 
+// cuBLAS, loaded on demand (only the tensor-cache path uses it: a plain library DGEMM)
+typedef void *cublasHandle_;
+struct CublasApi {
+  void *so = nullptr;
+  int (*Create)(cublasHandle_ *) = nullptr;
+  int (*Destroy)(cublasHandle_) = nullptr;
+  int (*SetStream)(cublasHandle_, cudaStream_t) = nullptr;
+  int (*Dgemm)(cublasHandle_, int, int, int, int, int, const double *, const double *, int, const double *, int,
+               const double *, double *, int) = nullptr;
+};
+CublasApi g_cublas;
+std::mutex g_cublas_mu;
+bool load_cublas() {
+  std::lock_guard<std::mutex> lk(g_cublas_mu);
+  if (g_cublas.so) return true;
+  void *so = nullptr;
+  for (const char *n : {"libcublas.so.12", "libcublas.so"})
+    if ((so = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
+  if (!so) return false;
+  g_cublas.Create = (int (*)(cublasHandle_ *))dlsym(so, "cublasCreate_v2");
+  g_cublas.Destroy = (int (*)(cublasHandle_))dlsym(so, "cublasDestroy_v2");
+  g_cublas.SetStream = (int (*)(cublasHandle_, cudaStream_t))dlsym(so, "cublasSetStream_v2");
+  g_cublas.Dgemm = (int (*)(cublasHandle_, int, int, int, int, int, const double *, const double *, int, const double *,
+                            int, const double *, double *, int))dlsym(so, "cublasDgemm_v2");
+  if (!g_cublas.Create || !g_cublas.Destroy || !g_cublas.SetStream || !g_cublas.Dgemm) return false;
+  g_cublas.so = so;
+  return true;
+}
+
 thread_local std::string g_create_error;
 
 }  // namespace
@@ -617,6 +677,10 @@ struct landau_s {
   int ntiles = 0;
   int64_t nsym_items = 0, nsym_slots = 0;
   bool coincident = false;   // two distinct quadrature points with identical (r, z) (never for one grid)
+  // tensor cache (NEXT-4)
+  bool tcache = false, tcache_valid = false;
+  double *d_U = nullptr;     // A1 (3N^2) | A2 (2N^2) | A3 (2N^2)
+  cublasHandle_ cublas = nullptr;
   // host staging for landau_jacobian_host: full-batch device buffers, two copy streams
   double *d_vals_tmp = nullptr;
   int64_t vals_tmp_cap = 0;
@@ -833,6 +897,34 @@ int launch_inner(landau_t h, int64_t nbatch) {
   const Plan &P = h->plan;
   const int64_t N = P.npts;
   const int64_t t0 = h->e0 * P.nqp, nt = (h->e1 - h->e0) * P.nqp;
+  if (h->tcache) {   // NEXT-4: cached tensors, three FP64 GEMMs
+    const int64_t n2 = N * N;
+    if (!h->tcache_valid) {
+      dim3 grid((unsigned)((N + 127) / 128), (unsigned)N);
+      tensor_fill_kernel<<<grid, 128, 0, h->stream>>>(N, h->d_r, h->d_z, h->d_U, h->d_U + 3 * n2, h->d_U + 5 * n2);
+      h->launches++;
+      KCHECK();
+      h->tcache_valid = true;
+    }
+    h->stats.nbatch = nbatch;
+    h->stats.targets = nt;
+    h->stats.sources = N;
+    h->stats.inner_path = 2;
+    h->stats.nsplit = 1;
+    h->stats.pair_evaluations = 0;
+    Timer t(h, LANDAU_T_INNER);
+    const double one = 1.0, zero = 0.0;
+    const int n = (int)N, nb = (int)nbatch;
+    double *G = h->d_G;   // [batch][5][N], Nc == N
+    int st = g_cublas.Dgemm(h->cublas, 0, 0, 3 * n, nb, n, &one, h->d_U, 3 * n, h->d_wT, 3 * n, &zero, G, 5 * n);
+    if (!st) st = g_cublas.Dgemm(h->cublas, 0, 0, n, nb, 2 * n, &one, h->d_U + 3 * n2, n, h->d_wT + N, 3 * n, &zero,
+                                 G + 3 * N, 5 * n);
+    if (!st) st = g_cublas.Dgemm(h->cublas, 0, 0, n, nb, 2 * n, &one, h->d_U + 5 * n2, n, h->d_wT + N, 3 * n, &zero,
+                                 G + 4 * N, 5 * n);
+    if (st) return fail(h, LANDAU_ECUDA, "cublasDgemm failed: " + std::to_string(st));
+    h->tlaunch[LANDAU_T_INNER] += 1;   // one inner stage (three cuBLAS kernels, not counted as ours)
+    return LANDAU_OK;
+  }
   InnerPlan ip;
   int rc = inner_plan(h, nbatch, ip);
   if (rc) return rc;
@@ -995,7 +1087,7 @@ int dispatch_build_direct(landau_t h, int64_t nbatch, double *out, int format) {
 // A whole build replays as one CUDA graph (launch-latency bound for small meshes) unless per-stage
 // timers are on, the legacy default stream is in use, or the build has a collective.
 int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
-  if (h->timing || !h->use_graphs || !h->stream || h->comm || !out)
+  if (h->timing || !h->use_graphs || !h->stream || h->comm || !out || h->tcache)
     return dispatch_build_direct(h, nbatch, out, format);
   for (auto &g : h->graphs)
     if (g.nbatch == nbatch && g.format == format && g.out == out && g.fin == h->fin) {
@@ -1272,6 +1364,8 @@ void landau_destroy(landau_t h) {
   cudaSetDevice(h->device);
   if (h->stream) cudaStreamSynchronize(h->stream);
   drop_graphs(h);
+  if (h->cublas && g_cublas.Destroy) g_cublas.Destroy(h->cublas);
+  cudaFree(h->d_U);
   if (h->s_h2d) cudaStreamDestroy(h->s_h2d);
   if (h->s_d2h) cudaStreamDestroy(h->s_d2h);
   for (auto e : h->ev_h2d) cudaEventDestroy(e);
@@ -1508,6 +1602,34 @@ int landau_get_timing(landau_t h, double *ms, int64_t *launches) {
     if (ms) ms[i] = acc[i];
     if (launches) launches[i] = h->tlaunch[i];
   }
+  return LANDAU_OK;
+}
+
+int landau_set_tensor_cache(landau_t h, int32_t enable) {
+  if (!h) return LANDAU_EINVAL;
+  if (h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!enable) {
+    drop_graphs(h);
+    CU(cudaStreamSynchronize(h->stream));
+    cudaFree(h->d_U);
+    h->d_U = nullptr;
+    h->tcache = h->tcache_valid = false;
+    return LANDAU_OK;
+  }
+  if (h->tcache) return LANDAU_OK;
+  const int64_t N = h->plan.npts;
+  if (h->world > 1 || h->Nc != N) return fail(h, LANDAU_EUNSUPPORTED, "tensor cache needs all targets on one GPU");
+  if (7 * N * N * (int64_t)sizeof(double) > (16LL << 30)) return fail(h, LANDAU_EUNSUPPORTED, "tensor cache > 16 GiB");
+  if (N > INT32_MAX / 5) return fail(h, LANDAU_EUNSUPPORTED, "mesh too large for the GEMM path");
+  if (!load_cublas()) return fail(h, LANDAU_EUNSUPPORTED, "cannot load libcublas.so.12");
+  if (!h->cublas) {
+    if (g_cublas.Create(&h->cublas)) return fail(h, LANDAU_ECUDA, "cublasCreate failed");
+    if (g_cublas.SetStream(h->cublas, h->stream)) return fail(h, LANDAU_ECUDA, "cublasSetStream failed");
+  }
+  CU(cudaMalloc(&h->d_U, sizeof(double) * 7 * N * N));
+  drop_graphs(h);
+  h->tcache = true;
+  h->tcache_valid = false;
   return LANDAU_OK;
 }
 

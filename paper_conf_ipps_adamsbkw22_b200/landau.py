@@ -81,6 +81,7 @@ def lib():
             "landau_get_timing": (C.c_int, [vp, Pd, P64]),
             "landau_get_launch_count": (C.c_int, [vp, P64]),
             "landau_get_stats": (C.c_int, [vp, C.POINTER(_Stats)]),
+            "landau_set_tensor_cache": (C.c_int, [vp, i32]),
             "landau_strerror": (C.c_char_p, [C.c_int]),
             "landau_last_error": (C.c_char_p, [vp]),
             "landau_version": (C.c_char_p, []),
@@ -271,6 +272,9 @@ class Landau:
         self._check(lib().landau_get_timing(self._h, _dptr(ms), n.ctypes.data_as(C.POINTER(C.c_int64))),
                     "landau_get_timing")
         return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(TIMERS)}
+
+    def set_tensor_cache(self, enable=True):
+        self._check(lib().landau_set_tensor_cache(self._h, int(bool(enable))), "landau_set_tensor_cache")
 
     def stats(self):
         st = _Stats()

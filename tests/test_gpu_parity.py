@@ -369,3 +369,34 @@ def test_full_parity_other_orders(order, mesh):
     assert np.all(np.abs(J - Jo) <= 1e-11 * Ja)
     d, m, e = _conservation(prob, h, J, fg)
     assert max(d, m, e) < 1e-13, (d, m, e)
+
+
+def test_tensor_cache_gemm_path_C4():
+    """NEXT-4 tensor cache: the batch's inner integral as FP64 GEMMs over cached tensor matrices
+    matches the oracle and the pairwise (symmetric) kernel."""
+    nb = 24
+    prob0 = inputs.config4_vertex(0)
+    h = L.Landau.from_problem(prob0, device=0)
+    nodes = h.all_nodes()
+    verts = [int(round(k * 1023 / (nb - 1))) for k in range(nb)]
+    probs = [inputs.config4_vertex(b) for b in verts]
+    F = torch.tensor(np.stack([inputs.coefficients(p, nodes) for p in probs]), device=DEV)
+    h.set_state_batched(F)
+    out = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
+    h.jacobian_batched(out)
+    ref = out.cpu().numpy()
+    h.set_tensor_cache(True)
+    h.jacobian_batched(out)
+    torch.cuda.synchronize()
+    assert h.stats()["inner_path"] == 2
+    Jc = out.cpu().numpy()
+    assert np.abs(Jc - ref).max() <= 1e-12 * np.abs(ref).max()
+    for k in (0, nb - 1):
+        o = Oracle(probs[k])
+        Jo, Ja = o.jacobian(o.coefficients())
+        assert np.all(np.abs(Jc[k] - Jo) <= 1e-11 * Ja)
+    h.jacobian_batched(out)      # cached tensors reused: bitwise repeatable
+    assert np.array_equal(out.cpu().numpy().view(np.uint64), Jc.view(np.uint64))
+    h.set_tensor_cache(False)
+    h.jacobian_batched(out)
+    assert h.stats()["inner_path"] == 1
