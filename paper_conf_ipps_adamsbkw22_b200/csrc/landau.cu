@@ -522,23 +522,36 @@ struct GatherDev {
   double fD[kMaxSpecies], fK[kMaxSpecies];   // a-3 species factors
 };
 
-template <int NB>
+template <int NB, int BPT>
 __global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ Cbuf, int64_t cbuf_bstride,
-                                double *__restrict__ out, int64_t out_bstride) {
-  const int b = blockIdx.y;
+                                double *__restrict__ out, int64_t out_bstride, int nbatch) {
+  // a thread gathers one slot for BPT batch items: the map (ptr, idx, w) is read once and the BPT
+  // element-matrix loads per contribution are independent (memory-level parallelism)
+  const int b0 = blockIdx.y * BPT;
   const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (s >= gm.nslots) return;
-  const double *C = Cbuf + (int64_t)b * cbuf_bstride;
+  const int nb = min(BPT, nbatch - b0);
+  const double *C = Cbuf + (int64_t)b0 * cbuf_bstride;
   const int64_t k0 = gm.ptr[s], k1 = gm.ptr[s + 1];
-  double sD = 0.0, sK = 0.0;
+  double sD[BPT], sK[BPT];
+#pragma unroll
+  for (int t = 0; t < BPT; t++) sD[t] = sK[t] = 0.0;
   for (int64_t k = k0; k < k1; k++) {
     const int64_t i = gm.idx[k];
     const double w = gm.w[k];
-    sD = fma(w, C[i], sD);
-    sK = fma(w, C[i + NB * NB], sK);
+#pragma unroll
+    for (int t = 0; t < BPT; t++)
+      if (t < nb) {
+        sD[t] = fma(w, __ldg(C + t * cbuf_bstride + i), sD[t]);
+        sK[t] = fma(w, __ldg(C + t * cbuf_bstride + i + NB * NB), sK[t]);
+      }
   }
-  double *o = out + (int64_t)b * out_bstride;
-  for (int q = 0; q < gm.nsp; q++) o[gm.out_off[q] + s] = fma(gm.fD[q], sD, gm.fK[q] * sK);
+#pragma unroll
+  for (int t = 0; t < BPT; t++)
+    if (t < nb) {
+      double *o = out + (int64_t)(b0 + t) * out_bstride;
+      for (int q = 0; q < gm.nsp; q++) o[gm.out_off[q] + s] = fma(gm.fD[q], sD[t], gm.fK[q] * sK[t]);
+    }
 }
 
 // mass gather (create time): out[s] = sum_k w_k M[idx_k]
@@ -1049,8 +1062,10 @@ int launch_assemble(landau_t h, int64_t nbatch, double *out, int format) {   // 
       gd.fK[q] = h->spc.fK[sp];
     }
     if (h->spc.grid_nsp[g] == 0 || m.nslots == 0) continue;
-    dim3 grid((unsigned)((m.nslots + 255) / 256), (unsigned)nbatch);
-    assemble_kernel<NB><<<grid, 256, 0, h->stream>>>(gd, h->d_C, P.ncell * 2 * NB * NB, out, out_bstride);
+    constexpr int BPT = 8;
+    dim3 grid((unsigned)((m.nslots + 127) / 128), (unsigned)((nbatch + BPT - 1) / BPT));
+    assemble_kernel<NB, BPT><<<grid, 128, 0, h->stream>>>(gd, h->d_C, P.ncell * 2 * NB * NB, out, out_bstride,
+                                                          (int)nbatch);
     h->launches++;
     h->tlaunch[LANDAU_T_ASSEMBLE]++;
     KCHECK();
