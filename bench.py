@@ -385,6 +385,37 @@ def main():
                         "DGEMMs (cuBLAS, FP64 tensor cores); same sums up to order, parity-tested"}}
         except Exception as e:   # the variant is optional: report why it did not run
             line["variants"] = {"tensor_cache_gemm": {"unavailable": str(e)[:200]}}
+    # configs[1] itself (one C2 grid, one build per step; launch-latency regime, CUDA-graph replay)
+    if args.workload == "C4" and rank == 0:
+        try:
+            p2 = inputs.config2()
+            h2 = L.Landau.from_problem(p2, device=local, stream=stream)
+            f2 = torch.tensor(inputs.coefficients(p2, h2.all_nodes()), device="cuda")
+            v2 = torch.empty(h2.nnz, dtype=torch.float64, device="cuda")
+            m2 = torch.empty(h2.nnz, dtype=torch.float64, device="cuda")
+            for _ in range(max(args.warmup, 3)):
+                h2.set_state(f2)
+                h2.jacobian(v2)
+                h2.mass(shift, m2)
+            torch.cuda.synchronize()
+            ev2 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+            for k in range(args.steps):
+                flush.fill_(float(k))
+                ev2[k][0].record(stream)
+                h2.set_state(f2)
+                h2.jacobian(v2)
+                h2.mass(shift, m2)
+                ev2[k][1].record(stream)
+            torch.cuda.synchronize()
+            ms2 = sum(a.elapsed_time(b) for a, b in ev2) / args.steps
+            line["c2_single_build"] = {"value": 1e3 / ms2, "unit": UNIT, "ms_per_step": ms2,
+                                       "pairs_per_s": 1e3 / ms2 * p2.npoints ** 2,
+                                       "inner_path": ["directed", "symmetric", "tensor cache"][h2.stats()["inner_path"]],
+                                       "note": "BASELINE configs[1]: one e+D Q3 AMR grid (N=1088) per step, "
+                                               "set_state + jacobian (CSR) + mass, CUDA-graph replay"}
+            h2.close()
+        except Exception as e:
+            line["c2_single_build"] = {"unavailable": str(e)[:200]}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         ns = args.cpu_sample or (8 if args.workload == "C4" else 1)
         line["cpu_baseline"] = cpu_baseline(args, desc, ns)

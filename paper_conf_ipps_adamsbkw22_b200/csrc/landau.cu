@@ -30,6 +30,9 @@ using namespace landau;
 #define LANDAU_SYM_UNROLL 2
 #endif
 constexpr int kSymUnroll = LANDAU_SYM_UNROLL;
+#ifndef LANDAU_SYM_HYBRID_COEF
+#define LANDAU_SYM_HYBRID_COEF 0
+#endif
 #ifndef LANDAU_SYM_SMEM_COEF
 #define LANDAU_SYM_SMEM_COEF 0
 #endif
@@ -321,6 +324,12 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t
   __syncthreads();
   const SmemCoef cf{reinterpret_cast<const double2 *>(s_coef), reinterpret_cast<const double2 *>(s_coef) + ELL_D_DEG + 1,
                     s_coef + 4 * (ELL_D_DEG + 1)};
+#elif LANDAU_SYM_HYBRID_COEF
+  __shared__ double s_coef[kNumPairCoef];
+  stage_pair_coef(s_coef);
+  __syncthreads();
+  HybridCoef cf;
+  load_hybrid_coef(s_coef, cf);
 #else
   __shared__ double s_coef[kNumPairCoef];
   stage_pair_coef(s_coef);

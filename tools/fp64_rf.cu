@@ -17,6 +17,9 @@ __global__ void k(double *out, double a, double b, long long *cyc) {
       if (V == 0) x[c] = fma(x[c], a, b);
       if (V == 1) x[c] = fma(x[c], y[c], z[c]);
       if (V == 2) x[c] = fma(x[c], y[c], b);
+      if (V == 3) x[c] = fma(y[0], x[c], z[c]);   // shared multiplier (operand reuse), distinct addend
+      if (V == 4) x[c] = x[c] * y[c];              // DMUL, two distinct registers
+      if (V == 5) x[c] = fma(x[c], y[c], x[c]);    // three operands, two distinct registers
     }
   }
   long long t1 = clock64();
@@ -33,10 +36,11 @@ template <int V> void run(double *o, long long *c, int sms) {
   long long h[1024]; cudaMemcpy(h, c, 8 * sms * bps, cudaMemcpyDeviceToHost);
   double mx = 0; for (int i = 0; i < sms * bps; i++) mx = h[i] > mx ? h[i] : mx;
   double lanes = (double)bps * threads * IT * CH / mx;
-  printf("\"v%d_dfma_lanes_per_sm_clk\": %.2f%s", V, lanes, V == 2 ? "" : ", ");
+  printf("\"v%d_lanes_per_sm_clk\": %.2f%s", V, lanes, V == 5 ? "" : ", ");
 }
 int main() {
   int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
   double *o; long long *c; cudaMalloc(&o, 8); cudaMalloc(&c, 8 * 1024);
-  printf("{"); run<0>(o, c, sms); run<1>(o, c, sms); run<2>(o, c, sms); printf("}\n");
+  printf("{"); run<0>(o, c, sms); run<1>(o, c, sms); run<2>(o, c, sms); run<3>(o, c, sms); run<4>(o, c, sms);
+  run<5>(o, c, sms); printf("}\n");
 }
