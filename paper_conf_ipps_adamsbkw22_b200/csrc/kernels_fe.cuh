@@ -1,0 +1,260 @@
+// kernels_fe.cuh -- finite-element kernels: point fields (a-1), element matrices (a-4), deterministic gather assembly (a-3 + a-5), mass (a-6)
+// (split out of landau.cu; included once, by landau.cu)
+#pragma once
+#include <cstdint>
+
+#include "kernels.cuh"
+
+namespace landau {
+
+
+// Per-handle data reaches the kernels as arguments (species table by value, basis tables through
+// global memory) -- no per-handle __constant__ state, so several handles can share a device and a
+// captured CUDA graph stays valid.
+
+// ------------------------------------------------------------------------------------------------
+// Reference tables in shared memory: thread-varying indices into __constant__ memory serialise, so
+// kernels that index the tables by thread copy them to shared memory once per block.
+// ------------------------------------------------------------------------------------------------
+template <int NB>
+__device__ __forceinline__ void load_tables(const double *__restrict__ tab, double (*s_phi)[NB], double (*s_dxi)[NB],
+                                            double (*s_deta)[NB]) {
+  for (int i = threadIdx.x; i < NB * NB; i += blockDim.x) {
+    s_phi[i / NB][i % NB] = tab[i];
+    s_dxi[i / NB][i % NB] = tab[NB * NB + i];
+    s_deta[i / NB][i % NB] = tab[2 * NB * NB + i];
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// N1: point fields.  A block handles EPB cells at a time (grid-stride over cells x batch); thread
+// (cell, a) first forms the combined element coefficients gD_a = sum_b e_b^2 f_b,a and
+// gK_a = sum_b e_b^2/m_b f_b,a through the extraction list (T_D, T_K are linear in f), then thread
+// (cell, q) interpolates: w T_D, w T_Kr, w T_Kz at its point.
+// ------------------------------------------------------------------------------------------------
+template <int NB, int EPB>
+__global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbatch, int64_t ndof_total,
+                                                         const double *__restrict__ f,
+                                                         const int32_t *__restrict__ ext_ptr,
+                                                         const int32_t *__restrict__ ext_dof,
+                                                         const double *__restrict__ ext_w,
+                                                         const int *__restrict__ cell_grid,
+                                                         const double *__restrict__ cell_h, const double *__restrict__ pw,
+                                                         const double *__restrict__ tab, const SpeciesConst sp_,
+                                                         double *__restrict__ wT, int64_t npts) {
+  // tables transposed ([k][q]): in phase 2 consecutive threads are consecutive q (conflict-free)
+  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
+  __shared__ double gD[EPB][NB], gK[EPB][NB];
+  for (int i = threadIdx.x; i < NB * NB; i += blockDim.x) {
+    s_phi[i % NB][i / NB] = tab[i];
+    s_dxi[i % NB][i / NB] = tab[NB * NB + i];
+    s_deta[i % NB][i / NB] = tab[2 * NB * NB + i];
+  }
+  const SpeciesConst &c_sp = sp_;
+  const int el = threadIdx.x / NB, a = threadIdx.x % NB;
+  const int64_t nchunks = (ncell + EPB - 1) / EPB;
+  for (int64_t it = blockIdx.x; it < nchunks * nbatch; it += gridDim.x) {
+    const int b = (int)(it / nchunks);
+    const int64_t e = (it % nchunks) * EPB + el;
+    const double *fb = f + (int64_t)b * ndof_total;
+    __syncthreads();
+    if (e < ncell) {
+      const int g = cell_grid[e];
+      const int32_t k0 = ext_ptr[e * NB + a], k1 = ext_ptr[e * NB + a + 1];
+      double sD = 0.0, sK = 0.0;
+      for (int s = 0; s < c_sp.grid_nsp[g]; s++) {
+        const int sp = c_sp.grid_sp[g][s];
+        const double *fs = fb + c_sp.soff[sp];
+        double v = 0.0;
+        for (int32_t k = k0; k < k1; k++) v = fma(ext_w[k], __ldg(fs + ext_dof[k]), v);
+        sD = fma(c_sp.e2[sp], v, sD);
+        sK = fma(c_sp.e2m[sp], v, sK);
+      }
+      gD[el][a] = sD;
+      gK[el][a] = sK;
+    }
+    __syncthreads();
+    if (e < ncell) {
+      const int q = a;   // NQP == NB for (p+1)^2 Gauss points
+      const int64_t pt = e * NB + q;
+      double td = 0.0, tr = 0.0, tz = 0.0;
+#pragma unroll
+      for (int k = 0; k < NB; k++) {
+        td = fma(s_phi[k][q], gD[el][k], td);
+        tr = fma(s_dxi[k][q], gK[el][k], tr);
+        tz = fma(s_deta[k][q], gK[el][k], tz);
+      }
+      const double w = pw[pt], ws = w * (2.0 / cell_h[e]);
+      double *o = wT + (int64_t)b * 3 * npts;
+      o[pt] = w * td;
+      o[npts + pt] = ws * tr;
+      o[2 * npts + pt] = ws * tz;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// N3: element matrices (species independent).  C^D[k,l] = (2/h)^2 sum_q gk . (w_q G_D(q)) . gl,
+// C^K[k,l] = (2/h) sum_q (gk . w_q G_K(q)) phi_l(q), gk the reference gradients.  A thread owns an
+// S x S block (S = p + 1) of both matrices of one cell, so each table value it loads from shared
+// memory feeds S outputs (the v0 one-entry-per-thread form was shared-memory-bandwidth bound);
+// a block handles EPB cells.  Per q:  u_l = A_rr gl_r + A_rz gl_z,  v_l = A_rz gl_r + A_zz gl_z,
+// t_k = gk_r K_r + gk_z K_z;  C^D[k,l] += gk_r u_l + gk_z v_l,  C^K[k,l] += t_k phi_l.
+// G is read in the chunked layout G[((i / Nc) * nbatch + b) * 5 + c][i % Nc] (Nc = N unless split).
+// ------------------------------------------------------------------------------------------------
+template <int NB, int S, int EPB>
+__global__ void __launch_bounds__(NB * EPB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
+                                                             int nbatch, int b0, int nb, const double *__restrict__ pw,
+                                                             const double *__restrict__ cell_h,
+                                                             const double *__restrict__ tab, double *__restrict__ Cbuf) {
+  static_assert(S * S == NB, "S = p + 1");
+  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];   // [q][k]
+  __shared__ double sA[EPB][5][NB];                                  // w_q G(q) per cell
+  load_tables<NB>(tab, s_phi, s_dxi, s_deta);
+  const int el = threadIdx.x / NB, t = threadIdx.x % NB;
+  const int k0 = (t / S) * S, l0 = (t % S) * S;
+  const int64_t nchunks = (ncell + EPB - 1) / EPB;
+  for (int64_t it = blockIdx.x; it < nchunks * nb; it += gridDim.x) {   // batch items b0 .. b0 + nb - 1
+    const int bc = (int)(it / nchunks), b = b0 + bc;
+    const int64_t e = (it % nchunks) * EPB + el;
+    __syncthreads();
+    if (e < ncell) {
+      const int64_t i = e * NB + t;
+      const int64_t chunk = i / Nc, off = i % Nc;
+      const double *Gb = G + ((chunk * nbatch + b) * 5) * Nc + off;
+      const double w = pw[i];
+#pragma unroll
+      for (int c = 0; c < 5; c++) sA[el][c][t] = w * Gb[c * Nc];
+    }
+    __syncthreads();
+    if (e >= ncell) continue;
+    double cd[S][S], ck[S][S];
+#pragma unroll
+    for (int a = 0; a < S; a++)
+#pragma unroll
+      for (int c = 0; c < S; c++) cd[a][c] = ck[a][c] = 0.0;
+#pragma unroll 2
+    for (int q = 0; q < NB; q++) {
+      const double Arr = sA[el][0][q], Arz = sA[el][1][q], Azz = sA[el][2][q], Kr = sA[el][3][q], Kz = sA[el][4][q];
+      double u[S], v[S], pl[S], gr[S], gz[S], tk[S];
+#pragma unroll
+      for (int c = 0; c < S; c++) {
+        const double glr = s_dxi[q][l0 + c], glz = s_deta[q][l0 + c];
+        u[c] = fma(Arr, glr, Arz * glz);
+        v[c] = fma(Arz, glr, Azz * glz);
+        pl[c] = s_phi[q][l0 + c];
+        gr[c] = s_dxi[q][k0 + c];
+        gz[c] = s_deta[q][k0 + c];
+        tk[c] = fma(gr[c], Kr, gz[c] * Kz);
+      }
+#pragma unroll
+      for (int a = 0; a < S; a++)
+#pragma unroll
+        for (int c = 0; c < S; c++) {
+          cd[a][c] = fma(gr[a], u[c], fma(gz[a], v[c], cd[a][c]));
+          ck[a][c] = fma(tk[a], pl[c], ck[a][c]);
+        }
+    }
+    const double sc = 2.0 / cell_h[e];
+    double *o = Cbuf + ((int64_t)bc * ncell + e) * 2 * NB * NB;
+#pragma unroll
+    for (int a = 0; a < S; a++)
+#pragma unroll
+      for (int c = 0; c < S; c++) {
+        o[(k0 + a) * NB + l0 + c] = cd[a][c] * sc * sc;
+        o[NB * NB + (k0 + a) * NB + l0 + c] = ck[a][c] * sc;
+      }
+  }
+}
+
+// Mass element matrices (create time): M[k,l] = sum_q w_q phi_k phi_l, stored in the [cell][2][NB^2]
+// layout (second half zero) so the same gather maps apply.
+template <int NB>
+__global__ void __launch_bounds__(NB * NB) mass_element_kernel(int64_t ncell, const double *__restrict__ pw,
+                                                                 const double *__restrict__ tab, double *__restrict__ Mbuf) {
+  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
+  load_tables<NB>(tab, s_phi, s_dxi, s_deta);
+  __syncthreads();
+  const int64_t e = blockIdx.x;
+  const int tid = threadIdx.x, k = tid / NB, l = tid % NB;
+  double m = 0.0;
+  for (int q = 0; q < NB; q++) m = fma(pw[e * NB + q] * s_phi[q][k], s_phi[q][l], m);
+  Mbuf[e * 2 * NB * NB + tid] = m;
+  Mbuf[e * 2 * NB * NB + NB * NB + tid] = 0.0;
+}
+
+// ------------------------------------------------------------------------------------------------
+// N4: deterministic gather.  For grid slot s (CSR nonzero or COO entry):
+//   sD = sum_k w_k C^D[idx_k], sK = sum_k w_k C^K[idx_k]   (fixed (cell, a, b) order)
+//   out[b][out_off(a) + s] = fD_a sD + fK_a sK   for every species a on the grid   (a-3 + a-5)
+// ------------------------------------------------------------------------------------------------
+struct GatherDev {
+  const int64_t *ptr;
+  const int32_t *idx;
+  const double *w;
+  int64_t nslots;
+  int nsp;                        // species on this grid
+  int64_t out_off[kMaxSpecies];   // output offset per species on this grid
+  double fD[kMaxSpecies], fK[kMaxSpecies];   // a-3 species factors
+};
+
+template <int NB, int BPT>
+__global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ Cbuf, int64_t cbuf_bstride,
+                                double *__restrict__ out, int64_t out_bstride, int nbatch) {
+  // a thread gathers one slot for BPT batch items: the map (ptr, idx, w) is read once and the BPT
+  // element-matrix loads per contribution are independent (memory-level parallelism)
+  const int b0 = blockIdx.y * BPT;
+  const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= gm.nslots) return;
+  const int nb = min(BPT, nbatch - b0);
+  const double *C = Cbuf + (int64_t)b0 * cbuf_bstride;
+  const int64_t k0 = gm.ptr[s], k1 = gm.ptr[s + 1];
+  double sD[BPT], sK[BPT];
+#pragma unroll
+  for (int t = 0; t < BPT; t++) sD[t] = sK[t] = 0.0;
+  for (int64_t k = k0; k < k1; k++) {
+    const int64_t i = gm.idx[k];
+    const double w = gm.w[k];
+#pragma unroll
+    for (int t = 0; t < BPT; t++)
+      if (t < nb) {
+        sD[t] = fma(w, __ldg(C + t * cbuf_bstride + i), sD[t]);
+        sK[t] = fma(w, __ldg(C + t * cbuf_bstride + i + NB * NB), sK[t]);
+      }
+  }
+#pragma unroll
+  for (int t = 0; t < BPT; t++)
+    if (t < nb) {
+      double *o = out + (int64_t)(b0 + t) * out_bstride;
+      for (int q = 0; q < gm.nsp; q++) o[gm.out_off[q] + s] = fma(gm.fD[q], sD[t], gm.fK[q] * sK[t]);
+    }
+}
+
+// mass gather (create time): out[s] = sum_k w_k M[idx_k]
+__global__ void mass_gather_kernel(const int64_t *__restrict__ ptr, const int32_t *__restrict__ idx,
+                                   const double *__restrict__ w, int64_t nslots, const double *__restrict__ M,
+                                   double *__restrict__ out) {
+  const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= nslots) return;
+  double v = 0.0;
+  for (int64_t k = ptr[s]; k < ptr[s + 1]; k++) v = fma(w[k], M[idx[k]], v);
+  out[s] = v;
+}
+
+// N5: out[o0 + i] = shift * M[i]
+__global__ void scale_copy_kernel(const double *__restrict__ M, double shift, int64_t n, double *__restrict__ out) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = shift * M[i];
+}
+
+// copy chunked G layout -> [b][5][N]
+__global__ void unchunk_kernel(const double *__restrict__ G, int64_t N, int64_t Nc, int nbatch, double *__restrict__ out) {
+  const int64_t total = (int64_t)nbatch * 5 * N;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = k / (5 * N), c = (k / N) % 5, i = k % N;
+    out[k] = G[(((i / Nc) * nbatch + b) * 5 + c) * Nc + (i % Nc)];
+  }
+}
+
+
+}  // namespace landau

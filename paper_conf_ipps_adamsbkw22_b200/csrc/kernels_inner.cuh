@@ -1,0 +1,325 @@
+// kernels_inner.cuh -- the inner integral (a-2): directed and symmetric pair kernels, split-j and slot reductions, tensor-cache fill
+// (split out of landau.cu; included once, by landau.cu)
+#pragma once
+#include <cstdint>
+
+#include "kernels.cuh"
+
+namespace landau {
+
+// build-time tuning knobs of the symmetric inner kernel (defaults = measured best on B200)
+#ifndef LANDAU_SYM_UNROLL
+#define LANDAU_SYM_UNROLL 2
+#endif
+constexpr int kSymUnroll = LANDAU_SYM_UNROLL;
+#ifndef LANDAU_SYM_HYBRID_COEF
+#define LANDAU_SYM_HYBRID_COEF 0
+#endif
+#ifndef LANDAU_SYM_SMEM_COEF
+#define LANDAU_SYM_SMEM_COEF 0
+#endif
+#ifndef LANDAU_SYM_WARPS
+#define LANDAU_SYM_WARPS 4
+#endif
+#ifndef LANDAU_SYM_MINB
+#define LANDAU_SYM_MINB 2
+#endif
+
+// ------------------------------------------------------------------------------------------------
+// N2: inner integral.  Work is warp-granular: a warp owns 32*TPT consecutive targets of one batch
+// item and one split of the source range (split-j), so the target tiling never pads across batch
+// items.  Sources are staged per warp through shared memory, 32 at a time (one per lane), and every
+// lane then reads the same source (broadcast LDS.128).  Coefficients of the elliptic fits live in
+// registers (see kernels.cuh).  out = [batch][nsplit][5][nt] partials (or G when nsplit == 1).
+// ------------------------------------------------------------------------------------------------
+constexpr int kInnerTB = 128;
+constexpr int kInnerWarps = kInnerTB / 32;
+
+template <int TPT, int MINB>
+__global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_t t0, int64_t nt, int64_t split_len,
+                                                             int nsplit, int64_t wtiles, int64_t nitems,
+                                                             const double *__restrict__ pr, const double *__restrict__ pz,
+                                                             const double *__restrict__ wT, double *__restrict__ out,
+                                                             int64_t out_bstride) {
+  __shared__ double2 s_rz[kInnerWarps][32], s_w[kInnerWarps][32], s_wz[kInnerWarps][32];   // (wkz, rb^2)
+  __shared__ double s_coef[kNumPairCoef];
+  stage_pair_coef(s_coef);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, cf);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t item = (int64_t)blockIdx.x * kInnerWarps + wid;
+  if (item >= nitems) return;   // whole warp: no block-level barrier follows
+  const int64_t b = item / (nsplit * wtiles);
+  const int64_t rem = item % (nsplit * wtiles);
+  const int split = (int)(rem / wtiles);
+  const int64_t wt = rem % wtiles;
+  const double *wb = wT + b * 3 * N;
+  int64_t ti[TPT];
+  double tr[TPT], tz[TPT], tr2[TPT];
+  Acc5 acc[TPT];
+#pragma unroll
+  for (int t = 0; t < TPT; t++) {
+    ti[t] = wt * 32 * TPT + t * 32 + lane;
+    const int64_t gi = t0 + (ti[t] < nt ? ti[t] : nt - 1);
+    tr[t] = pr[gi];
+    tz[t] = pz[gi];
+    tr2[t] = tr[t] * tr[t];
+    acc[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+  }
+  const int64_t j0 = (int64_t)split * split_len;
+  const int64_t j1 = min(N, j0 + split_len);
+  for (int64_t jt = j0; jt < j1; jt += 32) {
+    const int64_t j = jt + lane;
+    __syncwarp();
+    if (j < j1) {
+      const double rj = pr[j];
+      s_rz[wid][lane] = make_double2(rj, pz[j]);
+      s_w[wid][lane] = make_double2(wb[j], wb[N + j]);
+      s_wz[wid][lane] = make_double2(wb[2 * N + j], rj * rj);
+    }
+    __syncwarp();
+    const int n = (int)min((int64_t)32, j1 - jt);
+#pragma unroll 2
+    for (int k = 0; k < n; k++) {
+      const double2 rz = s_rz[wid][k], w = s_w[wid][k], wz = s_wz[wid][k];
+#pragma unroll
+      for (int t = 0; t < TPT; t++) landau_pair(tr[t], tz[t], tr2[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, cf, acc[t]);
+    }
+  }
+  double *o = out + b * out_bstride + (int64_t)split * 5 * nt;
+#pragma unroll
+  for (int t = 0; t < TPT; t++) {
+    if (ti[t] < nt) {
+      o[ti[t]] = acc[t].drr;
+      o[nt + ti[t]] = acc[t].drz;
+      o[2 * nt + ti[t]] = acc[t].dzz;
+      o[3 * nt + ti[t]] = acc[t].kr;
+      o[4 * nt + ti[t]] = acc[t].kz;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// N2 (symmetric): each unordered pair of points is evaluated once.  The points
+// are cut into T tiles of 32.  A warp item is one j-tile b (its 32 points and their reverse-sum
+// accumulators in warp-private shared memory) against one or two i-tiles a1 < a2 < b, or the
+// diagonal item (b, b).  Lane L holds target i = a*32 + L (forward sums in registers); at step k it
+// pairs with j = b*32 + ((L + k) mod 32), so the 32 lanes touch 32 distinct j each step
+// (conflict-free, no atomics).  Diagonal items run k = 1..16 (lanes < 16 only at k = 16) so every
+// unordered pair is visited exactly once.  Two i-tiles per item give two independent pair chains
+// per lane (the FP64 pipe needs the ILP) and share one accumulator update per step.
+// Every item writes 32-point partial "slots"; reduce_sym_kernel sums, for each tile, its slots in a
+// fixed host-built order -> bitwise reproducible.  part = [batch][nslots][5][32].
+// ------------------------------------------------------------------------------------------------
+constexpr int kSymWarps = LANDAU_SYM_WARPS;
+#ifndef LANDAU_SYM_NI
+#define LANDAU_SYM_NI 2
+#endif
+constexpr int kSymNI = LANDAU_SYM_NI;   // max i-tiles per item (independent pair chains per lane)
+static_assert(kSymNI >= 1 && kSymNI <= 3, "sym items carry 1..3 i-tiles");
+
+struct SymItem {   // host-built, see landau_create
+  int a[3];        // i-tiles (n of them, all < b); n == 0: the diagonal item (b, b)
+  int b, n;
+  int slot;        // first of the item's consecutive partial slots: one per i-tile (or the diagonal's
+                   // forward sums), then the j-tile's reverse sums
+};
+
+__device__ __forceinline__ void sym_load_i(const double *pr, const double *pz, const double *wb, int64_t N, int64_t i,
+                                           double zpad, double &r, double &z, double &wd, double &wkr, double &wkz) {
+  const bool v = i < N;   // padding: far away, zero weights -- contributes nothing, never read back
+  r = v ? pr[i] : 1.0;
+  z = v ? pz[i] : zpad;
+  wd = v ? wb[i] : 0.0;
+  wkr = v ? wb[N + i] : 0.0;
+  wkz = v ? wb[2 * N + i] : 0.0;
+}
+
+__device__ __forceinline__ void sym_store(double *o, int lane, const Acc5 &a) {
+  o[lane] = a.drr;
+  o[32 + lane] = a.drz;
+  o[64 + lane] = a.dzz;
+  o[96 + lane] = a.kr;
+  o[128 + lane] = a.kz;
+}
+
+// NI i-tiles against the warp's j-tile (NI independent pair chains per lane and step); DIAG: the
+// tile against itself, k = 1..16 (lanes < 16 only at k = 16) -- every unordered pair exactly once.
+// The reverse sums travel with their j: at step k lane L holds the accumulator of j = (L + k) mod 32
+// and hands it to lane L - 1 by a shuffle, so consecutive steps carry no memory fence and their
+// (long, independent) pair evaluations overlap; the j data itself is read-only shared memory.
+template <int NI, bool DIAG, bool MASK, class CF>
+__device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, const double *pz, const double *wb,
+                                        int64_t N, int lane, const double2 *s_rz, const double2 *s_w,
+                                        const double2 *s_wz, const CF &cf, double *o) {
+  double r[NI], z[NI], r2[NI], wd[NI], wkr[NI], wkz[NI];
+  Acc5 ai[NI];
+#pragma unroll
+  for (int t = 0; t < NI; t++) {
+    sym_load_i(pr, pz, wb, N, (int64_t)(DIAG ? it.b : it.a[t]) * 32 + lane, 1.0e6 + 64.0 * t + lane, r[t], z[t], wd[t],
+               wkr[t], wkz[t]);
+    r2[t] = r[t] * r[t];
+    ai[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+  }
+  constexpr int k0 = DIAG ? 1 : 0, k1 = DIAG ? 17 : 32;
+  const int src = (lane + 1) & 31;
+  Acc5 aj{0.0, 0.0, 0.0, 0.0, 0.0};
+  // diagonal items: steps 1..15 are unmasked, step 16 (lanes >= 16 would double-count) is peeled
+  constexpr int kmain = DIAG ? 16 : 32;
+#pragma unroll kSymUnroll
+  for (int k = k0; k < kmain; k++) {
+    const int jj = (lane + k) & 31;
+    const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
+#pragma unroll
+    for (int t = 0; t < NI; t++)
+      landau_pair_sym<CF, MASK>(r[t], z[t], r2[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, true, cf,
+                                ai[t], aj);
+    aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
+    aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
+    aj.dzz = __shfl_sync(0xffffffffu, aj.dzz, src);
+    aj.kr = __shfl_sync(0xffffffffu, aj.kr, src);
+    aj.kz = __shfl_sync(0xffffffffu, aj.kz, src);
+  }
+  if constexpr (DIAG) {
+    const int jj = (lane + 16) & 31;
+    const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
+    landau_pair_sym<CF, true>(r[0], z[0], r2[0], wd[0], wkr[0], wkz[0], rz.x, rz.y, wz.y, w.x, w.y, wz.x, lane < 16, cf,
+                              ai[0], aj);
+    aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
+    aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
+    aj.dzz = __shfl_sync(0xffffffffu, aj.dzz, src);
+    aj.kr = __shfl_sync(0xffffffffu, aj.kr, src);
+    aj.kz = __shfl_sync(0xffffffffu, aj.kz, src);
+  }
+#pragma unroll
+  for (int t = 0; t < NI; t++) sym_store(o + t * 160, lane, ai[t]);
+  // after the last hand-over lane L holds the reverse sums of j = (L + k1) mod 32
+  const int jf = (lane + k1) & 31;
+  double *oj = o + (DIAG ? 1 : NI) * 160;
+  oj[jf] = aj.drr;
+  oj[32 + jf] = aj.drz;
+  oj[64 + jf] = aj.dzz;
+  oj[96 + jf] = aj.kr;
+  oj[128 + jf] = aj.kz;
+}
+
+template <int MINB, bool MASK>
+__global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t N, int64_t nitems_b, int64_t nslots,
+                                                                         int64_t nitems,
+                                                                         const SymItem *__restrict__ items,
+                                                                         const double *__restrict__ pr,
+                                                                         const double *__restrict__ pz,
+                                                                         const double *__restrict__ wT,
+                                                                         double *__restrict__ part) {
+  __shared__ double2 s_rz[kSymWarps][32], s_w[kSymWarps][32], s_wz[kSymWarps][32];   // (wkz, rb^2)
+#if LANDAU_SYM_SMEM_COEF
+  __shared__ __align__(16) double s_coef[kNumSmemCoef];
+  stage_smem_coef(s_coef);
+  __syncthreads();
+  const SmemCoef cf{reinterpret_cast<const double2 *>(s_coef), reinterpret_cast<const double2 *>(s_coef) + ELL_D_DEG + 1,
+                    s_coef + 4 * (ELL_D_DEG + 1)};
+#elif LANDAU_SYM_HYBRID_COEF
+  __shared__ double s_coef[kNumPairCoef];
+  stage_pair_coef(s_coef);
+  __syncthreads();
+  HybridCoef cf;
+  load_hybrid_coef(s_coef, cf);
+#else
+  __shared__ double s_coef[kNumPairCoef];
+  stage_pair_coef(s_coef);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, cf);
+#endif
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  // persistent warps: grid-stride over the (batch item, work item) list
+  for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
+  const int64_t bb = item / nitems_b;
+  const SymItem it = items[item % nitems_b];
+  const double *wb = wT + bb * 3 * N;
+  __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
+  {
+    double r, z, wd, wkr, wkz;
+    sym_load_i(pr, pz, wb, N, (int64_t)it.b * 32 + lane, 2.0e6 + lane, r, z, wd, wkr, wkz);
+    s_rz[wid][lane] = make_double2(r, z);
+    s_w[wid][lane] = make_double2(wd, wkr);
+    s_wz[wid][lane] = make_double2(wkz, r * r);
+  }
+  __syncwarp();
+  double *o = part + (bb * nslots + it.slot) * 160;
+  switch (it.n) {
+    case 0: sym_run<1, true, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
+    case 1: sym_run<1, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
+    case 2:
+      if constexpr (kSymNI >= 2) sym_run<2, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
+      break;
+    default:
+      if constexpr (kSymNI >= 3)
+        sym_run<kSymNI, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
+      break;
+  }
+  }
+}
+
+// G[b][c][i] = sum of the partial slots of tile t = i / 32 in the fixed order of tile_slots.
+__global__ void reduce_sym_kernel(int64_t N, int64_t nslots, const int32_t *__restrict__ tile_ptr,
+                                  const int32_t *__restrict__ tile_slots, const double *__restrict__ part,
+                                  double *__restrict__ G, int64_t G_bstride, int nbatch) {
+  const int64_t total = (int64_t)nbatch * 5 * N;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = k / (5 * N), c = (k / N) % 5, i = k % N;
+    const int t = (int)(i / 32), lane = (int)(i % 32);
+    const double *pb = part + b * nslots * 160 + c * 32 + lane;
+    double s = 0.0;
+    for (int q = tile_ptr[t]; q < tile_ptr[t + 1]; q++) s += pb[(int64_t)tile_slots[q] * 160];
+    G[b * G_bstride + c * N + i] = s;
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// Tensor cache fill (NEXT-4): every ordered pair (i, j) once, written column-major for the GEMMs:
+//   A1 (3N x N): rows c N + i, c = 0,1,2 -> U^D_rr, U^D_rz, U^D_zz
+//   A2 (N x 2N): [U^K_rr | U^D_rz],  A3 (N x 2N): [U^K_zr | U^D_zz]
+// Coincident points (the diagonal and any twins) get zeros (Amb-3).
+// ------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(128) tensor_fill_kernel(int64_t N, const double *__restrict__ pr,
+                                                          const double *__restrict__ pz, double *__restrict__ A1,
+                                                          double *__restrict__ A2, double *__restrict__ A3) {
+  __shared__ double s_coef[kNumPairCoef];
+  stage_pair_coef(s_coef);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, cf);
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t j = blockIdx.y;
+  if (i >= N) return;
+  const double r = pr[i], z = pz[i], rb = pr[j], zb = pz[j];
+  bool ok;
+  double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
+  pair_tensors<PairCoef, true>(r, z, r * r, rb, zb, rb * rb, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
+  if (!ok) Udrr = Udrz = Udzz = Ukrr = Ukzr = 0.0;
+  A1[i + j * 3 * N] = Udrr;
+  A1[N + i + j * 3 * N] = Udrz;
+  A1[2 * N + i + j * 3 * N] = Udzz;
+  A2[i + j * N] = Ukrr;
+  A2[i + (N + j) * N] = Udrz;
+  A3[i + j * N] = Ukzr;
+  A3[i + (N + j) * N] = Udzz;
+}
+
+// N2r: G[b][c][i] = sum_{s = 0..nsplit-1} part[b][s][c][i] in fixed order (deterministic).
+__global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__ part, double *__restrict__ G,
+                              int64_t G_bstride, int nbatch) {
+  const int64_t total = (int64_t)nbatch * 5 * nt;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = k / (5 * nt), ci = k % (5 * nt);
+    const double *p = part + b * (int64_t)nsplit * 5 * nt + ci;
+    double s = 0.0;
+    for (int q = 0; q < nsplit; q++) s += p[(int64_t)q * 5 * nt];
+    G[b * G_bstride + ci] = s;
+  }
+}
+
+
+}  // namespace landau

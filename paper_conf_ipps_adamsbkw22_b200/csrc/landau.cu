@@ -1,11 +1,10 @@
-// landau.cu -- liblandau.so: the C ABI of include/landau.h and the sm_100a kernels of one build.
-//
-//   N1 field_kernel     a-1  f, grad f at the quadrature points -> w T_D, w T_K      (HBM/latency)
-//   N2 inner_kernel     a-2  pairwise U^D, U^K sums (split-j partials)               (FP64 pipe)
-//   N2r reduce_kernel   a-2  fixed-order sum of the split-j partials                 (HBM)
-//   N3 element_kernel   a-4  species-independent element matrices C^D_e, C^K_e       (FP64/L1)
-//   N4 assemble_kernel  a-3+a-5  species factors + deterministic gather into CSR/COO (HBM)
-//   N5 mass             a-6  element mass at create (cached), shift-scaled copy       (HBM)
+// landau.cu -- liblandau.so: the handle, the launch sequence of one build and the C ABI of
+// include/landau.h.  The sm_100a kernels live in
+//   kernels.cuh        FP64 pair body (cancellation-free U^D, U^K), coefficients, rcp/rsqrt/log
+//   kernels_inner.cuh  a-2: inner_sym_kernel (unordered pairs) / inner_kernel (ordered, split-j),
+//                      reduce_sym_kernel / reduce_kernel, tensor_fill_kernel (tensor cache)
+//   kernels_fe.cuh     a-1 field_kernel, a-4 element_kernel, a-3 + a-5 assemble_kernel, a-6 mass kernels
+//   dynload.h          NCCL (element split) and cuBLAS (tensor cache), loaded on demand
 // Citations: see include/landau.h and DESIGN.md.
 #include <cuda_runtime.h>
 #include <dlfcn.h>
@@ -25,638 +24,10 @@
 
 using namespace landau;
 
-// build-time tuning knobs of the symmetric inner kernel (defaults = measured best on B200)
-#ifndef LANDAU_SYM_UNROLL
-#define LANDAU_SYM_UNROLL 2
-#endif
-constexpr int kSymUnroll = LANDAU_SYM_UNROLL;
-#ifndef LANDAU_SYM_HYBRID_COEF
-#define LANDAU_SYM_HYBRID_COEF 0
-#endif
-#ifndef LANDAU_SYM_SMEM_COEF
-#define LANDAU_SYM_SMEM_COEF 0
-#endif
-#ifndef LANDAU_SYM_WARPS
-#define LANDAU_SYM_WARPS 4
-#endif
-#ifndef LANDAU_SYM_MINB
-#define LANDAU_SYM_MINB 2
-#endif
+#include "dynload.h"
+#include "kernels_fe.cuh"
+#include "kernels_inner.cuh"
 
-namespace {
-
-// Per-handle data reaches the kernels as arguments (species table by value, basis tables through
-// global memory) -- no per-handle __constant__ state, so several handles can share a device and a
-// captured CUDA graph stays valid.
-
-// ------------------------------------------------------------------------------------------------
-// Reference tables in shared memory: thread-varying indices into __constant__ memory serialise, so
-// kernels that index the tables by thread copy them to shared memory once per block.
-// ------------------------------------------------------------------------------------------------
-template <int NB>
-__device__ __forceinline__ void load_tables(const double *__restrict__ tab, double (*s_phi)[NB], double (*s_dxi)[NB],
-                                            double (*s_deta)[NB]) {
-  for (int i = threadIdx.x; i < NB * NB; i += blockDim.x) {
-    s_phi[i / NB][i % NB] = tab[i];
-    s_dxi[i / NB][i % NB] = tab[NB * NB + i];
-    s_deta[i / NB][i % NB] = tab[2 * NB * NB + i];
-  }
-}
-
-// ------------------------------------------------------------------------------------------------
-// N1: point fields.  A block handles EPB cells at a time (grid-stride over cells x batch); thread
-// (cell, a) first forms the combined element coefficients gD_a = sum_b e_b^2 f_b,a and
-// gK_a = sum_b e_b^2/m_b f_b,a through the extraction list (T_D, T_K are linear in f), then thread
-// (cell, q) interpolates: w T_D, w T_Kr, w T_Kz at its point.
-// ------------------------------------------------------------------------------------------------
-template <int NB, int EPB>
-__global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbatch, int64_t ndof_total,
-                                                         const double *__restrict__ f,
-                                                         const int32_t *__restrict__ ext_ptr,
-                                                         const int32_t *__restrict__ ext_dof,
-                                                         const double *__restrict__ ext_w,
-                                                         const int *__restrict__ cell_grid,
-                                                         const double *__restrict__ cell_h, const double *__restrict__ pw,
-                                                         const double *__restrict__ tab, const SpeciesConst sp_,
-                                                         double *__restrict__ wT, int64_t npts) {
-  // tables transposed ([k][q]): in phase 2 consecutive threads are consecutive q (conflict-free)
-  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
-  __shared__ double gD[EPB][NB], gK[EPB][NB];
-  for (int i = threadIdx.x; i < NB * NB; i += blockDim.x) {
-    s_phi[i % NB][i / NB] = tab[i];
-    s_dxi[i % NB][i / NB] = tab[NB * NB + i];
-    s_deta[i % NB][i / NB] = tab[2 * NB * NB + i];
-  }
-  const SpeciesConst &c_sp = sp_;
-  const int el = threadIdx.x / NB, a = threadIdx.x % NB;
-  const int64_t nchunks = (ncell + EPB - 1) / EPB;
-  for (int64_t it = blockIdx.x; it < nchunks * nbatch; it += gridDim.x) {
-    const int b = (int)(it / nchunks);
-    const int64_t e = (it % nchunks) * EPB + el;
-    const double *fb = f + (int64_t)b * ndof_total;
-    __syncthreads();
-    if (e < ncell) {
-      const int g = cell_grid[e];
-      const int32_t k0 = ext_ptr[e * NB + a], k1 = ext_ptr[e * NB + a + 1];
-      double sD = 0.0, sK = 0.0;
-      for (int s = 0; s < c_sp.grid_nsp[g]; s++) {
-        const int sp = c_sp.grid_sp[g][s];
-        const double *fs = fb + c_sp.soff[sp];
-        double v = 0.0;
-        for (int32_t k = k0; k < k1; k++) v = fma(ext_w[k], __ldg(fs + ext_dof[k]), v);
-        sD = fma(c_sp.e2[sp], v, sD);
-        sK = fma(c_sp.e2m[sp], v, sK);
-      }
-      gD[el][a] = sD;
-      gK[el][a] = sK;
-    }
-    __syncthreads();
-    if (e < ncell) {
-      const int q = a;   // NQP == NB for (p+1)^2 Gauss points
-      const int64_t pt = e * NB + q;
-      double td = 0.0, tr = 0.0, tz = 0.0;
-#pragma unroll
-      for (int k = 0; k < NB; k++) {
-        td = fma(s_phi[k][q], gD[el][k], td);
-        tr = fma(s_dxi[k][q], gK[el][k], tr);
-        tz = fma(s_deta[k][q], gK[el][k], tz);
-      }
-      const double w = pw[pt], ws = w * (2.0 / cell_h[e]);
-      double *o = wT + (int64_t)b * 3 * npts;
-      o[pt] = w * td;
-      o[npts + pt] = ws * tr;
-      o[2 * npts + pt] = ws * tz;
-    }
-  }
-}
-
-// ------------------------------------------------------------------------------------------------
-// N2: inner integral.  Work is warp-granular: a warp owns 32*TPT consecutive targets of one batch
-// item and one split of the source range (split-j), so the target tiling never pads across batch
-// items.  Sources are staged per warp through shared memory, 32 at a time (one per lane), and every
-// lane then reads the same source (broadcast LDS.128).  Coefficients of the elliptic fits live in
-// registers (see kernels.cuh).  out = [batch][nsplit][5][nt] partials (or G when nsplit == 1).
-// ------------------------------------------------------------------------------------------------
-constexpr int kInnerTB = 128;
-constexpr int kInnerWarps = kInnerTB / 32;
-
-template <int TPT, int MINB>
-__global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_t t0, int64_t nt, int64_t split_len,
-                                                             int nsplit, int64_t wtiles, int64_t nitems,
-                                                             const double *__restrict__ pr, const double *__restrict__ pz,
-                                                             const double *__restrict__ wT, double *__restrict__ out,
-                                                             int64_t out_bstride) {
-  __shared__ double2 s_rz[kInnerWarps][32], s_w[kInnerWarps][32], s_wz[kInnerWarps][32];   // (wkz, rb^2)
-  __shared__ double s_coef[kNumPairCoef];
-  stage_pair_coef(s_coef);
-  __syncthreads();
-  PairCoef cf;
-  load_pair_coef(s_coef, cf);
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const int64_t item = (int64_t)blockIdx.x * kInnerWarps + wid;
-  if (item >= nitems) return;   // whole warp: no block-level barrier follows
-  const int64_t b = item / (nsplit * wtiles);
-  const int64_t rem = item % (nsplit * wtiles);
-  const int split = (int)(rem / wtiles);
-  const int64_t wt = rem % wtiles;
-  const double *wb = wT + b * 3 * N;
-  int64_t ti[TPT];
-  double tr[TPT], tz[TPT], tr2[TPT];
-  Acc5 acc[TPT];
-#pragma unroll
-  for (int t = 0; t < TPT; t++) {
-    ti[t] = wt * 32 * TPT + t * 32 + lane;
-    const int64_t gi = t0 + (ti[t] < nt ? ti[t] : nt - 1);
-    tr[t] = pr[gi];
-    tz[t] = pz[gi];
-    tr2[t] = tr[t] * tr[t];
-    acc[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
-  }
-  const int64_t j0 = (int64_t)split * split_len;
-  const int64_t j1 = min(N, j0 + split_len);
-  for (int64_t jt = j0; jt < j1; jt += 32) {
-    const int64_t j = jt + lane;
-    __syncwarp();
-    if (j < j1) {
-      const double rj = pr[j];
-      s_rz[wid][lane] = make_double2(rj, pz[j]);
-      s_w[wid][lane] = make_double2(wb[j], wb[N + j]);
-      s_wz[wid][lane] = make_double2(wb[2 * N + j], rj * rj);
-    }
-    __syncwarp();
-    const int n = (int)min((int64_t)32, j1 - jt);
-#pragma unroll 2
-    for (int k = 0; k < n; k++) {
-      const double2 rz = s_rz[wid][k], w = s_w[wid][k], wz = s_wz[wid][k];
-#pragma unroll
-      for (int t = 0; t < TPT; t++) landau_pair(tr[t], tz[t], tr2[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, cf, acc[t]);
-    }
-  }
-  double *o = out + b * out_bstride + (int64_t)split * 5 * nt;
-#pragma unroll
-  for (int t = 0; t < TPT; t++) {
-    if (ti[t] < nt) {
-      o[ti[t]] = acc[t].drr;
-      o[nt + ti[t]] = acc[t].drz;
-      o[2 * nt + ti[t]] = acc[t].dzz;
-      o[3 * nt + ti[t]] = acc[t].kr;
-      o[4 * nt + ti[t]] = acc[t].kz;
-    }
-  }
-}
-
-// ------------------------------------------------------------------------------------------------
-// N2 (symmetric): each unordered pair of points is evaluated once.  The points
-// are cut into T tiles of 32.  A warp item is one j-tile b (its 32 points and their reverse-sum
-// accumulators in warp-private shared memory) against one or two i-tiles a1 < a2 < b, or the
-// diagonal item (b, b).  Lane L holds target i = a*32 + L (forward sums in registers); at step k it
-// pairs with j = b*32 + ((L + k) mod 32), so the 32 lanes touch 32 distinct j each step
-// (conflict-free, no atomics).  Diagonal items run k = 1..16 (lanes < 16 only at k = 16) so every
-// unordered pair is visited exactly once.  Two i-tiles per item give two independent pair chains
-// per lane (the FP64 pipe needs the ILP) and share one accumulator update per step.
-// Every item writes 32-point partial "slots"; reduce_sym_kernel sums, for each tile, its slots in a
-// fixed host-built order -> bitwise reproducible.  part = [batch][nslots][5][32].
-// ------------------------------------------------------------------------------------------------
-constexpr int kSymWarps = LANDAU_SYM_WARPS;
-#ifndef LANDAU_SYM_NI
-#define LANDAU_SYM_NI 2
-#endif
-constexpr int kSymNI = LANDAU_SYM_NI;   // max i-tiles per item (independent pair chains per lane)
-static_assert(kSymNI >= 1 && kSymNI <= 3, "sym items carry 1..3 i-tiles");
-
-struct SymItem {   // host-built, see landau_create
-  int a[3];        // i-tiles (n of them, all < b); n == 0: the diagonal item (b, b)
-  int b, n;
-  int slot;        // first of the item's consecutive partial slots: one per i-tile (or the diagonal's
-                   // forward sums), then the j-tile's reverse sums
-};
-
-__device__ __forceinline__ void sym_load_i(const double *pr, const double *pz, const double *wb, int64_t N, int64_t i,
-                                           double zpad, double &r, double &z, double &wd, double &wkr, double &wkz) {
-  const bool v = i < N;   // padding: far away, zero weights -- contributes nothing, never read back
-  r = v ? pr[i] : 1.0;
-  z = v ? pz[i] : zpad;
-  wd = v ? wb[i] : 0.0;
-  wkr = v ? wb[N + i] : 0.0;
-  wkz = v ? wb[2 * N + i] : 0.0;
-}
-
-__device__ __forceinline__ void sym_store(double *o, int lane, const Acc5 &a) {
-  o[lane] = a.drr;
-  o[32 + lane] = a.drz;
-  o[64 + lane] = a.dzz;
-  o[96 + lane] = a.kr;
-  o[128 + lane] = a.kz;
-}
-
-// NI i-tiles against the warp's j-tile (NI independent pair chains per lane and step); DIAG: the
-// tile against itself, k = 1..16 (lanes < 16 only at k = 16) -- every unordered pair exactly once.
-// The reverse sums travel with their j: at step k lane L holds the accumulator of j = (L + k) mod 32
-// and hands it to lane L - 1 by a shuffle, so consecutive steps carry no memory fence and their
-// (long, independent) pair evaluations overlap; the j data itself is read-only shared memory.
-template <int NI, bool DIAG, bool MASK, class CF>
-__device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, const double *pz, const double *wb,
-                                        int64_t N, int lane, const double2 *s_rz, const double2 *s_w,
-                                        const double2 *s_wz, const CF &cf, double *o) {
-  double r[NI], z[NI], r2[NI], wd[NI], wkr[NI], wkz[NI];
-  Acc5 ai[NI];
-#pragma unroll
-  for (int t = 0; t < NI; t++) {
-    sym_load_i(pr, pz, wb, N, (int64_t)(DIAG ? it.b : it.a[t]) * 32 + lane, 1.0e6 + 64.0 * t + lane, r[t], z[t], wd[t],
-               wkr[t], wkz[t]);
-    r2[t] = r[t] * r[t];
-    ai[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
-  }
-  constexpr int k0 = DIAG ? 1 : 0, k1 = DIAG ? 17 : 32;
-  const int src = (lane + 1) & 31;
-  Acc5 aj{0.0, 0.0, 0.0, 0.0, 0.0};
-  // diagonal items: steps 1..15 are unmasked, step 16 (lanes >= 16 would double-count) is peeled
-  constexpr int kmain = DIAG ? 16 : 32;
-#pragma unroll kSymUnroll
-  for (int k = k0; k < kmain; k++) {
-    const int jj = (lane + k) & 31;
-    const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
-#pragma unroll
-    for (int t = 0; t < NI; t++)
-      landau_pair_sym<CF, MASK>(r[t], z[t], r2[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, true, cf,
-                                ai[t], aj);
-    aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
-    aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
-    aj.dzz = __shfl_sync(0xffffffffu, aj.dzz, src);
-    aj.kr = __shfl_sync(0xffffffffu, aj.kr, src);
-    aj.kz = __shfl_sync(0xffffffffu, aj.kz, src);
-  }
-  if constexpr (DIAG) {
-    const int jj = (lane + 16) & 31;
-    const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
-    landau_pair_sym<CF, true>(r[0], z[0], r2[0], wd[0], wkr[0], wkz[0], rz.x, rz.y, wz.y, w.x, w.y, wz.x, lane < 16, cf,
-                              ai[0], aj);
-    aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
-    aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
-    aj.dzz = __shfl_sync(0xffffffffu, aj.dzz, src);
-    aj.kr = __shfl_sync(0xffffffffu, aj.kr, src);
-    aj.kz = __shfl_sync(0xffffffffu, aj.kz, src);
-  }
-#pragma unroll
-  for (int t = 0; t < NI; t++) sym_store(o + t * 160, lane, ai[t]);
-  // after the last hand-over lane L holds the reverse sums of j = (L + k1) mod 32
-  const int jf = (lane + k1) & 31;
-  double *oj = o + (DIAG ? 1 : NI) * 160;
-  oj[jf] = aj.drr;
-  oj[32 + jf] = aj.drz;
-  oj[64 + jf] = aj.dzz;
-  oj[96 + jf] = aj.kr;
-  oj[128 + jf] = aj.kz;
-}
-
-template <int MINB, bool MASK>
-__global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t N, int64_t nitems_b, int64_t nslots,
-                                                                         int64_t nitems,
-                                                                         const SymItem *__restrict__ items,
-                                                                         const double *__restrict__ pr,
-                                                                         const double *__restrict__ pz,
-                                                                         const double *__restrict__ wT,
-                                                                         double *__restrict__ part) {
-  __shared__ double2 s_rz[kSymWarps][32], s_w[kSymWarps][32], s_wz[kSymWarps][32];   // (wkz, rb^2)
-#if LANDAU_SYM_SMEM_COEF
-  __shared__ __align__(16) double s_coef[kNumSmemCoef];
-  stage_smem_coef(s_coef);
-  __syncthreads();
-  const SmemCoef cf{reinterpret_cast<const double2 *>(s_coef), reinterpret_cast<const double2 *>(s_coef) + ELL_D_DEG + 1,
-                    s_coef + 4 * (ELL_D_DEG + 1)};
-#elif LANDAU_SYM_HYBRID_COEF
-  __shared__ double s_coef[kNumPairCoef];
-  stage_pair_coef(s_coef);
-  __syncthreads();
-  HybridCoef cf;
-  load_hybrid_coef(s_coef, cf);
-#else
-  __shared__ double s_coef[kNumPairCoef];
-  stage_pair_coef(s_coef);
-  __syncthreads();
-  PairCoef cf;
-  load_pair_coef(s_coef, cf);
-#endif
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  // persistent warps: grid-stride over the (batch item, work item) list
-  for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
-  const int64_t bb = item / nitems_b;
-  const SymItem it = items[item % nitems_b];
-  const double *wb = wT + bb * 3 * N;
-  __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
-  {
-    double r, z, wd, wkr, wkz;
-    sym_load_i(pr, pz, wb, N, (int64_t)it.b * 32 + lane, 2.0e6 + lane, r, z, wd, wkr, wkz);
-    s_rz[wid][lane] = make_double2(r, z);
-    s_w[wid][lane] = make_double2(wd, wkr);
-    s_wz[wid][lane] = make_double2(wkz, r * r);
-  }
-  __syncwarp();
-  double *o = part + (bb * nslots + it.slot) * 160;
-  switch (it.n) {
-    case 0: sym_run<1, true, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
-    case 1: sym_run<1, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o); break;
-    case 2:
-      if constexpr (kSymNI >= 2) sym_run<2, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
-      break;
-    default:
-      if constexpr (kSymNI >= 3)
-        sym_run<kSymNI, false, MASK>(it, pr, pz, wb, N, lane, s_rz[wid], s_w[wid], s_wz[wid], cf, o);
-      break;
-  }
-  }
-}
-
-// G[b][c][i] = sum of the partial slots of tile t = i / 32 in the fixed order of tile_slots.
-__global__ void reduce_sym_kernel(int64_t N, int64_t nslots, const int32_t *__restrict__ tile_ptr,
-                                  const int32_t *__restrict__ tile_slots, const double *__restrict__ part,
-                                  double *__restrict__ G, int64_t G_bstride, int nbatch) {
-  const int64_t total = (int64_t)nbatch * 5 * N;
-  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t b = k / (5 * N), c = (k / N) % 5, i = k % N;
-    const int t = (int)(i / 32), lane = (int)(i % 32);
-    const double *pb = part + b * nslots * 160 + c * 32 + lane;
-    double s = 0.0;
-    for (int q = tile_ptr[t]; q < tile_ptr[t + 1]; q++) s += pb[(int64_t)tile_slots[q] * 160];
-    G[b * G_bstride + c * N + i] = s;
-  }
-}
-
-// ------------------------------------------------------------------------------------------------
-// Tensor cache fill (NEXT-4): every ordered pair (i, j) once, written column-major for the GEMMs:
-//   A1 (3N x N): rows c N + i, c = 0,1,2 -> U^D_rr, U^D_rz, U^D_zz
-//   A2 (N x 2N): [U^K_rr | U^D_rz],  A3 (N x 2N): [U^K_zr | U^D_zz]
-// Coincident points (the diagonal and any twins) get zeros (Amb-3).
-// ------------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(128) tensor_fill_kernel(int64_t N, const double *__restrict__ pr,
-                                                          const double *__restrict__ pz, double *__restrict__ A1,
-                                                          double *__restrict__ A2, double *__restrict__ A3) {
-  __shared__ double s_coef[kNumPairCoef];
-  stage_pair_coef(s_coef);
-  __syncthreads();
-  PairCoef cf;
-  load_pair_coef(s_coef, cf);
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const int64_t j = blockIdx.y;
-  if (i >= N) return;
-  const double r = pr[i], z = pz[i], rb = pr[j], zb = pz[j];
-  bool ok;
-  double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
-  pair_tensors<PairCoef, true>(r, z, r * r, rb, zb, rb * rb, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
-  if (!ok) Udrr = Udrz = Udzz = Ukrr = Ukzr = 0.0;
-  A1[i + j * 3 * N] = Udrr;
-  A1[N + i + j * 3 * N] = Udrz;
-  A1[2 * N + i + j * 3 * N] = Udzz;
-  A2[i + j * N] = Ukrr;
-  A2[i + (N + j) * N] = Udrz;
-  A3[i + j * N] = Ukzr;
-  A3[i + (N + j) * N] = Udzz;
-}
-
-// N2r: G[b][c][i] = sum_{s = 0..nsplit-1} part[b][s][c][i] in fixed order (deterministic).
-__global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__ part, double *__restrict__ G,
-                              int64_t G_bstride, int nbatch) {
-  const int64_t total = (int64_t)nbatch * 5 * nt;
-  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t b = k / (5 * nt), ci = k % (5 * nt);
-    const double *p = part + b * (int64_t)nsplit * 5 * nt + ci;
-    double s = 0.0;
-    for (int q = 0; q < nsplit; q++) s += p[(int64_t)q * 5 * nt];
-    G[b * G_bstride + ci] = s;
-  }
-}
-
-// ------------------------------------------------------------------------------------------------
-// N3: element matrices (species independent).  C^D[k,l] = (2/h)^2 sum_q gk . (w_q G_D(q)) . gl,
-// C^K[k,l] = (2/h) sum_q (gk . w_q G_K(q)) phi_l(q), gk the reference gradients.  A thread owns an
-// S x S block (S = p + 1) of both matrices of one cell, so each table value it loads from shared
-// memory feeds S outputs (the v0 one-entry-per-thread form was shared-memory-bandwidth bound);
-// a block handles EPB cells.  Per q:  u_l = A_rr gl_r + A_rz gl_z,  v_l = A_rz gl_r + A_zz gl_z,
-// t_k = gk_r K_r + gk_z K_z;  C^D[k,l] += gk_r u_l + gk_z v_l,  C^K[k,l] += t_k phi_l.
-// G is read in the chunked layout G[((i / Nc) * nbatch + b) * 5 + c][i % Nc] (Nc = N unless split).
-// ------------------------------------------------------------------------------------------------
-template <int NB, int S, int EPB>
-__global__ void __launch_bounds__(NB * EPB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
-                                                             int nbatch, int b0, int nb, const double *__restrict__ pw,
-                                                             const double *__restrict__ cell_h,
-                                                             const double *__restrict__ tab, double *__restrict__ Cbuf) {
-  static_assert(S * S == NB, "S = p + 1");
-  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];   // [q][k]
-  __shared__ double sA[EPB][5][NB];                                  // w_q G(q) per cell
-  load_tables<NB>(tab, s_phi, s_dxi, s_deta);
-  const int el = threadIdx.x / NB, t = threadIdx.x % NB;
-  const int k0 = (t / S) * S, l0 = (t % S) * S;
-  const int64_t nchunks = (ncell + EPB - 1) / EPB;
-  for (int64_t it = blockIdx.x; it < nchunks * nb; it += gridDim.x) {   // batch items b0 .. b0 + nb - 1
-    const int bc = (int)(it / nchunks), b = b0 + bc;
-    const int64_t e = (it % nchunks) * EPB + el;
-    __syncthreads();
-    if (e < ncell) {
-      const int64_t i = e * NB + t;
-      const int64_t chunk = i / Nc, off = i % Nc;
-      const double *Gb = G + ((chunk * nbatch + b) * 5) * Nc + off;
-      const double w = pw[i];
-#pragma unroll
-      for (int c = 0; c < 5; c++) sA[el][c][t] = w * Gb[c * Nc];
-    }
-    __syncthreads();
-    if (e >= ncell) continue;
-    double cd[S][S], ck[S][S];
-#pragma unroll
-    for (int a = 0; a < S; a++)
-#pragma unroll
-      for (int c = 0; c < S; c++) cd[a][c] = ck[a][c] = 0.0;
-#pragma unroll 2
-    for (int q = 0; q < NB; q++) {
-      const double Arr = sA[el][0][q], Arz = sA[el][1][q], Azz = sA[el][2][q], Kr = sA[el][3][q], Kz = sA[el][4][q];
-      double u[S], v[S], pl[S], gr[S], gz[S], tk[S];
-#pragma unroll
-      for (int c = 0; c < S; c++) {
-        const double glr = s_dxi[q][l0 + c], glz = s_deta[q][l0 + c];
-        u[c] = fma(Arr, glr, Arz * glz);
-        v[c] = fma(Arz, glr, Azz * glz);
-        pl[c] = s_phi[q][l0 + c];
-        gr[c] = s_dxi[q][k0 + c];
-        gz[c] = s_deta[q][k0 + c];
-        tk[c] = fma(gr[c], Kr, gz[c] * Kz);
-      }
-#pragma unroll
-      for (int a = 0; a < S; a++)
-#pragma unroll
-        for (int c = 0; c < S; c++) {
-          cd[a][c] = fma(gr[a], u[c], fma(gz[a], v[c], cd[a][c]));
-          ck[a][c] = fma(tk[a], pl[c], ck[a][c]);
-        }
-    }
-    const double sc = 2.0 / cell_h[e];
-    double *o = Cbuf + ((int64_t)bc * ncell + e) * 2 * NB * NB;
-#pragma unroll
-    for (int a = 0; a < S; a++)
-#pragma unroll
-      for (int c = 0; c < S; c++) {
-        o[(k0 + a) * NB + l0 + c] = cd[a][c] * sc * sc;
-        o[NB * NB + (k0 + a) * NB + l0 + c] = ck[a][c] * sc;
-      }
-  }
-}
-
-// Mass element matrices (create time): M[k,l] = sum_q w_q phi_k phi_l, stored in the [cell][2][NB^2]
-// layout (second half zero) so the same gather maps apply.
-template <int NB>
-__global__ void __launch_bounds__(NB * NB) mass_element_kernel(int64_t ncell, const double *__restrict__ pw,
-                                                                 const double *__restrict__ tab, double *__restrict__ Mbuf) {
-  __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
-  load_tables<NB>(tab, s_phi, s_dxi, s_deta);
-  __syncthreads();
-  const int64_t e = blockIdx.x;
-  const int tid = threadIdx.x, k = tid / NB, l = tid % NB;
-  double m = 0.0;
-  for (int q = 0; q < NB; q++) m = fma(pw[e * NB + q] * s_phi[q][k], s_phi[q][l], m);
-  Mbuf[e * 2 * NB * NB + tid] = m;
-  Mbuf[e * 2 * NB * NB + NB * NB + tid] = 0.0;
-}
-
-// ------------------------------------------------------------------------------------------------
-// N4: deterministic gather.  For grid slot s (CSR nonzero or COO entry):
-//   sD = sum_k w_k C^D[idx_k], sK = sum_k w_k C^K[idx_k]   (fixed (cell, a, b) order)
-//   out[b][out_off(a) + s] = fD_a sD + fK_a sK   for every species a on the grid   (a-3 + a-5)
-// ------------------------------------------------------------------------------------------------
-struct GatherDev {
-  const int64_t *ptr;
-  const int32_t *idx;
-  const double *w;
-  int64_t nslots;
-  int nsp;                        // species on this grid
-  int64_t out_off[kMaxSpecies];   // output offset per species on this grid
-  double fD[kMaxSpecies], fK[kMaxSpecies];   // a-3 species factors
-};
-
-template <int NB, int BPT>
-__global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ Cbuf, int64_t cbuf_bstride,
-                                double *__restrict__ out, int64_t out_bstride, int nbatch) {
-  // a thread gathers one slot for BPT batch items: the map (ptr, idx, w) is read once and the BPT
-  // element-matrix loads per contribution are independent (memory-level parallelism)
-  const int b0 = blockIdx.y * BPT;
-  const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (s >= gm.nslots) return;
-  const int nb = min(BPT, nbatch - b0);
-  const double *C = Cbuf + (int64_t)b0 * cbuf_bstride;
-  const int64_t k0 = gm.ptr[s], k1 = gm.ptr[s + 1];
-  double sD[BPT], sK[BPT];
-#pragma unroll
-  for (int t = 0; t < BPT; t++) sD[t] = sK[t] = 0.0;
-  for (int64_t k = k0; k < k1; k++) {
-    const int64_t i = gm.idx[k];
-    const double w = gm.w[k];
-#pragma unroll
-    for (int t = 0; t < BPT; t++)
-      if (t < nb) {
-        sD[t] = fma(w, __ldg(C + t * cbuf_bstride + i), sD[t]);
-        sK[t] = fma(w, __ldg(C + t * cbuf_bstride + i + NB * NB), sK[t]);
-      }
-  }
-#pragma unroll
-  for (int t = 0; t < BPT; t++)
-    if (t < nb) {
-      double *o = out + (int64_t)(b0 + t) * out_bstride;
-      for (int q = 0; q < gm.nsp; q++) o[gm.out_off[q] + s] = fma(gm.fD[q], sD[t], gm.fK[q] * sK[t]);
-    }
-}
-
-// mass gather (create time): out[s] = sum_k w_k M[idx_k]
-__global__ void mass_gather_kernel(const int64_t *__restrict__ ptr, const int32_t *__restrict__ idx,
-                                   const double *__restrict__ w, int64_t nslots, const double *__restrict__ M,
-                                   double *__restrict__ out) {
-  const int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (s >= nslots) return;
-  double v = 0.0;
-  for (int64_t k = ptr[s]; k < ptr[s + 1]; k++) v = fma(w[k], M[idx[k]], v);
-  out[s] = v;
-}
-
-// N5: out[o0 + i] = shift * M[i]
-__global__ void scale_copy_kernel(const double *__restrict__ M, double shift, int64_t n, double *__restrict__ out) {
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    out[i] = shift * M[i];
-}
-
-// copy chunked G layout -> [b][5][N]
-__global__ void unchunk_kernel(const double *__restrict__ G, int64_t N, int64_t Nc, int nbatch, double *__restrict__ out) {
-  const int64_t total = (int64_t)nbatch * 5 * N;
-  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t b = k / (5 * N), c = (k / N) % 5, i = k % N;
-    out[k] = G[(((i / Nc) * nbatch + b) * 5 + c) * Nc + (i % Nc)];
-  }
-}
-
-// ------------------------------------------------------------------------------------------------
-// NCCL, loaded on demand (only LANDAU_DIST_ELEMENTS needs it)
-// ------------------------------------------------------------------------------------------------
-typedef struct {
-  char internal[128];
-} ncclUniqueId_;
-typedef void *ncclComm_;
-struct NcclApi {
-  void *so = nullptr;
-  int (*GetUniqueId)(ncclUniqueId_ *) = nullptr;
-  int (*CommInitRank)(ncclComm_ *, int, ncclUniqueId_, int) = nullptr;
-  int (*AllGather)(const void *, void *, size_t, int, ncclComm_, cudaStream_t) = nullptr;
-  int (*CommDestroy)(ncclComm_) = nullptr;
-  const char *(*GetErrorString)(int) = nullptr;
-};
-NcclApi g_nccl;
-std::mutex g_nccl_mu;
-bool load_nccl() {
-  std::lock_guard<std::mutex> lk(g_nccl_mu);
-  if (g_nccl.so) return true;
-  const char *names[] = {"libnccl.so.2", "libnccl.so"};
-  void *so = nullptr;
-  for (const char *n : names)
-    if ((so = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
-  if (!so) return false;
-  g_nccl.GetUniqueId = (int (*)(ncclUniqueId_ *))dlsym(so, "ncclGetUniqueId");
-  g_nccl.CommInitRank = (int (*)(ncclComm_ *, int, ncclUniqueId_, int))dlsym(so, "ncclCommInitRank");
-  g_nccl.AllGather = (int (*)(const void *, void *, size_t, int, ncclComm_, cudaStream_t))dlsym(so, "ncclAllGather");
-  g_nccl.CommDestroy = (int (*)(ncclComm_))dlsym(so, "ncclCommDestroy");
-  g_nccl.GetErrorString = (const char *(*)(int))dlsym(so, "ncclGetErrorString");
-  if (!g_nccl.GetUniqueId || !g_nccl.CommInitRank || !g_nccl.AllGather || !g_nccl.CommDestroy) return false;
-  g_nccl.so = so;
-  return true;
-}
-constexpr int kNcclFloat64 = 8;
-
-// cuBLAS, loaded on demand (only the tensor-cache path uses it: a plain library DGEMM)
-typedef void *cublasHandle_;
-struct CublasApi {
-  void *so = nullptr;
-  int (*Create)(cublasHandle_ *) = nullptr;
-  int (*Destroy)(cublasHandle_) = nullptr;
-  int (*SetStream)(cublasHandle_, cudaStream_t) = nullptr;
-  int (*Dgemm)(cublasHandle_, int, int, int, int, int, const double *, const double *, int, const double *, int,
-               const double *, double *, int) = nullptr;
-};
-CublasApi g_cublas;
-std::mutex g_cublas_mu;
-bool load_cublas() {
-  std::lock_guard<std::mutex> lk(g_cublas_mu);
-  if (g_cublas.so) return true;
-  void *so = nullptr;
-  for (const char *n : {"libcublas.so.12", "libcublas.so"})
-    if ((so = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
-  if (!so) return false;
-  g_cublas.Create = (int (*)(cublasHandle_ *))dlsym(so, "cublasCreate_v2");
-  g_cublas.Destroy = (int (*)(cublasHandle_))dlsym(so, "cublasDestroy_v2");
-  g_cublas.SetStream = (int (*)(cublasHandle_, cudaStream_t))dlsym(so, "cublasSetStream_v2");
-  g_cublas.Dgemm = (int (*)(cublasHandle_, int, int, int, int, int, const double *, const double *, int, const double *,
-                            int, const double *, double *, int))dlsym(so, "cublasDgemm_v2");
-  if (!g_cublas.Create || !g_cublas.Destroy || !g_cublas.SetStream || !g_cublas.Dgemm) return false;
-  g_cublas.so = so;
-  return true;
-}
-
-thread_local std::string g_create_error;
-
-}  // namespace
 
 // ==================================================================================================
 // handle
