@@ -33,6 +33,22 @@ METRIC = "Landau Jacobian builds/sec + pair-interactions/sec; FP64 % of peak, 1/
 UNIT = "builds/s"
 
 
+class StdoutToStderr:
+    """Route fd 1 to fd 2 while libraries initialise (NCCL may print its version on stdout), so that
+    rank 0's stdout carries exactly one JSON line."""
+
+    def __enter__(self):
+        sys.stdout.flush()
+        self._saved = os.dup(1)
+        os.dup2(2, 1)
+        return self
+
+    def __exit__(self, *a):
+        sys.stdout.flush()
+        os.dup2(self._saved, 1)
+        os.close(self._saved)
+
+
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -219,7 +235,8 @@ def main():
 
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        with StdoutToStderr():
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     stream = torch.cuda.current_stream()
     desc, prob0, items = workload(args, world, rank)
     dist_desc = None
@@ -233,7 +250,8 @@ def main():
         items = [prob0]
         desc = dict(desc, workload="C5: one e+D Q4 mesh (4352 cells, N=108800), target cells split over the GPUs, "
                                    "NCCL all-gather of G")
-    h = L.Landau.from_problem(prob0, device=local, stream=stream, dist=dist_desc)
+    with StdoutToStderr():
+        h = L.Landau.from_problem(prob0, device=local, stream=stream, dist=dist_desc)
     if args.tensor_cache:
         h.set_tensor_cache(True)
         desc = dict(desc, variant="NEXT-4 tensor cache: inner integral as FP64 GEMMs over cached tensors")
