@@ -223,6 +223,15 @@ struct InnerPlan {
   int64_t wtiles, nsplit, split_len;
 };
 
+// minimum (batch x symmetric work items) per SM for the symmetric kernel (LANDAU_SYM_MIN_ITEMS_PER_SM)
+int64_t sym_min_items_per_sm() {
+  static const int64_t v = [] {
+    const char *e = getenv("LANDAU_SYM_MIN_ITEMS_PER_SM");
+    return e ? (int64_t)atoll(e) : (int64_t)8 * kSymWarps;
+  }();
+  return v;
+}
+
 bool sym_enabled() {
   static const bool v = [] {
     const char *e = getenv("LANDAU_SYM");
@@ -248,7 +257,7 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
   const int variant = inner_variant();
   // symmetric path: all targets on this rank (no element split across ranks), enough work items to
   // fill the GPU, and partial slots within 24 GiB (C5: ~11 GiB of the 180 GB HBM)
-  ip.sym = sym_enabled() && h->world == 1 && h->nsym_items > 0 && nbatch * h->nsym_items >= 8LL * kSymWarps * num_sms(h) &&
+  ip.sym = sym_enabled() && h->world == 1 && h->nsym_items > 0 && nbatch * h->nsym_items >= sym_min_items_per_sm() * num_sms(h) &&
            nbatch * h->nsym_slots * 160 * (int64_t)sizeof(double) <= (24LL << 30);
   if (ip.sym) {
     ip.tpt = 1;
