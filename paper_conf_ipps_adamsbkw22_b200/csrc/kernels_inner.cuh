@@ -12,12 +12,6 @@ namespace landau {
 #define LANDAU_SYM_UNROLL 2
 #endif
 constexpr int kSymUnroll = LANDAU_SYM_UNROLL;
-#ifndef LANDAU_SYM_HYBRID_COEF
-#define LANDAU_SYM_HYBRID_COEF 0
-#endif
-#ifndef LANDAU_SYM_SMEM_COEF
-#define LANDAU_SYM_SMEM_COEF 0
-#endif
 #ifndef LANDAU_SYM_WARPS
 #define LANDAU_SYM_WARPS 4
 #endif
@@ -43,10 +37,11 @@ __global__ void __launch_bounds__(kInnerTB, MINB) inner_kernel(int64_t N, int64_
                                                              int64_t out_bstride) {
   __shared__ double2 s_rz[kInnerWarps][32], s_w[kInnerWarps][32], s_wz[kInnerWarps][32];   // (wkz, rb^2)
   __shared__ double s_coef[kNumPairCoef];
-  stage_pair_coef(s_coef);
+  __shared__ double2 s_ltab[kLogTab];
+  stage_pair_coef(s_coef, s_ltab);
   __syncthreads();
   PairCoef cf;
-  load_pair_coef(s_coef, cf);
+  load_pair_coef(s_coef, s_ltab, cf);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int64_t item = (int64_t)blockIdx.x * kInnerWarps + wid;
   if (item >= nitems) return;   // whole warp: no block-level barrier follows
@@ -149,10 +144,10 @@ __device__ __forceinline__ void sym_store(double *o, int lane, const Acc5 &a) {
 // The reverse sums travel with their j: at step k lane L holds the accumulator of j = (L + k) mod 32
 // and hands it to lane L - 1 by a shuffle, so consecutive steps carry no memory fence and their
 // (long, independent) pair evaluations overlap; the j data itself is read-only shared memory.
-template <int NI, bool DIAG, bool MASK, class CF>
+template <int NI, bool DIAG, bool MASK>
 __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, const double *pz, const double *wb,
                                         int64_t N, int lane, const double2 *s_rz, const double2 *s_w,
-                                        const double2 *s_wz, const CF &cf, double *o) {
+                                        const double2 *s_wz, const PairCoef &cf, double *o) {
   double r[NI], z[NI], r2[NI], wd[NI], wkr[NI], wkz[NI];
   Acc5 ai[NI];
 #pragma unroll
@@ -173,7 +168,7 @@ __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, con
     const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
 #pragma unroll
     for (int t = 0; t < NI; t++)
-      landau_pair_sym<CF, MASK>(r[t], z[t], r2[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, true, cf,
+      landau_pair_sym<MASK>(r[t], z[t], r2[t], wd[t], wkr[t], wkz[t], rz.x, rz.y, wz.y, w.x, w.y, wz.x, true, cf,
                                 ai[t], aj);
     aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
     aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
@@ -184,7 +179,7 @@ __device__ __forceinline__ void sym_run(const SymItem &it, const double *pr, con
   if constexpr (DIAG) {
     const int jj = (lane + 16) & 31;
     const double2 rz = s_rz[jj], w = s_w[jj], wz = s_wz[jj];
-    landau_pair_sym<CF, true>(r[0], z[0], r2[0], wd[0], wkr[0], wkz[0], rz.x, rz.y, wz.y, w.x, w.y, wz.x, lane < 16, cf,
+    landau_pair_sym<true>(r[0], z[0], r2[0], wd[0], wkr[0], wkz[0], rz.x, rz.y, wz.y, w.x, w.y, wz.x, lane < 16, cf,
                               ai[0], aj);
     aj.drr = __shfl_sync(0xffffffffu, aj.drr, src);
     aj.drz = __shfl_sync(0xffffffffu, aj.drz, src);
@@ -213,25 +208,12 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_sym_kernel(int64_t
                                                                          const double *__restrict__ wT,
                                                                          double *__restrict__ part) {
   __shared__ double2 s_rz[kSymWarps][32], s_w[kSymWarps][32], s_wz[kSymWarps][32];   // (wkz, rb^2)
-#if LANDAU_SYM_SMEM_COEF
-  __shared__ __align__(16) double s_coef[kNumSmemCoef];
-  stage_smem_coef(s_coef);
-  __syncthreads();
-  const SmemCoef cf{reinterpret_cast<const double2 *>(s_coef), reinterpret_cast<const double2 *>(s_coef) + ELL_D_DEG + 1,
-                    s_coef + 4 * (ELL_D_DEG + 1)};
-#elif LANDAU_SYM_HYBRID_COEF
-  __shared__ double s_coef[kNumPairCoef];
-  stage_pair_coef(s_coef);
-  __syncthreads();
-  HybridCoef cf;
-  load_hybrid_coef(s_coef, cf);
-#else
-  __shared__ double s_coef[kNumPairCoef];
-  stage_pair_coef(s_coef);
+__shared__ double s_coef[kNumPairCoef];
+  __shared__ double2 s_ltab[kLogTab];
+  stage_pair_coef(s_coef, s_ltab);
   __syncthreads();
   PairCoef cf;
-  load_pair_coef(s_coef, cf);
-#endif
+  load_pair_coef(s_coef, s_ltab, cf);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   // persistent warps: grid-stride over the (batch item, work item) list
   for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
@@ -287,17 +269,18 @@ __global__ void __launch_bounds__(128) tensor_fill_kernel(int64_t N, const doubl
                                                           const double *__restrict__ pz, double *__restrict__ A1,
                                                           double *__restrict__ A2, double *__restrict__ A3) {
   __shared__ double s_coef[kNumPairCoef];
-  stage_pair_coef(s_coef);
+  __shared__ double2 s_ltab[kLogTab];
+  stage_pair_coef(s_coef, s_ltab);
   __syncthreads();
   PairCoef cf;
-  load_pair_coef(s_coef, cf);
+  load_pair_coef(s_coef, s_ltab, cf);
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t j = blockIdx.y;
   if (i >= N) return;
   const double r = pr[i], z = pz[i], rb = pr[j], zb = pz[j];
   bool ok;
   double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
-  pair_tensors<PairCoef, true>(r, z, r * r, rb, zb, rb * rb, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
+  pair_tensors<true>(r, z, r * r, rb, zb, rb * rb, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
   if (!ok) Udrr = Udrz = Udzz = Ukrr = Ukzr = 0.0;
   A1[i + j * 3 * N] = Udrr;
   A1[N + i + j * 3 * N] = Udrz;
