@@ -143,10 +143,10 @@ def load_profile_traffic(workload):
 # FP64 FLOP (2*DFMA + DMUL + DADD) per pair evaluation, counted once from ncu
 # sm__sass_thread_inst_executed_op_{dfma,dmul,dadd}_pred_on of each inner kernel on the C4 workload
 # (profiles/r01_inner_ncu.txt):
-#   directed kernel:  187 FLOP per ordered (target, source) pair, N^2 per batch item
-#   symmetric kernel: 203 FLOP per unordered pair, N (N - 1) / 2 per batch item (both targets updated)
-FLOP_PER_PAIR_DIRECTED = 187.0
-FLOP_PER_PAIR_SYMMETRIC = 203.0
+#   directed kernel:  177 FLOP per ordered (target, source) pair, N^2 per batch item
+#   symmetric kernel: 193 FLOP per unordered pair, N (N - 1) / 2 per batch item (both targets updated)
+FLOP_PER_PAIR_DIRECTED = 177.0
+FLOP_PER_PAIR_SYMMETRIC = 193.0
 
 
 def cpu_baseline(args, desc, nsample):
