@@ -400,3 +400,34 @@ def test_tensor_cache_gemm_path_C4():
     h.set_tensor_cache(False)
     h.jacobian_batched(out)
     assert h.stats()["inner_path"] == 1
+
+
+def test_more_error_codes_and_coo_batched():
+    prob = inputs.config2()
+    h = L.Landau.from_problem(prob, device=0)
+    lib = L.lib()
+    import ctypes
+    assert lib.landau_set_state_batched(h._h, 0, ctypes.c_void_p(16)) == L.LANDAU_EINVAL
+    assert lib.landau_set_state_batched(h._h, 2, None) == L.LANDAU_EINVAL
+    assert lib.landau_mass(h._h, 1.0, None, L.LANDAU_CSR) == L.LANDAU_EINVAL
+    assert lib.landau_point_coeffs(h._h, None) == L.LANDAU_EINVAL
+    assert "set_state" in lib.landau_last_error(h._h).decode() or lib.landau_last_error(h._h)
+    # batched COO = per-vertex COO
+    nodes = h.all_nodes()
+    F = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in (3, 700)]), device=DEV)
+    h.set_state_batched(F)
+    out = torch.empty((2, h.ncoo), dtype=torch.float64, device=DEV)
+    h.jacobian_batched(out, L.LANDAU_COO)
+    torch.cuda.synchronize()
+    for k in range(2):
+        single = gpu_jacobian(h, F[k].cpu().numpy(), L.LANDAU_COO)
+        assert np.abs(single - out[k].cpu().numpy()).max() <= 1e-13 * np.abs(single).max()
+    # COO summed into the CSR pattern equals the CSR output
+    import scipy.sparse as sps
+    row, col = h.pattern(coo=True)
+    rp, ccol = h.pattern()
+    Jcoo = gpu_jacobian(h, F[0].cpu().numpy(), L.LANDAU_COO)
+    Jcsr = gpu_jacobian(h, F[0].cpu().numpy(), L.LANDAU_CSR)
+    A = sps.coo_matrix((Jcoo, (row, col)), shape=(h.ndof, h.ndof)).tocsr()
+    A.sort_indices()
+    assert np.abs(A.data - Jcsr).max() <= 1e-14 * np.abs(Jcsr).max()
