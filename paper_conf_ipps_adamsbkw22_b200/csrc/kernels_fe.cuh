@@ -102,8 +102,11 @@ __global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbat
 // t_k = gk_r K_r + gk_z K_z;  C^D[k,l] += gk_r u_l + gk_z v_l,  C^K[k,l] += t_k phi_l.
 // G is read in the chunked layout G[((i / Nc) * nbatch + b) * 5 + c][i % Nc] (Nc = N unless split).
 // ------------------------------------------------------------------------------------------------
+#ifndef LANDAU_EL_MINB
+#define LANDAU_EL_MINB 1
+#endif
 template <int NB, int S, int EPB>
-__global__ void __launch_bounds__(NB * EPB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
+__global__ void __launch_bounds__(NB * EPB, LANDAU_EL_MINB) element_kernel(int64_t ncell, const double *__restrict__ G, int64_t Nc,
                                                              int nbatch, int b0, int nb, const double *__restrict__ pw,
                                                              const double *__restrict__ cell_h,
                                                              const double *__restrict__ tab, double *__restrict__ Cbuf) {

@@ -420,7 +420,10 @@ int launch_element(landau_t h, int64_t nbatch, int64_t b0, int64_t nb) {
   const Plan &P = h->plan;
   Timer t(h, LANDAU_T_ELEMENT);
   constexpr int S = NB == 9 ? 3 : (NB == 16 ? 4 : 5);
-  constexpr int EPB = NB == 9 ? 14 : (NB == 16 ? 8 : 5);   // ~128 threads per block
+#ifndef LANDAU_EL_EPB16
+#define LANDAU_EL_EPB16 8
+#endif
+  constexpr int EPB = NB == 9 ? 14 : (NB == 16 ? LANDAU_EL_EPB16 : 5);   // ~128 threads per block
   const int64_t items = (P.ncell + EPB - 1) / EPB * nb;
   const unsigned grid = (unsigned)std::min<int64_t>(items, 16LL * num_sms(h));
   element_kernel<NB, S, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, (int)b0, (int)nb,
