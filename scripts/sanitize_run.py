@@ -1,0 +1,30 @@
+# small workloads for compute-sanitizer: every kernel of the library on C1, C3 and a symmetric batch
+import os, sys
+sys.path.insert(0, os.getcwd())
+import numpy as np, torch
+from paper_conf_ipps_adamsbkw22_b200 import inputs
+from paper_conf_ipps_adamsbkw22_b200 import landau as L
+for name in ("C1", "C3"):
+    p = inputs.CONFIGS[name]()
+    h = L.Landau.from_problem(p, device=0)
+    f = torch.tensor(inputs.coefficients(p, h.all_nodes()), device="cuda")
+    h.set_state(f)
+    for fmt, n in ((L.LANDAU_CSR, h.nnz), (L.LANDAU_COO, h.ncoo)):
+        v = torch.empty(n, dtype=torch.float64, device="cuda")
+        h.jacobian(v, fmt)
+        h.mass(2.0, v, fmt)
+    G = torch.empty((5, h.npoints), dtype=torch.float64, device="cuda")
+    h.point_coeffs(G)
+p0 = inputs.config4_vertex(0)
+h = L.Landau.from_problem(p0, device=0)
+nodes = h.all_nodes()
+F = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in range(16)]), device="cuda")
+os.environ["LANDAU_SYM_MIN_ITEMS_PER_SM"] = "0"
+h.set_state_batched(F)
+v = torch.empty((16, h.nnz), dtype=torch.float64, device="cuda")
+h.jacobian_batched(v)
+print("stats", h.stats())
+fh = F.cpu().pin_memory(); vh = torch.empty((16, h.nnz), dtype=torch.float64).pin_memory()
+h.jacobian_host(fh, vh)
+torch.cuda.synchronize()
+print("ok")
