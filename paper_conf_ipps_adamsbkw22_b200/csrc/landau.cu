@@ -908,7 +908,11 @@ int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, doubl
     CU(cudaStreamCreateWithFlags(&h->s_h2d, cudaStreamNonBlocking));
     CU(cudaStreamCreateWithFlags(&h->s_d2h, cudaStreamNonBlocking));
   }
-  const int64_t K = std::max<int64_t>(1, std::min<int64_t>(8, nbatch / 64));
+  static const int64_t kmax = [] {
+    const char *e = getenv("LANDAU_HOST_CHUNKS");
+    return e ? (int64_t)atoll(e) : (int64_t)8;   // 16 measured no better
+  }();
+  const int64_t K = std::max<int64_t>(1, std::min<int64_t>(kmax, nbatch / 64));
   const int64_t cb = (nbatch + K - 1) / K;
   while ((int64_t)h->ev_h2d.size() < K) {
     cudaEvent_t a, b;
