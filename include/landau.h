@@ -150,9 +150,10 @@ int landau_partition(int64_t nelem, int32_t world, int32_t rank, int64_t *e0, in
 int landau_nccl_unique_id(void *out128);
 
 /* Per-stage device timers (CUDA events on the handle's stream): stage = 0 field, 1 inner,
- * 2 reduce, 3 element, 4 assemble, 5 mass, 6 allgather.  enable resets the accumulators. */
+ * 2 reduce, 3 element, 4 assemble, 5 mass, 6 allgather, 7 band factor, 8 band solve.  enable resets
+ * the accumulators. */
 enum { LANDAU_T_FIELD = 0, LANDAU_T_INNER, LANDAU_T_REDUCE, LANDAU_T_ELEMENT, LANDAU_T_ASSEMBLE,
-       LANDAU_T_MASS, LANDAU_T_ALLGATHER, LANDAU_NTIMERS };
+       LANDAU_T_MASS, LANDAU_T_ALLGATHER, LANDAU_T_FACTOR, LANDAU_T_SOLVE, LANDAU_NTIMERS };
 int landau_set_timing(landau_t h, int32_t enable);
 /* ms[LANDAU_NTIMERS] total milliseconds, launches[LANDAU_NTIMERS] kernel launches (synchronises) */
 int landau_get_timing(landau_t h, double *ms, int64_t *launches);
@@ -169,6 +170,21 @@ int landau_get_launch_count(landau_t h, int64_t *count);
  * The same sums as the pairwise kernels up to summation order.  EUNSUPPORTED for element-split
  * handles or when 7 N^2 doubles exceed 16 GiB; enable = 0 frees the cache. */
 int landau_set_tensor_cache(landau_t h, int32_t enable);
+
+/* NEXT-2 (PAPER.md:1@24330-26180, §III-G): the paper's direct solver for the implicit
+ * step.  Each species block of A = shift * M - J is put in reverse Cuthill-McKee order and band
+ * storage (half-bandwidth B = UBW = LBW of the grid's pattern) and factored by the outer-product
+ * band LU without pivoting (Golub-Van Loan Alg. 4.3.1), one CTA per (batch item, species block);
+ * the solve is a forward/backward substitution, one warp per block.  Without pivoting the
+ * factorisation needs A to be safely non-singular on its leading minors, as it is for the shift of
+ * an implicit step (shift * M dominant); a zero pivot yields inf/nan in x, nothing aborts.
+ *   landau_band_info:      B and the RCM permutation perm[new] = old of one grid (host, may be NULL)
+ *   landau_band_factor_batched: J_csr_dev = [nbatch][nnz_csr] (e.g. from landau_jacobian_batched)
+ *   landau_band_solve_batched:  b_dev, x_dev = [nbatch][ndof] species-major (may alias); uses the
+ *                          last factorisation (ESTATE before any, or when nbatch differs) */
+int landau_band_info(landau_t h, int32_t grid, int32_t *bandwidth, int32_t *perm);
+int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const double *J_csr_dev);
+int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev);
 
 /* How the last build ran (for FLOP accounting and diagnostics). */
 typedef struct {

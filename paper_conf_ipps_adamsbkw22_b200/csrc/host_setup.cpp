@@ -330,6 +330,80 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
       G.rowptr[i + 1] = G.rowptr[i] + (int64_t)r.size();
       G.col.insert(G.col.end(), r.begin(), r.end());
     }
+    // ---- RCM ordering and band map (NEXT-2) ---------------------------------------------------
+    // reverse Cuthill-McKee: BFS from a pseudo-peripheral node, neighbours by increasing degree,
+    // every connected component in turn, then the order reversed (PAPER.md:1@25294, [23])
+    {
+      const int n = G.ndof;
+      std::vector<int> deg(n);
+      for (int i = 0; i < n; i++) deg[i] = (int)(G.rowptr[i + 1] - G.rowptr[i]);
+      auto bfs = [&](int root, std::vector<int> &order, std::vector<int> &level, std::vector<char> &seen) {
+        order.clear();
+        order.push_back(root);
+        seen[root] = 1;
+        level[root] = 0;
+        for (size_t h = 0; h < order.size(); h++) {
+          const int u = order[h];
+          std::vector<int> nb;
+          for (int64_t q = G.rowptr[u]; q < G.rowptr[u + 1]; q++) {
+            const int v = G.col[q];
+            if (!seen[v]) nb.push_back(v);
+          }
+          std::sort(nb.begin(), nb.end(), [&](int a, int b) { return deg[a] != deg[b] ? deg[a] < deg[b] : a < b; });
+          for (int v : nb)
+            if (!seen[v]) {
+              seen[v] = 1;
+              level[v] = level[u] + 1;
+              order.push_back(v);
+            }
+        }
+      };
+      std::vector<char> done(n, 0);
+      std::vector<int> cm, level(n, 0), order;
+      for (int start = 0; start < n; start++) {
+        if (done[start]) continue;
+        // pseudo-peripheral root (George-Liu): repeat BFS from a min-degree node of the last level
+        int root = start;
+        int last_depth = -1;
+        for (int it = 0; it < 8; it++) {
+          std::vector<char> seen(done);
+          bfs(root, order, level, seen);
+          const int depth = level[order.back()];
+          if (depth <= last_depth) break;
+          last_depth = depth;
+          int best = order.back();
+          for (int v : order)
+            if (level[v] == depth && deg[v] < deg[best]) best = v;
+          root = best;
+        }
+        std::vector<char> seen(done);
+        bfs(root, order, level, seen);
+        for (int v : order) {
+          done[v] = 1;
+          cm.push_back(v);
+        }
+      }
+      G.rcm_perm.assign(cm.rbegin(), cm.rend());
+      G.rcm_iperm.assign(n, 0);
+      for (int k = 0; k < n; k++) G.rcm_iperm[G.rcm_perm[k]] = k;
+      int B = 0, B0 = 0;
+      for (int i = 0; i < n; i++)
+        for (int64_t q = G.rowptr[i]; q < G.rowptr[i + 1]; q++) {
+          B = std::max(B, std::abs(G.rcm_iperm[i] - G.rcm_iperm[G.col[q]]));
+          B0 = std::max(B0, std::abs(i - G.col[q]));
+        }
+      if (B0 < B) {   // tiny meshes: the (z, r) numbering can beat RCM; keep the smaller band
+        for (int k = 0; k < n; k++) G.rcm_perm[k] = G.rcm_iperm[k] = k;
+        B = B0;
+      }
+      G.band = B;
+      G.band_slot.resize(G.col.size());
+      for (int i = 0; i < n; i++)
+        for (int64_t q = G.rowptr[i]; q < G.rowptr[i + 1]; q++) {
+          const int ni = G.rcm_iperm[i], nj = G.rcm_iperm[G.col[q]];
+          G.band_slot[q] = (int32_t)((int64_t)ni * (2 * B + 1) + (nj - ni + B));
+        }
+    }
     // ---- gather maps --------------------------------------------------------------------------
     // slot contributions: (cell, a, b) with P[a][i] P[b][j] != 0, in (cell, a, b) order
     GatherMap csr, coo;

@@ -32,6 +32,11 @@ struct GridPlan {
   std::vector<int64_t> rowptr;           // [ndof+1]
   std::vector<int> col;
   int64_t ncoo = 0;                      // sum_e n_e^2
+  // NEXT-2 band solver (PAPER.md:1@25294): reverse Cuthill-McKee ordering of this grid's DOF graph
+  std::vector<int> rcm_perm;             // [ndof] new -> old
+  std::vector<int> rcm_iperm;            // [ndof] old -> new
+  int band = 0;                          // half-bandwidth B = max |iperm(i) - iperm(j)| over the pattern
+  std::vector<int32_t> band_slot;        // [nnz] CSR slot -> row-major band index iperm(i) (2B+1) + iperm(j) - iperm(i) + B
 };
 
 // A gather map: output slot s = sum over its contributions (idx, w) of w * Celem[idx], in a fixed

@@ -27,6 +27,7 @@ using namespace landau;
 #include "dynload.h"
 #include "kernels_fe.cuh"
 #include "kernels_inner.cuh"
+#include "kernels_band.cuh"
 
 
 // ==================================================================================================
@@ -74,6 +75,14 @@ struct landau_s {
   bool tcache = false, tcache_valid = false;
   double *d_U = nullptr;     // A1 (3N^2) | A2 (2N^2) | A3 (2N^2)
   cublasHandle_ cublas = nullptr;
+  // band solver (NEXT-2)
+  std::vector<int32_t *> d_band_slot;   // per grid
+  BandDesc *d_band_desc = nullptr;      // per species
+  std::vector<BandDesc> band_desc;
+  int32_t *d_perm_all = nullptr;
+  int64_t *d_perm_off = nullptr, *d_vec_off = nullptr;
+  int64_t band_bstride = 0, band_cap = 0, band_nbatch = 0;
+  double *d_band = nullptr, *d_band_scratch = nullptr;
   // host staging for landau_jacobian_host: full-batch device buffers, two copy streams
   double *d_vals_tmp = nullptr;
   int64_t vals_tmp_cap = 0;
@@ -732,6 +741,26 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
         (rc = upload(h, &h->d_tile_slots, tslots)))
       return bail(rc);
   }
+  {   // band solver maps (NEXT-2)
+    h->d_band_slot.assign(P.ngrids, nullptr);
+    for (int g = 0; g < P.ngrids; g++)
+      if ((rc = upload(h, &h->d_band_slot[g], P.grids[g].band_slot))) return bail(rc);
+    std::vector<int32_t> perm_all;
+    std::vector<int64_t> perm_off, vec_off;
+    int64_t off = 0;
+    for (int a = 0; a < h->S; a++) {
+      const GridPlan &G = P.grids[h->sgrid[a]];
+      h->band_desc.push_back({off, G.ndof, G.band});
+      off += (int64_t)G.ndof * (2 * G.band + 1);
+      perm_off.push_back((int64_t)perm_all.size());
+      perm_all.insert(perm_all.end(), G.rcm_perm.begin(), G.rcm_perm.end());
+      vec_off.push_back(h->soff[a]);
+    }
+    h->band_bstride = off;
+    if ((rc = upload(h, &h->d_band_desc, h->band_desc)) || (rc = upload(h, &h->d_perm_all, perm_all)) ||
+        (rc = upload(h, &h->d_perm_off, perm_off)) || (rc = upload(h, &h->d_vec_off, vec_off)))
+      return bail(rc);
+  }
   h->d_csr.resize(P.ngrids);
   h->d_coo.resize(P.ngrids);
   h->d_mass_csr.assign(P.ngrids, nullptr);
@@ -773,6 +802,13 @@ void landau_destroy(landau_t h) {
   drop_graphs(h);
   if (h->cublas && g_cublas.Destroy) g_cublas.Destroy(h->cublas);
   cudaFree(h->d_U);
+  for (int32_t *p : h->d_band_slot) cudaFree(p);
+  cudaFree(h->d_band_desc);
+  cudaFree(h->d_perm_all);
+  cudaFree(h->d_perm_off);
+  cudaFree(h->d_vec_off);
+  cudaFree(h->d_band);
+  cudaFree(h->d_band_scratch);
   if (h->s_h2d) cudaStreamDestroy(h->s_h2d);
   if (h->s_d2h) cudaStreamDestroy(h->s_d2h);
   for (auto e : h->ev_h2d) cudaEventDestroy(e);
@@ -1023,6 +1059,13 @@ int landau_set_tensor_cache(landau_t h, int32_t enable) {
     drop_graphs(h);
     CU(cudaStreamSynchronize(h->stream));
     cudaFree(h->d_U);
+  for (int32_t *p : h->d_band_slot) cudaFree(p);
+  cudaFree(h->d_band_desc);
+  cudaFree(h->d_perm_all);
+  cudaFree(h->d_perm_off);
+  cudaFree(h->d_vec_off);
+  cudaFree(h->d_band);
+  cudaFree(h->d_band_scratch);
     h->d_U = nullptr;
     h->tcache = h->tcache_valid = false;
     return LANDAU_OK;
@@ -1041,6 +1084,78 @@ int landau_set_tensor_cache(landau_t h, int32_t enable) {
   drop_graphs(h);
   h->tcache = true;
   h->tcache_valid = false;
+  return LANDAU_OK;
+}
+
+int landau_band_info(landau_t h, int32_t grid, int32_t *bandwidth, int32_t *perm) {
+  if (!h || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
+  const GridPlan &G = h->plan.grids[grid];
+  if (bandwidth) *bandwidth = G.band;
+  if (perm) memcpy(perm, G.rcm_perm.data(), sizeof(int32_t) * G.ndof);
+  return LANDAU_OK;
+}
+
+int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const double *J_csr_dev) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !J_csr_dev) return fail(h, LANDAU_EINVAL, "band_factor: bad argument");
+  if (nbatch > h->band_cap) {
+    cudaFree(h->d_band);
+    cudaFree(h->d_band_scratch);
+    h->d_band = h->d_band_scratch = nullptr;
+    CU(cudaMalloc(&h->d_band, sizeof(double) * nbatch * h->band_bstride));
+    CU(cudaMalloc(&h->d_band_scratch, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
+    h->band_cap = nbatch;
+  }
+  Timer t(h, LANDAU_T_FACTOR);
+  CU(cudaMemsetAsync(h->d_band, 0, sizeof(double) * nbatch * h->band_bstride, h->stream));
+  for (int a = 0; a < h->S; a++) {
+    const int g = h->sgrid[a];
+    const int64_t nslots = (int64_t)h->plan.grids[g].col.size();
+    if (!nslots) continue;
+    const int blocks = (int)std::min<int64_t>((nslots * nbatch + 255) / 256, 16LL * num_sms(h));
+    band_fill_kernel<<<blocks, 256, 0, h->stream>>>(nslots, h->d_band_slot[g], h->d_mass_csr[g], J_csr_dev, h->nnz,
+                                                    h->snnz_off[a], shift, h->d_band, h->band_bstride,
+                                                    h->band_desc[a].off, (int)nbatch);
+    h->launches++;
+    KCHECK();
+  }
+  int maxB = 0;
+  for (auto &d : h->band_desc) {
+    maxB = std::max(maxB, d.B);
+    // one CTA per matrix: meant for vertex-grid sizes (C1-C4); a single large grid (C5) would need a
+    // multi-CTA factorisation (not built)
+    if ((double)d.n * d.B * d.B > 2e9) return fail(h, LANDAU_EUNSUPPORTED, "band factor: n B^2 too large for one CTA");
+  }
+  const size_t smem = sizeof(double) * std::max(maxB, 1);
+  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(band_factor_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  // a CTA per matrix; few warps per CTA and many CTAs per SM: the factorisation is a chain of n
+  // barrier-separated steps of B^2 updates, so concurrency across matrices hides the step latency
+  static const int band_threads = [] {
+    const char *e = getenv("LANDAU_BAND_THREADS");
+    return e ? atoi(e) : 512;   // measured: 1024 15.6 ms, 512 14.1 ms, 256 17.5 ms (C4 batch)
+  }();
+  const int threads = std::min(band_threads, std::max(64, ((maxB * maxB + 31) / 32) * 32));
+  band_factor_kernel<<<(unsigned)(nbatch * h->S), threads, smem, h->stream>>>(h->d_band, h->band_bstride,
+                                                                             h->d_band_desc, h->S);
+  h->launches++;
+  h->tlaunch[LANDAU_T_FACTOR]++;
+  KCHECK();
+  h->band_nbatch = nbatch;
+  return LANDAU_OK;
+}
+
+int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !b_dev || !x_dev) return fail(h, LANDAU_EINVAL, "band_solve: bad argument");
+  if (h->band_nbatch != nbatch) return fail(h, LANDAU_ESTATE, "band_solve: factor this batch first");
+  Timer t(h, LANDAU_T_SOLVE);
+  const int64_t warps = nbatch * h->S;
+  band_solve_kernel<<<(unsigned)((warps * 32 + 127) / 128), 128, 0, h->stream>>>(
+      h->d_band, h->band_bstride, h->d_band_desc, h->d_perm_all, h->d_perm_off, h->d_vec_off, h->ndof, b_dev,
+      h->d_band_scratch, x_dev, h->S, (int)nbatch);
+  h->launches++;
+  h->tlaunch[LANDAU_T_SOLVE]++;
+  KCHECK();
   return LANDAU_OK;
 }
 

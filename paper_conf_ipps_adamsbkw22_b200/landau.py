@@ -19,7 +19,7 @@ LANDAU_OK, LANDAU_EINVAL, LANDAU_ENOMEM, LANDAU_ECUDA, LANDAU_ENCCL, LANDAU_ESTA
 LANDAU_CSR, LANDAU_COO = 0, 1
 LANDAU_DIST_REPLICATE, LANDAU_DIST_BATCH, LANDAU_DIST_ELEMENTS = 0, 1, 2
 LANDAU_HOST_ONLY = -1
-TIMERS = ("field", "inner", "reduce", "element", "assemble", "mass", "allgather")
+TIMERS = ("field", "inner", "reduce", "element", "assemble", "mass", "allgather", "factor", "solve")
 
 _lib = None
 
@@ -82,6 +82,9 @@ def lib():
             "landau_get_launch_count": (C.c_int, [vp, P64]),
             "landau_get_stats": (C.c_int, [vp, C.POINTER(_Stats)]),
             "landau_set_tensor_cache": (C.c_int, [vp, i32]),
+            "landau_band_info": (C.c_int, [vp, i32, P32, P32]),
+            "landau_band_factor_batched": (C.c_int, [vp, i64, d, vp]),
+            "landau_band_solve_batched": (C.c_int, [vp, i64, vp, vp]),
             "landau_strerror": (C.c_char_p, [C.c_int]),
             "landau_last_error": (C.c_char_p, [vp]),
             "landau_version": (C.c_char_p, []),
@@ -272,6 +275,22 @@ class Landau:
         self._check(lib().landau_get_timing(self._h, _dptr(ms), n.ctypes.data_as(C.POINTER(C.c_int64))),
                     "landau_get_timing")
         return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(TIMERS)}
+
+    def band_info(self, g):
+        B = C.c_int32()
+        perm = np.zeros(self.grid_ndof(g), dtype=np.int32)
+        self._check(lib().landau_band_info(self._h, g, C.byref(B), perm.ctypes.data_as(C.POINTER(C.c_int32))),
+                    "landau_band_info")
+        return B.value, perm
+
+    def band_factor_batched(self, shift, J):
+        nb = J.shape[0] if J.dim() == 2 else 1
+        self._check(lib().landau_band_factor_batched(self._h, nb, float(shift), _tptr(J)), "landau_band_factor_batched")
+
+    def band_solve_batched(self, b, x):
+        nb = b.shape[0] if b.dim() == 2 else 1
+        self._check(lib().landau_band_solve_batched(self._h, nb, _tptr(b), _tptr(x)), "landau_band_solve_batched")
+        return x
 
     def set_tensor_cache(self, enable=True):
         self._check(lib().landau_set_tensor_cache(self._h, int(bool(enable))), "landau_set_tensor_cache")
