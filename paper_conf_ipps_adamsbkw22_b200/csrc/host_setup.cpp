@@ -397,12 +397,39 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
         B = B0;
       }
       G.band = B;
-      G.band_slot.resize(G.col.size());
-      for (int i = 0; i < n; i++)
-        for (int64_t q = G.rowptr[i]; q < G.rowptr[i + 1]; q++) {
-          const int ni = G.rcm_iperm[i], nj = G.rcm_iperm[G.col[q]];
-          G.band_slot[q] = (int32_t)((int64_t)ni * (2 * B + 1) + (nj - ni + B));
+      // entering-row entry lists (see host_setup.h); the pattern is symmetric, so A(j, i) is the CSR
+      // entry (perm j, perm i), found by a binary search in its sorted row
+      auto slot_of = [&](int r, int c) -> int32_t {
+        const int *b = G.col.data() + G.rowptr[r], *e = G.col.data() + G.rowptr[r + 1];
+        const int *f = std::lower_bound(b, e, c);
+        return (f != e && *f == c) ? (int32_t)(f - G.col.data()) : -1;
+      };
+      // the factorisation runs a window of P = Bp + 1 rows, P a multiple of 8 (kernels_band.cuh):
+      // positions are relative to the padded half-bandwidth Bp >= B (entries past B are zero)
+      const int Bp = (B + 1 + 7) / 8 * 8 - 1;
+      G.band_p = Bp;
+      G.ent_ptr.assign(1, 0);
+      G.ent_slot.clear();
+      G.ent_pos.clear();
+      G.ent_max = 0;
+      std::vector<std::pair<int, int32_t>> ent;
+      for (int ni = 0; ni < n; ni++) {
+        const int oi = G.rcm_perm[ni];
+        ent.clear();
+        for (int64_t q = G.rowptr[oi]; q < G.rowptr[oi + 1]; q++) {
+          const int nj = G.rcm_iperm[G.col[q]];
+          if (nj <= ni) ent.push_back({nj - ni + Bp, (int32_t)q});                         // A(i, j), row part
+          if (nj < ni) ent.push_back({Bp + 1 + nj - ni + Bp, slot_of(G.col[q], oi)});      // A(j, i), column part
         }
+        std::sort(ent.begin(), ent.end());
+        for (auto &e : ent) {
+          if (e.second < 0) return "band: CSR pattern is not symmetric";
+          G.ent_pos.push_back((uint16_t)e.first);
+          G.ent_slot.push_back(e.second);
+        }
+        G.ent_max = std::max(G.ent_max, (int)ent.size());
+        G.ent_ptr.push_back((int32_t)G.ent_slot.size());
+      }
     }
     // ---- gather maps --------------------------------------------------------------------------
     // slot contributions: (cell, a, b) with P[a][i] P[b][j] != 0, in (cell, a, b) order

@@ -36,7 +36,15 @@ struct GridPlan {
   std::vector<int> rcm_perm;             // [ndof] new -> old
   std::vector<int> rcm_iperm;            // [ndof] old -> new
   int band = 0;                          // half-bandwidth B = max |iperm(i) - iperm(j)| over the pattern
-  std::vector<int32_t> band_slot;        // [nnz] CSR slot -> row-major band index iperm(i) (2B+1) + iperm(j) - iperm(i) + B
+  // Entries in the order the register-window factorisation consumes them, relative to the padded
+  // half-bandwidth Bp = (B + 1 rounded up to 8) - 1: RCM row i "enters" with its lower row part
+  // A(i, j), j <= i (pos = j - i + Bp in 0..Bp) and its upper column part A(j, i), j < i
+  // (pos = Bp + 1 + j - i + Bp in Bp+1..2Bp).  ent_slot = CSR slot of the entry.
+  int band_p = 0;
+  std::vector<int32_t> ent_ptr;          // [ndof+1]
+  std::vector<int32_t> ent_slot;         // [nnz]
+  std::vector<uint16_t> ent_pos;         // [nnz]
+  int ent_max = 0;                       // max entries of one entering row
 };
 
 // A gather map: output slot s = sum over its contributions (idx, w) of w * Celem[idx], in a fixed

@@ -76,13 +76,17 @@ struct landau_s {
   double *d_U = nullptr;     // A1 (3N^2) | A2 (2N^2) | A3 (2N^2)
   cublasHandle_ cublas = nullptr;
   // band solver (NEXT-2)
-  std::vector<int32_t *> d_band_slot;   // per grid
+  std::vector<int32_t *> d_ent_ptr, d_ent_slot;   // per grid: entering-row entry lists (host_setup.h)
+  std::vector<uint16_t *> d_ent_pos;
+  int band_ent_max = 0;
+  int64_t ent_bstride = 0;
+  double *d_Aent = nullptr;
   BandDesc *d_band_desc = nullptr;      // per species
   std::vector<BandDesc> band_desc;
   int32_t *d_perm_all = nullptr;
   int64_t *d_perm_off = nullptr, *d_vec_off = nullptr;
   int64_t band_bstride = 0, band_cap = 0, band_nbatch = 0;
-  double *d_band = nullptr, *d_band_scratch = nullptr;
+  double *d_band = nullptr;   // step-major LU factors [batch][band_bstride] (kernels_band.cuh)
   // host staging for landau_jacobian_host: full-batch device buffers, two copy streams
   double *d_vals_tmp = nullptr;
   int64_t vals_tmp_cap = 0;
@@ -333,6 +337,7 @@ int launch_inner(landau_t h, int64_t nbatch) {
     if (!st) st = g_cublas.Dgemm(h->cublas, 0, 0, n, nb, 2 * n, &one, h->d_U + 5 * n2, n, h->d_wT + N, 3 * n, &zero,
                                  G + 4 * N, 5 * n);
     if (st) return fail(h, LANDAU_ECUDA, "cublasDgemm failed: " + std::to_string(st));
+    (void)cudaGetLastError();   // cuBLAS may leave a benign runtime error behind on success
     h->tlaunch[LANDAU_T_INNER] += 1;   // one inner stage (three cuBLAS kernels, not counted as ours)
     return LANDAU_OK;
   }
@@ -680,6 +685,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     *out = h;
     return LANDAU_OK;
   }
+  (void)cudaGetLastError();   // a non-sticky error left by other code (a library, a freed handle) is not ours
   cudaError_t ce = cudaSetDevice(cuda_device);
   if (ce != cudaSuccess) {
     std::string m = std::string("cudaSetDevice: ") + cudaGetErrorString(ce);
@@ -742,21 +748,30 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
       return bail(rc);
   }
   {   // band solver maps (NEXT-2)
-    h->d_band_slot.assign(P.ngrids, nullptr);
+    h->d_ent_ptr.assign(P.ngrids, nullptr);
+    h->d_ent_slot.assign(P.ngrids, nullptr);
+    h->d_ent_pos.assign(P.ngrids, nullptr);
     for (int g = 0; g < P.ngrids; g++)
-      if ((rc = upload(h, &h->d_band_slot[g], P.grids[g].band_slot))) return bail(rc);
+      if ((rc = upload(h, &h->d_ent_ptr[g], P.grids[g].ent_ptr)) || (rc = upload(h, &h->d_ent_slot[g], P.grids[g].ent_slot)) ||
+          (rc = upload(h, &h->d_ent_pos[g], P.grids[g].ent_pos)))
+        return bail(rc);
     std::vector<int32_t> perm_all;
     std::vector<int64_t> perm_off, vec_off;
-    int64_t off = 0;
+    int64_t off = 0, aoff = 0;
     for (int a = 0; a < h->S; a++) {
-      const GridPlan &G = P.grids[h->sgrid[a]];
-      h->band_desc.push_back({off, G.ndof, G.band});
-      off += (int64_t)G.ndof * (2 * G.band + 1);
+      const int g = h->sgrid[a];
+      const GridPlan &G = P.grids[g];
+      h->band_desc.push_back(
+          {off, aoff, h->d_ent_ptr[g], h->d_ent_pos[g], G.ndof, G.band_p, G.band_p + 1, (int)G.ent_slot.size()});
+      off += (int64_t)G.ndof * (2 * G.band_p + 1);
+      aoff += (int64_t)G.ent_slot.size();
+      h->band_ent_max = std::max(h->band_ent_max, G.ent_max);
       perm_off.push_back((int64_t)perm_all.size());
       perm_all.insert(perm_all.end(), G.rcm_perm.begin(), G.rcm_perm.end());
       vec_off.push_back(h->soff[a]);
     }
     h->band_bstride = off;
+    h->ent_bstride = aoff;
     if ((rc = upload(h, &h->d_band_desc, h->band_desc)) || (rc = upload(h, &h->d_perm_all, perm_all)) ||
         (rc = upload(h, &h->d_perm_off, perm_off)) || (rc = upload(h, &h->d_vec_off, vec_off)))
       return bail(rc);
@@ -802,13 +817,15 @@ void landau_destroy(landau_t h) {
   drop_graphs(h);
   if (h->cublas && g_cublas.Destroy) g_cublas.Destroy(h->cublas);
   cudaFree(h->d_U);
-  for (int32_t *p : h->d_band_slot) cudaFree(p);
+  for (int32_t *p : h->d_ent_ptr) cudaFree(p);
+  for (int32_t *p : h->d_ent_slot) cudaFree(p);
+  for (uint16_t *p : h->d_ent_pos) cudaFree(p);
+  cudaFree(h->d_Aent);
   cudaFree(h->d_band_desc);
   cudaFree(h->d_perm_all);
   cudaFree(h->d_perm_off);
   cudaFree(h->d_vec_off);
   cudaFree(h->d_band);
-  cudaFree(h->d_band_scratch);
   if (h->s_h2d) cudaStreamDestroy(h->s_h2d);
   if (h->s_d2h) cudaStreamDestroy(h->s_d2h);
   for (auto e : h->ev_h2d) cudaEventDestroy(e);
@@ -835,6 +852,7 @@ void landau_destroy(landau_t h) {
     cudaEventDestroy(u.second.second);
   }
   for (auto e : h->ev_pool) cudaEventDestroy(e);
+  (void)cudaGetLastError();   // teardown leaves no error behind for the next call
   delete h;
 }
 
@@ -1059,13 +1077,6 @@ int landau_set_tensor_cache(landau_t h, int32_t enable) {
     drop_graphs(h);
     CU(cudaStreamSynchronize(h->stream));
     cudaFree(h->d_U);
-  for (int32_t *p : h->d_band_slot) cudaFree(p);
-  cudaFree(h->d_band_desc);
-  cudaFree(h->d_perm_all);
-  cudaFree(h->d_perm_off);
-  cudaFree(h->d_vec_off);
-  cudaFree(h->d_band);
-  cudaFree(h->d_band_scratch);
     h->d_U = nullptr;
     h->tcache = h->tcache_valid = false;
     return LANDAU_OK;
@@ -1098,45 +1109,55 @@ int landau_band_info(landau_t h, int32_t grid, int32_t *bandwidth, int32_t *perm
 int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const double *J_csr_dev) {
   if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
   if (!h || nbatch < 1 || !J_csr_dev) return fail(h, LANDAU_EINVAL, "band_factor: bad argument");
+  int maxPp = 8, maxn = 0, maxent = 0;
+  for (auto &d : h->band_desc) {
+    maxPp = std::max(maxPp, d.Pp);
+    maxn = std::max(maxn, d.n);
+    maxent = std::max(maxent, d.nent);
+  }
+  // one CTA per matrix with the active window in registers: vertex-grid sizes (C1-C4); a single large
+  // grid (C5) would need a multi-CTA factorisation (not built)
+  if (maxPp > kBandMaxP) return fail(h, LANDAU_EUNSUPPORTED, "band factor: half-bandwidth above 127");
+  const int W = 2 * (maxPp - 1) + 1;
+  const size_t smem = sizeof(double) * (2 * maxPp + 2 + 2 * W + (kBandD + 1) * W) + sizeof(int32_t) * (maxn + 1) +
+                      sizeof(uint16_t) * maxent;
+  if (smem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
   if (nbatch > h->band_cap) {
     cudaFree(h->d_band);
-    cudaFree(h->d_band_scratch);
-    h->d_band = h->d_band_scratch = nullptr;
+    cudaFree(h->d_Aent);
+    h->d_band = h->d_Aent = nullptr;
     CU(cudaMalloc(&h->d_band, sizeof(double) * nbatch * h->band_bstride));
-    CU(cudaMalloc(&h->d_band_scratch, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
+    CU(cudaMalloc(&h->d_Aent, sizeof(double) * nbatch * std::max<int64_t>(h->ent_bstride, 1)));
     h->band_cap = nbatch;
   }
   Timer t(h, LANDAU_T_FACTOR);
-  CU(cudaMemsetAsync(h->d_band, 0, sizeof(double) * nbatch * h->band_bstride, h->stream));
   for (int a = 0; a < h->S; a++) {
     const int g = h->sgrid[a];
-    const int64_t nslots = (int64_t)h->plan.grids[g].col.size();
-    if (!nslots) continue;
-    const int blocks = (int)std::min<int64_t>((nslots * nbatch + 255) / 256, 16LL * num_sms(h));
-    band_fill_kernel<<<blocks, 256, 0, h->stream>>>(nslots, h->d_band_slot[g], h->d_mass_csr[g], J_csr_dev, h->nnz,
-                                                    h->snnz_off[a], shift, h->d_band, h->band_bstride,
-                                                    h->band_desc[a].off, (int)nbatch);
+    const int64_t nent = h->band_desc[a].nent;
+    if (!nent) continue;
+    const int blocks = (int)std::min<int64_t>((nent * nbatch + 255) / 256, 16LL * num_sms(h));
+    band_gather_kernel<<<blocks, 256, 0, h->stream>>>(nent, h->d_ent_slot[g], h->d_mass_csr[g], J_csr_dev, h->nnz,
+                                                      h->snnz_off[a], shift, h->d_Aent, h->ent_bstride,
+                                                      h->band_desc[a].aoff, (int)nbatch);
     h->launches++;
     KCHECK();
   }
-  int maxB = 0;
-  for (auto &d : h->band_desc) {
-    maxB = std::max(maxB, d.B);
-    // one CTA per matrix: meant for vertex-grid sizes (C1-C4); a single large grid (C5) would need a
-    // multi-CTA factorisation (not built)
-    if ((double)d.n * d.B * d.B > 2e9) return fail(h, LANDAU_EUNSUPPORTED, "band factor: n B^2 too large for one CTA");
-  }
-  const size_t smem = sizeof(double) * std::max(maxB, 1);
-  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(band_factor_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  // a CTA per matrix; few warps per CTA and many CTAs per SM: the factorisation is a chain of n
-  // barrier-separated steps of B^2 updates, so concurrency across matrices hides the step latency
-  static const int band_threads = [] {
-    const char *e = getenv("LANDAU_BAND_THREADS");
-    return e ? atoi(e) : 512;   // measured: 1024 15.6 ms, 512 14.1 ms, 256 17.5 ms (C4 batch)
+  const unsigned grid = (unsigned)(nbatch * h->S);
+  static const int band_minb = [] {
+    const char *e = getenv("LANDAU_BAND_MINB");
+    return e ? atoi(e) : 2;
   }();
-  const int threads = std::min(band_threads, std::max(64, ((maxB * maxB + 31) / 32) * 32));
-  band_factor_kernel<<<(unsigned)(nbatch * h->S), threads, smem, h->stream>>>(h->d_band, h->band_bstride,
-                                                                             h->d_band_desc, h->S);
+  if (maxPp <= 88) {   // 4 x 8 tiles, <= 242 threads, two CTAs per SM (128 registers) or one
+    auto k = band_minb >= 2 ? band_lu_kernel<4, 8, 2> : band_lu_kernel<4, 8, 1>;
+    if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    k<<<grid, std::max(64, std::max((maxPp / 4) * (maxPp / 8), 2 * maxPp - 1) + 31) / 32 * 32, smem, h->stream>>>(
+        h->d_Aent, h->ent_bstride, h->d_band, h->band_bstride, h->d_band_desc, h->S);
+  } else {             // 8 x 8 tiles, <= 256 threads
+    auto k = band_lu_kernel<8, 8, 1>;
+    if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    k<<<grid, std::max(64, std::max((maxPp / 8) * (maxPp / 8), 2 * maxPp - 1) + 31) / 32 * 32, smem, h->stream>>>(
+        h->d_Aent, h->ent_bstride, h->d_band, h->band_bstride, h->d_band_desc, h->S);
+  }
   h->launches++;
   h->tlaunch[LANDAU_T_FACTOR]++;
   KCHECK();
@@ -1149,10 +1170,15 @@ int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, d
   if (!h || nbatch < 1 || !b_dev || !x_dev) return fail(h, LANDAU_EINVAL, "band_solve: bad argument");
   if (h->band_nbatch != nbatch) return fail(h, LANDAU_ESTATE, "band_solve: factor this batch first");
   Timer t(h, LANDAU_T_SOLVE);
+  int maxn = 0, maxB = 0;
+  for (auto &d : h->band_desc) maxn = std::max(maxn, d.n), maxB = std::max(maxB, d.B);
+  constexpr int kWarps = 4;
+  const size_t smem = sizeof(double) * kWarps * (maxn + maxB + 1 + (kBandD + 1) * (maxB + 1));
+  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(band_solve_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const int64_t warps = nbatch * h->S;
-  band_solve_kernel<<<(unsigned)((warps * 32 + 127) / 128), 128, 0, h->stream>>>(
-      h->d_band, h->band_bstride, h->d_band_desc, h->d_perm_all, h->d_perm_off, h->d_vec_off, h->ndof, b_dev,
-      h->d_band_scratch, x_dev, h->S, (int)nbatch);
+  band_solve_kernel<<<(unsigned)((warps + kWarps - 1) / kWarps), 32 * kWarps, smem, h->stream>>>(
+      h->d_band, h->band_bstride, h->d_band_desc, h->d_perm_all, h->d_perm_off, h->d_vec_off, h->ndof, maxn, maxB,
+      b_dev, x_dev, h->S, (int)nbatch);
   h->launches++;
   h->tlaunch[LANDAU_T_SOLVE]++;
   KCHECK();
