@@ -424,7 +424,7 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
         std::sort(ent.begin(), ent.end());
         for (auto &e : ent) {
           if (e.second < 0) return "band: CSR pattern is not symmetric";
-          G.ent_pos.push_back((uint16_t)e.first);
+          G.ent_pos.push_back((uint16_t)((ni % 8) * (2 * Bp + 1) + e.first));
           G.ent_slot.push_back(e.second);
         }
         G.ent_max = std::max(G.ent_max, (int)ent.size());

@@ -39,7 +39,8 @@ struct GridPlan {
   // Entries in the order the register-window factorisation consumes them, relative to the padded
   // half-bandwidth Bp = (B + 1 rounded up to 8) - 1: RCM row i "enters" with its lower row part
   // A(i, j), j <= i (pos = j - i + Bp in 0..Bp) and its upper column part A(j, i), j < i
-  // (pos = Bp + 1 + j - i + Bp in Bp+1..2Bp).  ent_slot = CSR slot of the entry.
+  // (pos = Bp + 1 + j - i + Bp in Bp+1..2Bp).  ent_slot = CSR slot of the entry; ent_pos stores
+  // (i mod 8) (2 Bp + 1) + pos, the entry's place in the dense buffer of its group of 8 rows.
   int band_p = 0;
   std::vector<int32_t> ent_ptr;          // [ndof+1]
   std::vector<int32_t> ent_slot;         // [nnz]

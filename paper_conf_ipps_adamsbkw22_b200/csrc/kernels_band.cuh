@@ -45,16 +45,16 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
 
-// band_lu_kernel, warp 0: issue the entry values of entering row e into ring slot e mod (D+1) (an
-// empty commit group past n keeps one group per step)
-__device__ __forceinline__ void band_issue(int e, int n, const int32_t *sptr, const double *ae, double *ring, int W,
-                                           int lane) {
-  if (e < n) {
-    const int q0 = sptr[e], cnt = sptr[e + 1] - q0;
-    double *dst = ring + (e % (kBandD + 1)) * W;
-    for (int q = lane; q < cnt; q += 32) cp_async8(dst + q, ae + q0 + q);
-  }
-  cp_async_commit();
+constexpr int kBandE = 2;   // entry values per thread and group of 8 entering rows (host-checked)
+
+// 1 / a for a normal pivot: MUFU seed, two Newton steps (correctly rounded to within an ulp)
+__device__ __forceinline__ double rcp_newton(double a) {
+  double y;
+  asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(a));
+  double e = fma(-a, y, 1.0);
+  y = fma(y, e, y);
+  e = fma(-a, y, 1.0);
+  return fma(y, e, y);
 }
 
 // One CTA per (batch item, species block).  The P x P active square (P = B + 1, B the padded
@@ -63,45 +63,61 @@ __device__ __forceinline__ void band_issue(int e, int n, const int32_t *sptr, co
 // row/column i mod P.  Step k (pk = k mod P):
 //   b) the owners of physical row/column pk publish U(k, .), A(., k) and the pivot in shared memory;
 //   c) every thread applies the rank-1 update to its tile (the retiring row/column see zero
-//      multipliers) and threads 0..2B write one value each of the factor row LU[k]; warp 0 stages
-//      the entering row/column e = k + P: its entry values arrive by cp.async kBandD steps ahead and
-//      are scattered into a dense buffer (after the entries of row e - 2 are scattered back to zero);
-//   d) the owners of the retiring physical row/column load the entering one.
-// The step loop is unrolled by 8 (P is a multiple of 8, so pk mod R and pk mod C are compile-time
-// constants in each copy): the owners index their registers statically.  Two barriers per step,
-// FP64 FMAs on register operands, no integer division.  Steps k = -P .. -1 only load the window.
+//      multipliers) and threads 0..2B write one value each of the factor row LU[k];
+//   d) the owners of the retiring physical row/column load the entering row/column k + P from a
+//      dense buffer.
+// Steps run in groups of 8 (P is a multiple of 8, so pk mod R and pk mod C are compile-time constants
+// in each unrolled copy and the owners index their registers statically).  The 8 rows entering in
+// group g are staged in bulk, once per group: their entry values (contiguous in Aent) are loaded
+// into registers two groups ahead, scattered into dense buffer set g mod 3 at the first step of
+// group g - 1, and scattered back to zero at the first step of group g + 2.  One barrier per step,
+// FP64 FMAs on register operands, no integer division.  Groups of steps k < 0 only load the window.
 template <int kBandR, int kBandC, int MINB>
 __global__ void __launch_bounds__(256, MINB) band_lu_kernel(const double *__restrict__ Aent, int64_t ent_bstride,
                                                         double *__restrict__ LU, int64_t lu_bstride,
                                                         const BandDesc *__restrict__ desc, int nsp) {
-  static_assert(8 % kBandR == 0 || kBandR % 8 == 0, "tile rows divide or are divided by the unroll");
-  static_assert(kBandC == 8, "tile columns = the unroll");
+  static_assert(8 % kBandR == 0 || kBandR % 8 == 0, "tile rows divide or are divided by the group");
+  static_assert(kBandC == 8, "tile columns = the group");
   extern __shared__ double smem[];
   const int bi = blockIdx.x / nsp, a = blockIdx.x % nsp;
   const BandDesc d = desc[a];
   const int n = d.n, B = d.B, P = B + 1, W = 2 * B + 1;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int tid = threadIdx.x, T = blockDim.x;
   const int ntc = P / kBandC;
   const int tr = tid / ntc, tc = tid % ntc;
   const bool owner = tr < P / kBandR;
   const int pr0 = tr * kBandR, pc0 = tc * kBandC;
   // shared layout
-  double *a_s = smem;                       // [P]  column k (raw); the retiring entry is zero
-  double *u_s = a_s + P;                    // [P]  row k
-  double *piv_s = u_s + P;                  // [2]  pivot, 1 / pivot
-  double *dbuf = piv_s + 2;                 // [2][W] entering row (dense)
-  double *ring = dbuf + 2 * W;              // [kBandD + 1][W] entry values in flight
-  int32_t *sptr = (int32_t *)(ring + (kBandD + 1) * W);   // [n + 1]
+  // a_s / u_s / piv_s are double-buffered by step parity: a step needs one barrier only
+  double *a_s0 = smem;                      // [2][P]  column k (raw); the retiring entry is zero
+  double *u_s0 = a_s0 + 2 * P;              // [2][P]  row k
+  double *piv_s0 = u_s0 + 2 * P;            // [2][2]  pivot, 1 / pivot
+  double *dbuf = piv_s0 + 4;                // [3][8][W] entering rows (dense), one set per group
+  int32_t *sptr = (int32_t *)(dbuf + 24 * W);              // [n + 1]
   uint16_t *spos = (uint16_t *)(sptr + n + 1);             // [nent]
-  for (int i = tid; i < 2 * P; i += blockDim.x) a_s[i] = 0.0;
-  for (int i = tid; i < 2 * W; i += blockDim.x) dbuf[i] = 0.0;
-  for (int i = tid; i <= n; i += blockDim.x) sptr[i] = d.ent_ptr[i];
-  for (int i = tid; i < d.nent; i += blockDim.x) spos[i] = d.ent_pos[i];
+  for (int i = tid; i < 4 * P; i += T) a_s0[i] = 0.0;
+  for (int i = tid; i < 24 * W; i += T) dbuf[i] = 0.0;
+  for (int i = tid; i <= n; i += T) sptr[i] = d.ent_ptr[i];
+  for (int i = tid; i < d.nent; i += T) spos[i] = d.ent_pos[i];
   const double *ae = Aent + (int64_t)bi * ent_bstride + d.aoff;
   double *lu = LU + (int64_t)bi * lu_bstride + d.off;
+  const int ngroups = (n + 7) / 8;
+  auto grange = [&](int g, int &q0, int &q1) {   // entry range of the rows entering in group g
+    q0 = g < ngroups ? sptr[8 * g] : 0;
+    q1 = g < ngroups ? sptr[min(8 * g + 8, n)] : 0;
+  };
+  double vin[kBandE];   // entry values of group g + 1 (loaded one group ahead of their scatter)
   __syncthreads();
-  if (warp == 0)
-    for (int e = 0; e < kBandD; e++) band_issue(e, n, sptr, ae, ring, W, lane);
+  {   // prologue: group 0 scattered into set 0, group 1 loaded
+    int q0, q1;
+    grange(0, q0, q1);
+#pragma unroll
+    for (int m = 0; m < kBandE; m++)
+      if (q0 + tid + m * T < q1) dbuf[spos[q0 + tid + m * T]] = ae[q0 + tid + m * T];
+    grange(1, q0, q1);
+#pragma unroll
+    for (int m = 0; m < kBandE; m++) vin[m] = q0 + tid + m * T < q1 ? ae[q0 + tid + m * T] : 0.0;
+  }
   double cell[kBandR][kBandC];
 #pragma unroll
   for (int r = 0; r < kBandR; r++)
@@ -111,8 +127,9 @@ __global__ void __launch_bounds__(256, MINB) band_lu_kernel(const double *__rest
   // an L entry (physical row pk + t - B), both modulo P by one conditional subtraction
   const int tw = tid < W ? (tid <= B ? tid : tid - B) : 0;
 
-  int pkb = 0;   // (k mod P) of the first step of the unrolled group
-  for (int kb = -P; kb < n; kb += 8) {
+  int pkb = 0;   // (k mod P) of the group's first step
+  for (int kb = -P, g = 0; kb < n; kb += 8, g++) {
+    const double *dset = dbuf + (g % 3) * 8 * W;   // this group's entering rows
 #pragma unroll
     for (int u = 0; u < 8; u++) {
       const int k = kb + u, pk = pkb + u;
@@ -120,13 +137,22 @@ __global__ void __launch_bounds__(256, MINB) band_lu_kernel(const double *__rest
       const bool rowown = owner && tr == (pkb + u - rr) / kBandR;
       const bool colown = owner && tc == pkb / kBandC;
       const bool live = k >= 0 && k < n;
+      double *a_s = a_s0 + (u & 1) * P, *u_s = u_s0 + (u & 1) * P, *piv_s = piv_s0 + (u & 1) * 2;
+      if (u == 0 && g >= 2) {   // clear group g - 2's rows from set (g + 1) mod 3
+        int q0, q1;
+        grange(g - 2, q0, q1);
+        double *ds = dbuf + ((g + 1) % 3) * 8 * W;
+#pragma unroll
+        for (int m = 0; m < kBandE; m++)
+          if (q0 + tid + m * T < q1) ds[spos[q0 + tid + m * T]] = 0.0;
+      }
       if (live) {   // b) publish the pivot row and column
         if (rowown) {
 #pragma unroll
           for (int c = 0; c < kBandC; c++) u_s[pc0 + c] = (colown && c == cc) ? 0.0 : cell[rr][c];
           if (colown) {
             piv_s[0] = cell[rr][cc];
-            piv_s[1] = __drcp_rn(cell[rr][cc]);
+            piv_s[1] = rcp_newton(cell[rr][cc]);
           }
         }
         if (colown) {
@@ -135,28 +161,36 @@ __global__ void __launch_bounds__(256, MINB) band_lu_kernel(const double *__rest
         }
       }
       __syncthreads();
-      const int e = k + P;   // entering row
-      double *db = dbuf + (e & 1) * W;
-      if (warp == 0) {   // stage the entering row: clear row e - 2's entries, wait for row e's, scatter
-        if (e >= 2 && e - 2 < n)
-          for (int q = sptr[e - 2] + lane; q < sptr[e - 1]; q += 32) db[spos[q]] = 0.0;
-        band_issue(e + kBandD, n, sptr, ae, ring, W, lane);
-        cp_async_wait<kBandD>();
-        __syncwarp();
-        if (e < n) {
-          const int q0 = sptr[e], cnt = sptr[e + 1] - q0;
-          const double *src = ring + (e % (kBandD + 1)) * W;
-          for (int q = lane; q < cnt; q += 32) db[spos[q0 + q]] = src[q];
-        }
+      if (u == 0) {   // scatter group g + 1 into set (g + 1) mod 3; load group g + 2
+        int q0, q1;
+        grange(g + 1, q0, q1);
+        double *ds = dbuf + ((g + 1) % 3) * 8 * W;
+#pragma unroll
+        for (int m = 0; m < kBandE; m++)
+          if (q0 + tid + m * T < q1) ds[spos[q0 + tid + m * T]] = vin[m];
+        grange(g + 2, q0, q1);
+#pragma unroll
+        for (int m = 0; m < kBandE; m++) vin[m] = q0 + tid + m * T < q1 ? ae[q0 + tid + m * T] : 0.0;
       }
       if (live) {   // c) rank-1 update of the tile; threads 0..2B write step k's factor row
         const double rinv = piv_s[1];
         if (owner) {
           double l[kBandR], uu[kBandC];
+          // 16-byte loads: pr0, pc0 and P are multiples of 4
+          const double2 *a2 = reinterpret_cast<const double2 *>(a_s + pr0);
+          const double2 *u2 = reinterpret_cast<const double2 *>(u_s + pc0);
 #pragma unroll
-          for (int r = 0; r < kBandR; r++) l[r] = a_s[pr0 + r] * rinv;
+          for (int r = 0; r < kBandR / 2; r++) {
+            const double2 v = a2[r];
+            l[2 * r] = v.x * rinv;
+            l[2 * r + 1] = v.y * rinv;
+          }
 #pragma unroll
-          for (int c = 0; c < kBandC; c++) uu[c] = u_s[pc0 + c];
+          for (int c = 0; c < kBandC / 2; c++) {
+            const double2 v = u2[c];
+            uu[2 * c] = v.x;
+            uu[2 * c + 1] = v.y;
+          }
 #pragma unroll
           for (int r = 0; r < kBandR; r++)
 #pragma unroll
@@ -168,9 +202,11 @@ __global__ void __launch_bounds__(256, MINB) band_lu_kernel(const double *__rest
           lu[(int64_t)k * W + tid] = tid == 0 ? piv_s[0] : tid <= B ? u_s[j] : a_s[j] * rinv;
         }
       }
-      __syncthreads();
-      // d) the retiring physical row/column pk takes the entering row/column e = k + P; offset 0 of
-      //    the entering row is logical index k + 1, i.e. physical pk + 1 (mod P)
+      // (no barrier: the next step publishes into the other a_s / u_s buffer, and phase d only
+      // touches the owners' own registers)
+      // d) the retiring physical row/column pk takes the entering row/column k + P (row u of the
+      //    group's set); offset 0 of the entering row is logical k + 1, i.e. physical pk + 1 (mod P)
+      const double *db = dset + u * W;
       const int pk1 = pk + 1 == P ? 0 : pk + 1;
       if (colown) {
         int o = pr0 - pk1;   // offset of physical row pr0 in the entering column

@@ -765,7 +765,8 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
           {off, aoff, h->d_ent_ptr[g], h->d_ent_pos[g], G.ndof, G.band_p, G.band_p + 1, (int)G.ent_slot.size()});
       off += (int64_t)G.ndof * (2 * G.band_p + 1);
       aoff += (int64_t)G.ent_slot.size();
-      h->band_ent_max = std::max(h->band_ent_max, G.ent_max);
+      for (int r = 0; r < G.ndof; r += 8)   // entries of one group of 8 entering rows (kernels_band.cuh)
+        h->band_ent_max = std::max(h->band_ent_max, G.ent_ptr[std::min(r + 8, G.ndof)] - G.ent_ptr[r]);
       perm_off.push_back((int64_t)perm_all.size());
       perm_all.insert(perm_all.end(), G.rcm_perm.begin(), G.rcm_perm.end());
       vec_off.push_back(h->soff[a]);
@@ -1119,8 +1120,7 @@ int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const d
   // grid (C5) would need a multi-CTA factorisation (not built)
   if (maxPp > kBandMaxP) return fail(h, LANDAU_EUNSUPPORTED, "band factor: half-bandwidth above 127");
   const int W = 2 * (maxPp - 1) + 1;
-  const size_t smem = sizeof(double) * (2 * maxPp + 2 + 2 * W + (kBandD + 1) * W) + sizeof(int32_t) * (maxn + 1) +
-                      sizeof(uint16_t) * maxent;
+  const size_t smem = sizeof(double) * (4 * maxPp + 4 + 24 * W) + sizeof(int32_t) * (maxn + 1) + sizeof(uint16_t) * maxent;
   if (smem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
   if (nbatch > h->band_cap) {
     cudaFree(h->d_band);
@@ -1142,6 +1142,8 @@ int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const d
     h->launches++;
     KCHECK();
   }
+  const int threads_lu = std::max(64, (std::max((maxPp / (maxPp <= 88 ? 4 : 8)) * (maxPp / 8), 2 * maxPp - 1) + 31) / 32 * 32);
+  if (h->band_ent_max > kBandE * threads_lu) return fail(h, LANDAU_EUNSUPPORTED, "band factor: too many entries per row group");
   const unsigned grid = (unsigned)(nbatch * h->S);
   static const int band_minb = [] {
     const char *e = getenv("LANDAU_BAND_MINB");
@@ -1150,12 +1152,12 @@ int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const d
   if (maxPp <= 88) {   // 4 x 8 tiles, <= 242 threads, two CTAs per SM (128 registers) or one
     auto k = band_minb >= 2 ? band_lu_kernel<4, 8, 2> : band_lu_kernel<4, 8, 1>;
     if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    k<<<grid, std::max(64, std::max((maxPp / 4) * (maxPp / 8), 2 * maxPp - 1) + 31) / 32 * 32, smem, h->stream>>>(
+    k<<<grid, threads_lu, smem, h->stream>>>(
         h->d_Aent, h->ent_bstride, h->d_band, h->band_bstride, h->d_band_desc, h->S);
   } else {             // 8 x 8 tiles, <= 256 threads
     auto k = band_lu_kernel<8, 8, 1>;
     if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    k<<<grid, std::max(64, std::max((maxPp / 8) * (maxPp / 8), 2 * maxPp - 1) + 31) / 32 * 32, smem, h->stream>>>(
+    k<<<grid, threads_lu, smem, h->stream>>>(
         h->d_Aent, h->ent_bstride, h->d_band, h->band_bstride, h->d_band_desc, h->S);
   }
   h->launches++;
