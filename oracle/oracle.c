@@ -929,8 +929,10 @@ void oracle_jacobian_coo(const oracle_t *o, const double *f, const unsigned char
   jacobian_driver(o, f, mask, vals, absvals, 1);
 }
 
-/* O9: mass */
-static void mass_driver(const oracle_t *o, double shift, double *vals, int coo) {
+/* O9: mass, sum_q w phi_k phi_l (kind 0); O11: E_z advection, sum_q w phi_k d_z phi_l (kind 1) --
+ * the element matrix of Eq. 4's (0, e E_z / m) . grad f term tested with psi = phi_k, before the
+ * species factor e_a E_z / m_a (@8216-8654; same w = w_hat detJ r as the mass, Amb-2) */
+static void mass_driver(const oracle_t *o, double shift, double *vals, int coo, int kind) {
   int nqp = o->nqp, nb = o->nb;
   if (!coo)
     for (long long k = 0; k < o->nnz; k++) vals[k] = 0.0;
@@ -940,11 +942,13 @@ static void mass_driver(const oracle_t *o, double shift, double *vals, int coo) 
     long long coff = o->scoo_off[a];
     for (int c = 0; c < g->ncell; c++) {
       int n = g->ne[c];
+      ld s = 2.0L / (ld)g->h[c];
       ld *M = calloc((size_t)nb * nb, sizeof(ld));
       for (int q = 0; q < nqp; q++) {
         ld w = o->pw[g->pt0 + (long long)c * nqp + q];
         for (int k = 0; k < nb; k++)
-          for (int l = 0; l < nb; l++) M[k * nb + l] += w * o->phi[q * nb + k] * o->phi[q * nb + l];
+          for (int l = 0; l < nb; l++)
+            M[k * nb + l] += w * o->phi[q * nb + k] * (kind == 0 ? o->phi[q * nb + l] : s * o->deta[q * nb + l]);
       }
       ld *X = calloc((size_t)n * n * 2, sizeof(ld));
       expand(o, g, c, M, M, X, X + n * n);
@@ -964,8 +968,10 @@ static void mass_driver(const oracle_t *o, double shift, double *vals, int coo) 
     }
   }
 }
-void oracle_mass(const oracle_t *o, double shift, double *vals) { mass_driver(o, shift, vals, 0); }
-void oracle_mass_coo(const oracle_t *o, double shift, double *vals) { mass_driver(o, shift, vals, 1); }
+void oracle_mass(const oracle_t *o, double shift, double *vals) { mass_driver(o, shift, vals, 0, 0); }
+void oracle_mass_coo(const oracle_t *o, double shift, double *vals) { mass_driver(o, shift, vals, 1, 0); }
+void oracle_advection(const oracle_t *o, double *vals) { mass_driver(o, 1.0, vals, 0, 1); }
+void oracle_advection_coo(const oracle_t *o, double *vals) { mass_driver(o, 1.0, vals, 1, 1); }
 
 void oracle_set_threads(int n) {
 #ifdef _OPENMP

@@ -20,6 +20,7 @@
  *       @8833-9206);  O8 assembly J_a = sum_e P_e^T C_e P_e, species-block-diagonal (@11277)
  *   O9  mass matrix shift * sum_e P_e^T (sum_q w phi phi) P_e (@39757-39999)
  *   O10 condition scale: the same assembly with every product replaced by its absolute value.
+ *   O11 E_z advection matrix sum_e P_e^T (sum_q w phi_k d_z phi_l) P_e (Eq. 4, @8216-8654)
  * Pins: see tests/test_oracle_*.py (P1-P9 of SURVEY.md §8(c)).
  */
 #ifndef LANDAU_ORACLE_H
@@ -76,6 +77,10 @@ void oracle_jacobian_coo(const oracle_t *o, const double *f, const unsigned char
 /* O9: CSR values [nnz] of shift * M for every species block */
 void oracle_mass(const oracle_t *o, double shift, double *vals);
 void oracle_mass_coo(const oracle_t *o, double shift, double *vals);
+/* O11: CSR / COO values of the unscaled E_z advection matrix sum_e P_e^T (sum_q w phi_k d_z phi_l) P_e
+ * for every species block (the caller applies e_a E_z / m_a; Eq. 4 @8216-8654) */
+void oracle_advection(const oracle_t *o, double *vals);
+void oracle_advection_coo(const oracle_t *o, double *vals);
 
 void oracle_set_threads(int n);
 int oracle_get_threads(void);

@@ -56,6 +56,8 @@ def lib():
         L.oracle_jacobian_coo.argtypes = [vp, _d, vp, _d, _d]
         L.oracle_mass.argtypes = [vp, C.c_double, _d]
         L.oracle_mass_coo.argtypes = [vp, C.c_double, _d]
+        L.oracle_advection.argtypes = [vp, _d]
+        L.oracle_advection_coo.argtypes = [vp, _d]
         L.oracle_set_threads.argtypes = [C.c_int]
         L.oracle_get_threads.restype = C.c_int
         _LIB = L
@@ -176,6 +178,47 @@ class Oracle:
         v = np.zeros(max(self.ncoo, 1))
         lib().oracle_mass_coo(self._h, float(shift), v)
         return v[: self.ncoo]
+
+    def advection(self):
+        """O11: unscaled E_z advection matrix (CSR values, every species block)."""
+        v = np.zeros(max(self.nnz, 1))
+        lib().oracle_advection(self._h, v)
+        return v[: self.nnz]
+
+    def advection_coo(self):
+        v = np.zeros(max(self.ncoo, 1))
+        lib().oracle_advection_coo(self._h, v)
+        return v[: self.ncoo]
+
+    def species_rows(self):
+        """species index of every row of the block-diagonal system (species-major blocks, @11277)"""
+        return np.concatenate([np.full(self.grid_ndof(int(g)), a, dtype=np.int64)
+                               for a, g in enumerate(self.prob.grid_of)])
+
+    def implicit_step(self, f_old, dt, Ez=0.0, iters=4):
+        """Backward-Euler step of Eq. 4 (no source) by the paper's quasi-Newton iteration (@10500-10978):
+        with the Jacobian J(f^k) recomputed about the current iterate,
+            (M/dt + E_z (e_a/m_a) A_E - J(f^k)) f^{k+1} = M f^old / dt,
+        i.e. Newton on F(f) = M (f - f^old)/dt + E_z (e/m) A_E f - C(f) with the approximate Jacobian
+        M/dt + E_z (e/m) A_E - J(f^k) (C(f^k) = J(f^k) f^k, Amb-4).  A sparse direct solve (a library
+        primitive) stands in for the paper's band LU.  Returns the iterates f^1..f^iters."""
+        import scipy.sparse as sps
+        import scipy.sparse.linalg as spla
+        rp, col = self.pattern()
+        n = self.ndof
+        M, Ae = self.mass(1.0), self.advection()
+        rows = np.repeat(np.arange(n), np.diff(rp))
+        eta = Ez * (np.asarray(self.prob.charge, float) / np.asarray(self.prob.mass, float))[self.species_rows()]
+        Mm = sps.csr_matrix((M, col, rp), shape=(n, n))
+        b = Mm @ np.asarray(f_old, float) / dt
+        f = np.array(f_old, dtype=np.float64)
+        out = []
+        for _ in range(iters):
+            J, _ = self.jacobian(f)
+            A = sps.csr_matrix((M / dt + eta[rows] * Ae - J, col, rp), shape=(n, n))
+            f = spla.spsolve(A.tocsc(), b)
+            out.append(f.copy())
+        return out
 
     def coefficients(self, with_noise=True):
         from paper_conf_ipps_adamsbkw22_b200 import inputs
