@@ -185,6 +185,29 @@ int landau_set_tensor_cache(landau_t h, int32_t enable);
 int landau_band_info(landau_t h, int32_t grid, int32_t *bandwidth, int32_t *perm);
 int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const double *J_csr_dev);
 int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev);
+/* The same factorisation of A = shift * M + E_z (e_a / m_a) A_E - J per species block a, with A_E the
+ * advection matrix below (the electric-field term of Eq. 4).  Ez = 0 is landau_band_factor_batched. */
+int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, double Ez, const double *J_csr_dev);
+
+/* E_z advection matrix of Eq. 4 (PAPER.md:1@8216-8654): the weak form of (0, e_a E_z / m_a) . grad f_a
+ * tested with psi = phi_k, i.e. per species block E_z (e_a / m_a) sum_e P_e^T (sum_q w phi_k d_z phi_l) P_e
+ * with the mass matrix's w (no 2 pi, Amb-2); charges in e, masses in m0, E_z in the same App.-A units
+ * as time.  values_dev: [nnz_csr] or [ncoo] device buffer (caller-owned); cached at create. */
+int landau_advection(landau_t h, double Ez, double *values_dev, int32_t format);
+
+/* NEXT-3: one backward-Euler step of Eq. 4 without source,
+ *   M (f^{n+1} - f^n) / dt + E_z (e/m) A_E f^{n+1} = C(f^{n+1}),   C(f) = J(f) f (Amb-4),
+ * solved by the paper's quasi-Newton iteration with the Jacobian fully recomputed about each iterate
+ * (PAPER.md:1@10500-10978): (M/dt + E_z (e/m) A_E - J(f^k)) f^{k+1} = M f^n / dt, every item of the
+ * batch independently, entirely on the device (set_state, Jacobian build, band LU, solve per
+ * iteration).  f_old_dev, f_new_dev: [nbatch][ndof] device buffers, distinct (f_new is overwritten;
+ * the iteration starts from f_old).  Stops after max_iter iterations, or earlier once every item's
+ * ||f^{k+1} - f^k|| / ||f^{k+1}|| <= rtol (rtol > 0 reads the norms back once per iteration; rtol <= 0
+ * runs exactly max_iter iterations with one read-back at the end).  iters (host, may be NULL): the
+ * iterations run; dnorm (host, may be NULL): the largest relative change of the last iteration.
+ * The handle's state afterwards is the last iterate f^{k} the final Jacobian was built about. */
+int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
+                                 double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm);
 
 /* How the last build ran (for FLOP accounting and diagnostics). */
 typedef struct {

@@ -25,15 +25,17 @@ struct BandDesc {             // per species block
   int n, B, Pp, nent;         // B: the half-bandwidth padded so that Pp = B + 1 is a multiple of 8
 };
 
-// Aent[b][aoff + e] = shift M[slot e] - J[b][J_off + slot e]: the block's entries in consumption order
+// Aent[b][aoff + e] = shift M[s] + eta A_E[s] - J[b][J_off + s], s = slot of entry e: the block's
+// entries in consumption order (eta = E_z e_a / m_a, the advection term of Eq. 4; 0 without a field)
 __global__ void band_gather_kernel(int64_t nent, const int32_t *__restrict__ ent_slot, const double *__restrict__ M,
-                                   const double *__restrict__ J, int64_t J_bstride, int64_t J_off, double shift,
-                                   double *__restrict__ Aent, int64_t ent_bstride, int64_t aoff, int nbatch) {
+                                   const double *__restrict__ AE, double eta, const double *__restrict__ J,
+                                   int64_t J_bstride, int64_t J_off, double shift, double *__restrict__ Aent,
+                                   int64_t ent_bstride, int64_t aoff, int nbatch) {
   const int64_t total = nent * nbatch;
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
     const int64_t b = k / nent, e = k % nent;
     const int32_t s = ent_slot[e];
-    Aent[b * ent_bstride + aoff + e] = fma(shift, M[s], -J[b * J_bstride + J_off + s]);
+    Aent[b * ent_bstride + aoff + e] = fma(shift, M[s], fma(eta, AE[s], -J[b * J_bstride + J_off + s]));
   }
 }
 

@@ -174,16 +174,24 @@ __global__ void __launch_bounds__(NB * EPB, LANDAU_EL_MINB) element_kernel(int64
 // layout (second half zero) so the same gather maps apply.
 template <int NB>
 __global__ void __launch_bounds__(NB * NB) mass_element_kernel(int64_t ncell, const double *__restrict__ pw,
+                                                                 const double *__restrict__ cell_h,
                                                                  const double *__restrict__ tab, double *__restrict__ Mbuf) {
+  // [cell][0][k][l] = sum_q w phi_k phi_l (mass, a-6); [cell][1][k][l] = sum_q w phi_k d_z phi_l (the
+  // E_z advection term of Eq. 4, @8216-8654, before its species factor e_a E_z / m_a)
   __shared__ double s_phi[NB][NB], s_dxi[NB][NB], s_deta[NB][NB];
   load_tables<NB>(tab, s_phi, s_dxi, s_deta);
   __syncthreads();
   const int64_t e = blockIdx.x;
   const int tid = threadIdx.x, k = tid / NB, l = tid % NB;
-  double m = 0.0;
-  for (int q = 0; q < NB; q++) m = fma(pw[e * NB + q] * s_phi[q][k], s_phi[q][l], m);
+  const double sz = 2.0 / cell_h[e];
+  double m = 0.0, adv = 0.0;
+  for (int q = 0; q < NB; q++) {
+    const double wp = pw[e * NB + q] * s_phi[q][k];
+    m = fma(wp, s_phi[q][l], m);
+    adv = fma(wp, sz * s_deta[q][l], adv);
+  }
   Mbuf[e * 2 * NB * NB + tid] = m;
-  Mbuf[e * 2 * NB * NB + NB * NB + tid] = 0.0;
+  Mbuf[e * 2 * NB * NB + NB * NB + tid] = adv;
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -234,6 +242,7 @@ __global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ C
 }
 
 // mass gather (create time): out[s] = sum_k w_k M[idx_k]
+// (M points at the mass half of the element buffer, or at M + NB^2 for the advection half)
 __global__ void mass_gather_kernel(const int64_t *__restrict__ ptr, const int32_t *__restrict__ idx,
                                    const double *__restrict__ w, int64_t nslots, const double *__restrict__ M,
                                    double *__restrict__ out) {
@@ -242,6 +251,51 @@ __global__ void mass_gather_kernel(const int64_t *__restrict__ ptr, const int32_
   double v = 0.0;
   for (int64_t k = ptr[s]; k < ptr[s + 1]; k++) v = fma(w[k], M[idx[k]], v);
   out[s] = v;
+}
+
+// NEXT-3: y[b][off + i] = scale * sum_q A[q] x[b][off + col[q]] over one species block's CSR rows
+// (one warp per row, lanes over its nonzeros, fixed-order shuffle reduction: deterministic)
+__global__ void block_spmv_kernel(const int64_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                 const double *__restrict__ A, int n, int64_t off, int64_t ndof, double scale,
+                                 const double *__restrict__ x, double *__restrict__ y, int nbatch) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (w >= (int64_t)nbatch * n) return;
+  const int64_t b = w / n;
+  const int i = (int)(w % n);
+  const double *xb = x + b * ndof + off;
+  double s = 0.0;
+  for (int64_t q = rowptr[i] + lane; q < rowptr[i + 1]; q += 32) s = fma(A[q], xb[col[q]], s);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if (lane == 0) y[b * ndof + off + i] = scale * s;
+}
+
+// NEXT-3: per batch item, out[b] = (sum (x - y)^2, sum x^2) in a fixed-order block reduction
+__global__ void __launch_bounds__(256) delta_norm_kernel(const double *__restrict__ x, const double *__restrict__ y,
+                                                         int64_t ndof, double *__restrict__ out) {
+  __shared__ double s_d[256], s_x[256];
+  const int64_t b = blockIdx.x;
+  double d = 0.0, xx = 0.0;
+  for (int64_t i = threadIdx.x; i < ndof; i += 256) {
+    const double xi = x[b * ndof + i], di = xi - y[b * ndof + i];
+    d = fma(di, di, d);
+    xx = fma(xi, xi, xx);
+  }
+  s_d[threadIdx.x] = d;
+  s_x[threadIdx.x] = xx;
+  __syncthreads();
+  for (int o = 128; o > 0; o >>= 1) {
+    if ((int)threadIdx.x < o) {
+      s_d[threadIdx.x] += s_d[threadIdx.x + o];
+      s_x[threadIdx.x] += s_x[threadIdx.x + o];
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    out[2 * b] = s_d[0];
+    out[2 * b + 1] = s_x[0];
+  }
 }
 
 // N5: out[o0 + i] = shift * M[i]

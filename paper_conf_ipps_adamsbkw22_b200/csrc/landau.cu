@@ -61,6 +61,12 @@ struct landau_s {
   };
   std::vector<DevMap> d_csr, d_coo;
   std::vector<double *> d_mass_csr, d_mass_coo;   // per grid
+  std::vector<double *> d_adv_csr, d_adv_coo;     // per grid: unscaled E_z advection matrix (NEXT-3)
+  std::vector<int64_t *> d_rowptr;                // per grid: CSR pattern of one species block
+  std::vector<int32_t *> d_col;
+  // implicit step (NEXT-3) workspace
+  double *d_Jwork = nullptr, *d_rhs = nullptr, *d_norms = nullptr, *h_norms = nullptr;
+  int64_t step_cap = 0;
   // device: state + workspace
   int64_t cap = 0, nbatch = 0, chunk = 1;
   bool have_state = false;
@@ -553,16 +559,17 @@ int build_mass(landau_t h) {
   const Plan &P = h->plan;
   double *Mbuf = nullptr;
   CU(cudaMalloc(&Mbuf, sizeof(double) * P.ncell * 2 * NB * NB));
-  mass_element_kernel<NB><<<(unsigned)P.ncell, NB * NB, 0, h->stream>>>(P.ncell, h->d_w, h->d_tab, Mbuf);
+  mass_element_kernel<NB><<<(unsigned)P.ncell, NB * NB, 0, h->stream>>>(P.ncell, h->d_w, h->d_h, h->d_tab, Mbuf);
   h->launches++;
   KCHECK();
   for (int g = 0; g < P.ngrids; g++) {
-    for (int f = 0; f < 2; f++) {
-      const auto &m = f == 0 ? h->d_csr[g] : h->d_coo[g];
-      double *&dst = f == 0 ? h->d_mass_csr[g] : h->d_mass_coo[g];
+    for (int f = 0; f < 4; f++) {   // mass CSR, mass COO, advection CSR, advection COO
+      const auto &m = f % 2 == 0 ? h->d_csr[g] : h->d_coo[g];
+      double *&dst = f == 0 ? h->d_mass_csr[g] : f == 1 ? h->d_mass_coo[g] : f == 2 ? h->d_adv_csr[g] : h->d_adv_coo[g];
       CU(cudaMalloc(&dst, sizeof(double) * std::max<int64_t>(m.nslots, 1)));
       if (m.nslots == 0) continue;
-      mass_gather_kernel<<<(unsigned)((m.nslots + 255) / 256), 256, 0, h->stream>>>(m.ptr, m.idx, m.w, m.nslots, Mbuf, dst);
+      mass_gather_kernel<<<(unsigned)((m.nslots + 255) / 256), 256, 0, h->stream>>>(m.ptr, m.idx, m.w, m.nslots,
+                                                                                    Mbuf + (f < 2 ? 0 : NB * NB), dst);
       h->launches++;
       KCHECK();
     }
@@ -781,6 +788,14 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
   h->d_coo.resize(P.ngrids);
   h->d_mass_csr.assign(P.ngrids, nullptr);
   h->d_mass_coo.assign(P.ngrids, nullptr);
+  h->d_adv_csr.assign(P.ngrids, nullptr);
+  h->d_adv_coo.assign(P.ngrids, nullptr);
+  h->d_rowptr.assign(P.ngrids, nullptr);
+  h->d_col.assign(P.ngrids, nullptr);
+  for (int g = 0; g < P.ngrids; g++) {
+    std::vector<int32_t> col(P.grids[g].col.begin(), P.grids[g].col.end());
+    if ((rc = upload(h, &h->d_rowptr[g], P.grids[g].rowptr)) || (rc = upload(h, &h->d_col[g], col))) return bail(rc);
+  }
   for (int g = 0; g < P.ngrids; g++) {
     for (int f = 0; f < 2; f++) {
       const GatherMap &m = f == 0 ? P.csr_map[g] : P.coo_map[g];
@@ -848,6 +863,14 @@ void landau_destroy(landau_t h) {
     }
   for (double *p : h->d_mass_csr) cudaFree(p);
   for (double *p : h->d_mass_coo) cudaFree(p);
+  for (double *p : h->d_adv_csr) cudaFree(p);
+  for (double *p : h->d_adv_coo) cudaFree(p);
+  for (int64_t *p : h->d_rowptr) cudaFree(p);
+  for (int32_t *p : h->d_col) cudaFree(p);
+  cudaFree(h->d_Jwork);
+  cudaFree(h->d_rhs);
+  cudaFree(h->d_norms);
+  if (h->h_norms) cudaFreeHost(h->h_norms);
   for (auto &u : h->ev_used) {
     cudaEventDestroy(u.second.first);
     cudaEventDestroy(u.second.second);
@@ -1022,6 +1045,25 @@ int landau_mass(landau_t h, double shift, double *values_dev, int32_t format) {
   return LANDAU_OK;
 }
 
+int landau_advection(landau_t h, double Ez, double *values_dev, int32_t format) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "advection: bad argument");
+  Timer t(h, LANDAU_T_MASS);
+  for (int a = 0; a < h->S; a++) {
+    const int g = h->sgrid[a];
+    const double *A = format == LANDAU_CSR ? h->d_adv_csr[g] : h->d_adv_coo[g];
+    const int64_t n = format == LANDAU_CSR ? (int64_t)h->plan.grids[g].col.size() : h->plan.grids[g].ncoo;
+    const int64_t off = format == LANDAU_CSR ? h->snnz_off[a] : h->scoo_off[a];
+    if (n == 0) continue;
+    const int blocks = (int)std::min<int64_t>((n + 255) / 256, 8LL * num_sms(h));
+    scale_copy_kernel<<<blocks, 256, 0, h->stream>>>(A, Ez * h->charge[a] / h->mass[a], n, values_dev + off);
+    h->launches++;
+    h->tlaunch[LANDAU_T_MASS]++;
+    KCHECK();
+  }
+  return LANDAU_OK;
+}
+
 int landau_point_coeffs_batched(landau_t h, int64_t nbatch, double *G_dev) {
   if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
   if (!h || !G_dev) return fail(h, LANDAU_EINVAL, "point_coeffs: bad argument");
@@ -1108,6 +1150,10 @@ int landau_band_info(landau_t h, int32_t grid, int32_t *bandwidth, int32_t *perm
 }
 
 int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const double *J_csr_dev) {
+  return landau_band_factor_field_batched(h, nbatch, shift, 0.0, J_csr_dev);
+}
+
+int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, double Ez, const double *J_csr_dev) {
   if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
   if (!h || nbatch < 1 || !J_csr_dev) return fail(h, LANDAU_EINVAL, "band_factor: bad argument");
   int maxPp = 8, maxn = 0, maxent = 0;
@@ -1136,7 +1182,8 @@ int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const d
     const int64_t nent = h->band_desc[a].nent;
     if (!nent) continue;
     const int blocks = (int)std::min<int64_t>((nent * nbatch + 255) / 256, 16LL * num_sms(h));
-    band_gather_kernel<<<blocks, 256, 0, h->stream>>>(nent, h->d_ent_slot[g], h->d_mass_csr[g], J_csr_dev, h->nnz,
+    band_gather_kernel<<<blocks, 256, 0, h->stream>>>(nent, h->d_ent_slot[g], h->d_mass_csr[g], h->d_adv_csr[g],
+                                                      Ez * h->charge[a] / h->mass[a], J_csr_dev, h->nnz,
                                                       h->snnz_off[a], shift, h->d_Aent, h->ent_bstride,
                                                       h->band_desc[a].aoff, (int)nbatch);
     h->launches++;
@@ -1184,6 +1231,63 @@ int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, d
   h->launches++;
   h->tlaunch[LANDAU_T_SOLVE]++;
   KCHECK();
+  return LANDAU_OK;
+}
+
+int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
+                                 double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm) {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !f_old_dev || !f_new_dev || f_old_dev == f_new_dev || max_iter < 1 || !(dt > 0))
+    return fail(h, LANDAU_EINVAL, "implicit_step: bad argument");
+  if (nbatch > h->step_cap) {
+    cudaFree(h->d_Jwork);
+    cudaFree(h->d_rhs);
+    cudaFree(h->d_norms);
+    if (h->h_norms) cudaFreeHost(h->h_norms);
+    h->d_Jwork = h->d_rhs = h->d_norms = h->h_norms = nullptr;
+    CU(cudaMalloc(&h->d_Jwork, sizeof(double) * nbatch * std::max<int64_t>(h->nnz, 1)));
+    CU(cudaMalloc(&h->d_rhs, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
+    CU(cudaMalloc(&h->d_norms, sizeof(double) * 2 * nbatch));
+    CU(cudaMallocHost(&h->h_norms, sizeof(double) * 2 * nbatch));
+    h->step_cap = nbatch;
+  }
+  // rhs = M f_old / dt (species blocks), initial iterate f_old
+  for (int a = 0; a < h->S; a++) {
+    const int g = h->sgrid[a];
+    const int n = h->plan.grids[g].ndof;
+    if (!n) continue;
+    const int64_t warps = nbatch * n;
+    block_spmv_kernel<<<(unsigned)((warps * 32 + 255) / 256), 256, 0, h->stream>>>(
+        h->d_rowptr[g], h->d_col[g], h->d_mass_csr[g], n, h->soff[a], h->ndof, 1.0 / dt, f_old_dev, h->d_rhs,
+        (int)nbatch);
+    h->launches++;
+    KCHECK();
+  }
+  CU(cudaMemcpyAsync(f_new_dev, f_old_dev, sizeof(double) * nbatch * h->ndof, cudaMemcpyDeviceToDevice, h->stream));
+  int it = 0;
+  double worst = 0.0;
+  for (it = 1; it <= max_iter; it++) {
+    // quasi-Newton iteration (@10500-10978): J about the current iterate, then
+    // (M/dt + E_z (e/m) A_E - J(f^k)) f^{k+1} = M f_old / dt  by the band LU
+    int rc = landau_set_state_batched(h, nbatch, f_new_dev);
+    if (!rc) rc = dispatch_build(h, nbatch, h->d_Jwork, LANDAU_CSR);
+    if (!rc) rc = landau_band_factor_field_batched(h, nbatch, 1.0 / dt, Ez, h->d_Jwork);
+    if (!rc) rc = landau_band_solve_batched(h, nbatch, h->d_rhs, f_new_dev);
+    if (rc) return rc;
+    delta_norm_kernel<<<(unsigned)nbatch, 256, 0, h->stream>>>(f_new_dev, h->d_f, h->ndof, h->d_norms);
+    h->launches++;
+    KCHECK();
+    if (rtol > 0 || it == max_iter) {
+      CU(cudaMemcpyAsync(h->h_norms, h->d_norms, sizeof(double) * 2 * nbatch, cudaMemcpyDeviceToHost, h->stream));
+      CU(cudaStreamSynchronize(h->stream));
+      worst = 0.0;
+      for (int64_t b = 0; b < nbatch; b++)
+        worst = std::max(worst, std::sqrt(h->h_norms[2 * b] / std::max(h->h_norms[2 * b + 1], 1e-300)));
+      if (rtol > 0 && worst <= rtol) break;
+    }
+  }
+  if (iters) *iters = std::min(it, (int)max_iter);
+  if (dnorm) *dnorm = worst;
   return LANDAU_OK;
 }
 

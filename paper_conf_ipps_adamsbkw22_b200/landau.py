@@ -85,6 +85,9 @@ def lib():
             "landau_band_info": (C.c_int, [vp, i32, P32, P32]),
             "landau_band_factor_batched": (C.c_int, [vp, i64, d, vp]),
             "landau_band_solve_batched": (C.c_int, [vp, i64, vp, vp]),
+            "landau_band_factor_field_batched": (C.c_int, [vp, i64, d, d, vp]),
+            "landau_advection": (C.c_int, [vp, d, vp, i32]),
+            "landau_implicit_step_batched": (C.c_int, [vp, i64, d, d, vp, vp, i32, d, P32, Pd]),
             "landau_strerror": (C.c_char_p, [C.c_int]),
             "landau_last_error": (C.c_char_p, [vp]),
             "landau_version": (C.c_char_p, []),
@@ -283,9 +286,27 @@ class Landau:
                     "landau_band_info")
         return B.value, perm
 
-    def band_factor_batched(self, shift, J):
+    def band_factor_batched(self, shift, J, Ez=0.0):
         nb = J.shape[0] if J.dim() == 2 else 1
-        self._check(lib().landau_band_factor_batched(self._h, nb, float(shift), _tptr(J)), "landau_band_factor_batched")
+        if Ez == 0.0:
+            self._check(lib().landau_band_factor_batched(self._h, nb, float(shift), _tptr(J)),
+                        "landau_band_factor_batched")
+        else:
+            self._check(lib().landau_band_factor_field_batched(self._h, nb, float(shift), float(Ez), _tptr(J)),
+                        "landau_band_factor_field_batched")
+
+    def advection(self, Ez, values, format=LANDAU_CSR):
+        self._check(lib().landau_advection(self._h, float(Ez), _tptr(values), format), "landau_advection")
+        return values
+
+    def implicit_step_batched(self, dt, f_old, f_new, Ez=0.0, max_iter=4, rtol=0.0):
+        """One backward-Euler step by quasi-Newton (include/landau.h); returns (iterations, max rel. change)."""
+        nb = f_old.shape[0] if f_old.dim() == 2 else 1
+        it, dn = C.c_int32(), C.c_double()
+        self._check(lib().landau_implicit_step_batched(self._h, nb, float(dt), float(Ez), _tptr(f_old), _tptr(f_new),
+                                                       int(max_iter), float(rtol), C.byref(it), C.byref(dn)),
+                    "landau_implicit_step_batched")
+        return it.value, dn.value
 
     def band_solve_batched(self, b, x):
         nb = b.shape[0] if b.dim() == 2 else 1

@@ -494,3 +494,101 @@ def test_band_lu_batched_C4():
     b2 = b.clone()
     h.band_solve_batched(b2, b2)
     assert torch.equal(b2, x)
+
+
+# ------------------------------------------------------------------------------------------------
+# NEXT-3: E_z advection matrix and the quasi-Newton implicit step
+# ------------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3"])
+def test_advection_parity(cfg):
+    """A_E (Eq. 4's field term) with its species factor E_z e_a / m_a, CSR and COO, against the oracle."""
+    prob, h, o, fg, fo = setup(cfg)
+    Ez = 0.37
+    eta = Ez * (np.asarray(prob.charge, float) / np.asarray(prob.mass, float))
+    rows = o.species_rows()
+    rp, col = o.pattern()
+    per_entry = eta[np.repeat(rows, np.diff(rp))]
+    ref = per_entry * o.advection()
+    out = torch.full((h.nnz,), float("nan"), dtype=torch.float64, device=DEV)
+    h.advection(Ez, out)
+    torch.cuda.synchronize()
+    assert np.abs(out.cpu().numpy() - ref).max() <= 1e-14 * np.abs(ref).max()
+    row, ccol = o.coo_pattern()
+    refc = eta[rows[row]] * o.advection_coo()
+    outc = torch.full((h.ncoo,), float("nan"), dtype=torch.float64, device=DEV)
+    h.advection(Ez, outc, L.LANDAU_COO)
+    torch.cuda.synchronize()
+    assert np.abs(outc.cpu().numpy() - refc).max() <= 1e-14 * np.abs(refc).max()
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C3"])
+def test_band_lu_with_field_matches_sparse_direct(cfg):
+    import scipy.sparse as sps
+    import scipy.sparse.linalg as spla
+    prob, h, o, fg, fo = setup(cfg)
+    J = gpu_jacobian(h, fg)
+    Mo, Ao = o.mass(1.0), o.advection()
+    rows = o.species_rows()
+    rp, col = o.pattern()
+    Ez, shift = 0.2, 10.0
+    eta = Ez * (np.asarray(prob.charge, float) / np.asarray(prob.mass, float))[np.repeat(rows, np.diff(rp))]
+    A = sps.csr_matrix((shift * Mo + eta * Ao - J, col, rp), shape=(o.ndof, o.ndof))
+    bvec = np.random.default_rng(3).standard_normal(o.ndof)
+    x_ref = spla.spsolve(A.tocsc(), bvec)
+    h.band_factor_batched(shift, torch.tensor(J, device=DEV).reshape(1, -1), Ez=Ez)
+    x = torch.empty((1, o.ndof), dtype=torch.float64, device=DEV)
+    h.band_solve_batched(torch.tensor(bvec, device=DEV).reshape(1, -1), x)
+    torch.cuda.synchronize()
+    assert np.linalg.norm(x.cpu().numpy()[0] - x_ref) <= 1e-9 * np.linalg.norm(x_ref)
+
+
+@pytest.mark.parametrize("cfg,dt,Ez", [("C1", 0.05, 0.0), ("C1", 0.05, 0.1), ("C3", 0.01, 0.1), ("C2", 0.02, 0.05)])
+def test_implicit_step_matches_oracle_iterates(cfg, dt, Ez):
+    """Every quasi-Newton iterate of the device step equals the oracle's iterate (same iteration count)."""
+    prob, h, o, fg, fo = setup(cfg)
+    its = o.implicit_step(fo, dt, Ez, iters=3)
+    f_old = torch.tensor(fg, device=DEV).reshape(1, -1)
+    f_new = torch.empty_like(f_old)
+    for k in (1, 3):
+        n_it, dn = h.implicit_step_batched(dt, f_old, f_new, Ez=Ez, max_iter=k, rtol=0.0)
+        torch.cuda.synchronize()
+        assert n_it == k
+        x = f_new.cpu().numpy()[0]
+        assert np.linalg.norm(x - its[k - 1]) <= 1e-10 * np.linalg.norm(its[k - 1]), (k, np.linalg.norm(x - its[k - 1]))
+        prev = its[k - 2] if k > 1 else fo
+        assert abs(dn - np.linalg.norm(its[k - 1] - prev) / np.linalg.norm(its[k - 1])) <= 1e-6 * dn
+
+
+def test_implicit_step_converges_and_conserves_C4_batch():
+    """Batched step over vertices with a tolerance: stops when every item's relative change <= rtol;
+    the converged step conserves density, momentum and energy of every vertex (no field)."""
+    import scipy.sparse as sps
+    nb = 4
+    prob0 = inputs.config4_vertex(0)
+    h = L.Landau.from_problem(prob0, device=0)
+    nodes = h.all_nodes()
+    # the quasi-Newton iteration converges linearly, slowly for the coldest vertices: hotter ones here
+    F = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in (600, 700, 800, 1023)]),
+                     device=DEV)
+    Fn = torch.empty_like(F)
+    dt = 0.002
+    n_it, dn = h.implicit_step_batched(dt, F, Fn, max_iter=40, rtol=1e-12)
+    torch.cuda.synchronize()
+    assert n_it < 40 and dn <= 1e-12
+    M = torch.empty(h.nnz, dtype=torch.float64, device=DEV)
+    h.mass(1.0, M)
+    rp, col = h.pattern()
+    Mm = sps.csr_matrix((M.cpu().numpy(), col, rp), shape=(h.ndof, h.ndof))
+    ng = h.grid_ndof(0)
+    r, z = np.concatenate([nodes[0][0]] * 2), np.concatenate([nodes[0][1]] * 2)
+    m = np.repeat(np.asarray(prob0.mass, float), ng)
+    for k in range(nb):
+        f0, f1 = F[k].cpu().numpy(), Fn[k].cpu().numpy()
+        d0, d1 = Mm @ f0, Mm @ f1
+        for a in range(2):
+            sl = slice(a * ng, (a + 1) * ng)
+            assert abs(d1[sl].sum() - d0[sl].sum()) <= 1e-12 * abs(d0[sl].sum())
+        psi = r * r + z * z
+        assert abs((m * psi * (d1 - d0)).sum()) <= 1e-10 * (m * psi * np.abs(d0)).sum()
+        assert abs((m * z * (d1 - d0)).sum()) <= 1e-10 * (m * np.abs(z) * np.abs(d0)).sum()
+        assert np.linalg.norm(f1 - f0) > 1e-6 * np.linalg.norm(f0)
