@@ -403,6 +403,38 @@ def main():
                         "DGEMMs (cuBLAS, FP64 tensor cores); same sums up to order, parity-tested"}}
         except Exception as e:   # the variant is optional: report why it did not run
             line["variants"] = {"tensor_cache_gemm": {"unavailable": str(e)[:200]}}
+    # NEXT-3: quasi-Newton backward-Euler iterations on the same batch (the paper's figure of merit,
+    # "Newton iterations per second", @37187): per iteration set_state + Jacobian + band LU + solve
+    if args.workload == "C4" and not args.tensor_cache and nloc:
+        try:
+            it_per_call = 2
+            Fn = torch.empty_like(F)
+            for _ in range(2):
+                h.implicit_step_batched(0.002, F, Fn, max_iter=it_per_call, rtol=0.0)
+            torch.cuda.synchronize()
+            h.set_timing(True)
+            nev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+            for k in range(args.steps):
+                flush.fill_(float(k))
+                nev[k][0].record(stream)
+                h.implicit_step_batched(0.002, F, Fn, max_iter=it_per_call, rtol=0.0)
+                nev[k][1].record(stream)
+            torch.cuda.synchronize()
+            nt = h.get_timing()
+            h.set_timing(False)
+            nms = torch.tensor([sum(a.elapsed_time(b) for a, b in nev)], dtype=torch.float64, device="cuda")
+            if world > 1:
+                dist.all_reduce(nms, op=dist.ReduceOp.MAX)
+            ms_it = float(nms.item()) / (args.steps * it_per_call)
+            line["newton"] = {
+                "value": total_builds / (ms_it / 1e3), "unit": "vertex Newton iterations/s", "ms_per_iteration": ms_it,
+                "stage_ms_per_iteration": {k: v[0] / (args.steps * it_per_call) for k, v in nt.items()},
+                "note": "SURVEY NEXT-3: backward-Euler step by quasi-Newton (Jacobian about each iterate, A = M/dt - J "
+                        "factored by the RCM band LU, solve), all vertices of the job per iteration, dt = 0.002, "
+                        f"{it_per_call} iterations per landau_implicit_step_batched call; context: the paper's V100 "
+                        "node figure is a different problem (10 species, 80 cells, CPU LU)"}
+        except Exception as e:
+            line["newton"] = {"unavailable": str(e)[:200]}
     # configs[1] itself (one C2 grid, one build per step; launch-latency regime, CUDA-graph replay)
     if args.workload == "C4" and rank == 0:
         try:
