@@ -209,11 +209,22 @@ int landau_advection(landau_t h, double Ez, double *values_dev, int32_t format);
 int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
                                  double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm);
 
+/* Mirror symmetry (v_par -> -v_par, i.e. z -> -z): when every grid's quadrature points come in pairs
+ * (r, z), (r, -z) (within 1e-12 R, no point on z = 0) -- true of every configuration of SURVEY §8(d)
+ * -- the batched (symmetric) inner integral evaluates each tensor once for four ordered interactions:
+ * reflection keeps lambda+-, x, m and every azimuthal integral and negates the rz / zr components,
+ * U(i', j') = F U(i, j) F with F = diag(1, -1), on top of the i <-> j symmetry (N^2/4 tensor
+ * evaluations per build instead of N^2/2).  The mirror point is placed at exactly (r, -z), a
+ * perturbation within the 1e-12 R detection tolerance.  On by default when available;
+ * enable = 0 selects the plain symmetric kernel, enable = 1 on a non-symmetric mesh is EUNSUPPORTED. */
+int landau_set_mirror(landau_t h, int32_t enable);
+
 /* How the last build ran (for FLOP accounting and diagnostics). */
 typedef struct {
   int32_t inner_path;        /* 0: directed pair kernel (every ordered pair, split-j when small);
                                 1: symmetric pair kernel (every unordered pair once, both targets);
-                                2: tensor cache + FP64 GEMM (landau_set_tensor_cache)              */
+                                2: tensor cache + FP64 GEMM (landau_set_tensor_cache);
+                                3: mirror-symmetric pair kernel (landau_set_mirror)                */
   int64_t nbatch;            /* batch items of the last build                                      */
   int64_t targets;           /* target points per batch item (all N unless element-split)          */
   int64_t sources;           /* source points per batch item (N)                                   */

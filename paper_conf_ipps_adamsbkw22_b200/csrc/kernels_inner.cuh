@@ -260,6 +260,243 @@ __global__ void reduce_sym_kernel(int64_t N, int64_t nslots, const int32_t *__re
 }
 
 // ------------------------------------------------------------------------------------------------
+// N2 (mirror-symmetric): meshes symmetric under v_par -> -v_par (z -> -z; every configuration of
+// SURVEY §8(d)) pair each point u of the upper half U (z > 0) with its mirror u' (detected and
+// symmetrised at create).  Reflection keeps lambda+-, x, m and every J integral and flips the sign of
+// the off-diagonal components:  U(i', j') = F U(i, j) F,  F = diag(1, -1) on (r, z).  So with
+//   A(u)  = (wT_D, wT_Kr, wT_Kz)(u),     Bf(u) = F-flipped weights of u' = (wT_D, wT_Kr, -wT_Kz)(u'),
+//   G(u) = Ga(u),  G(u') = F Gb(u)      (F on G: negate the rz and K_z components),
+// and U(i, j) the same-side tensor, V(i, j) = U(i, j') the cross tensor (source mirrored),
+//   Ga(i) = sum_j U(i,j) A(j) + V(i,j) F Bf(j),     Gb(i) = sum_j U(i,j) Bf(j) + V(i,j) F A(j).
+// One tensor evaluation serves four ordered interactions (the i <-> j symmetry of the symmetric
+// kernel on top): N^2 / 4 evaluations per build instead of N^2 / 2.  The reverse direction of a V
+// evaluation is F rev(V(i,j)) F, so V items accumulate it F-flipped (sources R1 = Bf(i), R2 = A(i))
+// and flip it when storing.  Items and slots as in inner_sym_kernel over the tiles of U, each item
+// once as a U item and once as a V item (it.v); a V diagonal item also pairs every point with its own
+// mirror (step 0, forward only).  part = [batch][nslots][2][5][32] (Ga, Gb).
+// ------------------------------------------------------------------------------------------------
+struct MirItem {   // host-built
+  int a[3];        // i-tiles (n of them, all < b); n == 0: the diagonal item (b, b)
+  int b, n;
+  int v;           // 0: same-side tensors U(i, j); 1: cross tensors V(i, j) = U(i, j')
+  int slot;        // first of the item's consecutive slots: one per i-tile (or the diagonal), then j's
+};
+
+struct Acc10 {
+  Acc5 a, b;
+};
+
+// wT gather of one U point's weight pair: A(u), Bf(u) (zero for padding)
+__device__ __forceinline__ void mir_weights(const double *wb, int64_t N, int64_t H, const int32_t *pu,
+                                            const int32_t *pm, int64_t u, double A[3], double Bf[3]) {
+  if (u < H) {
+    const int64_t p = pu[u], q = pm[u];
+    A[0] = wb[p];
+    A[1] = wb[N + p];
+    A[2] = wb[2 * N + p];
+    Bf[0] = wb[q];
+    Bf[1] = wb[N + q];
+    Bf[2] = -wb[2 * N + q];
+  } else {
+    A[0] = A[1] = A[2] = Bf[0] = Bf[1] = Bf[2] = 0.0;
+  }
+}
+
+__device__ __forceinline__ void acc_fwd(Acc5 &a, double Udrr, double Udrz, double Udzz, double Ukrr, double Ukzr,
+                                        double wd, double wkr, double wkz) {
+  a.drr = fma(wd, Udrr, a.drr);
+  a.drz = fma(wd, Udrz, a.drz);
+  a.dzz = fma(wd, Udzz, a.dzz);
+  a.kr = fma(Ukrr, wkr, fma(Udrz, wkz, a.kr));
+  a.kz = fma(Ukzr, wkr, fma(Udzz, wkz, a.kz));
+}
+
+// the reverse tensors of (i, j): U^D_rr(j,i) = Vdrr, U^D_rz(j,i) = Ukzr, U^D_zz, U^K_rr symmetric,
+// U^K_zr(j,i) = Udrz (see landau_pair_sym)
+__device__ __forceinline__ void acc_rev(Acc5 &a, double Vdrr, double Udrz, double Udzz, double Ukrr, double Ukzr,
+                                        double wd, double wkr, double wkz) {
+  a.drr = fma(wd, Vdrr, a.drr);
+  a.drz = fma(wd, Ukzr, a.drz);
+  a.dzz = fma(wd, Udzz, a.dzz);
+  a.kr = fma(Ukrr, wkr, fma(Ukzr, wkz, a.kr));
+  a.kz = fma(Udrz, wkr, fma(Udzz, wkz, a.kz));
+}
+
+__device__ __forceinline__ void acc_shfl(Acc5 &a, int src) {
+  a.drr = __shfl_sync(0xffffffffu, a.drr, src);
+  a.drz = __shfl_sync(0xffffffffu, a.drz, src);
+  a.dzz = __shfl_sync(0xffffffffu, a.dzz, src);
+  a.kr = __shfl_sync(0xffffffffu, a.kr, src);
+  a.kz = __shfl_sync(0xffffffffu, a.kz, src);
+}
+
+// store 5 x 32 sums at lane position pos; flip = negate the rz and K_z components (F)
+__device__ __forceinline__ void mir_store(double *o, int pos, const Acc5 &a, bool flip) {
+  const double sg = flip ? -1.0 : 1.0;
+  o[pos] = a.drr;
+  o[32 + pos] = sg * a.drz;
+  o[64 + pos] = a.dzz;
+  o[96 + pos] = a.kr;
+  o[128 + pos] = sg * a.kz;
+}
+
+template <int NI, bool DIAG, bool MASK>
+__device__ __forceinline__ void mir_run(const MirItem &it, const double *rU, const double *zU, const double *wb,
+                                        int64_t N, int64_t H, const int32_t *pu, const int32_t *pm, int lane,
+                                        const double2 *s_j, const PairCoef &cf, double *o) {
+  // lane data: target i of each i-tile, its reverse-source weights R1, R2 and its sums Ga, Gb
+  const bool V = it.v != 0;
+  double r[NI], z[NI], r2[NI], R1[NI][3], R2[NI][3];
+  Acc5 ga[NI], gb[NI];
+#pragma unroll
+  for (int t = 0; t < NI; t++) {
+    const int64_t i = (int64_t)(DIAG ? it.b : it.a[t]) * 32 + lane;
+    double A[3], Bf[3];
+    mir_weights(wb, N, H, pu, pm, i, A, Bf);
+    r[t] = i < H ? rU[i] : 1.0;
+    z[t] = i < H ? zU[i] : 1.0e6 + 64.0 * t + lane;   // padding: far away, zero weights
+    r2[t] = r[t] * r[t];
+#pragma unroll
+    for (int c = 0; c < 3; c++) {
+      R1[t][c] = V ? Bf[c] : A[c];
+      R2[t][c] = V ? A[c] : Bf[c];
+    }
+    ga[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+    gb[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+  }
+  const int src = (lane + 1) & 31;
+  Acc5 ja{0.0, 0.0, 0.0, 0.0, 0.0}, jb{0.0, 0.0, 0.0, 0.0, 0.0};
+  // diagonal: V items start at step 0 (each point with its own mirror, forward only); steps 1..15
+  // unmasked, step 16 peeled (lanes >= 16 would double-count)
+  const int k0 = DIAG ? (V ? 0 : 1) : 0;
+  constexpr int kmain = DIAG ? 16 : 32;
+#pragma unroll 1
+  for (int k = k0; k < kmain; k++) {
+    const int jj = (lane + k) & 31;
+    const double2 rz = s_j[jj * 5], w1 = s_j[jj * 5 + 1], w12 = s_j[jj * 5 + 2], w2 = s_j[jj * 5 + 3],
+                  rr2 = s_j[jj * 5 + 4];
+    const bool rev_on = !(DIAG && k == 0);
+#pragma unroll
+    for (int t = 0; t < NI; t++) {
+      bool ok;
+      double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
+      pair_tensors<MASK>(r[t], z[t], r2[t], rz.x, rz.y, rr2.x, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
+      const double m = (!MASK || ok) ? 1.0 : 0.0;
+      const double mr = rev_on ? m : 0.0;
+      acc_fwd(ga[t], Udrr, Udrz, Udzz, Ukrr, Ukzr, m * w1.x, m * w1.y, m * w12.x);
+      acc_fwd(gb[t], Udrr, Udrz, Udzz, Ukrr, Ukzr, m * w12.y, m * w2.x, m * w2.y);
+      acc_rev(ja, Vdrr, Udrz, Udzz, Ukrr, Ukzr, mr * R1[t][0], mr * R1[t][1], mr * R1[t][2]);
+      acc_rev(jb, Vdrr, Udrz, Udzz, Ukrr, Ukzr, mr * R2[t][0], mr * R2[t][1], mr * R2[t][2]);
+    }
+    acc_shfl(ja, src);
+    acc_shfl(jb, src);
+  }
+  if constexpr (DIAG) {
+    const int jj = (lane + 16) & 31;
+    const double2 rz = s_j[jj * 5], w1 = s_j[jj * 5 + 1], w12 = s_j[jj * 5 + 2], w2 = s_j[jj * 5 + 3],
+                  rr2 = s_j[jj * 5 + 4];
+    bool ok;
+    double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
+    pair_tensors<true>(r[0], z[0], r2[0], rz.x, rz.y, rr2.x, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
+    const double m = (ok && lane < 16) ? 1.0 : 0.0;
+    acc_fwd(ga[0], Udrr, Udrz, Udzz, Ukrr, Ukzr, m * w1.x, m * w1.y, m * w12.x);
+    acc_fwd(gb[0], Udrr, Udrz, Udzz, Ukrr, Ukzr, m * w12.y, m * w2.x, m * w2.y);
+    acc_rev(ja, Vdrr, Udrz, Udzz, Ukrr, Ukzr, m * R1[0][0], m * R1[0][1], m * R1[0][2]);
+    acc_rev(jb, Vdrr, Udrz, Udzz, Ukrr, Ukzr, m * R2[0][0], m * R2[0][1], m * R2[0][2]);
+    acc_shfl(ja, src);
+    acc_shfl(jb, src);
+  }
+#pragma unroll
+  for (int t = 0; t < NI; t++) {
+    mir_store(o + t * 320, lane, ga[t], false);
+    mir_store(o + t * 320 + 160, lane, gb[t], false);
+  }
+  // after the last hand-over lane L holds the reverse sums of j = (L + kend) mod 32
+  const int kend = DIAG ? 17 : 32;
+  const int jf = (lane + kend) & 31;
+  double *oj = o + (DIAG ? 1 : NI) * 320;
+  mir_store(oj, jf, ja, V);
+  mir_store(oj + 160, jf, jb, V);
+}
+
+template <int MINB, bool MASK>
+__global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_mir_kernel(int64_t N, int64_t H, int64_t nitems_b,
+                                                                         int64_t nslots, int64_t nitems,
+                                                                         const MirItem *__restrict__ items,
+                                                                         const double *__restrict__ rU,
+                                                                         const double *__restrict__ zU,
+                                                                         const int32_t *__restrict__ pu,
+                                                                         const int32_t *__restrict__ pm,
+                                                                         const double *__restrict__ wT,
+                                                                         double *__restrict__ part) {
+  __shared__ double2 s_j[kSymWarps][32 * 5];   // per j: (r, z_src), W1 (d, kr), (W1 kz, W2 d), W2 (kr, kz), (r^2, -)
+  __shared__ double s_coef[kNumPairCoef];
+  __shared__ double2 s_ltab[kLogTab];
+  stage_pair_coef(s_coef, s_ltab);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, s_ltab, cf);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
+    const int64_t bb = item / nitems_b;
+    const MirItem it = items[item % nitems_b];
+    const double *wb = wT + bb * 3 * N;
+    __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
+    {   // stage the j-tile: U items see j at (r, z) with W1 = A(j), W2 = Bf(j); V items see j' at
+        // (r, -z) with W1 = F Bf(j) (= the weights of j'), W2 = F A(j)
+      const int64_t j = (int64_t)it.b * 32 + lane;
+      double A[3], Bf[3];
+      mir_weights(wb, N, H, pu, pm, j, A, Bf);
+      const double r = j < H ? rU[j] : 1.0;
+      const double z = j < H ? zU[j] : 2.0e6 + lane;
+      double2 *d = &s_j[wid][lane * 5];
+      if (it.v) {
+        d[0] = make_double2(r, -z);
+        d[1] = make_double2(Bf[0], Bf[1]);
+        d[2] = make_double2(-Bf[2], A[0]);
+        d[3] = make_double2(A[1], -A[2]);
+      } else {
+        d[0] = make_double2(r, z);
+        d[1] = make_double2(A[0], A[1]);
+        d[2] = make_double2(A[2], Bf[0]);
+        d[3] = make_double2(Bf[1], Bf[2]);
+      }
+      d[4] = make_double2(r * r, 0.0);
+    }
+    __syncwarp();
+    double *o = part + (bb * nslots + it.slot) * 320;
+    switch (it.n) {
+      case 0: mir_run<1, true, MASK>(it, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, o); break;
+      case 1: mir_run<1, false, MASK>(it, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, o); break;
+      default:
+        if constexpr (kSymNI >= 2) mir_run<2, false, MASK>(it, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, o);
+        break;
+    }
+  }
+}
+
+// G[b][c][pu(u)] = sum of the Ga parts, G[b][c][pm(u)] = F (sum of the Gb parts), over the slots of
+// u's tile in the fixed order of tile_slots
+__global__ void reduce_mir_kernel(int64_t N, int64_t H, int64_t nslots, const int32_t *__restrict__ tile_ptr,
+                                  const int32_t *__restrict__ tile_slots, const int32_t *__restrict__ pu,
+                                  const int32_t *__restrict__ pm, const double *__restrict__ part,
+                                  double *__restrict__ G, int64_t G_bstride, int nbatch) {
+  const int64_t total = (int64_t)nbatch * 5 * H;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = k / (5 * H), c = (k / H) % 5, u = k % H;
+    const int t = (int)(u / 32), lane = (int)(u % 32);
+    const double *pbk = part + b * nslots * 320 + c * 32 + lane;
+    double sa = 0.0, sb = 0.0;
+    for (int q = tile_ptr[t]; q < tile_ptr[t + 1]; q++) {
+      sa += pbk[(int64_t)tile_slots[q] * 320];
+      sb += pbk[(int64_t)tile_slots[q] * 320 + 160];
+    }
+    G[b * G_bstride + c * N + pu[u]] = sa;
+    G[b * G_bstride + c * N + pm[u]] = (c == 1 || c == 4) ? -sb : sb;
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
 // Tensor cache fill (NEXT-4): every ordered pair (i, j) once, written column-major for the GEMMs:
 //   A1 (3N x N): rows c N + i, c = 0,1,2 -> U^D_rr, U^D_rz, U^D_zz
 //   A2 (N x 2N): [U^K_rr | U^D_rz],  A3 (N x 2N): [U^K_zr | U^D_zz]

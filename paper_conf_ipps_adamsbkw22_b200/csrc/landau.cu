@@ -76,6 +76,15 @@ struct landau_s {
   int32_t *d_tile_ptr = nullptr, *d_tile_slots = nullptr;
   int ntiles = 0;
   int64_t nsym_items = 0, nsym_slots = 0;
+  // mirror-symmetric inner kernel (meshes symmetric under z -> -z): upper-half points u, their
+  // original indices pu and mirrors pm, work items and slot map over the tiles of the upper half
+  bool mirror = false;     // the mesh is mirror-symmetric (maps built)
+  bool mirror_on = true;   // use inner_mir_kernel when the symmetric path runs (landau_set_mirror)
+  int64_t H = 0, nmir_items = 0, nmir_slots = 0;
+  double *d_rU = nullptr, *d_zU = nullptr;
+  int32_t *d_pu = nullptr, *d_pm = nullptr;
+  MirItem *d_mir_items = nullptr;
+  int32_t *d_mtile_ptr = nullptr, *d_mtile_slots = nullptr;
   bool coincident = false;   // two distinct quadrature points with identical (r, z) (never for one grid)
   // tensor cache (NEXT-4)
   bool tcache = false, tcache_valid = false;
@@ -259,6 +268,15 @@ bool sym_enabled() {
   return v;
 }
 
+// mirror-symmetric inner kernel when the mesh allows it (LANDAU_MIRROR=0 disables)
+bool mirror_enabled() {
+  static const bool v = [] {
+    const char *e = getenv("LANDAU_MIRROR");
+    return !(e && atoi(e) == 0);
+  }();
+  return v;
+}
+
 // inner-kernel variant (targets per thread, min blocks per SM); LANDAU_INNER_VARIANT overrides
 int inner_variant() {
   static const int v = [] {
@@ -283,7 +301,7 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
     ip.wtiles = h->ntiles;
     ip.nsplit = 1;
     ip.split_len = N;
-    const int64_t need = nbatch * h->nsym_slots * 160;
+    const int64_t need = (h->mirror && h->mirror_on) ? nbatch * h->nmir_slots * 320 : nbatch * h->nsym_slots * 160;
     if (need > h->part_cap) {
       drop_graphs(h);
       cudaFree(h->d_part);
@@ -358,12 +376,45 @@ int launch_inner(landau_t h, int64_t nbatch) {
   h->stats.sources = N;
   h->stats.inner_path = ip.sym ? 1 : 0;
   h->stats.nsplit = ip.sym ? 1 : ip.nsplit;
-  if (ip.sym) {
+  if (ip.sym && h->mirror && h->mirror_on) {
+    // tensor evaluations per batch item: U and V items over the T tiles of the upper half; diagonal
+    // items 16 (U) or 17 (V) steps x 32 lanes, the others 32 x 32 per i-tile
+    const int64_t T = (h->H + 31) / 32;
+    h->stats.pair_evaluations = T * 33 * 32 + 2 * (T * (T - 1) / 2) * 32 * 32;
+    h->stats.inner_path = 3;
+  } else if (ip.sym) {
     int64_t ev = 0;   // lane-steps per batch item: diagonal items 16 x 32, others 32 x 32 per i-tile
     ev = (int64_t)h->ntiles * 16 * 32 + (int64_t)h->ntiles * (h->ntiles - 1) / 2 * 32 * 32;
     h->stats.pair_evaluations = ev;
   } else {
     h->stats.pair_evaluations = ip.wtiles * 32 * ip.tpt * N;
+  }
+  if (ip.sym && h->mirror && h->mirror_on) {
+    {
+      Timer t(h, LANDAU_T_INNER);
+      const int64_t nitems = nbatch * h->nmir_items;
+      const unsigned grid = (unsigned)std::min<int64_t>((nitems + kSymWarps - 1) / kSymWarps, (int64_t)LANDAU_SYM_MINB * num_sms(h));
+      if (h->coincident)
+        inner_mir_kernel<LANDAU_SYM_MINB, true><<<grid, 32 * kSymWarps, 0, h->stream>>>(
+            N, h->H, h->nmir_items, h->nmir_slots, nitems, h->d_mir_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
+            h->d_part);
+      else
+        inner_mir_kernel<LANDAU_SYM_MINB, false><<<grid, 32 * kSymWarps, 0, h->stream>>>(
+            N, h->H, h->nmir_items, h->nmir_slots, nitems, h->d_mir_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
+            h->d_part);
+      h->launches++;
+      h->tlaunch[LANDAU_T_INNER]++;
+      KCHECK();
+    }
+    Timer t(h, LANDAU_T_REDUCE);
+    const int64_t total = nbatch * 5 * h->H;
+    const int blocks = (int)std::min<int64_t>((total + 255) / 256, 16LL * num_sms(h));
+    reduce_mir_kernel<<<blocks, 256, 0, h->stream>>>(N, h->H, h->nmir_slots, h->d_mtile_ptr, h->d_mtile_slots, h->d_pu,
+                                                     h->d_pm, h->d_part, G_own, 5 * h->Nc, (int)nbatch);
+    h->launches++;
+    h->tlaunch[LANDAU_T_REDUCE]++;
+    KCHECK();
+    return LANDAU_OK;
   }
   if (ip.sym) {
     {
@@ -754,6 +805,74 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
         (rc = upload(h, &h->d_tile_slots, tslots)))
       return bail(rc);
   }
+  if (world == 1 && mirror_enabled()) {   // mirror symmetry z -> -z of every grid (inner_mir_kernel)
+    std::vector<int32_t> pu, pm;
+    std::vector<double> rU, zU;
+    bool ok = true;
+    for (int g = 0; g < P.ngrids && ok; g++) {
+      const GridPlan &G = P.grids[g];
+      std::vector<int64_t> up, lo;
+      for (int64_t i = G.pt0; i < G.pt0 + G.ncell * P.nqp; i++) {
+        if (P.pz[i] > 0) up.push_back(i);
+        else if (P.pz[i] < 0) lo.push_back(i);
+        else ok = false;   // a point on z = 0 would be its own mirror
+      }
+      if (!ok || up.size() != lo.size()) {
+        ok = false;
+        break;
+      }
+      std::sort(up.begin(), up.end(), [&](int64_t a, int64_t b) {
+        return P.pr[a] != P.pr[b] ? P.pr[a] < P.pr[b] : P.pz[a] < P.pz[b];
+      });
+      std::sort(lo.begin(), lo.end(), [&](int64_t a, int64_t b) {
+        return P.pr[a] != P.pr[b] ? P.pr[a] < P.pr[b] : -P.pz[a] < -P.pz[b];
+      });
+      for (size_t k = 0; k < up.size() && ok; k++) {
+        const int64_t a = up[k], b = lo[k];
+        if (P.pr[a] != P.pr[b] || std::fabs(P.pz[a] + P.pz[b]) > 1e-12 * G.R) ok = false;
+        pu.push_back((int32_t)a);
+        pm.push_back((int32_t)b);
+        rU.push_back(P.pr[a]);
+        zU.push_back(P.pz[a]);   // the mirror sits at exactly (r, -z) for the inner integral
+      }
+    }
+    if (ok && !pu.empty()) {
+      const int64_t H = (int64_t)pu.size();
+      const int T = (int)((H + 31) / 32);
+      std::vector<MirItem> items;
+      std::vector<std::vector<int32_t>> slots_of(T);
+      int slot = 0;
+      for (int v = 0; v < 2; v++)
+        for (int b = 0; b < T; b++) {
+          items.push_back({{b, -1, -1}, b, 0, v, slot});
+          slots_of[b].push_back(slot);
+          slots_of[b].push_back(slot + 1);
+          slot += 2;
+          for (int a = 0; a < b; a += std::min(kSymNI, 2)) {
+            MirItem it{{-1, -1, -1}, b, std::min(std::min(kSymNI, 2), b - a), v, slot};
+            for (int t = 0; t < it.n; t++) {
+              it.a[t] = a + t;
+              slots_of[a + t].push_back(slot++);
+            }
+            slots_of[b].push_back(slot++);
+            items.push_back(it);
+          }
+        }
+      std::vector<int32_t> tptr(1, 0), tslots;
+      for (int t = 0; t < T; t++) {
+        tslots.insert(tslots.end(), slots_of[t].begin(), slots_of[t].end());
+        tptr.push_back((int32_t)tslots.size());
+      }
+      h->mirror = true;
+      h->H = H;
+      h->nmir_items = (int64_t)items.size();
+      h->nmir_slots = slot;
+      if ((rc = upload(h, &h->d_rU, rU)) || (rc = upload(h, &h->d_zU, zU)) || (rc = upload(h, &h->d_pu, pu)) ||
+          (rc = upload(h, &h->d_pm, pm)) || (rc = upload(h, &h->d_mir_items, items)) ||
+          (rc = upload(h, &h->d_mtile_ptr, tptr)) || (rc = upload(h, &h->d_mtile_slots, tslots)))
+        return bail(rc);
+    }
+  }
   {   // band solver maps (NEXT-2)
     h->d_ent_ptr.assign(P.ngrids, nullptr);
     h->d_ent_slot.assign(P.ngrids, nullptr);
@@ -853,6 +972,13 @@ void landau_destroy(landau_t h) {
   cudaFree(h->d_sym_items);
   cudaFree(h->d_tile_ptr);
   cudaFree(h->d_tile_slots);
+  cudaFree(h->d_rU);
+  cudaFree(h->d_zU);
+  cudaFree(h->d_pu);
+  cudaFree(h->d_pm);
+  cudaFree(h->d_mir_items);
+  cudaFree(h->d_mtile_ptr);
+  cudaFree(h->d_mtile_slots);
   cudaFree(h->d_ext_ptr);
   cudaFree(h->d_ext_dof);
   for (auto *v : {&h->d_csr, &h->d_coo})
@@ -1110,6 +1236,14 @@ int landau_get_timing(landau_t h, double *ms, int64_t *launches) {
     if (ms) ms[i] = acc[i];
     if (launches) launches[i] = h->tlaunch[i];
   }
+  return LANDAU_OK;
+}
+
+int landau_set_mirror(landau_t h, int32_t enable) {
+  if (!h) return LANDAU_EINVAL;
+  if (enable && !h->mirror) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: the mesh is not mirror-symmetric");
+  if (!h->host_only) drop_graphs(h);
+  h->mirror_on = enable != 0;
   return LANDAU_OK;
 }
 

@@ -82,6 +82,7 @@ def lib():
             "landau_get_launch_count": (C.c_int, [vp, P64]),
             "landau_get_stats": (C.c_int, [vp, C.POINTER(_Stats)]),
             "landau_set_tensor_cache": (C.c_int, [vp, i32]),
+            "landau_set_mirror": (C.c_int, [vp, i32]),
             "landau_band_info": (C.c_int, [vp, i32, P32, P32]),
             "landau_band_factor_batched": (C.c_int, [vp, i64, d, vp]),
             "landau_band_solve_batched": (C.c_int, [vp, i64, vp, vp]),
@@ -312,6 +313,9 @@ class Landau:
         nb = b.shape[0] if b.dim() == 2 else 1
         self._check(lib().landau_band_solve_batched(self._h, nb, _tptr(b), _tptr(x)), "landau_band_solve_batched")
         return x
+
+    def set_mirror(self, enable=True):
+        self._check(lib().landau_set_mirror(self._h, int(bool(enable))), "landau_set_mirror")
 
     def set_tensor_cache(self, enable=True):
         self._check(lib().landau_set_tensor_cache(self._h, int(bool(enable))), "landau_set_tensor_cache")

@@ -261,12 +261,15 @@ def test_graph_replay_matches_direct_launches():
     assert np.array_equal(b.view(np.uint64), c.view(np.uint64))
 
 
-def test_symmetric_kernel_batch_C4():
+@pytest.mark.parametrize("mirror", [True, False])
+def test_symmetric_kernel_batch_C4(mirror):
     """A batch large enough for the symmetric inner kernel (each unordered pair evaluated once, both
-    targets updated): vertices against the oracle, conservation, and bitwise determinism."""
+    targets updated; with mirror=True also each z-mirrored pair from the same tensor): vertices
+    against the oracle, conservation, and bitwise determinism."""
     nb = 24
     prob0 = inputs.config4_vertex(0)
     h = L.Landau.from_problem(prob0, device=0)
+    h.set_mirror(mirror)
     verts = [int(round(k * 1023 / (nb - 1))) for k in range(nb)]
     probs = [inputs.config4_vertex(b) for b in verts]
     nodes = h.all_nodes()
@@ -278,6 +281,7 @@ def test_symmetric_kernel_batch_C4():
     t = h.get_timing()
     h.set_timing(False)
     assert t["reduce"][1] == 1    # the symmetric path always reduces its partial slots
+    assert h.stats()["inner_path"] == (3 if mirror else 1)
     Jb = out.cpu().numpy()
     for k in (0, nb // 2, nb - 1):
         o = Oracle(probs[k])
@@ -334,8 +338,14 @@ def test_symmetric_kernel_with_coincident_points():
     out = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
     h.jacobian_batched(out)
     torch.cuda.synchronize()
-    assert h.stats()["inner_path"] == 1
+    assert h.stats()["inner_path"] == 3   # the twin mesh is z-symmetric too: masked mirror kernel
     Jb = out.cpu().numpy()
+    h.set_mirror(False)
+    out2 = torch.empty_like(out)
+    h.jacobian_batched(out2)
+    torch.cuda.synchronize()
+    assert h.stats()["inner_path"] == 1   # masked plain symmetric kernel
+    assert np.abs(out2.cpu().numpy() - Jb).max() <= 1e-13 * np.abs(Jb).max()
     for b in (0, nb - 1):
         p = inputs.Problem("twin", 3, prob.grids, prob.species, fmix=[[(1.0 + 0.01 * b, 1.0, 0.0)], [(1.0, 0.5, 0.0)]],
                            seed=99 + b)
@@ -399,7 +409,7 @@ def test_tensor_cache_gemm_path_C4():
     assert np.array_equal(out.cpu().numpy().view(np.uint64), Jc.view(np.uint64))
     h.set_tensor_cache(False)
     h.jacobian_batched(out)
-    assert h.stats()["inner_path"] == 1
+    assert h.stats()["inner_path"] in (1, 3)
 
 
 def test_more_error_codes_and_coo_batched():
@@ -592,3 +602,43 @@ def test_implicit_step_converges_and_conserves_C4_batch():
         assert abs((m * psi * (d1 - d0)).sum()) <= 1e-10 * (m * psi * np.abs(d0)).sum()
         assert abs((m * z * (d1 - d0)).sum()) <= 1e-10 * (m * np.abs(z) * np.abs(d0)).sum()
         assert np.linalg.norm(f1 - f0) > 1e-6 * np.linalg.norm(f0)
+
+
+def test_mirror_kernel_C3_C5_sampled_and_unsupported_mesh():
+    """Mirror kernel on the three-grid impurity case (C3, batched) against the oracle's point
+    coefficients; a mesh that is not z-symmetric refuses set_mirror(True) and still builds."""
+    prob, h0, o, fg, fo = setup("C3")
+    h = L.Landau.from_problem(prob, device=0)
+    nb = 64   # enough items for the batched (symmetric) path
+    F = torch.tensor(np.stack([fg] * nb), device=DEV)
+    h.set_state_batched(F)
+    G = torch.empty((nb, 5, h.npoints), dtype=torch.float64, device=DEV)
+    h.point_coeffs_batched(G)
+    torch.cuda.synchronize()
+    assert h.stats()["inner_path"] == 3
+    Go, Ga = o.point_coeffs(fo)
+    assert np.max(np.abs(G[nb - 1].cpu().numpy() - Go) / Ga) <= 1e-12
+    # an asymmetric mesh: the uniform 2 x 4 mesh with one upper cell split into four
+    R = inputs.R_E
+    cells = inputs.uniform_mesh(R, 2)
+    top = max(cells, key=lambda c: (c[1], c[0]))
+    cells.remove(top)
+    cells += inputs._split(top)
+    asym = inputs.Problem("asym", 2, [(R, cells)], [inputs.Species("e", 1.0, -1.0, 0)],
+                          fmix=[[(1.0, 1.0, 0.3)]], seed=7)
+    ha = L.Landau.from_problem(asym, device=0)
+    assert not _mesh_is_mirror(ha)
+    with pytest.raises(L.LandauError):
+        ha.set_mirror(True)
+    oa = Oracle(asym)
+    fa = oa.coefficients()
+    J = gpu_jacobian(ha, inputs.coefficients(asym, ha.all_nodes()))
+    Jo, Ja = oa.jacobian(fa)
+    assert np.all(np.abs(J - Jo) <= 1e-11 * Ja)
+
+
+def _mesh_is_mirror(h):
+    r, z, _ = h.points()
+    a = sorted(zip(r, z))
+    b = sorted(zip(r, -z))
+    return np.allclose(np.array(a), np.array(b), atol=1e-12)
