@@ -147,6 +147,9 @@ def load_profile_traffic(workload):
 #   symmetric kernel: 193 FLOP per unordered pair, N (N - 1) / 2 per batch item (both targets updated)
 FLOP_PER_PAIR_DIRECTED = 177.0
 FLOP_PER_PAIR_SYMMETRIC = 193.0
+# mirror-symmetric kernel: FP64 FLOP (2 DFMA + DMUL + DADD, ncu SASS counts on C4) per tensor
+# evaluation, (N/2)^2 evaluations per batch item (profiles/r01_flops_mirror.csv)
+FLOP_PER_EVAL_MIRROR = 222.8
 
 
 def cpu_baseline(args, desc, nsample):
@@ -339,6 +342,9 @@ def main():
     if st["inner_path"] == 2:   # GEMMs: 2 FLOP per multiply-add, 7 N^2 per batch item (three DGEMMs)
         flop_per_pair = 14.0
         flops_per_launch = 14.0 * st["nbatch"] * N * N
+    elif st["inner_path"] == 3:
+        flop_per_pair = FLOP_PER_EVAL_MIRROR
+        flops_per_launch = flop_per_pair * st["nbatch"] * (N // 2) ** 2
     elif st["inner_path"] == 1:
         flop_per_pair = FLOP_PER_PAIR_SYMMETRIC
         flops_per_launch = flop_per_pair * st["nbatch"] * N * (N - 1) / 2
@@ -351,12 +357,13 @@ def main():
     sm_max = clocks["sm_max_mhz"] or 1965.0
     peak = fp64_peak_tflops(props, sm_max)
     step_ms_lib = sum(v[0] for v in tim.values()) / args.steps
-    roof = {"bound": "alu", "kernel": "inner_sym_kernel / inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
+    roof = {"bound": "alu", "kernel": "inner_mir_kernel / inner_sym_kernel / inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
             "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None,
             "traffic": load_profile_traffic(args.workload),
             "peak_note": f"derived FP64 DFMA peak: {props.multi_processor_count} SMs x 64 lanes x 2 FLOP x {sm_max:.0f} MHz",
             "inner_path": ["directed (ordered pairs)", "symmetric (unordered pairs)",
-                           "tensor cache + FP64 DGEMM (cuBLAS)"][st["inner_path"]],
+                           "tensor cache + FP64 DGEMM (cuBLAS)",
+                           "mirror-symmetric (one tensor per unordered pair and its z-mirror)"][st["inner_path"]],
             "flop_per_pair": flop_per_pair, "flops_per_launch": flops_per_launch,
             "inner_ms_per_launch": inner_avg_s * 1e3,
             "inner_share_of_step": (inner_ms / args.steps) / ms_per_step if ms_per_step else None,
@@ -460,7 +467,7 @@ def main():
             ms2 = sum(a.elapsed_time(b) for a, b in ev2) / args.steps
             line["c2_single_build"] = {"value": 1e3 / ms2, "unit": UNIT, "ms_per_step": ms2,
                                        "pairs_per_s": 1e3 / ms2 * p2.npoints ** 2,
-                                       "inner_path": ["directed", "symmetric", "tensor cache"][h2.stats()["inner_path"]],
+                                       "inner_path": ["directed", "symmetric", "tensor cache", "mirror"][h2.stats()["inner_path"]],
                                        "note": "BASELINE configs[1]: one e+D Q3 AMR grid (N=1088) per step, "
                                                "set_state + jacobian (CSR) + mass, CUDA-graph replay"}
             h2.close()

@@ -12,11 +12,18 @@ namespace landau {
 #define LANDAU_SYM_UNROLL 2
 #endif
 constexpr int kSymUnroll = LANDAU_SYM_UNROLL;
+#ifndef LANDAU_MIR_UNROLL
+#define LANDAU_MIR_UNROLL 1
+#endif
+constexpr int kMirUnroll = LANDAU_MIR_UNROLL;
 #ifndef LANDAU_SYM_WARPS
-#define LANDAU_SYM_WARPS 4
+#define LANDAU_SYM_WARPS 8   // measured (mirror kernel, C4): 8 warps x 1 block 2.89 ms, 4 x 2 3.13, 2 x 4 3.16
 #endif
 #ifndef LANDAU_SYM_MINB
-#define LANDAU_SYM_MINB 2
+#define LANDAU_SYM_MINB 1
+#endif
+#ifndef LANDAU_MIR_UNROLL
+#define LANDAU_MIR_UNROLL 1
 #endif
 
 // ------------------------------------------------------------------------------------------------
@@ -370,7 +377,7 @@ __device__ __forceinline__ void mir_run(const MirItem &it, const double *rU, con
   // unmasked, step 16 peeled (lanes >= 16 would double-count)
   const int k0 = DIAG ? (V ? 0 : 1) : 0;
   constexpr int kmain = DIAG ? 16 : 32;
-#pragma unroll 1
+#pragma unroll kMirUnroll
   for (int k = k0; k < kmain; k++) {
     const int jj = (lane + k) & 31;
     const double2 rz = s_j[jj * 5], w1 = s_j[jj * 5 + 1], w12 = s_j[jj * 5 + 2], w2 = s_j[jj * 5 + 3],

@@ -255,7 +255,7 @@ struct InnerPlan {
 int64_t sym_min_items_per_sm() {
   static const int64_t v = [] {
     const char *e = getenv("LANDAU_SYM_MIN_ITEMS_PER_SM");
-    return e ? (int64_t)atoll(e) : (int64_t)8 * kSymWarps;
+    return e ? (int64_t)atoll(e) : (int64_t)4 * kSymWarps * LANDAU_SYM_MINB;   // 4 items per resident warp
   }();
   return v;
 }

@@ -1,0 +1,6 @@
+# time build variants of liblandau (build_variants/*.so) on the C4 bench, inner-stage ms
+for f in paper_conf_ipps_adamsbkw22_b200/liblandau.so build_variants/liblandau_*.so; do
+  n=$(basename $f .so)
+  LANDAU_LIB=$f python bench.py --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/v_$n.json 2>gpurun_out/v_$n.err
+  python -c "import json; d=json.load(open('gpurun_out/v_$n.json')); print('$n', round(d['value']), 'builds/s inner', round(d['stage_ms_per_step']['inner'],3), 'ms')" || tail -3 gpurun_out/v_$n.err
+done
