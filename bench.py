@@ -149,7 +149,7 @@ FLOP_PER_PAIR_DIRECTED = 177.0
 FLOP_PER_PAIR_SYMMETRIC = 193.0
 # mirror-symmetric kernel: FP64 FLOP (2 DFMA + DMUL + DADD, ncu SASS counts on C4) per tensor
 # evaluation, (N/2)^2 evaluations per batch item (profiles/r01_flops_mirror.csv)
-FLOP_PER_EVAL_MIRROR = 222.8
+FLOP_PER_EVAL_MIRROR = 223.9
 
 
 def cpu_baseline(args, desc, nsample):
