@@ -406,7 +406,7 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
       };
       // the factorisation runs a window of P = Bp + 1 rows, P a multiple of 8 (kernels_band.cuh):
       // positions are relative to the padded half-bandwidth Bp >= B (entries past B are zero)
-      const int Bp = (B + 1 + 7) / 8 * 8 - 1;
+      const int Bp = (B + 2 + 7) / 8 * 8 - 1;   // B + 2 <= P: the rank-2 kernel's row k+1 fits the window
       G.band_p = Bp;
       G.ent_ptr.assign(1, 0);
       G.ent_slot.clear();

@@ -234,6 +234,212 @@ __global__ void __launch_bounds__(256, MINB) band_lu_kernel(const double *__rest
   }
 }
 
+// Rank-2 variant: elimination steps k, k+1 (k even) share one barrier.  The owners of the two
+// retiring rows / columns (same tile row and tile column, since k is even and R, C are even) publish
+// them raw; the owner of the 2 x 2 corner publishes the pivots and L(k+1, k); every thread then
+// forms, for its own rows and columns,
+//   l0 = A(., k) / p0,  l1 = (A(., k+1) - l0 A(k, k+1)) / p1,  u0 = A(k, .),  u1 = A(k+1, .) - L(k+1,k) u0
+// and applies cell -= l0 u0 + l1 u1 (the same outer-product elimination, two steps fused).  Needs the
+// half-bandwidth padding B + 2 <= P so row k+1's band (to column k+1+B_true) lies in the window.
+template <int kBandR, int kBandC, int MINB>
+__global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__restrict__ Aent, int64_t ent_bstride,
+                                                         double *__restrict__ LU, int64_t lu_bstride,
+                                                         const BandDesc *__restrict__ desc, int nsp) {
+  static_assert(kBandR % 2 == 0 && (8 % kBandR == 0 || kBandR % 8 == 0), "tile rows: even, divide the group");
+  static_assert(kBandC == 8, "tile columns = the group");
+  extern __shared__ double smem[];
+  const int bi = blockIdx.x / nsp, a = blockIdx.x % nsp;
+  const BandDesc d = desc[a];
+  const int n = d.n, B = d.B, P = B + 1, W = 2 * B + 1;
+  const int tid = threadIdx.x, T = blockDim.x;
+  const int ntc = P / kBandC;
+  const int tr = tid / ntc, tc = tid % ntc;
+  const bool owner = tr < P / kBandR;
+  const int pr0 = tr * kBandR, pc0 = tc * kBandC;
+  // shared layout, double-buffered by pair parity: column k, column k+1 (raw), row k, row k+1 (raw),
+  // corner scalars (p0, 1/p0, L(k+1,k), p1, 1/p1, U(k,k+1), -, -)
+  double *sh0 = smem;
+  double *dbuf = sh0 + 2 * (4 * P + 8);     // [3][8][W] entering rows (dense), one set per group
+  int32_t *sptr = (int32_t *)(dbuf + 24 * W);              // [n + 1]
+  uint16_t *spos = (uint16_t *)(sptr + n + 1);             // [nent]
+  for (int i = tid; i < 2 * (4 * P + 8); i += T) sh0[i] = 0.0;
+  for (int i = tid; i < 24 * W; i += T) dbuf[i] = 0.0;
+  for (int i = tid; i <= n; i += T) sptr[i] = d.ent_ptr[i];
+  for (int i = tid; i < d.nent; i += T) spos[i] = d.ent_pos[i];
+  const double *ae = Aent + (int64_t)bi * ent_bstride + d.aoff;
+  double *lu = LU + (int64_t)bi * lu_bstride + d.off;
+  const int ngroups = (n + 7) / 8;
+  auto grange = [&](int g, int &q0, int &q1) {
+    q0 = g < ngroups ? sptr[8 * g] : 0;
+    q1 = g < ngroups ? sptr[min(8 * g + 8, n)] : 0;
+  };
+  double vin[kBandE];
+  __syncthreads();
+  {
+    int q0, q1;
+    grange(0, q0, q1);
+#pragma unroll
+    for (int m = 0; m < kBandE; m++)
+      if (q0 + tid + m * T < q1) dbuf[spos[q0 + tid + m * T]] = ae[q0 + tid + m * T];
+    grange(1, q0, q1);
+#pragma unroll
+    for (int m = 0; m < kBandE; m++) vin[m] = q0 + tid + m * T < q1 ? ae[q0 + tid + m * T] : 0.0;
+  }
+  double cell[kBandR][kBandC];
+#pragma unroll
+  for (int r = 0; r < kBandR; r++)
+#pragma unroll
+    for (int c = 0; c < kBandC; c++) cell[r][c] = 0.0;
+  // writer: thread t < W writes entry t of LU[k] and of LU[k+1]; U entries sit at physical column
+  // pk + t, L entries at physical row pk + t - B (mod P)
+  const int tw = tid < W ? (tid <= B ? tid : tid - B) : 0;
+
+  int pkb = 0;
+  for (int kb = -P, g = 0; kb < n; kb += 8, g++) {
+    const double *dset = dbuf + (g % 3) * 8 * W;
+#pragma unroll
+    for (int u = 0; u < 8; u += 2) {
+      const int k = kb + u, pk = pkb + u;
+      const int rr = u % kBandR, cc = u % kBandC;   // rows rr, rr+1 / columns cc, cc+1 of the tile
+      const bool rowown = owner && tr == (pkb + u - rr) / kBandR;
+      const bool colown = owner && tc == pkb / kBandC;
+      const bool live0 = k >= 0 && k < n, live1 = k + 1 < n;
+      double *sh = sh0 + ((u >> 1) & 1) * (4 * P + 8);
+      double *a0_s = sh, *a1_s = sh + P, *u0_s = sh + 2 * P, *u1_s = sh + 3 * P, *sc = sh + 4 * P;
+      if (u == 0 && g >= 2) {   // clear group g - 2's rows from set (g + 1) mod 3
+        int q0, q1;
+        grange(g - 2, q0, q1);
+        double *ds = dbuf + ((g + 1) % 3) * 8 * W;
+#pragma unroll
+        for (int m = 0; m < kBandE; m++)
+          if (q0 + tid + m * T < q1) ds[spos[q0 + tid + m * T]] = 0.0;
+      }
+      if (live0) {   // b) publish rows k, k+1 and columns k, k+1 (zero at the retiring positions)
+        if (rowown) {
+#pragma unroll
+          for (int c = 0; c < kBandC; c++) {
+            const bool ret = colown && (c == cc || c == cc + 1);
+            u0_s[pc0 + c] = ret ? 0.0 : cell[rr][c];
+            u1_s[pc0 + c] = ret ? 0.0 : cell[rr + 1][c];
+          }
+          if (colown) {   // the 2 x 2 corner
+            const double p0 = cell[rr][cc], ukk1 = cell[rr][cc + 1];
+            const double r0 = rcp_newton(p0);
+            const double l10 = cell[rr + 1][cc] * r0;
+            const double p1 = fma(-l10, ukk1, cell[rr + 1][cc + 1]);
+            sc[0] = p0;
+            sc[1] = r0;
+            sc[2] = l10;
+            sc[3] = p1;
+            sc[4] = live1 ? rcp_newton(p1) : 0.0;
+            sc[5] = ukk1;
+          }
+        }
+        if (colown) {
+#pragma unroll
+          for (int r = 0; r < kBandR; r++) {
+            const bool ret = rowown && (r == rr || r == rr + 1);
+            a0_s[pr0 + r] = ret ? 0.0 : cell[r][cc];
+            a1_s[pr0 + r] = ret ? 0.0 : cell[r][cc + 1];
+          }
+        }
+      }
+      __syncthreads();
+      if (u == 0) {   // scatter group g + 1 into set (g + 1) mod 3; load group g + 2
+        int q0, q1;
+        grange(g + 1, q0, q1);
+        double *ds = dbuf + ((g + 1) % 3) * 8 * W;
+#pragma unroll
+        for (int m = 0; m < kBandE; m++)
+          if (q0 + tid + m * T < q1) ds[spos[q0 + tid + m * T]] = vin[m];
+        grange(g + 2, q0, q1);
+#pragma unroll
+        for (int m = 0; m < kBandE; m++) vin[m] = q0 + tid + m * T < q1 ? ae[q0 + tid + m * T] : 0.0;
+      }
+      if (live0) {   // c) rank-2 update; threads 0..2B write LU[k] and LU[k+1]
+        const double r0 = sc[1], l10 = sc[2], r1 = sc[4], ukk1 = sc[5];
+        if (owner) {
+          double l0[kBandR], l1[kBandR], u0[kBandC], u1[kBandC];
+          const double2 *a02 = reinterpret_cast<const double2 *>(a0_s + pr0);
+          const double2 *a12 = reinterpret_cast<const double2 *>(a1_s + pr0);
+#pragma unroll
+          for (int r = 0; r < kBandR / 2; r++) {
+            const double2 x0 = a02[r], x1 = a12[r];
+            l0[2 * r] = x0.x * r0;
+            l0[2 * r + 1] = x0.y * r0;
+            l1[2 * r] = fma(-l0[2 * r], ukk1, x1.x) * r1;
+            l1[2 * r + 1] = fma(-l0[2 * r + 1], ukk1, x1.y) * r1;
+          }
+          const double2 *u02 = reinterpret_cast<const double2 *>(u0_s + pc0);
+          const double2 *u12 = reinterpret_cast<const double2 *>(u1_s + pc0);
+#pragma unroll
+          for (int c = 0; c < kBandC / 2; c++) {
+            const double2 y0 = u02[c], y1 = u12[c];
+            u0[2 * c] = y0.x;
+            u0[2 * c + 1] = y0.y;
+            u1[2 * c] = fma(-l10, y0.x, y1.x);
+            u1[2 * c + 1] = fma(-l10, y0.y, y1.y);
+          }
+#pragma unroll
+          for (int r = 0; r < kBandR; r++)
+#pragma unroll
+            for (int c = 0; c < kBandC; c++) cell[r][c] = fma(-l1[r], u1[c], fma(-l0[r], u0[c], cell[r][c]));
+        }
+        if (tid < W) {
+          int j = pk + tw;
+          j -= j >= P ? P : 0;
+          double v0, v1;
+          if (tid == 0) {
+            v0 = sc[0];
+            v1 = sc[3];
+          } else if (tid <= B) {   // U(k, k+t) and U(k+1, k+1+t): physical columns j and j + 1
+            int j1 = j + 1;
+            j1 -= j1 >= P ? P : 0;
+            v0 = tid == 1 ? ukk1 : u0_s[j];
+            v1 = fma(-l10, u0_s[j1], u1_s[j1]);
+          } else {                 // L(k+t, k) and L(k+1+t, k+1): physical rows j and j + 1
+            int j1 = j + 1;
+            j1 -= j1 >= P ? P : 0;
+            v0 = tid == B + 1 ? l10 : a0_s[j] * r0;
+            v1 = fma(-a0_s[j1] * r0, ukk1, a1_s[j1]) * r1;
+          }
+          lu[(int64_t)k * W + tid] = v0;
+          if (live1) lu[(int64_t)(k + 1) * W + tid] = v1;
+        }
+      }
+      // d) the retiring physical rows/columns pk, pk+1 take the entering rows/columns k+P, k+P+1
+      //    (rows u, u+1 of the group's set), in that order
+#pragma unroll
+      for (int h = 0; h < 2; h++) {
+        const double *db = dset + (u + h) * W;
+        const int pkh = pk + h;
+        const int pk1 = pkh + 1 == P ? 0 : pkh + 1;
+        const int rh = rr + h, ch = cc + h;
+        if (colown) {
+          int o = pr0 - pk1;
+          o += o < 0 ? P : 0;
+#pragma unroll
+          for (int r = 0; r < kBandR; r++) {
+            const int orr = o + r >= P ? o + r - P : o + r;
+            if (!(rowown && r == rh)) cell[r][ch] = db[B + 1 + orr];
+          }
+        }
+        if (rowown) {
+          int o = pc0 - pk1;
+          o += o < 0 ? P : 0;
+#pragma unroll
+          for (int c = 0; c < kBandC; c++) {
+            const int oc = o + c >= P ? o + c - P : o + c;
+            cell[rh][c] = db[oc];
+          }
+        }
+      }
+    }
+    pkb += 8;
+    pkb -= pkb == P ? P : 0;
+  }
+}
+
 // One warp per (batch item, species block): x = U^-1 L^-1 (P b) in the RCM order, un-permuted on
 // the way out.  y lives in shared memory; the factor rows stream through a per-warp cp.async ring
 // kBandD steps ahead (each step is a short dependent chain, so the loads must not sit on it).

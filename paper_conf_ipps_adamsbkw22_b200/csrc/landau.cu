@@ -1330,16 +1330,31 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
     const char *e = getenv("LANDAU_BAND_MINB");
     return e ? atoi(e) : 2;
   }();
-  if (maxPp <= 88) {   // 4 x 8 tiles, <= 242 threads, two CTAs per SM (128 registers) or one
-    auto k = band_minb >= 2 ? band_lu_kernel<4, 8, 2> : band_lu_kernel<4, 8, 1>;
-    if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    k<<<grid, threads_lu, smem, h->stream>>>(
-        h->d_Aent, h->ent_bstride, h->d_band, h->band_bstride, h->d_band_desc, h->S);
-  } else {             // 8 x 8 tiles, <= 256 threads
-    auto k = band_lu_kernel<8, 8, 1>;
-    if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    k<<<grid, threads_lu, smem, h->stream>>>(
-        h->d_Aent, h->ent_bstride, h->d_band, h->band_bstride, h->d_band_desc, h->S);
+  static const int band_rank = [] {   // 2: two elimination steps per barrier (band_lu2_kernel)
+    const char *e = getenv("LANDAU_BAND_RANK");
+    return e ? atoi(e) : 2;
+  }();
+  const size_t smem2 = sizeof(double) * (2 * (4 * maxPp + 8) + 24 * W) + sizeof(int32_t) * (maxn + 1) +
+                       sizeof(uint16_t) * maxent;
+  const void *kfn;
+  size_t ksmem = smem;
+  if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
+    kfn = band_rank == 2 ? (band_minb >= 2 ? (const void *)band_lu2_kernel<4, 8, 2> : (const void *)band_lu2_kernel<4, 8, 1>)
+                         : (band_minb >= 2 ? (const void *)band_lu_kernel<4, 8, 2> : (const void *)band_lu_kernel<4, 8, 1>);
+  else               // 8 x 8 tiles, <= 256 threads
+    kfn = band_rank == 2 ? (const void *)band_lu2_kernel<8, 8, 1> : (const void *)band_lu_kernel<8, 8, 1>;
+  if (band_rank == 2) ksmem = smem2;
+  if (ksmem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
+  if (ksmem > 48 * 1024) CU(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ksmem));
+  {
+    const double *a0 = h->d_Aent;
+    int64_t a1 = h->ent_bstride;
+    double *a2 = h->d_band;
+    int64_t a3 = h->band_bstride;
+    const BandDesc *a4 = h->d_band_desc;
+    int a5 = h->S;
+    void *args[] = {&a0, &a1, &a2, &a3, &a4, &a5};
+    CU(cudaLaunchKernel(kfn, dim3(grid), dim3(threads_lu), args, ksmem, h->stream));
   }
   h->launches++;
   h->tlaunch[LANDAU_T_FACTOR]++;
