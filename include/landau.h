@@ -168,7 +168,9 @@ int landau_get_launch_count(landau_t h, int64_t *count);
  *   [G_Drr; G_Drz; G_Dzz] = [U^D_rr; U^D_rz; U^D_zz] (3N x N) . W_D (N x batch)
  *   G_Kr = [U^K_rr  U^D_rz] (N x 2N) . [W_Kr; W_Kz],   G_Kz = [U^K_zr  U^D_zz] . [W_Kr; W_Kz].
  * The same sums as the pairwise kernels up to summation order.  EUNSUPPORTED for element-split
- * handles or when 7 N^2 doubles exceed 16 GiB; enable = 0 frees the cache. */
+ * handles or when 7 N^2 doubles exceed 16 GiB; enable = 0 frees the cache.  enable = 2 keeps the
+ * GEMM formulation but re-evaluates the tensors (every ordered pair) at every build: the cost of a
+ * build that shares nothing with the previous one. */
 int landau_set_tensor_cache(landau_t h, int32_t enable);
 
 /* NEXT-2 (PAPER.md:1@24330-26180, §III-G): the paper's direct solver for the implicit

@@ -88,6 +88,7 @@ struct landau_s {
   bool coincident = false;   // two distinct quadrature points with identical (r, z) (never for one grid)
   // tensor cache (NEXT-4)
   bool tcache = false, tcache_valid = false;
+  bool tcache_recompute = false;   // landau_set_tensor_cache(h, 2): evaluate the tensors in every build
   double *d_U = nullptr;     // A1 (3N^2) | A2 (2N^2) | A3 (2N^2)
   cublasHandle_ cublas = nullptr;
   // band solver (NEXT-2)
@@ -338,7 +339,7 @@ int launch_inner(landau_t h, int64_t nbatch) {
   const int64_t t0 = h->e0 * P.nqp, nt = (h->e1 - h->e0) * P.nqp;
   if (h->tcache) {   // NEXT-4: cached tensors, three FP64 GEMMs
     const int64_t n2 = N * N;
-    if (!h->tcache_valid) {
+    if (!h->tcache_valid || h->tcache_recompute) {
       dim3 grid((unsigned)((N + 127) / 128), (unsigned)N);
       tensor_fill_kernel<<<grid, 128, 0, h->stream>>>(N, h->d_r, h->d_z, h->d_U, h->d_U + 3 * n2, h->d_U + 5 * n2);
       h->launches++;
@@ -1258,7 +1259,11 @@ int landau_set_tensor_cache(landau_t h, int32_t enable) {
     h->tcache = h->tcache_valid = false;
     return LANDAU_OK;
   }
-  if (h->tcache) return LANDAU_OK;
+  if (h->tcache) {
+    if (h->tcache_recompute != (enable == 2)) drop_graphs(h);
+    h->tcache_recompute = enable == 2;
+    return LANDAU_OK;
+  }
   const int64_t N = h->plan.npts;
   if (h->world > 1 || h->Nc != N) return fail(h, LANDAU_EUNSUPPORTED, "tensor cache needs all targets on one GPU");
   if (7 * N * N * (int64_t)sizeof(double) > (16LL << 30)) return fail(h, LANDAU_EUNSUPPORTED, "tensor cache > 16 GiB");
@@ -1272,6 +1277,7 @@ int landau_set_tensor_cache(landau_t h, int32_t enable) {
   drop_graphs(h);
   h->tcache = true;
   h->tcache_valid = false;
+  h->tcache_recompute = enable == 2;
   return LANDAU_OK;
 }
 

@@ -318,7 +318,9 @@ class Landau:
         self._check(lib().landau_set_mirror(self._h, int(bool(enable))), "landau_set_mirror")
 
     def set_tensor_cache(self, enable=True):
-        self._check(lib().landau_set_tensor_cache(self._h, int(bool(enable))), "landau_set_tensor_cache")
+        """True: cache the tensors across builds; "recompute": GEMM path, tensors evaluated every build."""
+        mode = 2 if enable == "recompute" else int(bool(enable))
+        self._check(lib().landau_set_tensor_cache(self._h, mode), "landau_set_tensor_cache")
 
     def stats(self):
         st = _Stats()

@@ -407,6 +407,9 @@ def test_tensor_cache_gemm_path_C4():
         assert np.all(np.abs(Jc[k] - Jo) <= 1e-11 * Ja)
     h.jacobian_batched(out)      # cached tensors reused: bitwise repeatable
     assert np.array_equal(out.cpu().numpy().view(np.uint64), Jc.view(np.uint64))
+    h.set_tensor_cache("recompute")   # tensors re-evaluated in the build: the same values
+    h.jacobian_batched(out)
+    assert np.array_equal(out.cpu().numpy().view(np.uint64), Jc.view(np.uint64))
     h.set_tensor_cache(False)
     h.jacobian_batched(out)
     assert h.stats()["inner_path"] in (1, 3)
