@@ -150,6 +150,7 @@ FLOP_PER_PAIR_SYMMETRIC = 193.0
 # mirror-symmetric kernel: FP64 FLOP (2 DFMA + DMUL + DADD, ncu SASS counts on C4) per tensor
 # evaluation, (N/2)^2 evaluations per batch item (profiles/r01_flops_mirror.csv)
 FLOP_PER_EVAL_MIRROR = 223.9
+FLOP_PER_EVAL_VTX = 219.3   # inner_vtx_kernel, ncu SASS counts (profiles/r01_vtx_ncu.txt)
 
 
 def cpu_baseline(args, desc, nsample):
@@ -342,8 +343,8 @@ def main():
     if st["inner_path"] == 2:   # GEMMs: 2 FLOP per multiply-add, 7 N^2 per batch item (three DGEMMs)
         flop_per_pair = 14.0
         flops_per_launch = 14.0 * st["nbatch"] * N * N
-    elif st["inner_path"] == 3:
-        flop_per_pair = FLOP_PER_EVAL_MIRROR
+    elif st["inner_path"] in (3, 4):
+        flop_per_pair = FLOP_PER_EVAL_VTX if st["inner_path"] == 4 else FLOP_PER_EVAL_MIRROR
         flops_per_launch = flop_per_pair * st["nbatch"] * (N // 2) ** 2
     elif st["inner_path"] == 1:
         flop_per_pair = FLOP_PER_PAIR_SYMMETRIC
@@ -357,13 +358,14 @@ def main():
     sm_max = clocks["sm_max_mhz"] or 1965.0
     peak = fp64_peak_tflops(props, sm_max)
     step_ms_lib = sum(v[0] for v in tim.values()) / args.steps
-    roof = {"bound": "alu", "kernel": "inner_mir_kernel / inner_sym_kernel / inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
+    roof = {"bound": "alu", "kernel": "inner_vtx_kernel / inner_mir_kernel / inner_sym_kernel / inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
             "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None,
             "traffic": load_profile_traffic(args.workload),
             "peak_note": f"derived FP64 DFMA peak: {props.multi_processor_count} SMs x 64 lanes x 2 FLOP x {sm_max:.0f} MHz",
             "inner_path": ["directed (ordered pairs)", "symmetric (unordered pairs)",
                            "tensor cache + FP64 DGEMM (cuBLAS)",
-                           "mirror-symmetric (one tensor per unordered pair and its z-mirror)"][st["inner_path"]],
+                           "mirror-symmetric (one tensor per unordered pair and its z-mirror)",
+                           "mirror-symmetric, one CTA per vertex (sums in shared memory)"][st["inner_path"]],
             "flop_per_pair": flop_per_pair, "flops_per_launch": flops_per_launch,
             "inner_ms_per_launch": inner_avg_s * 1e3,
             "inner_share_of_step": (inner_ms / args.steps) / ms_per_step if ms_per_step else None,
@@ -486,7 +488,7 @@ def main():
             ms2 = sum(a.elapsed_time(b) for a, b in ev2) / args.steps
             line["c2_single_build"] = {"value": 1e3 / ms2, "unit": UNIT, "ms_per_step": ms2,
                                        "pairs_per_s": 1e3 / ms2 * p2.npoints ** 2,
-                                       "inner_path": ["directed", "symmetric", "tensor cache", "mirror"][h2.stats()["inner_path"]],
+                                       "inner_path": ["directed", "symmetric", "tensor cache", "mirror", "mirror per-vertex"][h2.stats()["inner_path"]],
                                        "note": "BASELINE configs[1]: one e+D Q3 AMR grid (N=1088) per step, "
                                                "set_state + jacobian (CSR) + mass, CUDA-graph replay"}
             h2.close()

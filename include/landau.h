@@ -217,8 +217,13 @@ int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double E
  * reflection keeps lambda+-, x, m and every azimuthal integral and negates the rz / zr components,
  * U(i', j') = F U(i, j) F with F = diag(1, -1), on top of the i <-> j symmetry (N^2/4 tensor
  * evaluations per build instead of N^2/2).  The mirror point is placed at exactly (r, -z), a
- * perturbation within the 1e-12 R detection tolerance.  On by default when available;
- * enable = 0 selects the plain symmetric kernel, enable = 1 on a non-symmetric mesh is EUNSUPPORTED. */
+ * perturbation within the 1e-12 R detection tolerance.  On by default when available.
+ * enable: 0 = plain symmetric kernel; 1 = mirror, automatic (batches of at least one vertex per SM run
+ * whole waves of the per-vertex kernel -- one CTA per batch item, sums in shared memory, no partial
+ * slots -- and a remainder below 0.9 of a wave on the slot kernel); 2 = mirror slot kernel only;
+ * 3 = per-vertex kernel for every batch size.  enable != 0 on a non-symmetric mesh, or 3 when a
+ * vertex's sums (80 B per upper-half point) exceed 160 KB of shared memory, is EUNSUPPORTED;
+ * enable outside 0..3 is EINVAL. */
 int landau_set_mirror(landau_t h, int32_t enable);
 
 /* How the last build ran (for FLOP accounting and diagnostics). */
@@ -226,7 +231,8 @@ typedef struct {
   int32_t inner_path;        /* 0: directed pair kernel (every ordered pair, split-j when small);
                                 1: symmetric pair kernel (every unordered pair once, both targets);
                                 2: tensor cache + FP64 GEMM (landau_set_tensor_cache);
-                                3: mirror-symmetric pair kernel (landau_set_mirror)                */
+                                3: mirror-symmetric pair kernel (landau_set_mirror)
+                                4: mirror-symmetric per-vertex kernel (+ slot kernel for a remainder) */
   int64_t nbatch;            /* batch items of the last build                                      */
   int64_t targets;           /* target points per batch item (all N unless element-split)          */
   int64_t sources;           /* source points per batch item (N)                                   */

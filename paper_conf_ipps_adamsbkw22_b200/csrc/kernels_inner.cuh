@@ -482,6 +482,185 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_mir_kernel(int64_t
   }
 }
 
+// ------------------------------------------------------------------------------------------------
+// N2 (mirror-symmetric, one CTA per batch item): for batches of small meshes (C4) the whole G of a
+// vertex fits in shared memory (Ga, Gb: 80 B per upper-half point), so a persistent CTA owns one
+// vertex at a time and accumulates there -- no partial slots in HBM and no reduction kernel.
+// Work items are tile pairs (a, b), each evaluating BOTH tensors of every (i in a, j in b): the
+// same-side U(i, j) and the cross V(i, j) = U(i, j') -- two independent pair chains per lane that
+// share the j-tile staging and the reverse-sum shuffles, with one set of accumulators: forward
+// Ga(i) += U A(j) + V F Bf(j), Gb(i) += U Bf(j) + V F A(j); reverse (F-flipped for V, see
+// inner_mir_kernel) Ga(j) += rev(U) A(i) + F rev(V) Bf(i), Gb(j) += rev(U) Bf(i) + F rev(V) A(i).
+// The host schedules the items in rounds whose tile sets are disjoint (round-robin tournament of
+// the tiles, then rounds of diagonal items), so the warps of a CTA add their sums into shared memory
+// without atomics and every target's partial sums arrive in a fixed order: bitwise reproducible.
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ void acc_rev_flip(Acc5 &a, double Vdrr, double Udrz, double Udzz, double Ukrr, double Ukzr,
+                                             double wd, double wkr, double wkz) {
+  a.drr = fma(wd, Vdrr, a.drr);
+  a.drz = fma(-wd, Ukzr, a.drz);
+  a.dzz = fma(wd, Udzz, a.dzz);
+  a.kr = fma(Ukrr, wkr, fma(Ukzr, wkz, a.kr));
+  a.kz = fma(-Udrz, wkr, fma(-Udzz, wkz, a.kz));
+}
+
+// one U+V step of lane target (r, z) against j-data (rj, zj, rj2, A(j), Bf(j)); i weights A(i), Bf(i)
+// mf: forward mask, mr: reverse mask (U part); mvf / mvr: the V part's masks
+template <bool MASK>
+__device__ __forceinline__ void vtx_step(double r, double z, double r2, const double Ai[3], const double Bi[3],
+                                         double rj, double zj, double rj2, double2 a01, double2 a2b0, double2 b12,
+                                         const PairCoef &cf, double mu_f, double mu_r, double mv_f, double mv_r,
+                                         Acc5 &ga, Acc5 &gb, Acc5 &ja, Acc5 &jb) {
+  bool oku, okv;
+  double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
+  double Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, Ydrr;
+  pair_tensors<MASK>(r, z, r2, rj, zj, rj2, cf, oku, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
+  pair_tensors<MASK>(r, z, r2, rj, -zj, rj2, cf, okv, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, Ydrr);
+  if (MASK) {
+    mu_f = oku ? mu_f : 0.0;
+    mu_r = oku ? mu_r : 0.0;
+    mv_f = okv ? mv_f : 0.0;
+    mv_r = okv ? mv_r : 0.0;
+  }
+  // U: sources A(j) -> Ga, Bf(j) -> Gb; reverse A(i) -> Ga(j), Bf(i) -> Gb(j)
+  acc_fwd(ga, Udrr, Udrz, Udzz, Ukrr, Ukzr, mu_f * a01.x, mu_f * a01.y, mu_f * a2b0.x);
+  acc_fwd(gb, Udrr, Udrz, Udzz, Ukrr, Ukzr, mu_f * a2b0.y, mu_f * b12.x, mu_f * b12.y);
+  acc_rev(ja, Vdrr, Udrz, Udzz, Ukrr, Ukzr, mu_r * Ai[0], mu_r * Ai[1], mu_r * Ai[2]);
+  acc_rev(jb, Vdrr, Udrz, Udzz, Ukrr, Ukzr, mu_r * Bi[0], mu_r * Bi[1], mu_r * Bi[2]);
+  // V (source j' at (rj, -zj)): F Bf(j) -> Ga, F A(j) -> Gb; reverse F rev(V) Bf(i) -> Ga(j), F rev(V) A(i) -> Gb(j)
+  acc_fwd(ga, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, mv_f * a2b0.y, mv_f * b12.x, -mv_f * b12.y);
+  acc_fwd(gb, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, mv_f * a01.x, mv_f * a01.y, -mv_f * a2b0.x);
+  acc_rev_flip(ja, Ydrr, Xdrz, Xdzz, Xkrr, Xkzr, mv_r * Bi[0], mv_r * Bi[1], mv_r * Bi[2]);
+  acc_rev_flip(jb, Ydrr, Xdrz, Xdzz, Xkrr, Xkzr, mv_r * Ai[0], mv_r * Ai[1], mv_r * Ai[2]);
+}
+
+__device__ __forceinline__ void vtx_add(double *sG, int64_t Hp, int64_t pos, const Acc5 &a) {
+  sG[pos] += a.drr;
+  sG[Hp + pos] += a.drz;
+  sG[2 * Hp + pos] += a.dzz;
+  sG[3 * Hp + pos] += a.kr;
+  sG[4 * Hp + pos] += a.kz;
+}
+
+// one (a, b) item of a vertex; s_j: the warp's staged j-tile b as (r, z), A01, (A2, Bf0), Bf12, (r^2, -);
+// sGa, sGb: the CTA's shared accumulators [5][Hp]
+template <bool DIAG, bool MASK>
+__device__ __forceinline__ void vtx_run(int a, int b, const double *rU, const double *zU, const double *wb, int64_t N,
+                                        int64_t H, int64_t Hp, const int32_t *pu, const int32_t *pm, int lane,
+                                        const double2 *s_j, const PairCoef &cf, double *sGa, double *sGb) {
+  const int64_t i = (int64_t)a * 32 + lane;
+  double Ai[3], Bi[3];
+  mir_weights(wb, N, H, pu, pm, i, Ai, Bi);
+  const double r = i < H ? rU[i] : 1.0;
+  const double z = i < H ? zU[i] : 1.0e6 + lane;   // padding: far away, zero weights
+  const double r2 = r * r;
+  Acc5 ga{0.0, 0.0, 0.0, 0.0, 0.0}, gb{0.0, 0.0, 0.0, 0.0, 0.0};
+  Acc5 ja{0.0, 0.0, 0.0, 0.0, 0.0}, jb{0.0, 0.0, 0.0, 0.0, 0.0};
+  const int src = (lane + 1) & 31;
+  if constexpr (DIAG) {   // step 0: each point with its own mirror (V forward only; U is the self pair)
+    const double2 rz = s_j[lane * 5], a01 = s_j[lane * 5 + 1], a2b0 = s_j[lane * 5 + 2], b12 = s_j[lane * 5 + 3],
+                  rr2 = s_j[lane * 5 + 4];
+    double Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, Ydrr;
+    bool okv;
+    pair_tensors<MASK>(r, z, r2, rz.x, -rz.y, rr2.x, cf, okv, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, Ydrr);
+    const double mv = (!MASK || okv) ? 1.0 : 0.0;
+    acc_fwd(ga, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, mv * a2b0.y, mv * b12.x, -mv * b12.y);
+    acc_fwd(gb, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, mv * a01.x, mv * a01.y, -mv * a2b0.x);
+  }
+  constexpr int k0 = DIAG ? 1 : 0, kmain = DIAG ? 16 : 32;
+#pragma unroll kMirUnroll
+  for (int k = k0; k < kmain; k++) {
+    const int jj = (lane + k) & 31;
+    const double2 rz = s_j[jj * 5], a01 = s_j[jj * 5 + 1], a2b0 = s_j[jj * 5 + 2], b12 = s_j[jj * 5 + 3],
+                  rr2 = s_j[jj * 5 + 4];
+    vtx_step<MASK>(r, z, r2, Ai, Bi, rz.x, rz.y, rr2.x, a01, a2b0, b12, cf, 1.0, 1.0, 1.0, 1.0, ga, gb, ja, jb);
+    acc_shfl(ja, src);
+    acc_shfl(jb, src);
+  }
+  if constexpr (DIAG) {   // step 16: lanes >= 16 would double-count
+    const int jj = (lane + 16) & 31;
+    const double2 rz = s_j[jj * 5], a01 = s_j[jj * 5 + 1], a2b0 = s_j[jj * 5 + 2], b12 = s_j[jj * 5 + 3],
+                  rr2 = s_j[jj * 5 + 4];
+    const double m = lane < 16 ? 1.0 : 0.0;
+    vtx_step<true>(r, z, r2, Ai, Bi, rz.x, rz.y, rr2.x, a01, a2b0, b12, cf, m, m, m, m, ga, gb, ja, jb);
+    acc_shfl(ja, src);
+    acc_shfl(jb, src);
+  }
+  vtx_add(sGa, Hp, i, ga);
+  vtx_add(sGb, Hp, i, gb);
+  if constexpr (DIAG) __syncwarp();   // forward and reverse sums of a diagonal item hit the same tile
+  // after the last hand-over lane L holds the reverse sums of j = (L + kend) mod 32
+  const int kend = DIAG ? 17 : 32;
+  const int64_t jf = (int64_t)b * 32 + ((lane + kend) & 31);
+  vtx_add(sGa, Hp, jf, ja);
+  vtx_add(sGb, Hp, jf, jb);
+}
+
+struct VtxItem {   // host-built: tiles (a, b) of the upper half; a == b: the diagonal item
+  int a, b;
+};
+
+template <bool MASK>
+__global__ void __launch_bounds__(32 * kSymWarps, 1) inner_vtx_kernel(int64_t N, int64_t H, int nrounds,
+                                                                      const int32_t *__restrict__ round_ptr,
+                                                                      const VtxItem *__restrict__ items,
+                                                                      const double *__restrict__ rU,
+                                                                      const double *__restrict__ zU,
+                                                                      const int32_t *__restrict__ pu,
+                                                                      const int32_t *__restrict__ pm,
+                                                                      const double *__restrict__ wT, int nbatch,
+                                                                      double *__restrict__ G, int64_t G_bstride) {
+  __shared__ double2 s_j[kSymWarps][32 * 5];
+  __shared__ double s_coef[kNumPairCoef];
+  __shared__ double2 s_ltab[kLogTab];
+  extern __shared__ double s_G[];   // Ga [5][Hp], Gb [5][Hp]
+  const int64_t Hp = (H + 31) / 32 * 32;
+  double *sGa = s_G, *sGb = s_G + 5 * Hp;
+  stage_pair_coef(s_coef, s_ltab);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, s_ltab, cf);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (int bb = blockIdx.x; bb < nbatch; bb += gridDim.x) {
+    const double *wb = wT + (int64_t)bb * 3 * N;
+    for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) s_G[k] = 0.0;
+    __syncthreads();
+    for (int rd = 0; rd < nrounds; rd++) {
+      for (int q = round_ptr[rd] + wid; q < round_ptr[rd + 1]; q += kSymWarps) {
+        const VtxItem it = items[q];
+        __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
+        {
+          const int64_t j = (int64_t)it.b * 32 + lane;
+          double A[3], Bf[3];
+          mir_weights(wb, N, H, pu, pm, j, A, Bf);
+          const double r = j < H ? rU[j] : 1.0;
+          const double z = j < H ? zU[j] : 2.0e6 + lane;
+          double2 *d = &s_j[wid][lane * 5];
+          d[0] = make_double2(r, z);
+          d[1] = make_double2(A[0], A[1]);
+          d[2] = make_double2(A[2], Bf[0]);
+          d[3] = make_double2(Bf[1], Bf[2]);
+          d[4] = make_double2(r * r, 0.0);
+        }
+        __syncwarp();
+        if (it.a == it.b)
+          vtx_run<true, MASK>(it.a, it.b, rU, zU, wb, N, H, Hp, pu, pm, lane, s_j[wid], cf, sGa, sGb);
+        else
+          vtx_run<false, MASK>(it.a, it.b, rU, zU, wb, N, H, Hp, pu, pm, lane, s_j[wid], cf, sGa, sGb);
+      }
+      __syncthreads();   // the next round's tiles may be this round's
+    }
+    double *Gb = G + (int64_t)bb * G_bstride;
+    for (int64_t k = threadIdx.x; k < 5 * H; k += blockDim.x) {
+      const int64_t c = k / H, u = k % H;
+      Gb[c * N + pu[u]] = sGa[c * Hp + u];
+      const double v = sGb[c * Hp + u];
+      Gb[c * N + pm[u]] = (c == 1 || c == 4) ? -v : v;
+    }
+    __syncthreads();   // the write-out reads s_G before the next vertex zeroes it
+  }
+}
+
 // G[b][c][pu(u)] = sum of the Ga parts, G[b][c][pm(u)] = F (sum of the Gb parts), over the slots of
 // u's tile in the fixed order of tile_slots
 __global__ void reduce_mir_kernel(int64_t N, int64_t H, int64_t nslots, const int32_t *__restrict__ tile_ptr,

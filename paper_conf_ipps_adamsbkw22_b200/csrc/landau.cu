@@ -80,7 +80,13 @@ struct landau_s {
   // original indices pu and mirrors pm, work items and slot map over the tiles of the upper half
   bool mirror = false;     // the mesh is mirror-symmetric (maps built)
   bool mirror_on = true;   // use inner_mir_kernel when the symmetric path runs (landau_set_mirror)
+  int mirror_mode = 1;     // 1: auto (per-vertex kernel for large batches), 2: slot kernel, 3: per-vertex kernel
   int64_t H = 0, nmir_items = 0, nmir_slots = 0;
+  // per-vertex mirror kernel (inner_vtx_kernel): round schedule of tile-pair items
+  VtxItem *d_vtx_items = nullptr;
+  int32_t *d_vtx_round_ptr = nullptr;
+  int nvtx_rounds = 0;
+  size_t vtx_smem = 0;     // dynamic shared memory (Ga, Gb); 0 when the vertex does not fit
   double *d_rU = nullptr, *d_zU = nullptr;
   int32_t *d_pu = nullptr, *d_pm = nullptr;
   MirItem *d_mir_items = nullptr;
@@ -278,6 +284,15 @@ bool mirror_enabled() {
   return v;
 }
 
+// per-vertex mirror kernel when the batch gives every SM at least this many vertices (LANDAU_VTX_MIN_BATCH_PER_SM)
+int64_t vtx_min_batch_per_sm() {
+  static const int64_t v = [] {
+    const char *e = getenv("LANDAU_VTX_MIN_BATCH_PER_SM");
+    return e ? (int64_t)atoll(e) : (int64_t)1;
+  }();
+  return v;
+}
+
 // inner-kernel variant (targets per thread, min blocks per SM); LANDAU_INNER_VARIANT overrides
 int inner_variant() {
   static const int v = [] {
@@ -390,32 +405,72 @@ int launch_inner(landau_t h, int64_t nbatch) {
   } else {
     h->stats.pair_evaluations = ip.wtiles * 32 * ip.tpt * N;
   }
-  if (ip.sym && h->mirror && h->mirror_on) {
-    {
-      Timer t(h, LANDAU_T_INNER);
-      const int64_t nitems = nbatch * h->nmir_items;
-      const unsigned grid = (unsigned)std::min<int64_t>((nitems + kSymWarps - 1) / kSymWarps, (int64_t)LANDAU_SYM_MINB * num_sms(h));
-      if (h->coincident)
-        inner_mir_kernel<LANDAU_SYM_MINB, true><<<grid, 32 * kSymWarps, 0, h->stream>>>(
-            N, h->H, h->nmir_items, h->nmir_slots, nitems, h->d_mir_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
-            h->d_part);
-      else
-        inner_mir_kernel<LANDAU_SYM_MINB, false><<<grid, 32 * kSymWarps, 0, h->stream>>>(
-            N, h->H, h->nmir_items, h->nmir_slots, nitems, h->d_mir_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
-            h->d_part);
-      h->launches++;
-      h->tlaunch[LANDAU_T_INNER]++;
-      KCHECK();
-    }
+  // mirror slot kernel over batch items [b0, b0 + nb): partial slots, then their reduction
+  auto mir_slots = [&](int64_t b0, int64_t nb) -> int {
+    const int64_t nitems = nb * h->nmir_items;
+    const double *wT = h->d_wT + b0 * 3 * N;
+    const unsigned grid = (unsigned)std::min<int64_t>((nitems + kSymWarps - 1) / kSymWarps, (int64_t)LANDAU_SYM_MINB * num_sms(h));
+    if (h->coincident)
+      inner_mir_kernel<LANDAU_SYM_MINB, true><<<grid, 32 * kSymWarps, 0, h->stream>>>(
+          N, h->H, h->nmir_items, h->nmir_slots, nitems, h->d_mir_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, wT, h->d_part);
+    else
+      inner_mir_kernel<LANDAU_SYM_MINB, false><<<grid, 32 * kSymWarps, 0, h->stream>>>(
+          N, h->H, h->nmir_items, h->nmir_slots, nitems, h->d_mir_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, wT, h->d_part);
+    h->launches++;
+    KCHECK();
+    return LANDAU_OK;
+  };
+  auto mir_reduce = [&](int64_t b0, int64_t nb) -> int {
     Timer t(h, LANDAU_T_REDUCE);
-    const int64_t total = nbatch * 5 * h->H;
+    const int64_t total = nb * 5 * h->H;
     const int blocks = (int)std::min<int64_t>((total + 255) / 256, 16LL * num_sms(h));
     reduce_mir_kernel<<<blocks, 256, 0, h->stream>>>(N, h->H, h->nmir_slots, h->d_mtile_ptr, h->d_mtile_slots, h->d_pu,
-                                                     h->d_pm, h->d_part, G_own, 5 * h->Nc, (int)nbatch);
+                                                     h->d_pm, h->d_part, G_own + b0 * 5 * h->Nc, 5 * h->Nc, (int)nb);
     h->launches++;
     h->tlaunch[LANDAU_T_REDUCE]++;
     KCHECK();
     return LANDAU_OK;
+  };
+  if (h->mirror && h->mirror_on && h->vtx_smem &&
+      (h->mirror_mode == 3 || (h->mirror_mode == 1 && ip.sym && nbatch >= vtx_min_batch_per_sm() * num_sms(h)))) {
+    // one CTA per vertex, sums in shared memory (no slots, no reduction kernel).  Auto mode runs
+    // whole waves of vertices this way and hands a remainder below 0.9 of a wave to the slot kernel,
+    // which spreads its items over every SM (a partial wave would leave SMs idle).
+    const int64_t T = (h->H + 31) / 32, S = num_sms(h);
+    h->stats.pair_evaluations = T * 33 * 32 + 2 * (T * (T - 1) / 2) * 32 * 32;
+    h->stats.nsplit = 1;
+    h->stats.inner_path = 4;
+    int64_t nv = nbatch;
+    if (h->mirror_mode == 1) {
+      const int64_t rem = nbatch % S;
+      if (rem && rem * 10 < 9 * S) nv = nbatch - rem;
+    }
+    {
+      Timer t(h, LANDAU_T_INNER);
+      const unsigned grid = (unsigned)std::min<int64_t>(nv, S);
+      if (h->coincident)
+        inner_vtx_kernel<true><<<grid, 32 * kSymWarps, h->vtx_smem, h->stream>>>(
+            N, h->H, h->nvtx_rounds, h->d_vtx_round_ptr, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
+            (int)nv, G_own, 5 * h->Nc);
+      else
+        inner_vtx_kernel<false><<<grid, 32 * kSymWarps, h->vtx_smem, h->stream>>>(
+            N, h->H, h->nvtx_rounds, h->d_vtx_round_ptr, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
+            (int)nv, G_own, 5 * h->Nc);
+      h->launches++;
+      h->tlaunch[LANDAU_T_INNER]++;   // one inner stage per build (the remainder's kernel is part of it)
+      KCHECK();
+      if (nv < nbatch && (rc = mir_slots(nv, nbatch - nv))) return rc;
+    }
+    if (nv < nbatch) return mir_reduce(nv, nbatch - nv);
+    return LANDAU_OK;
+  }
+  if (ip.sym && h->mirror && h->mirror_on) {
+    {
+      Timer t(h, LANDAU_T_INNER);
+      if ((rc = mir_slots(0, nbatch))) return rc;
+      h->tlaunch[LANDAU_T_INNER]++;
+    }
+    return mir_reduce(0, nbatch);
   }
   if (ip.sym) {
     {
@@ -864,6 +919,36 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
         tslots.insert(tslots.end(), slots_of[t].begin(), slots_of[t].end());
         tptr.push_back((int32_t)tslots.size());
       }
+      // per-vertex kernel schedule: round-robin tournament of the T tiles (circle method; rounds of
+      // disjoint tile pairs), then the diagonal items in rounds of kSymWarps
+      std::vector<VtxItem> vitems;
+      std::vector<int32_t> vround(1, 0);
+      {
+        const int Tp = T + (T & 1);
+        for (int rd = 0; rd + 1 < Tp; rd++) {
+          for (int q = 0; q < Tp / 2; q++) {
+            const int x = q == 0 ? Tp - 1 : (rd + q) % (Tp - 1);
+            const int y = q == 0 ? rd : (rd - q + Tp - 1) % (Tp - 1);
+            if (x < T && y < T) vitems.push_back({std::min(x, y), std::max(x, y)});
+          }
+          if ((int)vitems.size() > vround.back()) vround.push_back((int32_t)vitems.size());
+        }
+        for (int t = 0; t < T; t++) {
+          vitems.push_back({t, t});
+          if ((t + 1) % kSymWarps == 0 || t + 1 == T) vround.push_back((int32_t)vitems.size());
+        }
+      }
+      const size_t vsmem = (size_t)10 * T * 32 * sizeof(double);
+      h->vtx_smem = vsmem <= (size_t)160 * 1024 && T >= 2 ? vsmem : 0;
+      h->nvtx_rounds = (int)vround.size() - 1;
+      if (h->vtx_smem) {
+        if ((rc = upload(h, &h->d_vtx_items, vitems)) || (rc = upload(h, &h->d_vtx_round_ptr, vround))) return bail(rc);
+        if (!h->host_only) {
+          cudaError_t e1 = cudaFuncSetAttribute(inner_vtx_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)vsmem);
+          cudaError_t e2 = cudaFuncSetAttribute(inner_vtx_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)vsmem);
+          if (e1 != cudaSuccess || e2 != cudaSuccess) return bail(fail(h, LANDAU_ECUDA, "inner_vtx_kernel smem attribute"));
+        }
+      }
       h->mirror = true;
       h->H = H;
       h->nmir_items = (int64_t)items.size();
@@ -978,6 +1063,8 @@ void landau_destroy(landau_t h) {
   cudaFree(h->d_pu);
   cudaFree(h->d_pm);
   cudaFree(h->d_mir_items);
+  cudaFree(h->d_vtx_items);
+  cudaFree(h->d_vtx_round_ptr);
   cudaFree(h->d_mtile_ptr);
   cudaFree(h->d_mtile_slots);
   cudaFree(h->d_ext_ptr);
@@ -1242,9 +1329,12 @@ int landau_get_timing(landau_t h, double *ms, int64_t *launches) {
 
 int landau_set_mirror(landau_t h, int32_t enable) {
   if (!h) return LANDAU_EINVAL;
+  if (enable < 0 || enable > 3) return fail(h, LANDAU_EINVAL, "set_mirror: mode must be 0..3");
   if (enable && !h->mirror) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: the mesh is not mirror-symmetric");
+  if (enable == 3 && !h->vtx_smem) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: a vertex does not fit shared memory");
   if (!h->host_only) drop_graphs(h);
   h->mirror_on = enable != 0;
+  h->mirror_mode = enable ? enable : 1;
   return LANDAU_OK;
 }
 

@@ -315,7 +315,12 @@ class Landau:
         return x
 
     def set_mirror(self, enable=True):
-        self._check(lib().landau_set_mirror(self._h, int(bool(enable))), "landau_set_mirror")
+        """False: plain symmetric kernel; True: mirror kernel (auto: per-vertex for large batches);
+        "slots": mirror kernel with HBM partial slots; "vertex": per-vertex mirror kernel."""
+        mode = {"slots": 2, "vertex": 3}.get(enable) if isinstance(enable, str) else int(bool(enable))
+        if mode is None:
+            raise ValueError(f"set_mirror: unknown mode {enable!r}")
+        self._check(lib().landau_set_mirror(self._h, mode), "landau_set_mirror")
 
     def set_tensor_cache(self, enable=True):
         """True: cache the tensors across builds; "recompute": GEMM path, tensors evaluated every build."""

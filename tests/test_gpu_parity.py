@@ -261,7 +261,7 @@ def test_graph_replay_matches_direct_launches():
     assert np.array_equal(b.view(np.uint64), c.view(np.uint64))
 
 
-@pytest.mark.parametrize("mirror", [True, False])
+@pytest.mark.parametrize("mirror", [True, False, "vertex"])
 def test_symmetric_kernel_batch_C4(mirror):
     """A batch large enough for the symmetric inner kernel (each unordered pair evaluated once, both
     targets updated; with mirror=True also each z-mirrored pair from the same tensor): vertices
@@ -280,8 +280,9 @@ def test_symmetric_kernel_batch_C4(mirror):
     h.jacobian_batched(out)
     t = h.get_timing()
     h.set_timing(False)
-    assert t["reduce"][1] == 1    # the symmetric path always reduces its partial slots
-    assert h.stats()["inner_path"] == (3 if mirror else 1)
+    # the slot kernels reduce their partial slots; the per-vertex kernel sums in shared memory
+    assert t["reduce"][1] == (0 if mirror == "vertex" else 1)
+    assert h.stats()["inner_path"] == {True: 3, False: 1, "vertex": 4}[mirror]
     Jb = out.cpu().numpy()
     for k in (0, nb // 2, nb - 1):
         o = Oracle(probs[k])
@@ -346,6 +347,12 @@ def test_symmetric_kernel_with_coincident_points():
     torch.cuda.synchronize()
     assert h.stats()["inner_path"] == 1   # masked plain symmetric kernel
     assert np.abs(out2.cpu().numpy() - Jb).max() <= 1e-13 * np.abs(Jb).max()
+    h.set_mirror("vertex")
+    out3 = torch.empty_like(out)
+    h.jacobian_batched(out3)
+    torch.cuda.synchronize()
+    assert h.stats()["inner_path"] == 4   # masked per-vertex mirror kernel
+    assert np.abs(out3.cpu().numpy() - Jb).max() <= 1e-13 * np.abs(Jb).max()
     for b in (0, nb - 1):
         p = inputs.Problem("twin", 3, prob.grids, prob.species, fmix=[[(1.0 + 0.01 * b, 1.0, 0.0)], [(1.0, 0.5, 0.0)]],
                            seed=99 + b)
@@ -645,3 +652,68 @@ def _mesh_is_mirror(h):
     a = sorted(zip(r, z))
     b = sorted(zip(r, -z))
     return np.allclose(np.array(a), np.array(b), atol=1e-12)
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3"])
+def test_vertex_kernel_point_coeffs(cfg):
+    """Per-vertex mirror kernel (one CTA per batch item, sums in shared memory, round-robin tile
+    schedule) on a ragged tile set (C1: H = 36, two tiles), an odd tile count (C3: 15, three grids)
+    and the C2 mesh (17): point coefficients of every item against the oracle, single items and
+    batches, bitwise reproducible, and equal to the slot kernel up to summation order."""
+    prob, h0, o, fg, fo = setup(cfg)
+    h = L.Landau.from_problem(prob, device=0)
+    h.set_mirror("vertex")
+    Go, Ga = o.point_coeffs(fo)
+    for nb in (1, 5):
+        F = torch.tensor(np.stack([fg * (1.0 + 0.1 * k) for k in range(nb)]), device=DEV)
+        h.set_state_batched(F)
+        G = torch.empty((nb, 5, h.npoints), dtype=torch.float64, device=DEV)
+        h.point_coeffs_batched(G)
+        torch.cuda.synchronize()
+        assert h.stats()["inner_path"] == 4
+        Gn = G.cpu().numpy()
+        for k in range(nb):   # G is linear in f
+            assert np.max(np.abs(Gn[k] - (1.0 + 0.1 * k) * Go) / ((1.0 + 0.1 * k) * Ga)) <= 1e-12, (nb, k)
+        h.point_coeffs_batched(G)
+        assert np.array_equal(G.cpu().numpy().view(np.uint64), Gn.view(np.uint64))
+    h.set_mirror("slots")
+    G2 = torch.empty_like(G)
+    h.point_coeffs_batched(G2)
+    torch.cuda.synchronize()
+    assert np.max(np.abs(G2.cpu().numpy() - Gn) / Ga) <= 1e-13
+    J = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
+    h.set_mirror("vertex")
+    h.jacobian_batched(J)
+    Jo, Ja = o.jacobian(fo)
+    assert np.all(np.abs(J[0].cpu().numpy() - Jo) <= 1e-11 * Ja)
+
+
+def test_vertex_kernel_hybrid_remainder():
+    """Auto mode on a batch of one full wave plus a small remainder (S + 5 vertices, S = SM count):
+    the full wave runs one CTA per vertex, the remainder the slot kernel + reduction.  Vertices on
+    both sides against the oracle, and the whole batch against the slot kernel alone."""
+    S = torch.cuda.get_device_properties(0).multi_processor_count
+    nb = S + 5
+    prob0 = inputs.config4_vertex(0)
+    h = L.Landau.from_problem(prob0, device=0)
+    nodes = h.all_nodes()
+    verts = [(k * 1023) // (nb - 1) for k in range(nb)]
+    F = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in verts]), device=DEV)
+    h.set_state_batched(F)
+    out = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
+    h.set_timing(True)
+    h.jacobian_batched(out)
+    t = h.get_timing()
+    h.set_timing(False)
+    assert h.stats()["inner_path"] == 4
+    assert t["inner"][1] == 1 and t["reduce"][1] == 1   # one inner stage, the remainder reduced
+    Jb = out.cpu().numpy()
+    for k in (0, nb - 1):   # a per-vertex item and a remainder item
+        o = Oracle(inputs.config4_vertex(verts[k]))
+        Jo, Ja = o.jacobian(o.coefficients())
+        assert np.all(np.abs(Jb[k] - Jo) <= 1e-11 * Ja), verts[k]
+    h.set_mirror("slots")
+    out2 = torch.empty_like(out)
+    h.jacobian_batched(out2)
+    assert h.stats()["inner_path"] == 3
+    assert np.abs(out2.cpu().numpy() - Jb).max() <= 1e-13 * np.abs(Jb).max()
