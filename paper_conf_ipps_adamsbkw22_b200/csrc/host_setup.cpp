@@ -94,6 +94,13 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
   plan.tab_phi.resize(nqp * nb);
   plan.tab_dxi.resize(nqp * nb);
   plan.tab_deta.resize(nqp * nb);
+  plan.tab1_L.resize(nq * (p + 1));   // 1-D factors [Gauss point i][node a] (element_sf_kernel)
+  plan.tab1_D.resize(nq * (p + 1));
+  for (int i = 0; i < nq; i++)
+    for (int a = 0; a <= p; a++) {
+      plan.tab1_L[i * (p + 1) + a] = lagrange(p, a, xg[i]);
+      plan.tab1_D[i * (p + 1) + a] = lagrange_d(p, a, xg[i]);
+    }
   for (int qz = 0; qz < nq; qz++)
     for (int qr = 0; qr < nq; qr++)
       for (int b = 0; b <= p; b++)

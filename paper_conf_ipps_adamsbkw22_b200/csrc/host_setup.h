@@ -68,6 +68,8 @@ struct Plan {
   std::vector<double> pr, pz, pw;        // [npts]
   // reference tables at the Gauss points: [nqp][nb]
   std::vector<double> tab_phi, tab_dxi, tab_deta;
+  // their 1-D factors (q = qz * nq + qr, node n = b * (p+1) + a): l_a(x_i), l'_a(x_i) as [i][a]
+  std::vector<double> tab1_L, tab1_D;
   // field extraction per cell-local node: ext_ptr[ncell*nb+1] -> (dof in its grid, weight)
   std::vector<int32_t> ext_ptr, ext_dof;
   std::vector<double> ext_w;

@@ -551,10 +551,21 @@ int launch_element(landau_t h, int64_t nbatch, int64_t b0, int64_t nb) {
 #define LANDAU_EL_EPB16 8
 #endif
   constexpr int EPB = NB == 9 ? 14 : (NB == 16 ? LANDAU_EL_EPB16 : 5);   // ~128 threads per block
-  const int64_t items = (P.ncell + EPB - 1) / EPB * nb;
-  const unsigned grid = (unsigned)std::min<int64_t>(items, 16LL * num_sms(h));
-  element_kernel<NB, S, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, (int)b0, (int)nb,
-                                                                h->d_w, h->d_h, h->d_tab, h->d_C);
+  static const bool sf = [] {
+    const char *e = getenv("LANDAU_ELEMENT_SF");
+    return !(e && atoi(e) == 0);
+  }();
+  if (sf && P.ncell * nb < (1LL << 32)) {   // sum factorisation, one warp per cell
+    const int64_t items = P.ncell * nb;
+    const unsigned grid = (unsigned)std::min<int64_t>((items + kSfWarps - 1) / kSfWarps, 16LL * num_sms(h));
+    element_sf_kernel<S><<<grid, 32 * kSfWarps, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, (int)b0, (int)nb,
+                                                               h->d_w, h->d_h, h->d_tab + 3 * NB * NB, h->d_C);
+  } else {
+    const int64_t items = (P.ncell + EPB - 1) / EPB * nb;
+    const unsigned grid = (unsigned)std::min<int64_t>(items, 16LL * num_sms(h));
+    element_kernel<NB, S, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, (int)b0, (int)nb,
+                                                                  h->d_w, h->d_h, h->d_tab, h->d_C);
+  }
   h->launches++;
   h->tlaunch[LANDAU_T_ELEMENT]++;
   KCHECK();
@@ -820,6 +831,8 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     std::vector<double> tab(P.tab_phi);
     tab.insert(tab.end(), P.tab_dxi.begin(), P.tab_dxi.end());
     tab.insert(tab.end(), P.tab_deta.begin(), P.tab_deta.end());
+    tab.insert(tab.end(), P.tab1_L.begin(), P.tab1_L.end());   // at 3 NB^2: 1-D factors (element_sf_kernel)
+    tab.insert(tab.end(), P.tab1_D.begin(), P.tab1_D.end());
     if ((rc = upload(h, &h->d_tab, tab))) return bail(rc);
   }
   {   // do two distinct points share their coordinates (only possible across grids)?
