@@ -5,7 +5,7 @@ import csv
 import sys
 
 
-def main(path, skip_regex=None):
+def main(path, step_kernels=None, nstep=3):
     rows = list(csv.reader(open(path)))
     hi = [i for i, r in enumerate(rows) if "Kernel Name" in r][0]
     hdr, data = rows[hi], rows[hi + 1:]
@@ -17,6 +17,13 @@ def main(path, skip_regex=None):
         scale = {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3, "second": 1e6, "s": 1e6}.get(r[ui], 1.0)
         name = r[ki].split("(")[0].replace("(anonymous namespace)::", "")
         agg.setdefault(name, []).append(float(r[vi].replace(",", "")) * scale)
+    if step_kernels:   # the headline step: the first nstep launches of each of its kernels (it runs first)
+        print(f"{'kernel':48s} {'launches':>8s} {'mean_us':>10s} {'share of step':>14s}")
+        sel = {k: v[:nstep] for k, v in agg.items() if any(s in k for s in step_kernels)}
+        step = sum(sum(v) / len(v) for v in sel.values())
+        for k, v in sorted(sel.items(), key=lambda kv: -sum(kv[1]) / len(kv[1])):
+            print(f"{k:48s} {len(v):8d} {sum(v)/len(v):10.2f} {100*sum(v)/len(v)/step:13.1f}%")
+        print(f"{'step (sum of means)':48s} {'':8s} {step:10.2f}\n")
     tot = sum(sum(v) for v in agg.values())
     print(f"{'kernel':48s} {'launches':>8s} {'total_us':>12s} {'mean_us':>10s} {'share':>7s}")
     for k, v in sorted(agg.items(), key=lambda kv: -sum(kv[1])):
@@ -24,4 +31,4 @@ def main(path, skip_regex=None):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1])
+    main(sys.argv[1], sys.argv[2].split(",") if len(sys.argv) > 2 else None)

@@ -51,27 +51,30 @@ def main():
                     "J_err_over_Jabs": float(np.max(np.abs(J - Jo) / Ja)),
                     "J_maxerr_over_maxJ": float(np.abs(J - Jo).max() / np.abs(Jo).max()),
                     "conservation": {"density": d, "momentum": m, "energy": e}, "kernel": "directed (single build)"}
-    # C4 batch on the symmetric kernel
-    nb = 64
-    prob0 = inputs.config4_vertex(0)
-    h = L.Landau.from_problem(prob0, device=0)
-    nodes = h.all_nodes()
-    verts = [int(round(k * 1023 / (nb - 1))) for k in range(nb)]
-    probs = [inputs.config4_vertex(b) for b in verts]
-    F = torch.tensor(np.stack([inputs.coefficients(p, nodes) for p in probs]), device=DEV)
-    h.set_state_batched(F)
-    out = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
-    h.jacobian_batched(out)
-    Jb = out.cpu().numpy()
-    worst = {"J_err_over_Jabs": 0.0, "J_maxerr_over_maxJ": 0.0, "conservation_max": 0.0}
-    for k in (0, 21, 42, 63):
-        o = Oracle(probs[k])
-        Jo, Ja = o.jacobian(o.coefficients())
-        worst["J_err_over_Jabs"] = max(worst["J_err_over_Jabs"], float(np.max(np.abs(Jb[k] - Jo) / Ja)))
-        worst["J_maxerr_over_maxJ"] = max(worst["J_maxerr_over_maxJ"], float(np.abs(Jb[k] - Jo).max() / np.abs(Jo).max()))
-        worst["conservation_max"] = max(worst["conservation_max"],
-                                        max(_conservation(probs[k], h, Jb[k], inputs.coefficients(probs[k], nodes))))
-    rep["C4_batch64_symmetric"] = dict(worst, vertices_checked=[verts[k] for k in (0, 21, 42, 63)])
+    # C4 batch on the mirror slot kernel and on the per-vertex kernel (the headline path)
+    for mode, key in (("slots", "C4_batch64_mirror_slots"), ("vertex", "C4_batch64_vertex")):
+        nb = 64
+        prob0 = inputs.config4_vertex(0)
+        h = L.Landau.from_problem(prob0, device=0)
+        h.set_mirror(mode)
+        nodes = h.all_nodes()
+        verts = [int(round(k * 1023 / (nb - 1))) for k in range(nb)]
+        probs = [inputs.config4_vertex(b) for b in verts]
+        F = torch.tensor(np.stack([inputs.coefficients(p, nodes) for p in probs]), device=DEV)
+        h.set_state_batched(F)
+        out = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
+        h.jacobian_batched(out)
+        Jb = out.cpu().numpy()
+        worst = {"J_err_over_Jabs": 0.0, "J_maxerr_over_maxJ": 0.0, "conservation_max": 0.0,
+                 "inner_path": h.stats()["inner_path"]}
+        for k in (0, 21, 42, 63):
+            o = Oracle(probs[k])
+            Jo, Ja = o.jacobian(o.coefficients())
+            worst["J_err_over_Jabs"] = max(worst["J_err_over_Jabs"], float(np.max(np.abs(Jb[k] - Jo) / Ja)))
+            worst["J_maxerr_over_maxJ"] = max(worst["J_maxerr_over_maxJ"], float(np.abs(Jb[k] - Jo).max() / np.abs(Jo).max()))
+            worst["conservation_max"] = max(worst["conservation_max"],
+                                            max(_conservation(probs[k], h, Jb[k], inputs.coefficients(probs[k], nodes))))
+        rep[key] = dict(worst, vertices_checked=[verts[k] for k in (0, 21, 42, 63)])
     # C5 sampled cells
     prob = inputs.config5()
     h = L.Landau.from_problem(prob, device=0)
