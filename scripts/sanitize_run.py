@@ -1,4 +1,5 @@
-# small workloads for compute-sanitizer: every kernel of the library on C1, C3 and a symmetric batch
+# small workloads for compute-sanitizer: every kernel of the library on C1, C3 and a 16-vertex C4 batch
+# (symmetric, mirror-slot and per-vertex inner kernels; band LU, solve and the implicit step)
 import os, sys
 sys.path.insert(0, os.getcwd())
 import numpy as np, torch
@@ -26,5 +27,16 @@ h.jacobian_batched(v)
 print("stats", h.stats())
 fh = F.cpu().pin_memory(); vh = torch.empty((16, h.nnz), dtype=torch.float64).pin_memory()
 h.jacobian_host(fh, vh)
+for mode in ("slots", "vertex"):   # mirror slot kernel + reduction; per-vertex kernel
+    h.set_mirror(mode)
+    h.jacobian_batched(v)
+    print("stats", mode, h.stats())
+M = torch.empty(h.nnz, dtype=torch.float64, device="cuda"); h.mass(1.0, M)   # band LU, solve, implicit step
+shift = 2.0 * v.abs().max().item() / M.abs().max().item()
+h.band_factor_batched(shift, v)
+b = torch.randn((16, h.ndof), dtype=torch.float64, device="cuda"); x = torch.empty_like(b)
+h.band_solve_batched(b, x)
+fn = torch.empty_like(F)
+h.implicit_step_batched(0.002, F, fn, Ez=0.1, max_iter=2)
 torch.cuda.synchronize()
 print("ok")
