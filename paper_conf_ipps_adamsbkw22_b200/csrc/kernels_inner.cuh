@@ -596,12 +596,20 @@ __device__ __forceinline__ void vtx_run(int a, int b, const double *rU, const do
   vtx_add(sGb, Hp, jf, jb);
 }
 
+#ifndef LANDAU_VTX_WARPS
+#define LANDAU_VTX_WARPS 8
+#endif
+#ifndef LANDAU_VTX_MINB
+#define LANDAU_VTX_MINB 1
+#endif
+constexpr int kVtxWarps = LANDAU_VTX_WARPS, kVtxMinB = LANDAU_VTX_MINB;   // CTA shape, CTAs per SM
+
 struct VtxItem {   // host-built: tiles (a, b) of the upper half; a == b: the diagonal item
   int a, b;
 };
 
 template <bool MASK>
-__global__ void __launch_bounds__(32 * kSymWarps, 1) inner_vtx_kernel(int64_t N, int64_t H, int nrounds,
+__global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int64_t N, int64_t H, int nrounds,
                                                                       const int32_t *__restrict__ round_ptr,
                                                                       const VtxItem *__restrict__ items,
                                                                       const double *__restrict__ rU,
@@ -610,7 +618,7 @@ __global__ void __launch_bounds__(32 * kSymWarps, 1) inner_vtx_kernel(int64_t N,
                                                                       const int32_t *__restrict__ pm,
                                                                       const double *__restrict__ wT, int nbatch,
                                                                       double *__restrict__ G, int64_t G_bstride) {
-  __shared__ double2 s_j[kSymWarps][32 * 5];
+  __shared__ double2 s_j[kVtxWarps][32 * 5];
   __shared__ double s_coef[kNumPairCoef];
   __shared__ double2 s_ltab[kLogTab];
   extern __shared__ double s_G[];   // Ga [5][Hp], Gb [5][Hp]
@@ -626,7 +634,7 @@ __global__ void __launch_bounds__(32 * kSymWarps, 1) inner_vtx_kernel(int64_t N,
     for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) s_G[k] = 0.0;
     __syncthreads();
     for (int rd = 0; rd < nrounds; rd++) {
-      for (int q = round_ptr[rd] + wid; q < round_ptr[rd + 1]; q += kSymWarps) {
+      for (int q = round_ptr[rd] + wid; q < round_ptr[rd + 1]; q += kVtxWarps) {
         const VtxItem it = items[q];
         __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
         {

@@ -432,11 +432,11 @@ int launch_inner(landau_t h, int64_t nbatch) {
     return LANDAU_OK;
   };
   if (h->mirror && h->mirror_on && h->vtx_smem &&
-      (h->mirror_mode == 3 || (h->mirror_mode == 1 && ip.sym && nbatch >= vtx_min_batch_per_sm() * num_sms(h)))) {
+      (h->mirror_mode == 3 || (h->mirror_mode == 1 && ip.sym && nbatch >= vtx_min_batch_per_sm() * num_sms(h) * kVtxMinB))) {
     // one CTA per vertex, sums in shared memory (no slots, no reduction kernel).  Auto mode runs
     // whole waves of vertices this way and hands a remainder below 0.9 of a wave to the slot kernel,
     // which spreads its items over every SM (a partial wave would leave SMs idle).
-    const int64_t T = (h->H + 31) / 32, S = num_sms(h);
+    const int64_t T = (h->H + 31) / 32, S = (int64_t)num_sms(h) * kVtxMinB;   // vertices per wave
     h->stats.pair_evaluations = T * 33 * 32 + 2 * (T * (T - 1) / 2) * 32 * 32;
     h->stats.nsplit = 1;
     h->stats.inner_path = 4;
@@ -449,11 +449,11 @@ int launch_inner(landau_t h, int64_t nbatch) {
       Timer t(h, LANDAU_T_INNER);
       const unsigned grid = (unsigned)std::min<int64_t>(nv, S);
       if (h->coincident)
-        inner_vtx_kernel<true><<<grid, 32 * kSymWarps, h->vtx_smem, h->stream>>>(
+        inner_vtx_kernel<true><<<grid, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(
             N, h->H, h->nvtx_rounds, h->d_vtx_round_ptr, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
             (int)nv, G_own, 5 * h->Nc);
       else
-        inner_vtx_kernel<false><<<grid, 32 * kSymWarps, h->vtx_smem, h->stream>>>(
+        inner_vtx_kernel<false><<<grid, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(
             N, h->H, h->nvtx_rounds, h->d_vtx_round_ptr, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
             (int)nv, G_own, 5 * h->Nc);
       h->launches++;
@@ -933,7 +933,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
         tptr.push_back((int32_t)tslots.size());
       }
       // per-vertex kernel schedule: round-robin tournament of the T tiles (circle method; rounds of
-      // disjoint tile pairs), then the diagonal items in rounds of kSymWarps
+      // disjoint tile pairs), then the diagonal items in rounds of kVtxWarps
       std::vector<VtxItem> vitems;
       std::vector<int32_t> vround(1, 0);
       {
@@ -948,7 +948,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
         }
         for (int t = 0; t < T; t++) {
           vitems.push_back({t, t});
-          if ((t + 1) % kSymWarps == 0 || t + 1 == T) vround.push_back((int32_t)vitems.size());
+          if ((t + 1) % kVtxWarps == 0 || t + 1 == T) vround.push_back((int32_t)vitems.size());
         }
       }
       const size_t vsmem = (size_t)10 * T * 32 * sizeof(double);

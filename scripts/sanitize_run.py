@@ -29,6 +29,7 @@ fh = F.cpu().pin_memory(); vh = torch.empty((16, h.nnz), dtype=torch.float64).pi
 h.jacobian_host(fh, vh)
 for mode in ("slots", "vertex"):   # mirror slot kernel + reduction; per-vertex kernel
     h.set_mirror(mode)
+    h.set_state_batched(F)   # the host entry left its own (chunked) state behind
     h.jacobian_batched(v)
     print("stats", mode, h.stats())
 M = torch.empty(h.nnz, dtype=torch.float64, device="cuda"); h.mass(1.0, M)   # band LU, solve, implicit step
