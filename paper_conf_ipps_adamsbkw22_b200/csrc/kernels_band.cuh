@@ -256,16 +256,25 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
   const int tr = tid / ntc, tc = tid % ntc;
   const bool owner = tr < P / kBandR;
   const int pr0 = tr * kBandR, pc0 = tc * kBandC;
-  // shared layout, double-buffered by pair parity: column k, column k+1 (raw), row k, row k+1 (raw),
-  // corner scalars (p0, 1/p0, L(k+1,k), p1, 1/p1, U(k,k+1), -, -)
+  // shared layout, double-buffered by pair parity: column k, column k+1 (raw), row k, row k+1 (raw,
+  // padded: physical column j at upos(j) = j + 2 (j / 8), so the 16-byte loads of the tile columns
+  // hit distinct banks), corner scalars (p0, 1/p0, L(k+1,k), p1, 1/p1, U(k,k+1), -, -)
+  const int PU = P / 8 * 10, SHW = 2 * P + 2 * PU + 8, W4 = 4 * P;
+  auto upos = [](int j) { return j + (j >> 3) * 2; };
   double *sh0 = smem;
-  double *dbuf = sh0 + 2 * (4 * P + 8);     // [3][8][W] entering rows (dense), one set per group
-  int32_t *sptr = (int32_t *)(dbuf + 24 * W);              // [n + 1]
-  uint16_t *spos = (uint16_t *)(sptr + n + 1);             // [nent]
-  for (int i = tid; i < 2 * (4 * P + 8); i += T) sh0[i] = 0.0;
-  for (int i = tid; i < 24 * W; i += T) dbuf[i] = 0.0;
+  // [3][8][4P] entering rows (dense), one set per group: row part [0, P) and column part [2P, 3P),
+  // each stored twice (copy at +P) so the circular window offsets need no modulo
+  double *dbuf = sh0 + 2 * SHW;
+  int32_t *sptr = (int32_t *)(dbuf + 24 * W4);             // [n + 1]
+  uint16_t *spos = (uint16_t *)(sptr + n + 1);             // [nent] base position in a 4P row
+  for (int i = tid; i < 2 * SHW; i += T) sh0[i] = 0.0;
+  for (int i = tid; i < 24 * W4; i += T) dbuf[i] = 0.0;
   for (int i = tid; i <= n; i += T) sptr[i] = d.ent_ptr[i];
-  for (int i = tid; i < d.nent; i += T) spos[i] = d.ent_pos[i];
+  for (int i = tid; i < d.nent; i += T) {   // host position: row-in-group * W + p, p in 0..B (row
+    const int e = d.ent_pos[i];                 // part) or B+1..2B (column part)
+    const int rg = e / W, p = e - rg * W;
+    spos[i] = (uint16_t)(rg * W4 + (p <= B ? p : 2 * P + p - (B + 1)));
+  }
   const double *ae = Aent + (int64_t)bi * ent_bstride + d.aoff;
   double *lu = LU + (int64_t)bi * lu_bstride + d.off;
   const int ngroups = (n + 7) / 8;
@@ -280,7 +289,10 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
     grange(0, q0, q1);
 #pragma unroll
     for (int m = 0; m < kBandE; m++)
-      if (q0 + tid + m * T < q1) dbuf[spos[q0 + tid + m * T]] = ae[q0 + tid + m * T];
+      if (q0 + tid + m * T < q1) {
+        const int q = spos[q0 + tid + m * T];
+        dbuf[q] = dbuf[q + P] = ae[q0 + tid + m * T];
+      }
     grange(1, q0, q1);
 #pragma unroll
     for (int m = 0; m < kBandE; m++) vin[m] = q0 + tid + m * T < q1 ? ae[q0 + tid + m * T] : 0.0;
@@ -296,7 +308,7 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
 
   int pkb = 0;
   for (int kb = -P, g = 0; kb < n; kb += 8, g++) {
-    const double *dset = dbuf + (g % 3) * 8 * W;
+    const double *dset = dbuf + (g % 3) * 8 * W4;
 #pragma unroll
     for (int u = 0; u < 8; u += 2) {
       const int k = kb + u, pk = pkb + u;
@@ -304,23 +316,26 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
       const bool rowown = owner && tr == (pkb + u - rr) / kBandR;
       const bool colown = owner && tc == pkb / kBandC;
       const bool live0 = k >= 0 && k < n, live1 = k + 1 < n;
-      double *sh = sh0 + ((u >> 1) & 1) * (4 * P + 8);
-      double *a0_s = sh, *a1_s = sh + P, *u0_s = sh + 2 * P, *u1_s = sh + 3 * P, *sc = sh + 4 * P;
+      double *sh = sh0 + ((u >> 1) & 1) * SHW;
+      double *a0_s = sh, *a1_s = sh + P, *u0_s = sh + 2 * P, *u1_s = sh + 2 * P + PU, *sc = sh + 2 * P + 2 * PU;
       if (u == 0 && g >= 2) {   // clear group g - 2's rows from set (g + 1) mod 3
         int q0, q1;
         grange(g - 2, q0, q1);
-        double *ds = dbuf + ((g + 1) % 3) * 8 * W;
+        double *ds = dbuf + ((g + 1) % 3) * 8 * W4;
 #pragma unroll
         for (int m = 0; m < kBandE; m++)
-          if (q0 + tid + m * T < q1) ds[spos[q0 + tid + m * T]] = 0.0;
+          if (q0 + tid + m * T < q1) {
+            const int q = spos[q0 + tid + m * T];
+            ds[q] = ds[q + P] = 0.0;
+          }
       }
       if (live0) {   // b) publish rows k, k+1 and columns k, k+1 (zero at the retiring positions)
         if (rowown) {
 #pragma unroll
           for (int c = 0; c < kBandC; c++) {
             const bool ret = colown && (c == cc || c == cc + 1);
-            u0_s[pc0 + c] = ret ? 0.0 : cell[rr][c];
-            u1_s[pc0 + c] = ret ? 0.0 : cell[rr + 1][c];
+            u0_s[tc * 10 + c] = ret ? 0.0 : cell[rr][c];
+            u1_s[tc * 10 + c] = ret ? 0.0 : cell[rr + 1][c];
           }
           if (colown) {   // the 2 x 2 corner
             const double p0 = cell[rr][cc], ukk1 = cell[rr][cc + 1];
@@ -348,10 +363,13 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
       if (u == 0) {   // scatter group g + 1 into set (g + 1) mod 3; load group g + 2
         int q0, q1;
         grange(g + 1, q0, q1);
-        double *ds = dbuf + ((g + 1) % 3) * 8 * W;
+        double *ds = dbuf + ((g + 1) % 3) * 8 * W4;
 #pragma unroll
         for (int m = 0; m < kBandE; m++)
-          if (q0 + tid + m * T < q1) ds[spos[q0 + tid + m * T]] = vin[m];
+          if (q0 + tid + m * T < q1) {
+            const int q = spos[q0 + tid + m * T];
+            ds[q] = ds[q + P] = vin[m];
+          }
         grange(g + 2, q0, q1);
 #pragma unroll
         for (int m = 0; m < kBandE; m++) vin[m] = q0 + tid + m * T < q1 ? ae[q0 + tid + m * T] : 0.0;
@@ -370,8 +388,8 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
             l1[2 * r] = fma(-l0[2 * r], ukk1, x1.x) * r1;
             l1[2 * r + 1] = fma(-l0[2 * r + 1], ukk1, x1.y) * r1;
           }
-          const double2 *u02 = reinterpret_cast<const double2 *>(u0_s + pc0);
-          const double2 *u12 = reinterpret_cast<const double2 *>(u1_s + pc0);
+          const double2 *u02 = reinterpret_cast<const double2 *>(u0_s + tc * 10);
+          const double2 *u12 = reinterpret_cast<const double2 *>(u1_s + tc * 10);
 #pragma unroll
           for (int c = 0; c < kBandC / 2; c++) {
             const double2 y0 = u02[c], y1 = u12[c];
@@ -395,8 +413,8 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
           } else if (tid <= B) {   // U(k, k+t) and U(k+1, k+1+t): physical columns j and j + 1
             int j1 = j + 1;
             j1 -= j1 >= P ? P : 0;
-            v0 = tid == 1 ? ukk1 : u0_s[j];
-            v1 = fma(-l10, u0_s[j1], u1_s[j1]);
+            v0 = tid == 1 ? ukk1 : u0_s[upos(j)];
+            v1 = fma(-l10, u0_s[upos(j1)], u1_s[upos(j1)]);
           } else {                 // L(k+t, k) and L(k+1+t, k+1): physical rows j and j + 1
             int j1 = j + 1;
             j1 -= j1 >= P ? P : 0;
@@ -411,27 +429,24 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
       //    (rows u, u+1 of the group's set), in that order
 #pragma unroll
       for (int h = 0; h < 2; h++) {
-        const double *db = dset + (u + h) * W;
+        const double *db = dset + (u + h) * W4;
         const int pkh = pk + h;
         const int pk1 = pkh + 1 == P ? 0 : pkh + 1;
         const int rh = rr + h, ch = cc + h;
         if (colown) {
           int o = pr0 - pk1;
           o += o < 0 ? P : 0;
+          const double *dc = db + 2 * P + o;   // duplicated column part: no wrap
 #pragma unroll
-          for (int r = 0; r < kBandR; r++) {
-            const int orr = o + r >= P ? o + r - P : o + r;
-            if (!(rowown && r == rh)) cell[r][ch] = db[B + 1 + orr];
-          }
+          for (int r = 0; r < kBandR; r++)
+            if (!(rowown && r == rh)) cell[r][ch] = dc[r];
         }
         if (rowown) {
           int o = pc0 - pk1;
           o += o < 0 ? P : 0;
+          const double *dr = db + o;           // duplicated row part: no wrap
 #pragma unroll
-          for (int c = 0; c < kBandC; c++) {
-            const int oc = o + c >= P ? o + c - P : o + c;
-            cell[rh][c] = db[oc];
-          }
+          for (int c = 0; c < kBandC; c++) cell[rh][c] = dr[c];
         }
       }
     }

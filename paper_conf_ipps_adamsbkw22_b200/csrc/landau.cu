@@ -1443,8 +1443,8 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
     const char *e = getenv("LANDAU_BAND_RANK");
     return e ? atoi(e) : 2;
   }();
-  const size_t smem2 = sizeof(double) * (2 * (4 * maxPp + 8) + 24 * W) + sizeof(int32_t) * (maxn + 1) +
-                       sizeof(uint16_t) * maxent;
+  const size_t smem2 = sizeof(double) * (2 * (2 * maxPp + 2 * (maxPp / 8 * 10) + 8) + 24 * 4 * maxPp) +
+                       sizeof(int32_t) * (maxn + 1) + sizeof(uint16_t) * maxent;
   const void *kfn;
   size_t ksmem = smem;
   if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
