@@ -431,7 +431,10 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
         std::sort(ent.begin(), ent.end());
         for (auto &e : ent) {
           if (e.second < 0) return "band: CSR pattern is not symmetric";
-          G.ent_pos.push_back((uint16_t)((ni % 8) * (2 * Bp + 1) + e.first));
+          // kernel layout (band_lu2_kernel): row-in-group * 4P, row part p in [0, P), column part
+          // at 2P + (p - P) (each stored twice by the kernel, the copy at +P)
+          const int P = Bp + 1, p = e.first;
+          G.ent_pos.push_back((uint16_t)((ni % 8) * 4 * P + (p < P ? p : 2 * P + p - P)));
           G.ent_slot.push_back(e.second);
         }
         G.ent_max = std::max(G.ent_max, (int)ent.size());

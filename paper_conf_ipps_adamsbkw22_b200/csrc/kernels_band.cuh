@@ -62,179 +62,17 @@ __device__ __forceinline__ double rcp_newton(double a) {
 // One CTA per (batch item, species block).  The P x P active square (P = B + 1, B the padded
 // half-bandwidth, P a multiple of 8) of the outer-product elimination lives in REGISTERS, cut into
 // R x C tiles, one per thread, addressed circularly: logical row/column i sits in physical
-// row/column i mod P.  Step k (pk = k mod P):
-//   b) the owners of physical row/column pk publish U(k, .), A(., k) and the pivot in shared memory;
-//   c) every thread applies the rank-1 update to its tile (the retiring row/column see zero
-//      multipliers) and threads 0..2B write one value each of the factor row LU[k];
-//   d) the owners of the retiring physical row/column load the entering row/column k + P from a
-//      dense buffer.
-// Steps run in groups of 8 (P is a multiple of 8, so pk mod R and pk mod C are compile-time constants
-// in each unrolled copy and the owners index their registers statically).  The 8 rows entering in
+// row/column i mod P.  Per step: the owners of the retiring physical row/column publish them in
+// shared memory, every thread applies the update to its tile (the retiring row/column see zero
+// multipliers), threads 0..2B write the factor rows, and the owners of the retiring row/column load
+// the entering row/column k + P from a dense buffer.  Steps run in groups of 8 (P is a multiple of
+// 8, so the owners index their registers statically in each unrolled copy).  The 8 rows entering in
 // group g are staged in bulk, once per group: their entry values (contiguous in Aent) are loaded
 // into registers two groups ahead, scattered into dense buffer set g mod 3 at the first step of
-// group g - 1, and scattered back to zero at the first step of group g + 2.  One barrier per step,
-// FP64 FMAs on register operands, no integer division.  Groups of steps k < 0 only load the window.
-template <int kBandR, int kBandC, int MINB>
-__global__ void __launch_bounds__(256, MINB) band_lu_kernel(const double *__restrict__ Aent, int64_t ent_bstride,
-                                                        double *__restrict__ LU, int64_t lu_bstride,
-                                                        const BandDesc *__restrict__ desc, int nsp) {
-  static_assert(8 % kBandR == 0 || kBandR % 8 == 0, "tile rows divide or are divided by the group");
-  static_assert(kBandC == 8, "tile columns = the group");
-  extern __shared__ double smem[];
-  const int bi = blockIdx.x / nsp, a = blockIdx.x % nsp;
-  const BandDesc d = desc[a];
-  const int n = d.n, B = d.B, P = B + 1, W = 2 * B + 1;
-  const int tid = threadIdx.x, T = blockDim.x;
-  const int ntc = P / kBandC;
-  const int tr = tid / ntc, tc = tid % ntc;
-  const bool owner = tr < P / kBandR;
-  const int pr0 = tr * kBandR, pc0 = tc * kBandC;
-  // shared layout
-  // a_s / u_s / piv_s are double-buffered by step parity: a step needs one barrier only
-  double *a_s0 = smem;                      // [2][P]  column k (raw); the retiring entry is zero
-  double *u_s0 = a_s0 + 2 * P;              // [2][P]  row k
-  double *piv_s0 = u_s0 + 2 * P;            // [2][2]  pivot, 1 / pivot
-  double *dbuf = piv_s0 + 4;                // [3][8][W] entering rows (dense), one set per group
-  int32_t *sptr = (int32_t *)(dbuf + 24 * W);              // [n + 1]
-  uint16_t *spos = (uint16_t *)(sptr + n + 1);             // [nent]
-  for (int i = tid; i < 4 * P; i += T) a_s0[i] = 0.0;
-  for (int i = tid; i < 24 * W; i += T) dbuf[i] = 0.0;
-  for (int i = tid; i <= n; i += T) sptr[i] = d.ent_ptr[i];
-  for (int i = tid; i < d.nent; i += T) spos[i] = d.ent_pos[i];
-  const double *ae = Aent + (int64_t)bi * ent_bstride + d.aoff;
-  double *lu = LU + (int64_t)bi * lu_bstride + d.off;
-  const int ngroups = (n + 7) / 8;
-  auto grange = [&](int g, int &q0, int &q1) {   // entry range of the rows entering in group g
-    q0 = g < ngroups ? sptr[8 * g] : 0;
-    q1 = g < ngroups ? sptr[min(8 * g + 8, n)] : 0;
-  };
-  double vin[kBandE];   // entry values of group g + 1 (loaded one group ahead of their scatter)
-  __syncthreads();
-  {   // prologue: group 0 scattered into set 0, group 1 loaded
-    int q0, q1;
-    grange(0, q0, q1);
-#pragma unroll
-    for (int m = 0; m < kBandE; m++)
-      if (q0 + tid + m * T < q1) dbuf[spos[q0 + tid + m * T]] = ae[q0 + tid + m * T];
-    grange(1, q0, q1);
-#pragma unroll
-    for (int m = 0; m < kBandE; m++) vin[m] = q0 + tid + m * T < q1 ? ae[q0 + tid + m * T] : 0.0;
-  }
-  double cell[kBandR][kBandC];
-#pragma unroll
-  for (int r = 0; r < kBandR; r++)
-#pragma unroll
-    for (int c = 0; c < kBandC; c++) cell[r][c] = 0.0;
-  // the thread's entry of the factor row LU[k] (t = tid < W): a U entry (physical column pk + t) or
-  // an L entry (physical row pk + t - B), both modulo P by one conditional subtraction
-  const int tw = tid < W ? (tid <= B ? tid : tid - B) : 0;
-
-  int pkb = 0;   // (k mod P) of the group's first step
-  for (int kb = -P, g = 0; kb < n; kb += 8, g++) {
-    const double *dset = dbuf + (g % 3) * 8 * W;   // this group's entering rows
-#pragma unroll
-    for (int u = 0; u < 8; u++) {
-      const int k = kb + u, pk = pkb + u;
-      const int rr = u % kBandR, cc = u % kBandC;   // compile-time after unrolling
-      const bool rowown = owner && tr == (pkb + u - rr) / kBandR;
-      const bool colown = owner && tc == pkb / kBandC;
-      const bool live = k >= 0 && k < n;
-      double *a_s = a_s0 + (u & 1) * P, *u_s = u_s0 + (u & 1) * P, *piv_s = piv_s0 + (u & 1) * 2;
-      if (u == 0 && g >= 2) {   // clear group g - 2's rows from set (g + 1) mod 3
-        int q0, q1;
-        grange(g - 2, q0, q1);
-        double *ds = dbuf + ((g + 1) % 3) * 8 * W;
-#pragma unroll
-        for (int m = 0; m < kBandE; m++)
-          if (q0 + tid + m * T < q1) ds[spos[q0 + tid + m * T]] = 0.0;
-      }
-      if (live) {   // b) publish the pivot row and column
-        if (rowown) {
-#pragma unroll
-          for (int c = 0; c < kBandC; c++) u_s[pc0 + c] = (colown && c == cc) ? 0.0 : cell[rr][c];
-          if (colown) {
-            piv_s[0] = cell[rr][cc];
-            piv_s[1] = rcp_newton(cell[rr][cc]);
-          }
-        }
-        if (colown) {
-#pragma unroll
-          for (int r = 0; r < kBandR; r++) a_s[pr0 + r] = (rowown && r == rr) ? 0.0 : cell[r][cc];
-        }
-      }
-      __syncthreads();
-      if (u == 0) {   // scatter group g + 1 into set (g + 1) mod 3; load group g + 2
-        int q0, q1;
-        grange(g + 1, q0, q1);
-        double *ds = dbuf + ((g + 1) % 3) * 8 * W;
-#pragma unroll
-        for (int m = 0; m < kBandE; m++)
-          if (q0 + tid + m * T < q1) ds[spos[q0 + tid + m * T]] = vin[m];
-        grange(g + 2, q0, q1);
-#pragma unroll
-        for (int m = 0; m < kBandE; m++) vin[m] = q0 + tid + m * T < q1 ? ae[q0 + tid + m * T] : 0.0;
-      }
-      if (live) {   // c) rank-1 update of the tile; threads 0..2B write step k's factor row
-        const double rinv = piv_s[1];
-        if (owner) {
-          double l[kBandR], uu[kBandC];
-          // 16-byte loads: pr0, pc0 and P are multiples of 4
-          const double2 *a2 = reinterpret_cast<const double2 *>(a_s + pr0);
-          const double2 *u2 = reinterpret_cast<const double2 *>(u_s + pc0);
-#pragma unroll
-          for (int r = 0; r < kBandR / 2; r++) {
-            const double2 v = a2[r];
-            l[2 * r] = v.x * rinv;
-            l[2 * r + 1] = v.y * rinv;
-          }
-#pragma unroll
-          for (int c = 0; c < kBandC / 2; c++) {
-            const double2 v = u2[c];
-            uu[2 * c] = v.x;
-            uu[2 * c + 1] = v.y;
-          }
-#pragma unroll
-          for (int r = 0; r < kBandR; r++)
-#pragma unroll
-            for (int c = 0; c < kBandC; c++) cell[r][c] = fma(-l[r], uu[c], cell[r][c]);
-        }
-        if (tid < W) {
-          int j = pk + tw;
-          j -= j >= P ? P : 0;
-          lu[(int64_t)k * W + tid] = tid == 0 ? piv_s[0] : tid <= B ? u_s[j] : a_s[j] * rinv;
-        }
-      }
-      // (no barrier: the next step publishes into the other a_s / u_s buffer, and phase d only
-      // touches the owners' own registers)
-      // d) the retiring physical row/column pk takes the entering row/column k + P (row u of the
-      //    group's set); offset 0 of the entering row is logical k + 1, i.e. physical pk + 1 (mod P)
-      const double *db = dset + u * W;
-      const int pk1 = pk + 1 == P ? 0 : pk + 1;
-      if (colown) {
-        int o = pr0 - pk1;   // offset of physical row pr0 in the entering column
-        o += o < 0 ? P : 0;
-#pragma unroll
-        for (int r = 0; r < kBandR; r++) {
-          const int orr = o + r >= P ? o + r - P : o + r;
-          if (!(rowown && r == rr)) cell[r][cc] = db[B + 1 + orr];
-        }
-      }
-      if (rowown) {
-        int o = pc0 - pk1;
-        o += o < 0 ? P : 0;
-#pragma unroll
-        for (int c = 0; c < kBandC; c++) {
-          const int oc = o + c >= P ? o + c - P : o + c;
-          cell[rr][c] = db[oc];
-        }
-      }
-    }
-    pkb += 8;
-    pkb -= pkb == P ? P : 0;
-  }
-}
-
-// Rank-2 variant: elimination steps k, k+1 (k even) share one barrier.  The owners of the two
+// group g - 1, and scattered back to zero at the first step of group g + 2; each entering row is
+// stored twice (row part at [0, P) and [P, 2P), column part at [2P, 3P) and [3P, 4P)) so the
+// circular window offsets need no modulo.  Groups of steps k < 0 only load the window.
+// Elimination steps k, k+1 (k even) share one barrier.  The owners of the two
 // retiring rows / columns (same tile row and tile column, since k is even and R, C are even) publish
 // them raw; the owner of the 2 x 2 corner publishes the pivots and L(k+1, k); every thread then
 // forms, for its own rows and columns,
@@ -270,11 +108,7 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
   for (int i = tid; i < 2 * SHW; i += T) sh0[i] = 0.0;
   for (int i = tid; i < 24 * W4; i += T) dbuf[i] = 0.0;
   for (int i = tid; i <= n; i += T) sptr[i] = d.ent_ptr[i];
-  for (int i = tid; i < d.nent; i += T) {   // host position: row-in-group * W + p, p in 0..B (row
-    const int e = d.ent_pos[i];                 // part) or B+1..2B (column part)
-    const int rg = e / W, p = e - rg * W;
-    spos[i] = (uint16_t)(rg * W4 + (p <= B ? p : 2 * P + p - (B + 1)));
-  }
+  for (int i = tid; i < d.nent; i += T) spos[i] = d.ent_pos[i];
   const double *ae = Aent + (int64_t)bi * ent_bstride + d.aoff;
   double *lu = LU + (int64_t)bi * lu_bstride + d.off;
   const int ngroups = (n + 7) / 8;

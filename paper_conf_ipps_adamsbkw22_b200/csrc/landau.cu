@@ -1408,8 +1408,10 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
   // one CTA per matrix with the active window in registers: vertex-grid sizes (C1-C4); a single large
   // grid (C5) would need a multi-CTA factorisation (not built)
   if (maxPp > kBandMaxP) return fail(h, LANDAU_EUNSUPPORTED, "band factor: half-bandwidth above 127");
-  const int W = 2 * (maxPp - 1) + 1;
-  const size_t smem = sizeof(double) * (4 * maxPp + 4 + 24 * W) + sizeof(int32_t) * (maxn + 1) + sizeof(uint16_t) * maxent;
+  // band_lu2_kernel's shared memory: pivot rows/columns (double-buffered, padded), 3 x 8 dense
+  // entering rows of 4P, the entry lists
+  const size_t smem = sizeof(double) * (2 * (2 * maxPp + 2 * (maxPp / 8 * 10) + 8) + 24 * 4 * maxPp) +
+                      sizeof(int32_t) * (maxn + 1) + sizeof(uint16_t) * maxent;
   if (smem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
   if (nbatch > h->band_cap) {
     cudaFree(h->d_band);
@@ -1439,20 +1441,12 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
     const char *e = getenv("LANDAU_BAND_MINB");
     return e ? atoi(e) : 2;
   }();
-  static const int band_rank = [] {   // 2: two elimination steps per barrier (band_lu2_kernel)
-    const char *e = getenv("LANDAU_BAND_RANK");
-    return e ? atoi(e) : 2;
-  }();
-  const size_t smem2 = sizeof(double) * (2 * (2 * maxPp + 2 * (maxPp / 8 * 10) + 8) + 24 * 4 * maxPp) +
-                       sizeof(int32_t) * (maxn + 1) + sizeof(uint16_t) * maxent;
   const void *kfn;
-  size_t ksmem = smem;
+  const size_t ksmem = smem;
   if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
-    kfn = band_rank == 2 ? (band_minb >= 2 ? (const void *)band_lu2_kernel<4, 8, 2> : (const void *)band_lu2_kernel<4, 8, 1>)
-                         : (band_minb >= 2 ? (const void *)band_lu_kernel<4, 8, 2> : (const void *)band_lu_kernel<4, 8, 1>);
+    kfn = band_minb >= 2 ? (const void *)band_lu2_kernel<4, 8, 2> : (const void *)band_lu2_kernel<4, 8, 1>;
   else               // 8 x 8 tiles, <= 256 threads
-    kfn = band_rank == 2 ? (const void *)band_lu2_kernel<8, 8, 1> : (const void *)band_lu_kernel<8, 8, 1>;
-  if (band_rank == 2) ksmem = smem2;
+    kfn = (const void *)band_lu2_kernel<8, 8, 1>;
   if (ksmem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
   if (ksmem > 48 * 1024) CU(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ksmem));
   {
