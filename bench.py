@@ -3,8 +3,9 @@
 
 Workload (default, BASELINE.json configs[3] built on configs[1]): a batch of 1024 independent
 spatial-vertex velocity grids, each the e + D Q3 AMR C2 grid (68 cells, N = 1,088 points, 601 DOFs
-per species) with its own thermal-quench-shaped f; the batch is split evenly over the ranks with no
-communication (1024 / world vertices per GPU: strong scaling of a fixed job).
+per species) with its own thermal-quench-shaped f.  The vertices are independent problems, so they are
+sharded over the ranks with no communication: --batch vertices per GPU (default 1024), a job of
+--batch x world vertices ("scaling": "weak"); --strong splits a fixed job of --batch vertices instead.
 
 One step = the whole hot path (SURVEY.md §8(a) a-1 .. a-6) for the local batch:
     landau_set_state_batched -> landau_jacobian_batched (CSR) -> landau_mass (CSR)
@@ -56,7 +57,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="landau", choices=["landau", "reference"])
     ap.add_argument("--workload", default="C4", choices=["C4", "C1", "C2", "C3", "C5"])
-    ap.add_argument("--batch", type=int, default=1024, help="C4 vertices in the whole job")
+    ap.add_argument("--batch", type=int, default=1024, help="C4 vertices per GPU (--strong: in the whole job)")
+    ap.add_argument("--strong", action="store_true", help="C4: split a fixed job of --batch vertices over the GPUs")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle vertices for cpu_baseline (0 = auto)")
     ap.add_argument("--tensor-cache", action="store_true",
@@ -64,16 +66,21 @@ def parse():
     return ap.parse_args()
 
 
+def job_vertices(args, world):
+    """C4 vertices in the whole job: --batch per GPU (weak scaling), or --batch in all (--strong)."""
+    return args.batch if args.strong else args.batch * world
+
+
 def workload(args, world, rank):
     """(name, problem for the mesh, list of per-item problems of this rank, pairs per build)."""
     from paper_conf_ipps_adamsbkw22_b200 import inputs
     if args.workload == "C4":
-        B = args.batch
+        B = job_vertices(args, world)
         lo, hi = rank * B // world, (rank + 1) * B // world
         items = [inputs.config4_vertex(b, B) for b in range(lo, hi)]
         desc = {"workload": f"C4: {B} x C2 vertex grids (e+D, Q3 AMR 68 cells, N=1088, thermal-quench f), "
                             f"{B // world} per GPU, no communication",
-                "vertices": B, "points_per_vertex": 1088, "order": 3, "species": 2,
+                "vertices": B, "vertices_per_gpu": B // world, "points_per_vertex": 1088, "order": 3, "species": 2,
                 "l2": "flushed between timed steps (256 MiB write)"}
         return desc, items[0] if items else inputs.config4_vertex(0, B), items
     p = inputs.CONFIGS[args.workload]()
@@ -195,7 +202,7 @@ def run_reference(args, world, rank):
     from paper_conf_ipps_adamsbkw22_b200 import inputs
     desc, prob0, _ = workload(args, world, 0)
     desc = dict(desc, parallelism=f"batch-shard x{world}" if world > 1 else "1 GPU")
-    B = args.batch
+    B = job_vertices(args, world)
     times = []
     n_per_step = 1
     for k in range(args.warmup + args.steps):
@@ -215,8 +222,8 @@ def run_reference(args, world, rank):
     N = 1088 if args.workload == "C4" else prob0.npoints
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / len(times),
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": desc, "pairs_per_s": value * N * N,
+            "higher_is_better": True, "scaling": "strong" if args.strong else "weak", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic", "config": desc, "pairs_per_s": value * N * N,
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": get_threads(), "kind": "oracle",
                              "sample": f"1 vertex Jacobian per step ({args.workload}), full oracle"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -310,8 +317,8 @@ def main():
         dist.barrier()
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms = float(t.item())
-    total_builds = args.batch if args.workload == "C4" else 1
-    scaling = "strong"
+    total_builds = job_vertices(args, world) if args.workload == "C4" else 1
+    scaling = "strong" if (args.strong or args.workload != "C4") else "weak"
     ms_per_step = total_ms / args.steps
     value = total_builds / (ms_per_step / 1e3)
     pairs_per_build = N * N
@@ -373,7 +380,7 @@ def main():
     stage_ms = {k: v[0] / args.steps for k, v in tim.items()}
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": scaling,
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": dict(desc, parallelism=(f"element-split x{world}" if args.workload == "C5" else
                                               f"batch-shard x{world}") if world > 1 else "1 GPU"),

@@ -28,3 +28,21 @@ def test_reference_arm_other_ranks_exit_quietly():
     out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--steps", "1",
                           "--warmup", "0"], capture_output=True, text=True, timeout=120, cwd=ROOT, env=env)
     assert out.returncode == 0 and out.stdout.strip() == ""
+
+
+def test_c4_sharding_weak_and_strong():
+    """C4 vertices are independent problems: by default every rank builds its own --batch vertices
+    (weak scaling, a job of batch x world); --strong splits a fixed job.  The ranks' vertex ranges
+    are disjoint and cover the job, and world 1 is the BASELINE configs[3] batch either way."""
+    import argparse
+    sys.path.insert(0, ROOT)
+    import bench
+    for strong, world, job in ((False, 1, 16), (False, 2, 32), (True, 2, 16), (True, 4, 16)):
+        args = argparse.Namespace(batch=16, strong=strong, workload="C4")
+        assert bench.job_vertices(args, world) == job
+        seen = []
+        for rank in range(world):
+            desc, _, items = bench.workload(args, world, rank)
+            assert desc["vertices"] == job and len(items) == job // world
+            seen += [it.seed for it in items]
+        assert sorted(seen) == [20220 + b for b in range(job)]
