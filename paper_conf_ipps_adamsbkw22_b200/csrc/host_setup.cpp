@@ -460,7 +460,7 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
       std::vector<std::vector<std::pair<int32_t, double>>> cslot(ne * ne);
       for (int a = 0; a < nb; a++)
         for (int bb = 0; bb < nb; bb++) {
-          const int32_t idx = (int32_t)(ge * 2 * nb * nb + a * nb + bb);
+          const int32_t idx = (int32_t)(ge * 2 * nb * nb + 2 * (a * nb + bb));   // [cell][k][l][D|K] interleaved
           for (int i = 0; i < ne; i++) {
             double pa = Pc[a * ne + i];
             if (pa == 0.0) continue;

@@ -49,7 +49,8 @@ struct GridPlan {
 };
 
 // A gather map: output slot s = sum over its contributions (idx, w) of w * Celem[idx], in a fixed
-// order (cell, a, b).  idx = e * 2 Nb^2 + a * Nb + b indexes the [cell][2][Nb][Nb] element buffer.
+// order (cell, a, b).  idx = e * 2 Nb^2 + 2 (a * Nb + b) indexes the [cell][Nb][Nb][2] element buffer
+// (C^D and C^K of an entry side by side: one 16-byte load per contribution).
 struct GatherMap {
   std::vector<int64_t> ptr;   // [nslots+1]
   std::vector<int32_t> idx;

@@ -164,8 +164,7 @@ __global__ void __launch_bounds__(NB * EPB, LANDAU_EL_MINB) element_kernel(int64
     for (int a = 0; a < S; a++)
 #pragma unroll
       for (int c = 0; c < S; c++) {
-        o[(k0 + a) * NB + l0 + c] = cd[a][c] * sc * sc;
-        o[NB * NB + (k0 + a) * NB + l0 + c] = ck[a][c] * sc;
+        reinterpret_cast<double2 *>(o)[(k0 + a) * NB + l0 + c] = make_double2(cd[a][c] * sc * sc, ck[a][c] * sc);
       }
   }
 }
@@ -263,15 +262,14 @@ __global__ void __launch_bounds__(32 * kSfWarps) element_sf_kernel(int64_t ncell
           ck = fma(PLL[qr], sT[wid][5][bd][qr], ck);
         }
         const int k = (bd / S) * S + x, l = (bd % S) * S + y;
-        o[k * NB + l] = cd * sc2;
-        o[NB * NB + k * NB + l] = ck * sc;
+        reinterpret_cast<double2 *>(o)[k * NB + l] = make_double2(cd * sc2, ck * sc);   // (C^D, C^K) interleaved
       }
     }
   }
 }
 
-// Mass element matrices (create time): M[k,l] = sum_q w_q phi_k phi_l, stored in the [cell][2][NB^2]
-// layout (second half zero) so the same gather maps apply.
+// Mass element matrices (create time): M[k,l] = sum_q w_q phi_k phi_l, stored in the element-buffer
+// layout [cell][k][l][2] (interleaved with the advection matrix) so the same gather maps apply.
 template <int NB>
 __global__ void __launch_bounds__(NB * NB) mass_element_kernel(int64_t ncell, const double *__restrict__ pw,
                                                                  const double *__restrict__ cell_h,
@@ -290,8 +288,8 @@ __global__ void __launch_bounds__(NB * NB) mass_element_kernel(int64_t ncell, co
     m = fma(wp, s_phi[q][l], m);
     adv = fma(wp, sz * s_deta[q][l], adv);
   }
-  Mbuf[e * 2 * NB * NB + tid] = m;
-  Mbuf[e * 2 * NB * NB + NB * NB + tid] = adv;
+  Mbuf[e * 2 * NB * NB + 2 * tid] = m;   // [cell][k][l][mass | advection], the element-buffer layout
+  Mbuf[e * 2 * NB * NB + 2 * tid + 1] = adv;
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -329,8 +327,9 @@ __global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ C
 #pragma unroll
     for (int t = 0; t < BPT; t++)
       if (t < nb) {
-        sD[t] = fma(w, __ldg(C + t * cbuf_bstride + i), sD[t]);
-        sK[t] = fma(w, __ldg(C + t * cbuf_bstride + i + NB * NB), sK[t]);
+        const double2 v = __ldg(reinterpret_cast<const double2 *>(C + t * cbuf_bstride + i));   // (C^D, C^K)
+        sD[t] = fma(w, v.x, sD[t]);
+        sK[t] = fma(w, v.y, sK[t]);
       }
   }
 #pragma unroll
@@ -342,7 +341,7 @@ __global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ C
 }
 
 // mass gather (create time): out[s] = sum_k w_k M[idx_k]
-// (M points at the mass half of the element buffer, or at M + NB^2 for the advection half)
+// (M points at the mass entries of the element buffer, or at M + 1 for the interleaved advection ones)
 __global__ void mass_gather_kernel(const int64_t *__restrict__ ptr, const int32_t *__restrict__ idx,
                                    const double *__restrict__ w, int64_t nslots, const double *__restrict__ M,
                                    double *__restrict__ out) {

@@ -687,7 +687,7 @@ int build_mass(landau_t h) {
       CU(cudaMalloc(&dst, sizeof(double) * std::max<int64_t>(m.nslots, 1)));
       if (m.nslots == 0) continue;
       mass_gather_kernel<<<(unsigned)((m.nslots + 255) / 256), 256, 0, h->stream>>>(m.ptr, m.idx, m.w, m.nslots,
-                                                                                    Mbuf + (f < 2 ? 0 : NB * NB), dst);
+                                                                                    Mbuf + (f < 2 ? 0 : 1), dst);
       h->launches++;
       KCHECK();
     }
