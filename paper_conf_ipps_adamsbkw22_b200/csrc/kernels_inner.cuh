@@ -495,43 +495,56 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_mir_kernel(int64_t
 // the tiles, then rounds of diagonal items), so the warps of a CTA add their sums into shared memory
 // without atomics and every target's partial sums arrive in a fixed order: bitwise reproducible.
 // ------------------------------------------------------------------------------------------------
-__device__ __forceinline__ void acc_rev_flip(Acc5 &a, double Vdrr, double Udrz, double Udzz, double Ukrr, double Ukzr,
-                                             double wd, double wkr, double wkz) {
-  a.drr = fma(wd, Vdrr, a.drr);
-  a.drz = fma(-wd, Ukzr, a.drz);
-  a.dzz = fma(wd, Udzz, a.dzz);
-  a.kr = fma(Ukrr, wkr, fma(Ukzr, wkz, a.kr));
-  a.kz = fma(-Udrz, wkr, fma(-Udzz, wkz, a.kz));
-}
-
-// one U+V step of lane target (r, z) against j-data (rj, zj, rj2, A(j), Bf(j)); i weights A(i), Bf(i)
-// mf: forward mask, mr: reverse mask (U part); mvf / mvr: the V part's masks
-template <bool MASK>
-__device__ __forceinline__ void vtx_step(double r, double z, double r2, const double Ai[3], const double Bi[3],
-                                         double rj, double zj, double rj2, double2 a01, double2 a2b0, double2 b12,
-                                         const PairCoef &cf, double mu_f, double mu_r, double mv_f, double mv_r,
-                                         Acc5 &ga, Acc5 &gb, Acc5 &ja, Acc5 &jb) {
-  bool oku, okv;
-  double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
+// One U+V step in sum/difference form.  Every accumulated term has the shape
+//   Ga += A U + B (s X),   Gb += B U + A (s X)      (U: same-side tensor, X: cross tensor, s = +-1),
+// so with hp = (A + B)/2, hm = (A - B)/2 the pair is carried as P += hp (U + s X), M += hm (U - s X)
+// (Ga = P + M, Gb = P - M at the end of the item).  The reverse sums have the same shape with the i
+// weights, and the nine (U, X, s) combinations of the 5 + 5 + reverse tensor components reduce to six
+// sums/differences (S2 = D5, S3 = D7, ...): 12 DADD + 28 DFMA per step instead of 56 DFMA, and half
+// the DFMAs that read three distinct registers (register-file bank reads).
+// j-data: (rj, zj, rj^2) and its staged weights hp(j) = (p01.x, p01.y, p2m0.x), hm(j) = (p2m0.y, m12.x,
+// m12.y); i weights hpi, hmi.  msk scales both tensors (diagonal-step masks); REV = false: forward only.
+template <bool MASK, bool REV, bool UON>
+__device__ __forceinline__ void vtx_step(double r, double z, double r2, const double hpi[3], const double hmi[3],
+                                         double rj, double zj, double rj2, double2 p01, double2 p2m0, double2 m12,
+                                         const PairCoef &cf, double msk, Acc5 &P, Acc5 &M, Acc5 &PJ, Acc5 &MJ) {
+  bool oku = true, okv;
+  double Udrr = 0.0, Udrz = 0.0, Udzz = 0.0, Ukrr = 0.0, Ukzr = 0.0, Vdrr = 0.0;
   double Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, Ydrr;
-  pair_tensors<MASK>(r, z, r2, rj, zj, rj2, cf, oku, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
+  if constexpr (UON) pair_tensors<MASK>(r, z, r2, rj, zj, rj2, cf, oku, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
   pair_tensors<MASK>(r, z, r2, rj, -zj, rj2, cf, okv, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, Ydrr);
-  if (MASK) {
-    mu_f = oku ? mu_f : 0.0;
-    mu_r = oku ? mu_r : 0.0;
-    mv_f = okv ? mv_f : 0.0;
-    mv_r = okv ? mv_r : 0.0;
+  const double mu = (!MASK || oku) ? msk : 0.0, mv = (!MASK || okv) ? msk : 0.0;
+  Udrr *= mu; Udrz *= mu; Udzz *= mu; Ukrr *= mu; Ukzr *= mu; Vdrr *= mu;
+  Xdrr *= mv; Xdrz *= mv; Xdzz *= mv; Xkrr *= mv; Xkzr *= mv; Ydrr *= mv;
+  const double S1 = Udrr + Xdrr, D1 = Udrr - Xdrr;   // (drr, +)
+  const double S2 = Udrz + Xdrz, D2 = Udrz - Xdrz;   // (drz, +); (drz, -) = (D2, S2)
+  const double S3 = Udzz + Xdzz, D3 = Udzz - Xdzz;   // (dzz, +); (dzz, -) = (D3, S3)
+  const double S4 = Ukrr + Xkrr, D4 = Ukrr - Xkrr;   // (krr, +)
+  const double S6 = Ukzr + Xkzr, D6 = Ukzr - Xkzr;   // (kzr, +); (kzr, -) = (D6, S6)
+  // forward: weights of j
+  P.drr = fma(p01.x, S1, P.drr);
+  M.drr = fma(p2m0.y, D1, M.drr);
+  P.drz = fma(p01.x, S2, P.drz);
+  M.drz = fma(p2m0.y, D2, M.drz);
+  P.dzz = fma(p01.x, S3, P.dzz);
+  M.dzz = fma(p2m0.y, D3, M.dzz);
+  P.kr = fma(p01.y, S4, fma(p2m0.x, D2, P.kr));
+  M.kr = fma(m12.x, D4, fma(m12.y, S2, M.kr));
+  P.kz = fma(p01.y, S6, fma(p2m0.x, D3, P.kz));
+  M.kz = fma(m12.x, D6, fma(m12.y, S3, M.kz));
+  if constexpr (REV) {   // reverse: weights of i
+    const double S8 = Vdrr + Ydrr, D8 = Vdrr - Ydrr;   // (rev drr, +)
+    PJ.drr = fma(hpi[0], S8, PJ.drr);
+    MJ.drr = fma(hmi[0], D8, MJ.drr);
+    PJ.drz = fma(hpi[0], D6, PJ.drz);
+    MJ.drz = fma(hmi[0], S6, MJ.drz);
+    PJ.dzz = fma(hpi[0], S3, PJ.dzz);
+    MJ.dzz = fma(hmi[0], D3, MJ.dzz);
+    PJ.kr = fma(hpi[1], S4, fma(hpi[2], S6, PJ.kr));
+    MJ.kr = fma(hmi[1], D4, fma(hmi[2], D6, MJ.kr));
+    PJ.kz = fma(hpi[1], D2, fma(hpi[2], D3, PJ.kz));
+    MJ.kz = fma(hmi[1], S2, fma(hmi[2], S3, MJ.kz));
   }
-  // U: sources A(j) -> Ga, Bf(j) -> Gb; reverse A(i) -> Ga(j), Bf(i) -> Gb(j)
-  acc_fwd(ga, Udrr, Udrz, Udzz, Ukrr, Ukzr, mu_f * a01.x, mu_f * a01.y, mu_f * a2b0.x);
-  acc_fwd(gb, Udrr, Udrz, Udzz, Ukrr, Ukzr, mu_f * a2b0.y, mu_f * b12.x, mu_f * b12.y);
-  acc_rev(ja, Vdrr, Udrz, Udzz, Ukrr, Ukzr, mu_r * Ai[0], mu_r * Ai[1], mu_r * Ai[2]);
-  acc_rev(jb, Vdrr, Udrz, Udzz, Ukrr, Ukzr, mu_r * Bi[0], mu_r * Bi[1], mu_r * Bi[2]);
-  // V (source j' at (rj, -zj)): F Bf(j) -> Ga, F A(j) -> Gb; reverse F rev(V) Bf(i) -> Ga(j), F rev(V) A(i) -> Gb(j)
-  acc_fwd(ga, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, mv_f * a2b0.y, mv_f * b12.x, -mv_f * b12.y);
-  acc_fwd(gb, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, mv_f * a01.x, mv_f * a01.y, -mv_f * a2b0.x);
-  acc_rev_flip(ja, Ydrr, Xdrz, Xdzz, Xkrr, Xkzr, mv_r * Bi[0], mv_r * Bi[1], mv_r * Bi[2]);
-  acc_rev_flip(jb, Ydrr, Xdrz, Xdzz, Xkrr, Xkzr, mv_r * Ai[0], mv_r * Ai[1], mv_r * Ai[2]);
 }
 
 __device__ __forceinline__ void vtx_add(double *sG, int64_t Hp, int64_t pos, const Acc5 &a) {
@@ -542,58 +555,63 @@ __device__ __forceinline__ void vtx_add(double *sG, int64_t Hp, int64_t pos, con
   sG[4 * Hp + pos] += a.kz;
 }
 
-// one (a, b) item of a vertex; s_j: the warp's staged j-tile b as (r, z), A01, (A2, Bf0), Bf12, (r^2, -);
-// sGa, sGb: the CTA's shared accumulators [5][Hp]
+// Ga = P + M into sGa, Gb = P - M into sGb
+__device__ __forceinline__ void vtx_add_pm(double *sGa, double *sGb, int64_t Hp, int64_t pos, const Acc5 &P,
+                                           const Acc5 &M) {
+  vtx_add(sGa, Hp, pos, Acc5{P.drr + M.drr, P.drz + M.drz, P.dzz + M.dzz, P.kr + M.kr, P.kz + M.kz});
+  vtx_add(sGb, Hp, pos, Acc5{P.drr - M.drr, P.drz - M.drz, P.dzz - M.dzz, P.kr - M.kr, P.kz - M.kz});
+}
+
+// one (a, b) item of a vertex; s_j: the warp's staged j-tile b as (r, z), (hp_d, hp_kr), (hp_kz, hm_d),
+// (hm_kr, hm_kz), (r^2, -); sGa, sGb: the CTA's shared accumulators [5][Hp]
 template <bool DIAG, bool MASK>
 __device__ __forceinline__ void vtx_run(int a, int b, const double *rU, const double *zU, const double *wb, int64_t N,
                                         int64_t H, int64_t Hp, const int32_t *pu, const int32_t *pm, int lane,
                                         const double2 *s_j, const PairCoef &cf, double *sGa, double *sGb) {
   const int64_t i = (int64_t)a * 32 + lane;
-  double Ai[3], Bi[3];
+  double Ai[3], Bi[3], hpi[3], hmi[3];
   mir_weights(wb, N, H, pu, pm, i, Ai, Bi);
+#pragma unroll
+  for (int c = 0; c < 3; c++) {
+    hpi[c] = 0.5 * (Ai[c] + Bi[c]);
+    hmi[c] = 0.5 * (Ai[c] - Bi[c]);
+  }
   const double r = i < H ? rU[i] : 1.0;
   const double z = i < H ? zU[i] : 1.0e6 + lane;   // padding: far away, zero weights
   const double r2 = r * r;
-  Acc5 ga{0.0, 0.0, 0.0, 0.0, 0.0}, gb{0.0, 0.0, 0.0, 0.0, 0.0};
-  Acc5 ja{0.0, 0.0, 0.0, 0.0, 0.0}, jb{0.0, 0.0, 0.0, 0.0, 0.0};
+  Acc5 P{0.0, 0.0, 0.0, 0.0, 0.0}, M{0.0, 0.0, 0.0, 0.0, 0.0};
+  Acc5 PJ{0.0, 0.0, 0.0, 0.0, 0.0}, MJ{0.0, 0.0, 0.0, 0.0, 0.0};
   const int src = (lane + 1) & 31;
   if constexpr (DIAG) {   // step 0: each point with its own mirror (V forward only; U is the self pair)
-    const double2 rz = s_j[lane * 5], a01 = s_j[lane * 5 + 1], a2b0 = s_j[lane * 5 + 2], b12 = s_j[lane * 5 + 3],
+    const double2 rz = s_j[lane * 5], p01 = s_j[lane * 5 + 1], p2m0 = s_j[lane * 5 + 2], m12 = s_j[lane * 5 + 3],
                   rr2 = s_j[lane * 5 + 4];
-    double Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, Ydrr;
-    bool okv;
-    pair_tensors<MASK>(r, z, r2, rz.x, -rz.y, rr2.x, cf, okv, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, Ydrr);
-    const double mv = (!MASK || okv) ? 1.0 : 0.0;
-    acc_fwd(ga, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, mv * a2b0.y, mv * b12.x, -mv * b12.y);
-    acc_fwd(gb, Xdrr, Xdrz, Xdzz, Xkrr, Xkzr, mv * a01.x, mv * a01.y, -mv * a2b0.x);
+    vtx_step<MASK, false, false>(r, z, r2, hpi, hmi, rz.x, rz.y, rr2.x, p01, p2m0, m12, cf, 1.0, P, M, PJ, MJ);
   }
   constexpr int k0 = DIAG ? 1 : 0, kmain = DIAG ? 16 : 32;
 #pragma unroll kMirUnroll
   for (int k = k0; k < kmain; k++) {
     const int jj = (lane + k) & 31;
-    const double2 rz = s_j[jj * 5], a01 = s_j[jj * 5 + 1], a2b0 = s_j[jj * 5 + 2], b12 = s_j[jj * 5 + 3],
+    const double2 rz = s_j[jj * 5], p01 = s_j[jj * 5 + 1], p2m0 = s_j[jj * 5 + 2], m12 = s_j[jj * 5 + 3],
                   rr2 = s_j[jj * 5 + 4];
-    vtx_step<MASK>(r, z, r2, Ai, Bi, rz.x, rz.y, rr2.x, a01, a2b0, b12, cf, 1.0, 1.0, 1.0, 1.0, ga, gb, ja, jb);
-    acc_shfl(ja, src);
-    acc_shfl(jb, src);
+    vtx_step<MASK, true, true>(r, z, r2, hpi, hmi, rz.x, rz.y, rr2.x, p01, p2m0, m12, cf, 1.0, P, M, PJ, MJ);
+    acc_shfl(PJ, src);
+    acc_shfl(MJ, src);
   }
   if constexpr (DIAG) {   // step 16: lanes >= 16 would double-count
     const int jj = (lane + 16) & 31;
-    const double2 rz = s_j[jj * 5], a01 = s_j[jj * 5 + 1], a2b0 = s_j[jj * 5 + 2], b12 = s_j[jj * 5 + 3],
+    const double2 rz = s_j[jj * 5], p01 = s_j[jj * 5 + 1], p2m0 = s_j[jj * 5 + 2], m12 = s_j[jj * 5 + 3],
                   rr2 = s_j[jj * 5 + 4];
-    const double m = lane < 16 ? 1.0 : 0.0;
-    vtx_step<true>(r, z, r2, Ai, Bi, rz.x, rz.y, rr2.x, a01, a2b0, b12, cf, m, m, m, m, ga, gb, ja, jb);
-    acc_shfl(ja, src);
-    acc_shfl(jb, src);
+    vtx_step<true, true, true>(r, z, r2, hpi, hmi, rz.x, rz.y, rr2.x, p01, p2m0, m12, cf, lane < 16 ? 1.0 : 0.0, P,
+                               M, PJ, MJ);
+    acc_shfl(PJ, src);
+    acc_shfl(MJ, src);
   }
-  vtx_add(sGa, Hp, i, ga);
-  vtx_add(sGb, Hp, i, gb);
+  vtx_add_pm(sGa, sGb, Hp, i, P, M);
   if constexpr (DIAG) __syncwarp();   // forward and reverse sums of a diagonal item hit the same tile
   // after the last hand-over lane L holds the reverse sums of j = (L + kend) mod 32
   const int kend = DIAG ? 17 : 32;
   const int64_t jf = (int64_t)b * 32 + ((lane + kend) & 31);
-  vtx_add(sGa, Hp, jf, ja);
-  vtx_add(sGb, Hp, jf, jb);
+  vtx_add_pm(sGa, sGb, Hp, jf, PJ, MJ);
 }
 
 #ifndef LANDAU_VTX_WARPS
@@ -643,11 +661,11 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
           mir_weights(wb, N, H, pu, pm, j, A, Bf);
           const double r = j < H ? rU[j] : 1.0;
           const double z = j < H ? zU[j] : 2.0e6 + lane;
-          double2 *d = &s_j[wid][lane * 5];
+          double2 *d = &s_j[wid][lane * 5];   // (r, z), hp = (A + Bf)/2, hm = (A - Bf)/2, (r^2, -)
           d[0] = make_double2(r, z);
-          d[1] = make_double2(A[0], A[1]);
-          d[2] = make_double2(A[2], Bf[0]);
-          d[3] = make_double2(Bf[1], Bf[2]);
+          d[1] = make_double2(0.5 * (A[0] + Bf[0]), 0.5 * (A[1] + Bf[1]));
+          d[2] = make_double2(0.5 * (A[2] + Bf[2]), 0.5 * (A[0] - Bf[0]));
+          d[3] = make_double2(0.5 * (A[1] - Bf[1]), 0.5 * (A[2] - Bf[2]));
           d[4] = make_double2(r * r, 0.0);
         }
         __syncwarp();
