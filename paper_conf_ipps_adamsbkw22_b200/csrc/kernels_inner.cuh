@@ -282,18 +282,6 @@ __global__ void reduce_sym_kernel(int64_t N, int64_t nslots, const int32_t *__re
 // once as a U item and once as a V item (it.v); a V diagonal item also pairs every point with its own
 // mirror (step 0, forward only).  part = [batch][nslots][2][5][32] (Ga, Gb).
 // ------------------------------------------------------------------------------------------------
-struct MirItem {   // host-built
-  int a[3];        // i-tiles (n of them, all < b); n == 0: the diagonal item (b, b)
-  int b, n;
-  int v;           // 0: same-side tensors U(i, j); 1: cross tensors V(i, j) = U(i, j')
-  int slot;        // first of the item's consecutive slots: one per i-tile (or the diagonal), then j's
-};
-
-struct Acc10 {
-  Acc5 a, b;
-};
-
-// wT gather of one U point's weight pair: A(u), Bf(u) (zero for padding)
 __device__ __forceinline__ void mir_weights(const double *wb, int64_t N, int64_t H, const int32_t *pu,
                                             const int32_t *pm, int64_t u, double A[3], double Bf[3]) {
   if (u < H) {
@@ -307,26 +295,6 @@ __device__ __forceinline__ void mir_weights(const double *wb, int64_t N, int64_t
   } else {
     A[0] = A[1] = A[2] = Bf[0] = Bf[1] = Bf[2] = 0.0;
   }
-}
-
-__device__ __forceinline__ void acc_fwd(Acc5 &a, double Udrr, double Udrz, double Udzz, double Ukrr, double Ukzr,
-                                        double wd, double wkr, double wkz) {
-  a.drr = fma(wd, Udrr, a.drr);
-  a.drz = fma(wd, Udrz, a.drz);
-  a.dzz = fma(wd, Udzz, a.dzz);
-  a.kr = fma(Ukrr, wkr, fma(Udrz, wkz, a.kr));
-  a.kz = fma(Ukzr, wkr, fma(Udzz, wkz, a.kz));
-}
-
-// the reverse tensors of (i, j): U^D_rr(j,i) = Vdrr, U^D_rz(j,i) = Ukzr, U^D_zz, U^K_rr symmetric,
-// U^K_zr(j,i) = Udrz (see landau_pair_sym)
-__device__ __forceinline__ void acc_rev(Acc5 &a, double Vdrr, double Udrz, double Udzz, double Ukrr, double Ukzr,
-                                        double wd, double wkr, double wkz) {
-  a.drr = fma(wd, Vdrr, a.drr);
-  a.drz = fma(wd, Ukzr, a.drz);
-  a.dzz = fma(wd, Udzz, a.dzz);
-  a.kr = fma(Ukrr, wkr, fma(Ukzr, wkz, a.kr));
-  a.kz = fma(Udrz, wkr, fma(Udzz, wkz, a.kz));
 }
 
 __device__ __forceinline__ void acc_shfl(Acc5 &a, int src) {
@@ -345,141 +313,6 @@ __device__ __forceinline__ void mir_store(double *o, int pos, const Acc5 &a, boo
   o[64 + pos] = a.dzz;
   o[96 + pos] = a.kr;
   o[128 + pos] = sg * a.kz;
-}
-
-template <int NI, bool DIAG, bool MASK>
-__device__ __forceinline__ void mir_run(const MirItem &it, const double *rU, const double *zU, const double *wb,
-                                        int64_t N, int64_t H, const int32_t *pu, const int32_t *pm, int lane,
-                                        const double2 *s_j, const PairCoef &cf, double *o) {
-  // lane data: target i of each i-tile, its reverse-source weights R1, R2 and its sums Ga, Gb
-  const bool V = it.v != 0;
-  double r[NI], z[NI], r2[NI], R1[NI][3], R2[NI][3];
-  Acc5 ga[NI], gb[NI];
-#pragma unroll
-  for (int t = 0; t < NI; t++) {
-    const int64_t i = (int64_t)(DIAG ? it.b : it.a[t]) * 32 + lane;
-    double A[3], Bf[3];
-    mir_weights(wb, N, H, pu, pm, i, A, Bf);
-    r[t] = i < H ? rU[i] : 1.0;
-    z[t] = i < H ? zU[i] : 1.0e6 + 64.0 * t + lane;   // padding: far away, zero weights
-    r2[t] = r[t] * r[t];
-#pragma unroll
-    for (int c = 0; c < 3; c++) {
-      R1[t][c] = V ? Bf[c] : A[c];
-      R2[t][c] = V ? A[c] : Bf[c];
-    }
-    ga[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
-    gb[t] = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
-  }
-  const int src = (lane + 1) & 31;
-  Acc5 ja{0.0, 0.0, 0.0, 0.0, 0.0}, jb{0.0, 0.0, 0.0, 0.0, 0.0};
-  // diagonal: V items start at step 0 (each point with its own mirror, forward only); steps 1..15
-  // unmasked, step 16 peeled (lanes >= 16 would double-count)
-  const int k0 = DIAG ? (V ? 0 : 1) : 0;
-  constexpr int kmain = DIAG ? 16 : 32;
-#pragma unroll kMirUnroll
-  for (int k = k0; k < kmain; k++) {
-    const int jj = (lane + k) & 31;
-    const double2 rz = s_j[jj * 5], w1 = s_j[jj * 5 + 1], w12 = s_j[jj * 5 + 2], w2 = s_j[jj * 5 + 3],
-                  rr2 = s_j[jj * 5 + 4];
-    const bool rev_on = !(DIAG && k == 0);
-#pragma unroll
-    for (int t = 0; t < NI; t++) {
-      bool ok;
-      double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
-      pair_tensors<MASK>(r[t], z[t], r2[t], rz.x, rz.y, rr2.x, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
-      const double m = (!MASK || ok) ? 1.0 : 0.0;
-      const double mr = rev_on ? m : 0.0;
-      acc_fwd(ga[t], Udrr, Udrz, Udzz, Ukrr, Ukzr, m * w1.x, m * w1.y, m * w12.x);
-      acc_fwd(gb[t], Udrr, Udrz, Udzz, Ukrr, Ukzr, m * w12.y, m * w2.x, m * w2.y);
-      acc_rev(ja, Vdrr, Udrz, Udzz, Ukrr, Ukzr, mr * R1[t][0], mr * R1[t][1], mr * R1[t][2]);
-      acc_rev(jb, Vdrr, Udrz, Udzz, Ukrr, Ukzr, mr * R2[t][0], mr * R2[t][1], mr * R2[t][2]);
-    }
-    acc_shfl(ja, src);
-    acc_shfl(jb, src);
-  }
-  if constexpr (DIAG) {
-    const int jj = (lane + 16) & 31;
-    const double2 rz = s_j[jj * 5], w1 = s_j[jj * 5 + 1], w12 = s_j[jj * 5 + 2], w2 = s_j[jj * 5 + 3],
-                  rr2 = s_j[jj * 5 + 4];
-    bool ok;
-    double Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr;
-    pair_tensors<true>(r[0], z[0], r2[0], rz.x, rz.y, rr2.x, cf, ok, Udrr, Udrz, Udzz, Ukrr, Ukzr, Vdrr);
-    const double m = (ok && lane < 16) ? 1.0 : 0.0;
-    acc_fwd(ga[0], Udrr, Udrz, Udzz, Ukrr, Ukzr, m * w1.x, m * w1.y, m * w12.x);
-    acc_fwd(gb[0], Udrr, Udrz, Udzz, Ukrr, Ukzr, m * w12.y, m * w2.x, m * w2.y);
-    acc_rev(ja, Vdrr, Udrz, Udzz, Ukrr, Ukzr, m * R1[0][0], m * R1[0][1], m * R1[0][2]);
-    acc_rev(jb, Vdrr, Udrz, Udzz, Ukrr, Ukzr, m * R2[0][0], m * R2[0][1], m * R2[0][2]);
-    acc_shfl(ja, src);
-    acc_shfl(jb, src);
-  }
-#pragma unroll
-  for (int t = 0; t < NI; t++) {
-    mir_store(o + t * 320, lane, ga[t], false);
-    mir_store(o + t * 320 + 160, lane, gb[t], false);
-  }
-  // after the last hand-over lane L holds the reverse sums of j = (L + kend) mod 32
-  const int kend = DIAG ? 17 : 32;
-  const int jf = (lane + kend) & 31;
-  double *oj = o + (DIAG ? 1 : NI) * 320;
-  mir_store(oj, jf, ja, V);
-  mir_store(oj + 160, jf, jb, V);
-}
-
-template <int MINB, bool MASK>
-__global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_mir_kernel(int64_t N, int64_t H, int64_t nitems_b,
-                                                                         int64_t nslots, int64_t nitems,
-                                                                         const MirItem *__restrict__ items,
-                                                                         const double *__restrict__ rU,
-                                                                         const double *__restrict__ zU,
-                                                                         const int32_t *__restrict__ pu,
-                                                                         const int32_t *__restrict__ pm,
-                                                                         const double *__restrict__ wT,
-                                                                         double *__restrict__ part) {
-  __shared__ double2 s_j[kSymWarps][32 * 5];   // per j: (r, z_src), W1 (d, kr), (W1 kz, W2 d), W2 (kr, kz), (r^2, -)
-  __shared__ double s_coef[kNumPairCoef];
-  __shared__ double2 s_ltab[kLogTab];
-  stage_pair_coef(s_coef, s_ltab);
-  __syncthreads();
-  PairCoef cf;
-  load_pair_coef(s_coef, s_ltab, cf);
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
-    const int64_t bb = item / nitems_b;
-    const MirItem it = items[item % nitems_b];
-    const double *wb = wT + bb * 3 * N;
-    __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
-    {   // stage the j-tile: U items see j at (r, z) with W1 = A(j), W2 = Bf(j); V items see j' at
-        // (r, -z) with W1 = F Bf(j) (= the weights of j'), W2 = F A(j)
-      const int64_t j = (int64_t)it.b * 32 + lane;
-      double A[3], Bf[3];
-      mir_weights(wb, N, H, pu, pm, j, A, Bf);
-      const double r = j < H ? rU[j] : 1.0;
-      const double z = j < H ? zU[j] : 2.0e6 + lane;
-      double2 *d = &s_j[wid][lane * 5];
-      if (it.v) {
-        d[0] = make_double2(r, -z);
-        d[1] = make_double2(Bf[0], Bf[1]);
-        d[2] = make_double2(-Bf[2], A[0]);
-        d[3] = make_double2(A[1], -A[2]);
-      } else {
-        d[0] = make_double2(r, z);
-        d[1] = make_double2(A[0], A[1]);
-        d[2] = make_double2(A[2], Bf[0]);
-        d[3] = make_double2(Bf[1], Bf[2]);
-      }
-      d[4] = make_double2(r * r, 0.0);
-    }
-    __syncwarp();
-    double *o = part + (bb * nslots + it.slot) * 320;
-    switch (it.n) {
-      case 0: mir_run<1, true, MASK>(it, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, o); break;
-      case 1: mir_run<1, false, MASK>(it, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, o); break;
-      default:
-        if constexpr (kSymNI >= 2) mir_run<2, false, MASK>(it, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, o);
-        break;
-    }
-  }
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -562,12 +395,15 @@ __device__ __forceinline__ void vtx_add_pm(double *sGa, double *sGb, int64_t Hp,
   vtx_add(sGb, Hp, pos, Acc5{P.drr - M.drr, P.drz - M.drz, P.dzz - M.dzz, P.kr - M.kr, P.kz - M.kz});
 }
 
-// one (a, b) item of a vertex; s_j: the warp's staged j-tile b as (r, z), (hp_d, hp_kr), (hp_kz, hm_d),
-// (hm_kr, hm_kz), (r^2, -); sGa, sGb: the CTA's shared accumulators [5][Hp]
+// One (a, b) item: lane L's target i = 32 a + L against j = 32 b + (L + k) mod 32, both tensor families;
+// returns the forward sums of i (P, M) and the reverse sums of j = 32 b + (L + kend(DIAG)) mod 32
+// (PJ, MJ), kend = 17 for the diagonal item and 32 (i.e. L) otherwise.  s_j: the warp's staged j-tile b
+// as (r, z), (hp_d, hp_kr), (hp_kz, hm_d), (hm_kr, hm_kz), (r^2, -).
 template <bool DIAG, bool MASK>
-__device__ __forceinline__ void vtx_run(int a, int b, const double *rU, const double *zU, const double *wb, int64_t N,
-                                        int64_t H, int64_t Hp, const int32_t *pu, const int32_t *pm, int lane,
-                                        const double2 *s_j, const PairCoef &cf, double *sGa, double *sGb) {
+__device__ __forceinline__ void vtx_item(int a, const double *rU, const double *zU, const double *wb, int64_t N,
+                                         int64_t H, const int32_t *pu, const int32_t *pm, int lane,
+                                         const double2 *s_j, const PairCoef &cf, Acc5 &P, Acc5 &M, Acc5 &PJ,
+                                         Acc5 &MJ) {
   const int64_t i = (int64_t)a * 32 + lane;
   double Ai[3], Bi[3], hpi[3], hmi[3];
   mir_weights(wb, N, H, pu, pm, i, Ai, Bi);
@@ -579,8 +415,7 @@ __device__ __forceinline__ void vtx_run(int a, int b, const double *rU, const do
   const double r = i < H ? rU[i] : 1.0;
   const double z = i < H ? zU[i] : 1.0e6 + lane;   // padding: far away, zero weights
   const double r2 = r * r;
-  Acc5 P{0.0, 0.0, 0.0, 0.0, 0.0}, M{0.0, 0.0, 0.0, 0.0, 0.0};
-  Acc5 PJ{0.0, 0.0, 0.0, 0.0, 0.0}, MJ{0.0, 0.0, 0.0, 0.0, 0.0};
+  P = M = PJ = MJ = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
   const int src = (lane + 1) & 31;
   if constexpr (DIAG) {   // step 0: each point with its own mirror (V forward only; U is the self pair)
     const double2 rz = s_j[lane * 5], p01 = s_j[lane * 5 + 1], p2m0 = s_j[lane * 5 + 2], m12 = s_j[lane * 5 + 3],
@@ -606,12 +441,65 @@ __device__ __forceinline__ void vtx_run(int a, int b, const double *rU, const do
     acc_shfl(PJ, src);
     acc_shfl(MJ, src);
   }
-  vtx_add_pm(sGa, sGb, Hp, i, P, M);
-  if constexpr (DIAG) __syncwarp();   // forward and reverse sums of a diagonal item hit the same tile
-  // after the last hand-over lane L holds the reverse sums of j = (L + kend) mod 32
-  const int kend = DIAG ? 17 : 32;
-  const int64_t jf = (int64_t)b * 32 + ((lane + kend) & 31);
-  vtx_add_pm(sGa, sGb, Hp, jf, PJ, MJ);
+}
+
+// stage j-tile b of batch item wb into the warp's buffer (see vtx_item)
+__device__ __forceinline__ void vtx_stage_j(int b, const double *rU, const double *zU, const double *wb, int64_t N,
+                                            int64_t H, const int32_t *pu, const int32_t *pm, int lane, double2 *d) {
+  const int64_t j = (int64_t)b * 32 + lane;
+  double A[3], Bf[3];
+  mir_weights(wb, N, H, pu, pm, j, A, Bf);
+  const double r = j < H ? rU[j] : 1.0;
+  const double z = j < H ? zU[j] : 2.0e6 + lane;
+  d += lane * 5;   // (r, z), hp = (A + Bf)/2, hm = (A - Bf)/2, (r^2, -)
+  d[0] = make_double2(r, z);
+  d[1] = make_double2(0.5 * (A[0] + Bf[0]), 0.5 * (A[1] + Bf[1]));
+  d[2] = make_double2(0.5 * (A[2] + Bf[2]), 0.5 * (A[0] - Bf[0]));
+  d[3] = make_double2(0.5 * (A[1] - Bf[1]), 0.5 * (A[2] - Bf[2]));
+  d[4] = make_double2(r * r, 0.0);
+}
+
+// N2 (mirror-symmetric, partial-sum slots): the same (a, b) items as the per-vertex kernel, spread
+// over every warp of the GPU (batches below one vertex per SM, single large meshes such as C5); each
+// item stores Ga, Gb of its i-tile (slot 2q) and of its j-tile (slot 2q + 1), reduce_mir_kernel sums
+// each tile's slots in a fixed host-built order.  part = [batch][nslots][2][5][32].
+template <int MINB, bool MASK>
+__global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_mir_kernel(int64_t N, int64_t H, int64_t nitems_b,
+                                                                         int64_t nslots, int64_t nitems,
+                                                                         const int2 *__restrict__ items,
+                                                                         const double *__restrict__ rU,
+                                                                         const double *__restrict__ zU,
+                                                                         const int32_t *__restrict__ pu,
+                                                                         const int32_t *__restrict__ pm,
+                                                                         const double *__restrict__ wT,
+                                                                         double *__restrict__ part) {
+  __shared__ double2 s_j[kSymWarps][32 * 5];
+  __shared__ double s_coef[kNumPairCoef];
+  __shared__ double2 s_ltab[kLogTab];
+  stage_pair_coef(s_coef, s_ltab);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, s_ltab, cf);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
+    const int64_t bb = item / nitems_b, q = item % nitems_b;
+    const int2 it = items[q];
+    const double *wb = wT + bb * 3 * N;
+    __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
+    vtx_stage_j(it.y, rU, zU, wb, N, H, pu, pm, lane, s_j[wid]);
+    __syncwarp();
+    Acc5 P, M, PJ, MJ;
+    if (it.x == it.y)
+      vtx_item<true, MASK>(it.x, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
+    else
+      vtx_item<false, MASK>(it.x, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
+    double *o = part + (bb * nslots + 2 * q) * 320;
+    const int jf = (lane + (it.x == it.y ? 17 : 32)) & 31;
+    mir_store(o, lane, Acc5{P.drr + M.drr, P.drz + M.drz, P.dzz + M.dzz, P.kr + M.kr, P.kz + M.kz}, false);
+    mir_store(o + 160, lane, Acc5{P.drr - M.drr, P.drz - M.drz, P.dzz - M.dzz, P.kr - M.kr, P.kz - M.kz}, false);
+    mir_store(o + 320, jf, Acc5{PJ.drr + MJ.drr, PJ.drz + MJ.drz, PJ.dzz + MJ.dzz, PJ.kr + MJ.kr, PJ.kz + MJ.kz}, false);
+    mir_store(o + 480, jf, Acc5{PJ.drr - MJ.drr, PJ.drz - MJ.drz, PJ.dzz - MJ.dzz, PJ.kr - MJ.kr, PJ.kz - MJ.kz}, false);
+  }
 }
 
 #ifndef LANDAU_VTX_WARPS
@@ -655,24 +543,16 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
       for (int q = round_ptr[rd] + wid; q < round_ptr[rd + 1]; q += kVtxWarps) {
         const VtxItem it = items[q];
         __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
-        {
-          const int64_t j = (int64_t)it.b * 32 + lane;
-          double A[3], Bf[3];
-          mir_weights(wb, N, H, pu, pm, j, A, Bf);
-          const double r = j < H ? rU[j] : 1.0;
-          const double z = j < H ? zU[j] : 2.0e6 + lane;
-          double2 *d = &s_j[wid][lane * 5];   // (r, z), hp = (A + Bf)/2, hm = (A - Bf)/2, (r^2, -)
-          d[0] = make_double2(r, z);
-          d[1] = make_double2(0.5 * (A[0] + Bf[0]), 0.5 * (A[1] + Bf[1]));
-          d[2] = make_double2(0.5 * (A[2] + Bf[2]), 0.5 * (A[0] - Bf[0]));
-          d[3] = make_double2(0.5 * (A[1] - Bf[1]), 0.5 * (A[2] - Bf[2]));
-          d[4] = make_double2(r * r, 0.0);
-        }
+        vtx_stage_j(it.b, rU, zU, wb, N, H, pu, pm, lane, s_j[wid]);
         __syncwarp();
+        Acc5 P, M, PJ, MJ;
         if (it.a == it.b)
-          vtx_run<true, MASK>(it.a, it.b, rU, zU, wb, N, H, Hp, pu, pm, lane, s_j[wid], cf, sGa, sGb);
+          vtx_item<true, MASK>(it.a, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
         else
-          vtx_run<false, MASK>(it.a, it.b, rU, zU, wb, N, H, Hp, pu, pm, lane, s_j[wid], cf, sGa, sGb);
+          vtx_item<false, MASK>(it.a, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
+        vtx_add_pm(sGa, sGb, Hp, (int64_t)it.a * 32 + lane, P, M);
+        if (it.a == it.b) __syncwarp();   // forward and reverse sums of a diagonal item hit the same tile
+        vtx_add_pm(sGa, sGb, Hp, (int64_t)it.b * 32 + ((lane + (it.a == it.b ? 17 : 32)) & 31), PJ, MJ);
       }
       __syncthreads();   // the next round's tiles may be this round's
     }

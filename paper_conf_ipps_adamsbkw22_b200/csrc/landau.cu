@@ -89,7 +89,7 @@ struct landau_s {
   size_t vtx_smem = 0;     // dynamic shared memory (Ga, Gb); 0 when the vertex does not fit
   double *d_rU = nullptr, *d_zU = nullptr;
   int32_t *d_pu = nullptr, *d_pm = nullptr;
-  MirItem *d_mir_items = nullptr;
+  int2 *d_mir_items = nullptr;
   int32_t *d_mtile_ptr = nullptr, *d_mtile_slots = nullptr;
   bool coincident = false;   // two distinct quadrature points with identical (r, z) (never for one grid)
   // tensor cache (NEXT-4)
@@ -908,25 +908,18 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     if (ok && !pu.empty()) {
       const int64_t H = (int64_t)pu.size();
       const int T = (int)((H + 31) / 32);
-      std::vector<MirItem> items;
+      // slot-kernel items: every tile pair (a <= b) once, U and V together; item q stores the sums of
+      // its i-tile a in slot 2q and of its j-tile b in slot 2q + 1
+      std::vector<int2> items;
       std::vector<std::vector<int32_t>> slots_of(T);
-      int slot = 0;
-      for (int v = 0; v < 2; v++)
-        for (int b = 0; b < T; b++) {
-          items.push_back({{b, -1, -1}, b, 0, v, slot});
-          slots_of[b].push_back(slot);
-          slots_of[b].push_back(slot + 1);
-          slot += 2;
-          for (int a = 0; a < b; a += std::min(kSymNI, 2)) {
-            MirItem it{{-1, -1, -1}, b, std::min(std::min(kSymNI, 2), b - a), v, slot};
-            for (int t = 0; t < it.n; t++) {
-              it.a[t] = a + t;
-              slots_of[a + t].push_back(slot++);
-            }
-            slots_of[b].push_back(slot++);
-            items.push_back(it);
-          }
+      for (int b = 0; b < T; b++)
+        for (int a = 0; a <= b; a++) {
+          const int q = (int)items.size();
+          items.push_back(make_int2(a, b));
+          slots_of[a].push_back(2 * q);
+          slots_of[b].push_back(2 * q + 1);
         }
+      const int slot = 2 * (int)items.size();
       std::vector<int32_t> tptr(1, 0), tslots;
       for (int t = 0; t < T; t++) {
         tslots.insert(tslots.end(), slots_of[t].begin(), slots_of[t].end());
