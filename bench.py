@@ -156,8 +156,8 @@ FLOP_PER_PAIR_DIRECTED = 177.0
 FLOP_PER_PAIR_SYMMETRIC = 193.0
 # mirror-symmetric kernel: FP64 FLOP (2 DFMA + DMUL + DADD, ncu SASS counts on C4) per tensor
 # evaluation, (N/2)^2 evaluations per batch item (profiles/r01_flops_mirror.csv)
-FLOP_PER_EVAL_MIRROR = 222.9   # inner_mir_kernel (slot kernel)
-FLOP_PER_EVAL_VTX = 219.3      # inner_vtx_kernel (per-vertex kernel; profiles/r01_flops_vtx.csv)
+FLOP_PER_EVAL_MIRROR = 198.7   # inner_mir_kernel (slot kernel; profiles/r01_flops_mirror.csv)
+FLOP_PER_EVAL_VTX = 199.0      # inner_vtx_kernel (per-vertex kernel; profiles/r01_flops_vtx.csv)
 
 
 def cpu_baseline(args, desc, nsample):
