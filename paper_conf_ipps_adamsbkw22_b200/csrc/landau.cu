@@ -329,10 +329,19 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
   }
   ip.tpt = variant == 0 ? 1 : (variant == 4 ? 4 : 2);
   ip.wtiles = (nt + 32 * ip.tpt - 1) / (32 * ip.tpt);
-  // split-j so that small problems still fill the machine: aim for >= 12 warps per SM
-  const int64_t want = 12LL * num_sms(h);
+  // split-j so that small problems still fill the machine: aim for >= LANDAU_SPLIT_WARPS_PER_SM
+  // warps per SM, splits of at least LANDAU_SPLIT_MIN sources
+  static const int64_t split_wps = [] {
+    const char *e = getenv("LANDAU_SPLIT_WARPS_PER_SM");
+    return e ? (int64_t)atoll(e) : (int64_t)12;
+  }();
+  static const int64_t split_min = [] {
+    const char *e = getenv("LANDAU_SPLIT_MIN");
+    return e ? (int64_t)atoll(e) : (int64_t)32;
+  }();
+  const int64_t want = split_wps * num_sms(h);
   int64_t nsplit = std::max<int64_t>(1, (want + ip.wtiles * nbatch - 1) / (ip.wtiles * nbatch));
-  nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, N / 32));
+  nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, N / split_min));
   ip.split_len = (N + nsplit - 1) / nsplit;
   ip.nsplit = (N + ip.split_len - 1) / ip.split_len;
   if (ip.nsplit > 1) {
