@@ -240,7 +240,11 @@ int launch_field(landau_t h, int64_t nbatch) {
   constexpr int EPB = NB == 9 ? 8 : (NB == 16 ? 8 : 4);
   const Plan &P = h->plan;
   const int64_t items = (P.ncell + EPB - 1) / EPB * nbatch;
-  const unsigned grid = (unsigned)std::min<int64_t>(items, 8LL * num_sms(h));
+  static const int64_t blocks_per_sm = [] {   // grid cap (LANDAU_FIELD_BLOCKS_PER_SM)
+    const char *e = getenv("LANDAU_FIELD_BLOCKS_PER_SM");
+    return e ? (int64_t)atoll(e) : (int64_t)8;
+  }();
+  const unsigned grid = (unsigned)std::min<int64_t>(items, blocks_per_sm * num_sms(h));
   Timer t(h, LANDAU_T_FIELD);
   field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->fin ? h->fin : h->d_f,
                                                           h->d_ext_ptr, h->d_ext_dof,
