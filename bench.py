@@ -158,6 +158,7 @@ FLOP_PER_PAIR_SYMMETRIC = 193.0
 # evaluation, (N/2)^2 evaluations per batch item (profiles/r01_flops_mirror.csv)
 FLOP_PER_EVAL_MIRROR = 198.7   # inner_mir_kernel (slot kernel; profiles/r01_flops_mirror.csv)
 FLOP_PER_EVAL_VTX = 199.0      # inner_vtx_kernel (per-vertex kernel; profiles/r01_flops_vtx.csv)
+FLOP_PER_EVAL_MDIR = 187.4     # inner_mdir_kernel (mirror directed, per padded U or V evaluation; profiles/r01_flops_mdir.csv)
 
 
 def cpu_baseline(args, desc, nsample):
@@ -350,6 +351,9 @@ def main():
     if st["inner_path"] == 2:   # GEMMs: 2 FLOP per multiply-add, 7 N^2 per batch item (three DGEMMs)
         flop_per_pair = 14.0
         flops_per_launch = 14.0 * st["nbatch"] * N * N
+    elif st["inner_path"] == 5:
+        flop_per_pair = FLOP_PER_EVAL_MDIR
+        flops_per_launch = flop_per_pair * st["nbatch"] * st["pair_evaluations"]
     elif st["inner_path"] in (3, 4):
         flop_per_pair = FLOP_PER_EVAL_VTX if st["inner_path"] == 4 else FLOP_PER_EVAL_MIRROR
         flops_per_launch = flop_per_pair * st["nbatch"] * (N // 2) ** 2
@@ -372,7 +376,8 @@ def main():
             "inner_path": ["directed (ordered pairs)", "symmetric (unordered pairs)",
                            "tensor cache + FP64 DGEMM (cuBLAS)",
                            "mirror-symmetric (one tensor per unordered pair and its z-mirror)",
-                           "mirror-symmetric, one CTA per vertex (sums in shared memory)"][st["inner_path"]],
+                           "mirror-symmetric, one CTA per vertex (sums in shared memory)",
+                           "mirror-symmetric directed (U + V per target and source, forward sums)"][st["inner_path"]],
             "flop_per_pair": flop_per_pair, "flops_per_launch": flops_per_launch,
             "inner_ms_per_launch": inner_avg_s * 1e3,
             "inner_share_of_step": (inner_ms / args.steps) / ms_per_step if ms_per_step else None,
@@ -495,7 +500,7 @@ def main():
             ms2 = sum(a.elapsed_time(b) for a, b in ev2) / args.steps
             line["c2_single_build"] = {"value": 1e3 / ms2, "unit": UNIT, "ms_per_step": ms2,
                                        "pairs_per_s": 1e3 / ms2 * p2.npoints ** 2,
-                                       "inner_path": ["directed", "symmetric", "tensor cache", "mirror", "mirror per-vertex"][h2.stats()["inner_path"]],
+                                       "inner_path": ["directed", "symmetric", "tensor cache", "mirror", "mirror per-vertex", "mirror directed"][h2.stats()["inner_path"]],
                                        "note": "BASELINE configs[1]: one e+D Q3 AMR grid (N=1088) per step, "
                                                "set_state + jacobian (CSR) + mass, CUDA-graph replay"}
             h2.close()

@@ -567,6 +567,120 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
   }
 }
 
+// ------------------------------------------------------------------------------------------------
+// N2 (mirror-symmetric, directed): single builds and batches too small for the pair kernels.  A warp
+// owns 32 upper-half targets u of one batch item and one split of the upper-half sources j, staged 32
+// at a time and read by every lane at once (broadcast); each step evaluates U(u, j) and V(u, j) and
+// accumulates forward only, in the sum/difference form of vtx_step -- half the tensor evaluations of
+// the directed kernel (H^2 U + V pairs instead of N^2 ordered pairs), no shuffles.  The self pair
+// (U(u, u)) and any coincident points are masked.  nsplit == 1: G written directly; otherwise
+// partials [batch][nsplit][2][5][Hp] for reduce_mdir_kernel.
+// ------------------------------------------------------------------------------------------------
+constexpr int kMdirWarps = 4;
+
+__global__ void __launch_bounds__(32 * kMdirWarps) inner_mdir_kernel(int64_t N, int64_t H, int64_t wtiles,
+                                                                    int64_t split_len, int nsplit, int64_t nitems,
+                                                                    const double *__restrict__ rU,
+                                                                    const double *__restrict__ zU,
+                                                                    const int32_t *__restrict__ pu,
+                                                                    const int32_t *__restrict__ pm,
+                                                                    const double *__restrict__ wT,
+                                                                    double *__restrict__ G, int64_t G_bstride,
+                                                                    double *__restrict__ part) {
+  __shared__ double2 s_j[kMdirWarps][32 * 5];
+  __shared__ double s_coef[kNumPairCoef];
+  __shared__ double2 s_ltab[kLogTab];
+  stage_pair_coef(s_coef, s_ltab);
+  __syncthreads();
+  PairCoef cf;
+  load_pair_coef(s_coef, s_ltab, cf);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t item = (int64_t)blockIdx.x * kMdirWarps + wid;
+  if (item >= nitems) return;   // whole warp: no block-level barrier follows
+  const int64_t b = item / (nsplit * wtiles), rem = item % (nsplit * wtiles);
+  const int sp = (int)(rem / wtiles);
+  const int64_t u = (rem % wtiles) * 32 + lane;
+  const double *wb = wT + b * 3 * N;
+  const double r = u < H ? rU[u] : 1.0;
+  const double z = u < H ? zU[u] : 1.0e6 + lane;   // padding: far away, never stored
+  const double r2 = r * r;
+  const double nohp[3] = {0.0, 0.0, 0.0};
+  Acc5 P{0.0, 0.0, 0.0, 0.0, 0.0}, M{0.0, 0.0, 0.0, 0.0, 0.0}, PJ, MJ;
+  const int64_t j0 = (int64_t)sp * split_len, j1 = min(H, j0 + split_len);
+  double2 *sj = s_j[wid];
+  for (int64_t jt = j0; jt < j1; jt += 32) {
+    __syncwarp();
+    {   // stage sources jt .. jt + 31 (zero weights past j1)
+      const int64_t j = jt + lane;
+      double A[3], Bf[3];
+      mir_weights(wb, N, j1, pu, pm, j, A, Bf);
+      const double rj = j < j1 ? rU[j] : 1.0;
+      const double zj = j < j1 ? zU[j] : 2.0e6 + lane;
+      double2 *d = sj + lane * 5;
+      d[0] = make_double2(rj, zj);
+      d[1] = make_double2(0.5 * (A[0] + Bf[0]), 0.5 * (A[1] + Bf[1]));
+      d[2] = make_double2(0.5 * (A[2] + Bf[2]), 0.5 * (A[0] - Bf[0]));
+      d[3] = make_double2(0.5 * (A[1] - Bf[1]), 0.5 * (A[2] - Bf[2]));
+      d[4] = make_double2(rj * rj, 0.0);
+    }
+    __syncwarp();
+    const int n = (int)min((int64_t)32, j1 - jt);
+    for (int k = 0; k < n; k++) {
+      const double2 rz = sj[k * 5], p01 = sj[k * 5 + 1], p2m0 = sj[k * 5 + 2], m12 = sj[k * 5 + 3],
+                    rr2 = sj[k * 5 + 4];
+      vtx_step<true, false, true>(r, z, r2, nohp, nohp, rz.x, rz.y, rr2.x, p01, p2m0, m12, cf, 1.0, P, M, PJ, MJ);
+    }
+  }
+  if (u >= H) return;
+  const Acc5 ga{P.drr + M.drr, P.drz + M.drz, P.dzz + M.dzz, P.kr + M.kr, P.kz + M.kz};
+  const Acc5 gb{P.drr - M.drr, P.drz - M.drz, P.dzz - M.dzz, P.kr - M.kr, P.kz - M.kz};
+  if (nsplit == 1) {   // G(pu) = Ga, G(pm) = F Gb
+    double *Gb = G + b * G_bstride;
+    const int64_t p = pu[u], q = pm[u];
+    Gb[p] = ga.drr;
+    Gb[N + p] = ga.drz;
+    Gb[2 * N + p] = ga.dzz;
+    Gb[3 * N + p] = ga.kr;
+    Gb[4 * N + p] = ga.kz;
+    Gb[q] = gb.drr;
+    Gb[N + q] = -gb.drz;
+    Gb[2 * N + q] = gb.dzz;
+    Gb[3 * N + q] = gb.kr;
+    Gb[4 * N + q] = -gb.kz;
+  } else {
+    const int64_t Hp = wtiles * 32;
+    double *o = part + ((b * nsplit + sp) * 10) * Hp + u;
+    o[0] = ga.drr;
+    o[Hp] = ga.drz;
+    o[2 * Hp] = ga.dzz;
+    o[3 * Hp] = ga.kr;
+    o[4 * Hp] = ga.kz;
+    o[5 * Hp] = gb.drr;
+    o[6 * Hp] = gb.drz;
+    o[7 * Hp] = gb.dzz;
+    o[8 * Hp] = gb.kr;
+    o[9 * Hp] = gb.kz;
+  }
+}
+
+// G[b][c][pu(u)] = sum over splits of Ga, G[b][c][pm(u)] = F (sum of Gb), splits in order
+__global__ void reduce_mdir_kernel(int64_t N, int64_t H, int64_t Hp, int nsplit, const int32_t *__restrict__ pu,
+                                   const int32_t *__restrict__ pm, const double *__restrict__ part,
+                                   double *__restrict__ G, int64_t G_bstride, int nbatch) {
+  const int64_t total = (int64_t)nbatch * 5 * H;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = k / (5 * H), c = (k / H) % 5, u = k % H;
+    const double *pb = part + b * nsplit * 10 * Hp + c * Hp + u;
+    double sa = 0.0, sb = 0.0;
+    for (int q = 0; q < nsplit; q++) {
+      sa += pb[(int64_t)q * 10 * Hp];
+      sb += pb[(int64_t)q * 10 * Hp + 5 * Hp];
+    }
+    G[b * G_bstride + c * N + pu[u]] = sa;
+    G[b * G_bstride + c * N + pm[u]] = (c == 1 || c == 4) ? -sb : sb;
+  }
+}
+
 // G[b][c][pu(u)] = sum of the Ga parts, G[b][c][pm(u)] = F (sum of the Gb parts), over the slots of
 // u's tile in the fixed order of tile_slots
 __global__ void reduce_mir_kernel(int64_t N, int64_t H, int64_t nslots, const int32_t *__restrict__ tile_ptr,

@@ -258,6 +258,7 @@ int launch_field(landau_t h, int64_t nbatch) {
 
 struct InnerPlan {
   bool sym;   // symmetric pair evaluation (whole point set as targets, enough tile pairs to fill the GPU)
+  bool mdir = false;   // mirror-symmetric directed kernel (single builds / small batches on z-mirror meshes)
   int tpt;
   int64_t wtiles, nsplit, split_len;
 };
@@ -328,6 +329,40 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
       h->d_part = nullptr;
       CU(cudaMalloc(&h->d_part, sizeof(double) * need));
       h->part_cap = need;
+    }
+    return LANDAU_OK;
+  }
+  static const bool mdir_on = [] {
+    const char *e = getenv("LANDAU_MDIR");
+    return !(e && atoi(e) == 0);
+  }();
+  if (mdir_on && h->mirror && h->mirror_on) {   // targets and sources: the H upper-half points
+    const int64_t T = (h->H + 31) / 32;
+    ip.mdir = true;
+    ip.tpt = 1;
+    ip.wtiles = T;
+    static const int64_t mdir_wps = [] {   // warps per SM to aim for, minimum sources per split
+      const char *e = getenv("LANDAU_MDIR_WARPS_PER_SM");
+      return e ? (int64_t)atoll(e) : (int64_t)12;
+    }();
+    static const int64_t mdir_min = [] {
+      const char *e = getenv("LANDAU_MDIR_SPLIT_MIN");
+      return e ? (int64_t)atoll(e) : (int64_t)16;   // measured: 16 best on C2/C3 (finer splits cost reduction time)
+    }();
+    const int64_t want = mdir_wps * num_sms(h);
+    int64_t nsplit = std::max<int64_t>(1, (want + T * nbatch - 1) / (T * nbatch));
+    nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, h->H / mdir_min));
+    ip.split_len = (h->H + nsplit - 1) / nsplit;
+    ip.nsplit = (h->H + ip.split_len - 1) / ip.split_len;
+    if (ip.nsplit > 1) {
+      const int64_t need = nbatch * ip.nsplit * 10 * T * 32;
+      if (need > h->part_cap) {
+        drop_graphs(h);
+        cudaFree(h->d_part);
+        h->d_part = nullptr;
+        CU(cudaMalloc(&h->d_part, sizeof(double) * need));
+        h->part_cap = need;
+      }
     }
     return LANDAU_OK;
   }
@@ -508,6 +543,39 @@ int launch_inner(landau_t h, int64_t nbatch) {
     h->launches++;
     h->tlaunch[LANDAU_T_REDUCE]++;
     KCHECK();
+    return LANDAU_OK;
+  }
+  if (ip.mdir) {   // mirror-symmetric directed kernel
+    const int64_t T = ip.wtiles;
+    h->stats.inner_path = 5;
+    h->stats.nsplit = nsplit;
+    h->stats.pair_evaluations = T * 32 * h->H * 2;   // U + V per (target, source), padded targets
+    {
+      Timer t(h, LANDAU_T_INNER);
+      const int64_t nitems = nbatch * nsplit * T;
+      const unsigned grid = (unsigned)((nitems + kMdirWarps - 1) / kMdirWarps);
+      inner_mdir_kernel<<<grid, 32 * kMdirWarps, 0, h->stream>>>(N, h->H, T, split_len, (int)nsplit, nitems, h->d_rU,
+                                                                 h->d_zU, h->d_pu, h->d_pm, h->d_wT, G_own, 5 * h->Nc,
+                                                                 h->d_part);
+      h->launches++;
+      h->tlaunch[LANDAU_T_INNER]++;
+      KCHECK();
+    }
+    if (nsplit > 1) {
+      Timer t(h, LANDAU_T_REDUCE);
+      const int64_t total = nbatch * 5 * h->H;
+      const int blocks = (int)std::min<int64_t>((total + 255) / 256, 16LL * num_sms(h));
+      reduce_mdir_kernel<<<blocks, 256, 0, h->stream>>>(N, h->H, T * 32, (int)nsplit, h->d_pu, h->d_pm, h->d_part, G_own,
+                                                        5 * h->Nc, (int)nbatch);
+      h->launches++;
+      h->tlaunch[LANDAU_T_REDUCE]++;
+      KCHECK();
+    }
+    if (h->comm) {   // LANDAU_DIST_ELEMENTS at world 1: the (trivial) exchange step
+      Timer t(h, LANDAU_T_ALLGATHER);
+      int rc2 = g_nccl.AllGather(G_own, h->d_G, (size_t)(nbatch * 5 * h->Nc), kNcclFloat64, h->comm, h->stream);
+      if (rc2 != 0) return fail(h, LANDAU_ENCCL, "ncclAllGather failed");
+    }
     return LANDAU_OK;
   }
   double *out;
