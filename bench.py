@@ -372,6 +372,7 @@ def main():
     roof = {"bound": "alu", "kernel": "inner_vtx_kernel / inner_mir_kernel / inner_sym_kernel / inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
             "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None,
             "traffic": load_profile_traffic(args.workload),
+            "fp64_pipe_active_ncu": load_profile_traffic(args.workload + "_fp64_pipe_active"),
             "peak_note": f"derived FP64 DFMA peak: {props.multi_processor_count} SMs x 64 lanes x 2 FLOP x {sm_max:.0f} MHz",
             "inner_path": ["directed (ordered pairs)", "symmetric (unordered pairs)",
                            "tensor cache + FP64 DGEMM (cuBLAS)",
