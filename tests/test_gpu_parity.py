@@ -717,3 +717,42 @@ def test_vertex_kernel_hybrid_remainder():
     h.jacobian_batched(out2)
     assert h.stats()["inner_path"] == 3
     assert np.abs(out2.cpu().numpy() - Jb).max() <= 1e-13 * np.abs(Jb).max()
+
+
+def test_mirror_directed_kernel_unsplit():
+    """The mirror-symmetric directed kernel writes G directly when one source split suffices (a batch
+    large enough to fill the GPU with target tiles alone); the pair kernels are switched off in a
+    child process (LANDAU_SYM=0 is read once per process) so the path runs, and each item is checked
+    against the oracle."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import os, sys, numpy as np, torch
+sys.path.insert(0, os.getcwd())
+from oracle.oracle import Oracle
+from paper_conf_ipps_adamsbkw22_b200 import inputs
+from paper_conf_ipps_adamsbkw22_b200 import landau as L
+nb = 160
+p0 = inputs.config4_vertex(0)
+h = L.Landau.from_problem(p0, device=0)
+nodes = h.all_nodes()
+verts = [0, 511, 1023]
+F = np.stack([inputs.coefficients(inputs.config4_vertex(verts[k % 3]), nodes) for k in range(nb)])
+h.set_state_batched(torch.tensor(F, device="cuda"))
+G = torch.empty((nb, 5, h.npoints), dtype=torch.float64, device="cuda")
+h.point_coeffs_batched(G)
+torch.cuda.synchronize()
+st = h.stats()
+assert st["inner_path"] == 5 and st["nsplit"] == 1, st
+for k in range(3):
+    o = Oracle(inputs.config4_vertex(verts[k]))
+    Go, Ga = o.point_coeffs(o.coefficients())
+    e = float(np.max(np.abs(G[k].cpu().numpy() - Go) / Ga))
+    assert e <= 1e-12, (k, e)
+print("ok")
+'''
+    env = dict(os.environ, LANDAU_SYM="0")
+    out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600, env=env,
+                         cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    assert out.returncode == 0 and out.stdout.strip().endswith("ok"), out.stderr[-3000:]
