@@ -260,8 +260,8 @@ def main():
             dist_desc = {"rank": 0, "world": 1, "mode": L.LANDAU_DIST_ELEMENTS,
                          "nccl_unique_id": L.landau_nccl_unique_id()}
         items = [prob0]
-        desc = dict(desc, workload="C5: one e+D Q4 mesh (4352 cells, N=108800), target cells split over the GPUs, "
-                                   "NCCL all-gather of G")
+        desc = dict(desc, workload="C5: one e+D Q4 mesh (4352 cells, N=108800), LANDAU_DIST_ELEMENTS: the mirror "
+                                   "kernel's tile pairs split over the GPUs, NCCL all-reduce of the partial G")
     with StdoutToStderr():
         h = L.Landau.from_problem(prob0, device=local, stream=stream, dist=dist_desc)
     if args.tensor_cache:
@@ -356,7 +356,9 @@ def main():
         flops_per_launch = flop_per_pair * st["nbatch"] * st["pair_evaluations"]
     elif st["inner_path"] in (3, 4):
         flop_per_pair = FLOP_PER_EVAL_VTX if st["inner_path"] == 4 else FLOP_PER_EVAL_MIRROR
-        flops_per_launch = flop_per_pair * st["nbatch"] * (N // 2) ** 2
+        # (N/2)^2 U + V evaluations per batch item (+ the N/2 self-mirror pairs and tile padding); with
+        # the pair split, this rank's share
+        flops_per_launch = flop_per_pair * st["nbatch"] * st["pair_evaluations"]
     elif st["inner_path"] == 1:
         flop_per_pair = FLOP_PER_PAIR_SYMMETRIC
         flops_per_launch = flop_per_pair * st["nbatch"] * N * (N - 1) / 2

@@ -90,8 +90,14 @@ typedef struct {
   const void *nccl_unique_id;  /* 128 bytes from landau_nccl_unique_id on rank 0, broadcast by the
                                   caller (torch.distributed); only read for LANDAU_DIST_ELEMENTS   */
   int32_t mode;                /* LANDAU_DIST_*: REPLICATE and BATCH need no communicator (the
-                                  caller splits batches); ELEMENTS splits target cells into world
-                                  contiguous equal ranges and all-gathers G over NCCL              */
+                                  caller splits batches); ELEMENTS distributes one mesh's inner
+                                  integral over the ranks: on a z-mirror mesh (every configuration
+                                  of SURVEY §8(d)) the upper-half tile pairs are split into world
+                                  contiguous equal-work ranges (landau_pair_partition) and the
+                                  partial G summed by one NCCL all-reduce; otherwise the target
+                                  cells are split into world contiguous equal ranges
+                                  (landau_partition) and G all-gathered over NCCL.  Every rank then
+                                  forms the element matrices and the full CSR/COO itself.          */
 } landau_dist_t;
 
 /* cuda_device = LANDAU_HOST_ONLY builds only the host-side plan (sizes, nodes, points, patterns can
@@ -146,6 +152,13 @@ int landau_point_coeffs_batched(landau_t h, int64_t nbatch, double *G_dev);
 /* Element split (LANDAU_DIST_ELEMENTS): contiguous cell range [e0, e1) owned by a rank for a mesh
  * of nelem cells; pure host arithmetic, usable without a GPU. */
 int landau_partition(int64_t nelem, int32_t world, int32_t rank, int64_t *e0, int64_t *e1);
+/* Pair split (LANDAU_DIST_ELEMENTS on a z-mirror mesh): the mirror kernel's items -- tile pairs
+ * (a, b), a <= b, in the order b = 0.., a = 0..b, ntiles (T) upper-half tiles of 32 points,
+ * T (T + 1) / 2 items -- weighted 2 per pair and 1 per diagonal item (half its steps); rank takes
+ * the contiguous item range [q0, q1) whose weight prefix covers [rank T^2 / world,
+ * (rank + 1) T^2 / world).  Pure host arithmetic.  EINVAL: ntiles < 0, world < 1, rank outside
+ * [0, world), NULL outputs. */
+int landau_pair_partition(int64_t ntiles, int32_t world, int32_t rank, int64_t *q0, int64_t *q1);
 /* 128-byte NCCL unique id (rank 0 only; loads libnccl.so.2 on demand). */
 int landau_nccl_unique_id(void *out128);
 

@@ -19,6 +19,7 @@ struct NcclApi {
   int (*GetUniqueId)(ncclUniqueId_ *) = nullptr;
   int (*CommInitRank)(ncclComm_ *, int, ncclUniqueId_, int) = nullptr;
   int (*AllGather)(const void *, void *, size_t, int, ncclComm_, cudaStream_t) = nullptr;
+  int (*AllReduce)(const void *, void *, size_t, int, int, ncclComm_, cudaStream_t) = nullptr;
   int (*CommDestroy)(ncclComm_) = nullptr;
   const char *(*GetErrorString)(int) = nullptr;
 };
@@ -35,13 +36,16 @@ bool load_nccl() {
   g_nccl.GetUniqueId = (int (*)(ncclUniqueId_ *))dlsym(so, "ncclGetUniqueId");
   g_nccl.CommInitRank = (int (*)(ncclComm_ *, int, ncclUniqueId_, int))dlsym(so, "ncclCommInitRank");
   g_nccl.AllGather = (int (*)(const void *, void *, size_t, int, ncclComm_, cudaStream_t))dlsym(so, "ncclAllGather");
+  g_nccl.AllReduce = (int (*)(const void *, void *, size_t, int, int, ncclComm_, cudaStream_t))dlsym(so, "ncclAllReduce");
   g_nccl.CommDestroy = (int (*)(ncclComm_))dlsym(so, "ncclCommDestroy");
   g_nccl.GetErrorString = (const char *(*)(int))dlsym(so, "ncclGetErrorString");
-  if (!g_nccl.GetUniqueId || !g_nccl.CommInitRank || !g_nccl.AllGather || !g_nccl.CommDestroy) return false;
+  if (!g_nccl.GetUniqueId || !g_nccl.CommInitRank || !g_nccl.AllGather || !g_nccl.AllReduce || !g_nccl.CommDestroy)
+    return false;
   g_nccl.so = so;
   return true;
 }
 constexpr int kNcclFloat64 = 8;
+constexpr int kNcclSum = 0;
 
 // cuBLAS, loaded on demand (only the tensor-cache path uses it: a plain library DGEMM)
 typedef void *cublasHandle_;

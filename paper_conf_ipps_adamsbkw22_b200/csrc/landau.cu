@@ -79,6 +79,8 @@ struct landau_s {
   // mirror-symmetric inner kernel (meshes symmetric under z -> -z): upper-half points u, their
   // original indices pu and mirrors pm, work items and slot map over the tiles of the upper half
   bool mirror = false;     // the mesh is mirror-symmetric (maps built)
+  bool dist_pairs = false; // element-split mode on a mirror mesh: tile pairs split over ranks + all-reduce
+  int64_t mir_evals = 0;   // tensor evaluations per batch item of this handle's slot-kernel items
   bool mirror_on = true;   // use inner_mir_kernel when the symmetric path runs (landau_set_mirror)
   int mirror_mode = 1;     // 1: auto (per-vertex kernel for large batches), 2: slot kernel, 3: per-vertex kernel
   int64_t H = 0, nmir_items = 0, nmir_slots = 0;
@@ -317,6 +319,7 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
   // fill the GPU, and partial slots within 24 GiB (C5: ~11 GiB of the 180 GB HBM)
   ip.sym = sym_enabled() && h->world == 1 && h->nsym_items > 0 && nbatch * h->nsym_items >= sym_min_items_per_sm() * num_sms(h) &&
            nbatch * h->nsym_slots * 160 * (int64_t)sizeof(double) <= (24LL << 30);
+  if (h->dist_pairs) ip.sym = true;   // the rank's share of the mirror items (slot kernel)
   if (ip.sym) {
     ip.tpt = 1;
     ip.wtiles = h->ntiles;
@@ -434,17 +437,17 @@ int launch_inner(landau_t h, int64_t nbatch) {
   if (rc) return rc;
   const int variant = inner_variant();
   const int64_t wtiles = ip.wtiles, nsplit = ip.nsplit, split_len = ip.split_len;
-  double *G_own = h->d_G + (int64_t)h->rank * nbatch * 5 * h->Nc;   // [world][batch][5][Nc]
+  // [world][batch][5][Nc] chunks (element split), or the one full [batch][5][N] block (pair split)
+  double *G_own = h->d_G + (h->dist_pairs ? 0 : (int64_t)h->rank * nbatch * 5 * h->Nc);
   h->stats.nbatch = nbatch;
   h->stats.targets = nt;
   h->stats.sources = N;
   h->stats.inner_path = ip.sym ? 1 : 0;
   h->stats.nsplit = ip.sym ? 1 : ip.nsplit;
   if (ip.sym && h->mirror && h->mirror_on) {
-    // tensor evaluations per batch item: U and V items over the T tiles of the upper half; diagonal
-    // items 16 (U) or 17 (V) steps x 32 lanes, the others 32 x 32 per i-tile
-    const int64_t T = (h->H + 31) / 32;
-    h->stats.pair_evaluations = T * 33 * 32 + 2 * (T * (T - 1) / 2) * 32 * 32;
+    // tensor evaluations per batch item (this rank's items): U + V items over the T tiles of the upper
+    // half; diagonal items 16 (U) + 17 (V) steps x 32 lanes, the others 2 x 32 x 32
+    h->stats.pair_evaluations = h->mir_evals;
     h->stats.inner_path = 3;
   } else if (ip.sym) {
     int64_t ev = 0;   // lane-steps per batch item: diagonal items 16 x 32, others 32 x 32 per i-tile
@@ -515,10 +518,18 @@ int launch_inner(landau_t h, int64_t nbatch) {
   if (ip.sym && h->mirror && h->mirror_on) {
     {
       Timer t(h, LANDAU_T_INNER);
-      if ((rc = mir_slots(0, nbatch))) return rc;
+      if (h->nmir_items && (rc = mir_slots(0, nbatch))) return rc;
       h->tlaunch[LANDAU_T_INNER]++;
     }
-    return mir_reduce(0, nbatch);
+    if ((rc = mir_reduce(0, nbatch))) return rc;
+    if (h->dist_pairs) {   // the exchange step: sum the ranks' partial G (every rank gets all of G)
+      Timer t(h, LANDAU_T_ALLGATHER);
+      const int rc2 = g_nccl.AllReduce(G_own, G_own, (size_t)(nbatch * 5 * h->Nc), kNcclFloat64, kNcclSum, h->comm,
+                                       h->stream);
+      if (rc2 != 0)
+        return fail(h, LANDAU_ENCCL, std::string("ncclAllReduce: ") + (g_nccl.GetErrorString ? g_nccl.GetErrorString(rc2) : "error"));
+    }
+    return LANDAU_OK;
   }
   if (ip.sym) {
     {
@@ -810,6 +821,28 @@ int landau_partition(int64_t nelem, int32_t world, int32_t rank, int64_t *e0, in
   return LANDAU_OK;
 }
 
+int landau_pair_partition(int64_t ntiles, int32_t world, int32_t rank, int64_t *q0, int64_t *q1) {
+  if (ntiles < 0 || world < 1 || rank < 0 || rank >= world || !q0 || !q1) return LANDAU_EINVAL;
+  // items in the slot kernel's order (b = 0.., a = 0..b), weight 2 per pair, 1 per diagonal item
+  // (half the steps); rank r takes the items whose weight prefix lies in [r W / world, (r+1) W / world)
+  const int64_t nitems = ntiles * (ntiles + 1) / 2, wtot = ntiles * ntiles;   // 2 T(T-1)/2 + T
+  const int64_t w0 = wtot * rank / world, w1 = wtot * (rank + 1) / world;
+  int64_t q = 0, acc = 0, lo = -1, hi = nitems;
+  for (int64_t b = 0; b < ntiles; b++)
+    for (int64_t a = 0; a <= b; a++, q++) {
+      if (lo < 0 && acc >= w0) lo = q;
+      if (acc >= w1) {
+        hi = q;
+        b = ntiles;
+        break;
+      }
+      acc += a == b ? 1 : 2;
+    }
+  *q0 = lo < 0 ? nitems : lo;
+  *q1 = std::max(*q0, hi);
+  return LANDAU_OK;
+}
+
 int landau_nccl_unique_id(void *out128) {
   if (!out128) return LANDAU_EINVAL;
   if (!load_nccl()) return LANDAU_ENCCL;
@@ -955,7 +988,9 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
         (rc = upload(h, &h->d_tile_slots, tslots)))
       return bail(rc);
   }
-  if (world == 1 && mirror_enabled()) {   // mirror symmetry z -> -z of every grid (inner_mir_kernel)
+  // mirror symmetry z -> -z of every grid (inner_mir_kernel); with several ranks (element split) the
+  // tile pairs are split over the ranks and the partial G summed by one all-reduce (pair split)
+  if ((world == 1 || mode == LANDAU_DIST_ELEMENTS) && mirror_enabled()) {
     std::vector<int32_t> pu, pm;
     std::vector<double> rU, zU;
     bool ok = true;
@@ -991,10 +1026,19 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
       const int T = (int)((H + 31) / 32);
       // slot-kernel items: every tile pair (a <= b) once, U and V together; item q stores the sums of
       // its i-tile a in slot 2q and of its j-tile b in slot 2q + 1
+      // (world > 1: this rank's share of the items, landau_pair_partition, with local slot numbers)
       std::vector<int2> items;
       std::vector<std::vector<int32_t>> slots_of(T);
+      int64_t iq0 = 0, iq1 = (int64_t)T * (T + 1) / 2, qg = 0;
+      if (world > 1) landau_pair_partition(T, world, rank, &iq0, &iq1);
+      if (world == 1)
+        if (const char *e = getenv("LANDAU_PAIR_SPLIT_EMULATE")) {   // test hook: "world:rank" -- this
+          int ew = 1, er = 0;                                         // rank's items only, no all-reduce
+          if (sscanf(e, "%d:%d", &ew, &er) == 2 && ew >= 1 && er >= 0 && er < ew) landau_pair_partition(T, ew, er, &iq0, &iq1);
+        }
       for (int b = 0; b < T; b++)
-        for (int a = 0; a <= b; a++) {
+        for (int a = 0; a <= b; a++, qg++) {
+          if (qg < iq0 || qg >= iq1) continue;
           const int q = (int)items.size();
           items.push_back(make_int2(a, b));
           slots_of[a].push_back(2 * q);
@@ -1026,7 +1070,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
         }
       }
       const size_t vsmem = (size_t)10 * T * 32 * sizeof(double);
-      h->vtx_smem = vsmem <= (size_t)160 * 1024 && T >= 2 ? vsmem : 0;
+      h->vtx_smem = world == 1 && vsmem <= (size_t)160 * 1024 && T >= 2 ? vsmem : 0;
       h->nvtx_rounds = (int)vround.size() - 1;
       if (h->vtx_smem) {
         if ((rc = upload(h, &h->d_vtx_items, vitems)) || (rc = upload(h, &h->d_vtx_round_ptr, vround))) return bail(rc);
@@ -1040,10 +1084,17 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
       h->H = H;
       h->nmir_items = (int64_t)items.size();
       h->nmir_slots = slot;
+      for (const int2 &it : items) h->mir_evals += it.x == it.y ? 33 * 32 : 2 * 32 * 32;
       if ((rc = upload(h, &h->d_rU, rU)) || (rc = upload(h, &h->d_zU, zU)) || (rc = upload(h, &h->d_pu, pu)) ||
           (rc = upload(h, &h->d_pm, pm)) || (rc = upload(h, &h->d_mir_items, items)) ||
           (rc = upload(h, &h->d_mtile_ptr, tptr)) || (rc = upload(h, &h->d_mtile_slots, tslots)))
         return bail(rc);
+      if (world > 1) {   // pair split: every rank targets every point, G summed by an all-reduce
+        h->dist_pairs = true;
+        h->Nc = P.npts;
+        h->e0 = 0;
+        h->e1 = P.ncell;
+      }
     }
   }
   {   // band solver maps (NEXT-2)
@@ -1419,6 +1470,8 @@ int landau_set_mirror(landau_t h, int32_t enable) {
   if (enable < 0 || enable > 3) return fail(h, LANDAU_EINVAL, "set_mirror: mode must be 0..3");
   if (enable && !h->mirror) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: the mesh is not mirror-symmetric");
   if (enable == 3 && !h->vtx_smem) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: a vertex does not fit shared memory");
+  if (h->dist_pairs && enable != 1 && enable != 2)
+    return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: the pair split runs the mirror slot kernel");
   if (!h->host_only) drop_graphs(h);
   h->mirror_on = enable != 0;
   h->mirror_mode = enable ? enable : 1;

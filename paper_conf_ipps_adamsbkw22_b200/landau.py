@@ -76,6 +76,7 @@ def lib():
             "landau_point_coeffs": (C.c_int, [vp, vp]),
             "landau_point_coeffs_batched": (C.c_int, [vp, i64, vp]),
             "landau_partition": (C.c_int, [i64, i32, i32, P64, P64]),
+            "landau_pair_partition": (C.c_int, [i64, i32, i32, P64, P64]),
             "landau_nccl_unique_id": (C.c_int, [vp]),
             "landau_set_timing": (C.c_int, [vp, i32]),
             "landau_get_timing": (C.c_int, [vp, Pd, P64]),
@@ -115,6 +116,15 @@ def landau_partition(nelem, world, rank):
     if rc:
         raise LandauError(rc, "landau_partition")
     return e0.value, e1.value
+
+
+def landau_pair_partition(ntiles, world, rank):
+    """Item range [q0, q1) of the pair split (LANDAU_DIST_ELEMENTS on a z-mirror mesh)."""
+    q0, q1 = C.c_int64(), C.c_int64()
+    rc = lib().landau_pair_partition(int(ntiles), int(world), int(rank), C.byref(q0), C.byref(q1))
+    if rc:
+        raise LandauError(rc, "landau_pair_partition")
+    return q0.value, q1.value
 
 
 def landau_nccl_unique_id():

@@ -49,6 +49,25 @@ def test_partition_covers_cells_once(nelem, world):
         L.landau_partition(nelem, world, world)
 
 
+@pytest.mark.parametrize("ntiles,world", [(17, 1), (17, 2), (1700, 8), (5, 3), (2, 8), (0, 2)])
+def test_pair_partition_covers_items_once_balanced(ntiles, world):
+    """Pair split: the ranks' item ranges tile [0, T(T+1)/2) in order, and each rank's weight (2 per
+    tile pair, 1 per diagonal item) is within one pair of T^2 / world."""
+    items = [(a, b) for b in range(ntiles) for a in range(b + 1)]
+    wt = np.array([1 if a == b else 2 for a, b in items], dtype=np.int64)
+    prev = 0
+    for r in range(world):
+        q0, q1 = L.landau_pair_partition(ntiles, world, r)
+        assert q0 == prev and q0 <= q1 <= len(items)
+        prev = q1
+        if len(items) and world <= len(items):
+            assert abs(int(wt[q0:q1].sum()) - ntiles * ntiles / world) <= 2
+    assert prev == len(items)
+    for bad in ((ntiles, world, world), (ntiles, 0, 0), (-1, world, 0)):
+        with pytest.raises(L.LandauError):
+            L.landau_pair_partition(*bad)
+
+
 def _host(prob):
     return L.Landau.from_problem(prob, device=L.LANDAU_HOST_ONLY)
 

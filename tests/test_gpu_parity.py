@@ -756,3 +756,38 @@ print("ok")
     out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600, env=env,
                          cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     assert out.returncode == 0 and out.stdout.strip().endswith("ok"), out.stderr[-3000:]
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_pair_split_partials_sum_to_G(world, monkeypatch):
+    """Pair split (LANDAU_DIST_ELEMENTS on a mirror mesh): each rank runs only its landau_pair_partition
+    share of the slot kernel's items and the ranks' partial G are summed by the all-reduce.  One GPU
+    emulates the ranks (LANDAU_PAIR_SPLIT_EMULATE, read at create): the partials must add up to the
+    full G, which matches the oracle."""
+    prob, h0, o, fg, fo = setup("C3")
+    nb = 64   # enough items for the slot kernel
+    F = torch.tensor(np.stack([fg] * nb), device=DEV)
+
+    def G_of(env):
+        if env:
+            monkeypatch.setenv("LANDAU_PAIR_SPLIT_EMULATE", env)
+        else:
+            monkeypatch.delenv("LANDAU_PAIR_SPLIT_EMULATE", raising=False)
+        h = L.Landau.from_problem(prob, device=0)
+        h.set_mirror("slots")
+        h.set_state_batched(F)
+        G = torch.empty((nb, 5, h.npoints), dtype=torch.float64, device=DEV)
+        h.point_coeffs_batched(G)
+        torch.cuda.synchronize()
+        assert h.stats()["inner_path"] == 3
+        ev = h.stats()["pair_evaluations"]
+        h.close()
+        return G.cpu().numpy(), ev
+
+    Gfull, evfull = G_of(None)
+    parts = [G_of(f"{world}:{r}") for r in range(world)]
+    assert sum(e for _, e in parts) == evfull
+    Gsum = sum(g for g, _ in parts)
+    Go, Ga = o.point_coeffs(fo)
+    assert np.max(np.abs(Gsum[0] - Go) / Ga) <= 1e-12
+    assert np.max(np.abs(Gsum - Gfull) / Ga) <= 1e-13
