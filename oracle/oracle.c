@@ -283,6 +283,58 @@ void oracle_inner(long long n, const double *r, const double *z, const double *w
 }
 
 /* ------------------------------------------------------------------------------------------ */
+/* O12: the inner integral with the 3D Cartesian Landau tensor of Eq. 3    */
+/* (@7593), U(u) = (|u|^2 I - u u^T) / |u|^3, u = v_i - v_j, straight from the definition: no     */
+/* azimuthal integration, no elliptic integrals.  "A full 3D model is supported in the library"   */
+/* (@7997-8072).  Per target i, over sources j with v_j != v_i (Amb-3), in j order (Neumaier):    */
+/*   G_D(i) = sum_j wTD_j U(v_i - v_j)       (xx, xy, xz, yy, yz, zz)                          */
+/*   G_K(i) = sum_j U(v_i - v_j) wTK_j       (x, y, z)                                         */
+/* with wTD = w T_D, wTK = w T_K premultiplied by the caller (Eqs. 7-8 with the 3D tensor).      */
+/* ------------------------------------------------------------------------------------------ */
+void oracle_tensor3d(double ux, double uy, double uz, double out[6]) {
+  const ld u[3] = {ux, uy, uz};
+  const ld s2 = u[0] * u[0] + u[1] * u[1] + u[2] * u[2];
+  const ld s3 = s2 * sqrtl(s2);
+  int k = 0;
+  for (int a = 0; a < 3; a++)
+    for (int b = a; b < 3; b++) out[k++] = (double)(((a == b ? s2 : 0.0L) - u[a] * u[b]) / s3);
+}
+
+void oracle_inner3d(long long n, const double *x, const double *y, const double *z, const double *wTD,
+                    const double *wTKx, const double *wTKy, const double *wTKz, double *G, double *Gabs) {
+#pragma omp parallel for schedule(dynamic, 16)
+  for (long long i = 0; i < n; i++) {
+    nsum_t acc[9], aac[9];
+    memset(acc, 0, sizeof acc);
+    memset(aac, 0, sizeof aac);
+    for (long long j = 0; j < n; j++) {
+      if (x[j] == x[i] && y[j] == y[i] && z[j] == z[i]) continue;
+      const ld u[3] = {(ld)x[i] - x[j], (ld)y[i] - y[j], (ld)z[i] - z[j]};
+      const ld s2 = u[0] * u[0] + u[1] * u[1] + u[2] * u[2];
+      const ld s3 = s2 * sqrtl(s2);
+      ld U[3][3];
+      for (int a = 0; a < 3; a++)
+        for (int b = 0; b < 3; b++) U[a][b] = ((a == b ? s2 : 0.0L) - u[a] * u[b]) / s3;
+      const ld wd = wTD[j], wk[3] = {wTKx[j], wTKy[j], wTKz[j]};
+      int k = 0;
+      for (int a = 0; a < 3; a++)
+        for (int b = a; b < 3; b++, k++) {
+          nadd(&acc[k], wd * U[a][b]);
+          nadd(&aac[k], fabsl(wd * U[a][b]));
+        }
+      for (int a = 0; a < 3; a++) {
+        nadd(&acc[6 + a], U[a][0] * wk[0] + U[a][1] * wk[1] + U[a][2] * wk[2]);
+        nadd(&aac[6 + a], fabsl(U[a][0] * wk[0]) + fabsl(U[a][1] * wk[1]) + fabsl(U[a][2] * wk[2]));
+      }
+    }
+    for (int c = 0; c < 9; c++) {
+      if (G) G[c * n + i] = (double)nval(&acc[c]);
+      if (Gabs) Gabs[c * n + i] = (double)nval(&aac[c]);
+    }
+  }
+}
+
+/* ------------------------------------------------------------------------------------------ */
 /* O1: FE space on the quadtree                                                                */
 /* ------------------------------------------------------------------------------------------ */
 static int pos_cmp(const void *a, const void *b) {

@@ -21,7 +21,8 @@
  *   O9  mass matrix shift * sum_e P_e^T (sum_q w phi phi) P_e (@39757-39999)
  *   O10 condition scale: the same assembly with every product replaced by its absolute value.
  *   O11 E_z advection matrix sum_e P_e^T (sum_q w phi_k d_z phi_l) P_e (Eq. 4, @8216-8654)
- * Pins: see tests/test_oracle_*.py (P1-P9 of SURVEY.md §8(c)).
+ *   O12 the inner integral with the 3D Cartesian tensor of Eq. 3 (@7997-8072)
+ * Pins: see tests/test_oracle_*.py (P1-P9 of SURVEY.md §8(c); P13 for O12).
  */
 #ifndef LANDAU_ORACLE_H
 #define LANDAU_ORACLE_H
@@ -52,6 +53,13 @@ void oracle_points(const oracle_t *o, double *r, double *z, double *w);
 void oracle_pattern(const oracle_t *o, long long *rowptr, int *col);
 /* COO pattern: per species, per cell, the cell's sorted distinct DOFs x same, row-major */
 void oracle_coo_pattern(const oracle_t *o, int *row, int *col);
+
+/* O12: U(u) of Eq. 3 in 3D Cartesian velocity space, (xx, xy, xz, yy, yz, zz). */
+void oracle_tensor3d(double ux, double uy, double uz, double out[6]);
+/* O12: G = [9][n] = (G_D xx, xy, xz, yy, yz, zz, G_K x, y, z) at every point (wTD = w T_D and
+ * wTK = w T_K premultiplied), coincident points excluded; Gabs: the sums of absolute values. */
+void oracle_inner3d(long long n, const double *x, const double *y, const double *z, const double *wTD,
+                    const double *wTKx, const double *wTKy, const double *wTKz, double *G, double *Gabs);
 
 /* U^D_rr, U^D_rz, U^D_zz, U^K_rr, U^K_zr at target (r, z), source (rb, zb). */
 void oracle_tensor(double r, double z, double rb, double zb, double out[5]);

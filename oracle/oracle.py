@@ -58,6 +58,8 @@ def lib():
         L.oracle_mass_coo.argtypes = [vp, C.c_double, _d]
         L.oracle_advection.argtypes = [vp, _d]
         L.oracle_advection_coo.argtypes = [vp, _d]
+        L.oracle_tensor3d.argtypes = [C.c_double, C.c_double, C.c_double, _d]
+        L.oracle_inner3d.argtypes = [C.c_longlong, _d, _d, _d, _d, _d, _d, _d, _d, _d]
         L.oracle_set_threads.argtypes = [C.c_int]
         L.oracle_get_threads.restype = C.c_int
         _LIB = L
@@ -72,6 +74,24 @@ def tensor(r, z, rb, zb):
     out = np.zeros(5)
     lib().oracle_tensor(float(r), float(z), float(rb), float(zb), out)
     return out
+
+
+def tensor3d(u):
+    """O12: the 3D Cartesian Landau tensor U(u) of Eq. 3 as (xx, xy, xz, yy, yz, zz)."""
+    out = np.zeros(6)
+    lib().oracle_tensor3d(float(u[0]), float(u[1]), float(u[2]), out)
+    return out
+
+
+def inner3d(x, y, z, wTD, wTK):
+    """O12: (G [9][n], Gabs [9][n]) of the 3D Cartesian inner integral (wTK: [3][n])."""
+    x, y, z, wTD = (np.ascontiguousarray(a, dtype=np.float64) for a in (x, y, z, wTD))
+    wTK = np.ascontiguousarray(wTK, dtype=np.float64)
+    n = x.size
+    G = np.zeros(9 * n)
+    Ga = np.zeros(9 * n)
+    lib().oracle_inner3d(n, x, y, z, wTD, wTK[0].copy(), wTK[1].copy(), wTK[2].copy(), G, Ga)
+    return G.reshape(9, n), Ga.reshape(9, n)
 
 
 def inner(r, z, w, TD, TKr, TKz, targets=None, with_abs=False):
