@@ -239,6 +239,20 @@ int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double E
  * enable outside 0..3 is EINVAL. */
 int landau_set_mirror(landau_t h, int32_t enable);
 
+/* NEXT-4: the inner integral with the 3D Cartesian Landau tensor of Eq. 3
+ * (PAPER.md:1@7593, "a full 3D model is supported in the library" @7997-8072), without azimuthal
+ * reduction or elliptic integrals: for every point i of a 3D velocity-space point set,
+ *   G_D(i) = sum_{j: v_j != v_i} wTD_j U(v_i - v_j),   G_K(i) = sum_j U(v_i - v_j) wTK_j,
+ *   U(u) = (|u|^2 I - u u^T) / |u|^3.
+ * xyz_dev: [3][n] point coordinates (x, y, z rows); wTD_dev: [n] w T_D; wTK_dev: [3][n] w T_K
+ * (quadrature weights premultiplied, as in step a-1); G_dev: [9][n] output (G_D xx, xy, xz, yy, yz,
+ * zz, G_K x, y, z).  All device pointers owned by the caller, on the current CUDA device; enqueued on
+ * cuda_stream (temporary split-j partials come from the stream-ordered allocator).  Coincident
+ * points contribute nothing.  EINVAL: n < 0 or a NULL pointer with n > 0; ENOMEM: partials;
+ * ECUDA: launch failure.  Element matrices and assembly of a 3D model are not part of this call. */
+int landau3d_inner(int64_t n, const double *xyz_dev, const double *wTD_dev, const double *wTK_dev, double *G_dev,
+                   void *cuda_stream);
+
 /* How the last build ran (for FLOP accounting and diagnostics). */
 typedef struct {
   int32_t inner_path;        /* 0: directed pair kernel (every ordered pair, split-j when small);

@@ -28,6 +28,7 @@ using namespace landau;
 #include "kernels_fe.cuh"
 #include "kernels_inner.cuh"
 #include "kernels_band.cuh"
+#include "kernels_3d.cuh"
 
 
 // ==================================================================================================
@@ -819,6 +820,36 @@ int landau_partition(int64_t nelem, int32_t world, int32_t rank, int64_t *e0, in
   *e0 = std::min<int64_t>(nelem, (int64_t)rank * chunk);
   *e1 = std::min<int64_t>(nelem, (int64_t)(rank + 1) * chunk);
   return LANDAU_OK;
+}
+
+int landau3d_inner(int64_t n, const double *xyz_dev, const double *wTD_dev, const double *wTK_dev, double *G_dev,
+                   void *cuda_stream) {
+  if (n < 0 || (n > 0 && (!xyz_dev || !wTD_dev || !wTK_dev || !G_dev))) return LANDAU_EINVAL;
+  if (n == 0) return LANDAU_OK;
+  cudaStream_t st = (cudaStream_t)cuda_stream;
+  int dev = 0, sms = 148;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+    return LANDAU_ECUDA;
+  constexpr int TPT = 2;
+  const int64_t wtiles = (n + 32 * TPT - 1) / (32 * TPT);
+  int64_t nsplit = std::max<int64_t>(1, (12LL * sms + wtiles - 1) / wtiles);   // >= 12 warps per SM
+  nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, n / 32));
+  const int64_t split_len = (n + nsplit - 1) / nsplit;
+  nsplit = (n + split_len - 1) / split_len;
+  double *part = G_dev;
+  if (nsplit > 1 && cudaMallocAsync((void **)&part, sizeof(double) * nsplit * 9 * n, st) != cudaSuccess) return LANDAU_ENOMEM;
+  const int64_t nitems = nsplit * wtiles;
+  inner3d_kernel<TPT><<<(unsigned)((nitems + k3dWarps - 1) / k3dWarps), 32 * k3dWarps, 0, st>>>(
+      n, split_len, (int)nsplit, wtiles, nitems, xyz_dev, wTD_dev, wTK_dev, part);
+  cudaError_t e = cudaGetLastError();
+  if (nsplit > 1) {
+    if (e == cudaSuccess) {
+      reduce3d_kernel<<<(unsigned)std::min<int64_t>((9 * n + 255) / 256, 16LL * sms), 256, 0, st>>>(n, (int)nsplit, part, G_dev);
+      e = cudaGetLastError();
+    }
+    cudaFreeAsync(part, st);
+  }
+  return e == cudaSuccess ? LANDAU_OK : LANDAU_ECUDA;
 }
 
 int landau_pair_partition(int64_t ntiles, int32_t world, int32_t rank, int64_t *q0, int64_t *q1) {

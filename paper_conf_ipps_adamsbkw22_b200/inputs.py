@@ -264,3 +264,44 @@ def config5() -> Problem:
 
 
 CONFIGS = {"C1": config1, "C2": config2, "C3": config3, "C5": config5}
+
+
+# ------------------------------------------------------------------------------------------------
+# NEXT-4 (3D Cartesian variant): a point set and synthetic fields for the 3D inner integral
+# ------------------------------------------------------------------------------------------------
+def points3d(ncell: int = 4, order: int = 3, R: float = R_E):
+    """Tensor-product Gauss-Legendre points ((order+1)^3 per cube) of a uniform ncell^3 grid of cubes on
+    [-R, R]^3: xyz [3][n] and the quadrature weights w [n] (cube-major, then z, y, x)."""
+    q = order + 1
+    g, gw = np.polynomial.legendre.leggauss(q)
+    h = 2.0 * R / ncell
+    c0 = -R + h * np.arange(ncell)
+    X, Y, Z, W = [], [], [], []
+    for cz in c0:
+        for cy in c0:
+            for cx in c0:
+                for a in range(q):
+                    for b in range(q):
+                        for c in range(q):
+                            X.append(cx + 0.5 * h * (g[c] + 1.0))
+                            Y.append(cy + 0.5 * h * (g[b] + 1.0))
+                            Z.append(cz + 0.5 * h * (g[a] + 1.0))
+                            W.append(gw[a] * gw[b] * gw[c] * (0.5 * h) ** 3)
+    return np.array([X, Y, Z]), np.array(W)
+
+
+def fields3d(xyz, w, seed: int = 20222):
+    """Synthetic w T_D [n] and w T_K [3][n] with the shape of the thermal-quench case (a cold bulk
+    plus a drifting hot tail, electrons): a Maxwellian mix g(v) and its gradient, times the weights,
+    times (1 + 0.01 xi) with xi ~ U(-1, 1) from a seeded generator."""
+    x, y, z = xyz
+    rng = np.random.default_rng(seed)
+    g = np.zeros_like(x)
+    grad = np.zeros_like(xyz)
+    for n, T, u in ((5.0, 0.1, 0.0), (1.0, 1.0, 0.5 * VTH_E)):
+        th = theta(T, 1.0)
+        f = n * (math.pi * th) ** -1.5 * np.exp(-(x ** 2 + y ** 2 + (z - u) ** 2) / th)
+        g += f
+        grad += np.array([-2.0 * x / th * f, -2.0 * y / th * f, -2.0 * (z - u) / th * f])
+    xi = 1.0 + 0.01 * rng.uniform(-1.0, 1.0, size=x.size)
+    return w * g * xi, w * grad * xi

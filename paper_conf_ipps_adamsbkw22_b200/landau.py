@@ -77,6 +77,7 @@ def lib():
             "landau_point_coeffs_batched": (C.c_int, [vp, i64, vp]),
             "landau_partition": (C.c_int, [i64, i32, i32, P64, P64]),
             "landau_pair_partition": (C.c_int, [i64, i32, i32, P64, P64]),
+            "landau3d_inner": (C.c_int, [i64, vp, vp, vp, vp, vp]),
             "landau_nccl_unique_id": (C.c_int, [vp]),
             "landau_set_timing": (C.c_int, [vp, i32]),
             "landau_get_timing": (C.c_int, [vp, Pd, P64]),
@@ -125,6 +126,20 @@ def landau_pair_partition(ntiles, world, rank):
     if rc:
         raise LandauError(rc, "landau_pair_partition")
     return q0.value, q1.value
+
+
+def landau3d_inner(xyz, wTD, wTK, G, stream=None):
+    """NEXT-4: 3D Cartesian inner integral on device tensors xyz [3][n], wTD [n], wTK [3][n] -> G [9][n]
+    (float64, contiguous, on the current CUDA device)."""
+    import torch
+    n = int(wTD.numel())
+    for t, shape in ((xyz, (3, n)), (wTK, (3, n)), (G, (9, n))):
+        if tuple(t.shape) != shape or t.dtype != torch.float64 or not t.is_cuda or not t.is_contiguous():
+            raise ValueError(f"landau3d_inner: expected a contiguous float64 CUDA tensor of shape {shape}")
+    st = (stream or torch.cuda.current_stream()).cuda_stream
+    rc = lib().landau3d_inner(n, xyz.data_ptr(), wTD.data_ptr(), wTK.data_ptr(), G.data_ptr(), st)
+    if rc:
+        raise LandauError(rc, "landau3d_inner")
 
 
 def landau_nccl_unique_id():

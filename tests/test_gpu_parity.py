@@ -791,3 +791,27 @@ def test_pair_split_partials_sum_to_G(world, monkeypatch):
     Go, Ga = o.point_coeffs(fo)
     assert np.max(np.abs(Gsum[0] - Go) / Ga) <= 1e-12
     assert np.max(np.abs(Gsum - Gfull) / Ga) <= 1e-13
+
+
+@pytest.mark.parametrize("ncell,order,sub", [(3, 3, None), (2, 2, 173), (1, 2, 1)])
+def test_inner3d_matches_oracle(ncell, order, sub):
+    """NEXT-4: the 3D Cartesian inner integral (Eq. 3 directly) against oracle O12 on every point:
+    several target tiles and source splits, a ragged size (173 points), a single point, and a twin
+    point (coincident pairs excluded)."""
+    from oracle import oracle as O
+    xyz, w = inputs.points3d(ncell, order)
+    wTD, wTK = inputs.fields3d(xyz, w)
+    if sub is not None:
+        xyz, wTD, wTK = xyz[:, :sub].copy(), wTD[:sub].copy(), wTK[:, :sub].copy()
+    if xyz.shape[1] > 4:   # a twin of point 3 (distinct index, identical coordinates)
+        xyz = np.concatenate([xyz, xyz[:, 3:4]], axis=1)
+        wTD = np.concatenate([wTD, wTD[3:4]])
+        wTK = np.concatenate([wTK, wTK[:, 3:4]], axis=1)
+    n = xyz.shape[1]
+    G = torch.full((9, n), float("nan"), dtype=torch.float64, device=DEV)
+    L.landau3d_inner(torch.tensor(xyz, device=DEV), torch.tensor(wTD, device=DEV), torch.tensor(wTK, device=DEV), G)
+    torch.cuda.synchronize()
+    Go, Ga = O.inner3d(xyz[0], xyz[1], xyz[2], wTD, wTK)
+    Gg = G.cpu().numpy()
+    assert np.all(np.isfinite(Gg))
+    assert np.max(np.abs(Gg - Go) / np.maximum(Ga, 1e-300)) <= 1e-13
