@@ -158,6 +158,7 @@ FLOP_PER_PAIR_SYMMETRIC = 193.0
 # evaluation, (N/2)^2 evaluations per batch item (profiles/r01_flops_mirror.csv)
 FLOP_PER_EVAL_MIRROR = 198.7   # inner_mir_kernel (slot kernel; profiles/r01_flops_mirror.csv)
 FLOP_PER_EVAL_VTX = 199.0      # inner_vtx_kernel (per-vertex kernel; profiles/r01_flops_vtx.csv)
+FLOP_PER_PAIR_3D = 58.0        # inner3d_kernel, per ordered pair (profiles/r01_flops_3d.csv)
 FLOP_PER_EVAL_MDIR = 187.4     # inner_mdir_kernel (mirror directed, per padded U or V evaluation; profiles/r01_flops_mdir.csv)
 
 
@@ -446,6 +447,32 @@ def main():
                         "(the batch shares one mesh): no state carried across builds"}}
         except Exception as e:   # the variant is optional: report why it did not run
             line["variants"] = {"tensor_cache_gemm": {"unavailable": str(e)[:200]}}
+        # NEXT-4, the other variant: the inner integral with the 3D Cartesian tensor of Eq. 3
+        # (landau3d_inner) on a 3D point set of the thermal-quench shape, 8^3 Q3 cubes (N = 32768)
+        try:
+            xyz3, w3 = inputs.points3d(8, 3)
+            wTD3, wTK3 = inputs.fields3d(xyz3, w3)
+            n3 = int(w3.size)
+            X3, D3, K3 = (torch.tensor(a, device="cuda") for a in (xyz3, wTD3, wTK3))
+            G3 = torch.empty((9, n3), dtype=torch.float64, device="cuda")
+            for _ in range(2):
+                L.landau3d_inner(X3, D3, K3, G3, stream)
+            ev3 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+            for k in range(args.steps):
+                ev3[k][0].record(stream)
+                L.landau3d_inner(X3, D3, K3, G3, stream)
+                ev3[k][1].record(stream)
+            torch.cuda.synchronize()
+            ms3 = sum(a.elapsed_time(b) for a, b in ev3) / args.steps
+            line.setdefault("variants", {})["inner3d_cartesian"] = {
+                "value": n3 * n3 / (ms3 * 1e-3), "unit": "pairs/s",
+                "points": n3, "ms_per_launch": ms3,
+                "tflops": FLOP_PER_PAIR_3D * n3 * n3 / (ms3 * 1e-3) / 1e12,
+                "frac_of_fp64_peak": FLOP_PER_PAIR_3D * n3 * n3 / (ms3 * 1e-3) / 1e12 / peak,
+                "note": "SURVEY NEXT-4: G_D, G_K with U = (|u|^2 I - u u^T)/|u|^3 directly (no elliptic integrals), "
+                        "ordered pairs, parity-tested against oracle O12"}
+        except Exception as e:
+            line.setdefault("variants", {})["inner3d_cartesian"] = {"unavailable": str(e)[:200]}
     # NEXT-3: quasi-Newton backward-Euler iterations on the same batch (the paper's figure of merit,
     # "Newton iterations per second", @37187): per iteration set_state + Jacobian + band LU + solve
     if args.workload == "C4" and not args.tensor_cache and nloc:
