@@ -150,16 +150,16 @@ def load_profile_traffic(workload):
 # FP64 FLOP (2*DFMA + DMUL + DADD) per pair evaluation, counted once from ncu
 # sm__sass_thread_inst_executed_op_{dfma,dmul,dadd}_pred_on of each inner kernel on the C4 workload
 # (profiles/r01_inner_ncu.txt):
-#   directed kernel:  177 FLOP per ordered (target, source) pair, N^2 per batch item
-#   symmetric kernel: 193 FLOP per unordered pair, N (N - 1) / 2 per batch item (both targets updated)
-FLOP_PER_PAIR_DIRECTED = 177.0
-FLOP_PER_PAIR_SYMMETRIC = 193.0
+#   directed kernel:  173 FLOP per ordered (target, source) pair, N^2 per batch item
+#   symmetric kernel: 189 FLOP per unordered pair, N (N - 1) / 2 per batch item (both targets updated)
+FLOP_PER_PAIR_DIRECTED = 173.0
+FLOP_PER_PAIR_SYMMETRIC = 189.2
 # mirror-symmetric kernel: FP64 FLOP (2 DFMA + DMUL + DADD, ncu SASS counts on C4) per tensor
 # evaluation, (N/2)^2 evaluations per batch item (profiles/r01_flops_mirror.csv)
-FLOP_PER_EVAL_MIRROR = 198.7   # inner_mir_kernel (slot kernel; profiles/r01_flops_mirror.csv)
-FLOP_PER_EVAL_VTX = 199.0      # inner_vtx_kernel (per-vertex kernel; profiles/r01_flops_vtx.csv)
+FLOP_PER_EVAL_MIRROR = 194.7   # inner_mir_kernel (slot kernel; profiles/r01_flops_mirror.csv)
+FLOP_PER_EVAL_VTX = 195.0      # inner_vtx_kernel (per-vertex kernel; profiles/r01_flops_vtx.csv)
 FLOP_PER_PAIR_3D = 58.0        # inner3d_kernel, per ordered pair (profiles/r01_flops_3d.csv)
-FLOP_PER_EVAL_MDIR = 187.4     # inner_mdir_kernel (mirror directed, per padded U or V evaluation; profiles/r01_flops_mdir.csv)
+FLOP_PER_EVAL_MDIR = 183.2     # inner_mdir_kernel (mirror directed, per padded U or V evaluation; profiles/r01_flops_mdir.csv)
 
 
 def cpu_baseline(args, desc, nsample):
