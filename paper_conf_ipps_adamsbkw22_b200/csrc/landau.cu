@@ -685,10 +685,19 @@ int launch_assemble(landau_t h, int64_t nbatch, double *out, int format) {   // 
       gd.fK[q] = h->spc.fK[sp];
     }
     if (h->spc.grid_nsp[g] == 0 || m.nslots == 0) continue;
-    constexpr int BPT = 8;
-    dim3 grid((unsigned)((m.nslots + 127) / 128), (unsigned)((nbatch + BPT - 1) / BPT));
-    assemble_kernel<NB, BPT><<<grid, 128, 0, h->stream>>>(gd, h->d_C, P.ncell * 2 * NB * NB, out, out_bstride,
-                                                          (int)nbatch);
+    static const int bpt = [] {   // batch items per thread (LANDAU_ASM_BPT 1/2/4/8/16; C4: 4 0.191 ms, 8 0.201, 2 0.208, 16 0.453)
+      const char *e = getenv("LANDAU_ASM_BPT");
+      return e ? atoi(e) : 4;
+    }();
+#define LAUNCH_ASM(BPT)                                                                                          \
+  assemble_kernel<NB, BPT><<<dim3((unsigned)((m.nslots + 127) / 128), (unsigned)((nbatch + BPT - 1) / BPT)), 128, 0, \
+                             h->stream>>>(gd, h->d_C, P.ncell * 2 * NB * NB, out, out_bstride, (int)nbatch)
+    if (bpt == 4) LAUNCH_ASM(4);
+    else if (bpt == 2) LAUNCH_ASM(2);
+    else if (bpt == 1) LAUNCH_ASM(1);
+    else if (bpt == 16) LAUNCH_ASM(16);
+    else LAUNCH_ASM(8);
+#undef LAUNCH_ASM
     h->launches++;
     h->tlaunch[LANDAU_T_ASSEMBLE]++;
     KCHECK();
