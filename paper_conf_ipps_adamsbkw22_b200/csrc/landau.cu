@@ -839,7 +839,11 @@ int landau3d_inner(int64_t n, const double *xyz_dev, const double *wTD_dev, cons
   int dev = 0, sms = 148;
   if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
     return LANDAU_ECUDA;
-  constexpr int TPT = 2;
+  static const int tpt = [] {   // targets per lane (LANDAU_3D_TPT: 1, 2 or 4)
+    const char *e = getenv("LANDAU_3D_TPT");
+    return e ? atoi(e) : 2;
+  }();
+  const int TPT = tpt == 1 || tpt == 4 ? tpt : 2;
   const int64_t wtiles = (n + 32 * TPT - 1) / (32 * TPT);
   int64_t nsplit = std::max<int64_t>(1, (12LL * sms + wtiles - 1) / wtiles);   // >= 12 warps per SM
   nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, n / 32));
@@ -848,8 +852,13 @@ int landau3d_inner(int64_t n, const double *xyz_dev, const double *wTD_dev, cons
   double *part = G_dev;
   if (nsplit > 1 && cudaMallocAsync((void **)&part, sizeof(double) * nsplit * 9 * n, st) != cudaSuccess) return LANDAU_ENOMEM;
   const int64_t nitems = nsplit * wtiles;
-  inner3d_kernel<TPT><<<(unsigned)((nitems + k3dWarps - 1) / k3dWarps), 32 * k3dWarps, 0, st>>>(
-      n, split_len, (int)nsplit, wtiles, nitems, xyz_dev, wTD_dev, wTK_dev, part);
+  const unsigned grid3 = (unsigned)((nitems + k3dWarps - 1) / k3dWarps);
+  if (TPT == 1)
+    inner3d_kernel<1><<<grid3, 32 * k3dWarps, 0, st>>>(n, split_len, (int)nsplit, wtiles, nitems, xyz_dev, wTD_dev, wTK_dev, part);
+  else if (TPT == 4)
+    inner3d_kernel<4><<<grid3, 32 * k3dWarps, 0, st>>>(n, split_len, (int)nsplit, wtiles, nitems, xyz_dev, wTD_dev, wTK_dev, part);
+  else
+    inner3d_kernel<2><<<grid3, 32 * k3dWarps, 0, st>>>(n, split_len, (int)nsplit, wtiles, nitems, xyz_dev, wTD_dev, wTK_dev, part);
   cudaError_t e = cudaGetLastError();
   if (nsplit > 1) {
     if (e == cudaSuccess) {
