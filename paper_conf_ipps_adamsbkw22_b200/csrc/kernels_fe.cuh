@@ -183,7 +183,10 @@ __global__ void __launch_bounds__(NB * EPB, LANDAU_EL_MINB) element_kernel(int64
 // same pair plays (b, d) in step 1 and (a, c) in step 2); the 32 / S^2 lane groups split qr (step 1)
 // and (b, d) (step 2).
 // ------------------------------------------------------------------------------------------------
-constexpr int kSfWarps = 4;
+#ifndef LANDAU_SF_WARPS
+#define LANDAU_SF_WARPS 4
+#endif
+constexpr int kSfWarps = LANDAU_SF_WARPS;
 
 template <int S>
 __global__ void __launch_bounds__(32 * kSfWarps) element_sf_kernel(int64_t ncell, const double *__restrict__ G,

@@ -650,7 +650,11 @@ int launch_element(landau_t h, int64_t nbatch, int64_t b0, int64_t nb) {
   }();
   if (sf && P.ncell * nb < (1LL << 32)) {   // sum factorisation, one warp per cell
     const int64_t items = P.ncell * nb;
-    const unsigned grid = (unsigned)std::min<int64_t>((items + kSfWarps - 1) / kSfWarps, 16LL * num_sms(h));
+    static const int64_t sf_bps = [] {   // grid cap in blocks per SM (LANDAU_SF_BLOCKS_PER_SM)
+      const char *e = getenv("LANDAU_SF_BLOCKS_PER_SM");
+      return e ? (int64_t)atoll(e) : (int64_t)64;   // C4: 64 0.113 ms, 16 0.118 ms
+    }();
+    const unsigned grid = (unsigned)std::min<int64_t>((items + kSfWarps - 1) / kSfWarps, sf_bps * num_sms(h));
     element_sf_kernel<S><<<grid, 32 * kSfWarps, 0, h->stream>>>(P.ncell, h->d_G, h->Nc, (int)nbatch, (int)b0, (int)nb,
                                                                h->d_w, h->d_h, h->d_tab + 3 * NB * NB, h->d_C);
   } else {
