@@ -815,3 +815,28 @@ def test_inner3d_matches_oracle(ncell, order, sub):
     Gg = G.cpu().numpy()
     assert np.all(np.isfinite(Gg))
     assert np.max(np.abs(Gg - Go) / np.maximum(Ga, 1e-300)) <= 1e-13
+
+
+def test_bench_gpu_arm_json_line():
+    """The driver's contract for the GPU arm: one JSON line with the base keys, roofline, cpu_baseline,
+    e2e, clocks and a non-zero launch count of this library's kernels."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--steps", "3", "--warmup", "3"],
+                         capture_output=True, text=True, timeout=900, cwd=root)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "roofline", "cpu_baseline", "e2e", "clocks", "gpu_launches"):
+        assert k in d, k
+    assert d["value"] > 0 and d["steps"] == 3 and d["warmup"] == 3 and d["scaling"] == "weak"
+    r = d["roofline"]
+    assert r["bound"] == "alu" and 0 < r["frac"] < 1 and r["peak"] > 30
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0 and d["e2e"]["value"] > 0
+    assert d["gpu_launches"] > 0 and d["config"]["workload"].startswith("C4")
