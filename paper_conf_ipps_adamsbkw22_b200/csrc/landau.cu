@@ -1104,23 +1104,31 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
         tptr.push_back((int32_t)tslots.size());
       }
       // per-vertex kernel schedule: round-robin tournament of the T tiles (circle method; rounds of
-      // disjoint tile pairs), then the diagonal items in rounds of kVtxWarps
+      // disjoint tile pairs), then the diagonal items in rounds of kVtxWarps.  For odd T every round
+      // leaves one tile out (the bye); when the CTA has a warp to spare for it ((T + 1)/2 <=
+      // kVtxWarps), the bye tile's diagonal item joins that round (last, for the spare warp) and no
+      // diagonal rounds remain.
       std::vector<VtxItem> vitems;
       std::vector<int32_t> vround(1, 0);
       {
         const int Tp = T + (T & 1);
+        const bool bye_diag = (T & 1) && (T + 1) / 2 <= kVtxWarps;
         for (int rd = 0; rd + 1 < Tp; rd++) {
+          int bye = -1;
           for (int q = 0; q < Tp / 2; q++) {
             const int x = q == 0 ? Tp - 1 : (rd + q) % (Tp - 1);
             const int y = q == 0 ? rd : (rd - q + Tp - 1) % (Tp - 1);
             if (x < T && y < T) vitems.push_back({std::min(x, y), std::max(x, y)});
+            else bye = x < T ? x : y;
           }
+          if (bye_diag && bye >= 0) vitems.push_back({bye, bye});
           if ((int)vitems.size() > vround.back()) vround.push_back((int32_t)vitems.size());
         }
-        for (int t = 0; t < T; t++) {
-          vitems.push_back({t, t});
-          if ((t + 1) % kVtxWarps == 0 || t + 1 == T) vround.push_back((int32_t)vitems.size());
-        }
+        if (!bye_diag)
+          for (int t = 0; t < T; t++) {
+            vitems.push_back({t, t});
+            if ((t + 1) % kVtxWarps == 0 || t + 1 == T) vround.push_back((int32_t)vitems.size());
+          }
       }
       const size_t vsmem = (size_t)10 * T * 32 * sizeof(double);
       h->vtx_smem = world == 1 && vsmem <= (size_t)160 * 1024 && T >= 2 ? vsmem : 0;

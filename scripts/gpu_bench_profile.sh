@@ -13,3 +13,4 @@ M=sm__sass_thread_inst_executed_op_dfma_pred_on.sum,sm__sass_thread_inst_execute
 ncu --set full --metrics $M --clock-control none --import-source on -k regex:inner_vtx_kernel -s 1 -c 1 -o gpurun_out/inner_full python bench.py --steps 1 --warmup 1 --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"element_sf_kernel|assemble_kernel|field_kernel" -s 3 -c 3 -o gpurun_out/others_full python bench.py --steps 1 --warmup 1 --no-cpu-baseline > gpurun_out/ncu_others.log 2>&1
 tail -2 gpurun_out/ncu_full.log
+ncu --set full --clock-control none --import-source on -k regex:band_lu -s 2 -c 1 -o gpurun_out/band_full python scripts/band_timing.py 1024 > gpurun_out/band_ncu.log 2>&1
