@@ -1,5 +1,6 @@
 # small workloads for compute-sanitizer: every kernel of the library on C1, C3 and a 16-vertex C4 batch
-# (symmetric, mirror-slot and per-vertex inner kernels; band LU, solve and the implicit step)
+# (symmetric, mirror-slot, per-vertex and mirror-directed inner kernels; band LU, solve and the implicit
+# step; the 3D Cartesian inner integral; one emulated rank of the pair split)
 import os, sys
 sys.path.insert(0, os.getcwd())
 import numpy as np, torch
@@ -41,3 +42,19 @@ fn = torch.empty_like(F)
 h.implicit_step_batched(0.002, F, fn, Ez=0.1, max_iter=2)
 torch.cuda.synchronize()
 print("ok")
+# NEXT-4: the 3D Cartesian inner integral (split-j and direct)
+xyz3, w3 = inputs.points3d(2, 2)
+wTD3, wTK3 = inputs.fields3d(xyz3, w3)
+G3 = torch.empty((9, w3.size), dtype=torch.float64, device="cuda")
+L.landau3d_inner(torch.tensor(xyz3, device="cuda"), torch.tensor(wTD3, device="cuda"), torch.tensor(wTK3, device="cuda"), G3)
+# pair split (one emulated rank of two) on C3 through the slot kernel
+os.environ["LANDAU_PAIR_SPLIT_EMULATE"] = "2:1"
+p3 = inputs.CONFIGS["C3"]()
+h3 = L.Landau.from_problem(p3, device=0)
+h3.set_mirror("slots")
+f3 = torch.tensor(np.stack([inputs.coefficients(p3, h3.all_nodes())] * 4), device="cuda")
+h3.set_state_batched(f3)
+Gp = torch.empty((4, 5, h3.npoints), dtype=torch.float64, device="cuda")
+h3.point_coeffs_batched(Gp)
+torch.cuda.synchronize()
+print("ok 3d + pair split")
