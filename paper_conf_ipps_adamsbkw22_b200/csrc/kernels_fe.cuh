@@ -52,21 +52,42 @@ __global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbat
   }
   const SpeciesConst &c_sp = sp_;
   const int el = threadIdx.x / NB, a = threadIdx.x % NB;
+  // a block keeps one chunk of EPB cells and walks the batch items b = g, g + G, ... (blockIdx.x =
+  // g * nchunks + chunk), so the cell's extraction entries, grid, size and weights are loaded once
+  constexpr int kExt = 8;   // extraction entries cached in registers per node (more: read from memory)
   const int64_t nchunks = (ncell + EPB - 1) / EPB;
-  for (int64_t it = blockIdx.x; it < nchunks * nbatch; it += gridDim.x) {
-    const int b = (int)(it / nchunks);
-    const int64_t e = (it % nchunks) * EPB + el;
-    const double *fb = f + (int64_t)b * ndof_total;
+  const int64_t chunk = blockIdx.x % nchunks, G = gridDim.x / nchunks;
+  const int64_t e = chunk * EPB + el;
+  const bool live = e < ncell && (int64_t)blockIdx.x < G * nchunks;
+  int g = 0, nk = 0;
+  int32_t k0 = 0;
+  int32_t xd[kExt];
+  double xw[kExt], w = 0.0, ws = 0.0;
+  if (live) {
+    g = cell_grid[e];
+    k0 = ext_ptr[e * NB + a];
+    nk = ext_ptr[e * NB + a + 1] - k0;
+#pragma unroll
+    for (int k = 0; k < kExt; k++) {
+      xd[k] = k < nk ? ext_dof[k0 + k] : 0;
+      xw[k] = k < nk ? ext_w[k0 + k] : 0.0;
+    }
+    w = pw[e * NB + a];
+    ws = w * (2.0 / cell_h[e]);
+  }
+  for (int64_t b = blockIdx.x / nchunks; b < nbatch; b += G) {
+    const double *fb = f + b * ndof_total;
     __syncthreads();
-    if (e < ncell) {
-      const int g = cell_grid[e];
-      const int32_t k0 = ext_ptr[e * NB + a], k1 = ext_ptr[e * NB + a + 1];
+    if (live) {
       double sD = 0.0, sK = 0.0;
       for (int s = 0; s < c_sp.grid_nsp[g]; s++) {
         const int sp = c_sp.grid_sp[g][s];
         const double *fs = fb + c_sp.soff[sp];
         double v = 0.0;
-        for (int32_t k = k0; k < k1; k++) v = fma(ext_w[k], __ldg(fs + ext_dof[k]), v);
+#pragma unroll
+        for (int k = 0; k < kExt; k++)
+          if (k < nk) v = fma(xw[k], __ldg(fs + xd[k]), v);
+        for (int k = kExt; k < nk; k++) v = fma(ext_w[k0 + k], __ldg(fs + ext_dof[k0 + k]), v);
         sD = fma(c_sp.e2[sp], v, sD);
         sK = fma(c_sp.e2m[sp], v, sK);
       }
@@ -74,7 +95,7 @@ __global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbat
       gK[el][a] = sK;
     }
     __syncthreads();
-    if (e < ncell) {
+    if (live) {
       const int q = a;   // NQP == NB for (p+1)^2 Gauss points
       const int64_t pt = e * NB + q;
       double td = 0.0, tr = 0.0, tz = 0.0;
@@ -84,8 +105,7 @@ __global__ void __launch_bounds__(NB * EPB) field_kernel(int64_t ncell, int nbat
         tr = fma(s_dxi[k][q], gK[el][k], tr);
         tz = fma(s_deta[k][q], gK[el][k], tz);
       }
-      const double w = pw[pt], ws = w * (2.0 / cell_h[e]);
-      double *o = wT + (int64_t)b * 3 * npts;
+      double *o = wT + b * 3 * npts;
       o[pt] = w * td;
       o[npts + pt] = ws * tr;
       o[2 * npts + pt] = ws * tz;

@@ -247,7 +247,11 @@ int launch_field(landau_t h, int64_t nbatch) {
     const char *e = getenv("LANDAU_FIELD_BLOCKS_PER_SM");
     return e ? (int64_t)atoll(e) : (int64_t)8;
   }();
-  const unsigned grid = (unsigned)std::min<int64_t>(items, blocks_per_sm * num_sms(h));
+  // whole multiples of the chunk count: block g * nchunks + c keeps chunk c (see field_kernel)
+  const int64_t nchunks = (P.ncell + EPB - 1) / EPB;
+  const int64_t G = std::max<int64_t>(1, std::min<int64_t>(nbatch, blocks_per_sm * num_sms(h) / nchunks));
+  const unsigned grid = (unsigned)(G * nchunks);
+  (void)items;
   Timer t(h, LANDAU_T_FIELD);
   field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->fin ? h->fin : h->d_f,
                                                           h->d_ext_ptr, h->d_ext_dof,
