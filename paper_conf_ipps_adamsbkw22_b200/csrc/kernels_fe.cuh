@@ -426,6 +426,21 @@ __global__ void scale_copy_kernel(const double *__restrict__ M, double shift, in
     out[i] = shift * M[i];
 }
 
+// every species block in one launch: out[off_a + i] = scale_a * M_a[i], i < n_a (blockIdx.y = a)
+struct ScaleCopyDesc {
+  const double *M[kMaxSpecies];
+  int64_t n[kMaxSpecies], off[kMaxSpecies];
+  double scale[kMaxSpecies];
+};
+__global__ void scale_copy_species_kernel(const ScaleCopyDesc d, double *__restrict__ out) {
+  const int a = blockIdx.y;
+  const double *M = d.M[a];
+  const double sc = d.scale[a];
+  double *o = out + d.off[a];
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < d.n[a]; i += (int64_t)gridDim.x * blockDim.x)
+    o[i] = sc * M[i];
+}
+
 // copy chunked G layout -> [b][5][N]
 __global__ void unchunk_kernel(const double *__restrict__ G, int64_t N, int64_t Nc, int nbatch, double *__restrict__ out) {
   const int64_t total = (int64_t)nbatch * 5 * N;

@@ -1447,18 +1447,22 @@ int landau_mass(landau_t h, double shift, double *values_dev, int32_t format) {
   if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
   if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "mass: bad argument");
   Timer t(h, LANDAU_T_MASS);
-  for (int a = 0; a < h->S; a++) {
+  ScaleCopyDesc d{};
+  int64_t nmax = 0;
+  for (int a = 0; a < h->S; a++) {   // every species block in one launch
     const int g = h->sgrid[a];
-    const double *M = format == LANDAU_CSR ? h->d_mass_csr[g] : h->d_mass_coo[g];
-    const int64_t n = format == LANDAU_CSR ? (int64_t)h->plan.grids[g].col.size() : h->plan.grids[g].ncoo;
-    const int64_t off = format == LANDAU_CSR ? h->snnz_off[a] : h->scoo_off[a];
-    if (n == 0) continue;
-    const int blocks = (int)std::min<int64_t>((n + 255) / 256, 8LL * num_sms(h));
-    scale_copy_kernel<<<blocks, 256, 0, h->stream>>>(M, shift, n, values_dev + off);
-    h->launches++;
-    h->tlaunch[LANDAU_T_MASS]++;
-    KCHECK();
+    d.M[a] = format == LANDAU_CSR ? h->d_mass_csr[g] : h->d_mass_coo[g];
+    d.n[a] = format == LANDAU_CSR ? (int64_t)h->plan.grids[g].col.size() : h->plan.grids[g].ncoo;
+    d.off[a] = format == LANDAU_CSR ? h->snnz_off[a] : h->scoo_off[a];
+    d.scale[a] = shift;
+    nmax = std::max(nmax, d.n[a]);
   }
+  if (nmax == 0) return LANDAU_OK;
+  const int blocks = (int)std::min<int64_t>((nmax + 255) / 256, 8LL * num_sms(h));
+  scale_copy_species_kernel<<<dim3(blocks, h->S), 256, 0, h->stream>>>(d, values_dev);
+  h->launches++;
+  h->tlaunch[LANDAU_T_MASS]++;
+  KCHECK();
   return LANDAU_OK;
 }
 
