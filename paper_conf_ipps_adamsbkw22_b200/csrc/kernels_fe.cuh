@@ -208,22 +208,12 @@ __global__ void __launch_bounds__(NB * EPB, LANDAU_EL_MINB) element_kernel(int64
 #endif
 constexpr int kSfWarps = LANDAU_SF_WARPS;
 
+// per-lane products of the 1-D factors for the lane's index pair (x, y)
 template <int S>
-__global__ void __launch_bounds__(32 * kSfWarps) element_sf_kernel(int64_t ncell, const double *__restrict__ G,
-                                                                   int64_t Nc, int nbatch, int b0, int nb,
-                                                                   const double *__restrict__ pw,
-                                                                   const double *__restrict__ cell_h,
-                                                                   const double *__restrict__ tab1,
-                                                                   double *__restrict__ Cbuf) {
-  constexpr int NB = S * S, NG = 32 / NB;   // lane groups
-  static_assert(NG >= 1, "S <= 5");
-  __shared__ double sA[kSfWarps][5][NB];       // w_q G(q)
-  __shared__ double sT[kSfWarps][6][NB][S];    // T_t[(b,d)][qr]
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const int xy = lane % NB, grp = lane / NB;
-  const bool act = grp < NG;
-  const int x = xy / S, y = xy % S;
-  double PLL[S], PLD[S], PDL[S], PDD[S];
+__device__ __forceinline__ void sf_tables(const double *tab1, int lane, double PLL[S], double PLD[S], double PDL[S],
+                                          double PDD[S]) {
+  constexpr int NB = S * S;
+  const int xy = lane % NB, x = xy / S, y = xy % S;
 #pragma unroll
   for (int i = 0; i < S; i++) {
     const double Lx = tab1[i * S + x], Ly = tab1[i * S + y], Dx = tab1[NB + i * S + x], Dy = tab1[NB + i * S + y];
@@ -232,6 +222,73 @@ __global__ void __launch_bounds__(32 * kSfWarps) element_sf_kernel(int64_t ncell
     PDL[i] = Dx * Ly;
     PDD[i] = Dx * Dy;
   }
+}
+
+// one cell's C^D, C^K (both sum-factorised contractions) from sA = w_q G(q) [5][NB] (filled and
+// __syncwarp'ed by the caller); sT: the warp's [6][NB][S] scratch; o: the cell's [NB][NB][2] output
+template <int S>
+__device__ __forceinline__ void sf_cell(const double (*sA)[S * S], double (*sT)[S * S][S], int lane,
+                                        const double PLL[S], const double PLD[S], const double PDL[S],
+                                        const double PDD[S], double sc, double *o) {
+  constexpr int NB = S * S, NG = 32 / NB;   // lane groups
+  static_assert(NG >= 1, "S <= 5");
+  const int xy = lane % NB, grp = lane / NB, x = xy / S, y = xy % S;
+  const bool act = grp < NG;
+  if (act) {   // step 1: contract qz for (b, d) = (x, y)
+    for (int qr = grp; qr < S; qr += NG) {
+      double t1 = 0.0, t2 = 0.0, t3 = 0.0, t4 = 0.0, t5 = 0.0, t6 = 0.0;
+#pragma unroll
+      for (int qz = 0; qz < S; qz++) {
+        const int q = qz * S + qr;
+        const double arr = sA[0][q], arz = sA[1][q], azz = sA[2][q], kr = sA[3][q], kz = sA[4][q];
+        t1 = fma(PLL[qz], arr, t1);
+        t2 = fma(PLD[qz], arz, t2);
+        t3 = fma(PDL[qz], arz, t3);
+        t4 = fma(PDD[qz], azz, t4);
+        t5 = fma(PLL[qz], kr, t5);
+        t6 = fma(PDL[qz], kz, t6);
+      }
+      sT[0][xy][qr] = t1;
+      sT[1][xy][qr] = t2;
+      sT[2][xy][qr] = t3;
+      sT[3][xy][qr] = t4;
+      sT[4][xy][qr] = t5;
+      sT[5][xy][qr] = t6;
+    }
+  }
+  __syncwarp();
+  if (act) {   // step 2: contract qr for (a, c) = (x, y), every (b, d) of the lane's group
+    const double sc2 = sc * sc;
+    for (int bd = grp; bd < NB; bd += NG) {
+      double cd = 0.0, ck = 0.0;
+#pragma unroll
+      for (int qr = 0; qr < S; qr++) {
+        cd = fma(PDD[qr], sT[0][bd][qr], cd);
+        cd = fma(PDL[qr], sT[1][bd][qr], cd);
+        cd = fma(PLD[qr], sT[2][bd][qr], cd);
+        cd = fma(PLL[qr], sT[3][bd][qr], cd);
+        ck = fma(PDL[qr], sT[4][bd][qr], ck);
+        ck = fma(PLL[qr], sT[5][bd][qr], ck);
+      }
+      const int k = (bd / S) * S + x, l = (bd % S) * S + y;
+      reinterpret_cast<double2 *>(o)[k * NB + l] = make_double2(cd * sc2, ck * sc);   // (C^D, C^K) interleaved
+    }
+  }
+}
+
+template <int S>
+__global__ void __launch_bounds__(32 * kSfWarps) element_sf_kernel(int64_t ncell, const double *__restrict__ G,
+                                                                   int64_t Nc, int nbatch, int b0, int nb,
+                                                                   const double *__restrict__ pw,
+                                                                   const double *__restrict__ cell_h,
+                                                                   const double *__restrict__ tab1,
+                                                                   double *__restrict__ Cbuf) {
+  constexpr int NB = S * S;
+  __shared__ double sA[kSfWarps][5][NB];       // w_q G(q)
+  __shared__ double sT[kSfWarps][6][NB][S];    // T_t[(b,d)][qr]
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  double PLL[S], PLD[S], PDL[S], PDD[S];
+  sf_tables<S>(tab1, lane, PLL, PLD, PDL, PDD);
   const unsigned nc = (unsigned)ncell, nitems = (unsigned)(ncell * nb);   // < 2^32 (checked by the caller)
   for (unsigned it = blockIdx.x * kSfWarps + wid; it < nitems; it += gridDim.x * kSfWarps) {
     const int bc = (int)(it / nc), b = b0 + bc;
@@ -246,48 +303,7 @@ __global__ void __launch_bounds__(32 * kSfWarps) element_sf_kernel(int64_t ncell
       for (int c = 0; c < 5; c++) sA[wid][c][lane] = w * Gb[c * Nc];
     }
     __syncwarp();
-    if (act) {   // step 1: contract qz for (b, d) = (x, y)
-      for (int qr = grp; qr < S; qr += NG) {
-        double t1 = 0.0, t2 = 0.0, t3 = 0.0, t4 = 0.0, t5 = 0.0, t6 = 0.0;
-#pragma unroll
-        for (int qz = 0; qz < S; qz++) {
-          const int q = qz * S + qr;
-          const double arr = sA[wid][0][q], arz = sA[wid][1][q], azz = sA[wid][2][q], kr = sA[wid][3][q],
-                       kz = sA[wid][4][q];
-          t1 = fma(PLL[qz], arr, t1);
-          t2 = fma(PLD[qz], arz, t2);
-          t3 = fma(PDL[qz], arz, t3);
-          t4 = fma(PDD[qz], azz, t4);
-          t5 = fma(PLL[qz], kr, t5);
-          t6 = fma(PDL[qz], kz, t6);
-        }
-        sT[wid][0][xy][qr] = t1;
-        sT[wid][1][xy][qr] = t2;
-        sT[wid][2][xy][qr] = t3;
-        sT[wid][3][xy][qr] = t4;
-        sT[wid][4][xy][qr] = t5;
-        sT[wid][5][xy][qr] = t6;
-      }
-    }
-    __syncwarp();
-    if (act) {   // step 2: contract qr for (a, c) = (x, y), every (b, d) of the lane's group
-      const double sc = 2.0 / cell_h[e], sc2 = sc * sc;
-      double *o = Cbuf + ((int64_t)bc * ncell + e) * 2 * NB * NB;
-      for (int bd = grp; bd < NB; bd += NG) {
-        double cd = 0.0, ck = 0.0;
-#pragma unroll
-        for (int qr = 0; qr < S; qr++) {
-          cd = fma(PDD[qr], sT[wid][0][bd][qr], cd);
-          cd = fma(PDL[qr], sT[wid][1][bd][qr], cd);
-          cd = fma(PLD[qr], sT[wid][2][bd][qr], cd);
-          cd = fma(PLL[qr], sT[wid][3][bd][qr], cd);
-          ck = fma(PDL[qr], sT[wid][4][bd][qr], ck);
-          ck = fma(PLL[qr], sT[wid][5][bd][qr], ck);
-        }
-        const int k = (bd / S) * S + x, l = (bd % S) * S + y;
-        reinterpret_cast<double2 *>(o)[k * NB + l] = make_double2(cd * sc2, ck * sc);   // (C^D, C^K) interleaved
-      }
-    }
+    sf_cell<S>(sA[wid], sT[wid], lane, PLL, PLD, PDL, PDD, 2.0 / cell_h[e], Cbuf + ((int64_t)bc * ncell + e) * 2 * NB * NB);
   }
 }
 
