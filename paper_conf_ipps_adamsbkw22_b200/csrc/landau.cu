@@ -498,8 +498,12 @@ int launch_inner(landau_t h, int64_t nbatch) {
     h->stats.inner_path = 4;
     int64_t nv = nbatch;
     if (h->mirror_mode == 1) {
+      static const int64_t tail_pct = [] {   // remainder (% of a wave) below which the slot kernel takes it
+        const char *e = getenv("LANDAU_VTX_TAIL_PCT");
+        return e ? (int64_t)atoll(e) : (int64_t)90;
+      }();
       const int64_t rem = nbatch % S;
-      if (rem && rem * 10 < 9 * S) nv = nbatch - rem;
+      if (rem && rem * 100 < tail_pct * S) nv = nbatch - rem;
     }
     {
       Timer t(h, LANDAU_T_INNER);
