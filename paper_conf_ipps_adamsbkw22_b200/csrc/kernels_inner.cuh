@@ -399,7 +399,7 @@ __device__ __forceinline__ void vtx_add_pm(double *sGa, double *sGb, int64_t Hp,
 // returns the forward sums of i (P, M) and the reverse sums of j = 32 b + (L + kend(DIAG)) mod 32
 // (PJ, MJ), kend = 17 for the diagonal item and 32 (i.e. L) otherwise.  s_j: the warp's staged j-tile b
 // as (r, z), (hp_d, hp_kr), (hp_kz, hm_d), (hm_kr, hm_kz), (r^2, -).
-template <bool DIAG, bool MASK>
+template <bool DIAG, bool MASK, bool RESET_J = true>
 __device__ __forceinline__ void vtx_item(int a, const double *rU, const double *zU, const double *wb, int64_t N,
                                          int64_t H, const int32_t *pu, const int32_t *pm, int lane,
                                          const double2 *s_j, const PairCoef &cf, Acc5 &P, Acc5 &M, Acc5 &PJ,
@@ -415,7 +415,8 @@ __device__ __forceinline__ void vtx_item(int a, const double *rU, const double *
   const double r = i < H ? rU[i] : 1.0;
   const double z = i < H ? zU[i] : 1.0e6 + lane;   // padding: far away, zero weights
   const double r2 = r * r;
-  P = M = PJ = MJ = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+  P = M = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+  if constexpr (RESET_J) PJ = MJ = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};   // else: the j-tile's sums carry on
   const int src = (lane + 1) & 31;
   if constexpr (DIAG) {   // step 0: each point with its own mirror (V forward only; U is the self pair)
     const double2 rz = s_j[lane * 5], p01 = s_j[lane * 5 + 1], p2m0 = s_j[lane * 5 + 2], m12 = s_j[lane * 5 + 3],
@@ -459,14 +460,23 @@ __device__ __forceinline__ void vtx_stage_j(int b, const double *rU, const doubl
   d[4] = make_double2(r * r, 0.0);
 }
 
-// N2 (mirror-symmetric, partial-sum slots): the same (a, b) items as the per-vertex kernel, spread
-// over every warp of the GPU (batches below one vertex per SM, single large meshes such as C5); each
-// item stores Ga, Gb of its i-tile (slot 2q) and of its j-tile (slot 2q + 1), reduce_mir_kernel sums
-// each tile's slots in a fixed host-built order.  part = [batch][nslots][2][5][32].
+// N2 (mirror-symmetric, partial-sum slots): the per-vertex kernel's (a, b) U + V items spread over every
+// warp of the GPU (batches below one vertex per SM, single large meshes such as C5).  An item is a
+// j-tile b with a run of na consecutive i-tiles a0 .. a0+na-1 < b, evaluated one after the other: the
+// j-tile is staged once and its reverse sums carry on in registers across the run (after 32 steps
+// every lane holds its own j again), so the item writes na forward slots and one reverse slot
+// (slot0 .. slot0+na); na = 0 is the diagonal item (b, b) with slots slot0 (forward), slot0+1
+// (reverse).  reduce_mir_kernel sums each tile's slots in a fixed host-built order.
+// part = [batch][nslots][2][5][32].
+__device__ __forceinline__ void mir_store_pm(double *o, int pos, const Acc5 &P, const Acc5 &M) {
+  mir_store(o, pos, Acc5{P.drr + M.drr, P.drz + M.drz, P.dzz + M.dzz, P.kr + M.kr, P.kz + M.kz}, false);
+  mir_store(o + 160, pos, Acc5{P.drr - M.drr, P.drz - M.drz, P.dzz - M.dzz, P.kr - M.kr, P.kz - M.kz}, false);
+}
+
 template <int MINB, bool MASK>
 __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_mir_kernel(int64_t N, int64_t H, int64_t nitems_b,
                                                                          int64_t nslots, int64_t nitems,
-                                                                         const int2 *__restrict__ items,
+                                                                         const int4 *__restrict__ items,
                                                                          const double *__restrict__ rU,
                                                                          const double *__restrict__ zU,
                                                                          const int32_t *__restrict__ pu,
@@ -483,22 +493,26 @@ __global__ void __launch_bounds__(32 * kSymWarps, MINB) inner_mir_kernel(int64_t
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   for (int64_t item = (int64_t)blockIdx.x * kSymWarps + wid; item < nitems; item += (int64_t)gridDim.x * kSymWarps) {
     const int64_t bb = item / nitems_b, q = item % nitems_b;
-    const int2 it = items[q];
+    const int4 it = items[q];   // (a0, na, b, slot0)
     const double *wb = wT + bb * 3 * N;
     __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
-    vtx_stage_j(it.y, rU, zU, wb, N, H, pu, pm, lane, s_j[wid]);
+    vtx_stage_j(it.z, rU, zU, wb, N, H, pu, pm, lane, s_j[wid]);
     __syncwarp();
+    double *o = part + (bb * nslots + it.w) * 320;
     Acc5 P, M, PJ, MJ;
-    if (it.x == it.y)
-      vtx_item<true, MASK>(it.x, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
-    else
+    if (it.y == 0) {   // the diagonal item (b, b)
+      vtx_item<true, MASK>(it.z, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
+      mir_store_pm(o, lane, P, M);
+      mir_store_pm(o + 320, (lane + 17) & 31, PJ, MJ);
+    } else {
       vtx_item<false, MASK>(it.x, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
-    double *o = part + (bb * nslots + 2 * q) * 320;
-    const int jf = (lane + (it.x == it.y ? 17 : 32)) & 31;
-    mir_store(o, lane, Acc5{P.drr + M.drr, P.drz + M.drz, P.dzz + M.dzz, P.kr + M.kr, P.kz + M.kz}, false);
-    mir_store(o + 160, lane, Acc5{P.drr - M.drr, P.drz - M.drz, P.dzz - M.dzz, P.kr - M.kr, P.kz - M.kz}, false);
-    mir_store(o + 320, jf, Acc5{PJ.drr + MJ.drr, PJ.drz + MJ.drz, PJ.dzz + MJ.dzz, PJ.kr + MJ.kr, PJ.kz + MJ.kz}, false);
-    mir_store(o + 480, jf, Acc5{PJ.drr - MJ.drr, PJ.drz - MJ.drz, PJ.dzz - MJ.dzz, PJ.kr - MJ.kr, PJ.kz - MJ.kz}, false);
+      mir_store_pm(o, lane, P, M);
+      for (int t = 1; t < it.y; t++) {
+        vtx_item<false, MASK, false>(it.x + t, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
+        mir_store_pm(o + t * 320, lane, P, M);
+      }
+      mir_store_pm(o + it.y * 320, lane, PJ, MJ);   // after 32 steps per i-tile lane L holds j = 32 b + L
+    }
   }
 }
 

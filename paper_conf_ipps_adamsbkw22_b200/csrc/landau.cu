@@ -84,7 +84,7 @@ struct landau_s {
   int64_t mir_evals = 0;   // tensor evaluations per batch item of this handle's slot-kernel items
   bool mirror_on = true;   // use inner_mir_kernel when the symmetric path runs (landau_set_mirror)
   int mirror_mode = 1;     // 1: auto (per-vertex kernel for large batches), 2: slot kernel, 3: per-vertex kernel
-  int64_t H = 0, nmir_items = 0, nmir_slots = 0;
+  int64_t H = 0;
   // per-vertex mirror kernel (inner_vtx_kernel): round schedule of tile-pair items
   VtxItem *d_vtx_items = nullptr;
   int32_t *d_vtx_round_ptr = nullptr;
@@ -92,8 +92,13 @@ struct landau_s {
   size_t vtx_smem = 0;     // dynamic shared memory (Ga, Gb); 0 when the vertex does not fit
   double *d_rU = nullptr, *d_zU = nullptr;
   int32_t *d_pu = nullptr, *d_pm = nullptr;
-  int2 *d_mir_items = nullptr;
-  int32_t *d_mtile_ptr = nullptr, *d_mtile_slots = nullptr;
+  // slot-kernel item sets: [0] one i-tile per item (fine-grained: small batches), [1] runs of up to
+  // LANDAU_MIR_RUN i-tiles per j-tile (fewer slots and stagings: large work, e.g. C5)
+  struct MirSet {
+    int4 *items = nullptr;
+    int32_t *tile_ptr = nullptr, *tile_slots = nullptr;
+    int64_t nitems = 0, nslots = 0;
+  } mset[2];
   bool coincident = false;   // two distinct quadrature points with identical (r, z) (never for one grid)
   // tensor cache (NEXT-4)
   bool tcache = false, tcache_valid = false;
@@ -330,7 +335,8 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
     ip.wtiles = h->ntiles;
     ip.nsplit = 1;
     ip.split_len = N;
-    const int64_t need = (h->mirror && h->mirror_on) ? nbatch * h->nmir_slots * 320 : nbatch * h->nsym_slots * 160;
+    const int64_t need = (h->mirror && h->mirror_on) ? nbatch * std::max(h->mset[0].nslots, h->mset[1].nslots) * 320
+                                                     : nbatch * h->nsym_slots * 160;
     if (need > h->part_cap) {
       drop_graphs(h);
       cudaFree(h->d_part);
@@ -461,27 +467,34 @@ int launch_inner(landau_t h, int64_t nbatch) {
   } else {
     h->stats.pair_evaluations = ip.wtiles * 32 * ip.tpt * N;
   }
-  // mirror slot kernel over batch items [b0, b0 + nb): partial slots, then their reduction
+  // mirror slot kernel over batch items [b0, b0 + nb): partial slots, then their reduction; the item
+  // set with runs when the work is ample (>= 16 items per resident warp), single i-tiles otherwise
+  auto mir_set = [&](int64_t nb) -> const landau_s::MirSet & {
+    const landau_s::MirSet &r = h->mset[1];
+    return (r.nitems && nb * r.nitems >= 16LL * kSymWarps * LANDAU_SYM_MINB * num_sms(h)) ? r : h->mset[0];
+  };
   auto mir_slots = [&](int64_t b0, int64_t nb) -> int {
-    const int64_t nitems = nb * h->nmir_items;
+    const landau_s::MirSet &ms = mir_set(nb);
+    const int64_t nitems = nb * ms.nitems;
     const double *wT = h->d_wT + b0 * 3 * N;
     const unsigned grid = (unsigned)std::min<int64_t>((nitems + kSymWarps - 1) / kSymWarps, (int64_t)LANDAU_SYM_MINB * num_sms(h));
     if (h->coincident)
       inner_mir_kernel<LANDAU_SYM_MINB, true><<<grid, 32 * kSymWarps, 0, h->stream>>>(
-          N, h->H, h->nmir_items, h->nmir_slots, nitems, h->d_mir_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, wT, h->d_part);
+          N, h->H, ms.nitems, ms.nslots, nitems, ms.items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, wT, h->d_part);
     else
       inner_mir_kernel<LANDAU_SYM_MINB, false><<<grid, 32 * kSymWarps, 0, h->stream>>>(
-          N, h->H, h->nmir_items, h->nmir_slots, nitems, h->d_mir_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, wT, h->d_part);
+          N, h->H, ms.nitems, ms.nslots, nitems, ms.items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, wT, h->d_part);
     h->launches++;
     KCHECK();
     return LANDAU_OK;
   };
   auto mir_reduce = [&](int64_t b0, int64_t nb) -> int {
+    const landau_s::MirSet &ms = mir_set(nb);
     Timer t(h, LANDAU_T_REDUCE);
     const int64_t total = nb * 5 * h->H;
     const int blocks = (int)std::min<int64_t>((total + 255) / 256, 16LL * num_sms(h));
-    reduce_mir_kernel<<<blocks, 256, 0, h->stream>>>(N, h->H, h->nmir_slots, h->d_mtile_ptr, h->d_mtile_slots, h->d_pu,
-                                                     h->d_pm, h->d_part, G_own + b0 * 5 * h->Nc, 5 * h->Nc, (int)nb);
+    reduce_mir_kernel<<<blocks, 256, 0, h->stream>>>(N, h->H, ms.nslots, ms.tile_ptr, ms.tile_slots, h->d_pu, h->d_pm,
+                                                     h->d_part, G_own + b0 * 5 * h->Nc, 5 * h->Nc, (int)nb);
     h->launches++;
     h->tlaunch[LANDAU_T_REDUCE]++;
     KCHECK();
@@ -527,7 +540,7 @@ int launch_inner(landau_t h, int64_t nbatch) {
   if (ip.sym && h->mirror && h->mirror_on) {
     {
       Timer t(h, LANDAU_T_INNER);
-      if (h->nmir_items && (rc = mir_slots(0, nbatch))) return rc;
+      if (mir_set(nbatch).nitems && (rc = mir_slots(0, nbatch))) return rc;
       h->tlaunch[LANDAU_T_INNER]++;
     }
     if ((rc = mir_reduce(0, nbatch))) return rc;
@@ -1085,31 +1098,66 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
     if (ok && !pu.empty()) {
       const int64_t H = (int64_t)pu.size();
       const int T = (int)((H + 31) / 32);
-      // slot-kernel items: every tile pair (a <= b) once, U and V together; item q stores the sums of
-      // its i-tile a in slot 2q and of its j-tile b in slot 2q + 1
-      // (world > 1: this rank's share of the items, landau_pair_partition, with local slot numbers)
-      std::vector<int2> items;
-      std::vector<std::vector<int32_t>> slots_of(T);
-      int64_t iq0 = 0, iq1 = (int64_t)T * (T + 1) / 2, qg = 0;
+      // slot-kernel items: every tile pair (a <= b) once, U and V together, as runs of up to `run`
+      // consecutive i-tiles a0 .. a0+na-1 < b against one j-tile b (slots: na forward, then one
+      // reverse), and the diagonal items (b, b) (slots: forward, reverse); two sets (run 1 and
+      // LANDAU_MIR_RUN).  world > 1: this rank's share of the pairs (landau_pair_partition), local slots
+      static const int mir_run = [] {
+        const char *e = getenv("LANDAU_MIR_RUN");
+        const int v = e ? atoi(e) : 4;
+        return v < 1 ? 1 : v;
+      }();
+      int64_t iq0 = 0, iq1 = (int64_t)T * (T + 1) / 2;
       if (world > 1) landau_pair_partition(T, world, rank, &iq0, &iq1);
       if (world == 1)
         if (const char *e = getenv("LANDAU_PAIR_SPLIT_EMULATE")) {   // test hook: "world:rank" -- this
           int ew = 1, er = 0;                                         // rank's items only, no all-reduce
           if (sscanf(e, "%d:%d", &ew, &er) == 2 && ew >= 1 && er >= 0 && er < ew) landau_pair_partition(T, ew, er, &iq0, &iq1);
         }
-      for (int b = 0; b < T; b++)
-        for (int a = 0; a <= b; a++, qg++) {
-          if (qg < iq0 || qg >= iq1) continue;
-          const int q = (int)items.size();
-          items.push_back(make_int2(a, b));
-          slots_of[a].push_back(2 * q);
-          slots_of[b].push_back(2 * q + 1);
+      for (int set = 0; set < 2; set++) {
+        const int run = set == 0 ? 1 : mir_run;
+        if (set == 1 && run == 1) break;
+        std::vector<int4> items;
+        std::vector<std::vector<int32_t>> slots_of(T);
+        int slot = 0;
+        int64_t qg = 0;
+        for (int b = 0; b < T; b++) {
+          int run0 = -1, runn = 0;
+          auto flush = [&]() {
+            if (!runn) return;
+            items.push_back(make_int4(run0, runn, b, slot));
+            for (int t = 0; t < runn; t++) slots_of[run0 + t].push_back(slot++);
+            slots_of[b].push_back(slot++);
+            runn = 0;
+          };
+          for (int a = 0; a <= b; a++, qg++) {
+            if (qg < iq0 || qg >= iq1) continue;
+            if (a == b) {
+              flush();
+              items.push_back(make_int4(b, 0, b, slot));
+              slots_of[b].push_back(slot++);
+              slots_of[b].push_back(slot++);
+              continue;
+            }
+            if (runn && (a != run0 + runn || runn == run)) flush();
+            if (!runn) run0 = a;
+            runn++;
+          }
+          flush();
         }
-      const int slot = 2 * (int)items.size();
-      std::vector<int32_t> tptr(1, 0), tslots;
-      for (int t = 0; t < T; t++) {
-        tslots.insert(tslots.end(), slots_of[t].begin(), slots_of[t].end());
-        tptr.push_back((int32_t)tslots.size());
+        std::vector<int32_t> tptr(1, 0), tslots;
+        for (int t = 0; t < T; t++) {
+          tslots.insert(tslots.end(), slots_of[t].begin(), slots_of[t].end());
+          tptr.push_back((int32_t)tslots.size());
+        }
+        auto &ms = h->mset[set];
+        ms.nitems = (int64_t)items.size();
+        ms.nslots = slot;
+        if (set == 0)
+          for (const int4 &it : items) h->mir_evals += it.y == 0 ? 33 * 32 : (int64_t)it.y * 2 * 32 * 32;
+        if ((rc = upload(h, &ms.items, items)) || (rc = upload(h, &ms.tile_ptr, tptr)) ||
+            (rc = upload(h, &ms.tile_slots, tslots)))
+          return bail(rc);
       }
       // per-vertex kernel schedule: round-robin tournament of the T tiles (circle method; rounds of
       // disjoint tile pairs), then the diagonal items in rounds of kVtxWarps.  For odd T every round
@@ -1151,12 +1199,8 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
       }
       h->mirror = true;
       h->H = H;
-      h->nmir_items = (int64_t)items.size();
-      h->nmir_slots = slot;
-      for (const int2 &it : items) h->mir_evals += it.x == it.y ? 33 * 32 : 2 * 32 * 32;
       if ((rc = upload(h, &h->d_rU, rU)) || (rc = upload(h, &h->d_zU, zU)) || (rc = upload(h, &h->d_pu, pu)) ||
-          (rc = upload(h, &h->d_pm, pm)) || (rc = upload(h, &h->d_mir_items, items)) ||
-          (rc = upload(h, &h->d_mtile_ptr, tptr)) || (rc = upload(h, &h->d_mtile_slots, tslots)))
+          (rc = upload(h, &h->d_pm, pm)))
         return bail(rc);
       if (world > 1) {   // pair split: every rank targets every point, G summed by an all-reduce
         h->dist_pairs = true;
@@ -1269,11 +1313,13 @@ void landau_destroy(landau_t h) {
   cudaFree(h->d_zU);
   cudaFree(h->d_pu);
   cudaFree(h->d_pm);
-  cudaFree(h->d_mir_items);
+  for (auto &ms : h->mset) {
+    cudaFree(ms.items);
+    cudaFree(ms.tile_ptr);
+    cudaFree(ms.tile_slots);
+  }
   cudaFree(h->d_vtx_items);
   cudaFree(h->d_vtx_round_ptr);
-  cudaFree(h->d_mtile_ptr);
-  cudaFree(h->d_mtile_slots);
   cudaFree(h->d_ext_ptr);
   cudaFree(h->d_ext_dof);
   for (auto *v : {&h->d_csr, &h->d_coo})
