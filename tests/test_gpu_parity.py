@@ -840,3 +840,83 @@ def test_bench_gpu_arm_json_line():
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0 and d["e2e"]["value"] > 0
     assert d["gpu_launches"] > 0 and d["config"]["workload"].startswith("C4")
+
+
+def _balanced_random_mesh(rng, R, nsplit, mirror):
+    """Two R x R roots refined at random (mirror: every split applied to the z -> -z image too), then
+    2:1-balanced by splitting any cell with an edge neighbour more than one level finer."""
+    cells = [(0.0, -R, R), (0.0, 0.0, R)]
+    for _ in range(nsplit):
+        c = cells[rng.integers(len(cells))]
+        if c[2] < R / 32:
+            continue
+        todo = {c}
+        if mirror:
+            todo.add((c[0], -c[1] - c[2], c[2]))
+        cells = [x for x in cells if x not in todo] + [y for x in todo if x in cells for y in inputs._split(x)]
+    while True:
+        bad = None
+        for a in cells:
+            for b in cells:
+                if a[2] <= 2 * b[2]:
+                    continue
+                ra, za, ha = a
+                rb, zb, hb = b
+                touch_r = (abs(ra + ha - rb) < 1e-12 or abs(rb + hb - ra) < 1e-12) and zb < za + ha and zb + hb > za
+                touch_z = (abs(za + ha - zb) < 1e-12 or abs(zb + hb - za) < 1e-12) and rb < ra + ha and rb + hb > ra
+                if touch_r or touch_z:
+                    bad = a
+                    break
+            if bad:
+                break
+        if bad is None:
+            return cells
+        todo = {bad}
+        if mirror:
+            todo.add((bad[0], -bad[1] - bad[2], bad[2]))
+        cells = [x for x in cells if x not in todo] + [y for x in todo if x in cells for y in inputs._split(x)]
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3, 4, 5, 6])
+def test_random_meshes_every_inner_path(seed):
+    """Random 2:1-balanced quadtrees with hanging nodes (mirror-symmetric for odd seeds, asymmetric for
+    even ones), orders p = 2, 3, 4, one or two species: point coefficients of a small batch through the
+    inner kernels the mesh admits (per-vertex, mirror-directed, directed) against the oracle, and one
+    item's Jacobian."""
+    rng = np.random.default_rng(1000 + seed)
+    R = inputs.R_E
+    mirror = seed % 2 == 1
+    cells = _balanced_random_mesh(rng, R, int(rng.integers(3, 9)), mirror)
+    order = 2 + seed % 3
+    species = [inputs.Species("e", 1.0, -1.0, 0)]
+    fmix = [[(1.0, 1.0, 0.2)]]
+    if seed > 2:
+        species.append(inputs.Species("D", inputs.M_D, 1.0, 0))
+        fmix.append([(1.0, 1.0, 0.0)])
+    prob = inputs.Problem(f"rand{seed}", order, [(R, cells)], species, fmix=fmix, seed=seed)
+    o = Oracle(prob)
+    fo = o.coefficients()
+    Go, Ga = o.point_coeffs(fo)
+    h = L.Landau.from_problem(prob, device=0)
+    fg = inputs.coefficients(prob, h.all_nodes())
+    nb = 5
+    F = torch.tensor(np.stack([fg * (1.0 + 0.05 * k) for k in range(nb)]), device=DEV)
+    modes = ["vertex", "slots", True, False] if mirror else [False]
+    paths = set()
+    for mode in modes:
+        if mirror:
+            h.set_mirror(mode)
+        h.set_state_batched(F)
+        G = torch.empty((nb, 5, h.npoints), dtype=torch.float64, device=DEV)
+        h.point_coeffs_batched(G)
+        torch.cuda.synchronize()
+        paths.add(h.stats()["inner_path"])
+        Gn = G.cpu().numpy()
+        for k in (0, nb - 1):
+            sc = 1.0 + 0.05 * k
+            assert np.max(np.abs(Gn[k] - sc * Go) / (sc * Ga)) <= 1e-12, (mode, k)
+    if mirror:
+        assert {4, 5} <= paths, paths   # per-vertex and mirror-directed kernels both exercised
+    J = gpu_jacobian(h, fg)
+    Jo, Ja = o.jacobian(fo)
+    assert np.all(np.abs(J - Jo) <= 1e-11 * Ja)
