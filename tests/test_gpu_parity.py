@@ -920,3 +920,35 @@ def test_random_meshes_every_inner_path(seed):
     J = gpu_jacobian(h, fg)
     Jo, Ja = o.jacobian(fo)
     assert np.all(np.abs(J - Jo) <= 1e-11 * Ja)
+
+
+def test_pair_split_partials_sum_with_item_runs(monkeypatch):
+    """The pair split on a batch large enough for the slot kernel's i-tile runs on every rank (C4 mesh,
+    2048 vertices, slot mode): three emulated ranks' partial G sum to the full G of one handle (the
+    same sums in another grouping)."""
+    prob = inputs.config4_vertex(0)
+    nb = 2048   # each emulated rank still has >= 16 items per resident warp: the run item set
+    base = L.Landau.from_problem(prob, device=0)
+    nodes = base.all_nodes()
+    F1 = np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in range(0, 1024, 4)])
+    F = torch.tensor(np.concatenate([F1 * (1.0 + 0.01 * k) for k in range(nb // F1.shape[0])]), device=DEV)
+
+    def G_of(env):
+        if env:
+            monkeypatch.setenv("LANDAU_PAIR_SPLIT_EMULATE", env)
+        else:
+            monkeypatch.delenv("LANDAU_PAIR_SPLIT_EMULATE", raising=False)
+        h = L.Landau.from_problem(prob, device=0)
+        h.set_mirror("slots")
+        h.set_state_batched(F)
+        G = torch.empty((nb, 5, h.npoints), dtype=torch.float64, device=DEV)
+        h.point_coeffs_batched(G)
+        torch.cuda.synchronize()
+        assert h.stats()["inner_path"] == 3
+        h.close()
+        return G.cpu().numpy()
+
+    Gfull = G_of(None)
+    Gsum = sum(G_of(f"3:{r}") for r in range(3))
+    scale = np.abs(Gfull).max(axis=2, keepdims=True)
+    assert np.max(np.abs(Gsum - Gfull) / scale) <= 1e-12
