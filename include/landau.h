@@ -258,8 +258,10 @@ typedef struct {
   int32_t inner_path;        /* 0: directed pair kernel (every ordered pair, split-j when small);
                                 1: symmetric pair kernel (every unordered pair once, both targets);
                                 2: tensor cache + FP64 GEMM (landau_set_tensor_cache);
-                                3: mirror-symmetric pair kernel (landau_set_mirror)
-                                4: mirror-symmetric per-vertex kernel (+ slot kernel for a remainder) */
+                                3: mirror-symmetric pair kernel, partial-sum slots (landau_set_mirror;
+                                   with the pair split: this rank's share of the items)
+                                4: mirror-symmetric per-vertex kernel (+ slot kernel for a remainder)
+                                5: mirror-symmetric directed kernel (single builds, small batches) */
   int64_t nbatch;            /* batch items of the last build                                      */
   int64_t targets;           /* target points per batch item (all N unless element-split)          */
   int64_t sources;           /* source points per batch item (N)                                   */
