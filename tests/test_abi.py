@@ -144,3 +144,17 @@ def test_create_without_gpu_fails_loudly():
     with pytest.raises(L.LandauError) as ei:
         L.Landau.from_problem(inputs.config1(), device=0, stream=0)
     assert ei.value.code == L.LANDAU_ECUDA
+
+
+def test_argument_errors_without_gpu():
+    """Error codes the header documents, checked before any device work: set_mirror outside 0..3 is
+    EINVAL and the mirror on a host-only handle (no mirror maps) EUNSUPPORTED; landau3d_inner with
+    n < 0 or NULL pointers is EINVAL and with n = 0 a no-op."""
+    h = _host(inputs.config1())
+    lib = L.lib()
+    assert lib.landau_set_mirror(h._h, 7) == L.LANDAU_EINVAL
+    assert lib.landau_set_mirror(h._h, -1) == L.LANDAU_EINVAL
+    assert lib.landau_set_mirror(h._h, 1) == L.LANDAU_EUNSUPPORTED
+    assert lib.landau3d_inner(-1, None, None, None, None, None) == L.LANDAU_EINVAL
+    assert lib.landau3d_inner(5, None, None, None, None, None) == L.LANDAU_EINVAL
+    assert lib.landau3d_inner(0, None, None, None, None, None) == L.LANDAU_OK
