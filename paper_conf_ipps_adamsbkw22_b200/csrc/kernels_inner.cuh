@@ -685,13 +685,21 @@ __global__ void reduce_mdir_kernel(int64_t N, int64_t H, int64_t Hp, int nsplit,
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
     const int64_t b = k / (5 * H), c = (k / H) % 5, u = k % H;
     const double *pb = part + b * nsplit * 10 * Hp + c * Hp + u;
-    double sa = 0.0, sb = 0.0;
-    for (int q = 0; q < nsplit; q++) {
-      sa += pb[(int64_t)q * 10 * Hp];
-      sb += pb[(int64_t)q * 10 * Hp + 5 * Hp];
+    double sa[4] = {0.0, 0.0, 0.0, 0.0}, sb[4] = {0.0, 0.0, 0.0, 0.0};   // 4 independent chains, fixed order
+    int q = 0;
+    for (; q + 4 <= nsplit; q += 4)
+#pragma unroll
+      for (int m = 0; m < 4; m++) {
+        sa[m] += pb[(int64_t)(q + m) * 10 * Hp];
+        sb[m] += pb[(int64_t)(q + m) * 10 * Hp + 5 * Hp];
+      }
+    for (; q < nsplit; q++) {
+      sa[0] += pb[(int64_t)q * 10 * Hp];
+      sb[0] += pb[(int64_t)q * 10 * Hp + 5 * Hp];
     }
-    G[b * G_bstride + c * N + pu[u]] = sa;
-    G[b * G_bstride + c * N + pm[u]] = (c == 1 || c == 4) ? -sb : sb;
+    const double ta = (sa[0] + sa[1]) + (sa[2] + sa[3]), tb = (sb[0] + sb[1]) + (sb[2] + sb[3]);
+    G[b * G_bstride + c * N + pu[u]] = ta;
+    G[b * G_bstride + c * N + pm[u]] = (c == 1 || c == 4) ? -tb : tb;
   }
 }
 
@@ -706,13 +714,23 @@ __global__ void reduce_mir_kernel(int64_t N, int64_t H, int64_t nslots, const in
     const int64_t b = k / (5 * H), c = (k / H) % 5, u = k % H;
     const int t = (int)(u / 32), lane = (int)(u % 32);
     const double *pbk = part + b * nslots * 320 + c * 32 + lane;
-    double sa = 0.0, sb = 0.0;
-    for (int q = tile_ptr[t]; q < tile_ptr[t + 1]; q++) {
-      sa += pbk[(int64_t)tile_slots[q] * 320];
-      sb += pbk[(int64_t)tile_slots[q] * 320 + 160];
+    double sa[4] = {0.0, 0.0, 0.0, 0.0}, sb[4] = {0.0, 0.0, 0.0, 0.0};   // 4 independent chains, fixed order
+    const int q0 = tile_ptr[t], q1 = tile_ptr[t + 1];
+    int q = q0;
+    for (; q + 4 <= q1; q += 4)
+#pragma unroll
+      for (int m = 0; m < 4; m++) {
+        const int64_t sl = tile_slots[q + m];
+        sa[m] += pbk[sl * 320];
+        sb[m] += pbk[sl * 320 + 160];
+      }
+    for (; q < q1; q++) {
+      sa[0] += pbk[(int64_t)tile_slots[q] * 320];
+      sb[0] += pbk[(int64_t)tile_slots[q] * 320 + 160];
     }
-    G[b * G_bstride + c * N + pu[u]] = sa;
-    G[b * G_bstride + c * N + pm[u]] = (c == 1 || c == 4) ? -sb : sb;
+    const double ta = (sa[0] + sa[1]) + (sa[2] + sa[3]), tb = (sb[0] + sb[1]) + (sb[2] + sb[3]);
+    G[b * G_bstride + c * N + pu[u]] = ta;
+    G[b * G_bstride + c * N + pm[u]] = (c == 1 || c == 4) ? -tb : tb;
   }
 }
 
@@ -755,9 +773,13 @@ __global__ void reduce_kernel(int64_t nt, int nsplit, const double *__restrict__
   for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
     const int64_t b = k / (5 * nt), ci = k % (5 * nt);
     const double *p = part + b * (int64_t)nsplit * 5 * nt + ci;
-    double s = 0.0;
-    for (int q = 0; q < nsplit; q++) s += p[(int64_t)q * 5 * nt];
-    G[b * G_bstride + ci] = s;
+    double s4[4] = {0.0, 0.0, 0.0, 0.0};   // 4 independent chains, fixed order
+    int q = 0;
+    for (; q + 4 <= nsplit; q += 4)
+#pragma unroll
+      for (int m = 0; m < 4; m++) s4[m] += p[(int64_t)(q + m) * 5 * nt];
+    for (; q < nsplit; q++) s4[0] += p[(int64_t)q * 5 * nt];
+    G[b * G_bstride + ci] = (s4[0] + s4[1]) + (s4[2] + s4[3]);
   }
 }
 

@@ -258,9 +258,16 @@ int launch_field(landau_t h, int64_t nbatch) {
   const unsigned grid = (unsigned)(G * nchunks);
   (void)items;
   Timer t(h, LANDAU_T_FIELD);
-  field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->fin ? h->fin : h->d_f,
-                                                          h->d_ext_ptr, h->d_ext_dof,
-                                                          h->d_ext_w, h->d_cell_grid, h->d_h, h->d_w, h->d_tab, h->spc, h->d_wT, P.npts);
+  if (nchunks * nbatch < num_sms(h)) {   // small builds (a single C2 grid: 9 blocks): one cell per block
+    field_kernel<NB, 1><<<(unsigned)(P.ncell * std::max<int64_t>(1, std::min<int64_t>(nbatch, num_sms(h)))), NB, 0,
+                          h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->fin ? h->fin : h->d_f, h->d_ext_ptr,
+                                       h->d_ext_dof, h->d_ext_w, h->d_cell_grid, h->d_h, h->d_w, h->d_tab, h->spc,
+                                       h->d_wT, P.npts);
+  } else {
+    field_kernel<NB, EPB><<<grid, NB * EPB, 0, h->stream>>>(P.ncell, (int)nbatch, h->ndof, h->fin ? h->fin : h->d_f,
+                                                            h->d_ext_ptr, h->d_ext_dof, h->d_ext_w, h->d_cell_grid,
+                                                            h->d_h, h->d_w, h->d_tab, h->spc, h->d_wT, P.npts);
+  }
   h->launches++;
   h->tlaunch[LANDAU_T_FIELD]++;
   KCHECK();
