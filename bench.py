@@ -254,7 +254,8 @@ def main():
     desc, prob0, items = workload(args, world, rank)
     dist_desc = None
     if args.workload == "C5":
-        # one large mesh: target cells split over the ranks, one NCCL all-gather of G per build
+        # one large mesh: the mirror kernel's tile pairs split over the ranks, one NCCL all-reduce of
+        # the partial G per build (the pair split; the element split + all-gather on non-mirror meshes)
         if world > 1:
             dist_desc = L.make_dist(L.LANDAU_DIST_ELEMENTS)
         else:
