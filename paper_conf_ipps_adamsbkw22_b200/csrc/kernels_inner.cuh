@@ -677,29 +677,48 @@ __global__ void __launch_bounds__(32 * kMdirWarps) inner_mdir_kernel(int64_t N, 
   }
 }
 
-// G[b][c][pu(u)] = sum over splits of Ga, G[b][c][pm(u)] = F (sum of Gb), splits in order
-__global__ void reduce_mdir_kernel(int64_t N, int64_t H, int64_t Hp, int nsplit, const int32_t *__restrict__ pu,
-                                   const int32_t *__restrict__ pm, const double *__restrict__ part,
-                                   double *__restrict__ G, int64_t G_bstride, int nbatch) {
-  const int64_t total = (int64_t)nbatch * 5 * H;
-  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t b = k / (5 * H), c = (k / H) % 5, u = k % H;
+// G[b][c][pu(u)] = sum over splits of Ga, G[b][c][pm(u)] = F (sum of Gb).  One block per (b, c,
+// 32-target tile): warp w sums the splits q = w, w + 8, ... (independent loads in flight), then warp 0
+// adds the 8 warp sums in order -- a fixed summation order, so the result is deterministic.
+constexpr int kRedWarps = 8;
+
+__global__ void __launch_bounds__(32 * kRedWarps) reduce_mdir_kernel(int64_t N, int64_t H, int64_t Hp, int nsplit,
+                                                                   const int32_t *__restrict__ pu,
+                                                                   const int32_t *__restrict__ pm,
+                                                                   const double *__restrict__ part,
+                                                                   double *__restrict__ G, int64_t G_bstride,
+                                                                   int nbatch) {
+  __shared__ double2 s_w[kRedWarps][32];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t T = Hp / 32, nitems = (int64_t)nbatch * 5 * T;
+  for (int64_t it = blockIdx.x; it < nitems; it += gridDim.x) {
+    const int64_t b = it / (5 * T), c = (it / T) % 5, u = (it % T) * 32 + lane;
     const double *pb = part + b * nsplit * 10 * Hp + c * Hp + u;
-    double sa[4] = {0.0, 0.0, 0.0, 0.0}, sb[4] = {0.0, 0.0, 0.0, 0.0};   // 4 independent chains, fixed order
-    int q = 0;
-    for (; q + 4 <= nsplit; q += 4)
-#pragma unroll
-      for (int m = 0; m < 4; m++) {
-        sa[m] += pb[(int64_t)(q + m) * 10 * Hp];
-        sb[m] += pb[(int64_t)(q + m) * 10 * Hp + 5 * Hp];
-      }
-    for (; q < nsplit; q++) {
+    double sa[2] = {0.0, 0.0}, sb[2] = {0.0, 0.0};
+    int q = wid;
+    for (; q + kRedWarps < nsplit; q += 2 * kRedWarps) {
+      sa[0] += pb[(int64_t)q * 10 * Hp];
+      sb[0] += pb[(int64_t)q * 10 * Hp + 5 * Hp];
+      sa[1] += pb[(int64_t)(q + kRedWarps) * 10 * Hp];
+      sb[1] += pb[(int64_t)(q + kRedWarps) * 10 * Hp + 5 * Hp];
+    }
+    if (q < nsplit) {
       sa[0] += pb[(int64_t)q * 10 * Hp];
       sb[0] += pb[(int64_t)q * 10 * Hp + 5 * Hp];
     }
-    const double ta = (sa[0] + sa[1]) + (sa[2] + sa[3]), tb = (sb[0] + sb[1]) + (sb[2] + sb[3]);
-    G[b * G_bstride + c * N + pu[u]] = ta;
-    G[b * G_bstride + c * N + pm[u]] = (c == 1 || c == 4) ? -tb : tb;
+    s_w[wid][lane] = make_double2(sa[0] + sa[1], sb[0] + sb[1]);
+    __syncthreads();
+    if (wid == 0 && u < H) {
+      double ta = 0.0, tb = 0.0;
+#pragma unroll
+      for (int w = 0; w < kRedWarps; w++) {
+        ta += s_w[w][lane].x;
+        tb += s_w[w][lane].y;
+      }
+      G[b * G_bstride + c * N + pu[u]] = ta;
+      G[b * G_bstride + c * N + pm[u]] = (c == 1 || c == 4) ? -tb : tb;
+    }
+    __syncthreads();
   }
 }
 

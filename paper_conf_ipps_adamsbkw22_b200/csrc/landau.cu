@@ -603,9 +603,8 @@ int launch_inner(landau_t h, int64_t nbatch) {
     }
     if (nsplit > 1) {
       Timer t(h, LANDAU_T_REDUCE);
-      const int64_t total = nbatch * 5 * h->H;
-      const int blocks = (int)std::min<int64_t>((total + 255) / 256, 16LL * num_sms(h));
-      reduce_mdir_kernel<<<blocks, 256, 0, h->stream>>>(N, h->H, T * 32, (int)nsplit, h->d_pu, h->d_pm, h->d_part, G_own,
+      const int blocks = (int)std::min<int64_t>(nbatch * 5 * T, 16LL * num_sms(h));
+      reduce_mdir_kernel<<<blocks, 32 * kRedWarps, 0, h->stream>>>(N, h->H, T * 32, (int)nsplit, h->d_pu, h->d_pm, h->d_part, G_own,
                                                         5 * h->Nc, (int)nbatch);
       h->launches++;
       h->tlaunch[LANDAU_T_REDUCE]++;
