@@ -101,7 +101,41 @@ class Clocks:
         self._stop = threading.Event()
         self._t = None
 
+    # NVML clock-event reason bits (nvml.h nvmlClocksEventReason*)
+    NVML_BITS = {"sw_power_cap": 0x4, "hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40}
+
+    def _nvml_handle(self):
+        import pynvml
+        pynvml.nvmlInit()
+        idx = self.index
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES", "")
+        parts = [p.strip() for p in vis.split(",") if p.strip()]
+        if parts and all(p.isdigit() for p in parts) and idx < len(parts):
+            idx = int(parts[idx])
+        return pynvml, pynvml.nvmlDeviceGetHandleByIndex(idx)
+
     def _run(self):
+        # In-process NVML sampling every 5 ms, so that a timed region of a few tens of ms still gets
+        # several samples; nvidia-smi (one process per sample, ~50 ms) only when NVML is unavailable.
+        try:
+            nv, h = self._nvml_handle()
+            reasons_fn = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                nv.nvmlDeviceGetCurrentClocksThrottleReasons
+            mx = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+            while True:
+                sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
+                bits = reasons_fn(h)
+                self.rows.append([str(self.index), str(sm), str(mx), "", hex(bits)] +
+                                 ["Active" if bits & self.NVML_BITS[k] else "Not Active"
+                                  for k in ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown",
+                                            "sw_power_cap")])
+                if self._stop.wait(0.005):
+                    break
+            self.source = "nvml"
+            return
+        except Exception:
+            self.rows = []
+        self.source = "nvidia-smi"
         while not self._stop.is_set():
             try:
                 out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
@@ -129,7 +163,7 @@ class Clocks:
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[k] for r in self.rows for k in range(4) if len(r) > 5 + k and r[5 + k] == "Active"})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+                "reasons": reasons, "samples": len(self.rows), "source": getattr(self, "source", "nvidia-smi")}
 
 
 def fp64_peak_tflops(props, sm_max_mhz):
