@@ -46,3 +46,27 @@ def test_c4_sharding_weak_and_strong():
             assert desc["vertices"] == job and len(items) == job // world
             seen += [it.seed for it in items]
         assert sorted(seen) == [20220 + b for b in range(job)]
+
+
+def test_clock_summary_decodes_nvml_reason_bits():
+    """The clocks key: NVML clock-event reason bits (nvml.h: sw_power_cap 0x4, hw_slowdown 0x8,
+    sw_thermal_slowdown 0x20, hw_thermal_slowdown 0x40) become the reasons the driver rejects or notes;
+    the SM clock is the median over samples, the max clock the largest reported."""
+    sys.path.insert(0, ROOT)
+    import bench
+    c = bench.Clocks(0)
+    B = bench.Clocks.NVML_BITS
+
+    def row(sm, bits):
+        return ["0", str(sm), "1965", "", hex(bits)] + [
+            "Active" if bits & B[k] else "Not Active"
+            for k in ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")]
+
+    c.rows = [row(1965, 0), row(1900, B["sw_power_cap"]), row(1965, 0x1)]   # 0x1 = GPU idle: not a reason
+    c.source = "nvml"
+    s = c.summary()
+    assert s == {"sm_mhz": 1965.0, "sm_max_mhz": 1965.0, "reasons": ["sw_power_cap"], "samples": 3,
+                 "source": "nvml"}
+    c.rows = [row(1200, B["hw_thermal_slowdown"] | B["hw_slowdown"]), row(1300, B["sw_thermal_slowdown"])]
+    assert c.summary()["reasons"] == ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown"]
+    assert c.summary()["sm_mhz"] == 1250.0
