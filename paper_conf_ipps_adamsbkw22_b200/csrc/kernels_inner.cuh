@@ -695,7 +695,8 @@ __global__ void __launch_bounds__(32 * kRedWarps) reduce_mdir_kernel(int64_t N, 
     const int64_t b = it / (5 * T), c = (it / T) % 5, u = (it % T) * 32 + lane;
     const double *pb = part + b * nsplit * 10 * Hp + c * Hp + u;
     double sa[2] = {0.0, 0.0}, sb[2] = {0.0, 0.0};
-    int q = wid;
+    // lanes past H (the ragged last tile) never read: those slots are not written by the inner kernel
+    int q = u < H ? wid : nsplit;
     for (; q + kRedWarps < nsplit; q += 2 * kRedWarps) {
       sa[0] += pb[(int64_t)q * 10 * Hp];
       sb[0] += pb[(int64_t)q * 10 * Hp + 5 * Hp];
