@@ -225,19 +225,32 @@ int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double E
                                  double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm);
 
 /* Mirror symmetry (v_par -> -v_par, i.e. z -> -z): when every grid's quadrature points come in pairs
- * (r, z), (r, -z) (within 1e-12 R, no point on z = 0) -- true of every configuration of SURVEY §8(d)
- * -- the batched (symmetric) inner integral evaluates each tensor once for four ordered interactions:
- * reflection keeps lambda+-, x, m and every azimuthal integral and negates the rz / zr components,
+ * (r, z), (r, -z) BIT-EXACTLY (no point on z = 0; the dyadic meshes of every configuration of SURVEY
+ * §8(d) qualify, the cell-centre point formula keeps mirrored points exact negatives) the batched
+ * (symmetric) inner integral evaluates each tensor once for four ordered interactions: reflection keeps
+ * lambda+-, x, m and every azimuthal integral and negates the rz / zr components,
  * U(i', j') = F U(i, j) F with F = diag(1, -1), on top of the i <-> j symmetry (N^2/4 tensor
- * evaluations per build instead of N^2/2).  The mirror point is placed at exactly (r, -z), a
- * perturbation within the 1e-12 R detection tolerance.  On by default when available.
- * enable: 0 = plain symmetric kernel; 1 = mirror, automatic (batches of at least one vertex per SM run
- * whole waves of the per-vertex kernel -- one CTA per batch item, sums in shared memory, no partial
- * slots -- and a remainder below 0.9 of a wave on the slot kernel); 2 = mirror slot kernel only;
- * 3 = per-vertex kernel for every batch size.  enable != 0 on a non-symmetric mesh, or 3 when a
+ * evaluations per build instead of N^2/2).  A mesh symmetric only up to rounding is not detected (the
+ * general kernels run at the caller's exact points).  On by default when available.
+ * enable: 0 = plain symmetric kernel; 1 = mirror, automatic (batches with at least 8 round weights per
+ * SM -- C2: 32 vertices -- run the per-vertex kernel: one CTA per SM, a stream-K split of the batch's
+ * (vertex, round) work, sums in shared memory, a split vertex's two or more partials added in CTA order;
+ * smaller batches the slot kernel or, below that, the mirror-directed kernel); 2 = mirror slot kernel
+ * only; 3 = per-vertex kernel for every batch size (one CTA per vertex when the batch is below one
+ * vertex per SM: no vertex split).  enable != 0 on a non-symmetric mesh, or 3 when a
  * vertex's sums (80 B per upper-half point) exceed 160 KB of shared memory, is EUNSUPPORTED;
  * enable outside 0..3 is EINVAL. */
 int landau_set_mirror(landau_t h, int32_t enable);
+/* Whether the mesh is exactly z-mirror-symmetric (host logic, also on LANDAU_HOST_ONLY handles) and
+ * whether the mirror kernels are in use on this handle.  Either pointer may be NULL.  EINVAL: h NULL. */
+int landau_get_mirror(landau_t h, int32_t *mirror_symmetric, int32_t *mirror_active);
+/* The per-vertex kernel's stream-K schedule, for diagnostics and tests: nrounds (host,
+ * may be NULL) rounds per vertex; weight_prefix (host, [nrounds + 1], may be NULL) the cumulative round
+ * weights (a round of pair items weighs 2, of diagonal items 1); ctas (may be NULL) the CTAs of an
+ * automatic-mode launch.  Round rd of batch item v runs on CTA floor((v W + wp[rd]) ctas / (nbatch W)),
+ * W = wp[nrounds]; a vertex whose rounds share one CTA is summed in one fixed order, whatever the batch.
+ * EUNSUPPORTED when the per-vertex kernel is not available on this handle. */
+int landau_get_vtx_schedule(landau_t h, int32_t *nrounds, int32_t *weight_prefix, int32_t *ctas);
 
 /* NEXT-4: the inner integral with the 3D Cartesian Landau tensor of Eq. 3
  * (PAPER.md:1@7593, "a full 3D model is supported in the library" @7997-8072), without azimuthal

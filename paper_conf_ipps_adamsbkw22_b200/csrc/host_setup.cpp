@@ -5,6 +5,9 @@
 #include <cmath>
 #include <cstdio>
 #include <climits>
+#include <cstdlib>
+#include <cstring>
+#include <new>
 #include <functional>
 #include <map>
 #include <unordered_map>
@@ -81,6 +84,10 @@ struct ICell {
 std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, const double *radius, int order,
                        Plan &plan) {
   char msg[256];
+  // fault injection for the CPU test of the C ABI's exception safety (tests/test_abi.py): a host
+  // allocation failure inside the plan must come back as LANDAU_ENOMEM, not terminate the caller
+  if (const char *e = getenv("LANDAU_TEST_FAIL_ALLOC"))
+    if (!strcmp(e, "plan")) throw std::bad_alloc();
   const int p = order, nq = order + 1, nb = (p + 1) * (p + 1), nqp = nq * nq;
   plan = Plan();
   plan.p = p;
@@ -495,10 +502,14 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
       const double r0 = cc[3 * c], z0 = cc[3 * c + 1], h = cc[3 * c + 2];
       plan.cell_h.push_back(h);
       plan.cell_grid.push_back(g);
+      // points from the cell centre: with the exactly antisymmetric Gauss nodes (xg[n-1-i] = -xg[i])
+      // the points of a mirrored cell (z0' = -z0 - h exactly, as the dyadic meshes of inputs.py give)
+      // are the bit-exact negatives z' = -z, which the mirror kernels require (landau_create)
+      const double rc = r0 + 0.5 * h, zc = z0 + 0.5 * h, hh = 0.5 * h;
       for (int qz = 0; qz < nq; qz++)
         for (int qr = 0; qr < nq; qr++) {
-          double r = r0 + 0.5 * h * (xg[qr] + 1.0);
-          double z = z0 + 0.5 * h * (xg[qz] + 1.0);
+          double r = rc + hh * xg[qr];
+          double z = zc + hh * xg[qz];
           plan.pr.push_back(r);
           plan.pz.push_back(z);
           plan.pw.push_back(wg[qr] * wg[qz] * (0.25 * h * h) * r);

@@ -528,19 +528,63 @@ struct VtxItem {   // host-built: tiles (a, b) of the upper half; a == b: the di
   int a, b;
 };
 
+// Stream-K decomposition over (vertex, round) work.  The batch's rounds form one flattened sequence
+// (vertex-major, rounds in schedule order) with weights wp (a full round of pair items: 2, a round of
+// diagonal items: 1 -- their durations); round (v, rd) starting at weight g = v Wv + wp[rd] belongs to
+// CTA floor(g S / Wtot) of the S persistent CTAs, so every CTA gets a contiguous, equally heavy range
+// for any batch size (no partial last wave: 128 vertices on 148 SMs run 14.7 rounds per SM instead of
+// 17).  A vertex whose rounds lie in one CTA is summed in shared memory and written once, as before; a
+// vertex cut by a CTA boundary is summed per CTA into a partial slot (the CTA's first segment: slot
+// (c, 0), its last: (c, 1)), and the last CTA to finish one of its segments (an atomic counter per
+// vertex) adds the partials in CTA order -- a fixed order, so every build is bitwise reproducible.
+struct VtxSched {
+  int nbatch, nrounds, S;
+  int64_t Wv, Wtot;      // weight per vertex, whole batch
+};
+
+__device__ __forceinline__ int vtx_owner(const VtxSched &sc, const int32_t *wp, int64_t v, int rd) {
+  return (int)(((v * sc.Wv + wp[rd]) * (int64_t)sc.S) / sc.Wtot);
+}
+
+// first flattened round index f = v * nrounds + rd owned by CTA >= c (nbatch * nrounds if none)
+__device__ __forceinline__ int64_t vtx_first_round(const VtxSched &sc, const int32_t *wp, int c) {
+  int64_t lo = 0, hi = (int64_t)sc.nbatch * sc.nrounds;
+  while (lo < hi) {
+    const int64_t mid = (lo + hi) >> 1;
+    if (vtx_owner(sc, wp, mid / sc.nrounds, (int)(mid % sc.nrounds)) >= c) hi = mid;
+    else lo = mid + 1;
+  }
+  return lo;
+}
+
+// write a vertex's sums: G(pu) = Ga, G(pm) = F Gb  (F: negate the rz and K_z components)
+__device__ __forceinline__ void vtx_write_G(double *Gb, const double *sGa, const double *sGb, int64_t N, int64_t H,
+                                            int64_t Hp, const int32_t *pu, const int32_t *pm) {
+  for (int64_t k = threadIdx.x; k < 5 * H; k += blockDim.x) {
+    const int64_t c = k / H, u = k % H;
+    Gb[c * N + pu[u]] = sGa[c * Hp + u];
+    const double v = sGb[c * Hp + u];
+    Gb[c * N + pm[u]] = (c == 1 || c == 4) ? -v : v;
+  }
+}
+
 template <bool MASK>
-__global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int64_t N, int64_t H, int nrounds,
+__global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int64_t N, int64_t H, VtxSched sc,
                                                                       const int32_t *__restrict__ round_ptr,
+                                                                      const int32_t *__restrict__ wp,
                                                                       const VtxItem *__restrict__ items,
                                                                       const double *__restrict__ rU,
                                                                       const double *__restrict__ zU,
                                                                       const int32_t *__restrict__ pu,
                                                                       const int32_t *__restrict__ pm,
-                                                                      const double *__restrict__ wT, int nbatch,
-                                                                      double *__restrict__ G, int64_t G_bstride) {
+                                                                      const double *__restrict__ wT,
+                                                                      double *__restrict__ G, int64_t G_bstride,
+                                                                      double *__restrict__ part,
+                                                                      int32_t *__restrict__ counters) {
   __shared__ double2 s_j[kVtxWarps][32 * 5];
   __shared__ double s_coef[kNumPairCoef];
   __shared__ double2 s_ltab[kLogTab];
+  __shared__ int s_last;
   extern __shared__ double s_G[];   // Ga [5][Hp], Gb [5][Hp]
   const int64_t Hp = (H + 31) / 32 * 32;
   double *sGa = s_G, *sGb = s_G + 5 * Hp;
@@ -549,11 +593,18 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
   PairCoef cf;
   load_pair_coef(s_coef, s_ltab, cf);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  for (int bb = blockIdx.x; bb < nbatch; bb += gridDim.x) {
-    const double *wb = wT + (int64_t)bb * 3 * N;
+  const int c = blockIdx.x;
+  const int64_t f0 = vtx_first_round(sc, wp, c), f1 = vtx_first_round(sc, wp, c + 1);
+  int64_t f = f0;
+  while (f < f1) {
+    const int64_t v = f / sc.nrounds;
+    const int rd0 = (int)(f % sc.nrounds);
+    const int rd1 = (int)min((int64_t)sc.nrounds, f1 - v * sc.nrounds);   // this CTA's rounds [rd0, rd1) of v
+    f = v * sc.nrounds + rd1;
+    const double *wb = wT + v * 3 * N;
     for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) s_G[k] = 0.0;
     __syncthreads();
-    for (int rd = 0; rd < nrounds; rd++) {
+    for (int rd = rd0; rd < rd1; rd++) {
       for (int q = round_ptr[rd] + wid; q < round_ptr[rd + 1]; q += kVtxWarps) {
         const VtxItem it = items[q];
         __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
@@ -570,14 +621,29 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
       }
       __syncthreads();   // the next round's tiles may be this round's
     }
-    double *Gb = G + (int64_t)bb * G_bstride;
-    for (int64_t k = threadIdx.x; k < 5 * H; k += blockDim.x) {
-      const int64_t c = k / H, u = k % H;
-      Gb[c * N + pu[u]] = sGa[c * Hp + u];
-      const double v = sGb[c * Hp + u];
-      Gb[c * N + pm[u]] = (c == 1 || c == 4) ? -v : v;
+    const int cfirst = vtx_owner(sc, wp, v, 0), clast = vtx_owner(sc, wp, v, sc.nrounds - 1);
+    if (cfirst == clast) {   // the whole vertex ran here
+      vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, pu, pm);
+    } else {                 // one segment of a split vertex: partial slot, then the last one combines
+      double *slot = part + ((int64_t)c * 2 + (c == cfirst ? 1 : 0)) * 10 * Hp;
+      for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) slot[k] = s_G[k];
+      __threadfence();
+      __syncthreads();
+      if (threadIdx.x == 0) s_last = atomicAdd(&counters[v], 1) == clast - cfirst;
+      __syncthreads();
+      if (s_last) {
+        __threadfence();
+        for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) {   // partials in CTA order
+          double acc = __ldcg(part + ((int64_t)cfirst * 2 + 1) * 10 * Hp + k);
+          for (int cc = cfirst + 1; cc <= clast; cc++) acc += __ldcg(part + (int64_t)cc * 2 * 10 * Hp + k);
+          s_G[k] = acc;
+        }
+        __syncthreads();
+        vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, pu, pm);
+        if (threadIdx.x == 0) counters[v] = 0;   // ready for the next build
+      }
     }
-    __syncthreads();   // the write-out reads s_G before the next vertex zeroes it
+    __syncthreads();   // the write-out reads s_G before the next segment zeroes it
   }
 }
 

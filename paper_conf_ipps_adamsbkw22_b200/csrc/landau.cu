@@ -79,7 +79,9 @@ struct landau_s {
   int64_t nsym_items = 0, nsym_slots = 0;
   // mirror-symmetric inner kernel (meshes symmetric under z -> -z): upper-half points u, their
   // original indices pu and mirrors pm, work items and slot map over the tiles of the upper half
-  bool mirror = false;     // the mesh is mirror-symmetric (maps built)
+  bool mirror_sym = false; // every grid's points pair up bit-exactly under z -> -z (detect_mirror)
+  std::vector<int32_t> mir_pu, mir_pm;   // host copies of the pairing (upper half, mirror)
+  bool mirror = false;     // the mirror kernels are set up (maps built on the device)
   bool dist_pairs = false; // element-split mode on a mirror mesh: tile pairs split over ranks + all-reduce
   int64_t mir_evals = 0;   // tensor evaluations per batch item of this handle's slot-kernel items
   bool mirror_on = true;   // use inner_mir_kernel when the symmetric path runs (landau_set_mirror)
@@ -90,6 +92,11 @@ struct landau_s {
   int32_t *d_vtx_round_ptr = nullptr;
   int nvtx_rounds = 0;
   size_t vtx_smem = 0;     // dynamic shared memory (Ga, Gb); 0 when the vertex does not fit
+  int32_t *d_vtx_wp = nullptr;       // stream-K: prefix of the round weights [nrounds + 1]
+  int64_t vtx_Wv = 0;                // weight of one vertex
+  double *d_vtx_part = nullptr;      // stream-K partial slots [grid][2][10 Hp]
+  int32_t *d_vtx_cnt = nullptr;      // stream-K per-vertex arrival counters [cap] (zero between builds)
+  int64_t vtx_cnt_cap = 0;
   double *d_rU = nullptr, *d_zU = nullptr;
   int32_t *d_pu = nullptr, *d_pm = nullptr;
   // slot-kernel item sets: [0] one i-tile per item (fine-grained: small batches), [1] runs of up to
@@ -276,6 +283,7 @@ int launch_field(landau_t h, int64_t nbatch) {
 
 
 struct InnerPlan {
+  bool vtx = false;    // mirror-symmetric per-vertex kernel, stream-K over (vertex, round) work
   bool sym;   // symmetric pair evaluation (whole point set as targets, enough tile pairs to fill the GPU)
   bool mdir = false;   // mirror-symmetric directed kernel (single builds / small batches on z-mirror meshes)
   int tpt;
@@ -308,11 +316,12 @@ bool mirror_enabled() {
   return v;
 }
 
-// per-vertex mirror kernel when the batch gives every SM at least this many vertices (LANDAU_VTX_MIN_BATCH_PER_SM)
-int64_t vtx_min_batch_per_sm() {
+// per-vertex mirror kernel (automatic mode) when the batch gives every SM at least this much round
+// weight (a full round of pair items weighs 2; LANDAU_VTX_MIN_WEIGHT_PER_SM)
+int64_t vtx_min_weight_per_sm() {
   static const int64_t v = [] {
-    const char *e = getenv("LANDAU_VTX_MIN_BATCH_PER_SM");
-    return e ? (int64_t)atoll(e) : (int64_t)1;
+    const char *e = getenv("LANDAU_VTX_MIN_WEIGHT_PER_SM");
+    return e ? (int64_t)atoll(e) : (int64_t)8;
   }();
   return v;
 }
@@ -332,6 +341,29 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
   const Plan &P = h->plan;
   const int64_t N = P.npts, nt = (h->e1 - h->e0) * P.nqp;
   const int variant = inner_variant();
+  ip.vtx = h->mirror && h->mirror_on && h->vtx_smem && !h->dist_pairs &&
+           (h->mirror_mode == 3 ||
+            (h->mirror_mode == 1 && nbatch * h->vtx_Wv >= vtx_min_weight_per_sm() * num_sms(h) * kVtxMinB));
+  if (ip.vtx) {   // stream-K partial slots (one pair per CTA) and per-vertex arrival counters
+    if (!h->d_vtx_part) {
+      const int64_t Hp = (h->H + 31) / 32 * 32;
+      CU(cudaMalloc(&h->d_vtx_part, sizeof(double) * (int64_t)num_sms(h) * kVtxMinB * 2 * 10 * Hp));
+    }
+    if (nbatch > h->vtx_cnt_cap) {
+      drop_graphs(h);
+      cudaFree(h->d_vtx_cnt);
+      h->d_vtx_cnt = nullptr;
+      CU(cudaMalloc(&h->d_vtx_cnt, sizeof(int32_t) * nbatch));
+      CU(cudaMemsetAsync(h->d_vtx_cnt, 0, sizeof(int32_t) * nbatch, h->stream));
+      h->vtx_cnt_cap = nbatch;
+    }
+    ip.sym = false;
+    ip.tpt = 1;
+    ip.wtiles = (h->H + 31) / 32;
+    ip.nsplit = 1;
+    ip.split_len = h->H;
+    return LANDAU_OK;
+  }
   // symmetric path: all targets on this rank (no element split across ranks), enough work items to
   // fill the GPU, and partial slots within 24 GiB (C5: ~11 GiB of the 180 GB HBM)
   ip.sym = sym_enabled() && h->world == 1 && h->nsym_items > 0 && nbatch * h->nsym_items >= sym_min_items_per_sm() * num_sms(h) &&
@@ -507,41 +539,32 @@ int launch_inner(landau_t h, int64_t nbatch) {
     KCHECK();
     return LANDAU_OK;
   };
-  if (h->mirror && h->mirror_on && h->vtx_smem &&
-      (h->mirror_mode == 3 || (h->mirror_mode == 1 && ip.sym && nbatch >= vtx_min_batch_per_sm() * num_sms(h) * kVtxMinB))) {
-    // one CTA per vertex, sums in shared memory (no slots, no reduction kernel).  Auto mode runs
-    // whole waves of vertices this way and hands a remainder below 0.9 of a wave to the slot kernel,
-    // which spreads its items over every SM (a partial wave would leave SMs idle).
-    const int64_t T = (h->H + 31) / 32, S = (int64_t)num_sms(h) * kVtxMinB;   // vertices per wave
+  if (ip.vtx) {   // one CTA per SM, stream-K over the batch's (vertex, round) work, sums in shared memory
+    const int64_t T = (h->H + 31) / 32;
     h->stats.pair_evaluations = T * 33 * 32 + 2 * (T * (T - 1) / 2) * 32 * 32;
     h->stats.nsplit = 1;
     h->stats.inner_path = 4;
-    int64_t nv = nbatch;
-    if (h->mirror_mode == 1) {
-      static const int64_t tail_pct = [] {   // remainder (% of a wave) below which the slot kernel takes it
-        const char *e = getenv("LANDAU_VTX_TAIL_PCT");
-        return e ? (int64_t)atoll(e) : (int64_t)90;
-      }();
-      const int64_t rem = nbatch % S;
-      if (rem && rem * 100 < tail_pct * S) nv = nbatch - rem;
-    }
-    {
-      Timer t(h, LANDAU_T_INNER);
-      const unsigned grid = (unsigned)std::min<int64_t>(nv, S);
-      if (h->coincident)
-        inner_vtx_kernel<true><<<grid, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(
-            N, h->H, h->nvtx_rounds, h->d_vtx_round_ptr, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
-            (int)nv, G_own, 5 * h->Nc);
-      else
-        inner_vtx_kernel<false><<<grid, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(
-            N, h->H, h->nvtx_rounds, h->d_vtx_round_ptr, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
-            (int)nv, G_own, 5 * h->Nc);
-      h->launches++;
-      h->tlaunch[LANDAU_T_INNER]++;   // one inner stage per build (the remainder's kernel is part of it)
-      KCHECK();
-      if (nv < nbatch && (rc = mir_slots(nv, nbatch - nv))) return rc;
-    }
-    if (nv < nbatch) return mir_reduce(nv, nbatch - nv);
+    VtxSched sc;
+    sc.nbatch = (int)nbatch;
+    sc.nrounds = h->nvtx_rounds;
+    // automatic mode: every SM; mode 3 with a batch below one vertex per SM: one CTA per vertex (no
+    // vertex is split: the summation order of a lone build, used by the parity tests)
+    sc.S = num_sms(h) * kVtxMinB;
+    if (h->mirror_mode == 3 && nbatch < sc.S) sc.S = (int)nbatch;
+    sc.Wv = h->vtx_Wv;
+    sc.Wtot = nbatch * h->vtx_Wv;
+    Timer t(h, LANDAU_T_INNER);
+    if (h->coincident)
+      inner_vtx_kernel<true><<<sc.S, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(
+          N, h->H, sc, h->d_vtx_round_ptr, h->d_vtx_wp, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
+          G_own, 5 * h->Nc, h->d_vtx_part, h->d_vtx_cnt);
+    else
+      inner_vtx_kernel<false><<<sc.S, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(
+          N, h->H, sc, h->d_vtx_round_ptr, h->d_vtx_wp, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
+          G_own, 5 * h->Nc, h->d_vtx_part, h->d_vtx_cnt);
+    h->launches++;
+    h->tlaunch[LANDAU_T_INNER]++;
+    KCHECK();
     return LANDAU_OK;
   }
   if (ip.sym && h->mirror && h->mirror_on) {
@@ -553,6 +576,7 @@ int launch_inner(landau_t h, int64_t nbatch) {
     if ((rc = mir_reduce(0, nbatch))) return rc;
     if (h->dist_pairs) {   // the exchange step: sum the ranks' partial G (every rank gets all of G)
       Timer t(h, LANDAU_T_ALLGATHER);
+      h->tlaunch[LANDAU_T_ALLGATHER]++;   // stage count (a NCCL collective, not one of our kernels)
       const int rc2 = g_nccl.AllReduce(G_own, G_own, (size_t)(nbatch * 5 * h->Nc), kNcclFloat64, kNcclSum, h->comm,
                                        h->stream);
       if (rc2 != 0)
@@ -612,6 +636,7 @@ int launch_inner(landau_t h, int64_t nbatch) {
     }
     if (h->comm) {   // LANDAU_DIST_ELEMENTS at world 1: the (trivial) exchange step
       Timer t(h, LANDAU_T_ALLGATHER);
+      h->tlaunch[LANDAU_T_ALLGATHER]++;   // stage count (a NCCL collective, not one of our kernels)
       int rc2 = g_nccl.AllGather(G_own, h->d_G, (size_t)(nbatch * 5 * h->Nc), kNcclFloat64, h->comm, h->stream);
       if (rc2 != 0) return fail(h, LANDAU_ENCCL, "ncclAllGather failed");
     }
@@ -656,6 +681,7 @@ int launch_inner(landau_t h, int64_t nbatch) {
   }
   if (h->comm) {   // LANDAU_DIST_ELEMENTS: the exchange step (also run at world == 1)
     Timer t(h, LANDAU_T_ALLGATHER);
+      h->tlaunch[LANDAU_T_ALLGATHER]++;   // stage count (a NCCL collective, not one of our kernels)
     int rc = g_nccl.AllGather(G_own, h->d_G, (size_t)(nbatch * 5 * h->Nc), kNcclFloat64, h->comm, h->stream);
     if (rc != 0) return fail(h, LANDAU_ENCCL, std::string("ncclAllGather: ") + (g_nccl.GetErrorString ? g_nccl.GetErrorString(rc) : "error"));
   }
@@ -830,11 +856,76 @@ int build_mass(landau_t h) {
   return LANDAU_OK;
 }
 
+// Mirror symmetry z -> -z: every grid's quadrature points pair up as (r, z), (r, -z)
+// BIT-EXACTLY (no point on z = 0).  The mirror kernels evaluate the tensors of a point's mirror from
+// the point itself, so anything short of bit-exact equality would move the caller's points; meshes
+// that are symmetric only up to rounding take the general kernels.  pu: upper-half points (z > 0),
+// pm: their mirrors, grid by grid, each grid's pairs sorted by (r, z).
+bool detect_mirror(const Plan &P, std::vector<int32_t> &pu, std::vector<int32_t> &pm) {
+  pu.clear();
+  pm.clear();
+  for (int g = 0; g < P.ngrids; g++) {
+    const GridPlan &G = P.grids[g];
+    std::vector<int64_t> up, lo;
+    for (int64_t i = G.pt0; i < G.pt0 + G.ncell * P.nqp; i++) {
+      if (P.pz[i] > 0) up.push_back(i);
+      else if (P.pz[i] < 0) lo.push_back(i);
+      else return false;   // a point on z = 0 would be its own mirror
+    }
+    if (up.size() != lo.size()) return false;
+    auto by_rz = [&](int64_t a, int64_t b) { return P.pr[a] != P.pr[b] ? P.pr[a] < P.pr[b] : P.pz[a] < P.pz[b]; };
+    auto by_rmz = [&](int64_t a, int64_t b) { return P.pr[a] != P.pr[b] ? P.pr[a] < P.pr[b] : -P.pz[a] < -P.pz[b]; };
+    std::sort(up.begin(), up.end(), by_rz);
+    std::sort(lo.begin(), lo.end(), by_rmz);
+    for (size_t k = 0; k < up.size(); k++) {
+      const int64_t a = up[k], b = lo[k];
+      if (P.pr[a] != P.pr[b] || P.pz[b] != -P.pz[a]) return false;
+      if (k && P.pr[a] == P.pr[up[k - 1]] && P.pz[a] == P.pz[up[k - 1]]) return false;   // twins
+      pu.push_back((int32_t)a);
+      pm.push_back((int32_t)b);
+    }
+  }
+  return !pu.empty();
+}
+
+// Every C entry point runs its body through guarded(): the header promises that nothing throws or
+// aborts, so a std::bad_alloc (host vectors of a large mesh or batch) becomes LANDAU_ENOMEM and any
+// other exception LANDAU_EINVAL, and a handle's calls run on the handle's device whatever device is
+// current in the calling thread (restored afterwards).
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(landau_t h) {
+    int cur = 0;
+    if (h && !h->host_only && cudaGetDevice(&cur) == cudaSuccess && cur != h->device && cudaSetDevice(h->device) == cudaSuccess)
+      prev = cur;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+template <class F>
+int guarded(landau_t h, F &&body) {
+  try {
+    DeviceGuard g(h);
+    return body();
+  } catch (const std::bad_alloc &) {
+    return fail(h, LANDAU_ENOMEM, "host allocation failed (std::bad_alloc)");
+  } catch (const std::exception &e) {
+    return fail(h, LANDAU_EINVAL, std::string("exception: ") + e.what());
+  } catch (...) {
+    return fail(h, LANDAU_EINVAL, "unknown exception");
+  }
+}
+
 }  // namespace
 
 // ==================================================================================================
 // C ABI
 // ==================================================================================================
+static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, const landau_params_t *prm,
+                       int32_t cuda_device, void *cuda_stream, const landau_dist_t *dist);
+
 extern "C" {
 
 const char *landau_version(void) { return "landau-b200 0.1 (sm_100a, FP64)"; }
@@ -855,15 +946,18 @@ const char *landau_strerror(int code) {
 const char *landau_last_error(landau_t h) { return h ? h->err.c_str() : g_create_error.c_str(); }
 
 int landau_partition(int64_t nelem, int32_t world, int32_t rank, int64_t *e0, int64_t *e1) {
+  return guarded(nullptr, [&]() -> int {
   if (nelem < 0 || world < 1 || rank < 0 || rank >= world || !e0 || !e1) return LANDAU_EINVAL;
   const int64_t chunk = (nelem + world - 1) / world;
   *e0 = std::min<int64_t>(nelem, (int64_t)rank * chunk);
   *e1 = std::min<int64_t>(nelem, (int64_t)(rank + 1) * chunk);
   return LANDAU_OK;
+});
 }
 
 int landau3d_inner(int64_t n, const double *xyz_dev, const double *wTD_dev, const double *wTK_dev, double *G_dev,
                    void *cuda_stream) {
+  return guarded(nullptr, [&]() -> int {
   if (n < 0 || (n > 0 && (!xyz_dev || !wTD_dev || !wTK_dev || !G_dev))) return LANDAU_EINVAL;
   if (n == 0) return LANDAU_OK;
   cudaStream_t st = (cudaStream_t)cuda_stream;
@@ -899,9 +993,11 @@ int landau3d_inner(int64_t n, const double *xyz_dev, const double *wTD_dev, cons
     cudaFreeAsync(part, st);
   }
   return e == cudaSuccess ? LANDAU_OK : LANDAU_ECUDA;
+});
 }
 
 int landau_pair_partition(int64_t ntiles, int32_t world, int32_t rank, int64_t *q0, int64_t *q1) {
+  return guarded(nullptr, [&]() -> int {
   if (ntiles < 0 || world < 1 || rank < 0 || rank >= world || !q0 || !q1) return LANDAU_EINVAL;
   // items in the slot kernel's order (b = 0.., a = 0..b), weight 2 per pair, 1 per diagonal item
   // (half the steps); rank r takes the items whose weight prefix lies in [r W / world, (r+1) W / world)
@@ -921,20 +1017,650 @@ int landau_pair_partition(int64_t ntiles, int32_t world, int32_t rank, int64_t *
   *q0 = lo < 0 ? nitems : lo;
   *q1 = std::max(*q0, hi);
   return LANDAU_OK;
+});
 }
 
 int landau_nccl_unique_id(void *out128) {
+  return guarded(nullptr, [&]() -> int {
   if (!out128) return LANDAU_EINVAL;
   if (!load_nccl()) return LANDAU_ENCCL;
   ncclUniqueId_ id;
   if (g_nccl.GetUniqueId(&id) != 0) return LANDAU_ENCCL;
   memcpy(out128, &id, 128);
   return LANDAU_OK;
+});
 }
 
 int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_t *prm, int32_t cuda_device,
                   void *cuda_stream, const landau_dist_t *dist) {
   landau_t h = nullptr;
+  int rc, prev_dev = -1;
+  if (cuda_device != LANDAU_HOST_ONLY && cudaGetDevice(&prev_dev) != cudaSuccess) prev_dev = -1;
+  try {
+    rc = create_impl(h, out, mesh, prm, cuda_device, cuda_stream, dist);
+  } catch (const std::bad_alloc &) {
+    rc = fail(nullptr, LANDAU_ENOMEM, "landau_create: host allocation failed (std::bad_alloc)");
+  } catch (const std::exception &e) {
+    rc = fail(nullptr, LANDAU_EINVAL, std::string("landau_create: ") + e.what());
+  } catch (...) {
+    rc = fail(nullptr, LANDAU_EINVAL, "landau_create: unknown exception");
+  }
+  if (rc && h) {   // a throw left a partly built handle behind
+    const std::string m = g_create_error;
+    landau_destroy(h);
+    g_create_error = m;
+    if (out) *out = nullptr;
+  }
+  if (prev_dev >= 0) cudaSetDevice(prev_dev);   // the caller's current device is left as it was
+  return rc;
+}
+
+void landau_destroy(landau_t h) {
+  try {
+  if (!h) return;
+  if (h->host_only) {
+    delete h;
+    return;
+  }
+  cudaSetDevice(h->device);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  drop_graphs(h);
+  if (h->cublas && g_cublas.Destroy) g_cublas.Destroy(h->cublas);
+  cudaFree(h->d_U);
+  for (int32_t *p : h->d_ent_ptr) cudaFree(p);
+  for (int32_t *p : h->d_ent_slot) cudaFree(p);
+  for (uint16_t *p : h->d_ent_pos) cudaFree(p);
+  cudaFree(h->d_Aent);
+  cudaFree(h->d_band_desc);
+  cudaFree(h->d_perm_all);
+  cudaFree(h->d_perm_off);
+  cudaFree(h->d_vec_off);
+  cudaFree(h->d_band);
+  if (h->s_h2d) cudaStreamDestroy(h->s_h2d);
+  if (h->s_d2h) cudaStreamDestroy(h->s_d2h);
+  for (auto e : h->ev_h2d) cudaEventDestroy(e);
+  for (auto e : h->ev_built) cudaEventDestroy(e);
+  if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
+  for (double *p : {h->d_r, h->d_z, h->d_w, h->d_h, h->d_tab, h->d_ext_w, h->d_f, h->d_wT, h->d_part, h->d_G, h->d_C, h->d_vals_tmp})
+    cudaFree(p);
+  cudaFree(h->d_cell_grid);
+  cudaFree(h->d_sym_items);
+  cudaFree(h->d_tile_ptr);
+  cudaFree(h->d_tile_slots);
+  cudaFree(h->d_rU);
+  cudaFree(h->d_zU);
+  cudaFree(h->d_pu);
+  cudaFree(h->d_pm);
+  for (auto &ms : h->mset) {
+    cudaFree(ms.items);
+    cudaFree(ms.tile_ptr);
+    cudaFree(ms.tile_slots);
+  }
+  cudaFree(h->d_vtx_items);
+  cudaFree(h->d_vtx_round_ptr);
+  cudaFree(h->d_vtx_wp);
+  cudaFree(h->d_vtx_part);
+  cudaFree(h->d_vtx_cnt);
+  cudaFree(h->d_ext_ptr);
+  cudaFree(h->d_ext_dof);
+  for (auto *v : {&h->d_csr, &h->d_coo})
+    for (auto &m : *v) {
+      cudaFree(m.ptr);
+      cudaFree(m.idx);
+      cudaFree(m.w);
+    }
+  for (double *p : h->d_mass_csr) cudaFree(p);
+  for (double *p : h->d_mass_coo) cudaFree(p);
+  for (double *p : h->d_adv_csr) cudaFree(p);
+  for (double *p : h->d_adv_coo) cudaFree(p);
+  for (int64_t *p : h->d_rowptr) cudaFree(p);
+  for (int32_t *p : h->d_col) cudaFree(p);
+  cudaFree(h->d_Jwork);
+  cudaFree(h->d_rhs);
+  cudaFree(h->d_norms);
+  if (h->h_norms) cudaFreeHost(h->h_norms);
+  for (auto &u : h->ev_used) {
+    cudaEventDestroy(u.second.first);
+    cudaEventDestroy(u.second.second);
+  }
+  for (auto e : h->ev_pool) cudaEventDestroy(e);
+  (void)cudaGetLastError();   // teardown leaves no error behind for the next call
+  delete h;
+  } catch (...) {   // teardown never throws out of the C ABI
+  }
+}
+
+int landau_get_sizes(landau_t h, int64_t *ndof, int64_t *npoints, int64_t *nnz_csr, int64_t *ncoo) {
+  return guarded(h, [&]() -> int {
+  if (!h) return LANDAU_EINVAL;
+  if (ndof) *ndof = h->ndof;
+  if (npoints) *npoints = h->plan.npts;
+  if (nnz_csr) *nnz_csr = h->nnz;
+  if (ncoo) *ncoo = h->ncoo;
+  return LANDAU_OK;
+});
+}
+
+int landau_get_grid_ndof(landau_t h, int32_t grid, int64_t *ndof) {
+  return guarded(h, [&]() -> int {
+  if (!h || !ndof || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
+  *ndof = h->plan.grids[grid].ndof;
+  return LANDAU_OK;
+});
+}
+
+int landau_get_nodes(landau_t h, int32_t grid, double *r, double *z) {
+  return guarded(h, [&]() -> int {
+  if (!h || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
+  const auto &G = h->plan.grids[grid];
+  if (r) memcpy(r, G.node_r.data(), sizeof(double) * G.ndof);
+  if (z) memcpy(z, G.node_z.data(), sizeof(double) * G.ndof);
+  return LANDAU_OK;
+});
+}
+
+int landau_get_points(landau_t h, double *r, double *z, double *w) {
+  return guarded(h, [&]() -> int {
+  if (!h) return LANDAU_EINVAL;
+  const Plan &P = h->plan;
+  if (r) memcpy(r, P.pr.data(), sizeof(double) * P.npts);
+  if (z) memcpy(z, P.pz.data(), sizeof(double) * P.npts);
+  if (w) memcpy(w, P.pw.data(), sizeof(double) * P.npts);
+  return LANDAU_OK;
+});
+}
+
+int landau_get_pattern(landau_t h, int64_t *csr_rowptr, int32_t *csr_col, int32_t *coo_row, int32_t *coo_col) {
+  return guarded(h, [&]() -> int {
+  if (!h) return LANDAU_EINVAL;
+  const Plan &P = h->plan;
+  int64_t row = 0, k = 0, kc = 0;
+  if (csr_rowptr) csr_rowptr[0] = 0;
+  for (int a = 0; a < h->S; a++) {
+    const GridPlan &G = P.grids[h->sgrid[a]];
+    const int64_t off = h->soff[a];
+    for (int i = 0; i < G.ndof; i++, row++) {
+      for (int64_t q = G.rowptr[i]; q < G.rowptr[i + 1]; q++, k++)
+        if (csr_col) csr_col[k] = (int32_t)(off + G.col[q]);
+      if (csr_rowptr) csr_rowptr[row + 1] = k;
+    }
+    for (int64_t c = 0; c < G.ncell; c++) {
+      const int ne = G.ne[c];
+      const int *d = &G.edof[G.edof_off[c]];
+      for (int i = 0; i < ne; i++)
+        for (int j = 0; j < ne; j++, kc++) {
+          if (coo_row) coo_row[kc] = (int32_t)(off + d[i]);
+          if (coo_col) coo_col[kc] = (int32_t)(off + d[j]);
+        }
+    }
+  }
+  return LANDAU_OK;
+});
+}
+
+int landau_set_state_batched(landau_t h, int64_t nbatch, const double *f_dev) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !f_dev) return fail(h, LANDAU_EINVAL, "set_state: bad argument");
+  int rc = ensure_workspace(h, nbatch);
+  if (rc) return rc;
+  CU(cudaMemcpyAsync(h->d_f, f_dev, sizeof(double) * nbatch * h->ndof, cudaMemcpyDeviceToDevice, h->stream));
+  h->nbatch = nbatch;
+  h->have_state = true;
+  return LANDAU_OK;
+});
+}
+
+int landau_set_state(landau_t h, const double *f_dev) {
+  return guarded(h, [&]() -> int { return landau_set_state_batched(h, 1, f_dev); });
+}
+
+int landau_jacobian_batched(landau_t h, int64_t nbatch, double *values_dev, int32_t format) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "jacobian: bad argument");
+  if (!h->have_state || nbatch != h->nbatch) return fail(h, LANDAU_ESTATE, "jacobian: set_state first (batch size must match)");
+  return dispatch_build(h, nbatch, values_dev, format);
+});
+}
+
+int landau_jacobian(landau_t h, double *values_dev, int32_t format) {
+  return guarded(h, [&]() -> int {
+  if (h && h->have_state && h->nbatch != 1) return fail(h, LANDAU_ESTATE, "jacobian: state is batched");
+  return landau_jacobian_batched(h, 1, values_dev, format);
+});
+}
+
+// End-to-end entry: the batch is cut into K chunks; chunk c's upload (stream s_h2d), its build
+// (the handle's stream) and its download (stream s_d2h) are ordered by events, so downloads of
+// finished chunks overlap the builds of later ones.  Chunks are independent vertices, so the
+// values are identical to one whole-batch build up to the split-j / symmetric grouping (the same
+// for every chunk size at or above the symmetric threshold).
+int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, double *values_host, int32_t format) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !f_host || !values_host || (format != LANDAU_CSR && format != LANDAU_COO))
+    return fail(h, LANDAU_EINVAL, "jacobian_host: bad argument");
+  int rc = ensure_workspace(h, nbatch);
+  if (rc) return rc;
+  const int64_t nv = format == LANDAU_CSR ? h->nnz : h->ncoo;
+  if (nbatch * nv > h->vals_tmp_cap) {
+    drop_graphs(h);
+    cudaFree(h->d_vals_tmp);
+    h->d_vals_tmp = nullptr;
+    CU(cudaMalloc(&h->d_vals_tmp, sizeof(double) * nbatch * nv));
+    h->vals_tmp_cap = nbatch * nv;
+  }
+  if (!h->s_h2d) {
+    CU(cudaStreamCreateWithFlags(&h->s_h2d, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&h->s_d2h, cudaStreamNonBlocking));
+  }
+  static const int64_t kmax = [] {
+    const char *e = getenv("LANDAU_HOST_CHUNKS");
+    return e ? (int64_t)atoll(e) : (int64_t)8;   // 16 measured no better
+  }();
+  const int64_t K = std::max<int64_t>(1, std::min<int64_t>(kmax, nbatch / 64));
+  const int64_t cb = (nbatch + K - 1) / K;
+  while ((int64_t)h->ev_h2d.size() < K) {
+    cudaEvent_t a, b;
+    CU(cudaEventCreateWithFlags(&a, cudaEventDisableTiming));
+    CU(cudaEventCreateWithFlags(&b, cudaEventDisableTiming));
+    h->ev_h2d.push_back(a);
+    h->ev_built.push_back(b);
+  }
+  // the copies may only start once earlier work on the handle's stream is done with the buffers
+  CU(cudaEventRecord(h->ev_built[0], h->stream));
+  CU(cudaStreamWaitEvent(h->s_h2d, h->ev_built[0], 0));
+  CU(cudaStreamWaitEvent(h->s_d2h, h->ev_built[0], 0));
+  for (int64_t c = 0; c < K; c++) {
+    const int64_t b0 = c * cb, n = std::min(cb, nbatch - b0);
+    if (n <= 0) break;
+    CU(cudaMemcpyAsync(h->d_f + b0 * h->ndof, f_host + b0 * h->ndof, sizeof(double) * n * h->ndof,
+                       cudaMemcpyHostToDevice, h->s_h2d));
+    CU(cudaEventRecord(h->ev_h2d[c], h->s_h2d));
+    CU(cudaStreamWaitEvent(h->stream, h->ev_h2d[c], 0));
+    h->fin = h->d_f + b0 * h->ndof;
+    rc = dispatch_build(h, n, h->d_vals_tmp + b0 * nv, format);
+    h->fin = nullptr;
+    if (rc) return rc;
+    CU(cudaEventRecord(h->ev_built[c], h->stream));
+    CU(cudaStreamWaitEvent(h->s_d2h, h->ev_built[c], 0));
+    CU(cudaMemcpyAsync(values_host + b0 * nv, h->d_vals_tmp + b0 * nv, sizeof(double) * n * nv,
+                       cudaMemcpyDeviceToHost, h->s_d2h));
+  }
+  h->nbatch = cb;          // the device state now holds the last chunk's batch layout
+  h->have_state = false;   // (d_f holds the whole host batch, but not as one set_state)
+  CU(cudaStreamSynchronize(h->s_d2h));
+  CU(cudaStreamSynchronize(h->stream));
+  return LANDAU_OK;
+});
+}
+
+int landau_mass(landau_t h, double shift, double *values_dev, int32_t format) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "mass: bad argument");
+  Timer t(h, LANDAU_T_MASS);
+  ScaleCopyDesc d{};
+  int64_t nmax = 0;
+  for (int a = 0; a < h->S; a++) {   // every species block in one launch
+    const int g = h->sgrid[a];
+    d.M[a] = format == LANDAU_CSR ? h->d_mass_csr[g] : h->d_mass_coo[g];
+    d.n[a] = format == LANDAU_CSR ? (int64_t)h->plan.grids[g].col.size() : h->plan.grids[g].ncoo;
+    d.off[a] = format == LANDAU_CSR ? h->snnz_off[a] : h->scoo_off[a];
+    d.scale[a] = shift;
+    nmax = std::max(nmax, d.n[a]);
+  }
+  if (nmax == 0) return LANDAU_OK;
+  const int blocks = (int)std::min<int64_t>((nmax + 255) / 256, 8LL * num_sms(h));
+  scale_copy_species_kernel<<<dim3(blocks, h->S), 256, 0, h->stream>>>(d, values_dev);
+  h->launches++;
+  h->tlaunch[LANDAU_T_MASS]++;
+  KCHECK();
+  return LANDAU_OK;
+});
+}
+
+int landau_advection(landau_t h, double Ez, double *values_dev, int32_t format) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "advection: bad argument");
+  Timer t(h, LANDAU_T_MASS);
+  for (int a = 0; a < h->S; a++) {
+    const int g = h->sgrid[a];
+    const double *A = format == LANDAU_CSR ? h->d_adv_csr[g] : h->d_adv_coo[g];
+    const int64_t n = format == LANDAU_CSR ? (int64_t)h->plan.grids[g].col.size() : h->plan.grids[g].ncoo;
+    const int64_t off = format == LANDAU_CSR ? h->snnz_off[a] : h->scoo_off[a];
+    if (n == 0) continue;
+    const int blocks = (int)std::min<int64_t>((n + 255) / 256, 8LL * num_sms(h));
+    scale_copy_kernel<<<blocks, 256, 0, h->stream>>>(A, Ez * h->charge[a] / h->mass[a], n, values_dev + off);
+    h->launches++;
+    h->tlaunch[LANDAU_T_MASS]++;
+    KCHECK();
+  }
+  return LANDAU_OK;
+});
+}
+
+int landau_point_coeffs_batched(landau_t h, int64_t nbatch, double *G_dev) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || !G_dev) return fail(h, LANDAU_EINVAL, "point_coeffs: bad argument");
+  if (!h->have_state || nbatch != h->nbatch) return fail(h, LANDAU_ESTATE, "point_coeffs: set_state first");
+  int rc = dispatch_build(h, nbatch, nullptr, LANDAU_CSR);
+  if (rc) return rc;
+  const int64_t N = h->plan.npts;
+  if (h->Nc == N) {
+    CU(cudaMemcpyAsync(G_dev, h->d_G, sizeof(double) * nbatch * 5 * N, cudaMemcpyDeviceToDevice, h->stream));
+  } else {
+    const int64_t total = nbatch * 5 * N;
+    unchunk_kernel<<<(int)std::min<int64_t>((total + 255) / 256, 4096), 256, 0, h->stream>>>(h->d_G, N, h->Nc, (int)nbatch, G_dev);
+    h->launches++;
+    KCHECK();
+  }
+  return LANDAU_OK;
+});
+}
+
+int landau_point_coeffs(landau_t h, double *G_dev) {
+  return guarded(h, [&]() -> int { return landau_point_coeffs_batched(h, 1, G_dev); });
+}
+
+int landau_set_timing(landau_t h, int32_t enable) {
+  return guarded(h, [&]() -> int {
+  if (!h) return LANDAU_EINVAL;
+  for (auto &u : h->ev_used) {
+    h->ev_pool.push_back(u.second.first);
+    h->ev_pool.push_back(u.second.second);
+  }
+  h->ev_used.clear();
+  for (auto &x : h->tlaunch) x = 0;
+  h->timing = enable != 0;
+  return LANDAU_OK;
+});
+}
+
+int landau_get_timing(landau_t h, double *ms, int64_t *launches) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h) return LANDAU_EINVAL;
+  CU(cudaStreamSynchronize(h->stream));
+  double acc[LANDAU_NTIMERS] = {0};
+  for (auto &u : h->ev_used) {
+    float t = 0;
+    CU(cudaEventElapsedTime(&t, u.second.first, u.second.second));
+    acc[u.first] += t;
+  }
+  for (int i = 0; i < LANDAU_NTIMERS; i++) {
+    if (ms) ms[i] = acc[i];
+    if (launches) launches[i] = h->tlaunch[i];
+  }
+  return LANDAU_OK;
+});
+}
+
+int landau_set_mirror(landau_t h, int32_t enable) {
+  return guarded(h, [&]() -> int {
+  if (!h) return LANDAU_EINVAL;
+  if (enable < 0 || enable > 3) return fail(h, LANDAU_EINVAL, "set_mirror: mode must be 0..3");
+  if (enable && !h->mirror) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: the mesh is not mirror-symmetric");
+  if (enable == 3 && !h->vtx_smem) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: a vertex does not fit shared memory");
+  if (h->dist_pairs && enable != 1 && enable != 2)
+    return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: the pair split runs the mirror slot kernel");
+  if (!h->host_only) drop_graphs(h);
+  h->mirror_on = enable != 0;
+  h->mirror_mode = enable ? enable : 1;
+  return LANDAU_OK;
+});
+}
+
+int landau_set_tensor_cache(landau_t h, int32_t enable) {
+  return guarded(h, [&]() -> int {
+  if (!h) return LANDAU_EINVAL;
+  if (h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!enable) {
+    drop_graphs(h);
+    CU(cudaStreamSynchronize(h->stream));
+    cudaFree(h->d_U);
+    h->d_U = nullptr;
+    h->tcache = h->tcache_valid = false;
+    return LANDAU_OK;
+  }
+  if (h->tcache) {
+    if (h->tcache_recompute != (enable == 2)) drop_graphs(h);
+    h->tcache_recompute = enable == 2;
+    return LANDAU_OK;
+  }
+  const int64_t N = h->plan.npts;
+  if (h->world > 1 || h->Nc != N) return fail(h, LANDAU_EUNSUPPORTED, "tensor cache needs all targets on one GPU");
+  if (7 * N * N * (int64_t)sizeof(double) > (16LL << 30)) return fail(h, LANDAU_EUNSUPPORTED, "tensor cache > 16 GiB");
+  if (N > INT32_MAX / 5) return fail(h, LANDAU_EUNSUPPORTED, "mesh too large for the GEMM path");
+  if (!load_cublas()) return fail(h, LANDAU_EUNSUPPORTED, "cannot load libcublas.so.12");
+  if (!h->cublas) {
+    if (g_cublas.Create(&h->cublas)) return fail(h, LANDAU_ECUDA, "cublasCreate failed");
+    if (g_cublas.SetStream(h->cublas, h->stream)) return fail(h, LANDAU_ECUDA, "cublasSetStream failed");
+  }
+  CU(cudaMalloc(&h->d_U, sizeof(double) * 7 * N * N));
+  drop_graphs(h);
+  h->tcache = true;
+  h->tcache_valid = false;
+  h->tcache_recompute = enable == 2;
+  return LANDAU_OK;
+});
+}
+
+int landau_band_info(landau_t h, int32_t grid, int32_t *bandwidth, int32_t *perm) {
+  return guarded(h, [&]() -> int {
+  if (!h || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
+  const GridPlan &G = h->plan.grids[grid];
+  if (bandwidth) *bandwidth = G.band;
+  if (perm) memcpy(perm, G.rcm_perm.data(), sizeof(int32_t) * G.ndof);
+  return LANDAU_OK;
+});
+}
+
+int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const double *J_csr_dev) {
+  return guarded(h, [&]() -> int {
+  return landau_band_factor_field_batched(h, nbatch, shift, 0.0, J_csr_dev);
+});
+}
+
+int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, double Ez, const double *J_csr_dev) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !J_csr_dev) return fail(h, LANDAU_EINVAL, "band_factor: bad argument");
+  int maxPp = 8, maxn = 0, maxent = 0;
+  for (auto &d : h->band_desc) {
+    maxPp = std::max(maxPp, d.Pp);
+    maxn = std::max(maxn, d.n);
+    maxent = std::max(maxent, d.nent);
+  }
+  // one CTA per matrix with the active window in registers: vertex-grid sizes (C1-C4); a single large
+  // grid (C5) would need a multi-CTA factorisation (not built)
+  if (maxPp > kBandMaxP) return fail(h, LANDAU_EUNSUPPORTED, "band factor: half-bandwidth above 127");
+  // band_lu2_kernel's shared memory: pivot rows/columns (double-buffered, padded), 3 x 8 dense
+  // entering rows of 4P, the entry lists
+  const size_t smem = sizeof(double) * (2 * (2 * maxPp + 2 * (maxPp / 8 * 10) + 8) + 24 * 4 * maxPp) +
+                      sizeof(int32_t) * (maxn + 1) + sizeof(uint16_t) * maxent;
+  if (smem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
+  if (nbatch > h->band_cap) {
+    cudaFree(h->d_band);
+    cudaFree(h->d_Aent);
+    h->d_band = h->d_Aent = nullptr;
+    CU(cudaMalloc(&h->d_band, sizeof(double) * nbatch * h->band_bstride));
+    CU(cudaMalloc(&h->d_Aent, sizeof(double) * nbatch * std::max<int64_t>(h->ent_bstride, 1)));
+    h->band_cap = nbatch;
+  }
+  Timer t(h, LANDAU_T_FACTOR);
+  for (int a = 0; a < h->S; a++) {
+    const int g = h->sgrid[a];
+    const int64_t nent = h->band_desc[a].nent;
+    if (!nent) continue;
+    const int blocks = (int)std::min<int64_t>((nent * nbatch + 255) / 256, 16LL * num_sms(h));
+    band_gather_kernel<<<blocks, 256, 0, h->stream>>>(nent, h->d_ent_slot[g], h->d_mass_csr[g], h->d_adv_csr[g],
+                                                      Ez * h->charge[a] / h->mass[a], J_csr_dev, h->nnz,
+                                                      h->snnz_off[a], shift, h->d_Aent, h->ent_bstride,
+                                                      h->band_desc[a].aoff, (int)nbatch);
+    h->launches++;
+    KCHECK();
+  }
+  const int threads_lu = std::max(64, (std::max((maxPp / (maxPp <= 88 ? 4 : 8)) * (maxPp / 8), 2 * maxPp - 1) + 31) / 32 * 32);
+  if (h->band_ent_max > kBandE * threads_lu) return fail(h, LANDAU_EUNSUPPORTED, "band factor: too many entries per row group");
+  const unsigned grid = (unsigned)(nbatch * h->S);
+  static const int band_minb = [] {
+    const char *e = getenv("LANDAU_BAND_MINB");
+    return e ? atoi(e) : 2;
+  }();
+  const void *kfn;
+  const size_t ksmem = smem;
+  if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
+    kfn = band_minb >= 2 ? (const void *)band_lu2_kernel<4, 8, 2> : (const void *)band_lu2_kernel<4, 8, 1>;
+  else               // 8 x 8 tiles, <= 256 threads
+    kfn = (const void *)band_lu2_kernel<8, 8, 1>;
+  if (ksmem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
+  if (ksmem > 48 * 1024) CU(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ksmem));
+  {
+    const double *a0 = h->d_Aent;
+    int64_t a1 = h->ent_bstride;
+    double *a2 = h->d_band;
+    int64_t a3 = h->band_bstride;
+    const BandDesc *a4 = h->d_band_desc;
+    int a5 = h->S;
+    void *args[] = {&a0, &a1, &a2, &a3, &a4, &a5};
+    CU(cudaLaunchKernel(kfn, dim3(grid), dim3(threads_lu), args, ksmem, h->stream));
+  }
+  h->launches++;
+  h->tlaunch[LANDAU_T_FACTOR]++;
+  KCHECK();
+  h->band_nbatch = nbatch;
+  return LANDAU_OK;
+});
+}
+
+int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !b_dev || !x_dev) return fail(h, LANDAU_EINVAL, "band_solve: bad argument");
+  if (h->band_nbatch != nbatch) return fail(h, LANDAU_ESTATE, "band_solve: factor this batch first");
+  Timer t(h, LANDAU_T_SOLVE);
+  int maxn = 0, maxB = 0;
+  for (auto &d : h->band_desc) maxn = std::max(maxn, d.n), maxB = std::max(maxB, d.B);
+  constexpr int kWarps = 4;
+  const size_t smem = sizeof(double) * kWarps * (maxn + maxB + 1 + (kBandD + 1) * (maxB + 1));
+  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(band_solve_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int64_t warps = nbatch * h->S;
+  band_solve_kernel<<<(unsigned)((warps + kWarps - 1) / kWarps), 32 * kWarps, smem, h->stream>>>(
+      h->d_band, h->band_bstride, h->d_band_desc, h->d_perm_all, h->d_perm_off, h->d_vec_off, h->ndof, maxn, maxB,
+      b_dev, x_dev, h->S, (int)nbatch);
+  h->launches++;
+  h->tlaunch[LANDAU_T_SOLVE]++;
+  KCHECK();
+  return LANDAU_OK;
+});
+}
+
+int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
+                                 double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm) {
+  return guarded(h, [&]() -> int {
+  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+  if (!h || nbatch < 1 || !f_old_dev || !f_new_dev || f_old_dev == f_new_dev || max_iter < 1 || !(dt > 0))
+    return fail(h, LANDAU_EINVAL, "implicit_step: bad argument");
+  if (nbatch > h->step_cap) {
+    cudaFree(h->d_Jwork);
+    cudaFree(h->d_rhs);
+    cudaFree(h->d_norms);
+    if (h->h_norms) cudaFreeHost(h->h_norms);
+    h->d_Jwork = h->d_rhs = h->d_norms = h->h_norms = nullptr;
+    CU(cudaMalloc(&h->d_Jwork, sizeof(double) * nbatch * std::max<int64_t>(h->nnz, 1)));
+    CU(cudaMalloc(&h->d_rhs, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
+    CU(cudaMalloc(&h->d_norms, sizeof(double) * 2 * nbatch));
+    CU(cudaMallocHost(&h->h_norms, sizeof(double) * 2 * nbatch));
+    h->step_cap = nbatch;
+  }
+  // rhs = M f_old / dt (species blocks), initial iterate f_old
+  for (int a = 0; a < h->S; a++) {
+    const int g = h->sgrid[a];
+    const int n = h->plan.grids[g].ndof;
+    if (!n) continue;
+    const int64_t warps = nbatch * n;
+    block_spmv_kernel<<<(unsigned)((warps * 32 + 255) / 256), 256, 0, h->stream>>>(
+        h->d_rowptr[g], h->d_col[g], h->d_mass_csr[g], n, h->soff[a], h->ndof, 1.0 / dt, f_old_dev, h->d_rhs,
+        (int)nbatch);
+    h->launches++;
+    KCHECK();
+  }
+  CU(cudaMemcpyAsync(f_new_dev, f_old_dev, sizeof(double) * nbatch * h->ndof, cudaMemcpyDeviceToDevice, h->stream));
+  int it = 0;
+  double worst = 0.0;
+  for (it = 1; it <= max_iter; it++) {
+    // quasi-Newton iteration (@10500-10978): J about the current iterate, then
+    // (M/dt + E_z (e/m) A_E - J(f^k)) f^{k+1} = M f_old / dt  by the band LU
+    int rc = landau_set_state_batched(h, nbatch, f_new_dev);
+    if (!rc) rc = dispatch_build(h, nbatch, h->d_Jwork, LANDAU_CSR);
+    if (!rc) rc = landau_band_factor_field_batched(h, nbatch, 1.0 / dt, Ez, h->d_Jwork);
+    if (!rc) rc = landau_band_solve_batched(h, nbatch, h->d_rhs, f_new_dev);
+    if (rc) return rc;
+    delta_norm_kernel<<<(unsigned)nbatch, 256, 0, h->stream>>>(f_new_dev, h->d_f, h->ndof, h->d_norms);
+    h->launches++;
+    KCHECK();
+    if (rtol > 0 || it == max_iter) {
+      CU(cudaMemcpyAsync(h->h_norms, h->d_norms, sizeof(double) * 2 * nbatch, cudaMemcpyDeviceToHost, h->stream));
+      CU(cudaStreamSynchronize(h->stream));
+      worst = 0.0;
+      for (int64_t b = 0; b < nbatch; b++)
+        worst = std::max(worst, std::sqrt(h->h_norms[2 * b] / std::max(h->h_norms[2 * b + 1], 1e-300)));
+      if (rtol > 0 && worst <= rtol) break;
+    }
+  }
+  if (iters) *iters = std::min(it, (int)max_iter);
+  if (dnorm) *dnorm = worst;
+  return LANDAU_OK;
+});
+}
+
+int landau_get_vtx_schedule(landau_t h, int32_t *nrounds, int32_t *weight_prefix, int32_t *ctas) {
+  return guarded(h, [&]() -> int {
+  if (!h) return LANDAU_EINVAL;
+  if (!h->vtx_smem) return fail(h, LANDAU_EUNSUPPORTED, "vtx schedule: the per-vertex kernel is not available");
+  if (nrounds) *nrounds = h->nvtx_rounds;
+  if (weight_prefix) {
+    if (h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
+    CU(cudaMemcpy(weight_prefix, h->d_vtx_wp, sizeof(int32_t) * (h->nvtx_rounds + 1), cudaMemcpyDeviceToHost));
+  }
+  if (ctas) *ctas = h->host_only ? 0 : num_sms(h) * kVtxMinB;
+  return LANDAU_OK;
+});
+}
+
+int landau_get_mirror(landau_t h, int32_t *mirror_symmetric, int32_t *mirror_active) {
+  return guarded(h, [&]() -> int {
+  if (!h) return LANDAU_EINVAL;
+  if (mirror_symmetric) *mirror_symmetric = h->mirror_sym ? 1 : 0;
+  if (mirror_active) *mirror_active = (h->mirror && h->mirror_on) ? 1 : 0;
+  return LANDAU_OK;
+});
+}
+
+int landau_get_stats(landau_t h, landau_stats_t *stats) {
+  return guarded(h, [&]() -> int {
+  if (!h || !stats) return LANDAU_EINVAL;
+  *stats = h->stats;
+  return LANDAU_OK;
+});
+}
+
+int landau_get_launch_count(landau_t h, int64_t *count) {
+  return guarded(h, [&]() -> int {
+  if (!h || !count) return LANDAU_EINVAL;
+  *count = h->launches;
+  return LANDAU_OK;
+});
+}
+
+}  // extern "C"
+
+static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, const landau_params_t *prm, int32_t cuda_device,
+                void *cuda_stream, const landau_dist_t *dist) {
   if (!out || !mesh || !prm) return fail(h, LANDAU_EINVAL, "null argument");
   *out = nullptr;
   if (mesh->ngrids < 1 || mesh->ngrids > kMaxSpecies || !mesh->ncells || !mesh->cells || !mesh->radius)
@@ -964,6 +1690,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
   std::string msg = build_plan(mesh->ngrids, mesh->ncells, mesh->cells, mesh->radius, prm->order, h->plan);
   if (!msg.empty()) {
     delete h;
+    h = nullptr;
     return fail(nullptr, LANDAU_EINVAL, msg);
   }
   const Plan &P = h->plan;
@@ -999,6 +1726,7 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
   h->chunk_cells = (P.ncell + world - 1) / world;
   h->Nc = mode == LANDAU_DIST_ELEMENTS ? h->chunk_cells * P.nqp : P.npts;
   int rc;
+  h->mirror_sym = detect_mirror(P, h->mir_pu, h->mir_pm);
   if (cuda_device == LANDAU_HOST_ONLY) {
     h->host_only = true;
     *out = h;
@@ -1009,11 +1737,13 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
   if (ce != cudaSuccess) {
     std::string m = std::string("cudaSetDevice: ") + cudaGetErrorString(ce);
     delete h;
+    h = nullptr;
     return fail(nullptr, LANDAU_ECUDA, m);
   }
   auto bail = [&](int code) {
     std::string m = h->err;
     landau_destroy(h);
+    h = nullptr;
     return fail(nullptr, code, m);
   };
   if ((rc = upload(h, &h->d_r, P.pr)) || (rc = upload(h, &h->d_z, P.pz)) || (rc = upload(h, &h->d_w, P.pw)) ||
@@ -1071,35 +1801,12 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
   // mirror symmetry z -> -z of every grid (inner_mir_kernel); with several ranks (element split) the
   // tile pairs are split over the ranks and the partial G summed by one all-reduce (pair split)
   if ((world == 1 || mode == LANDAU_DIST_ELEMENTS) && mirror_enabled()) {
-    std::vector<int32_t> pu, pm;
+    const std::vector<int32_t> &pu = h->mir_pu, &pm = h->mir_pm;
     std::vector<double> rU, zU;
-    bool ok = true;
-    for (int g = 0; g < P.ngrids && ok; g++) {
-      const GridPlan &G = P.grids[g];
-      std::vector<int64_t> up, lo;
-      for (int64_t i = G.pt0; i < G.pt0 + G.ncell * P.nqp; i++) {
-        if (P.pz[i] > 0) up.push_back(i);
-        else if (P.pz[i] < 0) lo.push_back(i);
-        else ok = false;   // a point on z = 0 would be its own mirror
-      }
-      if (!ok || up.size() != lo.size()) {
-        ok = false;
-        break;
-      }
-      std::sort(up.begin(), up.end(), [&](int64_t a, int64_t b) {
-        return P.pr[a] != P.pr[b] ? P.pr[a] < P.pr[b] : P.pz[a] < P.pz[b];
-      });
-      std::sort(lo.begin(), lo.end(), [&](int64_t a, int64_t b) {
-        return P.pr[a] != P.pr[b] ? P.pr[a] < P.pr[b] : -P.pz[a] < -P.pz[b];
-      });
-      for (size_t k = 0; k < up.size() && ok; k++) {
-        const int64_t a = up[k], b = lo[k];
-        if (P.pr[a] != P.pr[b] || std::fabs(P.pz[a] + P.pz[b]) > 1e-12 * G.R) ok = false;
-        pu.push_back((int32_t)a);
-        pm.push_back((int32_t)b);
-        rU.push_back(P.pr[a]);
-        zU.push_back(P.pz[a]);   // the mirror sits at exactly (r, -z) for the inner integral
-      }
+    const bool ok = h->mirror_sym;
+    for (size_t k = 0; k < pu.size(); k++) {
+      rU.push_back(P.pr[pu[k]]);
+      zU.push_back(P.pz[pu[k]]);   // the mirror pm[k] sits at exactly (r, -z) (bit-exact, detect_mirror)
     }
     if (ok && !pu.empty()) {
       const int64_t H = (int64_t)pu.size();
@@ -1195,8 +1902,18 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
       const size_t vsmem = (size_t)10 * T * 32 * sizeof(double);
       h->vtx_smem = world == 1 && vsmem <= (size_t)160 * 1024 && T >= 2 ? vsmem : 0;
       h->nvtx_rounds = (int)vround.size() - 1;
+      // stream-K weights: a round lasts as long as its longest item (pair item 2, diagonal item 1)
+      std::vector<int32_t> vwp(1, 0);
+      for (int rd = 0; rd < h->nvtx_rounds; rd++) {
+        int w = 1;
+        for (int q = vround[rd]; q < vround[rd + 1]; q++) w = std::max(w, vitems[q].a == vitems[q].b ? 1 : 2);
+        vwp.push_back(vwp.back() + w);
+      }
+      h->vtx_Wv = vwp.back();
       if (h->vtx_smem) {
-        if ((rc = upload(h, &h->d_vtx_items, vitems)) || (rc = upload(h, &h->d_vtx_round_ptr, vround))) return bail(rc);
+        if ((rc = upload(h, &h->d_vtx_items, vitems)) || (rc = upload(h, &h->d_vtx_round_ptr, vround)) ||
+            (rc = upload(h, &h->d_vtx_wp, vwp)))
+          return bail(rc);
         if (!h->host_only) {
           cudaError_t e1 = cudaFuncSetAttribute(inner_vtx_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)vsmem);
           cudaError_t e2 = cudaFuncSetAttribute(inner_vtx_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)vsmem);
@@ -1284,527 +2001,3 @@ int landau_create(landau_t *out, const landau_mesh_t *mesh, const landau_params_
   return LANDAU_OK;
 }
 
-void landau_destroy(landau_t h) {
-  if (!h) return;
-  if (h->host_only) {
-    delete h;
-    return;
-  }
-  cudaSetDevice(h->device);
-  if (h->stream) cudaStreamSynchronize(h->stream);
-  drop_graphs(h);
-  if (h->cublas && g_cublas.Destroy) g_cublas.Destroy(h->cublas);
-  cudaFree(h->d_U);
-  for (int32_t *p : h->d_ent_ptr) cudaFree(p);
-  for (int32_t *p : h->d_ent_slot) cudaFree(p);
-  for (uint16_t *p : h->d_ent_pos) cudaFree(p);
-  cudaFree(h->d_Aent);
-  cudaFree(h->d_band_desc);
-  cudaFree(h->d_perm_all);
-  cudaFree(h->d_perm_off);
-  cudaFree(h->d_vec_off);
-  cudaFree(h->d_band);
-  if (h->s_h2d) cudaStreamDestroy(h->s_h2d);
-  if (h->s_d2h) cudaStreamDestroy(h->s_d2h);
-  for (auto e : h->ev_h2d) cudaEventDestroy(e);
-  for (auto e : h->ev_built) cudaEventDestroy(e);
-  if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
-  for (double *p : {h->d_r, h->d_z, h->d_w, h->d_h, h->d_tab, h->d_ext_w, h->d_f, h->d_wT, h->d_part, h->d_G, h->d_C, h->d_vals_tmp})
-    cudaFree(p);
-  cudaFree(h->d_cell_grid);
-  cudaFree(h->d_sym_items);
-  cudaFree(h->d_tile_ptr);
-  cudaFree(h->d_tile_slots);
-  cudaFree(h->d_rU);
-  cudaFree(h->d_zU);
-  cudaFree(h->d_pu);
-  cudaFree(h->d_pm);
-  for (auto &ms : h->mset) {
-    cudaFree(ms.items);
-    cudaFree(ms.tile_ptr);
-    cudaFree(ms.tile_slots);
-  }
-  cudaFree(h->d_vtx_items);
-  cudaFree(h->d_vtx_round_ptr);
-  cudaFree(h->d_ext_ptr);
-  cudaFree(h->d_ext_dof);
-  for (auto *v : {&h->d_csr, &h->d_coo})
-    for (auto &m : *v) {
-      cudaFree(m.ptr);
-      cudaFree(m.idx);
-      cudaFree(m.w);
-    }
-  for (double *p : h->d_mass_csr) cudaFree(p);
-  for (double *p : h->d_mass_coo) cudaFree(p);
-  for (double *p : h->d_adv_csr) cudaFree(p);
-  for (double *p : h->d_adv_coo) cudaFree(p);
-  for (int64_t *p : h->d_rowptr) cudaFree(p);
-  for (int32_t *p : h->d_col) cudaFree(p);
-  cudaFree(h->d_Jwork);
-  cudaFree(h->d_rhs);
-  cudaFree(h->d_norms);
-  if (h->h_norms) cudaFreeHost(h->h_norms);
-  for (auto &u : h->ev_used) {
-    cudaEventDestroy(u.second.first);
-    cudaEventDestroy(u.second.second);
-  }
-  for (auto e : h->ev_pool) cudaEventDestroy(e);
-  (void)cudaGetLastError();   // teardown leaves no error behind for the next call
-  delete h;
-}
-
-int landau_get_sizes(landau_t h, int64_t *ndof, int64_t *npoints, int64_t *nnz_csr, int64_t *ncoo) {
-  if (!h) return LANDAU_EINVAL;
-  if (ndof) *ndof = h->ndof;
-  if (npoints) *npoints = h->plan.npts;
-  if (nnz_csr) *nnz_csr = h->nnz;
-  if (ncoo) *ncoo = h->ncoo;
-  return LANDAU_OK;
-}
-
-int landau_get_grid_ndof(landau_t h, int32_t grid, int64_t *ndof) {
-  if (!h || !ndof || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
-  *ndof = h->plan.grids[grid].ndof;
-  return LANDAU_OK;
-}
-
-int landau_get_nodes(landau_t h, int32_t grid, double *r, double *z) {
-  if (!h || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
-  const auto &G = h->plan.grids[grid];
-  if (r) memcpy(r, G.node_r.data(), sizeof(double) * G.ndof);
-  if (z) memcpy(z, G.node_z.data(), sizeof(double) * G.ndof);
-  return LANDAU_OK;
-}
-
-int landau_get_points(landau_t h, double *r, double *z, double *w) {
-  if (!h) return LANDAU_EINVAL;
-  const Plan &P = h->plan;
-  if (r) memcpy(r, P.pr.data(), sizeof(double) * P.npts);
-  if (z) memcpy(z, P.pz.data(), sizeof(double) * P.npts);
-  if (w) memcpy(w, P.pw.data(), sizeof(double) * P.npts);
-  return LANDAU_OK;
-}
-
-int landau_get_pattern(landau_t h, int64_t *csr_rowptr, int32_t *csr_col, int32_t *coo_row, int32_t *coo_col) {
-  if (!h) return LANDAU_EINVAL;
-  const Plan &P = h->plan;
-  int64_t row = 0, k = 0, kc = 0;
-  if (csr_rowptr) csr_rowptr[0] = 0;
-  for (int a = 0; a < h->S; a++) {
-    const GridPlan &G = P.grids[h->sgrid[a]];
-    const int64_t off = h->soff[a];
-    for (int i = 0; i < G.ndof; i++, row++) {
-      for (int64_t q = G.rowptr[i]; q < G.rowptr[i + 1]; q++, k++)
-        if (csr_col) csr_col[k] = (int32_t)(off + G.col[q]);
-      if (csr_rowptr) csr_rowptr[row + 1] = k;
-    }
-    for (int64_t c = 0; c < G.ncell; c++) {
-      const int ne = G.ne[c];
-      const int *d = &G.edof[G.edof_off[c]];
-      for (int i = 0; i < ne; i++)
-        for (int j = 0; j < ne; j++, kc++) {
-          if (coo_row) coo_row[kc] = (int32_t)(off + d[i]);
-          if (coo_col) coo_col[kc] = (int32_t)(off + d[j]);
-        }
-    }
-  }
-  return LANDAU_OK;
-}
-
-int landau_set_state_batched(landau_t h, int64_t nbatch, const double *f_dev) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || nbatch < 1 || !f_dev) return fail(h, LANDAU_EINVAL, "set_state: bad argument");
-  int rc = ensure_workspace(h, nbatch);
-  if (rc) return rc;
-  CU(cudaMemcpyAsync(h->d_f, f_dev, sizeof(double) * nbatch * h->ndof, cudaMemcpyDeviceToDevice, h->stream));
-  h->nbatch = nbatch;
-  h->have_state = true;
-  return LANDAU_OK;
-}
-
-int landau_set_state(landau_t h, const double *f_dev) { return landau_set_state_batched(h, 1, f_dev); }
-
-int landau_jacobian_batched(landau_t h, int64_t nbatch, double *values_dev, int32_t format) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "jacobian: bad argument");
-  if (!h->have_state || nbatch != h->nbatch) return fail(h, LANDAU_ESTATE, "jacobian: set_state first (batch size must match)");
-  return dispatch_build(h, nbatch, values_dev, format);
-}
-
-int landau_jacobian(landau_t h, double *values_dev, int32_t format) {
-  if (h && h->have_state && h->nbatch != 1) return fail(h, LANDAU_ESTATE, "jacobian: state is batched");
-  return landau_jacobian_batched(h, 1, values_dev, format);
-}
-
-// End-to-end entry: the batch is cut into K chunks; chunk c's upload (stream s_h2d), its build
-// (the handle's stream) and its download (stream s_d2h) are ordered by events, so downloads of
-// finished chunks overlap the builds of later ones.  Chunks are independent vertices, so the
-// values are identical to one whole-batch build up to the split-j / symmetric grouping (the same
-// for every chunk size at or above the symmetric threshold).
-int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, double *values_host, int32_t format) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || nbatch < 1 || !f_host || !values_host || (format != LANDAU_CSR && format != LANDAU_COO))
-    return fail(h, LANDAU_EINVAL, "jacobian_host: bad argument");
-  int rc = ensure_workspace(h, nbatch);
-  if (rc) return rc;
-  const int64_t nv = format == LANDAU_CSR ? h->nnz : h->ncoo;
-  if (nbatch * nv > h->vals_tmp_cap) {
-    drop_graphs(h);
-    cudaFree(h->d_vals_tmp);
-    h->d_vals_tmp = nullptr;
-    CU(cudaMalloc(&h->d_vals_tmp, sizeof(double) * nbatch * nv));
-    h->vals_tmp_cap = nbatch * nv;
-  }
-  if (!h->s_h2d) {
-    CU(cudaStreamCreateWithFlags(&h->s_h2d, cudaStreamNonBlocking));
-    CU(cudaStreamCreateWithFlags(&h->s_d2h, cudaStreamNonBlocking));
-  }
-  static const int64_t kmax = [] {
-    const char *e = getenv("LANDAU_HOST_CHUNKS");
-    return e ? (int64_t)atoll(e) : (int64_t)8;   // 16 measured no better
-  }();
-  const int64_t K = std::max<int64_t>(1, std::min<int64_t>(kmax, nbatch / 64));
-  const int64_t cb = (nbatch + K - 1) / K;
-  while ((int64_t)h->ev_h2d.size() < K) {
-    cudaEvent_t a, b;
-    CU(cudaEventCreateWithFlags(&a, cudaEventDisableTiming));
-    CU(cudaEventCreateWithFlags(&b, cudaEventDisableTiming));
-    h->ev_h2d.push_back(a);
-    h->ev_built.push_back(b);
-  }
-  // the copies may only start once earlier work on the handle's stream is done with the buffers
-  CU(cudaEventRecord(h->ev_built[0], h->stream));
-  CU(cudaStreamWaitEvent(h->s_h2d, h->ev_built[0], 0));
-  CU(cudaStreamWaitEvent(h->s_d2h, h->ev_built[0], 0));
-  for (int64_t c = 0; c < K; c++) {
-    const int64_t b0 = c * cb, n = std::min(cb, nbatch - b0);
-    if (n <= 0) break;
-    CU(cudaMemcpyAsync(h->d_f + b0 * h->ndof, f_host + b0 * h->ndof, sizeof(double) * n * h->ndof,
-                       cudaMemcpyHostToDevice, h->s_h2d));
-    CU(cudaEventRecord(h->ev_h2d[c], h->s_h2d));
-    CU(cudaStreamWaitEvent(h->stream, h->ev_h2d[c], 0));
-    h->fin = h->d_f + b0 * h->ndof;
-    rc = dispatch_build(h, n, h->d_vals_tmp + b0 * nv, format);
-    h->fin = nullptr;
-    if (rc) return rc;
-    CU(cudaEventRecord(h->ev_built[c], h->stream));
-    CU(cudaStreamWaitEvent(h->s_d2h, h->ev_built[c], 0));
-    CU(cudaMemcpyAsync(values_host + b0 * nv, h->d_vals_tmp + b0 * nv, sizeof(double) * n * nv,
-                       cudaMemcpyDeviceToHost, h->s_d2h));
-  }
-  h->nbatch = cb;          // the device state now holds the last chunk's batch layout
-  h->have_state = false;   // (d_f holds the whole host batch, but not as one set_state)
-  CU(cudaStreamSynchronize(h->s_d2h));
-  CU(cudaStreamSynchronize(h->stream));
-  return LANDAU_OK;
-}
-
-int landau_mass(landau_t h, double shift, double *values_dev, int32_t format) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "mass: bad argument");
-  Timer t(h, LANDAU_T_MASS);
-  ScaleCopyDesc d{};
-  int64_t nmax = 0;
-  for (int a = 0; a < h->S; a++) {   // every species block in one launch
-    const int g = h->sgrid[a];
-    d.M[a] = format == LANDAU_CSR ? h->d_mass_csr[g] : h->d_mass_coo[g];
-    d.n[a] = format == LANDAU_CSR ? (int64_t)h->plan.grids[g].col.size() : h->plan.grids[g].ncoo;
-    d.off[a] = format == LANDAU_CSR ? h->snnz_off[a] : h->scoo_off[a];
-    d.scale[a] = shift;
-    nmax = std::max(nmax, d.n[a]);
-  }
-  if (nmax == 0) return LANDAU_OK;
-  const int blocks = (int)std::min<int64_t>((nmax + 255) / 256, 8LL * num_sms(h));
-  scale_copy_species_kernel<<<dim3(blocks, h->S), 256, 0, h->stream>>>(d, values_dev);
-  h->launches++;
-  h->tlaunch[LANDAU_T_MASS]++;
-  KCHECK();
-  return LANDAU_OK;
-}
-
-int landau_advection(landau_t h, double Ez, double *values_dev, int32_t format) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || !values_dev || (format != LANDAU_CSR && format != LANDAU_COO)) return fail(h, LANDAU_EINVAL, "advection: bad argument");
-  Timer t(h, LANDAU_T_MASS);
-  for (int a = 0; a < h->S; a++) {
-    const int g = h->sgrid[a];
-    const double *A = format == LANDAU_CSR ? h->d_adv_csr[g] : h->d_adv_coo[g];
-    const int64_t n = format == LANDAU_CSR ? (int64_t)h->plan.grids[g].col.size() : h->plan.grids[g].ncoo;
-    const int64_t off = format == LANDAU_CSR ? h->snnz_off[a] : h->scoo_off[a];
-    if (n == 0) continue;
-    const int blocks = (int)std::min<int64_t>((n + 255) / 256, 8LL * num_sms(h));
-    scale_copy_kernel<<<blocks, 256, 0, h->stream>>>(A, Ez * h->charge[a] / h->mass[a], n, values_dev + off);
-    h->launches++;
-    h->tlaunch[LANDAU_T_MASS]++;
-    KCHECK();
-  }
-  return LANDAU_OK;
-}
-
-int landau_point_coeffs_batched(landau_t h, int64_t nbatch, double *G_dev) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || !G_dev) return fail(h, LANDAU_EINVAL, "point_coeffs: bad argument");
-  if (!h->have_state || nbatch != h->nbatch) return fail(h, LANDAU_ESTATE, "point_coeffs: set_state first");
-  int rc = dispatch_build(h, nbatch, nullptr, LANDAU_CSR);
-  if (rc) return rc;
-  const int64_t N = h->plan.npts;
-  if (h->Nc == N) {
-    CU(cudaMemcpyAsync(G_dev, h->d_G, sizeof(double) * nbatch * 5 * N, cudaMemcpyDeviceToDevice, h->stream));
-  } else {
-    const int64_t total = nbatch * 5 * N;
-    unchunk_kernel<<<(int)std::min<int64_t>((total + 255) / 256, 4096), 256, 0, h->stream>>>(h->d_G, N, h->Nc, (int)nbatch, G_dev);
-    h->launches++;
-    KCHECK();
-  }
-  return LANDAU_OK;
-}
-
-int landau_point_coeffs(landau_t h, double *G_dev) { return landau_point_coeffs_batched(h, 1, G_dev); }
-
-int landau_set_timing(landau_t h, int32_t enable) {
-  if (!h) return LANDAU_EINVAL;
-  for (auto &u : h->ev_used) {
-    h->ev_pool.push_back(u.second.first);
-    h->ev_pool.push_back(u.second.second);
-  }
-  h->ev_used.clear();
-  for (auto &x : h->tlaunch) x = 0;
-  h->timing = enable != 0;
-  return LANDAU_OK;
-}
-
-int landau_get_timing(landau_t h, double *ms, int64_t *launches) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h) return LANDAU_EINVAL;
-  CU(cudaStreamSynchronize(h->stream));
-  double acc[LANDAU_NTIMERS] = {0};
-  for (auto &u : h->ev_used) {
-    float t = 0;
-    CU(cudaEventElapsedTime(&t, u.second.first, u.second.second));
-    acc[u.first] += t;
-  }
-  for (int i = 0; i < LANDAU_NTIMERS; i++) {
-    if (ms) ms[i] = acc[i];
-    if (launches) launches[i] = h->tlaunch[i];
-  }
-  return LANDAU_OK;
-}
-
-int landau_set_mirror(landau_t h, int32_t enable) {
-  if (!h) return LANDAU_EINVAL;
-  if (enable < 0 || enable > 3) return fail(h, LANDAU_EINVAL, "set_mirror: mode must be 0..3");
-  if (enable && !h->mirror) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: the mesh is not mirror-symmetric");
-  if (enable == 3 && !h->vtx_smem) return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: a vertex does not fit shared memory");
-  if (h->dist_pairs && enable != 1 && enable != 2)
-    return fail(h, LANDAU_EUNSUPPORTED, "set_mirror: the pair split runs the mirror slot kernel");
-  if (!h->host_only) drop_graphs(h);
-  h->mirror_on = enable != 0;
-  h->mirror_mode = enable ? enable : 1;
-  return LANDAU_OK;
-}
-
-int landau_set_tensor_cache(landau_t h, int32_t enable) {
-  if (!h) return LANDAU_EINVAL;
-  if (h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!enable) {
-    drop_graphs(h);
-    CU(cudaStreamSynchronize(h->stream));
-    cudaFree(h->d_U);
-    h->d_U = nullptr;
-    h->tcache = h->tcache_valid = false;
-    return LANDAU_OK;
-  }
-  if (h->tcache) {
-    if (h->tcache_recompute != (enable == 2)) drop_graphs(h);
-    h->tcache_recompute = enable == 2;
-    return LANDAU_OK;
-  }
-  const int64_t N = h->plan.npts;
-  if (h->world > 1 || h->Nc != N) return fail(h, LANDAU_EUNSUPPORTED, "tensor cache needs all targets on one GPU");
-  if (7 * N * N * (int64_t)sizeof(double) > (16LL << 30)) return fail(h, LANDAU_EUNSUPPORTED, "tensor cache > 16 GiB");
-  if (N > INT32_MAX / 5) return fail(h, LANDAU_EUNSUPPORTED, "mesh too large for the GEMM path");
-  if (!load_cublas()) return fail(h, LANDAU_EUNSUPPORTED, "cannot load libcublas.so.12");
-  if (!h->cublas) {
-    if (g_cublas.Create(&h->cublas)) return fail(h, LANDAU_ECUDA, "cublasCreate failed");
-    if (g_cublas.SetStream(h->cublas, h->stream)) return fail(h, LANDAU_ECUDA, "cublasSetStream failed");
-  }
-  CU(cudaMalloc(&h->d_U, sizeof(double) * 7 * N * N));
-  drop_graphs(h);
-  h->tcache = true;
-  h->tcache_valid = false;
-  h->tcache_recompute = enable == 2;
-  return LANDAU_OK;
-}
-
-int landau_band_info(landau_t h, int32_t grid, int32_t *bandwidth, int32_t *perm) {
-  if (!h || grid < 0 || grid >= h->plan.ngrids) return LANDAU_EINVAL;
-  const GridPlan &G = h->plan.grids[grid];
-  if (bandwidth) *bandwidth = G.band;
-  if (perm) memcpy(perm, G.rcm_perm.data(), sizeof(int32_t) * G.ndof);
-  return LANDAU_OK;
-}
-
-int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const double *J_csr_dev) {
-  return landau_band_factor_field_batched(h, nbatch, shift, 0.0, J_csr_dev);
-}
-
-int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, double Ez, const double *J_csr_dev) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || nbatch < 1 || !J_csr_dev) return fail(h, LANDAU_EINVAL, "band_factor: bad argument");
-  int maxPp = 8, maxn = 0, maxent = 0;
-  for (auto &d : h->band_desc) {
-    maxPp = std::max(maxPp, d.Pp);
-    maxn = std::max(maxn, d.n);
-    maxent = std::max(maxent, d.nent);
-  }
-  // one CTA per matrix with the active window in registers: vertex-grid sizes (C1-C4); a single large
-  // grid (C5) would need a multi-CTA factorisation (not built)
-  if (maxPp > kBandMaxP) return fail(h, LANDAU_EUNSUPPORTED, "band factor: half-bandwidth above 127");
-  // band_lu2_kernel's shared memory: pivot rows/columns (double-buffered, padded), 3 x 8 dense
-  // entering rows of 4P, the entry lists
-  const size_t smem = sizeof(double) * (2 * (2 * maxPp + 2 * (maxPp / 8 * 10) + 8) + 24 * 4 * maxPp) +
-                      sizeof(int32_t) * (maxn + 1) + sizeof(uint16_t) * maxent;
-  if (smem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
-  if (nbatch > h->band_cap) {
-    cudaFree(h->d_band);
-    cudaFree(h->d_Aent);
-    h->d_band = h->d_Aent = nullptr;
-    CU(cudaMalloc(&h->d_band, sizeof(double) * nbatch * h->band_bstride));
-    CU(cudaMalloc(&h->d_Aent, sizeof(double) * nbatch * std::max<int64_t>(h->ent_bstride, 1)));
-    h->band_cap = nbatch;
-  }
-  Timer t(h, LANDAU_T_FACTOR);
-  for (int a = 0; a < h->S; a++) {
-    const int g = h->sgrid[a];
-    const int64_t nent = h->band_desc[a].nent;
-    if (!nent) continue;
-    const int blocks = (int)std::min<int64_t>((nent * nbatch + 255) / 256, 16LL * num_sms(h));
-    band_gather_kernel<<<blocks, 256, 0, h->stream>>>(nent, h->d_ent_slot[g], h->d_mass_csr[g], h->d_adv_csr[g],
-                                                      Ez * h->charge[a] / h->mass[a], J_csr_dev, h->nnz,
-                                                      h->snnz_off[a], shift, h->d_Aent, h->ent_bstride,
-                                                      h->band_desc[a].aoff, (int)nbatch);
-    h->launches++;
-    KCHECK();
-  }
-  const int threads_lu = std::max(64, (std::max((maxPp / (maxPp <= 88 ? 4 : 8)) * (maxPp / 8), 2 * maxPp - 1) + 31) / 32 * 32);
-  if (h->band_ent_max > kBandE * threads_lu) return fail(h, LANDAU_EUNSUPPORTED, "band factor: too many entries per row group");
-  const unsigned grid = (unsigned)(nbatch * h->S);
-  static const int band_minb = [] {
-    const char *e = getenv("LANDAU_BAND_MINB");
-    return e ? atoi(e) : 2;
-  }();
-  const void *kfn;
-  const size_t ksmem = smem;
-  if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
-    kfn = band_minb >= 2 ? (const void *)band_lu2_kernel<4, 8, 2> : (const void *)band_lu2_kernel<4, 8, 1>;
-  else               // 8 x 8 tiles, <= 256 threads
-    kfn = (const void *)band_lu2_kernel<8, 8, 1>;
-  if (ksmem > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
-  if (ksmem > 48 * 1024) CU(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ksmem));
-  {
-    const double *a0 = h->d_Aent;
-    int64_t a1 = h->ent_bstride;
-    double *a2 = h->d_band;
-    int64_t a3 = h->band_bstride;
-    const BandDesc *a4 = h->d_band_desc;
-    int a5 = h->S;
-    void *args[] = {&a0, &a1, &a2, &a3, &a4, &a5};
-    CU(cudaLaunchKernel(kfn, dim3(grid), dim3(threads_lu), args, ksmem, h->stream));
-  }
-  h->launches++;
-  h->tlaunch[LANDAU_T_FACTOR]++;
-  KCHECK();
-  h->band_nbatch = nbatch;
-  return LANDAU_OK;
-}
-
-int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || nbatch < 1 || !b_dev || !x_dev) return fail(h, LANDAU_EINVAL, "band_solve: bad argument");
-  if (h->band_nbatch != nbatch) return fail(h, LANDAU_ESTATE, "band_solve: factor this batch first");
-  Timer t(h, LANDAU_T_SOLVE);
-  int maxn = 0, maxB = 0;
-  for (auto &d : h->band_desc) maxn = std::max(maxn, d.n), maxB = std::max(maxB, d.B);
-  constexpr int kWarps = 4;
-  const size_t smem = sizeof(double) * kWarps * (maxn + maxB + 1 + (kBandD + 1) * (maxB + 1));
-  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(band_solve_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  const int64_t warps = nbatch * h->S;
-  band_solve_kernel<<<(unsigned)((warps + kWarps - 1) / kWarps), 32 * kWarps, smem, h->stream>>>(
-      h->d_band, h->band_bstride, h->d_band_desc, h->d_perm_all, h->d_perm_off, h->d_vec_off, h->ndof, maxn, maxB,
-      b_dev, x_dev, h->S, (int)nbatch);
-  h->launches++;
-  h->tlaunch[LANDAU_T_SOLVE]++;
-  KCHECK();
-  return LANDAU_OK;
-}
-
-int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
-                                 double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm) {
-  if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || nbatch < 1 || !f_old_dev || !f_new_dev || f_old_dev == f_new_dev || max_iter < 1 || !(dt > 0))
-    return fail(h, LANDAU_EINVAL, "implicit_step: bad argument");
-  if (nbatch > h->step_cap) {
-    cudaFree(h->d_Jwork);
-    cudaFree(h->d_rhs);
-    cudaFree(h->d_norms);
-    if (h->h_norms) cudaFreeHost(h->h_norms);
-    h->d_Jwork = h->d_rhs = h->d_norms = h->h_norms = nullptr;
-    CU(cudaMalloc(&h->d_Jwork, sizeof(double) * nbatch * std::max<int64_t>(h->nnz, 1)));
-    CU(cudaMalloc(&h->d_rhs, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
-    CU(cudaMalloc(&h->d_norms, sizeof(double) * 2 * nbatch));
-    CU(cudaMallocHost(&h->h_norms, sizeof(double) * 2 * nbatch));
-    h->step_cap = nbatch;
-  }
-  // rhs = M f_old / dt (species blocks), initial iterate f_old
-  for (int a = 0; a < h->S; a++) {
-    const int g = h->sgrid[a];
-    const int n = h->plan.grids[g].ndof;
-    if (!n) continue;
-    const int64_t warps = nbatch * n;
-    block_spmv_kernel<<<(unsigned)((warps * 32 + 255) / 256), 256, 0, h->stream>>>(
-        h->d_rowptr[g], h->d_col[g], h->d_mass_csr[g], n, h->soff[a], h->ndof, 1.0 / dt, f_old_dev, h->d_rhs,
-        (int)nbatch);
-    h->launches++;
-    KCHECK();
-  }
-  CU(cudaMemcpyAsync(f_new_dev, f_old_dev, sizeof(double) * nbatch * h->ndof, cudaMemcpyDeviceToDevice, h->stream));
-  int it = 0;
-  double worst = 0.0;
-  for (it = 1; it <= max_iter; it++) {
-    // quasi-Newton iteration (@10500-10978): J about the current iterate, then
-    // (M/dt + E_z (e/m) A_E - J(f^k)) f^{k+1} = M f_old / dt  by the band LU
-    int rc = landau_set_state_batched(h, nbatch, f_new_dev);
-    if (!rc) rc = dispatch_build(h, nbatch, h->d_Jwork, LANDAU_CSR);
-    if (!rc) rc = landau_band_factor_field_batched(h, nbatch, 1.0 / dt, Ez, h->d_Jwork);
-    if (!rc) rc = landau_band_solve_batched(h, nbatch, h->d_rhs, f_new_dev);
-    if (rc) return rc;
-    delta_norm_kernel<<<(unsigned)nbatch, 256, 0, h->stream>>>(f_new_dev, h->d_f, h->ndof, h->d_norms);
-    h->launches++;
-    KCHECK();
-    if (rtol > 0 || it == max_iter) {
-      CU(cudaMemcpyAsync(h->h_norms, h->d_norms, sizeof(double) * 2 * nbatch, cudaMemcpyDeviceToHost, h->stream));
-      CU(cudaStreamSynchronize(h->stream));
-      worst = 0.0;
-      for (int64_t b = 0; b < nbatch; b++)
-        worst = std::max(worst, std::sqrt(h->h_norms[2 * b] / std::max(h->h_norms[2 * b + 1], 1e-300)));
-      if (rtol > 0 && worst <= rtol) break;
-    }
-  }
-  if (iters) *iters = std::min(it, (int)max_iter);
-  if (dnorm) *dnorm = worst;
-  return LANDAU_OK;
-}
-
-int landau_get_stats(landau_t h, landau_stats_t *stats) {
-  if (!h || !stats) return LANDAU_EINVAL;
-  *stats = h->stats;
-  return LANDAU_OK;
-}
-
-int landau_get_launch_count(landau_t h, int64_t *count) {
-  if (!h || !count) return LANDAU_EINVAL;
-  *count = h->launches;
-  return LANDAU_OK;
-}
-
-}  // extern "C"

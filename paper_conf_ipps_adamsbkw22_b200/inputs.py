@@ -40,6 +40,15 @@ def vth(T: float, m: float) -> float:
 # meshes
 # ----------------------------------------------------------------------------------------------
 
+def dyadic_radius(R: float, bits: int = 36) -> float:
+    """R rounded to `bits` significant binary digits (relative change <= 2^-bits ~ 1.5e-11).
+    Every cell coordinate R * k / 2^L with k < 2^(53 - bits) is then an exact double, so the
+    refinement sums are exact and the mesh is exactly mirror-symmetric under z -> -z in floating
+    point (the library's mirror kernels require bit-exact mirrored points)."""
+    m, e = math.frexp(R)
+    return math.ldexp(round(m * 2.0 ** bits), e - bits)
+
+
 def _roots(R: float):
     return [(0.0, -R, R), (0.0, 0.0, R)]
 
@@ -209,7 +218,7 @@ def coefficients(prob: Problem, nodes_per_grid, with_noise: bool = True) -> np.n
 # ----------------------------------------------------------------------------------------------
 # the five configurations of BASELINE.json (concretised in SURVEY.md §8(d))
 # ----------------------------------------------------------------------------------------------
-R_E = 5.0 * VTH_E            # 5 v_th,e (PAPER.md:1@26988)
+R_E = dyadic_radius(5.0 * VTH_E)   # 5 v_th,e (PAPER.md:1@26988), dyadic-rounded (exact mirror)
 
 
 def config1() -> Problem:
@@ -243,7 +252,7 @@ def config3() -> Problem:
     dens = [1.0, 0.9, 0.01]
     grids = []
     for s in sp:
-        R = 5.0 * vth(1.0, s.mass)
+        R = dyadic_radius(5.0 * vth(1.0, s.mass))
         grids.append((R, origin_chain(R, 3)))
     return Problem("C3", 3, grids, sp, fmix=[[(n, 1.0, 0.0)] for n in dens], seed=20221)
 

@@ -85,6 +85,8 @@ def lib():
             "landau_get_stats": (C.c_int, [vp, C.POINTER(_Stats)]),
             "landau_set_tensor_cache": (C.c_int, [vp, i32]),
             "landau_set_mirror": (C.c_int, [vp, i32]),
+            "landau_get_mirror": (C.c_int, [vp, P32, P32]),
+            "landau_get_vtx_schedule": (C.c_int, [vp, P32, P32, P32]),
             "landau_band_info": (C.c_int, [vp, i32, P32, P32]),
             "landau_band_factor_batched": (C.c_int, [vp, i64, d, vp]),
             "landau_band_solve_batched": (C.c_int, [vp, i64, vp, vp]),
@@ -161,6 +163,16 @@ def _tptr(t, dtype=None):
         raise ValueError("tensor must be contiguous")
     if t.dtype != (dtype or torch.float64):
         raise TypeError(f"expected {dtype or torch.float64}, got {t.dtype}")
+    return C.c_void_p(t.data_ptr())
+
+
+def _host_ptr(t, numel, where):
+    """host pointer of a CPU float64 contiguous torch tensor with exactly `numel` elements."""
+    import torch
+    if t.is_cuda or t.dtype != torch.float64 or not t.is_contiguous():
+        raise TypeError(f"{where}: expected a contiguous float64 CPU tensor")
+    if t.numel() != numel:
+        raise ValueError(f"{where}: expected {numel} elements, got {t.numel()}")
     return C.c_void_p(t.data_ptr())
 
 
@@ -258,41 +270,70 @@ class Landau:
         return rp, col[: self.nnz]
 
     # ---- device calls (torch tensors, float64, on this handle's device) --------------------------
+    def _dev(self, t, numel, where):
+        """Device pointer of a contiguous float64 CUDA tensor on this handle's device holding exactly
+        `numel` elements: the library trusts the sizes it is given, so they are checked here."""
+        if not t.is_cuda or t.device.index != self.device:
+            raise ValueError(f"{where}: tensor must live on cuda:{self.device}")
+        if t.numel() != numel:
+            raise ValueError(f"{where}: expected {numel} elements, got {t.numel()} (shape {tuple(t.shape)})")
+        return _tptr(t)
+
+    def _nvals(self, format):
+        if format not in (LANDAU_CSR, LANDAU_COO):
+            raise ValueError(f"unknown format {format!r}")
+        return self.nnz if format == LANDAU_CSR else self.ncoo
+
+    @staticmethod
+    def _nb(t):
+        return t.shape[0] if t.dim() >= 2 else 1
+
     def set_state(self, f):
-        self._check(lib().landau_set_state(self._h, _tptr(f)), "landau_set_state")
+        self._check(lib().landau_set_state(self._h, self._dev(f, self.ndof, "set_state")), "landau_set_state")
         self.nbatch = 1
 
     def set_state_batched(self, f):
-        nb = f.shape[0]
-        self._check(lib().landau_set_state_batched(self._h, nb, _tptr(f)), "landau_set_state_batched")
+        nb = self._nb(f)
+        self._check(lib().landau_set_state_batched(self._h, nb, self._dev(f, nb * self.ndof, "set_state_batched")),
+                    "landau_set_state_batched")
         self.nbatch = nb
 
     def jacobian(self, values, format=LANDAU_CSR):
-        self._check(lib().landau_jacobian(self._h, _tptr(values), format), "landau_jacobian")
+        self._check(lib().landau_jacobian(self._h, self._dev(values, self._nvals(format), "jacobian"), format),
+                    "landau_jacobian")
         return values
 
     def jacobian_batched(self, values, format=LANDAU_CSR):
-        self._check(lib().landau_jacobian_batched(self._h, values.shape[0], _tptr(values), format),
+        nb = self._nb(values)
+        self._check(lib().landau_jacobian_batched(self._h, nb, self._dev(values, nb * self._nvals(format),
+                                                                         "jacobian_batched"), format),
                     "landau_jacobian_batched")
         return values
 
     def jacobian_host(self, f_host, values_host, format=LANDAU_CSR):
-        """f_host: torch CPU tensor [nbatch, ndof] (pinned for async copies); values_host [nbatch, nnz]."""
-        nb = f_host.shape[0] if f_host.dim() == 2 else 1
-        self._check(lib().landau_jacobian_host(self._h, nb, C.c_void_p(f_host.data_ptr()),
-                                               C.c_void_p(values_host.data_ptr()), format), "landau_jacobian_host")
+        """f_host: CPU float64 tensor [nbatch, ndof] (pin it for asynchronous copies); values_host
+        [nbatch, nnz] (CSR) or [nbatch, ncoo] (COO), CPU float64."""
+        nb = self._nb(f_host)
+        fp = _host_ptr(f_host, nb * self.ndof, "jacobian_host f")
+        vp_ = _host_ptr(values_host, nb * self._nvals(format), "jacobian_host values")
+        self._check(lib().landau_jacobian_host(self._h, nb, fp, vp_, format), "landau_jacobian_host")
         return values_host
 
     def mass(self, shift, values, format=LANDAU_CSR):
-        self._check(lib().landau_mass(self._h, float(shift), _tptr(values), format), "landau_mass")
+        self._check(lib().landau_mass(self._h, float(shift), self._dev(values, self._nvals(format), "mass"), format),
+                    "landau_mass")
         return values
 
     def point_coeffs(self, G):
-        self._check(lib().landau_point_coeffs(self._h, _tptr(G)), "landau_point_coeffs")
+        self._check(lib().landau_point_coeffs(self._h, self._dev(G, 5 * self.npoints, "point_coeffs")),
+                    "landau_point_coeffs")
         return G
 
     def point_coeffs_batched(self, G):
-        self._check(lib().landau_point_coeffs_batched(self._h, G.shape[0], _tptr(G)), "landau_point_coeffs_batched")
+        nb = G.shape[0]
+        self._check(lib().landau_point_coeffs_batched(self._h, nb, self._dev(G, nb * 5 * self.npoints,
+                                                                             "point_coeffs_batched")),
+                    "landau_point_coeffs_batched")
         return G
 
     def set_timing(self, enable=True):
@@ -313,30 +354,35 @@ class Landau:
         return B.value, perm
 
     def band_factor_batched(self, shift, J, Ez=0.0):
-        nb = J.shape[0] if J.dim() == 2 else 1
+        nb = self._nb(J)
+        Jp = self._dev(J, nb * self.nnz, "band_factor_batched")
         if Ez == 0.0:
-            self._check(lib().landau_band_factor_batched(self._h, nb, float(shift), _tptr(J)),
-                        "landau_band_factor_batched")
+            self._check(lib().landau_band_factor_batched(self._h, nb, float(shift), Jp), "landau_band_factor_batched")
         else:
-            self._check(lib().landau_band_factor_field_batched(self._h, nb, float(shift), float(Ez), _tptr(J)),
+            self._check(lib().landau_band_factor_field_batched(self._h, nb, float(shift), float(Ez), Jp),
                         "landau_band_factor_field_batched")
 
     def advection(self, Ez, values, format=LANDAU_CSR):
-        self._check(lib().landau_advection(self._h, float(Ez), _tptr(values), format), "landau_advection")
+        self._check(lib().landau_advection(self._h, float(Ez), self._dev(values, self._nvals(format), "advection"),
+                                           format), "landau_advection")
         return values
 
     def implicit_step_batched(self, dt, f_old, f_new, Ez=0.0, max_iter=4, rtol=0.0):
         """One backward-Euler step by quasi-Newton (include/landau.h); returns (iterations, max rel. change)."""
-        nb = f_old.shape[0] if f_old.dim() == 2 else 1
+        nb = self._nb(f_old)
         it, dn = C.c_int32(), C.c_double()
-        self._check(lib().landau_implicit_step_batched(self._h, nb, float(dt), float(Ez), _tptr(f_old), _tptr(f_new),
+        self._check(lib().landau_implicit_step_batched(self._h, nb, float(dt), float(Ez),
+                                                       self._dev(f_old, nb * self.ndof, "implicit_step f_old"),
+                                                       self._dev(f_new, nb * self.ndof, "implicit_step f_new"),
                                                        int(max_iter), float(rtol), C.byref(it), C.byref(dn)),
                     "landau_implicit_step_batched")
         return it.value, dn.value
 
     def band_solve_batched(self, b, x):
-        nb = b.shape[0] if b.dim() == 2 else 1
-        self._check(lib().landau_band_solve_batched(self._h, nb, _tptr(b), _tptr(x)), "landau_band_solve_batched")
+        nb = self._nb(b)
+        self._check(lib().landau_band_solve_batched(self._h, nb, self._dev(b, nb * self.ndof, "band_solve b"),
+                                                    self._dev(x, nb * self.ndof, "band_solve x")),
+                    "landau_band_solve_batched")
         return x
 
     def set_mirror(self, enable=True):
@@ -346,6 +392,30 @@ class Landau:
         if mode is None:
             raise ValueError(f"set_mirror: unknown mode {enable!r}")
         self._check(lib().landau_set_mirror(self._h, mode), "landau_set_mirror")
+
+    def mirror(self):
+        """(exactly z-mirror-symmetric mesh, mirror kernels in use) -- see landau_get_mirror."""
+        a, b = C.c_int32(), C.c_int32()
+        self._check(lib().landau_get_mirror(self._h, C.byref(a), C.byref(b)), "landau_get_mirror")
+        return bool(a.value), bool(b.value)
+
+    def vtx_schedule(self):
+        """(round weight prefix [nrounds + 1], CTAs of an automatic launch) of the per-vertex kernel."""
+        nr, ct = C.c_int32(), C.c_int32()
+        self._check(lib().landau_get_vtx_schedule(self._h, C.byref(nr), None, None), "landau_get_vtx_schedule")
+        wp = np.zeros(nr.value + 1, dtype=np.int32)
+        self._check(lib().landau_get_vtx_schedule(self._h, None, wp.ctypes.data_as(C.POINTER(C.c_int32)),
+                                                  C.byref(ct)), "landau_get_vtx_schedule")
+        return wp, ct.value
+
+    def vtx_split_vertices(self, nbatch):
+        """Batch items whose rounds an automatic-mode build spreads over more than one CTA."""
+        wp, S = self.vtx_schedule()
+        W = int(wp[-1])
+        v = np.arange(nbatch, dtype=np.int64)
+        first = (v * W + int(wp[0])) * S // (nbatch * W)
+        last = (v * W + int(wp[-2])) * S // (nbatch * W)
+        return np.nonzero(first != last)[0]
 
     def set_tensor_cache(self, enable=True):
         """True: cache the tensors across builds; "recompute": GEMM path, tensors evaluated every build."""

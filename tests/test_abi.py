@@ -158,3 +158,70 @@ def test_argument_errors_without_gpu():
     assert lib.landau3d_inner(-1, None, None, None, None, None) == L.LANDAU_EINVAL
     assert lib.landau3d_inner(5, None, None, None, None, None) == L.LANDAU_EINVAL
     assert lib.landau3d_inner(0, None, None, None, None, None) == L.LANDAU_OK
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "C5"])
+def test_mirror_detection_is_bit_exact(cfg):
+    """Every configuration's mesh is exactly z-mirror-symmetric in floating point (dyadic radius,
+    cell-centre point formula), so the mirror kernels compute at the caller's own points: each point
+    (r, z) has a partner with bit-identical r and z' == -z."""
+    h = _host(inputs.CONFIGS[cfg]())
+    sym, active = h.mirror()
+    assert sym and not active          # host-only handle: detected, no device maps
+    r, z, _ = h.points()
+    pts = set(zip(r.tolist(), z.tolist()))
+    assert all((a, -b) in pts for a, b in zip(r.tolist(), z.tolist()))
+
+
+@pytest.mark.parametrize("shift", [1e-13, -2e-15, 1e-10])
+def test_mirror_detection_refuses_near_symmetric_mesh(shift):
+    """A mesh shifted by a few ulps-to-1e-10 R along z is still a valid quadtree (the cell lattice check
+    has a 1e-6 tolerance) but no longer exactly mirror-symmetric: the mirror kernels must not be used
+    (they would evaluate tensors at (r, -z) instead of the caller's point)."""
+    R = inputs.R_E
+    cells = [(a, b + shift * R, c) for a, b, c in inputs.c2_mesh(R)]
+    prob = inputs.Problem("shifted", 3, [(R, cells)], [inputs.Species("e", 1.0, -1.0, 0)], fmix=[[(1, 1, 0)]])
+    h = _host(prob)
+    assert h.mirror() == (False, False)
+    lib = L.lib()
+    assert lib.landau_set_mirror(h._h, 1) == L.LANDAU_EUNSUPPORTED
+
+
+def test_dyadic_radius_keeps_refinement_exact():
+    """inputs.dyadic_radius: a 36-significant-bit R changes the domain by <= 2^-36 relative and makes
+    every refinement coordinate an exact double (mirror cells satisfy z0' == -(z0 + h) exactly)."""
+    R = inputs.dyadic_radius(5.0 * inputs.VTH_E)
+    assert abs(R / (5.0 * inputs.VTH_E) - 1.0) <= 2.0 ** -36
+    cells = inputs.refine_uniform(inputs.c2_mesh(R), 3)
+    key = set(cells)
+    assert all((a, -(b + c), c) in key for a, b, c in cells)
+
+
+def test_host_allocation_failure_is_enomem(monkeypatch):
+    """The header promises that nothing throws or aborts: a std::bad_alloc inside the host plan
+    (forced by the LANDAU_TEST_FAIL_ALLOC fault-injection hook) comes back as LANDAU_ENOMEM with a
+    message, the process survives, and the next create succeeds."""
+    monkeypatch.setenv("LANDAU_TEST_FAIL_ALLOC", "plan")
+    with pytest.raises(L.LandauError) as ei:
+        _host(inputs.config1())
+    assert ei.value.code == L.LANDAU_ENOMEM
+    assert "bad_alloc" in L.lib().landau_last_error(None).decode()
+    monkeypatch.delenv("LANDAU_TEST_FAIL_ALLOC")
+    assert _host(inputs.config1()).npoints == 72
+
+
+def test_binding_checks_sizes_before_calling():
+    """The binding passes raw pointers, so it checks every tensor first: wrong element count, wrong
+    dtype or a CPU tensor where a device one is expected raise before the library is called."""
+    import torch
+    h = _host(inputs.config1())
+    with pytest.raises(ValueError):
+        h.set_state(torch.zeros(h.ndof))                   # CPU tensor for a device argument
+    with pytest.raises(ValueError):
+        h._dev(torch.zeros(3), h.ndof, "x")
+    with pytest.raises(TypeError):
+        h.jacobian_host(torch.zeros(h.ndof, dtype=torch.float32), torch.zeros(h.nnz, dtype=torch.float64))
+    with pytest.raises(ValueError):
+        h.jacobian_host(torch.zeros((1, h.ndof), dtype=torch.float64), torch.zeros((1, h.nnz - 1), dtype=torch.float64))
+    with pytest.raises(ValueError):
+        h._nvals(7)
