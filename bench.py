@@ -1,23 +1,29 @@
 #!/usr/bin/env python3
-"""Benchmark of the Landau Jacobian hot path on B200 (contract: see DESIGN.md §Measurement).
+"""Benchmark of the Landau Jacobian hot path on B200 (contract: see DESIGN.md §10 Measurement).
 
-Workload (default, BASELINE.json configs[3] built on configs[1]): a batch of 1024 independent
-spatial-vertex velocity grids, each the e + D Q3 AMR C2 grid (68 cells, N = 1,088 points, 601 DOFs
-per species) with its own thermal-quench-shaped f.  The vertices are independent problems, so they are
-sharded over the ranks with no communication: --batch vertices per GPU (default 1024), a job of
---batch x world vertices ("scaling": "weak"); --strong splits a fixed job of --batch vertices instead.
+Headline workload = BASELINE.json configs[3] built on configs[1]: a FIXED job of 1024 independent
+spatial-vertex velocity grids, each the e + D Q3 AMR C2 grid (68 cells, N = 1,088 points, 601 DOFs per
+species) with its own thermal-quench-shaped f, sharded over the ranks with no communication
+(1024/N vertices per GPU, "scaling": "strong" -- the driver's 1/2/4/8-GPU runs measure the
+">= 7x at 8 GPUs" target of north_star directly).  --weak gives every GPU its own --batch vertices.
 
 One step = the whole hot path (SURVEY.md §8(a) a-1 .. a-6) for the local batch:
     landau_set_state_batched -> landau_jacobian_batched (CSR) -> landau_mass (CSR)
 with the inputs already resident in HBM.  L2 (126 MB) is flushed between timed steps by writing a
-256 MiB buffer outside the timed events.  e2e repeats the step through landau_jacobian_host with
-pinned host buffers (H2D of f and D2H of every Jacobian value inside the timed region).
+256 MiB buffer outside the timed events.  ms_per_step is the median of the per-step CUDA-event times
+(max over ranks).  e2e repeats the step through landau_jacobian_host with pinned host buffers (H2D of f
+and D2H of every Jacobian value inside the timed region).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl landau|reference] [--workload C4|C2|C3|C5]
+Sub-lines of the same JSON line: "weak" (N > 1: 1024 vertices per GPU), "configs"
+(C1, C2, C3 single builds with their full-oracle cpu_baseline; C5 = one Q4 mesh of 108,800 points with
+the tile pairs of the mirror kernel split over the N GPUs and one NCCL all-reduce of the partial G per
+build, its roofline, its 32-element / 800-target oracle spot check as cpu_baseline and parity), the
+NEXT-3 Newton iterations and the NEXT-4 variants.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl landau|reference] [--workload C4|C1|C2|C3|C5]
 """
 import argparse
 import json
-import math
 import os
 import statistics
 import subprocess
@@ -32,6 +38,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "Landau Jacobian builds/sec + pair-interactions/sec; FP64 % of peak, 1/2/4/8 B200"
 UNIT = "builds/s"
+TIMERS_IN_LOOP = ("C4", "C5")
 
 
 class StdoutToStderr:
@@ -50,29 +57,31 @@ class StdoutToStderr:
         os.close(self._saved)
 
 
-def parse():
+def parse(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
-    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="landau", choices=["landau", "reference"])
     ap.add_argument("--workload", default="C4", choices=["C4", "C1", "C2", "C3", "C5"])
-    ap.add_argument("--batch", type=int, default=1024, help="C4 vertices per GPU (--strong: in the whole job)")
-    ap.add_argument("--strong", action="store_true", help="C4: split a fixed job of --batch vertices over the GPUs")
+    ap.add_argument("--batch", type=int, default=1024, help="C4 vertices in the whole job (--weak: per GPU)")
+    ap.add_argument("--weak", action="store_true", help="C4: --batch vertices per GPU instead of in the whole job")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-sample", type=int, default=0, help="oracle vertices for cpu_baseline (0 = auto)")
+    ap.add_argument("--no-sublines", action="store_true", help="headline only (no configs/variants/newton)")
+    ap.add_argument("--cpu-sample", type=int, default=16, help="oracle C4 vertices for cpu_baseline")
+    ap.add_argument("--c5-cells", type=int, default=32, help="C5 oracle spot check: seeded-random cells")
     ap.add_argument("--tensor-cache", action="store_true",
                     help="NEXT-4 variant: cached mesh tensors + FP64 GEMM inner integral (not the headline path)")
-    return ap.parse_args()
+    return ap.parse_args(argv)
 
 
 def job_vertices(args, world):
-    """C4 vertices in the whole job: --batch per GPU (weak scaling), or --batch in all (--strong)."""
-    return args.batch if args.strong else args.batch * world
+    """C4 vertices in the whole job: --batch in all (default, strong scaling) or per GPU (--weak)."""
+    return args.batch * world if args.weak else args.batch
 
 
 def workload(args, world, rank):
-    """(name, problem for the mesh, list of per-item problems of this rank, pairs per build)."""
+    """(description, problem for the mesh, list of per-item problems of this rank)."""
     from paper_conf_ipps_adamsbkw22_b200 import inputs
     if args.workload == "C4":
         B = job_vertices(args, world)
@@ -86,23 +95,29 @@ def workload(args, world, rank):
     p = inputs.CONFIGS[args.workload]()
     desc = {"workload": f"{args.workload} single build", "points": p.npoints, "order": p.order,
             "species": len(p.species), "l2": "flushed between timed steps (256 MiB write)"}
-    return desc, p, [p] if rank == 0 or world == 1 else []
+    return desc, p, [p] if rank == 0 or world == 1 or args.workload == "C5" else []
 
 
 class Clocks:
-    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    """SM clock and clock-event reasons sampled in-process through NVML every 5 ms (nvidia-smi when NVML
+    is unavailable) during the timed region (B200_PROFILING.md clocks line).  __enter__ returns only
+    after the first sample is taken; mark_start/mark_end bracket the timed region and summary() keeps
+    the samples inside it (all samples if the region saw none)."""
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
 
+    # NVML clock-event reason bits (nvml.h nvmlClocksEventReason*)
+    NVML_BITS = {"sw_power_cap": 0x4, "hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40}
+
     def __init__(self, index):
         self.index = index
         self.rows = []
+        self.times = []
+        self.t0 = self.t1 = None
         self._stop = threading.Event()
+        self._ready = threading.Event()
         self._t = None
-
-    # NVML clock-event reason bits (nvml.h nvmlClocksEventReason*)
-    NVML_BITS = {"sw_power_cap": 0x4, "hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40}
 
     def _nvml_handle(self):
         import pynvml
@@ -114,56 +129,70 @@ class Clocks:
             idx = int(parts[idx])
         return pynvml, pynvml.nvmlDeviceGetHandleByIndex(idx)
 
+    def _add(self, row):
+        self.rows.append(row)
+        self.times.append(time.perf_counter())
+        self._ready.set()
+
     def _run(self):
-        # In-process NVML sampling every 5 ms, so that a timed region of a few tens of ms still gets
-        # several samples; nvidia-smi (one process per sample, ~50 ms) only when NVML is unavailable.
         try:
             nv, h = self._nvml_handle()
             reasons_fn = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
                 nv.nvmlDeviceGetCurrentClocksThrottleReasons
             mx = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+            self.source = "nvml"
             while True:
                 sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
                 bits = reasons_fn(h)
-                self.rows.append([str(self.index), str(sm), str(mx), "", hex(bits)] +
-                                 ["Active" if bits & self.NVML_BITS[k] else "Not Active"
-                                  for k in ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown",
-                                            "sw_power_cap")])
+                self._add([str(self.index), str(sm), str(mx), "", hex(bits)] +
+                          ["Active" if bits & self.NVML_BITS[k] else "Not Active"
+                           for k in ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")])
                 if self._stop.wait(0.005):
-                    break
-            self.source = "nvml"
-            return
+                    return
         except Exception:
-            self.rows = []
+            self.rows, self.times = [], []
         self.source = "nvidia-smi"
         while not self._stop.is_set():
             try:
                 out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
                                       "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5).stdout
                 for line in out.strip().splitlines():
-                    self.rows.append([x.strip() for x in line.split(",")])
+                    self._add([x.strip() for x in line.split(",")])
             except Exception:
                 pass
+            self._ready.set()
             self._stop.wait(0.2)
 
     def __enter__(self):
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
+        self._ready.wait(timeout=15)   # the first sample exists before the timed region starts
         return self
+
+    def mark_start(self):
+        self.t0 = time.perf_counter()
+
+    def mark_end(self):
+        self.t1 = time.perf_counter()
+        time.sleep(0.006)               # one more sample at the region's end
 
     def __exit__(self, *a):
         self._stop.set()
         self._t.join(timeout=10)
 
     def summary(self):
-        if not self.rows:
+        rows = self.rows
+        if self.t0 is not None and self.t1 is not None and self.times:
+            inside = [r for r, t in zip(self.rows, self.times) if self.t0 - 0.006 <= t <= self.t1 + 0.006]
+            rows = inside or self.rows
+        if not rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
-        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[k] for r in self.rows for k in range(4) if len(r) > 5 + k and r[5 + k] == "Active"})
+        reasons = sorted({names[k] for r in rows for k in range(4) if len(r) > 5 + k and r[5 + k] == "Active"})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows), "source": getattr(self, "source", "nvidia-smi")}
+                "reasons": reasons, "samples": len(rows), "source": getattr(self, "source", "nvidia-smi")}
 
 
 def fp64_peak_tflops(props, sm_max_mhz):
@@ -172,62 +201,105 @@ def fp64_peak_tflops(props, sm_max_mhz):
     return props.multi_processor_count * 64 * 2 * sm_max_mhz * 1e6 / 1e12
 
 
-def load_profile_traffic(workload):
-    path = os.path.join(ROOT, "profiles", "inner_traffic.json")
+def load_profile_traffic(key):
     try:
-        d = json.load(open(path))
-        return d.get(workload)
+        return json.load(open(os.path.join(ROOT, "profiles", "inner_traffic.json"))).get(key)
     except Exception:
         return None
 
 
 # FP64 FLOP (2*DFMA + DMUL + DADD) per pair evaluation, counted once from ncu
 # sm__sass_thread_inst_executed_op_{dfma,dmul,dadd}_pred_on of each inner kernel on the C4 workload
-# (profiles/r01_inner_ncu.txt):
-#   directed kernel:  173 FLOP per ordered (target, source) pair, N^2 per batch item
-#   symmetric kernel: 189 FLOP per unordered pair, N (N - 1) / 2 per batch item (both targets updated)
-FLOP_PER_PAIR_DIRECTED = 173.0
-FLOP_PER_PAIR_SYMMETRIC = 189.2
-# mirror-symmetric kernel: FP64 FLOP (2 DFMA + DMUL + DADD, ncu SASS counts on C4) per tensor
-# evaluation, (N/2)^2 evaluations per batch item (profiles/r01_flops_mirror.csv)
-FLOP_PER_EVAL_MIRROR = 194.7   # inner_mir_kernel (slot kernel; profiles/r01_flops_mirror.csv)
-FLOP_PER_EVAL_VTX = 195.0      # inner_vtx_kernel (per-vertex kernel; profiles/r01_flops_vtx.csv)
-FLOP_PER_PAIR_3D = 58.0        # inner3d_kernel, per ordered pair (profiles/r01_flops_3d.csv)
-FLOP_PER_EVAL_MDIR = 183.2     # inner_mdir_kernel (mirror directed, per padded U or V evaluation; profiles/r01_flops_mdir.csv)
+# (profiles/r01_flops_*.csv):
+FLOP_PER_PAIR_DIRECTED = 173.0   # inner_kernel, per ordered (target, source) pair
+FLOP_PER_PAIR_SYMMETRIC = 189.2  # inner_sym_kernel, per unordered pair
+FLOP_PER_EVAL_MIRROR = 194.7     # inner_mir_kernel (slot kernel), per U or V tensor evaluation
+FLOP_PER_EVAL_VTX = 195.0        # inner_vtx_kernel (per-vertex kernel), per U or V tensor evaluation
+FLOP_PER_PAIR_3D = 58.0          # inner3d_kernel, per ordered pair
+FLOP_PER_EVAL_MDIR = 183.2       # inner_mdir_kernel (mirror directed), per padded U or V evaluation
+INNER_PATHS = ["directed (ordered pairs)", "symmetric (unordered pairs)", "tensor cache + FP64 DGEMM (cuBLAS)",
+               "mirror-symmetric slot kernel (one tensor per unordered pair and its z-mirror)",
+               "mirror-symmetric per-vertex kernel (stream-K over vertex rounds, sums in shared memory)",
+               "mirror-symmetric directed (U + V per target and source, forward sums)"]
 
 
-def cpu_baseline(args, desc, nsample):
-    from oracle.oracle import Oracle, get_threads
+def inner_flops(st, N):
+    """(FLOP per evaluation, FLOP per inner launch) from the library's stats of the last build."""
+    p = st["inner_path"]
+    if p == 2:
+        return 14.0, 14.0 * st["nbatch"] * N * N
+    if p == 5:
+        return FLOP_PER_EVAL_MDIR, FLOP_PER_EVAL_MDIR * st["nbatch"] * st["pair_evaluations"]
+    if p in (3, 4):
+        f = FLOP_PER_EVAL_VTX if p == 4 else FLOP_PER_EVAL_MIRROR
+        return f, f * st["nbatch"] * st["pair_evaluations"]
+    if p == 1:
+        return FLOP_PER_PAIR_SYMMETRIC, FLOP_PER_PAIR_SYMMETRIC * st["nbatch"] * N * (N - 1) / 2
+    return FLOP_PER_PAIR_DIRECTED, FLOP_PER_PAIR_DIRECTED * st["nbatch"] * st["targets"] * N
+
+
+def timed_steps(torch, stream, step, steps, flush, clk=None):
+    """Per-step CUDA-event times (ms) on the library's stream, L2 flushed before each step."""
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    torch.cuda.synchronize()
+    if clk:
+        clk.mark_start()
+    for k in range(steps):
+        flush.fill_(float(k))
+        evs[k][0].record(stream)
+        step()
+        evs[k][1].record(stream)
+    torch.cuda.synchronize()
+    if clk:
+        clk.mark_end()
+    return [a.elapsed_time(b) for a, b in evs]
+
+
+def max_over_ranks(torch, dist, world, x):
+    t = torch.tensor([float(x)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def oracle_c4_baseline(B, nsample):
+    """The oracle (full Jacobian incl. its |.| scale) on nsample C4 vertices b = 0, 68, ...,
+    all host cores, plus a 1-core figure on two of them."""
+    from oracle.oracle import Oracle, get_threads, set_threads
     from paper_conf_ipps_adamsbkw22_b200 import inputs
-    B = args.batch
-    if args.workload == "C4":
-        verts = [int(round(k * (B - 1) / max(nsample - 1, 1))) for k in range(nsample)]
-        probs = [inputs.config4_vertex(b, B) for b in verts]
-        sample = f"full oracle Jacobian (incl. |.| scale) of {nsample} of the {B} C4 vertices (b = {verts})"
-    else:
-        probs = [inputs.CONFIGS[args.workload]()]
-        sample = f"full oracle Jacobian of one {args.workload} build"
-    from oracle.oracle import set_threads
+    step = max(1, (B - 1) // max(nsample - 1, 1)) if nsample > 1 else 1
+    verts = [min(B - 1, k * step) for k in range(nsample)]
     t = 0.0
-    for p in probs:
-        o = Oracle(p)
+    for b in verts:
+        o = Oracle(inputs.config4_vertex(b, B))
         f = o.coefficients()
         t0 = time.perf_counter()
         o.jacobian(f)
         t += time.perf_counter() - t0
     cores = get_threads()
-    # the single-core figure of SURVEY §8(d), on the first two vertices of the sample
     set_threads(1)
     t1 = 0.0
-    for p in probs[:2]:
-        o = Oracle(p)
+    for b in verts[:2]:
+        o = Oracle(inputs.config4_vertex(b, B))
         f = o.coefficients()
         t0 = time.perf_counter()
         o.jacobian(f)
         t1 += time.perf_counter() - t0
     set_threads(cores)
-    return {"value": len(probs) / t, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
-            "seconds": t, "value_1core": min(2, len(probs)) / t1}
+    return {"value": len(verts) / t, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"full oracle Jacobian (incl. |.| scale) of {len(verts)} of the {B} C4 vertices (b = {verts})",
+            "seconds": t, "value_1core": min(2, len(verts)) / t1, "omp_num_threads": os.environ.get("OMP_NUM_THREADS"),
+            "nproc": os.cpu_count()}
+
+
+def oracle_full_build(prob):
+    """One full oracle Jacobian (with the |.| scale) of a single-build config: (J, Ja, seconds)."""
+    from oracle.oracle import Oracle
+    o = Oracle(prob)
+    f = o.coefficients()
+    t0 = time.perf_counter()
+    J, Ja = o.jacobian(f)
+    return o, J, Ja, time.perf_counter() - t0
 
 
 def run_reference(args, world, rank):
@@ -240,12 +312,8 @@ def run_reference(args, world, rank):
     desc = dict(desc, parallelism=f"batch-shard x{world}" if world > 1 else "1 GPU")
     B = job_vertices(args, world)
     times = []
-    n_per_step = 1
     for k in range(args.warmup + args.steps):
-        if args.workload == "C4":
-            p = inputs.config4_vertex((k * 97) % B, B)
-        else:
-            p = inputs.CONFIGS[args.workload]()
+        p = inputs.config4_vertex((k * 97) % B, B) if args.workload == "C4" else inputs.CONFIGS[args.workload]()
         o = Oracle(p)
         f = o.coefficients()
         t0 = time.perf_counter()
@@ -253,18 +321,126 @@ def run_reference(args, world, rank):
         dt = time.perf_counter() - t0
         if k >= args.warmup:
             times.append(dt)
-    T = sum(times)
-    value = n_per_step * len(times) / T
+    med = statistics.median(times)
+    value = 1.0 / med
     N = 1088 if args.workload == "C4" else prob0.npoints
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / len(times),
-            "higher_is_better": True, "scaling": "strong" if args.strong else "weak", "vs_baseline": None,
-            "dtype": "f64", "data": "synthetic", "config": desc, "pairs_per_s": value * N * N,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * med,
+            "higher_is_better": True, "scaling": "weak" if args.weak or args.workload != "C4" else "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "config": desc, "pairs_per_s": value * N * N,
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": get_threads(), "kind": "oracle",
-                             "sample": f"1 vertex Jacobian per step ({args.workload}), full oracle"},
+                             "sample": f"1 vertex Jacobian per step ({args.workload}), full oracle incl. |.| scale"},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
+
+
+def single_build_line(torch, L, inputs, name, local, stream, flush, steps, warmup, with_cpu):
+    """One C1/C2/C3 build per step (set_state + jacobian (CSR) + mass, CUDA-graph replay), and the full
+    oracle on the same config as its cpu_baseline."""
+    p = inputs.CONFIGS[name]()
+    h = L.Landau.from_problem(p, device=local, stream=stream)
+    f = torch.tensor(inputs.coefficients(p, h.all_nodes()), device="cuda")
+    v = torch.empty(h.nnz, dtype=torch.float64, device="cuda")
+    m = torch.empty(h.nnz, dtype=torch.float64, device="cuda")
+
+    def step():
+        h.set_state(f)
+        h.jacobian(v)
+        h.mass(1.0e3, m)
+
+    for _ in range(max(warmup, 3)):
+        step()
+    ts = timed_steps(torch, stream, step, steps, flush)
+    ms = statistics.median(ts)
+    st = h.stats()
+    out = {"value": 1e3 / ms, "unit": UNIT, "ms_per_step": ms, "ms_mean": statistics.mean(ts),
+           "points": p.npoints, "pairs_per_s": 1e3 / ms * p.npoints ** 2, "inner_path": INNER_PATHS[st["inner_path"]],
+           "note": f"BASELINE configs ({name}): one build per step, set_state + jacobian (CSR) + mass, CUDA-graph replay"}
+    if with_cpu:
+        o, Jo, Ja, secs = oracle_full_build(p)
+        from oracle.oracle import get_threads
+        Jg = v.cpu().numpy()
+        out["cpu_baseline"] = {"value": 1.0 / secs, "unit": UNIT, "cores": get_threads(), "kind": "oracle",
+                               "sample": f"one full {name} oracle Jacobian (incl. |.| scale)"}
+        out["parity_max_dJ_over_Jabs"] = float(np.max(np.abs(Jg - Jo) / Ja))
+    h.close()
+    return out
+
+
+def c5_line(torch, dist, L, inputs, world, rank, local, stream, flush, steps, warmup, ncheck, with_cpu, peak):
+    """C5: one e+D Q4 mesh (4,352 cells, N = 108,800).  LANDAU_DIST_ELEMENTS over the N ranks: the mirror
+    slot kernel's tile pairs are split (landau_pair_partition), each rank reduces a partial G over all
+    points and one ncclAllReduce sums them (the path's exchange step); element matrices and assembly
+    then run for every cell.  Timed per build (max over ranks), with the all-reduce's own event time,
+    the inner kernel's roofline, and (rank 0, outside the timed region) the oracle on every pair of the
+    points of ncheck seeded-random cells: their COO element blocks against the GPU (parity) and the
+    oracle time as cpu_baseline (SURVEY §8(d) spot check: 32 cells, 800 targets)."""
+    p = inputs.config5()
+    with StdoutToStderr():
+        if world > 1:
+            dd = L.make_dist(L.LANDAU_DIST_ELEMENTS)
+        else:
+            dd = {"rank": 0, "world": 1, "mode": L.LANDAU_DIST_ELEMENTS, "nccl_unique_id": L.landau_nccl_unique_id()}
+        h = L.Landau.from_problem(p, device=local, stream=stream, dist=dd)
+    F = torch.tensor(inputs.coefficients(p, h.all_nodes()), device="cuda")
+    v = torch.empty(h.nnz, dtype=torch.float64, device="cuda")
+    m = torch.empty(h.nnz, dtype=torch.float64, device="cuda")
+
+    def step():
+        h.set_state(F)
+        h.jacobian(v)
+        h.mass(1.0e3, m)
+
+    for _ in range(max(warmup, 2)):
+        step()
+    if world > 1:
+        dist.barrier()
+    h.set_timing(True)
+    ts = timed_steps(torch, stream, step, steps, flush)
+    tim = h.get_timing()
+    h.set_timing(False)
+    st = h.stats()
+    ms = max_over_ranks(torch, dist, world, statistics.median(ts))
+    N = h.npoints
+    fpe, fpl = inner_flops(st, N)
+    inner_s = tim["inner"][0] / max(tim["inner"][1], 1) / 1e3
+    ach = fpl / inner_s / 1e12 if tim["inner"][1] else None
+    out = {"value": 1e3 / ms, "unit": UNIT, "ms_per_step": ms, "points": N, "pairs_per_s": 1e3 / ms * N * N,
+           "parallelism": f"pair split x{world} + ncclAllReduce of G ({5 * N * 8 / 1e6:.2f} MB)" if world > 1
+           else "1 GPU (LANDAU_DIST_ELEMENTS handle at world 1: no exchange)",
+           "inner_path": INNER_PATHS[st["inner_path"]],
+           "stage_ms_per_step": {k: v_[0] / steps for k, v_ in tim.items() if v_[0]},
+           "allreduce_ms_per_step": tim["allgather"][0] / steps if tim["allgather"][1] else 0.0,
+           "roofline": {"bound": "alu", "kernel": "inner_mir_kernel (a-2, this rank's share of the tile pairs)",
+                        "achieved": ach, "peak": peak, "unit": "TFLOP/s", "frac": ach / peak if ach else None,
+                        "flop_per_eval": fpe, "flops_per_launch": fpl, "inner_ms_per_launch": inner_s * 1e3}}
+    if rank == 0 and ncheck > 0:
+        from oracle.oracle import Oracle, get_threads
+        Jc = torch.empty(h.ncoo, dtype=torch.float64, device="cuda")
+        h.jacobian(Jc, L.LANDAU_COO)
+        Jg = Jc.cpu().numpy()
+        o = Oracle(p)
+        ncell = len(p.grids[0][1])
+        cells = np.sort(np.random.default_rng(2022).choice(ncell, ncheck, replace=False))
+        mask = np.zeros(ncell, dtype=np.uint8)
+        mask[cells] = 1
+        t0 = time.perf_counter()
+        Jo, Ja = o.jacobian_coo(o.coefficients(), mask)
+        secs = time.perf_counter() - t0
+        sel = np.isfinite(Jo)
+        targets = ncheck * (p.order + 1) ** 2
+        out["parity"] = {"cells": int(ncheck), "targets": int(targets), "entries": int(sel.sum()),
+                         "max_dJ_over_Jabs": float(np.max(np.abs(Jg[sel] - Jo[sel]) / Ja[sel])),
+                         "bar": 1e-11}
+        if with_cpu:
+            out["cpu_baseline"] = {"value": targets / secs, "unit": "target points/s (all N sources each)",
+                                   "cores": get_threads(), "kind": "oracle",
+                                   "sample": f"oracle element blocks of {ncheck} seeded-random cells ({targets} targets x "
+                                             f"{N} sources, incl. |.| scale)", "seconds": secs,
+                                   "gpu_same_unit": N * 1e3 / ms}
+    h.close()
+    return out
 
 
 def main():
@@ -288,13 +464,9 @@ def main():
     desc, prob0, items = workload(args, world, rank)
     dist_desc = None
     if args.workload == "C5":
-        # one large mesh: the mirror kernel's tile pairs split over the ranks, one NCCL all-reduce of
-        # the partial G per build (the pair split; the element split + all-gather on non-mirror meshes)
-        if world > 1:
-            dist_desc = L.make_dist(L.LANDAU_DIST_ELEMENTS)
-        else:
-            dist_desc = {"rank": 0, "world": 1, "mode": L.LANDAU_DIST_ELEMENTS,
-                         "nccl_unique_id": L.landau_nccl_unique_id()}
+        with StdoutToStderr():
+            dist_desc = L.make_dist(L.LANDAU_DIST_ELEMENTS) if world > 1 else \
+                {"rank": 0, "world": 1, "mode": L.LANDAU_DIST_ELEMENTS, "nccl_unique_id": L.landau_nccl_unique_id()}
         items = [prob0]
         desc = dict(desc, workload="C5: one e+D Q4 mesh (4352 cells, N=108800), LANDAU_DIST_ELEMENTS: the mirror "
                                    "kernel's tile pairs split over the GPUs, NCCL all-reduce of the partial G")
@@ -312,6 +484,7 @@ def main():
     mvals = torch.empty(h.nnz, dtype=torch.float64, device="cuda")
     flush = torch.empty(256 * 1024 * 1024 // 8, dtype=torch.float64, device="cuda")
     shift = 1.0e3
+    props = torch.cuda.get_device_properties(local)
 
     def step():
         if nloc:
@@ -325,20 +498,13 @@ def main():
     if world > 1:
         dist.barrier()
     # Per-stage library timers (CUDA events on the library stream) run inside the timed region for
-    # large batches; small single builds replay as CUDA graphs, so their stage breakdown is taken in
-    # a separate pass right after the timed region.
-    in_loop_timers = args.workload in ("C4", "C5")
+    # the large workloads; small single builds replay as CUDA graphs, so their stage breakdown is taken
+    # in a separate pass right after the timed region.
+    in_loop_timers = args.workload in TIMERS_IN_LOOP
     h.set_timing(in_loop_timers)
     n0 = h.launch_count()
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     with Clocks(local) as clk:
-        torch.cuda.synchronize()
-        for k in range(args.steps):
-            flush.fill_(float(k))
-            evs[k][0].record(stream)
-            step()
-            evs[k][1].record(stream)
-        torch.cuda.synchronize()
+        ts = timed_steps(torch, stream, step, args.steps, flush, clk)
     launches = h.launch_count() - n0
     st = h.stats()   # how the timed builds ran (read before the e2e pass changes the batch layout)
     if not in_loop_timers:
@@ -348,15 +514,13 @@ def main():
             step()
     tim = h.get_timing()
     h.set_timing(False)
-    local_ms = sum(a.elapsed_time(b) for a, b in evs)
-    t = torch.tensor([local_ms], dtype=torch.float64, device="cuda")
+    local_med, local_mean = statistics.median(ts), statistics.mean(ts)
     if world > 1:
         dist.barrier()
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    total_ms = float(t.item())
+    ms_per_step = max_over_ranks(torch, dist, world, local_med)
+    ms_mean = max_over_ranks(torch, dist, world, local_mean)
     total_builds = job_vertices(args, world) if args.workload == "C4" else 1
-    scaling = "strong" if (args.strong or args.workload != "C4") else "weak"
-    ms_per_step = total_ms / args.steps
+    scaling = "weak" if (args.weak or args.workload != "C4") else "strong"
     value = total_builds / (ms_per_step / 1e3)
     pairs_per_build = N * N
 
@@ -366,124 +530,125 @@ def main():
     for _ in range(min(args.warmup, 2)):
         if nloc:
             h.jacobian_host(f_pin, v_pin)
-    e_ms = 0.0
+    ets = []
     for k in range(args.steps):
         flush.fill_(float(k))
+        torch.cuda.synchronize()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         if nloc:
             h.jacobian_host(f_pin, v_pin)
         b.record(stream)
         torch.cuda.synchronize()
-        e_ms += a.elapsed_time(b)
-    et = torch.tensor([e_ms], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(et, op=dist.ReduceOp.MAX)
-    e2e_value = total_builds / (float(et.item()) / args.steps / 1e3)
+        ets.append(a.elapsed_time(b))
+    e_ms = max_over_ranks(torch, dist, world, statistics.median(ets))
+    e2e_value = total_builds / (e_ms / 1e3)
 
     # ---- roofline of the dominant kernel (inner integral, FP64 pipe) --------------------------
     inner_ms, inner_n = tim["inner"]
     inner_avg_s = inner_ms / max(inner_n, 1) / 1e3
-    if st["inner_path"] == 2:   # GEMMs: 2 FLOP per multiply-add, 7 N^2 per batch item (three DGEMMs)
-        flop_per_pair = 14.0
-        flops_per_launch = 14.0 * st["nbatch"] * N * N
-    elif st["inner_path"] == 5:
-        flop_per_pair = FLOP_PER_EVAL_MDIR
-        flops_per_launch = flop_per_pair * st["nbatch"] * st["pair_evaluations"]
-    elif st["inner_path"] in (3, 4):
-        flop_per_pair = FLOP_PER_EVAL_VTX if st["inner_path"] == 4 else FLOP_PER_EVAL_MIRROR
-        # (N/2)^2 U + V evaluations per batch item (+ the N/2 self-mirror pairs and tile padding); with
-        # the pair split, this rank's share
-        flops_per_launch = flop_per_pair * st["nbatch"] * st["pair_evaluations"]
-    elif st["inner_path"] == 1:
-        flop_per_pair = FLOP_PER_PAIR_SYMMETRIC
-        flops_per_launch = flop_per_pair * st["nbatch"] * N * (N - 1) / 2
-    else:
-        flop_per_pair = FLOP_PER_PAIR_DIRECTED
-        flops_per_launch = flop_per_pair * st["nbatch"] * st["targets"] * N
+    flop_per_pair, flops_per_launch = inner_flops(st, N)
     achieved = flops_per_launch / inner_avg_s / 1e12 if inner_n else None
     clocks = clk.summary()
-    props = torch.cuda.get_device_properties(local)
     sm_max = clocks["sm_max_mhz"] or 1965.0
     peak = fp64_peak_tflops(props, sm_max)
-    step_ms_lib = sum(v[0] for v in tim.values()) / args.steps
-    roof = {"bound": "alu", "kernel": "inner_vtx_kernel / inner_mir_kernel / inner_sym_kernel / inner_kernel (a-2, FP64 pipe)", "achieved": achieved, "peak": peak,
-            "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None,
+    roof = {"bound": "alu", "kernel": "inner_vtx_kernel (a-2, FP64 pipe; inner_path says which kernel ran)",
+            "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": (achieved / peak) if achieved else None,
             "traffic": load_profile_traffic(args.workload),
             "fp64_pipe_active_ncu": load_profile_traffic(args.workload + "_fp64_pipe_active"),
-            "peak_note": f"derived FP64 DFMA peak: {props.multi_processor_count} SMs x 64 lanes x 2 FLOP x {sm_max:.0f} MHz",
-            "inner_path": ["directed (ordered pairs)", "symmetric (unordered pairs)",
-                           "tensor cache + FP64 DGEMM (cuBLAS)",
-                           "mirror-symmetric (one tensor per unordered pair and its z-mirror)",
-                           "mirror-symmetric, one CTA per vertex (sums in shared memory)",
-                           "mirror-symmetric directed (U + V per target and source, forward sums)"][st["inner_path"]],
+            "peak_note": f"derived FP64 DFMA peak: {props.multi_processor_count} SMs x 64 lanes x 2 FLOP x {sm_max:.0f} MHz "
+                         "(MEASURED_PEAKS.json has no FP64 figure; tools/fp64_peak.cu measured 36.96 TFLOP/s)",
+            "inner_path": INNER_PATHS[st["inner_path"]],
             "flop_per_pair": flop_per_pair, "flops_per_launch": flops_per_launch,
             "inner_ms_per_launch": inner_avg_s * 1e3,
-            "inner_share_of_step": (inner_ms / args.steps) / ms_per_step if ms_per_step else None,
+            "inner_share_of_step": (inner_ms / args.steps) / local_mean if local_mean else None,
             "pairs_per_s_inner": pairs_per_build * max(nloc, 1) / inner_avg_s * world if inner_n else None}
     stage_ms = {k: v[0] / args.steps for k, v in tim.items()}
 
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": scaling,
-            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": dict(desc, parallelism=(f"element-split x{world}" if args.workload == "C5" else
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "ms_per_step_mean": ms_mean,
+            "timing": "median of per-step CUDA-event times on the library stream, max over ranks",
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": dict(desc, parallelism=(f"pair split x{world}" if args.workload == "C5" else
                                               f"batch-shard x{world}") if world > 1 else "1 GPU"),
             "pairs_per_s": value * pairs_per_build, "roofline": roof, "stage_ms_per_step": stage_ms,
             "stage_timers": "in timed region" if in_loop_timers else "separate pass (graphs off)",
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(F_host.nbytes) * world,
-                    "d2h_bytes_per_step": int(v_pin.numel() * 8) * world, "api": "landau_jacobian_host"},
+                    "d2h_bytes_per_step": int(v_pin.numel() * 8) * world, "api": "landau_jacobian_host",
+                    "ms_per_step": e_ms},
             "gpu_launches": int(launches), "clocks": clocks}
-    # NEXT-4 variant on the same job (informational; the headline above is the pairwise path)
-    if args.workload == "C4" and not args.tensor_cache and nloc:
+    extras = args.workload == "C4" and not args.tensor_cache and not args.no_sublines
+
+    # ---- weak scaling sub-line (N > 1): every GPU its own 1024 vertices ---------------------------
+    if extras and world > 1:
+        try:
+            Bw = args.batch
+            hw = L.Landau.from_problem(prob0, device=local, stream=stream)
+            Fw = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b, Bw * world), nodes)
+                                        for b in range(rank * Bw, (rank + 1) * Bw)]), device="cuda")
+            vw = torch.empty((Bw, hw.nnz), dtype=torch.float64, device="cuda")
+
+            def wstep():
+                hw.set_state_batched(Fw)
+                hw.jacobian_batched(vw)
+                hw.mass(shift, mvals)
+            for _ in range(args.warmup):
+                wstep()
+            dist.barrier()
+            wms = max_over_ranks(torch, dist, world, statistics.median(timed_steps(torch, stream, wstep, args.steps, flush)))
+            line["weak"] = {"value": Bw * world / (wms / 1e3), "unit": UNIT, "ms_per_step": wms,
+                            "vertices_per_gpu": Bw, "vertices": Bw * world, "scaling": "weak"}
+            hw.close()
+            del Fw, vw
+        except Exception as e:
+            line["weak"] = {"unavailable": str(e)[:200]}
+
+    # ---- configs: C1-C3 single builds (rank 0) and C5 across all ranks ----------------------------
+    if extras:
+        cfgs = {}
+        if rank == 0:
+            for name in ("C1", "C2", "C3"):
+                try:
+                    cfgs[name] = single_build_line(torch, L, inputs, name, local, stream, flush, args.steps, args.warmup,
+                                                   world == 1 and not args.no_cpu_baseline)
+                except Exception as e:
+                    cfgs[name] = {"unavailable": str(e)[:200]}
+        try:
+            cfgs["C5"] = c5_line(torch, dist, L, inputs, world, rank, local, stream, flush, max(5, args.steps // 2),
+                                 args.warmup, args.c5_cells, world == 1 and not args.no_cpu_baseline, peak)
+        except Exception as e:
+            cfgs["C5"] = {"unavailable": str(e)[:200]}
+        line["configs"] = cfgs
+        if "C2" in cfgs:
+            line["c2_single_build"] = cfgs["C2"]
+
+    # ---- NEXT-4 variants on the same job (informational; the headline is the pairwise path) -------
+    if extras and nloc:
         try:
             h.set_tensor_cache(True)
             step()
-            torch.cuda.synchronize()
             h.set_timing(True)
-            vev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-            for k in range(args.steps):
-                flush.fill_(float(k))
-                vev[k][0].record(stream)
-                step()
-                vev[k][1].record(stream)
-            torch.cuda.synchronize()
+            vts = timed_steps(torch, stream, step, args.steps, flush)
             vt = h.get_timing()
             h.set_timing(False)
-            # the same GEMM formulation with the tensors re-evaluated inside every timed build
             h.set_tensor_cache("recompute")
             step()
-            torch.cuda.synchronize()
-            rev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-            for k in range(args.steps):
-                flush.fill_(float(k))
-                rev[k][0].record(stream)
-                step()
-                rev[k][1].record(stream)
-            torch.cuda.synchronize()
-            rms = torch.tensor([sum(a.elapsed_time(b) for a, b in rev)], dtype=torch.float64, device="cuda")
+            rts = timed_steps(torch, stream, step, args.steps, flush)
             h.set_tensor_cache(False)
-            vms = torch.tensor([sum(a.elapsed_time(b) for a, b in vev)], dtype=torch.float64, device="cuda")
-            if world > 1:
-                dist.all_reduce(vms, op=dist.ReduceOp.MAX)
-            vstep = float(vms.item()) / args.steps
-            if world > 1:
-                dist.all_reduce(rms, op=dist.ReduceOp.MAX)
-            rstep = float(rms.item()) / args.steps
+            vstep = max_over_ranks(torch, dist, world, statistics.median(vts))
+            rstep = max_over_ranks(torch, dist, world, statistics.median(rts))
             gemm_s = vt["inner"][0] / max(vt["inner"][1], 1) / 1e3
             line["variants"] = {"tensor_cache_gemm": {
                 "value": total_builds / (vstep / 1e3), "unit": UNIT, "ms_per_step": vstep,
-                "inner_ms_per_launch": gemm_s * 1e3,
-                "inner_tflops": 14.0 * nloc * N * N / gemm_s / 1e12,
+                "inner_ms_per_launch": gemm_s * 1e3, "inner_tflops": 14.0 * nloc * N * N / gemm_s / 1e12,
                 "note": "SURVEY NEXT-4: mesh tensors cached once (7 N^2 doubles), inner integral as three FP64 "
                         "DGEMMs (cuBLAS, FP64 tensor cores); same sums up to order, parity-tested"},
                 "tensor_gemm_recompute": {
                 "value": total_builds / (rstep / 1e3), "unit": UNIT, "ms_per_step": rstep,
                 "note": "the GEMM formulation with all N^2 tensors re-evaluated inside every timed build "
                         "(the batch shares one mesh): no state carried across builds"}}
-        except Exception as e:   # the variant is optional: report why it did not run
+        except Exception as e:
             line["variants"] = {"tensor_cache_gemm": {"unavailable": str(e)[:200]}}
-        # NEXT-4, the other variant: the inner integral with the 3D Cartesian tensor of Eq. 3
-        # (landau3d_inner) on a 3D point set of the thermal-quench shape, 8^3 Q3 cubes (N = 32768)
         try:
             xyz3, w3 = inputs.points3d(8, 3)
             wTD3, wTK3 = inputs.fields3d(xyz3, w3)
@@ -492,45 +657,30 @@ def main():
             G3 = torch.empty((9, n3), dtype=torch.float64, device="cuda")
             for _ in range(2):
                 L.landau3d_inner(X3, D3, K3, G3, stream)
-            ev3 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-            for k in range(args.steps):
-                ev3[k][0].record(stream)
-                L.landau3d_inner(X3, D3, K3, G3, stream)
-                ev3[k][1].record(stream)
-            torch.cuda.synchronize()
-            ms3 = sum(a.elapsed_time(b) for a, b in ev3) / args.steps
+            ms3 = statistics.median(timed_steps(torch, stream, lambda: L.landau3d_inner(X3, D3, K3, G3, stream),
+                                                args.steps, flush))
             line.setdefault("variants", {})["inner3d_cartesian"] = {
-                "value": n3 * n3 / (ms3 * 1e-3), "unit": "pairs/s",
-                "points": n3, "ms_per_launch": ms3,
+                "value": n3 * n3 / (ms3 * 1e-3), "unit": "pairs/s", "points": n3, "ms_per_launch": ms3,
                 "tflops": FLOP_PER_PAIR_3D * n3 * n3 / (ms3 * 1e-3) / 1e12,
                 "frac_of_fp64_peak": FLOP_PER_PAIR_3D * n3 * n3 / (ms3 * 1e-3) / 1e12 / peak,
                 "note": "SURVEY NEXT-4: G_D, G_K with U = (|u|^2 I - u u^T)/|u|^3 directly (no elliptic integrals), "
                         "ordered pairs, parity-tested against oracle O12"}
         except Exception as e:
             line.setdefault("variants", {})["inner3d_cartesian"] = {"unavailable": str(e)[:200]}
-    # NEXT-3: quasi-Newton backward-Euler iterations on the same batch (the paper's figure of merit,
-    # "Newton iterations per second", @37187): per iteration set_state + Jacobian + band LU + solve
-    if args.workload == "C4" and not args.tensor_cache and nloc:
+
+    # ---- NEXT-3: quasi-Newton backward-Euler iterations on the same batch --------------------------
+    if extras and nloc:
         try:
             it_per_call = 2
             Fn = torch.empty_like(F)
             for _ in range(2):
                 h.implicit_step_batched(0.002, F, Fn, max_iter=it_per_call, rtol=0.0)
-            torch.cuda.synchronize()
             h.set_timing(True)
-            nev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-            for k in range(args.steps):
-                flush.fill_(float(k))
-                nev[k][0].record(stream)
-                h.implicit_step_batched(0.002, F, Fn, max_iter=it_per_call, rtol=0.0)
-                nev[k][1].record(stream)
-            torch.cuda.synchronize()
+            nts = timed_steps(torch, stream, lambda: h.implicit_step_batched(0.002, F, Fn, max_iter=it_per_call, rtol=0.0),
+                              args.steps, flush)
             nt = h.get_timing()
             h.set_timing(False)
-            nms = torch.tensor([sum(a.elapsed_time(b) for a, b in nev)], dtype=torch.float64, device="cuda")
-            if world > 1:
-                dist.all_reduce(nms, op=dist.ReduceOp.MAX)
-            ms_it = float(nms.item()) / (args.steps * it_per_call)
+            ms_it = max_over_ranks(torch, dist, world, statistics.median(nts)) / it_per_call
             line["newton"] = {
                 "value": total_builds / (ms_it / 1e3), "unit": "vertex Newton iterations/s", "ms_per_iteration": ms_it,
                 "stage_ms_per_iteration": {k: v[0] / (args.steps * it_per_call) for k, v in nt.items()},
@@ -540,40 +690,15 @@ def main():
                         "node figure is a different problem (10 species, 80 cells, CPU LU)"}
         except Exception as e:
             line["newton"] = {"unavailable": str(e)[:200]}
-    # configs[1] itself (one C2 grid, one build per step; launch-latency regime, CUDA-graph replay)
-    if args.workload == "C4" and rank == 0:
-        try:
-            p2 = inputs.config2()
-            h2 = L.Landau.from_problem(p2, device=local, stream=stream)
-            f2 = torch.tensor(inputs.coefficients(p2, h2.all_nodes()), device="cuda")
-            v2 = torch.empty(h2.nnz, dtype=torch.float64, device="cuda")
-            m2 = torch.empty(h2.nnz, dtype=torch.float64, device="cuda")
-            for _ in range(max(args.warmup, 3)):
-                h2.set_state(f2)
-                h2.jacobian(v2)
-                h2.mass(shift, m2)
-            torch.cuda.synchronize()
-            ev2 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-            for k in range(args.steps):
-                flush.fill_(float(k))
-                ev2[k][0].record(stream)
-                h2.set_state(f2)
-                h2.jacobian(v2)
-                h2.mass(shift, m2)
-                ev2[k][1].record(stream)
-            torch.cuda.synchronize()
-            ms2 = sum(a.elapsed_time(b) for a, b in ev2) / args.steps
-            line["c2_single_build"] = {"value": 1e3 / ms2, "unit": UNIT, "ms_per_step": ms2,
-                                       "pairs_per_s": 1e3 / ms2 * p2.npoints ** 2,
-                                       "inner_path": ["directed", "symmetric", "tensor cache", "mirror", "mirror per-vertex", "mirror directed"][h2.stats()["inner_path"]],
-                                       "note": "BASELINE configs[1]: one e+D Q3 AMR grid (N=1088) per step, "
-                                               "set_state + jacobian (CSR) + mass, CUDA-graph replay"}
-            h2.close()
-        except Exception as e:
-            line["c2_single_build"] = {"unavailable": str(e)[:200]}
+
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        ns = args.cpu_sample or (8 if args.workload == "C4" else 1)
-        line["cpu_baseline"] = cpu_baseline(args, desc, ns)
+        if args.workload == "C4":
+            line["cpu_baseline"] = oracle_c4_baseline(job_vertices(args, world), args.cpu_sample)
+        elif args.workload in ("C1", "C2", "C3"):
+            _, _, _, secs = oracle_full_build(prob0)
+            from oracle.oracle import get_threads
+            line["cpu_baseline"] = {"value": 1.0 / secs, "unit": UNIT, "cores": get_threads(), "kind": "oracle",
+                                    "sample": f"one full {args.workload} oracle Jacobian (incl. |.| scale)"}
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

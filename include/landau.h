@@ -238,7 +238,7 @@ int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double E
  * smaller batches the slot kernel or, below that, the mirror-directed kernel); 2 = mirror slot kernel
  * only; 3 = per-vertex kernel for every batch size (one CTA per vertex when the batch is below one
  * vertex per SM: no vertex split).  enable != 0 on a non-symmetric mesh, or 3 when a
- * vertex's sums (80 B per upper-half point) exceed 160 KB of shared memory, is EUNSUPPORTED;
+ * vertex's sums and staged inputs (168 B per upper-half point) exceed 200 KB of shared memory, is EUNSUPPORTED;
  * enable outside 0..3 is EINVAL. */
 int landau_set_mirror(landau_t h, int32_t enable);
 /* Whether the mesh is exactly z-mirror-symmetric (host logic, also on LANDAU_HOST_ONLY handles) and

@@ -528,6 +528,41 @@ struct VtxItem {   // host-built: tiles (a, b) of the upper half; a == b: the di
   int a, b;
 };
 
+// One (a, b) item reading both tiles from the CTA's staged copy of the vertex (s_i: tile a, s_j: tile b,
+// 32 points x 5 double2 each, layout of vtx_stage_j); otherwise exactly vtx_item (same steps, same order).
+template <bool DIAG, bool MASK>
+__device__ __forceinline__ void vtx_item_staged(const double2 *s_i, const double2 *s_j, int lane, const PairCoef &cf,
+                                                Acc5 &P, Acc5 &M, Acc5 &PJ, Acc5 &MJ) {
+  const double2 irz = s_i[lane * 5], ip01 = s_i[lane * 5 + 1], ip2m0 = s_i[lane * 5 + 2], im12 = s_i[lane * 5 + 3],
+                ir2 = s_i[lane * 5 + 4];
+  const double hpi[3] = {ip01.x, ip01.y, ip2m0.x}, hmi[3] = {ip2m0.y, im12.x, im12.y};
+  const double r = irz.x, z = irz.y, r2 = ir2.x;
+  P = M = PJ = MJ = Acc5{0.0, 0.0, 0.0, 0.0, 0.0};
+  const int src = (lane + 1) & 31;
+  if constexpr (DIAG) {   // step 0: each point with its own mirror (V forward only; U is the self pair)
+    vtx_step<MASK, false, false>(r, z, r2, hpi, hmi, irz.x, irz.y, ir2.x, ip01, ip2m0, im12, cf, 1.0, P, M, PJ, MJ);
+  }
+  constexpr int k0 = DIAG ? 1 : 0, kmain = DIAG ? 16 : 32;
+#pragma unroll kMirUnroll
+  for (int k = k0; k < kmain; k++) {
+    const int jj = (lane + k) & 31;
+    const double2 rz = s_j[jj * 5], p01 = s_j[jj * 5 + 1], p2m0 = s_j[jj * 5 + 2], m12 = s_j[jj * 5 + 3],
+                  rr2 = s_j[jj * 5 + 4];
+    vtx_step<MASK, true, true>(r, z, r2, hpi, hmi, rz.x, rz.y, rr2.x, p01, p2m0, m12, cf, 1.0, P, M, PJ, MJ);
+    acc_shfl(PJ, src);
+    acc_shfl(MJ, src);
+  }
+  if constexpr (DIAG) {   // step 16: lanes >= 16 would double-count
+    const int jj = (lane + 16) & 31;
+    const double2 rz = s_j[jj * 5], p01 = s_j[jj * 5 + 1], p2m0 = s_j[jj * 5 + 2], m12 = s_j[jj * 5 + 3],
+                  rr2 = s_j[jj * 5 + 4];
+    vtx_step<true, true, true>(r, z, r2, hpi, hmi, rz.x, rz.y, rr2.x, p01, p2m0, m12, cf, lane < 16 ? 1.0 : 0.0, P,
+                               M, PJ, MJ);
+    acc_shfl(PJ, src);
+    acc_shfl(MJ, src);
+  }
+}
+
 // Stream-K decomposition over (vertex, round) work.  The batch's rounds form one flattened sequence
 // (vertex-major, rounds in schedule order) with weights wp (a full round of pair items: 2, a round of
 // diagonal items: 1 -- their durations); round (v, rd) starting at weight g = v Wv + wp[rd] belongs to
@@ -546,27 +581,31 @@ __device__ __forceinline__ int vtx_owner(const VtxSched &sc, const int32_t *wp, 
   return (int)(((v * sc.Wv + wp[rd]) * (int64_t)sc.S) / sc.Wtot);
 }
 
-// first flattened round index f = v * nrounds + rd owned by CTA >= c (nbatch * nrounds if none)
+// first flattened round index f = v * nrounds + rd owned by CTA >= c (nbatch * nrounds if none):
+// owner(v, rd) >= c  <=>  v Wv + wp[rd] >= g_c = ceil(c Wtot / S)
 __device__ __forceinline__ int64_t vtx_first_round(const VtxSched &sc, const int32_t *wp, int c) {
-  int64_t lo = 0, hi = (int64_t)sc.nbatch * sc.nrounds;
-  while (lo < hi) {
-    const int64_t mid = (lo + hi) >> 1;
-    if (vtx_owner(sc, wp, mid / sc.nrounds, (int)(mid % sc.nrounds)) >= c) hi = mid;
-    else lo = mid + 1;
-  }
-  return lo;
+  const int64_t g = ((int64_t)c * sc.Wtot + sc.S - 1) / sc.S;
+  const int64_t v = g / sc.Wv, rem = g - v * sc.Wv;
+  int rd = 0;
+  while (rd < sc.nrounds && wp[rd] < rem) rd++;
+  return v * sc.nrounds + rd;
 }
 
-// write a vertex's sums: G(pu) = Ga, G(pm) = F Gb  (F: negate the rz and K_z components)
+// write a vertex's sums: G(pu) = Ga, G(pm) = F Gb  (F: negate the rz and K_z components); pu, pm in smem
 __device__ __forceinline__ void vtx_write_G(double *Gb, const double *sGa, const double *sGb, int64_t N, int64_t H,
-                                            int64_t Hp, const int32_t *pu, const int32_t *pm) {
+                                            int64_t Hp, const int32_t *s_pu, const int32_t *s_pm) {
   for (int64_t k = threadIdx.x; k < 5 * H; k += blockDim.x) {
-    const int64_t c = k / H, u = k % H;
-    Gb[c * N + pu[u]] = sGa[c * Hp + u];
+    const int64_t c = k / H, u = k - c * H;
+    Gb[c * N + s_pu[u]] = sGa[c * Hp + u];
     const double v = sGb[c * Hp + u];
-    Gb[c * N + pm[u]] = (c == 1 || c == 4) ? -v : v;
+    Gb[c * N + s_pm[u]] = (c == 1 || c == 4) ? -v : v;
   }
 }
+
+// Dynamic shared memory of inner_vtx_kernel for H upper-half points (Hp = H rounded up to 32): the sums
+// Ga, Gb [5][Hp] each, the staged vertex [Hp][5] double2 (geometry once per CTA, weights per vertex)
+// and the mirror maps pu, pm [Hp] int32.
+__host__ __device__ constexpr size_t vtx_smem_bytes(int64_t Hp) { return (size_t)Hp * (20 * 8 + 2 * 4); }
 
 template <bool MASK>
 __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int64_t N, int64_t H, VtxSched sc,
@@ -581,14 +620,25 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
                                                                       double *__restrict__ G, int64_t G_bstride,
                                                                       double *__restrict__ part,
                                                                       int32_t *__restrict__ counters) {
-  __shared__ double2 s_j[kVtxWarps][32 * 5];
   __shared__ double s_coef[kNumPairCoef];
   __shared__ double2 s_ltab[kLogTab];
   __shared__ int s_last;
-  extern __shared__ double s_G[];   // Ga [5][Hp], Gb [5][Hp]
+  extern __shared__ double s_G[];   // Ga [5][Hp], Gb [5][Hp] | staged vertex [Hp][5] double2 | pu, pm [Hp]
   const int64_t Hp = (H + 31) / 32 * 32;
   double *sGa = s_G, *sGb = s_G + 5 * Hp;
+  double2 *s_V = reinterpret_cast<double2 *>(s_G + 10 * Hp);
+  int32_t *s_pu = reinterpret_cast<int32_t *>(s_G + 20 * Hp), *s_pm = s_pu + Hp;
   stage_pair_coef(s_coef, s_ltab);
+  // the mesh part of the staged vertex (r, z, r^2) and the mirror maps, once per CTA; padding points
+  // sit far away (z = 1e6 + 2 L: distinct from each other and from every mirror) with zero weights
+  for (int64_t u = threadIdx.x; u < Hp; u += blockDim.x) {
+    const bool v = u < H;
+    const double r = v ? rU[u] : 1.0, z = v ? zU[u] : 1.0e6 + 2.0 * (double)(u & 31);
+    s_V[u * 5] = make_double2(r, z);
+    s_V[u * 5 + 4] = make_double2(r * r, 0.0);
+    s_pu[u] = v ? pu[u] : 0;
+    s_pm[u] = v ? pm[u] : 0;
+  }
   __syncthreads();
   PairCoef cf;
   load_pair_coef(s_coef, s_ltab, cf);
@@ -598,23 +648,36 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
   int64_t f = f0;
   while (f < f1) {
     const int64_t v = f / sc.nrounds;
-    const int rd0 = (int)(f % sc.nrounds);
+    const int rd0 = (int)(f - v * sc.nrounds);
     const int rd1 = (int)min((int64_t)sc.nrounds, f1 - v * sc.nrounds);   // this CTA's rounds [rd0, rd1) of v
     f = v * sc.nrounds + rd1;
+    // stage the vertex's weights: hp = (A + Bf)/2, hm = (A - Bf)/2 with A = wT(u), Bf = F wT(u')
     const double *wb = wT + v * 3 * N;
+    for (int64_t u = threadIdx.x; u < Hp; u += blockDim.x) {
+      double A[3] = {0.0, 0.0, 0.0}, B[3] = {0.0, 0.0, 0.0};
+      if (u < H) {
+        const int64_t p = s_pu[u], q = s_pm[u];
+        A[0] = wb[p];
+        A[1] = wb[N + p];
+        A[2] = wb[2 * N + p];
+        B[0] = wb[q];
+        B[1] = wb[N + q];
+        B[2] = -wb[2 * N + q];
+      }
+      s_V[u * 5 + 1] = make_double2(0.5 * (A[0] + B[0]), 0.5 * (A[1] + B[1]));
+      s_V[u * 5 + 2] = make_double2(0.5 * (A[2] + B[2]), 0.5 * (A[0] - B[0]));
+      s_V[u * 5 + 3] = make_double2(0.5 * (A[1] - B[1]), 0.5 * (A[2] - B[2]));
+    }
     for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) s_G[k] = 0.0;
     __syncthreads();
     for (int rd = rd0; rd < rd1; rd++) {
       for (int q = round_ptr[rd] + wid; q < round_ptr[rd + 1]; q += kVtxWarps) {
         const VtxItem it = items[q];
-        __syncwarp();   // the previous item's readers are done with the warp's j-tile buffer
-        vtx_stage_j(it.b, rU, zU, wb, N, H, pu, pm, lane, s_j[wid]);
-        __syncwarp();
         Acc5 P, M, PJ, MJ;
         if (it.a == it.b)
-          vtx_item<true, MASK>(it.a, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
+          vtx_item_staged<true, MASK>(s_V + it.a * 32 * 5, s_V + it.b * 32 * 5, lane, cf, P, M, PJ, MJ);
         else
-          vtx_item<false, MASK>(it.a, rU, zU, wb, N, H, pu, pm, lane, s_j[wid], cf, P, M, PJ, MJ);
+          vtx_item_staged<false, MASK>(s_V + it.a * 32 * 5, s_V + it.b * 32 * 5, lane, cf, P, M, PJ, MJ);
         vtx_add_pm(sGa, sGb, Hp, (int64_t)it.a * 32 + lane, P, M);
         if (it.a == it.b) __syncwarp();   // forward and reverse sums of a diagonal item hit the same tile
         vtx_add_pm(sGa, sGb, Hp, (int64_t)it.b * 32 + ((lane + (it.a == it.b ? 17 : 32)) & 31), PJ, MJ);
@@ -623,7 +686,7 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
     }
     const int cfirst = vtx_owner(sc, wp, v, 0), clast = vtx_owner(sc, wp, v, sc.nrounds - 1);
     if (cfirst == clast) {   // the whole vertex ran here
-      vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, pu, pm);
+      vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, s_pu, s_pm);
     } else {                 // one segment of a split vertex: partial slot, then the last one combines
       double *slot = part + ((int64_t)c * 2 + (c == cfirst ? 1 : 0)) * 10 * Hp;
       for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) slot[k] = s_G[k];
@@ -633,17 +696,35 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
       __syncthreads();
       if (s_last) {
         __threadfence();
-        for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) {   // partials in CTA order
-          double acc = __ldcg(part + ((int64_t)cfirst * 2 + 1) * 10 * Hp + k);
-          for (int cc = cfirst + 1; cc <= clast; cc++) acc += __ldcg(part + (int64_t)cc * 2 * 10 * Hp + k);
-          s_G[k] = acc;
+        const double *p0 = part + ((int64_t)cfirst * 2 + 1) * 10 * Hp;
+        constexpr int kU = 8;   // independent loads in flight per thread
+        for (int64_t k0 = threadIdx.x; k0 < 10 * Hp; k0 += kU * blockDim.x) {   // partials in CTA order
+          double acc[kU];
+#pragma unroll
+          for (int m = 0; m < kU; m++) {
+            const int64_t k = k0 + m * blockDim.x;
+            acc[m] = k < 10 * Hp ? __ldcg(p0 + k) : 0.0;
+          }
+          for (int cc = cfirst + 1; cc <= clast; cc++) {
+            const double *pc = part + (int64_t)cc * 2 * 10 * Hp;
+#pragma unroll
+            for (int m = 0; m < kU; m++) {
+              const int64_t k = k0 + m * blockDim.x;
+              if (k < 10 * Hp) acc[m] += __ldcg(pc + k);
+            }
+          }
+#pragma unroll
+          for (int m = 0; m < kU; m++) {
+            const int64_t k = k0 + m * blockDim.x;
+            if (k < 10 * Hp) s_G[k] = acc[m];
+          }
         }
         __syncthreads();
-        vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, pu, pm);
+        vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, s_pu, s_pm);
         if (threadIdx.x == 0) counters[v] = 0;   // ready for the next build
       }
     }
-    __syncthreads();   // the write-out reads s_G before the next segment zeroes it
+    __syncthreads();   // the write-out reads s_G (and items read s_V) before the next segment rewrites them
   }
 }
 

@@ -343,7 +343,8 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
   const int variant = inner_variant();
   ip.vtx = h->mirror && h->mirror_on && h->vtx_smem && !h->dist_pairs &&
            (h->mirror_mode == 3 ||
-            (h->mirror_mode == 1 && nbatch * h->vtx_Wv >= vtx_min_weight_per_sm() * num_sms(h) * kVtxMinB));
+            (h->mirror_mode == 1 && sym_enabled() &&
+             nbatch * h->vtx_Wv >= vtx_min_weight_per_sm() * num_sms(h) * kVtxMinB));
   if (ip.vtx) {   // stream-K partial slots (one pair per CTA) and per-vertex arrival counters
     if (!h->d_vtx_part) {
       const int64_t Hp = (h->H + 31) / 32 * 32;
@@ -1899,8 +1900,8 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
             if ((t + 1) % kVtxWarps == 0 || t + 1 == T) vround.push_back((int32_t)vitems.size());
           }
       }
-      const size_t vsmem = (size_t)10 * T * 32 * sizeof(double);
-      h->vtx_smem = world == 1 && vsmem <= (size_t)160 * 1024 && T >= 2 ? vsmem : 0;
+      const size_t vsmem = vtx_smem_bytes((int64_t)T * 32);
+      h->vtx_smem = world == 1 && vsmem <= (size_t)200 * 1024 && T >= 2 ? vsmem : 0;
       h->nvtx_rounds = (int)vround.size() - 1;
       // stream-K weights: a round lasts as long as its longest item (pair item 2, diagonal item 1)
       std::vector<int32_t> vwp(1, 0);

@@ -30,15 +30,15 @@ def test_reference_arm_other_ranks_exit_quietly():
     assert out.returncode == 0 and out.stdout.strip() == ""
 
 
-def test_c4_sharding_weak_and_strong():
-    """C4 vertices are independent problems: by default every rank builds its own --batch vertices
-    (weak scaling, a job of batch x world); --strong splits a fixed job.  The ranks' vertex ranges
-    are disjoint and cover the job, and world 1 is the BASELINE configs[3] batch either way."""
-    import argparse
+def test_c4_sharding_strong_and_weak():
+    """C4 vertices are independent problems: by default a fixed job of --batch vertices (BASELINE
+    configs[3]: 1024) is split over the ranks (strong scaling); --weak gives every rank its own --batch
+    vertices.  The ranks' vertex ranges are disjoint and cover the job, and world 1 is the same batch
+    either way."""
     sys.path.insert(0, ROOT)
     import bench
-    for strong, world, job in ((False, 1, 16), (False, 2, 32), (True, 2, 16), (True, 4, 16)):
-        args = argparse.Namespace(batch=16, strong=strong, workload="C4")
+    for weak, world, job in ((False, 1, 16), (False, 2, 16), (False, 4, 16), (True, 1, 16), (True, 2, 32)):
+        args = bench.parse(["--batch", "16"] + (["--weak"] if weak else []))
         assert bench.job_vertices(args, world) == job
         seen = []
         for rank in range(world):
@@ -46,6 +46,24 @@ def test_c4_sharding_weak_and_strong():
             assert desc["vertices"] == job and len(items) == job // world
             seen += [it.seed for it in items]
         assert sorted(seen) == [20220 + b for b in range(job)]
+    assert bench.parse([]).batch == 1024 and not bench.parse([]).weak
+
+
+def test_clock_region_filter_and_handshake():
+    """Clocks keeps only the samples taken inside the timed region (mark_start/mark_end) and falls
+    back to all samples when the region saw none."""
+    sys.path.insert(0, ROOT)
+    import bench
+    c = bench.Clocks(0)
+    c.source = "nvml"
+    row = lambda sm: ["0", str(sm), "1965", "", "0x0", "Not Active", "Not Active", "Not Active", "Not Active"]
+    c.rows = [row(1000), row(1965), row(1965), row(1200)]
+    c.times = [0.0, 10.0, 10.5, 20.0]
+    c.t0, c.t1 = 9.9, 10.6
+    s = c.summary()
+    assert s["samples"] == 2 and s["sm_mhz"] == 1965.0
+    c.t0, c.t1 = 30.0, 31.0
+    assert c.summary()["samples"] == 4
 
 
 def test_clock_summary_decodes_nvml_reason_bits():
