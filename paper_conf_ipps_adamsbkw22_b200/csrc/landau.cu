@@ -857,6 +857,22 @@ int build_mass(landau_t h) {
   return LANDAU_OK;
 }
 
+// The dynamic shared-memory limit of inner_vtx_kernel is a per-function attribute shared by every
+// handle on a device, so it only ever grows: the largest need of any handle created so far (setting a
+// small handle's size would make a larger handle's launches fail).
+bool raise_vtx_smem_attr(int device, size_t bytes) {
+  static std::mutex mu;
+  static size_t cur[64] = {0};
+  std::lock_guard<std::mutex> lk(mu);
+  size_t &c = cur[device & 63];
+  if (bytes <= c) return true;
+  if (cudaFuncSetAttribute(inner_vtx_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess ||
+      cudaFuncSetAttribute(inner_vtx_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess)
+    return false;
+  c = bytes;
+  return true;
+}
+
 // Mirror symmetry z -> -z: every grid's quadrature points pair up as (r, z), (r, -z)
 // BIT-EXACTLY (no point on z = 0).  The mirror kernels evaluate the tensors of a point's mirror from
 // the point itself, so anything short of bit-exact equality would move the caller's points; meshes
@@ -1916,9 +1932,7 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
             (rc = upload(h, &h->d_vtx_wp, vwp)))
           return bail(rc);
         if (!h->host_only) {
-          cudaError_t e1 = cudaFuncSetAttribute(inner_vtx_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)vsmem);
-          cudaError_t e2 = cudaFuncSetAttribute(inner_vtx_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)vsmem);
-          if (e1 != cudaSuccess || e2 != cudaSuccess) return bail(fail(h, LANDAU_ECUDA, "inner_vtx_kernel smem attribute"));
+          if (!raise_vtx_smem_attr(cuda_device, vsmem)) return bail(fail(h, LANDAU_ECUDA, "inner_vtx_kernel smem attribute"));
         }
       }
       h->mirror = true;

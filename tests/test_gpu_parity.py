@@ -1019,3 +1019,20 @@ def test_pair_split_partials_sum_with_item_runs(monkeypatch):
     Gsum = sum(G_of(f"3:{r}") for r in range(3))
     scale = np.abs(Gfull).max(axis=2, keepdims=True)
     assert np.max(np.abs(Gsum - Gfull) / scale) <= 1e-12
+
+
+def test_vertex_kernel_smem_limit_survives_smaller_handles():
+    """The per-vertex kernel's dynamic shared-memory limit is a per-function attribute shared by all
+    handles: creating a handle with a smaller mesh after a larger one must not break the larger
+    handle's launches (regression: the bench's Newton sub-line failed after the C1 config line)."""
+    big = L.Landau.from_problem(inputs.config4_vertex(0), device=0)
+    small = L.Landau.from_problem(inputs.config1(), device=0)   # 10.7 KB vs 91 KB of shared memory
+    big.set_mirror("vertex")
+    f = inputs.coefficients(inputs.config4_vertex(0), big.all_nodes())
+    F = torch.tensor(np.stack([f] * 4), device=DEV)
+    big.set_state_batched(F)
+    out = torch.empty((4, big.nnz), dtype=torch.float64, device=DEV)
+    big.jacobian_batched(out)
+    torch.cuda.synchronize()
+    assert big.stats()["inner_path"] == 4 and np.all(np.isfinite(out.cpu().numpy()))
+    small.close()
