@@ -78,6 +78,28 @@ struct Plan {
   std::vector<GatherMap> csr_map, coo_map;
 };
 
+// Phased gather maps of the fused element + assembly kernel (tail_kernel, kernels_fe.cuh): each grid's
+// cells are cut into phases of at most `cap` cells (cells sorted by their z centre, so a z-mirror
+// mesh splits at z = 0 and few slots straddle two phases); a phase's element matrices live in shared
+// memory, cell c of the phase at local offset c * 2 Nb^2.  Per phase, the output slots it touches
+// (sorted) with their contributions restricted to the phase, in the gather map's (cell, a, b) order,
+// and a mode: 0 direct (every contribution in this phase: write), 1 first phase of a straddling slot
+// (keep the partial sum in shared memory, cross id x), 2 middle (add), 3 last (add the partial, write).
+struct PhaseMaps {
+  std::vector<int32_t> grid_phase_ptr;   // [ngrids + 1] phases of each grid
+  std::vector<int32_t> cell_ptr;         // [nphases + 1] into cells
+  std::vector<int32_t> cells;            // global cell index, phase by phase
+  std::vector<int32_t> slot_ptr;         // [nphases + 1] into slot / mode_x / cptr
+  std::vector<int32_t> slot;             // grid-local output slot
+  std::vector<int32_t> mode_x;           // mode | (cross id << 2)
+  std::vector<int32_t> cptr;             // [total phase slots + 1] into cidx / cw
+  std::vector<int32_t> cidx;             // element-matrix index in the phase's shared buffer (doubles)
+  std::vector<double> cw;
+  int max_cells = 0, max_cross = 0;
+};
+// cap >= 1 cells per phase; returns "" or an error (more than INT32_MAX entries).
+std::string build_phase_maps(const Plan &plan, const std::vector<GatherMap> &maps, int cap, PhaseMaps &out);
+
 // Build the plan.  Returns "" on success or an error message (the mesh is invalid).
 std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, const double *radius, int order,
                        Plan &plan);

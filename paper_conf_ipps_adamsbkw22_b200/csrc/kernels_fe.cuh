@@ -379,6 +379,100 @@ __global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ C
     }
 }
 
+// ------------------------------------------------------------------------------------------------
+// N3 + N4 fused (batches of small meshes, C4): a persistent CTA owns one batch item at a time and
+// walks each grid's phases (host_setup.h PhaseMaps: groups of cells by z, a z-mirror mesh splits at
+// z = 0).  Per phase its warps compute the phase's element matrices (C^D, C^K) by sum factorisation
+// (sf_cell) into SHARED memory -- the two-kernel form writes and reads them through HBM (285 MB each
+// way per C4 build) -- then every thread gathers output slots of the phase from shared memory: a slot
+// whose contributions all lie in the phase is written; a slot straddling phases keeps its partial sum
+// in shared memory from its first to its last phase.  Every slot sums its contributions in the
+// gather map's fixed (cell, a, b) order within a phase and the phases in order: deterministic.
+// ------------------------------------------------------------------------------------------------
+struct TailDev {
+  const int32_t *grid_phase_ptr, *cell_ptr, *cells, *slot_ptr, *slot, *mode_x, *cptr, *cidx;
+  const double *cw;
+  int ngrids, max_cells, max_cross;
+};
+
+template <int S>
+__host__ __device__ constexpr int tail_warps() { return S == 5 ? 8 : 16; }
+
+// dynamic shared memory: element matrices of max_cells cells | sA [warps][5][NB] | sT [warps][6][NB][S]
+// | straddling-slot partials [max_cross][2]
+template <int S>
+__host__ __device__ constexpr size_t tail_smem_bytes(int max_cells, int max_cross) {
+  return sizeof(double) * ((size_t)max_cells * 2 * S * S * S * S + (size_t)tail_warps<S>() * (5 * S * S + 6 * S * S * S) +
+                           2 * (size_t)max_cross);
+}
+
+template <int S>
+__global__ void __launch_bounds__(32 * tail_warps<S>(), 1) tail_kernel(const double *__restrict__ G, int64_t N,
+                                                                       int nbatch, const double *__restrict__ pw,
+                                                                       const double *__restrict__ cell_h,
+                                                                       const double *__restrict__ tab1, const TailDev td,
+                                                                       const GatherDev *__restrict__ maps,
+                                                                       double *__restrict__ out, int64_t out_bstride) {
+  constexpr int NB = S * S, W = tail_warps<S>();
+  extern __shared__ double s_tail[];
+  double *sC = s_tail;
+  double(*sA)[5][NB] = reinterpret_cast<double(*)[5][NB]>(sC + (size_t)td.max_cells * 2 * NB * NB);
+  double(*sT)[6][NB][S] = reinterpret_cast<double(*)[6][NB][S]>(sC + (size_t)td.max_cells * 2 * NB * NB + W * 5 * NB);
+  double2 *sX = reinterpret_cast<double2 *>(sC + (size_t)td.max_cells * 2 * NB * NB + W * (5 * NB + 6 * NB * S));
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  double PLL[S], PLD[S], PDL[S], PDD[S];
+  sf_tables<S>(tab1, lane, PLL, PLD, PDL, PDD);
+  for (int b = blockIdx.x; b < nbatch; b += gridDim.x) {
+    const double *Gb = G + (int64_t)b * 5 * N;
+    double *ob = out + (int64_t)b * out_bstride;
+    for (int g = 0; g < td.ngrids; g++) {
+      const GatherDev &gm = maps[g];
+      for (int ph = td.grid_phase_ptr[g]; ph < td.grid_phase_ptr[g + 1]; ph++) {
+        const int c0 = td.cell_ptr[ph], nc = td.cell_ptr[ph + 1] - c0;
+        for (int lc = wid; lc < nc; lc += W) {   // a-4: one warp per cell
+          const int64_t e = td.cells[c0 + lc];
+          __syncwarp();   // the previous cell's readers are done with sA / sT
+          if (lane < NB) {
+            const int64_t i = e * NB + lane;
+            const double w = pw[i];
+#pragma unroll
+            for (int c = 0; c < 5; c++) sA[wid][c][lane] = w * Gb[c * N + i];
+          }
+          __syncwarp();
+          sf_cell<S>(sA[wid], sT[wid], lane, PLL, PLD, PDL, PDD, 2.0 / cell_h[e], sC + (size_t)lc * 2 * NB * NB);
+        }
+        __syncthreads();   // the phase's element matrices are complete
+        const int s0 = td.slot_ptr[ph], s1 = td.slot_ptr[ph + 1];
+        for (int i = s0 + threadIdx.x; i < s1; i += blockDim.x) {   // a-3 + a-5
+          double sD = 0.0, sK = 0.0;
+          for (int k = td.cptr[i]; k < td.cptr[i + 1]; k++) {
+            const double w = td.cw[k];
+            const double2 v = *reinterpret_cast<const double2 *>(sC + td.cidx[k]);   // (C^D, C^K)
+            sD = fma(w, v.x, sD);
+            sK = fma(w, v.y, sK);
+          }
+          const int mx = td.mode_x[i], mode = mx & 3, x = mx >> 2;
+          if (mode == 1) {
+            sX[x] = make_double2(sD, sK);
+            continue;
+          }
+          if (mode == 2) {
+            sX[x] = make_double2(sX[x].x + sD, sX[x].y + sK);
+            continue;
+          }
+          if (mode == 3) {
+            sD = sX[x].x + sD;
+            sK = sX[x].y + sK;
+          }
+          const int64_t s = td.slot[i];
+          for (int q = 0; q < gm.nsp; q++) ob[gm.out_off[q] + s] = fma(gm.fD[q], sD, gm.fK[q] * sK);
+        }
+        __syncthreads();   // the next phase overwrites the element matrices
+      }
+    }
+  }
+}
+
 // mass gather (create time): out[s] = sum_k w_k M[idx_k]
 // (M points at the mass entries of the element buffer, or at M + 1 for the interleaved advection ones)
 __global__ void mass_gather_kernel(const int64_t *__restrict__ ptr, const int32_t *__restrict__ idx,

@@ -61,6 +61,16 @@ struct landau_s {
     int64_t nslots = 0;
   };
   std::vector<DevMap> d_csr, d_coo;
+  GatherDev *d_gmaps[2] = {nullptr, nullptr};   // per format (CSR, COO): the grids' gather maps (tail_kernel)
+  // tail_kernel (fused a-4 + a-5) phased gather maps per format; tail_ok: built and fit shared memory
+  struct TailMaps {
+    int32_t *grid_phase_ptr = nullptr, *cell_ptr = nullptr, *cells = nullptr, *slot_ptr = nullptr, *slot = nullptr,
+            *mode_x = nullptr, *cptr = nullptr, *cidx = nullptr;
+    double *cw = nullptr;
+    int max_cells = 0, max_cross = 0;
+  } tmaps[2];
+  bool tail_ok = false;
+  size_t tail_smem = 0;
   std::vector<double *> d_mass_csr, d_mass_coo;   // per grid
   std::vector<double *> d_adv_csr, d_adv_coo;     // per grid: unscaled E_z advection matrix (NEXT-3)
   std::vector<int64_t *> d_rowptr;                // per grid: CSR pattern of one species block
@@ -281,6 +291,24 @@ int launch_field(landau_t h, int64_t nbatch) {
   return LANDAU_OK;
 }
 
+
+// N3 + N4 fused into tail_kernel (one CTA per batch item, element matrices in an L2-resident scratch)
+// for batches of small meshes: all targets on this GPU, at least LANDAU_TAIL_MIN_BATCH items (fewer
+// items would leave most SMs idle: the two-kernel form spreads the cells), <= 1 MB of element matrices
+// per item.  LANDAU_TAIL=0 disables it.
+bool use_tail(landau_t h, int64_t nbatch) {
+  static const bool on = [] {
+    const char *e = getenv("LANDAU_TAIL");
+    return !(e && atoi(e) == 0);
+  }();
+  static const int64_t min_batch = [] {
+    const char *e = getenv("LANDAU_TAIL_MIN_BATCH");
+    return e ? (int64_t)atoll(e) : (int64_t)16;
+  }();
+  return on && h->tail_ok && h->Nc == h->plan.npts && h->world == 1 && nbatch >= min_batch;
+}
+
+int64_t tail_grid(landau_t h, int64_t nbatch) { return std::min<int64_t>(nbatch, num_sms(h)); }
 
 struct InnerPlan {
   bool vtx = false;    // mirror-symmetric per-vertex kernel, stream-K over (vertex, round) work
@@ -764,11 +792,33 @@ int launch_assemble(landau_t h, int64_t nbatch, double *out, int format) {   // 
 }
 
 template <int NB>
+int launch_tail(landau_t h, int64_t nbatch, double *out, int format) {
+  const Plan &P = h->plan;
+  constexpr int S = NB == 9 ? 3 : (NB == 16 ? 4 : 5);
+  Timer t(h, LANDAU_T_ELEMENT);   // a-4 and a-5 in one kernel: timed as the element stage
+  const int64_t out_bstride = format == LANDAU_CSR ? h->nnz : h->ncoo;
+  const auto &m = h->tmaps[format == LANDAU_CSR ? 0 : 1];
+  TailDev td{m.grid_phase_ptr, m.cell_ptr, m.cells, m.slot_ptr, m.slot, m.mode_x, m.cptr, m.cidx, m.cw,
+             P.ngrids, m.max_cells, m.max_cross};
+  const size_t smem = tail_smem_bytes<S>(m.max_cells, m.max_cross);
+  // > 48 KB of dynamic shared memory: the attribute is per device and cheap to set, so on every call
+  CU(cudaFuncSetAttribute(tail_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  tail_kernel<S><<<(unsigned)tail_grid(h, nbatch), 32 * tail_warps<S>(), smem, h->stream>>>(
+      h->d_G, P.npts, (int)nbatch, h->d_w, h->d_h, h->d_tab + 3 * NB * NB, td, h->d_gmaps[format == LANDAU_CSR ? 0 : 1],
+      out, out_bstride);
+  h->launches++;
+  h->tlaunch[LANDAU_T_ELEMENT]++;
+  KCHECK();
+  return LANDAU_OK;
+}
+
+template <int NB>
 int build_jacobian(landau_t h, int64_t nbatch, double *out, int format) {
   int rc;
   if ((rc = launch_field<NB>(h, nbatch))) return rc;
   if ((rc = launch_inner(h, nbatch))) return rc;
   if (!out) return LANDAU_OK;   // point_coeffs: G only
+  if (use_tail(h, nbatch)) return launch_tail<NB>(h, nbatch, out, format);
   // a-4 + a-5 in batch chunks whose element matrices stay resident in L2 between the two kernels
   const int64_t nb = h->chunk;
   const int64_t out_bstride = format == LANDAU_CSR ? h->nnz : h->ncoo;
@@ -1115,6 +1165,12 @@ void landau_destroy(landau_t h) {
   }
   cudaFree(h->d_vtx_items);
   cudaFree(h->d_vtx_round_ptr);
+  cudaFree(h->d_gmaps[0]);
+  cudaFree(h->d_gmaps[1]);
+  for (auto &m : h->tmaps)
+    for (void *q : {(void *)m.grid_phase_ptr, (void *)m.cell_ptr, (void *)m.cells, (void *)m.slot_ptr, (void *)m.slot,
+                    (void *)m.mode_x, (void *)m.cptr, (void *)m.cidx, (void *)m.cw})
+      cudaFree(q);
   cudaFree(h->d_vtx_wp);
   cudaFree(h->d_vtx_part);
   cudaFree(h->d_vtx_cnt);
@@ -1996,6 +2052,61 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
       auto &d = f == 0 ? h->d_csr[g] : h->d_coo[g];
       if ((rc = upload(h, &d.ptr, m.ptr)) || (rc = upload(h, &d.idx, m.idx)) || (rc = upload(h, &d.w, m.w))) return bail(rc);
       d.nslots = (int64_t)m.ptr.size() - 1;
+    }
+  }
+  for (int f = 0; f < 2; f++) {   // the grids' gather maps with their species factors (tail_kernel)
+    std::vector<GatherDev> gms(P.ngrids);
+    for (int g = 0; g < P.ngrids; g++) {
+      const auto &m = f == 0 ? h->d_csr[g] : h->d_coo[g];
+      GatherDev &gd = gms[g];
+      gd = GatherDev{};
+      gd.ptr = m.ptr;
+      gd.idx = m.idx;
+      gd.w = m.w;
+      gd.nslots = m.nslots;
+      gd.nsp = h->spc.grid_nsp[g];
+      for (int q = 0; q < gd.nsp; q++) {
+        const int sp = h->spc.grid_sp[g][q];
+        gd.out_off[q] = f == 0 ? h->snnz_off[sp] : h->scoo_off[sp];
+        gd.fD[q] = h->spc.fD[sp];
+        gd.fK[q] = h->spc.fK[sp];
+      }
+    }
+    if ((rc = upload(h, &h->d_gmaps[f], gms))) return bail(rc);
+  }
+  {   // tail_kernel's phased maps: phases of as many cells as fit the shared memory left beside the
+      // sum-factorisation scratch (meshes of up to ~128 cells per grid; larger meshes keep two kernels)
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, cuda_device);
+    const int S = P.p + 1, nb = P.nb;
+    const size_t fixed = P.nb == 25 ? tail_smem_bytes<5>(0, 0) : P.nb == 16 ? tail_smem_bytes<4>(0, 0) : tail_smem_bytes<3>(0, 0);
+    const size_t per_cell = sizeof(double) * 2 * nb * nb, cross_reserve = 16 * 1024;
+    const int cap = optin > (int)(fixed + cross_reserve) ? (int)((optin - fixed - cross_reserve) / per_cell) : 0;
+    int64_t max_grid_cells = 0;
+    for (int g = 0; g < P.ngrids; g++) max_grid_cells = std::max(max_grid_cells, P.grids[g].ncell);
+    (void)S;
+    if (cap >= 4 && max_grid_cells <= 8LL * cap) {
+      bool ok = true;
+      for (int f = 0; f < 2 && ok; f++) {
+        PhaseMaps pm;
+        if (!build_phase_maps(P, f == 0 ? P.csr_map : P.coo_map, cap, pm).empty()) {
+          ok = false;
+          break;
+        }
+        auto &m = h->tmaps[f];
+        m.max_cells = pm.max_cells;
+        m.max_cross = pm.max_cross;
+        if ((rc = upload(h, &m.grid_phase_ptr, pm.grid_phase_ptr)) || (rc = upload(h, &m.cell_ptr, pm.cell_ptr)) ||
+            (rc = upload(h, &m.cells, pm.cells)) || (rc = upload(h, &m.slot_ptr, pm.slot_ptr)) ||
+            (rc = upload(h, &m.slot, pm.slot)) || (rc = upload(h, &m.mode_x, pm.mode_x)) ||
+            (rc = upload(h, &m.cptr, pm.cptr)) || (rc = upload(h, &m.cidx, pm.cidx)) || (rc = upload(h, &m.cw, pm.cw)))
+          return bail(rc);
+        const size_t need = P.nb == 25 ? tail_smem_bytes<5>(m.max_cells, m.max_cross)
+                            : P.nb == 16 ? tail_smem_bytes<4>(m.max_cells, m.max_cross)
+                                         : tail_smem_bytes<3>(m.max_cells, m.max_cross);
+        if (need > (size_t)optin) ok = false;
+      }
+      h->tail_ok = ok;
     }
   }
   switch (P.nb) {

@@ -1036,3 +1036,55 @@ def test_vertex_kernel_smem_limit_survives_smaller_handles():
     torch.cuda.synchronize()
     assert big.stats()["inner_path"] == 4 and np.all(np.isfinite(out.cpu().numpy()))
     small.close()
+
+
+_TAIL_CHILD = r'''
+import os, sys, numpy as np, torch
+sys.path.insert(0, os.getcwd())
+from paper_conf_ipps_adamsbkw22_b200 import inputs
+from paper_conf_ipps_adamsbkw22_b200 import landau as L
+fmt, nb, path = int(sys.argv[1]), int(sys.argv[2]), sys.argv[3]
+h = L.Landau.from_problem(inputs.config4_vertex(0), device=0)
+h.set_mirror("slots")
+nodes = h.all_nodes()
+verts = [(k * 1023) // (nb - 1) for k in range(nb)]
+F = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in verts]), device="cuda")
+h.set_state_batched(F)
+out = torch.full((nb, h.nnz if fmt == 0 else h.ncoo), float("nan"), dtype=torch.float64, device="cuda")
+h.set_timing(True)
+h.jacobian_batched(out, fmt)
+t = h.get_timing()
+np.save(path, out.cpu().numpy())
+print("stages", t["element"][1], t["assemble"][1])
+'''
+
+
+@pytest.mark.parametrize("fmt", [L.LANDAU_CSR, L.LANDAU_COO])
+def test_fused_tail_kernel_equals_two_kernel_path(fmt, tmp_path):
+    """Batches of >= 16 small meshes run a-4 + a-5 as one kernel (tail_kernel: each phase's element
+    matrices in shared memory, then the gather); LANDAU_TAIL=0 runs element_sf_kernel + assemble_kernel.
+    On the same G (slot kernel for a-2, batch-invariant) the values agree: slots inside one phase bit
+    for bit (same contractions, same gather order), slots straddling the z = 0 phase cut up to the
+    grouping of their sum; and the tail's values match the oracle."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    nb = 20
+    res = {}
+    for tail in ("1", "0"):
+        path = str(tmp_path / f"J{tail}.npy")
+        out = subprocess.run([sys.executable, "-c", _TAIL_CHILD, str(fmt), str(nb), path], capture_output=True,
+                             text=True, timeout=600, cwd=root, env=dict(os.environ, LANDAU_TAIL=tail))
+        assert out.returncode == 0, out.stderr[-3000:]
+        res[tail] = (np.load(path), out.stdout.split())
+    assert res["1"][1][-2:] == ["1", "0"] and res["0"][1][-2:] == ["1", "1"]   # fused vs element + assemble
+    Jt, J2 = res["1"][0], res["0"][0]
+    assert np.all(np.isfinite(Jt))
+    same = Jt.view(np.uint64) == J2.view(np.uint64)
+    assert same.mean() > 0.9
+    assert np.max(np.abs(Jt - J2)) <= 1e-15 * np.abs(J2).max()
+    verts = [(k * 1023) // (nb - 1) for k in range(nb)]
+    o = Oracle(inputs.config4_vertex(verts[7]))
+    Jo, Ja = o.jacobian(o.coefficients()) if fmt == L.LANDAU_CSR else o.jacobian_coo(o.coefficients())
+    assert np.all(np.abs(Jt[7] - Jo) <= 1e-11 * Ja)
