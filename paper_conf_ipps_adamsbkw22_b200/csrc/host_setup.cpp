@@ -527,44 +527,27 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
 
 std::string build_phase_maps(const Plan &plan, const std::vector<GatherMap> &maps, int cap, PhaseMaps &out) {
   out = PhaseMaps();
-  const int nb = plan.nb, nqp = plan.nqp;
+  const int nb = plan.nb;
   const int64_t csz = 2LL * nb * nb;   // doubles per cell in the element buffer
   out.grid_phase_ptr.push_back(0);
-  out.cell_ptr.push_back(0);
   out.slot_ptr.push_back(0);
-  out.cptr.push_back(0);
-  std::vector<int32_t> phase_of(plan.ncell, -1), local_of(plan.ncell, -1);
   for (int g = 0; g < plan.ngrids; g++) {
     const GridPlan &G = plan.grids[g];
-    // cells by z centre (the mean z of the cell's points), then index: ties keep input order
-    std::vector<int64_t> order(G.ncell);
-    std::vector<double> zc(G.ncell, 0.0);
-    for (int64_t c = 0; c < G.ncell; c++) {
-      order[c] = c;
-      for (int q = 0; q < nqp; q++) zc[c] += plan.pz[G.pt0 + c * nqp + q];
-    }
-    std::stable_sort(order.begin(), order.end(), [&](int64_t a, int64_t b) { return zc[a] < zc[b]; });
-    const int nph = (int)((G.ncell + cap - 1) / cap), per = (int)((G.ncell + nph - 1) / nph);   // balanced phases
-    const int ph0 = (int)out.cell_ptr.size() - 1;
-    for (int64_t k = 0; k < G.ncell; k++) {
-      const int64_t ge = G.cell0 + order[k];
-      const int ph = (int)(k / per);
-      phase_of[ge] = ph0 + ph;
-      local_of[ge] = (int32_t)(k % per);
-      out.cells.push_back((int32_t)ge);
-      if ((k + 1) % per == 0 || k + 1 == G.ncell) out.cell_ptr.push_back((int32_t)out.cells.size());
-      out.max_cells = std::max(out.max_cells, (int)(k % per) + 1);
-    }
-    const int ph1 = (int)out.cell_ptr.size() - 1;
+    const int nph = (int)((G.ncell + cap - 1) / cap), per = (int)((G.ncell + nph - 1) / nph);   // balanced
+    const int ph0 = (int)out.cell_ptr.size();
+    for (int64_t c = 0; c < G.ncell; c += per) out.cell_ptr.push_back((int32_t)(G.cell0 + c));
+    out.max_cells = std::max(out.max_cells, per);
+    const int ph1 = (int)out.cell_ptr.size();
     out.grid_phase_ptr.push_back(ph1);
-    // per slot: the phases it touches (first, last), a cross id when they differ
+    auto phase_of = [&](int64_t ge) { return ph0 + (int)((ge - G.cell0) / per); };
     const GatherMap &m = maps[g];
     const int64_t nslots = (int64_t)m.ptr.size() - 1;
-    std::vector<int32_t> pfirst(nslots, INT32_MAX), plast(nslots, -1), xid(nslots, -1);
+    std::vector<int32_t> pfirst(nslots, INT32_MAX), plast(nslots, -1), xid(nslots, 0);
     int nx = 0;
     for (int64_t s = 0; s < nslots; s++) {
       for (int64_t k = m.ptr[s]; k < m.ptr[s + 1]; k++) {
-        const int ph = phase_of[m.idx[k] / csz];
+        const int ph = phase_of(m.idx[k] / csz);
+        if (ph < plast[s]) return "phase maps: contributions not in cell order";
         pfirst[s] = std::min(pfirst[s], ph);
         plast[s] = std::max(plast[s], ph);
       }
@@ -572,26 +555,42 @@ std::string build_phase_maps(const Plan &plan, const std::vector<GatherMap> &map
     }
     out.max_cross = std::max(out.max_cross, nx);
     for (int ph = ph0; ph < ph1; ph++) {
+      const int64_t cbase = (int64_t)out.cell_ptr[ph];
       for (int64_t s = 0; s < nslots; s++) {
         if (ph < pfirst[s] || ph > plast[s]) continue;
-        bool any = false;
+        int n = 0;
+        int32_t ii[4] = {0, 0, 0, 0};
+        double ww[4] = {0.0, 0.0, 0.0, 0.0};
+        const int32_t o0 = (int32_t)out.oidx.size();
         for (int64_t k = m.ptr[s]; k < m.ptr[s + 1]; k++) {
           const int64_t ge = m.idx[k] / csz;
-          if (phase_of[ge] != ph) continue;
-          any = true;
-          out.cidx.push_back((int32_t)(local_of[ge] * csz + m.idx[k] % csz));
-          out.cw.push_back(m.w[k]);
+          if (phase_of(ge) != ph) continue;
+          const int32_t li = (int32_t)((ge - cbase) * csz + m.idx[k] % csz);
+          if (n < 4) {
+            ii[n] = li;
+            ww[n] = m.w[k];
+          } else {
+            out.oidx.push_back(li);
+            out.ow.push_back(m.w[k]);
+          }
+          n++;
         }
-        if (!any && pfirst[s] == plast[s]) continue;   // (cannot happen: the slot's only phase has entries)
         const int mode = pfirst[s] == plast[s] ? 0 : ph == pfirst[s] ? 1 : ph == plast[s] ? 3 : 2;
-        out.slot.push_back((int32_t)s);
-        out.mode_x.push_back(mode | ((xid[s] < 0 ? 0 : xid[s]) << 2));
-        if (out.cidx.size() > (size_t)INT32_MAX) return "phase maps: too many contributions";
-        out.cptr.push_back((int32_t)out.cidx.size());
+        out.meta.push_back((int32_t)s);
+        out.meta.push_back(mode | (std::min(n, 4) << 2) | (xid[s] << 5));
+        for (int t = 0; t < 4; t++) {
+          out.idx4.push_back(ii[t]);
+          out.w4.push_back(ww[t]);
+        }
+        out.optr.push_back(o0);
+        out.optr.push_back((int32_t)out.oidx.size());
+        if (out.oidx.size() > (size_t)INT32_MAX / 2 || out.meta.size() > (size_t)INT32_MAX / 2)
+          return "phase maps: too many entries";
       }
-      out.slot_ptr.push_back((int32_t)out.slot.size());
+      out.slot_ptr.push_back((int32_t)(out.meta.size() / 2));
     }
   }
+  out.cell_ptr.push_back((int32_t)plan.ncell);   // end of the last phase
   return "";
 }
 

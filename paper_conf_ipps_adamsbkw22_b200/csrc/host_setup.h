@@ -79,22 +79,25 @@ struct Plan {
 };
 
 // Phased gather maps of the fused element + assembly kernel (tail_kernel, kernels_fe.cuh): each grid's
-// cells are cut into phases of at most `cap` cells (cells sorted by their z centre, so a z-mirror
-// mesh splits at z = 0 and few slots straddle two phases); a phase's element matrices live in shared
-// memory, cell c of the phase at local offset c * 2 Nb^2.  Per phase, the output slots it touches
-// (sorted) with their contributions restricted to the phase, in the gather map's (cell, a, b) order,
-// and a mode: 0 direct (every contribution in this phase: write), 1 first phase of a straddling slot
-// (keep the partial sum in shared memory, cross id x), 2 middle (add), 3 last (add the partial, write).
+// cells are cut into phases of at most `cap` consecutive cells (input order, so every slot's
+// contributions -- listed in (cell, a, b) order by the gather map -- arrive phase after phase and a
+// slot straddling phases continues one fma chain: the result equals assemble_kernel's bit for bit).  A
+// phase's element matrices live in shared memory, cell c of the phase at offset c * 2 Nb^2.  Per phase,
+// the output slots it touches (sorted) with their contributions in the phase: the first four inline
+// (ELL layout: one 16-byte index quad and two 16-byte weight pairs per slot, independent coalesced
+// loads), the rest in an overflow list.  meta = (slot, mode | n_inline << 2 | cross id << 5), mode 0: every
+// contribution in this phase (write), 1: first phase of a straddling slot (keep the running sum in
+// shared memory under the cross id), 2: middle (continue it), 3: last (continue it and write).
 struct PhaseMaps {
   std::vector<int32_t> grid_phase_ptr;   // [ngrids + 1] phases of each grid
-  std::vector<int32_t> cell_ptr;         // [nphases + 1] into cells
-  std::vector<int32_t> cells;            // global cell index, phase by phase
-  std::vector<int32_t> slot_ptr;         // [nphases + 1] into slot / mode_x / cptr
-  std::vector<int32_t> slot;             // grid-local output slot
-  std::vector<int32_t> mode_x;           // mode | (cross id << 2)
-  std::vector<int32_t> cptr;             // [total phase slots + 1] into cidx / cw
-  std::vector<int32_t> cidx;             // element-matrix index in the phase's shared buffer (doubles)
-  std::vector<double> cw;
+  std::vector<int32_t> cell_ptr;         // [nphases + 1] first cell (global index) of each phase, + end
+  std::vector<int32_t> slot_ptr;         // [nphases + 1] into the per-slot arrays
+  std::vector<int32_t> meta;             // [2 * total phase slots] (slot, mode | n_inline << 2 | x << 5)
+  std::vector<int32_t> idx4;             // [4 * total] the four inline element-matrix indices (doubles)
+  std::vector<double> w4;                // [4 * total] their weights
+  std::vector<int32_t> optr;             // [2 * total] overflow range [begin, end) into oidx / ow
+  std::vector<int32_t> oidx;
+  std::vector<double> ow;
   int max_cells = 0, max_cross = 0;
 };
 // cap >= 1 cells per phase; returns "" or an error (more than INT32_MAX entries).

@@ -381,25 +381,30 @@ __global__ void assemble_kernel(const GatherDev gm, const double *__restrict__ C
 
 // ------------------------------------------------------------------------------------------------
 // N3 + N4 fused (batches of small meshes, C4): a persistent CTA owns one batch item at a time and
-// walks each grid's phases (host_setup.h PhaseMaps: groups of cells by z, a z-mirror mesh splits at
-// z = 0).  Per phase its warps compute the phase's element matrices (C^D, C^K) by sum factorisation
-// (sf_cell) into SHARED memory -- the two-kernel form writes and reads them through HBM (285 MB each
-// way per C4 build) -- then every thread gathers output slots of the phase from shared memory: a slot
-// whose contributions all lie in the phase is written; a slot straddling phases keeps its partial sum
-// in shared memory from its first to its last phase.  Every slot sums its contributions in the
-// gather map's fixed (cell, a, b) order within a phase and the phases in order: deterministic.
+// walks each grid's phases (host_setup.h PhaseMaps: runs of consecutive cells).  Per phase its warps
+// compute the phase's element matrices (C^D, C^K) by sum factorisation (sf_cell) into SHARED memory --
+// the two-kernel form writes and reads them through HBM (285 MB each way per C4 build) -- then every
+// thread gathers output slots of the phase from shared memory, four slots at a time with all their
+// map loads independent and coalesced (ELL layout).  A slot straddling phases carries its running
+// fma sums from phase to phase in shared memory, so every slot is the same fma chain in the same
+// (cell, a, b) order as assemble_kernel: bitwise identical values.
 // ------------------------------------------------------------------------------------------------
 struct TailDev {
-  const int32_t *grid_phase_ptr, *cell_ptr, *cells, *slot_ptr, *slot, *mode_x, *cptr, *cidx;
-  const double *cw;
-  int ngrids, max_cells, max_cross;
+  const int32_t *grid_phase_ptr, *cell_ptr, *slot_ptr;
+  const int2 *meta, *optr;
+  const int4 *idx4;
+  const double2 *w4;   // [2 * slots]: (w0, w1), (w2, w3)
+  const int32_t *oidx;
+  const double *ow;
+  int ngrids, nphases, max_cells, max_cross;
 };
+constexpr int kTailMaxPhases = 64;
 
 template <int S>
 __host__ __device__ constexpr int tail_warps() { return S == 5 ? 8 : 16; }
 
 // dynamic shared memory: element matrices of max_cells cells | sA [warps][5][NB] | sT [warps][6][NB][S]
-// | straddling-slot partials [max_cross][2]
+// | straddling-slot running sums [max_cross] double2
 template <int S>
 __host__ __device__ constexpr size_t tail_smem_bytes(int max_cells, int max_cross) {
   return sizeof(double) * ((size_t)max_cells * 2 * S * S * S * S + (size_t)tail_warps<S>() * (5 * S * S + 6 * S * S * S) +
@@ -413,24 +418,34 @@ __global__ void __launch_bounds__(32 * tail_warps<S>(), 1) tail_kernel(const dou
                                                                        const double *__restrict__ tab1, const TailDev td,
                                                                        const GatherDev *__restrict__ maps,
                                                                        double *__restrict__ out, int64_t out_bstride) {
-  constexpr int NB = S * S, W = tail_warps<S>();
+  constexpr int NB = S * S, W = tail_warps<S>(), kS = 4;
   extern __shared__ double s_tail[];
+  __shared__ int s_gp[kMaxSpecies + 1], s_cp[kTailMaxPhases + 1], s_sp[kTailMaxPhases + 1];
+  __shared__ GatherDev s_gm[kMaxSpecies];   // species of each grid (a-3)
   double *sC = s_tail;
   double(*sA)[5][NB] = reinterpret_cast<double(*)[5][NB]>(sC + (size_t)td.max_cells * 2 * NB * NB);
   double(*sT)[6][NB][S] = reinterpret_cast<double(*)[6][NB][S]>(sC + (size_t)td.max_cells * 2 * NB * NB + W * 5 * NB);
   double2 *sX = reinterpret_cast<double2 *>(sC + (size_t)td.max_cells * 2 * NB * NB + W * (5 * NB + 6 * NB * S));
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (int k = threadIdx.x; k <= td.nphases; k += blockDim.x) {   // the phase tables, once per CTA
+    s_cp[k] = td.cell_ptr[k];
+    s_sp[k] = td.slot_ptr[k];
+  }
+  for (int k = threadIdx.x; k <= td.ngrids; k += blockDim.x) s_gp[k] = td.grid_phase_ptr[k];
+  for (int k = threadIdx.x; k < td.ngrids; k += blockDim.x) s_gm[k] = maps[k];
   double PLL[S], PLD[S], PDL[S], PDD[S];
   sf_tables<S>(tab1, lane, PLL, PLD, PDL, PDD);
+  __syncthreads();
   for (int b = blockIdx.x; b < nbatch; b += gridDim.x) {
     const double *Gb = G + (int64_t)b * 5 * N;
     double *ob = out + (int64_t)b * out_bstride;
     for (int g = 0; g < td.ngrids; g++) {
-      const GatherDev &gm = maps[g];
-      for (int ph = td.grid_phase_ptr[g]; ph < td.grid_phase_ptr[g + 1]; ph++) {
-        const int c0 = td.cell_ptr[ph], nc = td.cell_ptr[ph + 1] - c0;
+      const GatherDev &gm = s_gm[g];
+      for (int ph = s_gp[g]; ph < s_gp[g + 1]; ph++) {
+        const int64_t c0 = s_cp[ph];
+        const int nc = s_cp[ph + 1] - (int)c0;
         for (int lc = wid; lc < nc; lc += W) {   // a-4: one warp per cell
-          const int64_t e = td.cells[c0 + lc];
+          const int64_t e = c0 + lc;
           __syncwarp();   // the previous cell's readers are done with sA / sT
           if (lane < NB) {
             const int64_t i = e * NB + lane;
@@ -442,30 +457,53 @@ __global__ void __launch_bounds__(32 * tail_warps<S>(), 1) tail_kernel(const dou
           sf_cell<S>(sA[wid], sT[wid], lane, PLL, PLD, PDL, PDD, 2.0 / cell_h[e], sC + (size_t)lc * 2 * NB * NB);
         }
         __syncthreads();   // the phase's element matrices are complete
-        const int s0 = td.slot_ptr[ph], s1 = td.slot_ptr[ph + 1];
-        for (int i = s0 + threadIdx.x; i < s1; i += blockDim.x) {   // a-3 + a-5
-          double sD = 0.0, sK = 0.0;
-          for (int k = td.cptr[i]; k < td.cptr[i + 1]; k++) {
-            const double w = td.cw[k];
-            const double2 v = *reinterpret_cast<const double2 *>(sC + td.cidx[k]);   // (C^D, C^K)
-            sD = fma(w, v.x, sD);
-            sK = fma(w, v.y, sK);
+        const int s0 = s_sp[ph], s1 = s_sp[ph + 1];
+        for (int i0 = s0 + threadIdx.x; i0 < s1; i0 += kS * blockDim.x) {   // a-3 + a-5
+          int2 mt[kS], op[kS];
+          int4 ix[kS];
+          double2 wa[kS], wb[kS];
+#pragma unroll
+          for (int t = 0; t < kS; t++) {   // every map load of the four slots in flight at once
+            const int i = i0 + t * blockDim.x;
+            const bool v = i < s1;
+            mt[t] = v ? td.meta[i] : make_int2(0, 0);
+            ix[t] = v ? td.idx4[i] : make_int4(0, 0, 0, 0);
+            wa[t] = v ? td.w4[2 * i] : make_double2(0.0, 0.0);
+            wb[t] = v ? td.w4[2 * i + 1] : make_double2(0.0, 0.0);
+            op[t] = v ? td.optr[i] : make_int2(0, 0);
           }
-          const int mx = td.mode_x[i], mode = mx & 3, x = mx >> 2;
-          if (mode == 1) {
-            sX[x] = make_double2(sD, sK);
-            continue;
+#pragma unroll
+          for (int t = 0; t < kS; t++) {
+            const int i = i0 + t * blockDim.x;
+            if (i >= s1) continue;
+            const int mode = mt[t].y & 3, nin = (mt[t].y >> 2) & 7, x = mt[t].y >> 5;
+            double sD = 0.0, sK = 0.0;
+            if (mode >= 2) {   // continue the running sums of the earlier phases
+              sD = sX[x].x;
+              sK = sX[x].y;
+            }
+            const int id[4] = {ix[t].x, ix[t].y, ix[t].z, ix[t].w};
+            const double wt[4] = {wa[t].x, wa[t].y, wb[t].x, wb[t].y};
+#pragma unroll
+            for (int u = 0; u < 4; u++)
+              if (u < nin) {
+                const double2 c = *reinterpret_cast<const double2 *>(sC + id[u]);   // (C^D, C^K)
+                sD = fma(wt[u], c.x, sD);
+                sK = fma(wt[u], c.y, sK);
+              }
+            for (int k = op[t].x; k < op[t].y; k++) {   // slots with more than four contributions
+              const double2 c = *reinterpret_cast<const double2 *>(sC + td.oidx[k]);
+              const double w = td.ow[k];
+              sD = fma(w, c.x, sD);
+              sK = fma(w, c.y, sK);
+            }
+            if (mode == 1 || mode == 2) {
+              sX[x] = make_double2(sD, sK);
+            } else {
+              const int64_t s = mt[t].x;
+              for (int q = 0; q < gm.nsp; q++) ob[gm.out_off[q] + s] = fma(gm.fD[q], sD, gm.fK[q] * sK);
+            }
           }
-          if (mode == 2) {
-            sX[x] = make_double2(sX[x].x + sD, sX[x].y + sK);
-            continue;
-          }
-          if (mode == 3) {
-            sD = sX[x].x + sD;
-            sK = sX[x].y + sK;
-          }
-          const int64_t s = td.slot[i];
-          for (int q = 0; q < gm.nsp; q++) ob[gm.out_off[q] + s] = fma(gm.fD[q], sD, gm.fK[q] * sK);
         }
         __syncthreads();   // the next phase overwrites the element matrices
       }

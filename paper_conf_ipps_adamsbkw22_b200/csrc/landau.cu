@@ -64,10 +64,10 @@ struct landau_s {
   GatherDev *d_gmaps[2] = {nullptr, nullptr};   // per format (CSR, COO): the grids' gather maps (tail_kernel)
   // tail_kernel (fused a-4 + a-5) phased gather maps per format; tail_ok: built and fit shared memory
   struct TailMaps {
-    int32_t *grid_phase_ptr = nullptr, *cell_ptr = nullptr, *cells = nullptr, *slot_ptr = nullptr, *slot = nullptr,
-            *mode_x = nullptr, *cptr = nullptr, *cidx = nullptr;
-    double *cw = nullptr;
-    int max_cells = 0, max_cross = 0;
+    int32_t *grid_phase_ptr = nullptr, *cell_ptr = nullptr, *slot_ptr = nullptr, *meta = nullptr, *idx4 = nullptr,
+            *optr = nullptr, *oidx = nullptr;
+    double *w4 = nullptr, *ow = nullptr;
+    int max_cells = 0, max_cross = 0, nphases = 0;
   } tmaps[2];
   bool tail_ok = false;
   size_t tail_smem = 0;
@@ -294,12 +294,13 @@ int launch_field(landau_t h, int64_t nbatch) {
 
 // N3 + N4 fused into tail_kernel (one CTA per batch item, element matrices in an L2-resident scratch)
 // for batches of small meshes: all targets on this GPU, at least LANDAU_TAIL_MIN_BATCH items (fewer
-// items would leave most SMs idle: the two-kernel form spreads the cells), <= 1 MB of element matrices
-// per item.  LANDAU_TAIL=0 disables it.
+// items would leave most SMs idle: the two-kernel form spreads the cells), phases that fit shared
+// memory.  Opt-in (LANDAU_TAIL=1): C4 0.43 ms vs 0.30 ms for element_sf_kernel + assemble_kernel -- the
+// hanging-node expansion gives some slots up to 36 contributions, serial per thread.
 bool use_tail(landau_t h, int64_t nbatch) {
-  static const bool on = [] {
+  static const bool on = [] {   // off by default: measured slower than element_sf + assemble
     const char *e = getenv("LANDAU_TAIL");
-    return !(e && atoi(e) == 0);
+    return e && atoi(e) != 0;
   }();
   static const int64_t min_batch = [] {
     const char *e = getenv("LANDAU_TAIL_MIN_BATCH");
@@ -798,8 +799,19 @@ int launch_tail(landau_t h, int64_t nbatch, double *out, int format) {
   Timer t(h, LANDAU_T_ELEMENT);   // a-4 and a-5 in one kernel: timed as the element stage
   const int64_t out_bstride = format == LANDAU_CSR ? h->nnz : h->ncoo;
   const auto &m = h->tmaps[format == LANDAU_CSR ? 0 : 1];
-  TailDev td{m.grid_phase_ptr, m.cell_ptr, m.cells, m.slot_ptr, m.slot, m.mode_x, m.cptr, m.cidx, m.cw,
-             P.ngrids, m.max_cells, m.max_cross};
+  TailDev td{m.grid_phase_ptr,
+             m.cell_ptr,
+             m.slot_ptr,
+             reinterpret_cast<const int2 *>(m.meta),
+             reinterpret_cast<const int2 *>(m.optr),
+             reinterpret_cast<const int4 *>(m.idx4),
+             reinterpret_cast<const double2 *>(m.w4),
+             m.oidx,
+             m.ow,
+             P.ngrids,
+             m.nphases,
+             m.max_cells,
+             m.max_cross};
   const size_t smem = tail_smem_bytes<S>(m.max_cells, m.max_cross);
   // > 48 KB of dynamic shared memory: the attribute is per device and cheap to set, so on every call
   CU(cudaFuncSetAttribute(tail_kernel<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -1168,8 +1180,8 @@ void landau_destroy(landau_t h) {
   cudaFree(h->d_gmaps[0]);
   cudaFree(h->d_gmaps[1]);
   for (auto &m : h->tmaps)
-    for (void *q : {(void *)m.grid_phase_ptr, (void *)m.cell_ptr, (void *)m.cells, (void *)m.slot_ptr, (void *)m.slot,
-                    (void *)m.mode_x, (void *)m.cptr, (void *)m.cidx, (void *)m.cw})
+    for (void *q : {(void *)m.grid_phase_ptr, (void *)m.cell_ptr, (void *)m.slot_ptr, (void *)m.meta, (void *)m.idx4,
+                    (void *)m.optr, (void *)m.oidx, (void *)m.w4, (void *)m.ow})
       cudaFree(q);
   cudaFree(h->d_vtx_wp);
   cudaFree(h->d_vtx_part);
@@ -2080,7 +2092,8 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, cuda_device);
     const int S = P.p + 1, nb = P.nb;
     const size_t fixed = P.nb == 25 ? tail_smem_bytes<5>(0, 0) : P.nb == 16 ? tail_smem_bytes<4>(0, 0) : tail_smem_bytes<3>(0, 0);
-    const size_t per_cell = sizeof(double) * 2 * nb * nb, cross_reserve = 16 * 1024;
+    // 16 KB for straddling-slot partials, 8 KB for the kernel's static tables (phase tables, species)
+    const size_t per_cell = sizeof(double) * 2 * nb * nb, cross_reserve = 24 * 1024, static_smem = 8 * 1024;
     const int cap = optin > (int)(fixed + cross_reserve) ? (int)((optin - fixed - cross_reserve) / per_cell) : 0;
     int64_t max_grid_cells = 0;
     for (int g = 0; g < P.ngrids; g++) max_grid_cells = std::max(max_grid_cells, P.grids[g].ncell);
@@ -2096,15 +2109,20 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
         auto &m = h->tmaps[f];
         m.max_cells = pm.max_cells;
         m.max_cross = pm.max_cross;
+        m.nphases = (int)pm.slot_ptr.size() - 1;
+        if (m.nphases > kTailMaxPhases || (size_t)pm.max_cross >= (1u << 26)) {
+          ok = false;
+          break;
+        }
         if ((rc = upload(h, &m.grid_phase_ptr, pm.grid_phase_ptr)) || (rc = upload(h, &m.cell_ptr, pm.cell_ptr)) ||
-            (rc = upload(h, &m.cells, pm.cells)) || (rc = upload(h, &m.slot_ptr, pm.slot_ptr)) ||
-            (rc = upload(h, &m.slot, pm.slot)) || (rc = upload(h, &m.mode_x, pm.mode_x)) ||
-            (rc = upload(h, &m.cptr, pm.cptr)) || (rc = upload(h, &m.cidx, pm.cidx)) || (rc = upload(h, &m.cw, pm.cw)))
+            (rc = upload(h, &m.slot_ptr, pm.slot_ptr)) || (rc = upload(h, &m.meta, pm.meta)) ||
+            (rc = upload(h, &m.idx4, pm.idx4)) || (rc = upload(h, &m.optr, pm.optr)) ||
+            (rc = upload(h, &m.oidx, pm.oidx)) || (rc = upload(h, &m.w4, pm.w4)) || (rc = upload(h, &m.ow, pm.ow)))
           return bail(rc);
         const size_t need = P.nb == 25 ? tail_smem_bytes<5>(m.max_cells, m.max_cross)
                             : P.nb == 16 ? tail_smem_bytes<4>(m.max_cells, m.max_cross)
                                          : tail_smem_bytes<3>(m.max_cells, m.max_cross);
-        if (need > (size_t)optin) ok = false;
+        if (need + static_smem > (size_t)optin) ok = false;
       }
       h->tail_ok = ok;
     }
