@@ -292,7 +292,7 @@ int launch_field(landau_t h, int64_t nbatch) {
 }
 
 
-// N3 + N4 fused into tail_kernel (one CTA per batch item, element matrices in an L2-resident scratch)
+// N3 + N4 fused into tail_kernel (one CTA per batch item, each phase's element matrices in shared memory)
 // for batches of small meshes: all targets on this GPU, at least LANDAU_TAIL_MIN_BATCH items (fewer
 // items would leave most SMs idle: the two-kernel form spreads the cells), phases that fit shared
 // memory.  Opt-in (LANDAU_TAIL=1): C4 0.43 ms vs 0.30 ms for element_sf_kernel + assemble_kernel -- the

@@ -83,3 +83,74 @@ def test_element_split_and_sharding_gloo(name):
     for lo, hi in ranges:
         cover[lo:hi] += 1
     assert np.all(cover == 1)
+
+
+# ---------------------------------------------------------------------------------------------------
+# Pair split (LANDAU_DIST_ELEMENTS on a z-mirror mesh, the C5 path): rank r runs the slot kernel's items
+# (tile pairs a <= b of the upper half, U and V tensors, both directions) in its landau_pair_partition
+# range and reduces a partial G over ALL points; one all-reduce (sum) gives every rank the full G.
+# Here the oracle stands in for the kernels: a rank's partial G at a target t sums the sources in the
+# tiles its items pair with t's tile (upper points and their mirrors), and the gloo all-reduce of the
+# [5][N] partials must reproduce the oracle's full G.
+# ---------------------------------------------------------------------------------------------------
+def _mirror_tiles(r, z, grid_of_point):
+    """The library's upper-half ordering (landau_create / detect_mirror): per grid, the points with z > 0
+    sorted by (r, z), grids concatenated; tile = position // 32.  Returns the tile of every point (a
+    mirror point takes its partner's tile)."""
+    tile = np.full(r.size, -1)
+    pos = 0
+    for g in np.unique(grid_of_point):
+        up = [i for i in np.nonzero(grid_of_point == g)[0] if z[i] > 0]
+        up.sort(key=lambda i: (r[i], z[i]))
+        lo = {(r[i], z[i]): i for i in np.nonzero(grid_of_point == g)[0] if z[i] < 0}
+        for i in up:
+            tile[i] = pos // 32
+            tile[lo[(r[i], -z[i])]] = pos // 32
+            pos += 1
+    return tile, (pos + 31) // 32
+
+
+def _pair_split_worker(rank, port, out_q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=WORLD)
+    try:
+        from oracle.oracle import Oracle, inner
+        prob = inputs.config3()
+        o = Oracle(prob)
+        f = o.coefficients()
+        r, z, w = o.points()
+        TD, TKr, TKz = o.point_fields(f)
+        gop = np.repeat(np.arange(len(prob.grids)), [o.npoints // len(prob.grids)] * len(prob.grids))
+        tile, T = _mirror_tiles(r, z, gop)
+        q0, q1 = L.landau_pair_partition(T, WORLD, rank)
+        items = [(a, b) for b in range(T) for a in range(b + 1)][q0:q1]
+        partner = [set() for _ in range(T)]
+        for a, b in items:
+            partner[a].add(b)
+            partner[b].add(a)
+        part = np.zeros((5, o.npoints))
+        for A in range(T):
+            if not partner[A]:
+                continue
+            tg = np.nonzero(tile == A)[0]
+            src = np.isin(tile, sorted(partner[A]))
+            part[:, tg] = inner(r, z, w * src, TD, TKr, TKz, targets=tg)
+        t = torch.from_numpy(part)
+        dist.all_reduce(t)                      # the exchange step: sum of the ranks' partial G
+        counts = [None] * WORLD
+        dist.all_gather_object(counts, (q1 - q0, sum(1 if a == b else 2 for a, b in items)))
+        if rank == 0:
+            G, Ga = o.point_coeffs(f)
+            out_q.put((float(np.max(np.abs(t.numpy() - G) / Ga)), counts, T))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_pair_split_partials_allreduce_gloo():
+    ctx = mp.get_context("spawn")
+    q = ctx.SimpleQueue()
+    mp.start_processes(_pair_split_worker, args=(_free_port(), q), nprocs=WORLD, join=True, start_method="spawn")
+    err, counts, T = q.get()
+    assert sum(c for c, _ in counts) == T * (T + 1) // 2          # every tile pair exactly once
+    assert all(abs(wt - T * T / WORLD) <= 2 for _, wt in counts)   # balanced work (pair 2, diagonal 1)
+    assert err <= 1e-13, err
