@@ -671,12 +671,17 @@ def main():
     # ---- NEXT-3: quasi-Newton backward-Euler iterations on the same batch --------------------------
     if extras and nloc:
         try:
-            it_per_call = 2
+            it_per_call, dt_n = 2, 0.002
             Fn = torch.empty_like(F)
+            # the thermal-quench source of Eq. 4 (a cold pulse injecting 5x the initial density over 10
+            # steps, reading R-7): the first step's rate x each vertex's cold-Maxwellian shape
+            rate = 5.0 * inputs.quench_pulse_fraction(0.0, dt_n, 10 * dt_n) / dt_n
+            Src = torch.tensor(np.stack([rate * inputs.quench_source_shape(p, nodes) for p in items]), device="cuda")
             for _ in range(2):
-                h.implicit_step_batched(0.002, F, Fn, max_iter=it_per_call, rtol=0.0)
+                h.implicit_step_batched(dt_n, F, Fn, max_iter=it_per_call, rtol=0.0, src=Src)
             h.set_timing(True)
-            nts = timed_steps(torch, stream, lambda: h.implicit_step_batched(0.002, F, Fn, max_iter=it_per_call, rtol=0.0),
+            nts = timed_steps(torch, stream,
+                              lambda: h.implicit_step_batched(dt_n, F, Fn, max_iter=it_per_call, rtol=0.0, src=Src),
                               args.steps, flush)
             nt = h.get_timing()
             h.set_timing(False)
@@ -685,7 +690,8 @@ def main():
                 "value": total_builds / (ms_it / 1e3), "unit": "vertex Newton iterations/s", "ms_per_iteration": ms_it,
                 "stage_ms_per_iteration": {k: v[0] / (args.steps * it_per_call) for k, v in nt.items()},
                 "note": "SURVEY NEXT-3: backward-Euler step by quasi-Newton (Jacobian about each iterate, A = M/dt - J "
-                        "factored by the RCM band LU, solve), all vertices of the job per iteration, dt = 0.002, "
+                        "factored by the RCM band LU, solve) with the thermal-quench source of Eq. 4 (cold pulse, "
+                        "R-7), all vertices of the job per iteration, dt = 0.002, "
                         f"{it_per_call} iterations per landau_implicit_step_batched call; context: the paper's V100 "
                         "node figure is a different problem (10 species, 80 cells, CPU LU)"}
         except Exception as e:

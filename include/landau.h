@@ -223,6 +223,17 @@ int landau_advection(landau_t h, double Ez, double *values_dev, int32_t format);
  * The handle's state afterwards is the last iterate f^{k} the final Jacobian was built about. */
 int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
                                  double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm);
+/* The same step with the source term S_a(t) of Eq. 1 / Eq. 4 (PAPER.md:1@6337, @8216; the thermal-quench
+ * "pulse of cold ions ... injected with the source term in (4)", @34560): src_dev [nbatch][ndof]
+ * (device, species-major, may be NULL = no source) holds the FE coefficients sigma of S_a at t^{n+1};
+ * (psi_k, S_a) = (M sigma)_k with the mass matrix's weighted L2 product (Amb-2), so each iterate solves
+ *   (M/dt + E_z (e_a/m_a) A_E - J(f^k)) f^{k+1} = M (f^n / dt + sigma)
+ * and every iterate satisfies the per-species density balance
+ *   1^T [M (f^{k+1} - f^n)/dt + E_z (e_a/m_a) A_E f^{k+1}] = 1^T M sigma   (1^T J = 0).
+ * The time profile and shape of the source are the caller's (R-7).  Errors as above. */
+int landau_implicit_step_source_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
+                                        const double *src_dev, double *f_new_dev, int32_t max_iter, double rtol,
+                                        int32_t *iters, double *dnorm);
 
 /* Mirror symmetry (v_par -> -v_par, i.e. z -> -z): when every grid's quadrature points come in pairs
  * (r, z), (r, -z) BIT-EXACTLY (no point on z = 0; the dyadic meshes of every configuration of SURVEY

@@ -215,12 +215,14 @@ class Oracle:
         return np.concatenate([np.full(self.grid_ndof(int(g)), a, dtype=np.int64)
                                for a, g in enumerate(self.prob.grid_of)])
 
-    def implicit_step(self, f_old, dt, Ez=0.0, iters=4):
-        """Backward-Euler step of Eq. 4 (no source) by the paper's quasi-Newton iteration (@10500-10978):
-        with the Jacobian J(f^k) recomputed about the current iterate,
-            (M/dt + E_z (e_a/m_a) A_E - J(f^k)) f^{k+1} = M f^old / dt,
-        i.e. Newton on F(f) = M (f - f^old)/dt + E_z (e/m) A_E f - C(f) with the approximate Jacobian
-        M/dt + E_z (e/m) A_E - J(f^k) (C(f^k) = J(f^k) f^k, Amb-4).  A sparse direct solve (a library
+    def implicit_step(self, f_old, dt, Ez=0.0, iters=4, src=None):
+        """Backward-Euler step of Eq. 4 by the paper's quasi-Newton iteration (@10500-10978): with the
+        Jacobian J(f^k) recomputed about the current iterate,
+            (M/dt + E_z (e_a/m_a) A_E - J(f^k)) f^{k+1} = M f^old / dt + M sigma,
+        i.e. Newton on F(f) = M (f - f^old)/dt + E_z (e/m) A_E f - C(f) - (psi, S) with the approximate
+        Jacobian M/dt + E_z (e/m) A_E - J(f^k) (C(f^k) = J(f^k) f^k, Amb-4).  sigma: the FE coefficients
+        of the source S_a(t^{n+1}) of Eq. 1 / Eq. 4 (None: no source); (psi_k, S_a) = (M sigma)_k, the
+        weighted L2 product of the mass matrix (Amb-2, R-7).  A sparse direct solve (a library
         primitive) stands in for the paper's band LU.  Returns the iterates f^1..f^iters."""
         import scipy.sparse as sps
         import scipy.sparse.linalg as spla
@@ -231,6 +233,8 @@ class Oracle:
         eta = Ez * (np.asarray(self.prob.charge, float) / np.asarray(self.prob.mass, float))[self.species_rows()]
         Mm = sps.csr_matrix((M, col, rp), shape=(n, n))
         b = Mm @ np.asarray(f_old, float) / dt
+        if src is not None:
+            b = b + Mm @ np.asarray(src, float)
         f = np.array(f_old, dtype=np.float64)
         out = []
         for _ in range(iters):

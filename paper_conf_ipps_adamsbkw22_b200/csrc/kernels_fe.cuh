@@ -568,6 +568,13 @@ __global__ void __launch_bounds__(256) delta_norm_kernel(const double *__restric
   }
 }
 
+// NEXT-3: z = a x + y (the implicit step's f_old / dt + sigma)
+__global__ void axpby_kernel(int64_t n, double a, const double *__restrict__ x, const double *__restrict__ y,
+                             double *__restrict__ z) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    z[i] = fma(a, x[i], y[i]);
+}
+
 // N5: out[o0 + i] = shift * M[i]
 __global__ void scale_copy_kernel(const double *__restrict__ M, double shift, int64_t n, double *__restrict__ out) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)

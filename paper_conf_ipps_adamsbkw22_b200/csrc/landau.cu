@@ -77,6 +77,7 @@ struct landau_s {
   std::vector<int32_t *> d_col;
   // implicit step (NEXT-3) workspace
   double *d_Jwork = nullptr, *d_rhs = nullptr, *d_norms = nullptr, *h_norms = nullptr;
+  double *d_srcx = nullptr;   // f_old / dt + sigma (implicit step with a source)
   int64_t step_cap = 0;
   // device: state + workspace
   int64_t cap = 0, nbatch = 0, chunk = 1;
@@ -1203,6 +1204,7 @@ void landau_destroy(landau_t h) {
   cudaFree(h->d_Jwork);
   cudaFree(h->d_rhs);
   cudaFree(h->d_norms);
+  cudaFree(h->d_srcx);
   if (h->h_norms) cudaFreeHost(h->h_norms);
   for (auto &u : h->ev_used) {
     cudaEventDestroy(u.second.first);
@@ -1646,6 +1648,13 @@ int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, d
 
 int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
                                  double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm) {
+  return landau_implicit_step_source_batched(h, nbatch, dt, Ez, f_old_dev, nullptr, f_new_dev, max_iter, rtol, iters,
+                                             dnorm);
+}
+
+int landau_implicit_step_source_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
+                                        const double *src_dev, double *f_new_dev, int32_t max_iter, double rtol,
+                                        int32_t *iters, double *dnorm) {
   return guarded(h, [&]() -> int {
   if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
   if (!h || nbatch < 1 || !f_old_dev || !f_new_dev || f_old_dev == f_new_dev || max_iter < 1 || !(dt > 0))
@@ -1660,16 +1669,31 @@ int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double E
     CU(cudaMalloc(&h->d_rhs, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
     CU(cudaMalloc(&h->d_norms, sizeof(double) * 2 * nbatch));
     CU(cudaMallocHost(&h->h_norms, sizeof(double) * 2 * nbatch));
+    cudaFree(h->d_srcx);
+    h->d_srcx = nullptr;
+    CU(cudaMalloc(&h->d_srcx, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
     h->step_cap = nbatch;
   }
-  // rhs = M f_old / dt (species blocks), initial iterate f_old
+  // rhs = M f_old / dt (species blocks) or, with a source, M (f_old / dt + sigma) (Eq. 4's (psi, S_a) =
+  // M sigma, R-7); initial iterate f_old
+  const double *xin = f_old_dev;
+  double rscale = 1.0 / dt;
+  if (src_dev) {
+    const int64_t n = nbatch * h->ndof;
+    axpby_kernel<<<(unsigned)std::min<int64_t>((n + 255) / 256, 16LL * num_sms(h)), 256, 0, h->stream>>>(
+        n, 1.0 / dt, f_old_dev, src_dev, h->d_srcx);
+    h->launches++;
+    KCHECK();
+    xin = h->d_srcx;
+    rscale = 1.0;
+  }
   for (int a = 0; a < h->S; a++) {
     const int g = h->sgrid[a];
     const int n = h->plan.grids[g].ndof;
     if (!n) continue;
     const int64_t warps = nbatch * n;
     block_spmv_kernel<<<(unsigned)((warps * 32 + 255) / 256), 256, 0, h->stream>>>(
-        h->d_rowptr[g], h->d_col[g], h->d_mass_csr[g], n, h->soff[a], h->ndof, 1.0 / dt, f_old_dev, h->d_rhs,
+        h->d_rowptr[g], h->d_col[g], h->d_mass_csr[g], n, h->soff[a], h->ndof, rscale, xin, h->d_rhs,
         (int)nbatch);
     h->launches++;
     KCHECK();

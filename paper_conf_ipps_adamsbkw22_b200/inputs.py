@@ -216,6 +216,34 @@ def coefficients(prob: Problem, nodes_per_grid, with_noise: bool = True) -> np.n
 
 
 # ----------------------------------------------------------------------------------------------
+# NEXT-3 thermal-quench source S_a(t) of Eq. 1 / Eq. 4 (PAPER.md:1@6337, @8216): "a pulse of cold ions
+# is injected with the source term" (@34560), "the profile n_e is the prescribed sinusoidal source
+# function", "the total mass injected by the model is five times the initial density" (@35736).
+# Readings (R-7): every species is injected (quasi-neutral: electrons with the ions), as a
+# Maxwellian at the cold temperature Tc of the quench bulk, with the cumulative sinusoidal profile
+# P(t) = (1 - cos(pi t / t_pulse)) / 2 (0 -> 1 over the pulse); a backward-Euler step [t, t + dt]
+# injects (P(t + dt) - P(t)) of the total, so the injected amounts telescope exactly.
+# ----------------------------------------------------------------------------------------------
+def quench_pulse_fraction(t0: float, t1: float, t_pulse: float) -> float:
+    """Fraction of the pulse's total injection that falls in [t0, t1] (cumulative sinusoidal profile)."""
+    P = lambda t: 0.5 * (1.0 - math.cos(math.pi * min(max(t, 0.0), t_pulse) / t_pulse))
+    return P(t1) - P(t0)
+
+
+def quench_source_shape(prob: Problem, nodes_per_grid, Tc: float = 0.1, density=None) -> np.ndarray:
+    """FE coefficients (species-major, the caller's DOF numbering) of the cold Maxwellians a quench
+    pulse injects: species a at temperature Tc with density[a] (default: the initial density of the
+    species' recipe, sum of its Maxwellian components).  The step's source is sigma = fraction x
+    factor x shape (factor = 5 for the paper's five-fold injection)."""
+    out = []
+    for a, sp in enumerate(prob.species):
+        r, z = nodes_per_grid[sp.grid]
+        n = density[a] if density is not None else sum(c[0] for c in prob.fmix[a])
+        out.append(maxwellian(r, z, n, Tc, sp.mass))
+    return np.ascontiguousarray(np.concatenate(out), dtype=np.float64)
+
+
+# ----------------------------------------------------------------------------------------------
 # the five configurations of BASELINE.json (concretised in SURVEY.md §8(d))
 # ----------------------------------------------------------------------------------------------
 R_E = dyadic_radius(5.0 * VTH_E)   # 5 v_th,e (PAPER.md:1@26988), dyadic-rounded (exact mirror)

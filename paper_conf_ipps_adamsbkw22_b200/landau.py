@@ -93,6 +93,7 @@ def lib():
             "landau_band_factor_field_batched": (C.c_int, [vp, i64, d, d, vp]),
             "landau_advection": (C.c_int, [vp, d, vp, i32]),
             "landau_implicit_step_batched": (C.c_int, [vp, i64, d, d, vp, vp, i32, d, P32, Pd]),
+            "landau_implicit_step_source_batched": (C.c_int, [vp, i64, d, d, vp, vp, vp, i32, d, P32, Pd]),
             "landau_strerror": (C.c_char_p, [C.c_int]),
             "landau_last_error": (C.c_char_p, [vp]),
             "landau_version": (C.c_char_p, []),
@@ -367,15 +368,21 @@ class Landau:
                                            format), "landau_advection")
         return values
 
-    def implicit_step_batched(self, dt, f_old, f_new, Ez=0.0, max_iter=4, rtol=0.0):
-        """One backward-Euler step by quasi-Newton (include/landau.h); returns (iterations, max rel. change)."""
+    def implicit_step_batched(self, dt, f_old, f_new, Ez=0.0, max_iter=4, rtol=0.0, src=None):
+        """One backward-Euler step by quasi-Newton (include/landau.h); src: the FE coefficients of the
+        source S_a(t^{n+1}) (same shape as f_old) or None.  Returns (iterations, max rel. change)."""
         nb = self._nb(f_old)
         it, dn = C.c_int32(), C.c_double()
-        self._check(lib().landau_implicit_step_batched(self._h, nb, float(dt), float(Ez),
-                                                       self._dev(f_old, nb * self.ndof, "implicit_step f_old"),
-                                                       self._dev(f_new, nb * self.ndof, "implicit_step f_new"),
-                                                       int(max_iter), float(rtol), C.byref(it), C.byref(dn)),
-                    "landau_implicit_step_batched")
+        fo = self._dev(f_old, nb * self.ndof, "implicit_step f_old")
+        fn = self._dev(f_new, nb * self.ndof, "implicit_step f_new")
+        if src is None:
+            rc = lib().landau_implicit_step_batched(self._h, nb, float(dt), float(Ez), fo, fn, int(max_iter),
+                                                    float(rtol), C.byref(it), C.byref(dn))
+        else:
+            sp = self._dev(src, nb * self.ndof, "implicit_step src")
+            rc = lib().landau_implicit_step_source_batched(self._h, nb, float(dt), float(Ez), fo, sp, fn, int(max_iter),
+                                                           float(rtol), C.byref(it), C.byref(dn))
+        self._check(rc, "landau_implicit_step_batched")
         return it.value, dn.value
 
     def band_solve_batched(self, b, x):

@@ -586,6 +586,41 @@ def test_implicit_step_matches_oracle_iterates(cfg, dt, Ez):
         assert abs(dn - np.linalg.norm(its[k - 1] - prev) / np.linalg.norm(its[k - 1])) <= 1e-6 * dn
 
 
+@pytest.mark.parametrize("cfg,dt,Ez", [("C1", 0.05, 0.1), ("C2", 0.02, 0.0), ("C3", 0.01, 0.1)])
+def test_implicit_step_with_quench_source_matches_oracle(cfg, dt, Ez):
+    """NEXT-3 with the source S_a(t) of Eq. 4 (a cold Maxwellian pulse, reading R-7): every device
+    iterate equals the oracle's iterate with the same source (each side interpolates the shape at its
+    own DOF nodes), and the device iterate satisfies the per-species density balance
+    1^T [M (f^1 - f^0)/dt + eta A_E f^1] = 1^T M sigma."""
+    import scipy.sparse as sps
+    prob, h, o, fg, fo = setup(cfg)
+    frac = 5.0 * inputs.quench_pulse_fraction(0.0, dt, 4 * dt) / dt   # rate for the first step of a 4-step pulse
+    sig_o = frac * inputs.quench_source_shape(prob, o.all_nodes())
+    sig_g = frac * inputs.quench_source_shape(prob, h.all_nodes())
+    its = o.implicit_step(fo, dt, Ez, iters=2, src=sig_o)
+    f_old = torch.tensor(fg, device=DEV).reshape(1, -1)
+    f_new = torch.empty_like(f_old)
+    n_it, dn = h.implicit_step_batched(dt, f_old, f_new, Ez=Ez, max_iter=2, rtol=0.0,
+                                       src=torch.tensor(sig_g, device=DEV).reshape(1, -1))
+    torch.cuda.synchronize()
+    x = f_new.cpu().numpy()[0]
+    assert n_it == 2 and np.linalg.norm(x - its[1]) <= 1e-10 * np.linalg.norm(its[1])
+    M = torch.empty(h.nnz, dtype=torch.float64, device=DEV)
+    A = torch.empty(h.nnz, dtype=torch.float64, device=DEV)
+    h.mass(1.0, M)
+    h.advection(Ez, A)
+    rp, col = h.pattern()
+    Mm = sps.csr_matrix((M.cpu().numpy(), col, rp), shape=(h.ndof, h.ndof))
+    Am = sps.csr_matrix((A.cpu().numpy(), col, rp), shape=(h.ndof, h.ndof))
+    R = Mm @ (x - fg) / dt + Am @ x - Mm @ sig_g
+    start = 0
+    for sp in prob.species:
+        nd = h.grid_ndof(sp.grid)
+        sl = slice(start, start + nd)
+        assert abs(R[sl].sum()) <= 1e-12 * (np.abs(Mm) @ np.abs(x))[sl].sum() / dt
+        start += nd
+
+
 def test_implicit_step_converges_and_conserves_C4_batch():
     """Batched step over vertices with a tolerance: stops when every item's relative change <= rtol;
     the converged step conserves density, momentum and energy of every vertex (no field)."""

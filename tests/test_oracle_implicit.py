@@ -110,3 +110,63 @@ def test_P12_negative_control_first_iterate_not_converged():
     its = o.implicit_step(f0, 0.05, 0.0, iters=1)
     dens, mom, en = _balances(o, prob, f0, its[0], 0.05, 0.0)
     assert dens <= 1e-13 and en > 1e-8
+
+
+# ---------------------------------------------------------------------------------------------------
+# P14: the thermal-quench source S_a(t) of Eq. 1 / Eq. 4 (PAPER.md:1@6337, @8216, @34560, @35736)
+# ---------------------------------------------------------------------------------------------------
+def _source(o, prob, f0, t0, t1, t_pulse, factor=5.0):
+    """sigma for the step [t0, t1]: the cold-Maxwellian shape scaled so that the whole pulse injects
+    factor x the initial discrete density of each species (reading R-7), divided by the step."""
+    M, _ = _mats(o)
+    rows = o.species_rows()
+    shape = inputs.quench_source_shape(prob, o.all_nodes())
+    Ms, Mf0 = M @ shape, M @ f0
+    scale = np.array([Mf0[rows == a].sum() / Ms[rows == a].sum() for a in range(len(prob.species))])[rows]
+    return factor * inputs.quench_pulse_fraction(t0, t1, t_pulse) / (t1 - t0) * scale * shape
+
+
+@pytest.mark.parametrize("cfg,Ez", [("config1", 0.0), ("config3", 0.1)])
+def test_P14_source_density_balance_every_iterate(cfg, Ez):
+    """With the source, each quasi-Newton iterate satisfies the per-species density balance
+    1^T [M (f^{k+1} - f^n)/dt + eta A_E f^{k+1}] = 1^T M sigma exactly (1^T J = 0); without the source
+    term in the step the same balance misses by the injected amount (negative control)."""
+    prob = getattr(inputs, cfg)()
+    o = Oracle(prob)
+    f0 = o.coefficients()
+    dt = 0.02
+    sig = _source(o, prob, f0, 0.0, dt, 4 * dt)
+    M, A = _mats(o)
+    rows = o.species_rows()
+    eta = Ez * (np.asarray(prob.charge, float) / np.asarray(prob.mass, float))[rows]
+    Msig = M @ sig
+    for f in o.implicit_step(f0, dt, Ez, iters=3, src=sig):
+        R = M @ (f - f0) / dt + eta * (A @ f)
+        for a in range(len(prob.species)):
+            sel = rows == a
+            scale = (np.abs(M) @ (np.abs(f) + np.abs(f0)))[sel].sum() / dt
+            assert abs(R[sel].sum() - Msig[sel].sum()) <= 1e-13 * scale
+    f = o.implicit_step(f0, dt, Ez, iters=1)[0]
+    R = M @ (f - f0) / dt + eta * (A @ f)
+    assert abs(R[rows == 0].sum() - Msig[rows == 0].sum()) > 1e-3 * abs(Msig[rows == 0].sum())
+
+
+def test_P14_pulse_injects_five_times_the_initial_density():
+    """A whole pulse (4 backward-Euler steps, cumulative sinusoidal profile) injects exactly five times
+    each species' initial density (@35736: "the total mass injected by the model is five times the
+    initial density, which is observed to high accuracy"): with 1^T J = 0 and no field the discrete
+    density after the pulse is 6 x the initial one to roundoff, whatever the iterates' convergence."""
+    prob = inputs.config3()
+    o = Oracle(prob)
+    f = o.coefficients()
+    f0 = f.copy()
+    M, _ = _mats(o)
+    rows = o.species_rows()
+    dt, K = 0.01, 4
+    for n in range(K):
+        sig = _source(o, prob, f0, n * dt, (n + 1) * dt, K * dt)
+        f = o.implicit_step(f, dt, 0.0, iters=2, src=sig)[-1]
+    Mf0, Mf = M @ f0, M @ f
+    for a in range(len(prob.species)):
+        n0, n1 = Mf0[rows == a].sum(), Mf[rows == a].sum()
+        assert abs(n1 - 6.0 * n0) <= 1e-12 * n1, (a, n1 / n0)
