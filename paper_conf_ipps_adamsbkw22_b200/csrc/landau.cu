@@ -28,6 +28,7 @@ using namespace landau;
 #include "kernels_fe.cuh"
 #include "kernels_inner.cuh"
 #include "kernels_band.cuh"
+#include "kernels_single.cuh"
 #include "kernels_3d.cuh"
 
 
@@ -312,6 +313,9 @@ bool use_tail(landau_t h, int64_t nbatch) {
 
 int64_t tail_grid(landau_t h, int64_t nbatch) { return std::min<int64_t>(nbatch, num_sms(h)); }
 
+bool fused_single_enabled();
+bool fused_single_ok(landau_t h, int64_t nbatch);
+
 struct InnerPlan {
   bool vtx = false;    // mirror-symmetric per-vertex kernel, stream-K over (vertex, round) work
   bool sym;   // symmetric pair evaluation (whole point set as targets, enough tile pairs to fill the GPU)
@@ -433,9 +437,18 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
       const char *e = getenv("LANDAU_MDIR_SPLIT_MIN");
       return e ? (int64_t)atoll(e) : (int64_t)16;   // measured: 16 best on C2/C3 (finer splits cost reduction time)
     }();
-    const int64_t want = mdir_wps * num_sms(h);
-    int64_t nsplit = std::max<int64_t>(1, (want + T * nbatch - 1) / (T * nbatch));
-    nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, h->H / mdir_min));
+    // the fused single-build kernel wants one CTA item (a target tile and a group of 8 source splits)
+    // per SM; the stand-alone kernel LANDAU_MDIR_WARPS_PER_SM warps per SM with >= 16 sources per split
+    const bool fused = fused_single_ok(h, nbatch);
+    int64_t nsplit;
+    if (fused) {   // fused kernel: groups of 8 splits per CTA, one CTA item per SM, splits >= 8 sources
+      const int64_t ngroups = std::max<int64_t>(1, num_sms(h) / (T * nbatch));
+      nsplit = std::min<int64_t>(ngroups * kSbWarps, std::max<int64_t>(1, h->H / 8));
+    } else {
+      const int64_t want = mdir_wps * num_sms(h);
+      nsplit = std::max<int64_t>(1, (want + T * nbatch - 1) / (T * nbatch));
+      nsplit = std::min<int64_t>(nsplit, std::max<int64_t>(1, h->H / mdir_min));
+    }
     ip.split_len = (h->H + nsplit - 1) / nsplit;
     ip.nsplit = (h->H + ip.split_len - 1) / ip.split_len;
     if (ip.nsplit > 1) {
@@ -825,9 +838,93 @@ int launch_tail(landau_t h, int64_t nbatch, double *out, int format) {
   return LANDAU_OK;
 }
 
+// Whole small builds as ONE cooperative launch (kernels_single.cuh): the mirror-directed path of single
+// builds / tiny batches on Q2-Q3 meshes, CSR or COO, when no per-stage timers are requested.
+// LANDAU_FUSED_SINGLE=0 disables it.
+bool fused_single_enabled() {
+  static const bool v = [] {
+    const char *e = getenv("LANDAU_FUSED_SINGLE");
+    return !(e && atoi(e) == 0);
+  }();
+  return v;
+}
+
+bool fused_single_ok(landau_t h, int64_t nbatch) {
+  // latency-bound builds only: at most one target tile per SM (C2: up to 8 vertices)
+  return fused_single_enabled() && h->plan.nb <= 16 && !h->timing && !h->comm && !h->tcache && h->world == 1 &&
+         h->Nc == h->plan.npts && nbatch <= h->chunk && h->mirror && h->mirror_on &&
+         nbatch * ((h->H + 31) / 32) <= num_sms(h);
+}
+
+template <int NB>
+int launch_single(landau_t h, int64_t nbatch, const InnerPlan &ip, double *out, int format) {
+  if constexpr (NB > 16) {
+    return fail(h, LANDAU_EUNSUPPORTED, "fused single build: Q2/Q3 only");
+  } else {
+    const Plan &P = h->plan;
+    SingleBuildArgs a{};
+    a.ncell = P.ncell;
+    a.ndof_total = h->ndof;
+    a.nbatch = (int)nbatch;
+    a.f = h->fin ? h->fin : h->d_f;
+    a.ext_ptr = h->d_ext_ptr;
+    a.ext_dof = h->d_ext_dof;
+    a.ext_w = h->d_ext_w;
+    a.cell_grid = h->d_cell_grid;
+    a.cell_h = h->d_h;
+    a.pw = h->d_w;
+    a.tab = h->d_tab;
+    a.tab1 = h->d_tab + 3 * NB * NB;
+    a.sp = h->spc;
+    a.wT = h->d_wT;
+    a.npts = P.npts;
+    a.H = h->H;
+    a.T = ip.wtiles;
+    a.split_len = ip.split_len;
+    a.nsplit = (int)ip.nsplit;
+    a.rU = h->d_rU;
+    a.zU = h->d_zU;
+    a.pu = h->d_pu;
+    a.pm = h->d_pm;
+    a.G = h->d_G;
+    a.part = h->d_part;
+    a.Cbuf = h->d_C;
+    a.maps = h->d_gmaps[format == LANDAU_CSR ? 0 : 1];
+    a.ngrids = P.ngrids;
+    a.out = out;
+    a.out_bstride = format == LANDAU_CSR ? h->nnz : h->ncoo;
+    const int64_t inner_items = nbatch * ip.wtiles * ((ip.nsplit + kSbWarps - 1) / kSbWarps);   // CTA items
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(num_sms(h), inner_items));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(32 * kSbWarps);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = h->stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    CU(cudaLaunchKernelEx(&cfg, single_build_kernel<NB>, a));
+    h->launches++;
+    h->stats.nbatch = nbatch;
+    h->stats.targets = P.npts;
+    h->stats.sources = P.npts;
+    h->stats.inner_path = 5;
+    h->stats.nsplit = ip.nsplit;
+    h->stats.pair_evaluations = ip.wtiles * 32 * h->H * 2;
+    return LANDAU_OK;
+  }
+}
+
 template <int NB>
 int build_jacobian(landau_t h, int64_t nbatch, double *out, int format) {
   int rc;
+  if (out && fused_single_ok(h, nbatch)) {
+    InnerPlan ip;
+    if ((rc = inner_plan(h, nbatch, ip))) return rc;
+    if (ip.mdir && !ip.vtx && !ip.sym) return launch_single<NB>(h, nbatch, ip, out, format);
+  }
   if ((rc = launch_field<NB>(h, nbatch))) return rc;
   if ((rc = launch_inner(h, nbatch))) return rc;
   if (!out) return LANDAU_OK;   // point_coeffs: G only
