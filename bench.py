@@ -63,7 +63,7 @@ def parse(argv=None):
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="landau", choices=["landau", "reference"])
-    ap.add_argument("--workload", default="C4", choices=["C4", "C1", "C2", "C3", "C5"])
+    ap.add_argument("--workload", default="C4", choices=["C4", "C1", "C2", "C3", "C5", "C2ncu"])
     ap.add_argument("--batch", type=int, default=1024, help="C4 vertices in the whole job (--weak: per GPU)")
     ap.add_argument("--weak", action="store_true", help="C4: --batch vertices per GPU instead of in the whole job")
     ap.add_argument("--no-cpu-baseline", action="store_true")

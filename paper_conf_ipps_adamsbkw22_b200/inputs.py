@@ -300,7 +300,16 @@ def config5() -> Problem:
     return p
 
 
-CONFIGS = {"C1": config1, "C2": config2, "C3": config3, "C5": config5}
+def config2ncu() -> Problem:
+    """C2-ncu: the C2 problem on its mesh refined uniformly once (272 cells, N = 4,352),
+    the analogue of the paper's 320-cell problem sized to fill the GPU for Nsight Compute (@40473)."""
+    p = config2()
+    p.name = "C2ncu"
+    p.grids = [(R_E, refine_uniform(c2_mesh(), 1))]
+    return p
+
+
+CONFIGS = {"C1": config1, "C2": config2, "C3": config3, "C5": config5, "C2ncu": config2ncu}
 
 
 # ------------------------------------------------------------------------------------------------
