@@ -1,0 +1,4 @@
+for F in 1 0; do for B in 1024 128; do
+LANDAU_FIELD_VTX=$F timeout 300 python bench.py --batch $B --no-sublines --no-cpu-baseline 2>/dev/null | python -c "import json,sys; d=json.loads(sys.stdin.read().strip().splitlines()[-1]); print('FV$F B$B', round(d['value']), round(d['ms_per_step'],4), round(d['roofline']['frac'],3), {k: round(v,4) for k,v in d['stage_ms_per_step'].items() if v})"
+done; done
+timeout 900 python -m pytest tests/ -x -q -m gpu 2>&1 | tail -3
