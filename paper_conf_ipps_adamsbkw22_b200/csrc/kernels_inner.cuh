@@ -624,6 +624,19 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
   __shared__ double2 s_ltab[kLogTab];
   __shared__ int s_last;
   extern __shared__ double s_G[];   // Ga [5][Hp], Gb [5][Hp] | staged vertex [Hp][5] double2 | pu, pm [Hp]
+#ifdef LANDAU_VTX_TRACE   // build variant: per-CTA timeline (globaltimer ns) printed at exit (scripts/vtx_trace.py)
+  unsigned long long tr_[24];
+  int ntr_ = 0;
+#define VTX_MARK(tag)                                                                                   \
+  if (threadIdx.x == 0 && ntr_ < 24) {                                                                  \
+    unsigned long long t_;                                                                              \
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                                              \
+    tr_[ntr_++] = (t_ << 4) | (tag);                                                                    \
+  }
+#else
+#define VTX_MARK(tag)
+#endif
+  VTX_MARK(0);
   const int64_t Hp = (H + 31) / 32 * 32;
   double *sGa = s_G, *sGb = s_G + 5 * Hp;
   double2 *s_V = reinterpret_cast<double2 *>(s_G + 10 * Hp);
@@ -646,6 +659,7 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
   const int c = blockIdx.x;
   const int64_t f0 = vtx_first_round(sc, wp, c), f1 = vtx_first_round(sc, wp, c + 1);
   int64_t f = f0;
+  VTX_MARK(1);
   while (f < f1) {
     const int64_t v = f / sc.nrounds;
     const int rd0 = (int)(f - v * sc.nrounds);
@@ -670,6 +684,7 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
     }
     for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) s_G[k] = 0.0;
     __syncthreads();
+    VTX_MARK(2);
     for (int rd = rd0; rd < rd1; rd++) {
       for (int q = round_ptr[rd] + wid; q < round_ptr[rd + 1]; q += kVtxWarps) {
         const VtxItem it = items[q];
@@ -684,6 +699,7 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
       }
       __syncthreads();   // the next round's tiles may be this round's
     }
+    VTX_MARK(3);
     const int cfirst = vtx_owner(sc, wp, v, 0), clast = vtx_owner(sc, wp, v, sc.nrounds - 1);
     if (cfirst == clast) {   // the whole vertex ran here
       vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, s_pu, s_pm);
@@ -722,10 +738,19 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
         __syncthreads();
         vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, s_pu, s_pm);
         if (threadIdx.x == 0) counters[v] = 0;   // ready for the next build
+        VTX_MARK(5);
       }
     }
     __syncthreads();   // the write-out reads s_G (and items read s_V) before the next segment rewrites them
+    VTX_MARK(4);
   }
+#ifdef LANDAU_VTX_TRACE
+  if (threadIdx.x == 0) {
+    unsigned smid_;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid_));
+    for (int i = 0; i < ntr_; i++) printf("VTX %d %d %llu %llu %u\n", c, i, tr_[i] & 15, tr_[i] >> 4, smid_);
+  }
+#endif
 }
 
 // ------------------------------------------------------------------------------------------------
