@@ -1,7 +1,12 @@
 # small workloads for compute-sanitizer: every kernel of the library on C1, C3 and a 16-vertex C4 batch
 # (symmetric, mirror-slot, per-vertex and mirror-directed inner kernels; band LU, solve and the implicit
-# step; the 3D Cartesian inner integral; one emulated rank of the pair split)
+# step with and without the quench source; the 3D Cartesian inner integral; one emulated rank of the pair
+# split), the fused single-build kernel (C1, C3 without timers), the element/assembly kernels (timed
+# builds), and a 200-vertex batch (more vertices than SMs: the per-vertex kernel loops over several
+# vertices per CTA and splits some between CTAs).  Argument "tail": LANDAU_TAIL=1 (the fused tail kernel).
 import os, sys
+if len(sys.argv) > 1 and sys.argv[1] == "tail":
+    os.environ["LANDAU_TAIL"] = "1"
 sys.path.insert(0, os.getcwd())
 import numpy as np, torch
 from paper_conf_ipps_adamsbkw22_b200 import inputs
@@ -17,6 +22,10 @@ for name in ("C1", "C3"):
         h.mass(2.0, v, fmt)
     G = torch.empty((5, h.npoints), dtype=torch.float64, device="cuda")
     h.point_coeffs(G)
+    h.set_timing(True)   # the multi-kernel single build (field, mdir, reduce, element, assemble)
+    v = torch.empty(h.nnz, dtype=torch.float64, device="cuda")
+    h.jacobian(v)
+    h.set_timing(False)
 p0 = inputs.config4_vertex(0)
 h = L.Landau.from_problem(p0, device=0)
 nodes = h.all_nodes()
@@ -40,8 +49,19 @@ b = torch.randn((16, h.ndof), dtype=torch.float64, device="cuda"); x = torch.emp
 h.band_solve_batched(b, x)
 fn = torch.empty_like(F)
 h.implicit_step_batched(0.002, F, fn, Ez=0.1, max_iter=2)
+src = torch.tensor(np.stack([inputs.quench_source_shape(inputs.config4_vertex(b), nodes) for b in range(16)]), device="cuda")
+h.implicit_step_batched(0.002, F, fn, Ez=0.1, max_iter=2, src=src)
 torch.cuda.synchronize()
 print("ok")
+# more vertices than SMs: several vertices per CTA, some split between CTAs (automatic mode)
+h.set_mirror(True)
+nb = 200
+F2 = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in range(nb)]), device="cuda")
+h.set_state_batched(F2)
+v2 = torch.empty((nb, h.nnz), dtype=torch.float64, device="cuda")
+h.jacobian_batched(v2)
+torch.cuda.synchronize()
+print("stats 200", h.stats(), "split", len(h.vtx_split_vertices(nb)))
 # NEXT-4: the 3D Cartesian inner integral (split-j and direct)
 xyz3, w3 = inputs.points3d(2, 2)
 wTD3, wTK3 = inputs.fields3d(xyz3, w3)

@@ -47,10 +47,17 @@ def main():
         J = run(h, fg)
         Jo, Ja = o.jacobian(fo)
         d, m, e = _conservation(prob, h, J, fg)
-        rep[cfg] = {"G_err_over_Gabs": float(np.max(np.abs(G - Go) / Ga)),
+        eg = np.abs(G - Go) / Ga
+        worst = np.unravel_index(int(np.argmax(eg)), eg.shape)
+        r, z, _ = h.points()
+        rep[cfg] = {"G_err_over_Gabs": float(eg.max()),
+                    "G_worst_point": {"component": int(worst[0]), "r": float(r[worst[1]]), "z": float(z[worst[1]]),
+                                      "r_over_R": float(r[worst[1]] / prob.grids[0][0])},
                     "J_err_over_Jabs": float(np.max(np.abs(J - Jo) / Ja)),
                     "J_maxerr_over_maxJ": float(np.abs(J - Jo).max() / np.abs(Jo).max()),
-                    "conservation": {"density": d, "momentum": m, "energy": e}, "kernel": "directed (single build)"}
+                    "conservation": {"density": d, "momentum": m, "energy": e},
+                    "kernel": ["directed", "symmetric", "tensor cache", "mirror slot", "per-vertex",
+                               "mirror-directed (single build: one cooperative kernel)"][h.stats()["inner_path"]]}
     # C4 batch on the mirror slot kernel and on the per-vertex kernel (the headline path)
     for mode, key in (("slots", "C4_batch64_mirror_slots"), ("vertex", "C4_batch64_vertex")):
         nb = 64
@@ -75,6 +82,27 @@ def main():
             worst["conservation_max"] = max(worst["conservation_max"],
                                             max(_conservation(probs[k], h, Jb[k], inputs.coefficients(probs[k], nodes))))
         rep[key] = dict(worst, vertices_checked=[verts[k] for k in (0, 21, 42, 63)])
+    # the headline batch: 1024 vertices in automatic mode (per-vertex kernel, stream-K)
+    nb = 1024
+    prob0 = inputs.config4_vertex(0, nb)
+    h = L.Landau.from_problem(prob0, device=0)
+    nodes = h.all_nodes()
+    F = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b, nb), nodes) for b in range(nb)]), device=DEV)
+    h.set_state_batched(F)
+    out = torch.empty((nb, h.nnz), dtype=torch.float64, device=DEV)
+    h.jacobian_batched(out)
+    Jb = out.cpu().numpy()
+    split = set(int(x) for x in h.vtx_split_vertices(nb))
+    sample = [0, 148, 500, 1023] + sorted(split)[:2]
+    worst = {"J_err_over_Jabs": 0.0, "conservation_max": 0.0, "inner_path": h.stats()["inner_path"]}
+    for b in sample:
+        o = Oracle(inputs.config4_vertex(b, nb))
+        Jo, Ja = o.jacobian(o.coefficients())
+        worst["J_err_over_Jabs"] = max(worst["J_err_over_Jabs"], float(np.max(np.abs(Jb[b] - Jo) / Ja)))
+        worst["conservation_max"] = max(worst["conservation_max"],
+                                        max(_conservation(inputs.config4_vertex(b, nb), h, Jb[b],
+                                                          inputs.coefficients(inputs.config4_vertex(b, nb), nodes))))
+    rep["C4_headline_1024"] = dict(worst, vertices_checked=sample, vertices_split_between_ctas=len(split))
     # C5 sampled cells
     prob = inputs.config5()
     h = L.Landau.from_problem(prob, device=0)
@@ -82,7 +110,7 @@ def main():
     fg, fo = inputs.coefficients(prob, h.all_nodes()), o.coefficients()
     rng = np.random.default_rng(2022)
     ncell = len(prob.grids[0][1])
-    cells = np.sort(rng.choice(ncell, 8, replace=False))
+    cells = np.sort(rng.choice(ncell, 32, replace=False))
     nqp = (prob.order + 1) ** 2
     targets = (cells[:, None] * nqp + np.arange(nqp)[None, :]).ravel()
     G = run(h, fg, G=True)
