@@ -1132,3 +1132,17 @@ def test_fused_tail_kernel_equals_two_kernel_path(fmt, tmp_path):
     o = Oracle(inputs.config4_vertex(verts[7]))
     Jo, Ja = o.jacobian(o.coefficients()) if fmt == L.LANDAU_CSR else o.jacobian_coo(o.coefficients())
     assert np.all(np.abs(Jt[7] - Jo) <= 1e-11 * Ja)
+
+
+def test_rz_cancellation_stress_uniform_density():
+    """The two tensor components whose azimuthal integrands change sign (U^D_rz, U^K_zr) are the only
+    ones whose GPU error grows beyond roundoff of G^abs (profiles/r02_parity_analysis.md): with a
+    uniform density (f = 1 on every DOF, G_rz a sum of nearly cancelling ring integrals) the C2 G_D,rz
+    error reaches ~7e-13 G^abs, still inside the 1e-12 parity bound, while rr, zz and both K
+    components stay at roundoff."""
+    prob, h, o, fg, fo = setup("C2")
+    G = gpu_G(h, np.ones_like(fg))
+    Go, Ga = o.point_coeffs(np.ones_like(fo))
+    e = np.max(np.abs(G - Go) / Ga, axis=1)
+    assert e[1] <= 1e-12, e
+    assert e[0] <= 1e-14 and e[2] <= 1e-14 and e[3] <= 1e-14 and e[4] <= 1e-14, e
