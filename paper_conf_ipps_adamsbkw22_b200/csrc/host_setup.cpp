@@ -397,6 +397,53 @@ std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, c
           cm.push_back(v);
         }
       }
+      // connected grids up to 2048 DOFs: the Cuthill-McKee order from EVERY root, keep the smallest
+      // bandwidth (George-Liu's pseudo-peripheral root is a heuristic: 81 on the C2/C4 grid against
+      // 78 for the best root, and the band kernel's window is B + 2 rounded up to 8: 88 -> 80, 17%
+      // fewer FLOP per step).  A root is abandoned as soon as its partial order reaches the best B.
+      if ((int)cm.size() == n && n > 1 && n <= 2048 && !getenv("LANDAU_RCM_PERIPHERAL")) {
+        std::vector<int> sadj(G.col.size());   // neighbours by (degree, id), self excluded below
+        for (int i = 0; i < n; i++) {
+          std::copy(G.col.begin() + G.rowptr[i], G.col.begin() + G.rowptr[i + 1], sadj.begin() + G.rowptr[i]);
+          std::sort(sadj.begin() + G.rowptr[i], sadj.begin() + G.rowptr[i + 1],
+                    [&](int a, int b) { return deg[a] != deg[b] ? deg[a] < deg[b] : a < b; });
+        }
+        auto band_of = [&](const std::vector<int> &ord, std::vector<int> &pos) {
+          for (int k = 0; k < n; k++) pos[ord[k]] = k;
+          int b = 0;
+          for (int i = 0; i < n; i++)
+            for (int64_t q = G.rowptr[i]; q < G.rowptr[i + 1]; q++) b = std::max(b, std::abs(pos[i] - pos[G.col[q]]));
+          return b;
+        };
+        std::vector<int> pos(n, -1), ord, best = cm;
+        int bestB = band_of(cm, pos);
+        ord.reserve(n);
+        for (int root = 0; root < n; root++) {
+          std::fill(pos.begin(), pos.end(), -1);
+          ord.clear();
+          ord.push_back(root);
+          pos[root] = 0;
+          bool cut = false;
+          for (size_t h = 0; h < ord.size() && !cut; h++) {
+            const int u = ord[h];
+            for (int64_t q = G.rowptr[u]; q < G.rowptr[u + 1]; q++) {
+              const int v = sadj[q];
+              if (pos[v] >= 0) continue;
+              pos[v] = (int)ord.size();
+              ord.push_back(v);
+              // u is v's lowest-placed neighbour (BFS), so this edge is v's widest to the front
+              if (pos[v] - (int)h >= bestB) {
+                cut = true;
+                break;
+              }
+            }
+          }
+          if (cut || (int)ord.size() != n) continue;
+          bestB = band_of(ord, pos);
+          best = ord;
+        }
+        cm = best;
+      }
       G.rcm_perm.assign(cm.rbegin(), cm.rend());
       G.rcm_iperm.assign(n, 0);
       for (int k = 0; k < n; k++) G.rcm_iperm[G.rcm_perm[k]] = k;

@@ -1688,7 +1688,11 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
     h->launches++;
     KCHECK();
   }
-  const int threads_lu = std::max(64, (std::max((maxPp / (maxPp <= 88 ? 4 : 8)) * (maxPp / 8), 2 * maxPp - 1) + 31) / 32 * 32);
+  // threads: the tile owners, the 2B + 1 factor-row writers, and enough to stage one group's entering
+  // entries kBandE per thread (threads past the tiles own none and only stage and write)
+  const int tiles_lu = (maxPp / (maxPp <= 88 ? 4 : 8)) * (maxPp / 8);
+  const int stage_lu = (h->band_ent_max + kBandE - 1) / kBandE;
+  const int threads_lu = std::min(256, std::max(64, (std::max(std::max(tiles_lu, 2 * maxPp - 1), stage_lu) + 31) / 32 * 32));
   if (h->band_ent_max > kBandE * threads_lu) return fail(h, LANDAU_EUNSUPPORTED, "band factor: too many entries per row group");
   const unsigned grid = (unsigned)(nbatch * h->S);
   static const int band_minb = [] {
