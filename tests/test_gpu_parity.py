@@ -230,6 +230,7 @@ def test_launch_counter_and_timers():
     h.set_timing(True)
     gpu_jacobian(h, fg)
     t = h.get_timing()
+    h.set_timing(False)   # the cached handle goes back to the untimed (fused single-build) path
     assert h.launch_count() > n0
     assert t["inner"][1] == 1 and t["inner"][0] > 0
 
@@ -240,15 +241,26 @@ def test_element_split_mode_single_rank():
     prob, h, o, fg, fo = setup("C2")
     dist = {"rank": 0, "world": 1, "mode": L.LANDAU_DIST_ELEMENTS, "nccl_unique_id": L.landau_nccl_unique_id()}
     hd = L.Landau.from_problem(prob, device=0, dist=dist)
+    # a handle with a communicator never runs the fused single-build kernel: compare with the plain
+    # handle's multi-kernel build (stage timers on select it), bit for bit, and with its fused build
+    # within rounding (the fused kernel groups the source splits differently)
+    h.set_timing(True)
     a = gpu_jacobian(h, fg)
+    h.set_timing(False)
+    a_fused = gpu_jacobian(h, fg)
     b = gpu_jacobian(hd, fg)
     assert np.array_equal(a.view(np.uint64), b.view(np.uint64))
+    _, Ja = o.jacobian(fo)
+    assert np.max(np.abs(a_fused - b) / Ja) <= 1e-14
     hd.set_timing(True)
     gpu_jacobian(hd, fg)
     tm = hd.get_timing()
     assert tm["allgather"][1] == 1 and tm["allgather"][0] > 0.0   # one timed exchange step per build
     Gd = gpu_G(hd, fg)
-    assert np.array_equal(Gd, gpu_G(h, fg))
+    h.set_timing(True)   # the split rule of the multi-kernel build, as on the communicator handle
+    Gh = gpu_G(h, fg)
+    h.set_timing(False)
+    assert np.array_equal(Gd, Gh)
 
 
 @pytest.mark.parametrize("cfg,fmt", [("C1", L.LANDAU_CSR), ("C2", L.LANDAU_CSR), ("C3", L.LANDAU_CSR), ("C2", L.LANDAU_COO)])
