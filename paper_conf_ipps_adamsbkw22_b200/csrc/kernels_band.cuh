@@ -289,6 +289,247 @@ __global__ void __launch_bounds__(256, MINB) band_lu2_kernel(const double *__res
   }
 }
 
+// ---- column-warp factorisation with look-ahead (round 2) ------------------------------------------
+// The same outer-product band LU (Golub-Van Loan Alg. 4.3.1, rank-1 steps) and the same step-major
+// factor rows as band_lu2_kernel, with the P x P window (P = 8 NC, a template constant) distributed so
+// that the per-step synchronisation is a producer/consumer hand-off instead of a CTA barrier:
+//   * warp w owns the physical columns w + 8 c (c < NC: cyclic, so consecutive pivots belong to
+//     different warps); lane l owns the physical rows l + 32 m (m < MR = ceil(P / 32)):
+//     cell[m][c] = window(l + 32 m, w + 8 c);
+//   * step k (pivot at physical index pk = k mod P) needs the multipliers l_k (P values) from the
+//     warp owning column pk, and the pivot row's values in each warp's own columns, which the warp's
+//     lane pk mod 32 holds -- so only l_k crosses warps, through a shared-memory ring, guarded by the
+//     named barrier 1 + k mod 9: its producer bar.arrive()s, the other warps bar.sync();
+//   * look-ahead: during step k the owner of column pk + 1 applies step k to that column first, forms
+//     l_{k+1} = column / pivot and publishes it before updating its other columns, so the next step's
+//     hand-off overlaps the current step's rank-1 update;
+//   * every 8 steps one CTA barrier stages the next group's entering rows (dense, indexed by physical
+//     position, three sets) and writes the previous group's factor rows from the l / u rings
+//     (coalesced); it also bounds how far any warp runs ahead (9 barrier ids, 16 ring slots suffice).
+// Retiring row pk: l_k = 0 there, so the update leaves the entering row (written just before) intact;
+// retiring column pk: updated like the others, then overwritten by the entering column.
+constexpr int kCwRing = 16;   // ring slots of l_k / row-k values (>= 8 steps of a group + look-ahead + lag)
+
+__device__ __forceinline__ void named_sync(int id, int cnt) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(cnt) : "memory"); }
+__device__ __forceinline__ void named_arrive(int id, int cnt) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(cnt) : "memory"); }
+
+template <int NC>
+__global__ void __launch_bounds__(256, 2) band_lu_cw_kernel(const double *__restrict__ Aent, int64_t ent_bstride,
+                                                            double *__restrict__ LU, int64_t lu_bstride,
+                                                            const BandDesc *__restrict__ desc, int nsp) {
+  constexpr int P = 8 * NC, W = 2 * P - 1, MR = (P + 31) / 32, T = 256;
+  extern __shared__ double smem[];
+  const int bi = blockIdx.x / nsp, a = blockIdx.x % nsp;
+  const BandDesc d = desc[a];   // d.B + 1 == P (host-checked)
+  const int n = d.n;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  double *Lr = smem;                      // [kCwRing][P] l_k by physical row (0 at the pivot row)
+  double *Ur = Lr + kCwRing * P;          // [kCwRing][P] row k, warp-major: column w + 8 c at w NC + c
+  double *eb = Ur + kCwRing * P;          // [3][8][2P] entering rows: row part [0, P) warp-major, column part [P, 2P)
+  const double *ae = Aent + (int64_t)bi * ent_bstride + d.aoff;
+  double *lu = LU + (int64_t)bi * lu_bstride + d.off;
+  const int ngroups = (n + 7) / 8;
+  for (int i = tid; i < 3 * 16 * P; i += T) eb[i] = 0.0;
+  // an entry of group g (entering rows 8g..8g+7): its dense index from the band_lu2 position code
+  // (ri 4P + (row part: p | column part: 2P + p - P)), whose logical index is ni + p - 2B - 1 (column
+  // part) or ni + p - B (row part) with B = P - 1, i.e. physical (ni + p + 1) mod P either way
+  auto stage = [&](int g, double *v, int *ix) {
+#pragma unroll
+    for (int m = 0; m < kBandE; m++) {
+      v[m] = 0.0;
+      ix[m] = -1;
+    }
+    if (g >= ngroups) return;
+    const int q0 = d.ent_ptr[8 * g], q1 = d.ent_ptr[min(8 * g + 8, n)];
+#pragma unroll
+    for (int m = 0; m < kBandE; m++) {
+      const int q = q0 + tid + m * T;
+      if (q < q1) {
+        const int code = d.ent_pos[q];
+        const int ri = code / (4 * P), qq = code - ri * 4 * P;
+        const bool isrow = qq < P;
+        const int pp = isrow ? qq : qq - P;
+        const int phys = (8 * g + ri + pp + 1) % P;   // row part stored warp-major: (phys % 8) NC + phys / 8
+        ix[m] = ri * 2 * P + (isrow ? (phys & 7) * NC + (phys >> 3) : P + phys);
+        v[m] = ae[q];
+      }
+    }
+  };
+  double vin[kBandE];
+  int vix[kBandE];
+  __syncthreads();
+  for (int g0 = 0; g0 < 2; g0++) {   // groups 0 and 1 into sets 0 and 1; group 2 waits in registers
+    stage(g0, vin, vix);
+#pragma unroll
+    for (int m = 0; m < kBandE; m++)
+      if (vix[m] >= 0) eb[g0 * 16 * P + vix[m]] = vin[m];
+  }
+  stage(2, vin, vix);
+  // factor rows of steps [k0, k0 + 8) from the rings: t < P: U(k, k + t), t >= P: L(k + t - P + 1, k)
+  auto write_rows = [&](int k0) {
+    for (int r = 0; r < 8; r++) {
+      const int kk = k0 + r;
+      if (kk < 0 || kk >= n) continue;
+      const int pkk = kk % P, sl = kk & (kCwRing - 1);
+      for (int t = tid; t < W; t += T) {
+        int j = pkk + (t < P ? t : t - P + 1);
+        j -= j >= P ? P : 0;
+        lu[(int64_t)kk * W + t] = t < P ? Ur[sl * P + (j & 7) * NC + (j >> 3)] : Lr[sl * P + j];
+      }
+    }
+  };
+  auto group_barrier = [&](int g, int kb) {   // stage group g + 1, clear set (g + 2) % 3, rows of group g - 1
+    __syncthreads();
+#pragma unroll
+    for (int m = 0; m < kBandE; m++)
+      if (vix[m] >= 0) eb[((g + 1) % 3) * 16 * P + vix[m]] = vin[m];
+    double2 *cs = reinterpret_cast<double2 *>(eb + ((g + 2) % 3) * 16 * P);
+    for (int i = tid; i < 8 * P; i += T) cs[i] = make_double2(0.0, 0.0);
+    stage(g + 2, vin, vix);
+    write_rows(kb - 8);
+    __syncthreads();
+  };
+
+  double cell[MR][NC];
+#pragma unroll
+  for (int m = 0; m < MR; m++)
+#pragma unroll
+    for (int c = 0; c < NC; c++) cell[m][c] = 0.0;
+  const int c0 = w * NC;   // this warp's segment of a warp-major row (Ur, entering row parts)
+  // the pivot row's values of this warp's columns -> ring slot sl (lane rl of slot rm holds them)
+  // (16-byte accesses for even NC: c0, the ring rows and the dense rows are 16-byte aligned)
+  auto put_row = [&](double *dst, int rl, int rm) {
+#pragma unroll
+    for (int m = 0; m < MR; m++)
+      if (m == rm && lane == rl) {
+        if constexpr (NC % 2 == 0) {
+#pragma unroll
+          for (int c = 0; c < NC; c += 2) reinterpret_cast<double2 *>(dst)[c / 2] = make_double2(cell[m][c], cell[m][c + 1]);
+        } else {
+#pragma unroll
+          for (int c = 0; c < NC; c++) dst[c] = cell[m][c];
+        }
+      }
+  };
+  auto take_row = [&](const double *src, int rl, int rm) {   // the entering row into lane rl, slot rm
+#pragma unroll
+    for (int m = 0; m < MR; m++)
+      if (m == rm && lane == rl) {
+        if constexpr (NC % 2 == 0) {
+#pragma unroll
+          for (int c = 0; c < NC; c += 2) {
+            const double2 v = reinterpret_cast<const double2 *>(src)[c / 2];
+            cell[m][c] = v.x;
+            cell[m][c + 1] = v.y;
+          }
+        } else {
+#pragma unroll
+          for (int c = 0; c < NC; c++) cell[m][c] = src[c];
+        }
+      }
+  };
+  auto take_col = [&](const double *src, int oc, int pk) {    // the entering column into column oc
+#pragma unroll
+    for (int c = 0; c < NC; c++)
+      if (c == oc) {
+#pragma unroll
+        for (int m = 0; m < MR; m++) {
+          const int row = lane + 32 * m;
+          if ((m < MR - 1 || row < P) && row != pk) cell[m][c] = src[row];
+        }
+      }
+  };
+  // l_{k+1} from column pn (physical) with step k applied: multipliers l, the old pivot row's value at
+  // column pn from lane rl (slot rm), whose row is the entering row from this step on (value ev)
+  auto produce = [&](const double *l, int pn, int rl, int rm, double ev, double *dst) {
+    const int nc = pn >> 3;
+#pragma unroll
+    for (int c = 0; c < NC; c++)
+      if (c == nc) {
+        double uv = cell[0][c];
+#pragma unroll
+        for (int m = 1; m < MR; m++) uv = rm == m ? cell[m][c] : uv;
+        uv = __shfl_sync(0xffffffffu, uv, rl);
+        double t[MR];
+#pragma unroll
+        for (int m = 0; m < MR; m++) t[m] = (m == rm && lane == rl) ? ev : fma(-l[m], uv, cell[m][c]);
+        const int prm = pn >> 5;
+        double tv = t[0];
+#pragma unroll
+        for (int m = 1; m < MR; m++) tv = prm == m ? t[m] : tv;
+        const double pv = __shfl_sync(0xffffffffu, tv, pn & 31);
+        const double r = rcp_newton(pv);
+#pragma unroll
+        for (int m = 0; m < MR; m++) {
+          const int row = lane + 32 * m;
+          if (m < MR - 1 || row < P) dst[row] = row == pn ? 0.0 : t[m] * r;
+        }
+      }
+  };
+
+  // ---- steps k = -P .. -1: the first P rows / columns enter the window; l_0 at the end ----
+  int pk = 0, g = 0;
+  for (int kb = -P; kb < 0; kb += 8, g++) {
+    if (g > 0) group_barrier(g, kb);
+    else __syncthreads();
+    const double *es = eb + (g % 3) * 16 * P;
+#pragma unroll 1
+    for (int u = 0; u < 8; u++, pk++) {   // pk = k + P < P
+      take_row(es + u * 2 * P + c0, pk & 31, pk >> 5);
+      if (w == (pk & 7)) take_col(es + u * 2 * P + P, pk >> 3, pk);
+    }
+  }
+  pk = 0;
+  if (w == 0 && n > 0) {   // l_0 (column 0 belongs to warp 0); nothing to apply yet
+    const double z[MR] = {};
+    produce(z, 0, 32, MR, 0.0, Lr);
+    __syncwarp();
+    named_arrive(1, T);
+  }
+  // ---- steps k = 0 .. n - 1 ----
+  int bid = 1;   // named barrier of step k: 1 + k mod 9
+  for (int kb = 0; kb < n; kb += 8, g++) {
+    group_barrier(g, kb);
+    const double *es = eb + (g % 3) * 16 * P;
+#pragma unroll 1
+    for (int u = 0; u < 8; u++) {
+      const int k = kb + u;
+      if (k >= n) break;
+      const int ow = pk & 7, oc = pk >> 3;         // owner warp / column slot of the retiring column
+      const int rl = pk & 31, rm = pk >> 5;        // owner lane / slot of the retiring row
+      const int sl = k & (kCwRing - 1);
+      const int pn = pk + 1 == P ? 0 : pk + 1;
+      const int bid1 = bid == 9 ? 1 : bid + 1;
+      if (w != ow) named_sync(bid, T);
+      double l[MR], uu[NC];
+#pragma unroll
+      for (int m = 0; m < MR; m++) {
+        const int row = lane + 32 * m;
+        l[m] = (m < MR - 1 || row < P) ? Lr[sl * P + row] : 0.0;
+      }
+      if (k + 1 < n && w == (pn & 7)) {   // look-ahead first: l_{k+1} (the next step's only hand-off)
+        produce(l, pn, rl, rm, es[u * 2 * P + (pn & 7) * NC + (pn >> 3)], Lr + ((k + 1) & (kCwRing - 1)) * P);
+        __syncwarp();
+        named_arrive(bid1, T);
+      }
+      put_row(Ur + sl * P + c0, rl, rm);
+      __syncwarp();
+#pragma unroll
+      for (int c = 0; c < NC; c++) uu[c] = Ur[sl * P + c0 + c];
+      take_row(es + u * 2 * P + c0, rl, rm);   // the entering row k + P takes physical row pk
+#pragma unroll
+      for (int m = 0; m < MR; m++)             // rank-1 update (column pn again: the same fma)
+#pragma unroll
+        for (int c = 0; c < NC; c++) cell[m][c] = fma(-l[m], uu[c], cell[m][c]);
+      if (w == ow) take_col(es + u * 2 * P + P, oc, pk);   // the entering column k + P
+      pk = pn;
+      bid = bid1;
+    }
+  }
+  __syncthreads();
+  write_rows(8 * ((n - 1) / 8));   // the last group's rows
+}
+
 // One warp per (batch item, species block): x = U^-1 L^-1 (P b) in the RCM order, un-permuted on
 // the way out.  y lives in shared memory; the factor rows stream through a per-warp cp.async ring
 // kBandD steps ahead (each step is a short dependent chain, so the loads must not sit on it).

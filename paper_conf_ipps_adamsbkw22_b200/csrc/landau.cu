@@ -1699,9 +1699,26 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
     const char *e = getenv("LANDAU_BAND_MINB");
     return e ? atoi(e) : 2;
   }();
+  static const bool band_cw = [] {   // opt-in: the column-warp kernel measured slower
+    const char *e = getenv("LANDAU_BAND_CW");
+    return e && atoi(e) != 0;
+  }();
   const void *kfn;
-  const size_t ksmem = smem;
-  if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
+  size_t ksmem = smem;
+  unsigned threads = (unsigned)threads_lu;
+  bool same_p = true;
+  for (auto &d : h->band_desc) same_p = same_p && d.Pp == maxPp;
+  static const void *const cw_kernels[12] = {
+      (const void *)band_lu_cw_kernel<1>, (const void *)band_lu_cw_kernel<2>,  (const void *)band_lu_cw_kernel<3>,
+      (const void *)band_lu_cw_kernel<4>, (const void *)band_lu_cw_kernel<5>,  (const void *)band_lu_cw_kernel<6>,
+      (const void *)band_lu_cw_kernel<7>, (const void *)band_lu_cw_kernel<8>,  (const void *)band_lu_cw_kernel<9>,
+      (const void *)band_lu_cw_kernel<10>, (const void *)band_lu_cw_kernel<11>, (const void *)band_lu_cw_kernel<12>};
+  if (band_cw && same_p && maxPp <= 96 && maxPp % 8 == 0 && h->band_ent_max <= kBandE * 256) {
+    // column-warp kernel with look-ahead: 8 warps of P / 8 columns (one window width per launch)
+    kfn = cw_kernels[maxPp / 8 - 1];
+    ksmem = sizeof(double) * (2 * kCwRing + 48) * maxPp;
+    threads = 256;
+  } else if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
     kfn = band_minb >= 2 ? (const void *)band_lu2_kernel<4, 8, 2> : (const void *)band_lu2_kernel<4, 8, 1>;
   else               // 8 x 8 tiles, <= 256 threads
     kfn = (const void *)band_lu2_kernel<8, 8, 1>;
@@ -1715,7 +1732,7 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
     const BandDesc *a4 = h->d_band_desc;
     int a5 = h->S;
     void *args[] = {&a0, &a1, &a2, &a3, &a4, &a5};
-    CU(cudaLaunchKernel(kfn, dim3(grid), dim3(threads_lu), args, ksmem, h->stream));
+    CU(cudaLaunchKernel(kfn, dim3(grid), dim3(threads), args, ksmem, h->stream));
   }
   h->launches++;
   h->tlaunch[LANDAU_T_FACTOR]++;

@@ -1158,3 +1158,59 @@ def test_rz_cancellation_stress_uniform_density():
     e = np.max(np.abs(G - Go) / Ga, axis=1)
     assert e[1] <= 1e-12, e
     assert e[0] <= 1e-14 and e[2] <= 1e-14 and e[3] <= 1e-14 and e[4] <= 1e-14, e
+
+
+_BAND_CHILD = r'''
+import os, sys, numpy as np, torch
+sys.path.insert(0, os.getcwd())
+from paper_conf_ipps_adamsbkw22_b200 import inputs
+from paper_conf_ipps_adamsbkw22_b200 import landau as L
+path, nb = sys.argv[1], int(sys.argv[2])
+h = L.Landau.from_problem(inputs.config4_vertex(0), device=0)
+nodes = h.all_nodes()
+F = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in range(0, 1024, 1024 // nb)]),
+                 device="cuda")
+h.set_state_batched(F)
+J = torch.empty((nb, h.nnz), dtype=torch.float64, device="cuda")
+h.jacobian_batched(J)
+Mv = torch.empty(h.nnz, dtype=torch.float64, device="cuda")
+h.mass(1.0, Mv)
+shift = float(J.abs().max()) / float(Mv.abs().max())
+h.band_factor_batched(shift, J)
+b = torch.tensor(np.random.default_rng(5).standard_normal((nb, h.ndof)), device="cuda")
+x = torch.empty_like(b)
+h.band_solve_batched(b, x)
+np.savez(path, x=x.cpu().numpy(), b=b.cpu().numpy(), J=J.cpu().numpy(), shift=shift)
+'''
+
+
+def test_band_column_warp_kernel_matches():
+    """The opt-in column-warp band factorisation (LANDAU_BAND_CW=1: warps own cyclic columns, the
+    multipliers handed over through named barriers, look-ahead on the next pivot column) solves the
+    same C4 systems as the default register-tile kernel: both agree with a sparse direct solve of the
+    same A = shift M - J (the rank-1 and rank-2 eliminations round differently)."""
+    import os
+    import subprocess
+    import sys
+    import tempfile
+    import scipy.sparse as sps
+    import scipy.sparse.linalg as spla
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = {}
+    with tempfile.TemporaryDirectory() as td:
+        for cw in ("1", "0"):
+            path = os.path.join(td, f"x{cw}.npz")
+            out = subprocess.run([sys.executable, "-c", _BAND_CHILD, path, "4"], capture_output=True, text=True,
+                                 timeout=600, cwd=root, env=dict(os.environ, LANDAU_BAND_CW=cw))
+            assert out.returncode == 0, out.stderr[-3000:]
+            res[cw] = dict(np.load(path))
+    o = Oracle(inputs.config4_vertex(0))
+    rp, col = o.pattern()
+    M = o.mass(1.0)
+    for k in range(4):
+        J = res["0"]["J"][k]
+        assert np.array_equal(J, res["1"]["J"][k])
+        A = sps.csr_matrix((res["0"]["shift"] * M - J, col, rp), shape=(o.ndof, o.ndof))
+        x_ref = spla.spsolve(A.tocsc(), res["0"]["b"][k])
+        for cw in ("0", "1"):
+            assert np.max(np.abs(res[cw]["x"][k] - x_ref)) <= 1e-10 * np.max(np.abs(x_ref))
