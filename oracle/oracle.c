@@ -1039,3 +1039,330 @@ int oracle_get_threads(void) {
   return 1;
 #endif
 }
+
+/* ------------------------------------------------------------------------------------------ */
+/* O13 (SURVEY §8(f) NEXT-4 completed: "a full 3D model is supported in the library"           */
+/* @7997-8072): the Landau Jacobian in 3D Cartesian velocity space -- O1-O8 and O10 with the    */
+/* tensor of O12, on a uniform grid of ncell^3 Q_p cubes over [-R, R]^3 (no hanging nodes, no   */
+/* r weight: the Cartesian weak form of Eq. 4 @8216-8560 is int psi ... dv over R^3):           */
+/*   DOFs   the lattice of M = ncell p + 1 equispaced nodes per direction,                      */
+/*          dof(ix, iy, iz) = (iz M + iy) M + ix at (-R + ix h/p, -R + iy h/p, -R + iz h/p)      */
+/*   points (p+1)^3 Gauss-Legendre points per cube, w = w_a w_b w_c (h/2)^3                     */
+/*   O3/O4  T_D = sum_b e_b^2 f_b, T_K = sum_b e_b^2 (m0/m_b) grad f_b at every point            */
+/*   O12    G_D(i) = sum_{j: v_j != v_i} w_j T_D(j) U(v_i - v_j), G_K(i) = sum_j U w_j T_K(j)      */
+/*   O6/O7  C_e[k][l] = sum_q w_q (grad phi_k . D~ grad phi_l + (grad phi_k . K~) phi_l),       */
+/*          D~ = -nu e_a^2 (m0/m_a)^2 G_D, K~ = nu e_a^2 (m0/m_a) G_K (the forms of Eqs. 5-6)    */
+/*   O8     J_a = sum_e C_e added at (dof_k, dof_l), species-block-diagonal, CSR rows sorted      */
+/*   O10    the same with every product in absolute value (fields from |phi| |f|)               */
+/* ------------------------------------------------------------------------------------------ */
+/* 1D: the lattice indices sharing a cube with lattice index i: [lo, hi] */
+static void o3_range(int ncell, int p, long long i, long long *lo, long long *hi) {
+  long long c0 = i / p, c1 = c0;
+  if (i % p == 0 && c0 > 0) c0--;  /* a cube boundary node belongs to the cubes on both sides */
+  if (c1 >= ncell) c1 = ncell - 1;
+  *lo = c0 * p;
+  *hi = (c1 + 1) * p;
+}
+
+void oracle3d_sizes(int ncell, int order, long long *ndof, long long *npoints, long long *nnz) {
+  long long M = (long long)ncell * order + 1, s = 0;
+  for (long long i = 0; i < M; i++) {
+    long long lo, hi;
+    o3_range(ncell, order, i, &lo, &hi);
+    s += hi - lo + 1;
+  }
+  if (ndof) *ndof = M * M * M;
+  if (npoints) *npoints = (long long)ncell * ncell * ncell * (order + 1) * (order + 1) * (order + 1);
+  if (nnz) *nnz = s * s * s; /* the pattern is the tensor product of the 1D ones */
+}
+
+void oracle3d_pattern(int ncell, int order, long long *rowptr, int *col) {
+  long long M = (long long)ncell * order + 1, k = 0;
+  rowptr[0] = 0;
+  for (long long iz = 0; iz < M; iz++)
+    for (long long iy = 0; iy < M; iy++)
+      for (long long ix = 0; ix < M; ix++) {
+        long long lx, hx, ly, hy, lz, hz;
+        o3_range(ncell, order, ix, &lx, &hx);
+        o3_range(ncell, order, iy, &ly, &hy);
+        o3_range(ncell, order, iz, &lz, &hz);
+        for (long long jz = lz; jz <= hz; jz++)
+          for (long long jy = ly; jy <= hy; jy++)
+            for (long long jx = lx; jx <= hx; jx++) col[k++] = (int)((jz * M + jy) * M + jx);
+        rowptr[(iz * M + iy) * M + ix + 1] = k;
+      }
+}
+
+void oracle3d_nodes(int ncell, int order, double R, double *xyz) {
+  long long M = (long long)ncell * order + 1, nd = M * M * M;
+  ld d = 2.0L * (ld)R / ((ld)ncell * order);
+  for (long long iz = 0; iz < M; iz++)
+    for (long long iy = 0; iy < M; iy++)
+      for (long long ix = 0; ix < M; ix++) {
+        long long k = (iz * M + iy) * M + ix;
+        xyz[k] = (double)(-(ld)R + ix * d);
+        xyz[nd + k] = (double)(-(ld)R + iy * d);
+        xyz[2 * nd + k] = (double)(-(ld)R + iz * d);
+      }
+}
+
+static long long o3_find(const long long *rowptr, const int *col, long long row, int c) {
+  long long lo = rowptr[row], hi = rowptr[row + 1] - 1;
+  while (lo <= hi) {
+    long long mid = (lo + hi) / 2;
+    if (col[mid] == c) return mid;
+    if (col[mid] < c) lo = mid + 1;
+    else hi = mid - 1;
+  }
+  return -1;
+}
+
+/* the grid: points (coordinates, weights), reference basis at the Gauss points, cube DOFs */
+typedef struct {
+  int p, s1, nb, nq, ncell;
+  long long M, nc3, ndof, N, nnz;
+  ld h, s; /* cube side, 2 / h */
+  double *x, *y, *z;
+  ld *w;
+  ld *bas;        /* [q][n][phi, d/dx, d/dy, d/dz] (physical gradients) */
+  long long *dofs; /* [cube][nb] */
+} o3grid_t;
+
+static void o3_grid(int ncell, int order, double R, o3grid_t *g) {
+  const int p = order, s1 = p + 1, nb = s1 * s1 * s1;
+  g->p = p;
+  g->s1 = s1;
+  g->nb = nb;
+  g->nq = nb;
+  g->ncell = ncell;
+  g->M = (long long)ncell * p + 1;
+  g->nc3 = (long long)ncell * ncell * ncell;
+  oracle3d_sizes(ncell, order, &g->ndof, &g->N, &g->nnz);
+  g->h = 2.0L * (ld)R / ncell;
+  g->s = 2.0L / g->h;
+  ld xg[8], wg[8];
+  gauss_legendre(s1, xg, wg);
+  g->x = malloc(sizeof(double) * 3 * g->N);
+  g->y = g->x + g->N;
+  g->z = g->x + 2 * g->N;
+  g->w = malloc(sizeof(ld) * g->N);
+  g->bas = malloc(sizeof(ld) * 4 * (size_t)nb * nb);
+  g->dofs = malloc(sizeof(long long) * g->nc3 * nb);
+  for (int qa = 0; qa < s1; qa++) /* Gauss index along z, y, x */
+    for (int qb = 0; qb < s1; qb++)
+      for (int qc = 0; qc < s1; qc++) {
+        int q = (qa * s1 + qb) * s1 + qc;
+        for (int k = 0; k < s1; k++)
+          for (int j = 0; j < s1; j++)
+            for (int i = 0; i < s1; i++) {
+              int n = (k * s1 + j) * s1 + i;
+              ld Lx = lag(p, i, xg[qc]), Ly = lag(p, j, xg[qb]), Lz = lag(p, k, xg[qa]);
+              ld *b = g->bas + 4 * ((size_t)q * nb + n);
+              b[0] = Lx * Ly * Lz;
+              b[1] = g->s * dlag(p, i, xg[qc]) * Ly * Lz;
+              b[2] = g->s * Lx * dlag(p, j, xg[qb]) * Lz;
+              b[3] = g->s * Lx * Ly * dlag(p, k, xg[qa]);
+            }
+      }
+  for (long long cz = 0; cz < ncell; cz++)
+    for (long long cy = 0; cy < ncell; cy++)
+      for (long long cx = 0; cx < ncell; cx++) {
+        long long c = (cz * ncell + cy) * ncell + cx;
+        for (int k = 0; k < s1; k++)
+          for (int j = 0; j < s1; j++)
+            for (int i = 0; i < s1; i++)
+              g->dofs[c * nb + (k * s1 + j) * s1 + i] = ((cz * p + k) * g->M + (cy * p + j)) * g->M + (cx * p + i);
+        for (int qa = 0; qa < s1; qa++)
+          for (int qb = 0; qb < s1; qb++)
+            for (int qc = 0; qc < s1; qc++) {
+              long long pt = c * g->nq + (qa * s1 + qb) * s1 + qc;
+              g->x[pt] = (double)(-(ld)R + g->h * cx + 0.5L * g->h * (xg[qc] + 1.0L));
+              g->y[pt] = (double)(-(ld)R + g->h * cy + 0.5L * g->h * (xg[qb] + 1.0L));
+              g->z[pt] = (double)(-(ld)R + g->h * cz + 0.5L * g->h * (xg[qa] + 1.0L));
+              g->w[pt] = wg[qa] * wg[qb] * wg[qc] * (0.5L * g->h) * (0.5L * g->h) * (0.5L * g->h);
+            }
+      }
+}
+
+static void o3_free(o3grid_t *g) {
+  free(g->x);
+  free(g->w);
+  free(g->bas);
+  free(g->dofs);
+}
+
+/* O3, O4 at every point: T[8][N] = T_D, T_Kx, T_Ky, T_Kz (not multiplied by w), then the |.| versions */
+static void o3_fields(const o3grid_t *g, int S, const double *mass, const double *charge, const double *f, ld *T) {
+  const long long N = g->N;
+  for (long long k = 0; k < 8 * N; k++) T[k] = 0.0L;
+#pragma omp parallel for schedule(static)
+  for (long long pt = 0; pt < N; pt++) {
+    long long c = pt / g->nq;
+    int q = (int)(pt % g->nq);
+    for (int a = 0; a < S; a++) {
+      ld e2 = (ld)charge[a] * (ld)charge[a], im = 1.0L / (ld)mass[a];
+      ld v[4] = {0, 0, 0, 0}, va[4] = {0, 0, 0, 0};
+      for (int n = 0; n < g->nb; n++) {
+        ld fv = f[(long long)a * g->ndof + g->dofs[c * g->nb + n]];
+        const ld *b = g->bas + 4 * ((size_t)q * g->nb + n);
+        for (int t = 0; t < 4; t++) {
+          v[t] += b[t] * fv;
+          va[t] += fabsl(b[t]) * fabsl(fv);
+        }
+      }
+      T[pt] += e2 * v[0];
+      T[4 * N + pt] += e2 * va[0];
+      for (int t = 1; t < 4; t++) {
+        T[t * N + pt] += e2 * im * v[t];
+        T[(4 + t) * N + pt] += e2 * im * va[t];
+      }
+    }
+  }
+}
+
+/* O12 at every point: G[18][N] = signed sums from w T, then |.| sums from w |T|^abs */
+static void o3_inner(const o3grid_t *g, const ld *T, ld *G) {
+  const long long N = g->N;
+  const double *x = g->x, *y = g->y, *z = g->z;
+#pragma omp parallel for schedule(dynamic, 8)
+  for (long long i = 0; i < N; i++) {
+    nsum_t acc[9], aac[9];
+    memset(acc, 0, sizeof acc);
+    memset(aac, 0, sizeof aac);
+    for (long long j = 0; j < N; j++) {
+      if (x[j] == x[i] && y[j] == y[i] && z[j] == z[i]) continue; /* Amb-3 */
+      const ld u[3] = {(ld)x[i] - x[j], (ld)y[i] - y[j], (ld)z[i] - z[j]};
+      const ld s2 = u[0] * u[0] + u[1] * u[1] + u[2] * u[2], s3 = s2 * sqrtl(s2);
+      ld U[3][3];
+      for (int a = 0; a < 3; a++)
+        for (int b = 0; b < 3; b++) U[a][b] = ((a == b ? s2 : 0.0L) - u[a] * u[b]) / s3;
+      const ld wj = g->w[j];
+      int k = 0;
+      for (int a = 0; a < 3; a++)
+        for (int b = a; b < 3; b++, k++) {
+          nadd(&acc[k], wj * T[j] * U[a][b]);
+          nadd(&aac[k], wj * T[4 * N + j] * fabsl(U[a][b]));
+        }
+      for (int a = 0; a < 3; a++) {
+        nadd(&acc[6 + a], wj * (U[a][0] * T[N + j] + U[a][1] * T[2 * N + j] + U[a][2] * T[3 * N + j]));
+        nadd(&aac[6 + a], wj * (fabsl(U[a][0]) * T[5 * N + j] + fabsl(U[a][1]) * T[6 * N + j] + fabsl(U[a][2]) * T[7 * N + j]));
+      }
+    }
+    for (int c = 0; c < 9; c++) {
+      G[c * N + i] = nval(&acc[c]);
+      G[(9 + c) * N + i] = nval(&aac[c]);
+    }
+  }
+}
+
+/* O6-O8 (+O10 when Ga != NULL): per species the element matrices from G at the cube's points, added
+ * at (dof_k, dof_l) of the CSR pattern; vals [S][nnz] */
+static void o3_assemble(const o3grid_t *g, int S, const double *mass, const double *charge, double nu, const ld *G,
+                        const ld *Ga, double *vals, double *absvals) {
+  const long long N = g->N, nnz = g->nnz;
+  const int nb = g->nb, nq = g->nq;
+  long long *rowptr = malloc(sizeof(long long) * (g->ndof + 1));
+  int *col = malloc(sizeof(int) * nnz);
+  oracle3d_pattern(g->ncell, g->p, rowptr, col);
+  ld *acc = calloc((size_t)2 * S * nnz, sizeof(ld));
+  const int sym[3][3] = {{0, 1, 2}, {1, 3, 4}, {2, 4, 5}};
+#pragma omp parallel for schedule(static)
+  for (int a = 0; a < S; a++) {
+    ld e2 = (ld)charge[a] * (ld)charge[a], im = 1.0L / (ld)mass[a];
+    ld fD = -(ld)nu * e2 * im * im, fK = (ld)nu * e2 * im; /* O6 */
+    ld *C = malloc(sizeof(ld) * 2 * nb * nb);
+    for (long long c = 0; c < g->nc3; c++) {
+      for (int k = 0; k < 2 * nb * nb; k++) C[k] = 0.0L;
+      for (int q = 0; q < nq; q++) { /* O7 */
+        long long pt = c * nq + q;
+        ld D[3][3], K[3], Da[3][3], Ka[3];
+        for (int r = 0; r < 3; r++) {
+          for (int t = 0; t < 3; t++) {
+            D[r][t] = fD * G[sym[r][t] * N + pt];
+            Da[r][t] = Ga ? fabsl(fD) * Ga[sym[r][t] * N + pt] : 0.0L;
+          }
+          K[r] = fK * G[(6 + r) * N + pt];
+          Ka[r] = Ga ? fabsl(fK) * Ga[(6 + r) * N + pt] : 0.0L;
+        }
+        for (int k = 0; k < nb; k++) {
+          const ld *bk = g->bas + 4 * ((size_t)q * nb + k);
+          for (int l = 0; l < nb; l++) {
+            const ld *bl = g->bas + 4 * ((size_t)q * nb + l);
+            ld v = 0.0L, va = 0.0L;
+            for (int r = 0; r < 3; r++) {
+              for (int t = 0; t < 3; t++) {
+                v += bk[1 + r] * D[r][t] * bl[1 + t];
+                va += fabsl(bk[1 + r]) * Da[r][t] * fabsl(bl[1 + t]);
+              }
+              v += bk[1 + r] * K[r] * bl[0];
+              va += fabsl(bk[1 + r]) * Ka[r] * fabsl(bl[0]);
+            }
+            C[k * nb + l] += g->w[pt] * v;
+            C[nb * nb + k * nb + l] += fabsl(g->w[pt]) * va;
+          }
+        }
+      }
+      for (int k = 0; k < nb; k++) /* O8 */
+        for (int l = 0; l < nb; l++) {
+          long long at = o3_find(rowptr, col, g->dofs[c * nb + k], (int)g->dofs[c * nb + l]);
+          acc[(long long)a * nnz + at] += C[k * nb + l];
+          acc[(long long)(S + a) * nnz + at] += C[nb * nb + k * nb + l];
+        }
+    }
+    free(C);
+  }
+  for (long long k = 0; k < (long long)S * nnz; k++) {
+    vals[k] = (double)acc[k];
+    if (absvals) absvals[k] = (double)acc[(long long)S * nnz + k];
+  }
+  free(acc);
+  free(col);
+  free(rowptr);
+}
+
+void oracle3d_points(int ncell, int order, double R, double *xyz, double *w) {
+  o3grid_t g;
+  o3_grid(ncell, order, R, &g);
+  for (long long k = 0; k < g.N; k++) {
+    xyz[k] = g.x[k];
+    xyz[g.N + k] = g.y[k];
+    xyz[2 * g.N + k] = g.z[k];
+    w[k] = (double)g.w[k];
+  }
+  o3_free(&g);
+}
+
+void oracle3d_fields(int ncell, int order, double R, int S, const double *mass, const double *charge, const double *f,
+                     double *T) {
+  o3grid_t g;
+  o3_grid(ncell, order, R, &g);
+  ld *t = malloc(sizeof(ld) * 8 * g.N);
+  o3_fields(&g, S, mass, charge, f, t);
+  for (long long k = 0; k < 4 * g.N; k++) T[k] = (double)t[k];
+  free(t);
+  o3_free(&g);
+}
+
+void oracle3d_assemble(int ncell, int order, double R, int S, const double *mass, const double *charge, double nu,
+                       const double *G, double *vals) {
+  o3grid_t g;
+  o3_grid(ncell, order, R, &g);
+  ld *Gl = malloc(sizeof(ld) * 9 * g.N);
+  for (long long k = 0; k < 9 * g.N; k++) Gl[k] = G[k];
+  o3_assemble(&g, S, mass, charge, nu, Gl, NULL, vals, NULL);
+  free(Gl);
+  o3_free(&g);
+}
+
+void oracle3d_jacobian(int ncell, int order, double R, int S, const double *mass, const double *charge, double nu,
+                       const double *f, double *vals, double *absvals) {
+  o3grid_t g;
+  o3_grid(ncell, order, R, &g);
+  ld *T = malloc(sizeof(ld) * 8 * g.N), *G = malloc(sizeof(ld) * 18 * g.N);
+  o3_fields(&g, S, mass, charge, f, T);
+  o3_inner(&g, T, G);
+  o3_assemble(&g, S, mass, charge, nu, G, G + 9 * g.N, vals, absvals);
+  free(G);
+  free(T);
+  o3_free(&g);
+}

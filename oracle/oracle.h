@@ -22,6 +22,7 @@
  *   O10 condition scale: the same assembly with every product replaced by its absolute value.
  *   O11 E_z advection matrix sum_e P_e^T (sum_q w phi_k d_z phi_l) P_e (Eq. 4, @8216-8654)
  *   O12 the inner integral with the 3D Cartesian tensor of Eq. 3 (@7997-8072)
+ *   O13 the whole 3D Cartesian Jacobian (O3-O8, O10 on a uniform grid of Q_p cubes, tensor of O12)
  * Pins: see tests/test_oracle_*.py (P1-P9 of SURVEY.md §8(c); P13 for O12).
  */
 #ifndef LANDAU_ORACLE_H
@@ -60,6 +61,26 @@ void oracle_tensor3d(double ux, double uy, double uz, double out[6]);
  * wTK = w T_K premultiplied), coincident points excluded; Gabs: the sums of absolute values. */
 void oracle_inner3d(long long n, const double *x, const double *y, const double *z, const double *wTD,
                     const double *wTKx, const double *wTKy, const double *wTKz, double *G, double *Gabs);
+
+/* O13: the 3D Cartesian Landau Jacobian (NEXT-4 completed, @7997-8072) on a uniform grid of
+ * ncell^3 Q_p cubes over [-R, R]^3: DOF dof(ix, iy, iz) = (iz M + iy) M + ix of the lattice of
+ * M = ncell p + 1 nodes per direction; (p+1)^3 Gauss points per cube; O3/O4 fields, O12 inner
+ * integral, O6/O7 element matrices grad phi_k . D~ grad phi_l + (grad phi_k . K~) phi_l, O8 assembly
+ * (no constraints), O10 |.| scale.  f = [S][ndof] (species-major), vals / absvals = [S][nnz] CSR values
+ * in the pattern of oracle3d_pattern (rows and columns ascending; absvals may be NULL). */
+void oracle3d_sizes(int ncell, int order, long long *ndof, long long *npoints, long long *nnz);
+void oracle3d_pattern(int ncell, int order, long long *rowptr, int *col);
+void oracle3d_nodes(int ncell, int order, double R, double *xyz);  /* [3][ndof] */
+/* the Gauss points [3][npoints] and weights [npoints] (cube-major; q = (a S + b) S + c along z, y, x) */
+void oracle3d_points(int ncell, int order, double R, double *xyz, double *w);
+/* O3/O4 alone: T [4][npoints] = T_D, T_Kx, T_Ky, T_Kz (not multiplied by w) */
+void oracle3d_fields(int ncell, int order, double R, int S, const double *mass, const double *charge, const double *f,
+                     double *T);
+/* O6-O8 alone, from a given G [9][npoints] (G_D xx, xy, xz, yy, yz, zz, G_K x, y, z): vals [S][nnz] */
+void oracle3d_assemble(int ncell, int order, double R, int S, const double *mass, const double *charge, double nu,
+                       const double *G, double *vals);
+void oracle3d_jacobian(int ncell, int order, double R, int S, const double *mass, const double *charge, double nu,
+                       const double *f, double *vals, double *absvals);
 
 /* U^D_rr, U^D_rz, U^D_zz, U^K_rr, U^K_zr at target (r, z), source (rb, zb). */
 void oracle_tensor(double r, double z, double rb, double zb, double out[5]);

@@ -60,6 +60,13 @@ def lib():
         L.oracle_advection_coo.argtypes = [vp, _d]
         L.oracle_tensor3d.argtypes = [C.c_double, C.c_double, C.c_double, _d]
         L.oracle_inner3d.argtypes = [C.c_longlong, _d, _d, _d, _d, _d, _d, _d, _d, _d]
+        L.oracle3d_sizes.argtypes = [C.c_int, C.c_int, P64, P64, P64]
+        L.oracle3d_pattern.argtypes = [C.c_int, C.c_int, _i64, _i32]
+        L.oracle3d_nodes.argtypes = [C.c_int, C.c_int, C.c_double, _d]
+        L.oracle3d_jacobian.argtypes = [C.c_int, C.c_int, C.c_double, C.c_int, _d, _d, C.c_double, _d, _d, _d]
+        L.oracle3d_points.argtypes = [C.c_int, C.c_int, C.c_double, _d, _d]
+        L.oracle3d_fields.argtypes = [C.c_int, C.c_int, C.c_double, C.c_int, _d, _d, _d, _d]
+        L.oracle3d_assemble.argtypes = [C.c_int, C.c_int, C.c_double, C.c_int, _d, _d, C.c_double, _d, _d]
         L.oracle_set_threads.argtypes = [C.c_int]
         L.oracle_get_threads.restype = C.c_int
         _LIB = L
@@ -247,3 +254,56 @@ class Oracle:
     def coefficients(self, with_noise=True):
         from paper_conf_ipps_adamsbkw22_b200 import inputs
         return inputs.coefficients(self.prob, self.all_nodes(), with_noise)
+
+
+class Oracle3D:
+    """O13: the 3D Cartesian Landau Jacobian on a uniform grid of ncell^3 Q_p cubes over [-R, R]^3
+    (oracle.h).  species: sequence of (mass, charge)."""
+
+    def __init__(self, ncell, order, R, species, nu=1.0):
+        self.ncell, self.order, self.R, self.nu = int(ncell), int(order), float(R), float(nu)
+        self.mass = np.array([m for m, _ in species], dtype=np.float64)
+        self.charge = np.array([e for _, e in species], dtype=np.float64)
+        a, b, c = (C.c_longlong() for _ in range(3))
+        lib().oracle3d_sizes(self.ncell, self.order, C.byref(a), C.byref(b), C.byref(c))
+        self.ndof, self.npoints, self.nnz = a.value, b.value, c.value
+
+    def pattern(self):
+        rp = np.zeros(self.ndof + 1, dtype=np.int64)
+        col = np.zeros(self.nnz, dtype=np.int32)
+        lib().oracle3d_pattern(self.ncell, self.order, rp, col)
+        return rp, col
+
+    def nodes(self):
+        xyz = np.zeros((3, self.ndof))
+        lib().oracle3d_nodes(self.ncell, self.order, self.R, xyz)
+        return xyz
+
+    def points(self):
+        xyz, w = np.zeros((3, self.npoints)), np.zeros(self.npoints)
+        lib().oracle3d_points(self.ncell, self.order, self.R, xyz, w)
+        return xyz, w
+
+    def fields(self, f):
+        """O3/O4: [4][npoints] = T_D, T_K (x, y, z), not multiplied by w"""
+        S = self.mass.size
+        f = np.ascontiguousarray(f, dtype=np.float64).reshape(S, self.ndof)
+        T = np.zeros((4, self.npoints))
+        lib().oracle3d_fields(self.ncell, self.order, self.R, S, self.mass, self.charge, f, T)
+        return T
+
+    def assemble(self, G):
+        """O6-O8 from a given G [9][npoints] -> [S][nnz]"""
+        S = self.mass.size
+        v = np.zeros((S, self.nnz))
+        lib().oracle3d_assemble(self.ncell, self.order, self.R, S, self.mass, self.charge, self.nu,
+                                np.ascontiguousarray(G, dtype=np.float64), v)
+        return v
+
+    def jacobian(self, f):
+        """f [S][ndof] -> (J, J^abs), each [S][nnz]"""
+        S = self.mass.size
+        f = np.ascontiguousarray(f, dtype=np.float64).reshape(S, self.ndof)
+        v, va = np.zeros((S, self.nnz)), np.zeros((S, self.nnz))
+        lib().oracle3d_jacobian(self.ncell, self.order, self.R, S, self.mass, self.charge, self.nu, f, v, va)
+        return v, va
