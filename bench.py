@@ -703,6 +703,28 @@ def main():
                         "ordered pairs, parity-tested against oracle O12"}
         except Exception as e:
             line.setdefault("variants", {})["inner3d_cartesian"] = {"unavailable": str(e)[:200]}
+        try:   # the whole 3D Jacobian (a-1, inner, a-4, a-3 + a-5) on the same 8^3 Q3 grid, two species
+            p3 = inputs.config3d(8, 3)
+            with torch.cuda.stream(stream):
+                h3 = L.Landau3D(p3.ncell, p3.order, p3.R, p3.species, p3.nu, device=local, stream=stream)
+            F3 = torch.tensor(inputs.coefficients3d(p3, h3.nodes()), device="cuda")
+            J3 = torch.empty((len(p3.species), h3.nnz), dtype=torch.float64, device="cuda")
+            for _ in range(2):
+                h3.jacobian(F3, J3)
+            ms3j = statistics.median(timed_steps(torch, stream, lambda: h3.jacobian(F3, J3), args.steps, flush))
+            h3.set_timing(True)
+            for _ in range(2):   # the second timed build (the first pays the partials pool's growth)
+                h3.jacobian(F3, J3)
+            st3 = h3.get_timing()
+            h3.set_timing(False)
+            line["variants"]["jacobian3d"] = {
+                "value": 1e3 / ms3j, "unit": "builds/s", "ms_per_step": ms3j, "points": h3.npoints, "ndof": h3.ndof,
+                "nnz_per_species": h3.nnz, "species": len(p3.species), "stage_ms": st3,
+                "note": "SURVEY NEXT-4 completed: 3D Cartesian Jacobian (field3d, inner3d, element3d, assembly) on "
+                        "8^3 Q3 cubes, e + a light ion; parity-tested against oracle O13 on 2^3/3^3 grids"}
+            h3.close()
+        except Exception as e:
+            line.setdefault("variants", {})["jacobian3d"] = {"unavailable": str(e)[:200]}
 
     # ---- NEXT-3: quasi-Newton backward-Euler iterations on the same batch --------------------------
     if extras and nloc:

@@ -277,6 +277,32 @@ int landau_get_vtx_schedule(landau_t h, int32_t *nrounds, int32_t *weight_prefix
 int landau3d_inner(int64_t n, const double *xyz_dev, const double *wTD_dev, const double *wTK_dev, double *G_dev,
                    void *cuda_stream);
 
+/* NEXT-4 completed ("a full 3D model is supported in the library", PAPER.md:1@7997-8072): the whole
+ * Landau Jacobian in 3D Cartesian velocity space -- a-1 point fields, the inner integral of
+ * landau3d_inner, a-4 element matrices (Eqs. 5-6 without the r weight: C^D_e[k][l] = sum_q w_q
+ * grad phi_k . G_D grad phi_l, C^K_e[k][l] = sum_q w_q (grad phi_k . G_K) phi_l), a-3 species factors
+ * and a-5 assembly -- on a uniform grid of ncell^3 Q_p cubes (order 2 or 3) over [-R, R]^3.
+ *   DOFs: the lattice of M = ncell p + 1 equispaced nodes per direction, dof = (iz M + iy) M + ix at
+ *   (-R + ix h/p, ...), h = 2R / ncell (landau3d_get_nodes: host [3][ndof]); (p+1)^3 Gauss points per
+ *   cube.  The CSR pattern (landau3d_get_pattern: host rowptr [ndof+1], col [nnz]) has rows and
+ *   columns ascending and is the same for every species block.
+ *   landau3d_create: species masses (m0 units, > 0) and charges [nspecies <= 16], nu; the handle is
+ *     tied to cuda_device and enqueues on cuda_stream.  EINVAL: bad sizes or parameters; ENOMEM.
+ *   landau3d_jacobian: f_dev [nspecies][ndof] (device, species-major) -> J_dev [nspecies][nnz] CSR
+ *     values of the species-block-diagonal Jacobian (device).  Enqueued; ECUDA on launch failure.
+ *   landau3d_set_timing / _get_timing: per-stage CUDA-event times of the last build (field, inner,
+ *     element, assemble; milliseconds; synchronises the stream when enabled). */
+typedef struct landau3d_s *landau3d_t;
+int landau3d_create(landau3d_t *out, int32_t ncell, int32_t order, double R, int32_t nspecies, const double *mass,
+                    const double *charge, double nu, int32_t cuda_device, void *cuda_stream);
+int landau3d_get_sizes(landau3d_t h, int64_t *ndof, int64_t *npoints, int64_t *nnz);
+int landau3d_get_pattern(landau3d_t h, int64_t *rowptr, int32_t *col);
+int landau3d_get_nodes(landau3d_t h, double *xyz);
+int landau3d_jacobian(landau3d_t h, const double *f_dev, double *J_dev);
+int landau3d_set_timing(landau3d_t h, int32_t enable);
+int landau3d_get_timing(landau3d_t h, float *ms4);
+void landau3d_destroy(landau3d_t h);
+
 /* How the last build ran (for FLOP accounting and diagnostics). */
 typedef struct {
   int32_t inner_path;        /* 0: directed pair kernel (every ordered pair, split-j when small);

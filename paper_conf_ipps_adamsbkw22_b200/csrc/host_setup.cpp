@@ -641,4 +641,96 @@ std::string build_phase_maps(const Plan &plan, const std::vector<GatherMap> &map
   return "";
 }
 
+std::string build_plan3d(int ncell, int order, double R, Plan3D &P) {
+  if (ncell < 1 || order < 2 || order > 3 || !(R > 0.0)) return "3d: ncell >= 1, order 2 or 3, R > 0";
+  const int p = order, S = p + 1, nb = S * S * S;
+  const int64_t M = (int64_t)ncell * p + 1, nc3 = (int64_t)ncell * ncell * ncell;
+  if (M * M * M > INT32_MAX || nc3 * nb * nb * 2 > INT32_MAX) return "3d: grid too large";
+  P = Plan3D{};
+  P.ncell = ncell;
+  P.p = p;
+  P.s1 = S;
+  P.nb = nb;
+  P.R = R;
+  P.h = 2.0 * R / ncell;
+  P.ndof = M * M * M;
+  P.npts = nc3 * nb;
+  std::vector<double> xg, wg;
+  gauss_legendre(S, xg, wg);
+  P.L1.resize(S * S);
+  P.D1.resize(S * S);
+  for (int i = 0; i < S; i++)
+    for (int a = 0; a < S; a++) {
+      P.L1[i * S + a] = lagrange(p, a, xg[i]);
+      P.D1[i * S + a] = lagrange_d(p, a, xg[i]);
+    }
+  P.xyz.resize(3 * P.npts);
+  P.w.resize(P.npts);
+  P.dofs.resize(nc3 * nb);
+  const double hh = 0.5 * P.h;
+  for (int64_t cz = 0; cz < ncell; cz++)
+    for (int64_t cy = 0; cy < ncell; cy++)
+      for (int64_t cx = 0; cx < ncell; cx++) {
+        const int64_t e = (cz * ncell + cy) * ncell + cx;
+        for (int k = 0; k < S; k++)
+          for (int j = 0; j < S; j++)
+            for (int i = 0; i < S; i++)
+              P.dofs[e * nb + (k * S + j) * S + i] = (int32_t)(((cz * p + k) * M + (cy * p + j)) * M + (cx * p + i));
+        for (int a = 0; a < S; a++)
+          for (int b = 0; b < S; b++)
+            for (int c = 0; c < S; c++) {
+              const int64_t pt = e * nb + (a * S + b) * S + c;
+              P.xyz[pt] = -R + P.h * cx + hh * (xg[c] + 1.0);
+              P.xyz[P.npts + pt] = -R + P.h * cy + hh * (xg[b] + 1.0);
+              P.xyz[2 * P.npts + pt] = -R + P.h * cz + hh * (xg[a] + 1.0);
+              P.w[pt] = wg[a] * wg[b] * wg[c] * hh * hh * hh;
+            }
+      }
+  // 1-D neighbour ranges: the lattice indices sharing a cube with i
+  std::vector<int64_t> lo(M), hi(M);
+  for (int64_t i = 0; i < M; i++) {
+    int64_t c0 = i / p, c1 = c0;
+    if (i % p == 0 && c0 > 0) c0--;
+    c1 = std::min<int64_t>(c1, ncell - 1);
+    lo[i] = c0 * p;
+    hi[i] = (c1 + 1) * p;
+  }
+  P.rowptr.assign(P.ndof + 1, 0);
+  for (int64_t iz = 0; iz < M; iz++)
+    for (int64_t iy = 0; iy < M; iy++)
+      for (int64_t ix = 0; ix < M; ix++) {
+        const int64_t r = (iz * M + iy) * M + ix;
+        P.rowptr[r + 1] = P.rowptr[r] + (hi[ix] - lo[ix] + 1) * (hi[iy] - lo[iy] + 1) * (hi[iz] - lo[iz] + 1);
+      }
+  P.nnz = P.rowptr[P.ndof];
+  if (P.nnz > INT32_MAX) return "3d: pattern too large";
+  P.col.resize(P.nnz);
+  for (int64_t iz = 0; iz < M; iz++)
+    for (int64_t iy = 0; iy < M; iy++)
+      for (int64_t ix = 0; ix < M; ix++) {
+        int64_t q = P.rowptr[(iz * M + iy) * M + ix];
+        for (int64_t jz = lo[iz]; jz <= hi[iz]; jz++)
+          for (int64_t jy = lo[iy]; jy <= hi[iy]; jy++)
+            for (int64_t jx = lo[ix]; jx <= hi[ix]; jx++) P.col[q++] = (int32_t)((jz * M + jy) * M + jx);
+      }
+  // gather map: contributions counted, then filled in cube order (stable per slot)
+  auto slot_of = [&](int32_t r, int32_t c) -> int64_t {
+    const int32_t *b = P.col.data() + P.rowptr[r], *en = P.col.data() + P.rowptr[r + 1];
+    return (int64_t)(std::lower_bound(b, en, c) - P.col.data());
+  };
+  P.map.ptr.assign(P.nnz + 1, 0);
+  for (int64_t e = 0; e < nc3; e++)
+    for (int k = 0; k < nb; k++)
+      for (int l = 0; l < nb; l++) P.map.ptr[slot_of(P.dofs[e * nb + k], P.dofs[e * nb + l]) + 1]++;
+  for (int64_t s = 0; s < P.nnz; s++) P.map.ptr[s + 1] += P.map.ptr[s];
+  std::vector<int64_t> fill(P.map.ptr.begin(), P.map.ptr.end() - 1);
+  P.map.idx.resize(P.map.ptr[P.nnz]);
+  P.map.w.assign(P.map.ptr[P.nnz], 1.0);
+  for (int64_t e = 0; e < nc3; e++)
+    for (int k = 0; k < nb; k++)
+      for (int l = 0; l < nb; l++)
+        P.map.idx[fill[slot_of(P.dofs[e * nb + k], P.dofs[e * nb + l])]++] = (int32_t)(e * 2 * nb * nb + 2 * (k * nb + l));
+  return "";
+}
+
 }  // namespace landau

@@ -103,6 +103,26 @@ struct PhaseMaps {
 // cap >= 1 cells per phase; returns "" or an error (more than INT32_MAX entries).
 std::string build_phase_maps(const Plan &plan, const std::vector<GatherMap> &maps, int cap, PhaseMaps &out);
 
+// NEXT-4 completed: the 3D Cartesian model on a uniform grid of ncell^3 Q_p cubes over [-R, R]^3
+// (kernels_3d_fe.cuh).  DOFs: the lattice of M = ncell p + 1 nodes per direction,
+// dof(ix, iy, iz) = (iz M + iy) M + ix; points cube-major, q = (a S + b) S + c (Gauss indices along
+// z, y, x), w = w_a w_b w_c (h/2)^3; local node n = (k S + j) S + i.  The CSR pattern: rows and
+// columns ascending (the tensor product of the 1-D patterns); the gather map lists, per CSR slot, the
+// element-buffer entries e 2 NB^2 + 2 (k NB + l) of every cube holding both DOFs, in cube order,
+// weight 1 (no constraints on a uniform grid).
+struct Plan3D {
+  int ncell = 0, p = 0, s1 = 0, nb = 0;
+  double R = 0.0, h = 0.0;
+  int64_t ndof = 0, npts = 0, nnz = 0;
+  std::vector<double> L1, D1;            // [S][S]: l_a(x_i), l'_a(x_i) at [i * S + a]
+  std::vector<double> xyz, w;            // [3][npts], [npts]
+  std::vector<int32_t> dofs;             // [ncube][nb]
+  std::vector<int64_t> rowptr;           // [ndof + 1]
+  std::vector<int32_t> col;              // [nnz]
+  GatherMap map;                         // [nnz] slots
+};
+std::string build_plan3d(int ncell, int order, double R, Plan3D &plan);
+
 // Build the plan.  Returns "" on success or an error message (the mesh is invalid).
 std::string build_plan(int ngrids, const int64_t *ncells, const double *cells, const double *radius, int order,
                        Plan &plan);

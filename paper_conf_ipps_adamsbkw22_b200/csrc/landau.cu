@@ -30,6 +30,7 @@ using namespace landau;
 #include "kernels_band.cuh"
 #include "kernels_single.cuh"
 #include "kernels_3d.cuh"
+#include "kernels_3d_fe.cuh"
 
 
 // ==================================================================================================
@@ -2287,3 +2288,217 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
   return LANDAU_OK;
 }
 
+
+// ==================================================================================================
+// NEXT-4 completed: the 3D Cartesian Landau Jacobian (landau3d_*, include/landau.h)
+// ==================================================================================================
+struct landau3d_s {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  landau::Plan3D P;
+  int S = 0;
+  landau::Species3D sp{};
+  landau::GatherDev gm{};
+  double *d_L1 = nullptr, *d_D1 = nullptr, *d_xyz = nullptr, *d_w = nullptr, *d_wTD = nullptr, *d_wTK = nullptr,
+         *d_G = nullptr, *d_C = nullptr, *d_mw = nullptr;
+  int32_t *d_dofs = nullptr, *d_idx = nullptr;
+  int64_t *d_ptr = nullptr;
+  float stage_ms[4] = {0, 0, 0, 0};   // field, inner, element, assemble of the last timed build
+  bool timing = false;
+};
+
+namespace {
+void free3d(landau3d_t h) {
+  for (void *p : {(void *)h->d_L1, (void *)h->d_D1, (void *)h->d_xyz, (void *)h->d_w, (void *)h->d_wTD, (void *)h->d_wTK,
+                  (void *)h->d_G, (void *)h->d_C, (void *)h->d_mw, (void *)h->d_dofs, (void *)h->d_idx, (void *)h->d_ptr})
+    if (p) cudaFree(p);
+}
+template <class T>
+int up3d(landau3d_t h, T **dst, const std::vector<T> &src) {
+  if (cudaMalloc((void **)dst, std::max<size_t>(src.size(), 1) * sizeof(T)) != cudaSuccess) return LANDAU_ENOMEM;
+  if (!src.empty() && cudaMemcpyAsync(*dst, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice, h->stream) != cudaSuccess)
+    return LANDAU_ECUDA;
+  return LANDAU_OK;
+}
+template <class F>
+int guarded3d(landau3d_t h, F &&body) {
+  try {
+    int prev = -1, cur = 0;
+    if (h && cudaGetDevice(&cur) == cudaSuccess && cur != h->device && cudaSetDevice(h->device) == cudaSuccess) prev = cur;
+    const int rc = body();
+    if (prev >= 0) cudaSetDevice(prev);
+    return rc;
+  } catch (const std::bad_alloc &) {
+    return LANDAU_ENOMEM;
+  } catch (...) {
+    return LANDAU_EINVAL;
+  }
+}
+template <int S1>
+int build3d(landau3d_t h, const double *f, double *J) {
+  using namespace landau;
+  const Plan3D &P = h->P;
+  cudaEvent_t ev[5];
+  if (h->timing)
+    for (auto &e : ev) cudaEventCreate(&e);
+  auto mark = [&](int i) {
+    if (h->timing) cudaEventRecord(ev[i], h->stream);
+  };
+  mark(0);
+  const unsigned gf = (unsigned)std::min<int64_t>((P.npts + 127) / 128, 148LL * 16);
+  field3d_kernel<S1><<<gf, 128, 0, h->stream>>>(P.npts, f, P.ndof, h->d_dofs, h->d_L1, h->d_D1, 2.0 / P.h, h->d_w, h->sp,
+                                                h->d_wTD, h->d_wTK);
+  if (cudaGetLastError() != cudaSuccess) return LANDAU_ECUDA;
+  mark(1);
+  int rc = landau3d_inner(P.npts, h->d_xyz, h->d_wTD, h->d_wTK, h->d_G, h->stream);
+  if (rc) return rc;
+  mark(2);
+  const int64_t ncube = (int64_t)P.ncell * P.ncell * P.ncell;
+  element3d_kernel<S1><<<(unsigned)std::min<int64_t>(ncube, 148LL * 8), k3dElThreads, 0, h->stream>>>(
+      ncube, h->d_G, P.npts, h->d_w, h->d_L1, h->d_D1, 2.0 / P.h, reinterpret_cast<double2 *>(h->d_C));
+  if (cudaGetLastError() != cudaSuccess) return LANDAU_ECUDA;
+  mark(3);
+  assemble_kernel<S1 * S1 * S1, 1><<<dim3((unsigned)((P.nnz + 127) / 128), 1), 128, 0, h->stream>>>(h->gm, h->d_C, 0, J,
+                                                                                                    0, 1);
+  if (cudaGetLastError() != cudaSuccess) return LANDAU_ECUDA;
+  mark(4);
+  if (h->timing) {
+    cudaEventSynchronize(ev[4]);
+    for (int i = 0; i < 4; i++) cudaEventElapsedTime(&h->stage_ms[i], ev[i], ev[i + 1]);
+    for (auto &e : ev) cudaEventDestroy(e);
+  }
+  return LANDAU_OK;
+}
+}  // namespace
+
+extern "C" {
+
+int landau3d_create(landau3d_t *out, int32_t ncell, int32_t order, double R, int32_t nspecies, const double *mass,
+                    const double *charge, double nu, int32_t cuda_device, void *cuda_stream) {
+  if (!out) return LANDAU_EINVAL;
+  *out = nullptr;
+  if (nspecies < 1 || nspecies > landau::kMaxSpecies || !mass || !charge) return LANDAU_EINVAL;
+  for (int a = 0; a < nspecies; a++)
+    if (!(mass[a] > 0.0)) return LANDAU_EINVAL;
+  landau3d_t h = nullptr;
+  int prev = -1;
+  const int rc = [&]() -> int {
+    try {
+      h = new landau3d_s();
+      const std::string err = landau::build_plan3d(ncell, order, R, h->P);
+      if (!err.empty()) return LANDAU_EINVAL;
+      int cur = 0;
+      if (cudaGetDevice(&cur) != cudaSuccess) return LANDAU_ECUDA;
+      if (cur != cuda_device) {
+        if (cudaSetDevice(cuda_device) != cudaSuccess) return LANDAU_ECUDA;
+        prev = cur;
+      }
+      h->device = cuda_device;
+      h->stream = (cudaStream_t)cuda_stream;
+      h->S = nspecies;
+      h->sp.S = nspecies;
+      h->gm.nsp = nspecies;
+      h->gm.nslots = h->P.nnz;
+      for (int a = 0; a < nspecies; a++) {   // a-1 sums and a-3 factors
+        const double e2 = charge[a] * charge[a], im = 1.0 / mass[a];
+        h->sp.e2[a] = e2;
+        h->sp.e2m[a] = e2 * im;
+        h->gm.out_off[a] = (int64_t)a * h->P.nnz;
+        h->gm.fD[a] = -nu * e2 * im * im;
+        h->gm.fK[a] = nu * e2 * im;
+      }
+      const landau::Plan3D &P = h->P;
+      const int64_t ncube = (int64_t)P.ncell * P.ncell * P.ncell;
+      int r;
+      if ((r = up3d(h, &h->d_L1, P.L1)) || (r = up3d(h, &h->d_D1, P.D1)) || (r = up3d(h, &h->d_xyz, P.xyz)) ||
+          (r = up3d(h, &h->d_w, P.w)) || (r = up3d(h, &h->d_dofs, P.dofs)) || (r = up3d(h, &h->d_ptr, P.map.ptr)) ||
+          (r = up3d(h, &h->d_idx, P.map.idx)) || (r = up3d(h, &h->d_mw, P.map.w)))
+        return r;
+      if (cudaMalloc(&h->d_wTD, sizeof(double) * P.npts) != cudaSuccess ||
+          cudaMalloc(&h->d_wTK, sizeof(double) * 3 * P.npts) != cudaSuccess ||
+          cudaMalloc(&h->d_G, sizeof(double) * 9 * P.npts) != cudaSuccess ||
+          cudaMalloc(&h->d_C, sizeof(double) * 2 * ncube * P.nb * P.nb) != cudaSuccess)
+        return LANDAU_ENOMEM;
+      h->gm.ptr = h->d_ptr;
+      h->gm.idx = h->d_idx;
+      h->gm.w = h->d_mw;
+      if (cudaStreamSynchronize(h->stream) != cudaSuccess) return LANDAU_ECUDA;
+      return LANDAU_OK;
+    } catch (const std::bad_alloc &) {
+      return LANDAU_ENOMEM;
+    } catch (...) {
+      return LANDAU_EINVAL;
+    }
+  }();
+  if (rc != LANDAU_OK) {
+    if (h) {
+      free3d(h);
+      delete h;
+    }
+  } else {
+    *out = h;
+  }
+  if (prev >= 0) cudaSetDevice(prev);
+  return rc;
+}
+
+int landau3d_get_sizes(landau3d_t h, int64_t *ndof, int64_t *npoints, int64_t *nnz) {
+  if (!h) return LANDAU_EINVAL;
+  if (ndof) *ndof = h->P.ndof;
+  if (npoints) *npoints = h->P.npts;
+  if (nnz) *nnz = h->P.nnz;
+  return LANDAU_OK;
+}
+
+int landau3d_get_pattern(landau3d_t h, int64_t *rowptr, int32_t *col) {
+  if (!h) return LANDAU_EINVAL;
+  if (rowptr) std::copy(h->P.rowptr.begin(), h->P.rowptr.end(), rowptr);
+  if (col) std::copy(h->P.col.begin(), h->P.col.end(), col);
+  return LANDAU_OK;
+}
+
+int landau3d_get_nodes(landau3d_t h, double *xyz) {
+  if (!h || !xyz) return LANDAU_EINVAL;
+  const landau::Plan3D &P = h->P;
+  const int64_t M = (int64_t)P.ncell * P.p + 1, nd = P.ndof;
+  const double d = P.h / P.p;
+  for (int64_t iz = 0; iz < M; iz++)
+    for (int64_t iy = 0; iy < M; iy++)
+      for (int64_t ix = 0; ix < M; ix++) {
+        const int64_t k = (iz * M + iy) * M + ix;
+        xyz[k] = -P.R + ix * d;
+        xyz[nd + k] = -P.R + iy * d;
+        xyz[2 * nd + k] = -P.R + iz * d;
+      }
+  return LANDAU_OK;
+}
+
+int landau3d_jacobian(landau3d_t h, const double *f_dev, double *J_dev) {
+  if (!h || !f_dev || !J_dev) return LANDAU_EINVAL;
+  return guarded3d(h, [&]() -> int { return h->P.s1 == 3 ? build3d<3>(h, f_dev, J_dev) : build3d<4>(h, f_dev, J_dev); });
+}
+
+int landau3d_set_timing(landau3d_t h, int32_t enable) {
+  if (!h) return LANDAU_EINVAL;
+  h->timing = enable != 0;
+  return LANDAU_OK;
+}
+
+int landau3d_get_timing(landau3d_t h, float *ms4) {
+  if (!h || !ms4) return LANDAU_EINVAL;
+  for (int i = 0; i < 4; i++) ms4[i] = h->stage_ms[i];
+  return LANDAU_OK;
+}
+
+void landau3d_destroy(landau3d_t h) {
+  if (!h) return;
+  try {
+    cudaSetDevice(h->device);
+    if (h->stream) cudaStreamSynchronize(h->stream);
+    free3d(h);
+    delete h;
+  } catch (...) {
+  }
+}
+
+}  // extern "C"

@@ -351,3 +351,43 @@ def fields3d(xyz, w, seed: int = 20222):
         grad += np.array([-2.0 * x / th * f, -2.0 * y / th * f, -2.0 * (z - u) / th * f])
     xi = 1.0 + 0.01 * rng.uniform(-1.0, 1.0, size=x.size)
     return w * g * xi, w * grad * xi
+
+
+# ------------------------------------------------------------------------------------------------
+# NEXT-4 completed: a 3D Cartesian Jacobian configuration (uniform ncell^3 Q_p cubes over [-R, R]^3)
+# ------------------------------------------------------------------------------------------------
+@dataclass
+class Problem3D:
+    name: str
+    ncell: int
+    order: int
+    R: float
+    species: list            # [(mass, charge)]
+    fmix: list               # per species [(n, T, u_z)]: Maxwellians drifting along z
+    seed: int = 20223
+    noise: float = 0.01
+    nu: float = 1.0
+
+
+def config3d(ncell: int = 4, order: int = 3) -> Problem3D:
+    """Electrons with the thermal-quench shape of C2 (cold bulk + drifting hot tail) and a light
+    synthetic ion (m = 4 m_e, T = 4 T_e, so that its Maxwellian is resolved on the electron-scale grid:
+    the test exercises the species factors, not a physical mass ratio), on [-R_E, R_E]^3."""
+    return Problem3D("C3D", ncell, order, R_E, [(1.0, -1.0), (4.0, 1.0)],
+                     fmix=[[(5.0, 0.1, 0.0), (1.0, 1.0, 0.5 * VTH_E)], [(6.0, 4.0, 0.0)]])
+
+
+def coefficients3d(prob: Problem3D, xyz, with_noise: bool = True) -> np.ndarray:
+    """[S][ndof] nodal values of each species' Maxwellian mix at the DOF nodes xyz [3][ndof] (whoever
+    owns the numbering), times (1 + noise xi), xi ~ U(-1, 1) from a seeded generator per species."""
+    x, y, z = (np.asarray(c, dtype=np.float64) for c in xyz)
+    out = []
+    for a, (m, _) in enumerate(prob.species):
+        v = np.zeros_like(x)
+        for (n, T, u) in prob.fmix[a]:
+            th = theta(T, m)
+            v = v + n * (math.pi * th) ** -1.5 * np.exp(-(x ** 2 + y ** 2 + (z - u) ** 2) / th)
+        if with_noise and prob.noise != 0.0:
+            v = v * (1.0 + prob.noise * np.random.default_rng(prob.seed + a).uniform(-1.0, 1.0, size=x.size))
+        out.append(v)
+    return np.ascontiguousarray(np.stack(out), dtype=np.float64)

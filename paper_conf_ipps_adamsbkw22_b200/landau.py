@@ -78,6 +78,14 @@ def lib():
             "landau_partition": (C.c_int, [i64, i32, i32, P64, P64]),
             "landau_pair_partition": (C.c_int, [i64, i32, i32, P64, P64]),
             "landau3d_inner": (C.c_int, [i64, vp, vp, vp, vp, vp]),
+            "landau3d_create": (C.c_int, [C.POINTER(vp), i32, i32, d, i32, Pd, Pd, d, i32, vp]),
+            "landau3d_get_sizes": (C.c_int, [vp, P64, P64, P64]),
+            "landau3d_get_pattern": (C.c_int, [vp, P64, P32]),
+            "landau3d_get_nodes": (C.c_int, [vp, Pd]),
+            "landau3d_jacobian": (C.c_int, [vp, vp, vp]),
+            "landau3d_set_timing": (C.c_int, [vp, i32]),
+            "landau3d_get_timing": (C.c_int, [vp, C.POINTER(C.c_float)]),
+            "landau3d_destroy": (None, [vp]),
             "landau_nccl_unique_id": (C.c_int, [vp]),
             "landau_set_timing": (C.c_int, [vp, i32]),
             "landau_get_timing": (C.c_int, [vp, Pd, P64]),
@@ -143,6 +151,69 @@ def landau3d_inner(xyz, wTD, wTK, G, stream=None):
     rc = lib().landau3d_inner(n, xyz.data_ptr(), wTD.data_ptr(), wTK.data_ptr(), G.data_ptr(), st)
     if rc:
         raise LandauError(rc, "landau3d_inner")
+
+
+class Landau3D:
+    """NEXT-4: the 3D Cartesian Landau Jacobian on a uniform grid of ncell^3 Q_p cubes over [-R, R]^3
+    (include/landau.h, landau3d_*).  species: sequence of (mass, charge).  Argument marshalling only."""
+
+    def __init__(self, ncell, order, R, species, nu=1.0, device=0, stream=None):
+        import torch
+        self.device = int(device)
+        self.nspecies = len(species)
+        mass = np.array([m for m, _ in species], dtype=np.float64)
+        charge = np.array([e for _, e in species], dtype=np.float64)
+        st = stream.cuda_stream if stream is not None else torch.cuda.current_stream(self.device).cuda_stream
+        self.stream = stream
+        h = C.c_void_p()
+        rc = lib().landau3d_create(C.byref(h), int(ncell), int(order), float(R), self.nspecies, _dptr(mass), _dptr(charge),
+                                   float(nu), self.device, C.c_void_p(st))
+        if rc:
+            raise LandauError(rc, "landau3d_create")
+        self._h = h
+        a, b, c = C.c_int64(), C.c_int64(), C.c_int64()
+        lib().landau3d_get_sizes(h, C.byref(a), C.byref(b), C.byref(c))
+        self.ndof, self.npoints, self.nnz = a.value, b.value, c.value
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().landau3d_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def pattern(self):
+        rp = np.zeros(self.ndof + 1, dtype=np.int64)
+        col = np.zeros(self.nnz, dtype=np.int32)
+        lib().landau3d_get_pattern(self._h, rp.ctypes.data_as(C.POINTER(C.c_int64)), col.ctypes.data_as(C.POINTER(C.c_int32)))
+        return rp, col
+
+    def nodes(self):
+        xyz = np.zeros((3, self.ndof))
+        lib().landau3d_get_nodes(self._h, _dptr(xyz))
+        return xyz
+
+    def jacobian(self, f, J):
+        """f [nspecies][ndof] -> J [nspecies][nnz] (contiguous float64 tensors on the handle's GPU)."""
+        for t, n, name in ((f, self.nspecies * self.ndof, "f"), (J, self.nspecies * self.nnz, "J")):
+            if not t.is_cuda or t.device.index != self.device or t.numel() != n:
+                raise ValueError(f"landau3d_jacobian: {name} must hold {n} values on cuda:{self.device}")
+        rc = lib().landau3d_jacobian(self._h, _tptr(f), _tptr(J))
+        if rc:
+            raise LandauError(rc, "landau3d_jacobian")
+
+    def set_timing(self, on):
+        lib().landau3d_set_timing(self._h, int(bool(on)))
+
+    def get_timing(self):
+        """per-stage ms of the last timed build: field, inner, element, assemble"""
+        ms = (C.c_float * 4)()
+        lib().landau3d_get_timing(self._h, ms)
+        return dict(zip(("field", "inner", "element", "assemble"), [float(x) for x in ms]))
 
 
 def landau_nccl_unique_id():

@@ -17,14 +17,14 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def header_symbols():
     txt = open(os.path.join(ROOT, "include", "landau.h")).read()
-    return sorted(set(re.findall(r"^\s*(?:int|void|const char \*)\s*(landau_\w+)\s*\(", txt, re.M)))
+    return sorted(set(re.findall(r"^\s*(?:int|void|const char \*)\s*(landau(?:_|3d_)\w+)\s*\(", txt, re.M)))
 
 
 def test_library_exports_every_declared_symbol():
     syms = header_symbols()
     assert len(syms) >= 20
     out = subprocess.run(["nm", "-D", "--defined-only", L.LIB_PATH], capture_output=True, text=True, check=True).stdout
-    exported = set(re.findall(r"\bT (landau_\w+)", out))
+    exported = set(re.findall(r"\bT (landau(?:_|3d_)\w+)", out))
     missing = [s for s in syms if s not in exported]
     assert not missing, missing
     lib = ctypes.CDLL(L.LIB_PATH)
