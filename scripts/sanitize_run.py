@@ -3,10 +3,13 @@
 # step with and without the quench source; the 3D Cartesian inner integral; one emulated rank of the pair
 # split), the fused single-build kernel (C1, C3 without timers), the element/assembly kernels (timed
 # builds), and a 200-vertex batch (more vertices than SMs: the per-vertex kernel loops over several
-# vertices per CTA and splits some between CTAs).  Argument "tail": LANDAU_TAIL=1 (the fused tail kernel).
+# vertices per CTA and splits some between CTAs), the 3D Cartesian Jacobian.  Argument "tail":
+# LANDAU_TAIL=1 (the fused tail kernel); "bandcw": LANDAU_BAND_CW=1 (the column-warp band factorisation).
 import os, sys
 if len(sys.argv) > 1 and sys.argv[1] == "tail":
     os.environ["LANDAU_TAIL"] = "1"
+if len(sys.argv) > 1 and sys.argv[1] == "bandcw":   # the opt-in column-warp band factorisation
+    os.environ["LANDAU_BAND_CW"] = "1"
 sys.path.insert(0, os.getcwd())
 import numpy as np, torch
 from paper_conf_ipps_adamsbkw22_b200 import inputs
@@ -78,3 +81,13 @@ Gp = torch.empty((4, 5, h3.npoints), dtype=torch.float64, device="cuda")
 h3.point_coeffs_batched(Gp)
 torch.cuda.synchronize()
 print("ok 3d + pair split")
+# NEXT-4 completed: the whole 3D Jacobian (field3d, inner3d, element3d, assembly), Q2 and Q3
+for nc, order in ((2, 2), (2, 3)):
+    p3d = inputs.config3d(nc, order)
+    h3d = L.Landau3D(p3d.ncell, p3d.order, p3d.R, p3d.species, p3d.nu, device=0)
+    F3d = torch.tensor(inputs.coefficients3d(p3d, h3d.nodes()), device="cuda")
+    J3d = torch.empty((len(p3d.species), h3d.nnz), dtype=torch.float64, device="cuda")
+    h3d.jacobian(F3d, J3d)
+    torch.cuda.synchronize()
+    h3d.close()
+print("ok 3d jacobian")
