@@ -87,7 +87,10 @@ __global__ void __launch_bounds__(32 * kSbWarps, 1) single_build_kernel(const Si
     u.fld.dxi[i % NB][i / NB] = a.tab[NB * NB + i];
     u.fld.deta[i % NB][i / NB] = a.tab[2 * NB * NB + i];
   }
-  {
+#ifndef LANDAU_SB_SKIP
+#define LANDAU_SB_SKIP 0
+#endif
+  if (!(LANDAU_SB_SKIP & 1)) {
     const int el = threadIdx.x / NB, q = threadIdx.x % NB;
     const int64_t nchunks = (a.ncell + EPB - 1) / EPB;
     for (int64_t it = blockIdx.x; it < nchunks * a.nbatch; it += gridDim.x) {
@@ -135,7 +138,7 @@ __global__ void __launch_bounds__(32 * kSbWarps, 1) single_build_kernel(const Si
   // ---- a-2 inner integral: a CTA item is (b, target tile t, group g of 8 source splits); warp w
   // evaluates split 8 g + w of the sources against the tile (inner_mdir_kernel's per-warp arithmetic),
   // the CTA adds its warps' sums in warp order in shared memory and writes one partial per group ------
-  {
+  if (!(LANDAU_SB_SKIP & 2)) {
     PairCoef cf;
     load_pair_coef(s_coef, s_ltab, cf);
     const int64_t N = a.npts, Hp = a.T * 32, ngroups = (a.nsplit + kSbWarps - 1) / kSbWarps;
@@ -213,7 +216,7 @@ __global__ void __launch_bounds__(32 * kSbWarps, 1) single_build_kernel(const Si
   // ---- a-2r: the groups' partials summed in group order (one thread per (b, component, point)) ----
   {
     const int64_t N = a.npts, Hp = a.T * 32, ngroups = (a.nsplit + kSbWarps - 1) / kSbWarps;
-    if (ngroups > 1) {
+    if (ngroups > 1 && !(LANDAU_SB_SKIP & 4)) {
       const int64_t total = (int64_t)a.nbatch * 10 * a.H;
       for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
         const int64_t b = k / (10 * a.H), c = (k / a.H) % 10, ut = k % a.H;
@@ -230,7 +233,7 @@ __global__ void __launch_bounds__(32 * kSbWarps, 1) single_build_kernel(const Si
   SB_STAMP();
 
   // ---- a-4 element matrices (element_sf_kernel's arithmetic, one warp per cell) -------------------
-  {
+  if (!(LANDAU_SB_SKIP & 8)) {
     double PLL[S], PLD[S], PDL[S], PDD[S];
     sf_tables<S>(a.tab1, lane, PLL, PLD, PDL, PDD);
     const int64_t N = a.npts, nitems = a.ncell * a.nbatch;
@@ -254,7 +257,7 @@ __global__ void __launch_bounds__(32 * kSbWarps, 1) single_build_kernel(const Si
   SB_STAMP();
 
   // ---- a-3 + a-5 assembly (assemble_kernel's arithmetic: one slot per thread) ----------------------
-  for (int g = 0; g < a.ngrids; g++) {
+  for (int g = 0; g < ((LANDAU_SB_SKIP & 16) ? 0 : a.ngrids); g++) {
     const GatherDev &gm = a.maps[g];
     const int64_t total = gm.nslots * a.nbatch;
     for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
