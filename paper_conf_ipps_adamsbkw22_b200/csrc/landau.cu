@@ -270,7 +270,7 @@ int launch_field(landau_t h, int64_t nbatch) {
   const int64_t items = (P.ncell + EPB - 1) / EPB * nbatch;
   static const int64_t blocks_per_sm = [] {   // grid cap (LANDAU_FIELD_BLOCKS_PER_SM)
     const char *e = getenv("LANDAU_FIELD_BLOCKS_PER_SM");
-    return e ? (int64_t)atoll(e) : (int64_t)8;
+    return e ? (int64_t)atoll(e) : (int64_t)6;   // C4 1024: 8 43.5 us, 6 35.4, 4 41.8; 128: 16.6, 13.9, 13.9
   }();
   // whole multiples of the chunk count: block g * nchunks + c keeps chunk c (see field_kernel)
   const int64_t nchunks = (P.ncell + EPB - 1) / EPB;
