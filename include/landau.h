@@ -262,6 +262,12 @@ int landau_get_mirror(landau_t h, int32_t *mirror_symmetric, int32_t *mirror_act
  * W = wp[nrounds]; a vertex whose rounds share one CTA is summed in one fixed order, whatever the batch.
  * EUNSUPPORTED when the per-vertex kernel is not available on this handle. */
 int landau_get_vtx_schedule(landau_t h, int32_t *nrounds, int32_t *weight_prefix, int32_t *ctas);
+/* The automatic-mode CTAs of the first and the last round of every vertex of an nbatch build (host,
+ * caller-allocated [nbatch] each; first != last: the vertex is split between CTAs and summed through
+ * partial slots).  A split vertex runs its rounds in its own order, chosen on the host so that every
+ * stream-K cut falls on a round boundary (exact balance); the others keep the canonical order of
+ * weight_prefix above.  EUNSUPPORTED as above. */
+int landau_get_vtx_split(landau_t h, int64_t nbatch, int32_t *first_cta, int32_t *last_cta);
 
 /* NEXT-4: the inner integral with the 3D Cartesian Landau tensor of Eq. 3
  * (PAPER.md:1@7593, "a full 3D model is supported in the library" @7997-8072), without azimuthal

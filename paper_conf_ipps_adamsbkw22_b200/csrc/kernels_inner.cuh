@@ -572,13 +572,18 @@ __device__ __forceinline__ void vtx_item_staged(const double2 *s_i, const double
 // vertex cut by a CTA boundary is summed per CTA into a partial slot (the CTA's first segment: slot
 // (c, 0), its last: (c, 1)), and the last CTA to finish one of its segments (an atomic counter per
 // vertex) adds the partials in CTA order -- a fixed order, so every build is bitwise reproducible.
+constexpr int kVtxMaxRounds = 64;   // rounds per vertex the per-vertex kernel supports (host-checked)
 struct VtxSched {
   int nbatch, nrounds, S;
   int64_t Wv, Wtot;      // weight per vertex, whole batch
 };
 
+// wp: the canonical weight prefix [nrounds + 1], or (PERV) the per-vertex prefixes [nbatch][nrounds + 1]
+// of host vtx_tables, where a vertex split between CTAs runs its rounds in an order whose boundaries
+// meet the cuts
+template <bool PERV = false>
 __device__ __forceinline__ int vtx_owner(const VtxSched &sc, const int32_t *wp, int64_t v, int rd) {
-  return (int)(((v * sc.Wv + wp[rd]) * (int64_t)sc.S) / sc.Wtot);
+  return (int)(((v * sc.Wv + wp[(PERV ? v * (sc.nrounds + 1) : 0) + rd]) * (int64_t)sc.S) / sc.Wtot);
 }
 
 // first flattened round index f = v * nrounds + rd owned by CTA >= c (nbatch * nrounds if none):
@@ -607,10 +612,11 @@ __device__ __forceinline__ void vtx_write_G(double *Gb, const double *sGa, const
 // and the mirror maps pu, pm [Hp] int32.
 __host__ __device__ constexpr size_t vtx_smem_bytes(int64_t Hp) { return (size_t)Hp * (20 * 8 + 2 * 4); }
 
-template <bool MASK>
+template <bool MASK, bool PERV>
 __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int64_t N, int64_t H, VtxSched sc,
                                                                       const int32_t *__restrict__ round_ptr,
                                                                       const int32_t *__restrict__ wp,
+                                                                      const int16_t *__restrict__ ord,
                                                                       const VtxItem *__restrict__ items,
                                                                       const double *__restrict__ rU,
                                                                       const double *__restrict__ zU,
@@ -623,6 +629,7 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
   __shared__ double s_coef[kNumPairCoef];
   __shared__ double2 s_ltab[kLogTab];
   __shared__ int s_last;
+  __shared__ int16_t s_ord[kVtxMaxRounds];   // the current vertex's round order
   extern __shared__ double s_G[];   // Ga [5][Hp], Gb [5][Hp] | staged vertex [Hp][5] double2 | pu, pm [Hp]
 #ifdef LANDAU_VTX_TRACE   // build variant: per-CTA timeline (globaltimer ns) printed at exit (scripts/vtx_trace.py)
   unsigned long long tr_[24];
@@ -657,7 +664,36 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
   load_pair_coef(s_coef, s_ltab, cf);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int c = blockIdx.x;
-  const int64_t f0 = vtx_first_round(sc, wp, c), f1 = vtx_first_round(sc, wp, c + 1);
+  // this CTA's range [f0, f1): the two cut vertices' weight prefixes are read in parallel into shared
+  // memory first (a serial scan through global memory costs a dependent L2 miss per round)
+  int64_t f0, f1;
+  if constexpr (!PERV) {
+    f0 = vtx_first_round(sc, wp, c);
+    f1 = vtx_first_round(sc, wp, c + 1);
+  } else {
+    __shared__ int32_t s_w[2][kVtxMaxRounds + 1];
+    int64_t vc[2];
+    for (int e = 0; e < 2; e++) {
+      const int64_t g = ((int64_t)(c + e) * sc.Wtot + sc.S - 1) / sc.S;
+      vc[e] = min(g / sc.Wv, (int64_t)sc.nbatch - 1);
+      for (int k = threadIdx.x; k <= sc.nrounds; k += blockDim.x) s_w[e][k] = wp[vc[e] * (sc.nrounds + 1) + k];
+    }
+    __syncthreads();
+    int64_t fr[2];
+    for (int e = 0; e < 2; e++) {
+      const int64_t g = ((int64_t)(c + e) * sc.Wtot + sc.S - 1) / sc.S;
+      const int64_t v = g / sc.Wv, rem = g - v * sc.Wv;
+      if (v >= sc.nbatch) {
+        fr[e] = (int64_t)sc.nbatch * sc.nrounds;
+      } else {
+        int rd = 0;
+        while (rd < sc.nrounds && s_w[e][rd] < rem) rd++;
+        fr[e] = v * sc.nrounds + rd;
+      }
+    }
+    f0 = fr[0];
+    f1 = fr[1];
+  }
   int64_t f = f0;
   VTX_MARK(1);
   while (f < f1) {
@@ -683,9 +719,12 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
       s_V[u * 5 + 3] = make_double2(0.5 * (A[1] - B[1]), 0.5 * (A[2] - B[2]));
     }
     for (int64_t k = threadIdx.x; k < 10 * Hp; k += blockDim.x) s_G[k] = 0.0;
+    if constexpr (PERV)
+      for (int k = threadIdx.x; k < sc.nrounds; k += blockDim.x) s_ord[k] = ord[v * sc.nrounds + k];
     __syncthreads();
     VTX_MARK(2);
-    for (int rd = rd0; rd < rd1; rd++) {
+    for (int rp = rd0; rp < rd1; rp++) {
+      const int rd = PERV ? (int)s_ord[rp] : rp;   // this vertex's round at position rp
       for (int q = round_ptr[rd] + wid; q < round_ptr[rd + 1]; q += kVtxWarps) {
         const VtxItem it = items[q];
         Acc5 P, M, PJ, MJ;
@@ -700,7 +739,7 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
       __syncthreads();   // the next round's tiles may be this round's
     }
     VTX_MARK(3);
-    const int cfirst = vtx_owner(sc, wp, v, 0), clast = vtx_owner(sc, wp, v, sc.nrounds - 1);
+    const int cfirst = vtx_owner<PERV>(sc, wp, v, 0), clast = vtx_owner<PERV>(sc, wp, v, sc.nrounds - 1);
     if (cfirst == clast) {   // the whole vertex ran here
       vtx_write_G(G + v * G_bstride, sGa, sGb, N, H, Hp, s_pu, s_pm);
     } else {                 // one segment of a split vertex: partial slot, then the last one combines

@@ -106,6 +106,12 @@ struct landau_s {
   int nvtx_rounds = 0;
   size_t vtx_smem = 0;     // dynamic shared memory (Ga, Gb); 0 when the vertex does not fit
   int32_t *d_vtx_wp = nullptr;       // stream-K: prefix of the round weights [nrounds + 1]
+  std::vector<int32_t> vtx_w;        // the rounds' weights (canonical order)
+  // per-batch stream-K tables (vtx_tables): round order and weight prefix per vertex, for (nbatch, S)
+  int16_t *d_vtx_ord = nullptr;
+  int32_t *d_vtx_wpv = nullptr;
+  int64_t vtx_tab_nb = -1;
+  int vtx_tab_S = -1;
   int64_t vtx_Wv = 0;                // weight of one vertex
   double *d_vtx_part = nullptr;      // stream-K partial slots [grid][2][10 Hp]
   int32_t *d_vtx_cnt = nullptr;      // stream-K per-vertex arrival counters [cap] (zero between builds)
@@ -494,6 +500,87 @@ int inner_plan(landau_t h, int64_t nbatch, InnerPlan &ip) {
   return LANDAU_OK;
 }
 
+
+// Stream-K tables of the per-vertex kernel for a batch of nbatch vertices on S CTAs.  The cuts
+// g_c = ceil(c Wtot / S) fall at arbitrary weight offsets; with the canonical round order (pair
+// rounds of weight 2, then diagonal rounds of weight 1) a cut inside a pair round gives one CTA a unit
+// more than its share (128 C2 vertices: 64 CTAs with 33 of 32 units).  A vertex with cuts inside it
+// (split between CTAs anyway) gets its own round order -- rounds of one vertex touch disjoint tiles
+// in any order -- built greedily so that every cut offset is a round boundary: from the previous
+// boundary s to the cut t, (t - s) mod 2 diagonal rounds and the rest pair rounds.  Vertices without
+// inner cuts keep the canonical order (a lone vertex's summation order).  ord [nbatch][R] = round per
+// position, wpv [nbatch][R+1] = weight prefix per position.
+// per-vertex orders pay where a CTA holds few vertices (the cut imbalance is a unit in ~Wv x vertices
+// per CTA); with more, the kernel variant reading the canonical prefix is the faster one (C4 1024
+// vertices: 2548 vs 2561 us; 128: 352.8 vs 347.9 us)
+bool vtx_use_perv(const landau_t h, int64_t nbatch, int S) {
+  static const bool reorder = [] {
+    const char *e = getenv("LANDAU_VTX_REORDER");
+    return !(e && atoi(e) == 0);
+  }();
+  return reorder && nbatch < 4LL * S;
+}
+
+void vtx_tables(const landau_t h, int64_t nbatch, int S, std::vector<int16_t> &ord, std::vector<int32_t> &wpv) {
+  const bool reorder = vtx_use_perv(h, nbatch, S);
+  const int R = h->nvtx_rounds;
+  const int64_t Wv = h->vtx_Wv, Wtot = nbatch * Wv;
+  ord.assign((size_t)nbatch * R, 0);
+  wpv.assign((size_t)nbatch * (R + 1), 0);
+  std::vector<int> twos, ones;
+  for (int r = 0; r < R; r++) (h->vtx_w[r] == 2 ? twos : ones).push_back(r);
+  std::vector<int64_t> cuts;
+  for (int64_t v = 0; v < nbatch; v++) {
+    cuts.clear();   // cut offsets strictly inside vertex v
+    const int64_t c0 = (v * Wv * S) / Wtot, c1 = ((v + 1) * Wv * S + Wtot - 1) / Wtot;
+    for (int64_t c = std::max<int64_t>(c0, 1); c <= c1; c++) {
+      const int64_t g = (c * Wtot + S - 1) / S;
+      if (g > v * Wv && g < (v + 1) * Wv) cuts.push_back(g - v * Wv);
+    }
+    int16_t *o = ord.data() + v * R;
+    int n = 0;
+    if (cuts.empty() || !reorder) {
+      for (int r = 0; r < R; r++) o[n++] = (int16_t)r;
+    } else {
+      size_t it = 0, io = 0;
+      int64_t pos = 0;
+      for (int64_t t : cuts) {
+        if (t <= pos) continue;
+        int64_t need = t - pos;
+        int b = (int)(need & 1);
+        if (b > (int)(ones.size() - io)) b = 0;
+        int64_t a = (need - b) / 2;
+        a = std::min<int64_t>(a, (int64_t)(twos.size() - it));
+        for (int64_t k = 0; k < a; k++, pos += 2) o[n++] = (int16_t)twos[it++];
+        for (int k = 0; k < b; k++, pos += 1) o[n++] = (int16_t)ones[io++];
+      }
+      while (it < twos.size()) o[n++] = (int16_t)twos[it++];
+      while (io < ones.size()) o[n++] = (int16_t)ones[io++];
+    }
+    int32_t *w = wpv.data() + v * (R + 1);
+    w[0] = 0;
+    for (int p = 0; p < R; p++) w[p + 1] = w[p] + h->vtx_w[o[p]];
+  }
+}
+
+int ensure_vtx_tables(landau_t h, int64_t nbatch, int S) {
+  if (h->vtx_tab_nb == nbatch && h->vtx_tab_S == S) return LANDAU_OK;
+  std::vector<int16_t> ord;
+  std::vector<int32_t> wpv;
+  vtx_tables(h, nbatch, S, ord, wpv);
+  drop_graphs(h);   // captured launches hold the old tables
+  cudaFree(h->d_vtx_ord);
+  cudaFree(h->d_vtx_wpv);
+  h->d_vtx_ord = nullptr;
+  h->d_vtx_wpv = nullptr;
+  h->vtx_tab_nb = -1;
+  int rc;
+  if ((rc = upload(h, &h->d_vtx_ord, ord)) || (rc = upload(h, &h->d_vtx_wpv, wpv))) return rc;
+  h->vtx_tab_nb = nbatch;
+  h->vtx_tab_S = S;
+  return LANDAU_OK;
+}
+
 int launch_inner(landau_t h, int64_t nbatch) {
   const Plan &P = h->plan;
   const int64_t N = P.npts;
@@ -598,15 +685,23 @@ int launch_inner(landau_t h, int64_t nbatch) {
     if (h->mirror_mode == 3 && nbatch < sc.S) sc.S = (int)nbatch;
     sc.Wv = h->vtx_Wv;
     sc.Wtot = nbatch * h->vtx_Wv;
+    const bool perv = vtx_use_perv(h, nbatch, sc.S);
+    if (perv && (rc = ensure_vtx_tables(h, nbatch, sc.S))) return rc;
+    const int32_t *wp = perv ? h->d_vtx_wpv : h->d_vtx_wp;
+    const int16_t *ord = perv ? h->d_vtx_ord : nullptr;
     Timer t(h, LANDAU_T_INNER);
-    if (h->coincident)
-      inner_vtx_kernel<true><<<sc.S, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(
-          N, h->H, sc, h->d_vtx_round_ptr, h->d_vtx_wp, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
-          G_own, 5 * h->Nc, h->d_vtx_part, h->d_vtx_cnt);
-    else
-      inner_vtx_kernel<false><<<sc.S, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(
-          N, h->H, sc, h->d_vtx_round_ptr, h->d_vtx_wp, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT,
-          G_own, 5 * h->Nc, h->d_vtx_part, h->d_vtx_cnt);
+#define LAUNCH_VTX(MASK, PERV)                                                                                   \
+  inner_vtx_kernel<MASK, PERV><<<sc.S, 32 * kVtxWarps, h->vtx_smem, h->stream>>>(                                \
+      N, h->H, sc, h->d_vtx_round_ptr, wp, ord, h->d_vtx_items, h->d_rU, h->d_zU, h->d_pu, h->d_pm, h->d_wT, G_own, \
+      5 * h->Nc, h->d_vtx_part, h->d_vtx_cnt)
+    if (h->coincident) {
+      if (perv) LAUNCH_VTX(true, true);
+      else LAUNCH_VTX(true, false);
+    } else {
+      if (perv) LAUNCH_VTX(false, true);
+      else LAUNCH_VTX(false, false);
+    }
+#undef LAUNCH_VTX
     h->launches++;
     h->tlaunch[LANDAU_T_INNER]++;
     KCHECK();
@@ -1027,8 +1122,10 @@ bool raise_vtx_smem_attr(int device, size_t bytes) {
   std::lock_guard<std::mutex> lk(mu);
   size_t &c = cur[device & 63];
   if (bytes <= c) return true;
-  if (cudaFuncSetAttribute(inner_vtx_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess ||
-      cudaFuncSetAttribute(inner_vtx_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess)
+  if (cudaFuncSetAttribute(inner_vtx_kernel<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess ||
+      cudaFuncSetAttribute(inner_vtx_kernel<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess ||
+      cudaFuncSetAttribute(inner_vtx_kernel<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess ||
+      cudaFuncSetAttribute(inner_vtx_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess)
     return false;
   c = bytes;
   return true;
@@ -1283,6 +1380,8 @@ void landau_destroy(landau_t h) {
                     (void *)m.optr, (void *)m.oidx, (void *)m.w4, (void *)m.ow})
       cudaFree(q);
   cudaFree(h->d_vtx_wp);
+  cudaFree(h->d_vtx_ord);
+  cudaFree(h->d_vtx_wpv);
   cudaFree(h->d_vtx_part);
   cudaFree(h->d_vtx_cnt);
   cudaFree(h->d_ext_ptr);
@@ -1860,6 +1959,25 @@ int landau_get_vtx_schedule(landau_t h, int32_t *nrounds, int32_t *weight_prefix
 });
 }
 
+int landau_get_vtx_split(landau_t h, int64_t nbatch, int32_t *first_cta, int32_t *last_cta) {
+  return guarded(h, [&]() -> int {
+  if (!h || nbatch < 1 || !first_cta || !last_cta) return fail(h, LANDAU_EINVAL, "vtx split: bad argument");
+  if (!h->vtx_smem) return fail(h, LANDAU_EUNSUPPORTED, "vtx schedule: the per-vertex kernel is not available");
+  const int S = h->host_only ? 148 * kVtxMinB : num_sms(h) * kVtxMinB;
+  std::vector<int16_t> ord;
+  std::vector<int32_t> wpv;
+  vtx_tables(h, nbatch, S, ord, wpv);
+  const int R = h->nvtx_rounds;
+  const int64_t Wtot = nbatch * h->vtx_Wv;
+  for (int64_t v = 0; v < nbatch; v++) {
+    const int32_t *w = wpv.data() + v * (R + 1);
+    first_cta[v] = (int32_t)(((v * h->vtx_Wv + w[0]) * S) / Wtot);
+    last_cta[v] = (int32_t)(((v * h->vtx_Wv + w[R - 1]) * S) / Wtot);
+  }
+  return LANDAU_OK;
+});
+}
+
 int landau_get_mirror(landau_t h, int32_t *mirror_symmetric, int32_t *mirror_active) {
   return guarded(h, [&]() -> int {
   if (!h) return LANDAU_EINVAL;
@@ -2128,7 +2246,7 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
           }
       }
       const size_t vsmem = vtx_smem_bytes((int64_t)T * 32);
-      h->vtx_smem = world == 1 && vsmem <= (size_t)200 * 1024 && T >= 2 ? vsmem : 0;
+      h->vtx_smem = world == 1 && vsmem <= (size_t)200 * 1024 && T >= 2 && (int)vround.size() - 1 <= kVtxMaxRounds ? vsmem : 0;
       h->nvtx_rounds = (int)vround.size() - 1;
       // stream-K weights: a round lasts as long as its longest item (pair item 2, diagonal item 1)
       std::vector<int32_t> vwp(1, 0);
@@ -2138,6 +2256,8 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
         vwp.push_back(vwp.back() + w);
       }
       h->vtx_Wv = vwp.back();
+      h->vtx_w.clear();
+      for (int rd = 0; rd < h->nvtx_rounds; rd++) h->vtx_w.push_back(vwp[rd + 1] - vwp[rd]);
       if (h->vtx_smem) {
         if ((rc = upload(h, &h->d_vtx_items, vitems)) || (rc = upload(h, &h->d_vtx_round_ptr, vround)) ||
             (rc = upload(h, &h->d_vtx_wp, vwp)))

@@ -95,6 +95,7 @@ def lib():
             "landau_set_mirror": (C.c_int, [vp, i32]),
             "landau_get_mirror": (C.c_int, [vp, P32, P32]),
             "landau_get_vtx_schedule": (C.c_int, [vp, P32, P32, P32]),
+            "landau_get_vtx_split": (C.c_int, [vp, i64, P32, P32]),
             "landau_band_info": (C.c_int, [vp, i32, P32, P32]),
             "landau_band_factor_batched": (C.c_int, [vp, i64, d, vp]),
             "landau_band_solve_batched": (C.c_int, [vp, i64, vp, vp]),
@@ -488,11 +489,9 @@ class Landau:
 
     def vtx_split_vertices(self, nbatch):
         """Batch items whose rounds an automatic-mode build spreads over more than one CTA."""
-        wp, S = self.vtx_schedule()
-        W = int(wp[-1])
-        v = np.arange(nbatch, dtype=np.int64)
-        first = (v * W + int(wp[0])) * S // (nbatch * W)
-        last = (v * W + int(wp[-2])) * S // (nbatch * W)
+        first, last = np.zeros(nbatch, dtype=np.int32), np.zeros(nbatch, dtype=np.int32)
+        self._check(lib().landau_get_vtx_split(self._h, int(nbatch), first.ctypes.data_as(C.POINTER(C.c_int32)),
+                                               last.ctypes.data_as(C.POINTER(C.c_int32))), "landau_get_vtx_split")
         return np.nonzero(first != last)[0]
 
     def set_tensor_cache(self, enable=True):
