@@ -218,13 +218,13 @@ def load_profile_traffic(key):
 
 # FP64 FLOP (2*DFMA + DMUL + DADD) per pair evaluation, counted once from ncu
 # sm__sass_thread_inst_executed_op_{dfma,dmul,dadd}_pred_on of each inner kernel on the C4 workload
-# (profiles/r01_flops_*.csv):
-FLOP_PER_PAIR_DIRECTED = 173.0   # inner_kernel, per ordered (target, source) pair
-FLOP_PER_PAIR_SYMMETRIC = 189.2  # inner_sym_kernel, per unordered pair
-FLOP_PER_EVAL_MIRROR = 194.7     # inner_mir_kernel (slot kernel), per U or V tensor evaluation
-FLOP_PER_EVAL_VTX = 195.0        # inner_vtx_kernel (per-vertex kernel), per U or V tensor evaluation
+# (profiles/r02_flops_*.csv with the degree-9 D fit):
+FLOP_PER_PAIR_DIRECTED = 169.0   # inner_kernel, per ordered (target, source) pair
+FLOP_PER_PAIR_SYMMETRIC = 185.2  # inner_sym_kernel, per unordered pair
+FLOP_PER_EVAL_MIRROR = 190.1     # inner_mir_kernel (slot kernel), per U or V tensor evaluation
+FLOP_PER_EVAL_VTX = 190.2        # inner_vtx_kernel (per-vertex kernel), per U or V tensor evaluation
 FLOP_PER_PAIR_3D = 58.0          # inner3d_kernel, per ordered pair
-FLOP_PER_EVAL_MDIR = 183.2       # inner_mdir_kernel (mirror directed), per padded U or V evaluation
+FLOP_PER_EVAL_MDIR = 179.2       # inner_mdir_kernel (mirror directed), per padded U or V evaluation
 INNER_PATHS = ["directed (ordered pairs)", "symmetric (unordered pairs)", "tensor cache + FP64 DGEMM (cuBLAS)",
                "mirror-symmetric slot kernel (one tensor per unordered pair and its z-mirror)",
                "mirror-symmetric per-vertex kernel (stream-K over vertex rounds, sums in shared memory)",
