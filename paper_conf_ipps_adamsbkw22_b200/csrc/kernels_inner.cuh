@@ -632,10 +632,10 @@ __global__ void __launch_bounds__(32 * kVtxWarps, kVtxMinB) inner_vtx_kernel(int
   __shared__ int16_t s_ord[kVtxMaxRounds];   // the current vertex's round order
   extern __shared__ double s_G[];   // Ga [5][Hp], Gb [5][Hp] | staged vertex [Hp][5] double2 | pu, pm [Hp]
 #ifdef LANDAU_VTX_TRACE   // build variant: per-CTA timeline (globaltimer ns) printed at exit (scripts/vtx_trace.py)
-  unsigned long long tr_[24];
+  unsigned long long tr_[64];
   int ntr_ = 0;
 #define VTX_MARK(tag)                                                                                   \
-  if (threadIdx.x == 0 && ntr_ < 24) {                                                                  \
+  if (threadIdx.x == 0 && ntr_ < 64) {                                                                  \
     unsigned long long t_;                                                                              \
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                                              \
     tr_[ntr_++] = (t_ << 4) | (tag);                                                                    \

@@ -1,4 +1,4 @@
-"""A/B of the overlapped C4 pipeline (LANDAU_OVERLAP = K chunks): per-step time of the whole Jacobian
+"""A/B of a library knob (env var ENVVAR, default LANDAU_OVERLAP = K chunks): per-step time of the whole Jacobian
 build (graph replay, median of per-step CUDA events, L2 flushed between steps) and the CSR values'
 largest difference from the K = 1 build, relative to max |J|.  Each K runs in its own process (the
 knob is read once).  Usage: python scripts/overlap_ab.py [B] K1 K2 ...   (first K is the reference)"""
@@ -32,9 +32,9 @@ ref = None
 import numpy as np
 for rep in range(int(os.environ.get("REPS", "2"))):
     for K in sys.argv[2:]:
-        out = f"/tmp/J_{K}.npy"
+        out = "/tmp/J_%d.npy" % sys.argv[2:].index(K)
         r = subprocess.run([sys.executable, "-c", CHILD, out, B], capture_output=True, text=True,
-                           env=dict(os.environ, LANDAU_OVERLAP=K))
+                           env=dict(os.environ, **{os.environ.get("ENVVAR", "LANDAU_OVERLAP"): K}))
         msg = r.stdout.strip() or r.stderr[-800:]
         if r.returncode == 0:
             Jv = np.load(out)
