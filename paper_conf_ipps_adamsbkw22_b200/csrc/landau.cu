@@ -1078,7 +1078,7 @@ int dispatch_build(landau_t h, int64_t nbatch, double *out, int format) {
   ce = cudaGraphInstantiate(&exec, graph, 0);
   cudaGraphDestroy(graph);
   if (ce != cudaSuccess) return fail(h, LANDAU_ECUDA, std::string("graph instantiate: ") + cudaGetErrorString(ce));
-  if (h->graphs.size() >= 16) {
+  if (h->graphs.size() >= 32) {   // (landau_jacobian_host keeps one graph per chunk: up to 16)
     cudaGraphExecDestroy(h->graphs.front().exec);
     h->graphs.erase(h->graphs.begin());
   }
@@ -1541,10 +1541,13 @@ int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, doubl
   }
   static const int64_t kmax = [] {
     const char *e = getenv("LANDAU_HOST_CHUNKS");
-    return e ? (int64_t)atoll(e) : (int64_t)8;   // 16 measured no better
+    // C4 1024 vertices (scripts/e2e_probe.py, one B200, D2H 56.7 GB/s): 8 chunks 4.65 ms, 16 4.48 ms,
+    // 32 4.88 ms; a shorter first chunk (16-48 vertices) 5.0-5.9 ms
+    return e ? (int64_t)atoll(e) : (int64_t)16;
   }();
-  const int64_t K = std::max<int64_t>(1, std::min<int64_t>(kmax, nbatch / 64));
-  const int64_t cb = (nbatch + K - 1) / K;
+  const int64_t K = std::max<int64_t>(1, std::min<int64_t>(kmax, nbatch / 32));
+  std::vector<int64_t> bnd{0};   // chunk boundaries (equal chunks)
+  for (int64_t c = 1; c <= K; c++) bnd.push_back(nbatch * c / K);
   while ((int64_t)h->ev_h2d.size() < K) {
     cudaEvent_t a, b;
     CU(cudaEventCreateWithFlags(&a, cudaEventDisableTiming));
@@ -1557,8 +1560,8 @@ int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, doubl
   CU(cudaStreamWaitEvent(h->s_h2d, h->ev_built[0], 0));
   CU(cudaStreamWaitEvent(h->s_d2h, h->ev_built[0], 0));
   for (int64_t c = 0; c < K; c++) {
-    const int64_t b0 = c * cb, n = std::min(cb, nbatch - b0);
-    if (n <= 0) break;
+    const int64_t b0 = bnd[c], n = bnd[c + 1] - bnd[c];
+    if (n <= 0) continue;
     CU(cudaMemcpyAsync(h->d_f + b0 * h->ndof, f_host + b0 * h->ndof, sizeof(double) * n * h->ndof,
                        cudaMemcpyHostToDevice, h->s_h2d));
     CU(cudaEventRecord(h->ev_h2d[c], h->s_h2d));
@@ -1572,7 +1575,7 @@ int landau_jacobian_host(landau_t h, int64_t nbatch, const double *f_host, doubl
     CU(cudaMemcpyAsync(values_host + b0 * nv, h->d_vals_tmp + b0 * nv, sizeof(double) * n * nv,
                        cudaMemcpyDeviceToHost, h->s_d2h));
   }
-  h->nbatch = cb;          // the device state now holds the last chunk's batch layout
+  h->nbatch = bnd.back() - bnd[bnd.size() - 2];   // the device state now holds the last chunk's batch layout
   h->have_state = false;   // (d_f holds the whole host batch, but not as one set_state)
   CU(cudaStreamSynchronize(h->s_d2h));
   CU(cudaStreamSynchronize(h->stream));
