@@ -2,8 +2,9 @@
 # (symmetric, mirror-slot, per-vertex and mirror-directed inner kernels; band LU, solve and the implicit
 # step with and without the quench source; the 3D Cartesian inner integral; one emulated rank of the pair
 # split), the fused single-build kernel (C1, C3 without timers), the element/assembly kernels (timed
-# builds), and a 200-vertex batch (more vertices than SMs: the per-vertex kernel loops over several
-# vertices per CTA and splits some between CTAs), the 3D Cartesian Jacobian.  Argument "tail":
+# builds), a 200-vertex batch (more vertices than SMs: the per-vertex kernel loops over several
+# vertices per CTA and splits some between CTAs) and a 640-vertex one (the headline's canonical-order
+# variant), the pipelined host entry point, the 3D Cartesian Jacobian.  Argument "tail":
 # LANDAU_TAIL=1 (the fused tail kernel); "bandcw": LANDAU_BAND_CW=1 (the column-warp band factorisation).
 import os, sys
 if len(sys.argv) > 1 and sys.argv[1] == "tail":
@@ -65,6 +66,19 @@ v2 = torch.empty((nb, h.nnz), dtype=torch.float64, device="cuda")
 h.jacobian_batched(v2)
 torch.cuda.synchronize()
 print("stats 200", h.stats(), "split", len(h.vtx_split_vertices(nb)))
+# the headline's variant: >= 4 vertices per CTA (canonical round order, several whole vertices per CTA)
+nb = 640
+F4 = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b % 200), nodes) for b in range(nb)]), device="cuda")
+h.set_state_batched(F4)
+v4 = torch.empty((nb, h.nnz), dtype=torch.float64, device="cuda")
+h.jacobian_batched(v4)
+torch.cuda.synchronize()
+print("stats 640", h.stats(), "split", len(h.vtx_split_vertices(nb)))
+# the end-to-end entry point: pipelined chunks (H2D, build, D2H on three streams)
+fh = F4[:256].cpu().pin_memory()
+vh = torch.empty((256, h.nnz), dtype=torch.float64).pin_memory()
+h.jacobian_host(fh, vh)
+print("ok host chunks")
 # NEXT-4: the 3D Cartesian inner integral (split-j and direct)
 xyz3, w3 = inputs.points3d(2, 2)
 wTD3, wTK3 = inputs.fields3d(xyz3, w3)
