@@ -28,6 +28,7 @@ using namespace landau;
 #include "kernels_fe.cuh"
 #include "kernels_inner.cuh"
 #include "kernels_band.cuh"
+#include "kernels_band_mma.cuh"
 #include "kernels_single.cuh"
 #include "kernels_3d.cuh"
 #include "kernels_3d_fe.cuh"
@@ -1816,7 +1817,20 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
       (const void *)band_lu_cw_kernel<4>, (const void *)band_lu_cw_kernel<5>,  (const void *)band_lu_cw_kernel<6>,
       (const void *)band_lu_cw_kernel<7>, (const void *)band_lu_cw_kernel<8>,  (const void *)band_lu_cw_kernel<9>,
       (const void *)band_lu_cw_kernel<10>, (const void *)band_lu_cw_kernel<11>, (const void *)band_lu_cw_kernel<12>};
-  if (band_cw && same_p && maxPp <= 96 && maxPp % 8 == 0 && h->band_ent_max <= kBandE * 256) {
+  static const bool band_mma = [] {   // the blocked DMMA factorisation (kernels_band_mma.cuh)
+    const char *e = getenv("LANDAU_BAND_MMA");
+    return !(e && atoi(e) == 0);
+  }();
+#define BM(NT) (const void *)band_lu_mma_kernel<NT>
+  static const void *const mma_kernels[18] = {nullptr, nullptr, nullptr, BM(3),  BM(4),  BM(5),  BM(6),  BM(7),  BM(8),
+                                              BM(9),   BM(10),  BM(11),  BM(12), BM(13), BM(14), BM(15), BM(16), BM(17)};
+#undef BM
+  const int mma_nt = maxPp / 8 + 1;
+  if (band_mma && same_p && maxPp % 8 == 0 && mma_nt >= 3 && mma_nt <= 17) {
+    kfn = mma_kernels[mma_nt];
+    ksmem = sizeof(double) * band_mma_smem_doubles(mma_nt);
+    threads = 32 * kBmWarps;
+  } else if (band_cw && same_p && maxPp <= 96 && maxPp % 8 == 0 && h->band_ent_max <= kBandE * 256) {
     // column-warp kernel with look-ahead: 8 warps of P / 8 columns (one window width per launch)
     kfn = cw_kernels[maxPp / 8 - 1];
     ksmem = sizeof(double) * (2 * kCwRing + 48) * maxPp;
