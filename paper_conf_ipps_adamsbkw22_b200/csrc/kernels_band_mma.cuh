@@ -44,7 +44,8 @@ constexpr int kBmWarps = 8;
 constexpr int kBmE = 2;    // entering entries per thread and group of 8 indices (host-checked)
 constexpr int kBmTS = 72;  // panel tile stride: 8 rows of 9 (padded: conflict-free row loads in phase B)
 
-// diagonal -> (warp, first accumulator slot), longest diagonals first to the least-loaded warp
+// diagonal -> (warp, first accumulator slot): the main diagonal on warp 0; the others longest first to
+// the least-loaded of warps 1-7
 template <int NT>
 struct BmPlan {
   int warp[2 * NT - 1], off[2 * NT - 1], load[kBmWarps];
@@ -53,10 +54,13 @@ template <int NT>
 constexpr BmPlan<NT> bm_plan() {
   BmPlan<NT> pl{};
   for (int w = 0; w < kBmWarps; w++) pl.load[w] = 0;
-  for (int a = 0; a < 2 * NT - 1; a++) {
+  pl.warp[NT - 1] = 0;   // the main diagonal alone on warp 0, which also factors the next corner
+  pl.off[NT - 1] = 0;
+  pl.load[0] = NT;
+  for (int a = 1; a < 2 * NT - 1; a++) {
     const int d = (a + 1) / 2 * (a % 2 ? 1 : -1), len = NT - (d < 0 ? -d : d);
-    int best = 0;
-    for (int w = 1; w < kBmWarps; w++)
+    int best = 1;
+    for (int w = 2; w < kBmWarps; w++)
       if (pl.load[w] < pl.load[best]) best = w;
     pl.warp[d + NT - 1] = best;
     pl.off[d + NT - 1] = pl.load[best];
@@ -83,9 +87,9 @@ __device__ __forceinline__ void bm_for_diags(F &&f) {
 }
 
 // shared memory (doubles): panels [2 parities][2][NT][72], fragments of -L21 and U12 [2][NT][2][32],
-// factored corner (64) + pivot reciprocals (8), entering buffers [2 parities][2][8][8 NT]
+// factored corner (64) + pivot reciprocals (8) [2 parities], entering buffers [2 parities][2][8][8 NT]
 __host__ __device__ constexpr int band_mma_smem_doubles(int NT) {
-  return 4 * NT * kBmTS + 2 * NT * 64 + 72 + 4 * 8 * 8 * NT;
+  return 4 * NT * kBmTS + 2 * NT * 64 + 2 * 72 + 4 * 8 * 8 * NT;
 }
 
 struct BmArgs {
@@ -97,24 +101,56 @@ struct BmArgs {
   double *pan0, *lfr, *ufr, *cor, *ebuf0;
 };
 
+// LU of the 8 x 8 corner held as a DMMA accumulator fragment (lane: row g, columns c0, c0 + 1), in
+// place (U on and above the diagonal, L below), pivots shared by shuffles; writes it row-major to cr[64]
+// and the pivot reciprocals to cr[64 + t]
+__device__ __forceinline__ void bm_corner_lu(double &v0, double &v1, double *cr, int lane) {
+  const int g = lane >> 2, c0 = 2 * (lane & 3);
+#pragma unroll
+  for (int t = 0; t < 8; t++) {
+    const double sel = (t & 1) ? v1 : v0;
+    const double piv = __shfl_sync(0xffffffffu, sel, 4 * t + (t >> 1));
+    const double at = __shfl_sync(0xffffffffu, sel, 4 * g + (t >> 1));
+    const double u0 = __shfl_sync(0xffffffffu, v0, 4 * t + (lane & 3));
+    const double u1 = __shfl_sync(0xffffffffu, v1, 4 * t + (lane & 3));
+    const double rp = rcp_newton(piv);
+    if (lane == 0) cr[64 + t] = rp;
+    const double l = at * rp;
+    const bool below = g > t;
+    v0 = below ? (c0 > t ? fma(-l, u0, v0) : (c0 == t ? l : v0)) : v0;
+    v1 = below ? (c0 + 1 > t ? fma(-l, u1, v1) : (c0 + 1 == t ? l : v1)) : v1;
+  }
+  cr[g * 8 + c0] = v0;
+  cr[g * 8 + c0 + 1] = v1;
+}
+
 // the warp-specialised pieces (accumulator indices static): publish the first tile of each owned
 // diagonal (phase A), the rank-8 DMMA update (phase C), the shift + entering tiles (phase C)
 template <int NT, int WID, int TPW>
 __device__ __forceinline__ void bm_publish(double (&acc)[TPW][2], double *colp, double *rowp, int g, int c0) {
   bm_for_diags<NT, WID>([&](auto dc, auto mc) {
     constexpr int d = decltype(dc)::value, m0 = decltype(mc)::value;
-    double *t = d > 0 ? rowp + d * kBmTS : colp + (d < 0 ? -d : 0) * kBmTS;
-    t[g * 9 + c0] = acc[m0][0];
-    t[g * 9 + c0 + 1] = acc[m0][1];
+    if constexpr (d != 0) {   // (the corner was factored ahead, in the previous panel's phase C)
+      double *t = d > 0 ? rowp + d * kBmTS : colp + (-d) * kBmTS;
+      t[g * 9 + c0] = acc[m0][0];
+      t[g * 9 + c0 + 1] = acc[m0][1];
+    }
   });
 }
 template <int NT, int WID, int TPW>
-__device__ __forceinline__ void bm_update(double (&acc)[TPW][2], const double *lfr, const double *ufr, int lane) {
+__device__ __forceinline__ void bm_update(double (&acc)[TPW][2], const double *lfr, const double *ufr, int lane,
+                                          double *cnext) {
   bm_for_diags<NT, WID>([&](auto dc, auto mc) {
     constexpr int d = decltype(dc)::value, m0 = decltype(mc)::value;
     constexpr int len = NT - (d < 0 ? -d : d), I0 = d < 0 ? -d : 0, J0 = d > 0 ? d : 0;
+    constexpr int i0 = d == 0 ? 2 : 1;
+    if constexpr (d == 0) {   // look-ahead: update tile (1, 1) first and factor it -- the next corner
+      dmma_8x8x4(acc[m0 + 1][0], acc[m0 + 1][1], lfr[64 + lane], ufr[64 + lane]);
+      dmma_8x8x4(acc[m0 + 1][0], acc[m0 + 1][1], lfr[96 + lane], ufr[96 + lane]);
+      if (cnext) bm_corner_lu(acc[m0 + 1][0], acc[m0 + 1][1], cnext, lane);
+    }
 #pragma unroll
-    for (int i = 1; i < len; i++) {
+    for (int i = i0; i < len; i++) {
       const double *fa = lfr + (I0 + i) * 64, *fb = ufr + (J0 + i) * 64;
       dmma_8x8x4(acc[m0 + i][0], acc[m0 + i][1], fa[lane], fb[lane]);
       dmma_8x8x4(acc[m0 + i][0], acc[m0 + i][1], fa[32 + lane], fb[32 + lane]);
@@ -193,11 +229,13 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
       }
     }
   };
+  // ep / (4P) by a multiply: ep < 32 P <= 4096, so the rounding error ep / 2^24 stays below 1 / (4P)
+  const unsigned qmul = (1u << 24) / (unsigned)(4 * P) + 1u;
   auto scatter_group = [&](double *er) {   // dense rows er[q][col] (row parts), er[8 Q + q][row] (column parts)
 #pragma unroll
     for (int m = 0; m < kBmE; m++)
       if (ep[m] >= 0) {
-        const int q = ep[m] / (4 * P), s = ep[m] - q * 4 * P;
+        const int q = (int)(((unsigned)ep[m] * qmul) >> 24), s = ep[m] - q * 4 * P;   // q = ep / 4P
         if (s < P) er[q * Q + q + 1 + s] = ev[m];                  // A(i, j), j = i - Bp + s: window column q + 1 + s
         else er[8 * Q + q * Q + q + s - 2 * P + 1] = ev[m];        // A(j, i), j = i + s - 3P + 1: window row q + s - 2P + 1
       }
@@ -226,36 +264,13 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
     }
     load_group(p + 1 + NT);
     asm volatile("bar.sync 0, %0;" ::"n"(32 * kBmWarps) : "memory");
-    // ---- B: panel factorisation (warps 0-6), clear the next entering buffer (warp 7)
-    if (warp == 7) {
-      for (int i = lane; i < 2 * 8 * Q; i += 32) er1[i] = 0.0;
+    // ---- B: L21 and U12 from the corner factored ahead (warps 1-6); warps 0 and 7 clear the next
+    // entering buffer
+    double *cor = A.cor + par * 72;
+    if (warp == 0 || warp == 7) {
+      for (int i = (warp ? 32 : 0) + lane; i < 2 * 8 * Q; i += 64) er1[i] = 0.0;
     } else if (p >= 0) {
-      double *cor = A.cor;
-      if (warp == 0) {   // corner LU: lane holds row g, columns c0, c0 + 1
-        double v0 = colp[g * 9 + c0], v1 = colp[g * 9 + c0 + 1];
-#pragma unroll
-        for (int t = 0; t < 8; t++) {
-          const double sel = (t & 1) ? v1 : v0;
-          const double piv = __shfl_sync(0xffffffffu, sel, 4 * t + (t >> 1));
-          const double at = __shfl_sync(0xffffffffu, sel, 4 * g + (t >> 1));
-          const double u0 = __shfl_sync(0xffffffffu, v0, 4 * t + (lane & 3));
-          const double u1 = __shfl_sync(0xffffffffu, v1, 4 * t + (lane & 3));
-          const double rp = rcp_newton(piv);
-          if (lane == 0) cor[64 + t] = rp;
-          if (g > t) {
-            const double l = at * rp;
-            if (c0 > t) v0 = fma(-l, u0, v0);
-            else if (c0 == t) v0 = l;
-            if (c0 + 1 > t) v1 = fma(-l, u1, v1);
-            else if (c0 + 1 == t) v1 = l;
-          }
-        }
-        cor[g * 8 + c0] = v0;
-        cor[g * 8 + c0 + 1] = v1;
-        __threadfence_block();
-        asm volatile("bar.arrive 1, %0;" ::"n"(32 * 7) : "memory");
-      } else {
-        asm volatile("bar.sync 1, %0;" ::"n"(32 * 7) : "memory");
+      {
         if (warp <= 3) {   // L21 = A21 U11^-1: window row r = 8 + (tid - 32)
           const int r = 8 + tid - 32;
           if (r < Q) {
@@ -300,7 +315,8 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
     asm volatile("bar.sync 0, %0;" ::"n"(32 * kBmWarps) : "memory");
     // ---- C: rank-8 trailing update of the tiles with I, J >= 1 (all but the first of each diagonal)
     if (p >= 0) {
-#define BM_UPD(w) bm_update<NT, w, TPW>(acc, A.lfr, A.ufr, lane)
+    double *cnext = p + 1 < A.npan ? A.cor + (par ^ 1) * 72 : nullptr;
+#define BM_UPD(w) bm_update<NT, w, TPW>(acc, A.lfr, A.ufr, lane, cnext)
       BM_SWITCH(BM_UPD)
 #undef BM_UPD
       // factor row k + warp: (U(t, t), U(t, t+1 .. t+Bp), L(t+1 .. t+Bp, t)) in window coordinates
@@ -310,13 +326,13 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
         for (int s = lane; s < W; s += 32) {
           double v;
           if (s == 0) {
-            v = A.cor[t * 9];
+            v = cor[t * 9];
           } else if (s <= Bp) {
             const int c = t + s;
-            v = c < 8 ? A.cor[t * 8 + c] : rowp[(c >> 3) * kBmTS + t * 9 + (c & 7)];
+            v = c < 8 ? cor[t * 8 + c] : rowp[(c >> 3) * kBmTS + t * 9 + (c & 7)];
           } else {
             const int r = t + s - Bp;
-            v = r < 8 ? A.cor[r * 8 + t] : colp[(r >> 3) * kBmTS + (r & 7) * 9 + t];
+            v = r < 8 ? cor[r * 8 + t] : colp[(r >> 3) * kBmTS + (r & 7) * 9 + t];
           }
           out[s] = v;
         }
@@ -328,6 +344,7 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
 #define BM_SH(w) bm_shift<NT, w, TPW>(acc, er, g, c0, k1, n)
     BM_SWITCH(BM_SH)
 #undef BM_SH
+    if (p == -1 && warp == 0) bm_corner_lu(acc[0][0], acc[0][1], A.cor, lane);   // the first corner
     scatter_group(er1);
   }
 }
@@ -356,7 +373,7 @@ __global__ void __launch_bounds__(32 * kBmWarps, NT <= 12 ? 2 : 1) band_lu_mma_k
   A.lfr = A.pan0 + 4 * NT * kBmTS;
   A.ufr = A.lfr + NT * 64;
   A.cor = A.ufr + NT * 64;
-  A.ebuf0 = A.cor + 72;
+  A.ebuf0 = A.cor + 2 * 72;
   bm_body<NT>(A);
 }
 

@@ -1826,15 +1826,17 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
                                               BM(9),   BM(10),  BM(11),  BM(12), BM(13), BM(14), BM(15), BM(16), BM(17)};
 #undef BM
   const int mma_nt = maxPp / 8 + 1;
-  if (band_mma && same_p && maxPp % 8 == 0 && mma_nt >= 3 && mma_nt <= 17) {
-    kfn = mma_kernels[mma_nt];
-    ksmem = sizeof(double) * band_mma_smem_doubles(mma_nt);
-    threads = 32 * kBmWarps;
-  } else if (band_cw && same_p && maxPp <= 96 && maxPp % 8 == 0 && h->band_ent_max <= kBandE * 256) {
+  if (band_cw && same_p && maxPp <= 96 && maxPp % 8 == 0 && h->band_ent_max <= kBandE * 256) {
     // column-warp kernel with look-ahead: 8 warps of P / 8 columns (one window width per launch)
     kfn = cw_kernels[maxPp / 8 - 1];
     ksmem = sizeof(double) * (2 * kCwRing + 48) * maxPp;
     threads = 256;
+  } else if (band_mma && same_p && maxPp % 8 == 0 && mma_nt >= 3 && mma_nt <= 17 &&
+             h->band_ent_max <= kBmE * 32 * kBmWarps) {
+    // blocked factorisation, DMMA trailing updates (kernels_band_mma.cuh): C4 2.0 ms vs 3.2 ms
+    kfn = mma_kernels[mma_nt];
+    ksmem = sizeof(double) * band_mma_smem_doubles(mma_nt);
+    threads = 32 * kBmWarps;
   } else if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
     kfn = band_minb >= 2 ? (const void *)band_lu2_kernel<4, 8, 2> : (const void *)band_lu2_kernel<4, 8, 1>;
   else               // 8 x 8 tiles, <= 256 threads

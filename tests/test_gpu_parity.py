@@ -1184,11 +1184,12 @@ np.savez(path, x=x.cpu().numpy(), b=b.cpu().numpy(), J=J.cpu().numpy(), shift=sh
 '''
 
 
-def test_band_column_warp_kernel_matches():
-    """The opt-in column-warp band factorisation (LANDAU_BAND_CW=1: warps own cyclic columns, the
-    multipliers handed over through named barriers, look-ahead on the next pivot column) solves the
-    same C4 systems as the default register-tile kernel: both agree with a sparse direct solve of the
-    same A = shift M - J (the rank-1 and rank-2 eliminations round differently)."""
+def test_band_factorisation_kernels_match():
+    """The three band factorisations solve the same C4 systems: the default blocked DMMA kernel
+    (band_lu_mma_kernel: 8-column panels, rank-8 trailing updates on the FP64 tensor cores), the
+    register-tile rank-2 kernel (LANDAU_BAND_MMA=0) and the opt-in column-warp kernel
+    (LANDAU_BAND_CW=1); each agrees with a sparse direct solve of the same A = shift M - J (the
+    eliminations round differently), and the Jacobians they factor are identical."""
     import os
     import subprocess
     import sys
@@ -1196,24 +1197,25 @@ def test_band_column_warp_kernel_matches():
     import scipy.sparse as sps
     import scipy.sparse.linalg as spla
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    variants = {"mma": {}, "rt": {"LANDAU_BAND_MMA": "0"}, "cw": {"LANDAU_BAND_CW": "1"}}
     res = {}
     with tempfile.TemporaryDirectory() as td:
-        for cw in ("1", "0"):
-            path = os.path.join(td, f"x{cw}.npz")
+        for name, env in variants.items():
+            path = os.path.join(td, f"x_{name}.npz")
             out = subprocess.run([sys.executable, "-c", _BAND_CHILD, path, "4"], capture_output=True, text=True,
-                                 timeout=600, cwd=root, env=dict(os.environ, LANDAU_BAND_CW=cw))
+                                 timeout=600, cwd=root, env=dict(os.environ, **env))
             assert out.returncode == 0, out.stderr[-3000:]
-            res[cw] = dict(np.load(path))
+            res[name] = dict(np.load(path))
     o = Oracle(inputs.config4_vertex(0))
     rp, col = o.pattern()
     M = o.mass(1.0)
     for k in range(4):
-        J = res["0"]["J"][k]
-        assert np.array_equal(J, res["1"]["J"][k])
-        A = sps.csr_matrix((res["0"]["shift"] * M - J, col, rp), shape=(o.ndof, o.ndof))
-        x_ref = spla.spsolve(A.tocsc(), res["0"]["b"][k])
-        for cw in ("0", "1"):
-            assert np.max(np.abs(res[cw]["x"][k] - x_ref)) <= 1e-10 * np.max(np.abs(x_ref))
+        J = res["mma"]["J"][k]
+        A = sps.csr_matrix((res["mma"]["shift"] * M - J, col, rp), shape=(o.ndof, o.ndof))
+        x_ref = spla.spsolve(A.tocsc(), res["mma"]["b"][k])
+        for name in variants:
+            assert np.array_equal(J, res[name]["J"][k])
+            assert np.max(np.abs(res[name]["x"][k] - x_ref)) <= 1e-10 * np.max(np.abs(x_ref)), name
 
 
 @pytest.mark.parametrize("ncell,order", [(2, 2), (2, 3), (3, 3)])
