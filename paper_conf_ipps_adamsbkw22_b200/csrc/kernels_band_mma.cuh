@@ -249,6 +249,12 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
     scatter_group(er);
     asm volatile("bar.sync 0, %0;" ::"n"(32 * kBmWarps) : "memory");
   }
+#ifdef LANDAU_BM_TRACE   // build variant: clock64 per phase, printed by lane 0 of every warp of CTA 0
+  long long tph[6] = {0, 0, 0, 0, 0, 0}, t_ = clock64();
+#define BM_T(i) { const long long t2_ = clock64(); tph[i] += t2_ - t_; t_ = t2_; }
+#else
+#define BM_T(i)
+#endif
   for (int p = -NT; p < A.npan; p++) {
     const int par = p & 1;
     double *colp = A.pan0 + par * 2 * NT * kBmTS;   // tiles (I, 0): element (r, c) at I*72 + r*9 + c
@@ -263,7 +269,9 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
 #undef BM_PUB
     }
     load_group(p + 1 + NT);
+    BM_T(0)
     asm volatile("bar.sync 0, %0;" ::"n"(32 * kBmWarps) : "memory");
+    BM_T(1)
     // ---- B: L21 and U12 from the corner factored ahead (warps 1-6); warps 0 and 7 clear the next
     // entering buffer
     double *cor = A.cor + par * 72;
@@ -312,7 +320,9 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
         }
       }
     }
+    BM_T(2)
     asm volatile("bar.sync 0, %0;" ::"n"(32 * kBmWarps) : "memory");
+    BM_T(3)
     // ---- C: rank-8 trailing update of the tiles with I, J >= 1 (all but the first of each diagonal)
     if (p >= 0) {
     double *cnext = p + 1 < A.npan ? A.cor + (par ^ 1) * 72 : nullptr;
@@ -345,8 +355,14 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
     BM_SWITCH(BM_SH)
 #undef BM_SH
     if (p == -1 && warp == 0) bm_corner_lu(acc[0][0], acc[0][1], A.cor, lane);   // the first corner
+    BM_T(4)
     scatter_group(er1);
+    BM_T(5)
   }
+#ifdef LANDAU_BM_TRACE
+  if (blockIdx.x == 0 && lane == 0)
+    printf("BM warp %d A %lld barA %lld B %lld barB %lld C %lld scatter %lld\n", warp, tph[0], tph[1], tph[2], tph[3], tph[4], tph[5]);
+#endif
 }
 
 template <int NT>
