@@ -14,7 +14,10 @@ namespace landau {
 
 // register window: each thread owns an R x C tile of the (B+1) x (B+1) active square, at most 256
 // threads per CTA: 4 x 8 tiles for B + 1 <= 88 (two CTAs per SM), 8 x 8 tiles for B + 1 <= 128
-constexpr int kBandD = 6;        // cp.async prefetch distance, in elimination steps
+#ifndef LANDAU_BAND_D
+#define LANDAU_BAND_D 6
+#endif
+constexpr int kBandD = LANDAU_BAND_D;   // cp.async prefetch distance, in elimination steps
 constexpr int kBandMaxP = 128;
 
 struct BandDesc {             // per species block
