@@ -541,7 +541,8 @@ __global__ void __launch_bounds__(256, 2) band_lu_cw_kernel(const double *__rest
 __global__ void band_solve_kernel(const double *__restrict__ LU, int64_t lu_bstride, const BandDesc *__restrict__ desc,
                                   const int32_t *__restrict__ perm_all, const int64_t *__restrict__ perm_off,
                                   const int64_t *__restrict__ vec_off, int64_t ndof, int nmax, int Bmax,
-                                  const double *__restrict__ rhs, double *__restrict__ x, int nsp, int nbatch) {
+                                  const double *__restrict__ rhs, double *__restrict__ x, int nsp, int nbatch,
+                                  const double *__restrict__ yfwd) {
   extern __shared__ double sm[];
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -556,16 +557,22 @@ __global__ void band_solve_kernel(const double *__restrict__ LU, int64_t lu_bstr
   double *xb = x + (int64_t)b * ndof + vec_off[a];
   double *y = sm + (int64_t)wib * (nmax + Bmax + 1 + (kBandD + 1) * RW);
   double *ring = y + nmax + Bmax + 1;
-  for (int i = lane; i < n + B + 1; i += 32) y[i] = i < n ? bb[perm[i]] : 0.0;   // zero pads past n
+  if (yfwd) {   // the fused factorisation already eliminated forward: y = L^-1 b (RCM order)
+    const double *yb = yfwd + (int64_t)b * ndof + vec_off[a];
+    for (int i = lane; i < n + B + 1; i += 32) y[i] = i < n ? yb[i] : 0.0;
+  } else {
+    for (int i = lane; i < n + B + 1; i += 32) y[i] = i < n ? bb[perm[i]] : 0.0;   // zero pads past n
+  }
   // forward: ring rows hold L(k+1..k+B, k) = LU[k][B+1..2B]
   auto issue_f = [&](int k) {
     if (k < n)
       for (int t = lane; t < B; t += 32) cp_async8(ring + (k % (kBandD + 1)) * RW + t, A + (int64_t)k * W + B + 1 + t);
     cp_async_commit();
   };
-  for (int k = 0; k < kBandD; k++) issue_f(k);
-  for (int k = 0; k < n; k++) {
-    issue_f(k + kBandD);
+  const int nf = yfwd ? 0 : n;   // forward steps
+  for (int k = 0; k < kBandD; k++) issue_f(k < nf ? k : n);
+  for (int k = 0; k < nf; k++) {
+    issue_f(k + kBandD < nf ? k + kBandD : n);
     cp_async_wait<kBandD>();
     __syncwarp();
     const double *row = ring + (k % (kBandD + 1)) * RW;

@@ -99,6 +99,8 @@ struct BmArgs {
   const uint16_t *ent_pos;
   int n, Bp, P, W, npan;
   double *pan0, *lfr, *ufr, *cor, *ebuf0;
+  double *bs;         // FWD: the right-hand side in RCM order (shared memory), eliminated in place
+  double *yout;       // FWD: L^-1 b (RCM order) for the backward substitution
 };
 
 // LU of the 8 x 8 corner held as a DMMA accumulator fragment (lane: row g, columns c0, c0 + 1), in
@@ -193,7 +195,7 @@ __device__ __forceinline__ void bm_shift(double (&acc)[TPW][2], const double *er
     default: CALL(7); break;         \
   }
 
-template <int NT>
+template <int NT, bool FWD>
 __device__ __forceinline__ void bm_body(const BmArgs &A) {
   constexpr BmPlan<NT> PL = bm_plan<NT>();
   constexpr int Q = 8 * NT;
@@ -277,6 +279,20 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
     double *cor = A.cor + par * 72;
     if (warp == 0 || warp == 7) {
       for (int i = (warp ? 32 : 0) + lane; i < 2 * 8 * Q; i += 64) er1[i] = 0.0;
+      if (FWD && warp == 0 && lane == 0 && p >= 0) {   // forward elimination of the panel's rows: y = L11^-1 b
+        double y[8];
+#pragma unroll
+        for (int t = 0; t < 8; t++) {
+          double v = k + t < n ? A.bs[k + t] : 0.0;
+#pragma unroll
+          for (int s2 = 0; s2 < t; s2++) v = fma(-cor[t * 8 + s2], y[s2], v);
+          y[t] = v;
+          if (k + t < n) {
+            A.bs[k + t] = v;
+            A.yout[k + t] = v;
+          }
+        }
+      }
     } else if (p >= 0) {
       {
         if (warp <= 3) {   // L21 = A21 U11^-1: window row r = 8 + (tid - 32)
@@ -329,11 +345,22 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
 #define BM_UPD(w) bm_update<NT, w, TPW>(acc, A.lfr, A.ufr, lane, cnext)
       BM_SWITCH(BM_UPD)
 #undef BM_UPD
-      // factor row k + warp: (U(t, t), U(t, t+1 .. t+Bp), L(t+1 .. t+Bp, t)) in window coordinates
+      if (FWD && warp >= 1 && warp <= 3) {   // b(rows below the panel) -= L21 y
+        const int r = 8 + tid - 32;
+        if (r < Q && k + r < n) {
+          const double *row = colp + (r >> 3) * kBmTS + (r & 7) * 9;
+          double v = A.bs[k + r];
+#pragma unroll
+          for (int c = 0; c < 8; c++) v = fma(-row[c], k + c < n ? A.bs[k + c] : 0.0, v);
+          A.bs[k + r] = v;
+        }
+      }
+      // factor row k + warp: (U(t, t), U(t, t+1 .. t+Bp), L(t+1 .. t+Bp, t)) in window coordinates; with
+      // FWD the L part is not needed (the forward elimination is done) and not written
       const int t = warp;
       if (k + t < n) {
         double *out = A.lu + (int64_t)(k + t) * W;
-        for (int s = lane; s < W; s += 32) {
+        for (int s = lane; s < (FWD ? Bp + 1 : W); s += 32) {
           double v;
           if (s == 0) {
             v = cor[t * 9];
@@ -365,13 +392,21 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
 #endif
 }
 
-template <int NT>
+// FWD (the implicit step): also eliminate the right-hand side rhs [batch][ndof] (species blocks at
+// vec_off, original order; perm maps RCM -> original) and write y = L^-1 b (RCM order) to yout in the
+// same layout; only the U part of the factor rows is written, for band_solve_kernel's backward pass
+template <int NT, bool FWD>
 __global__ void __launch_bounds__(32 * kBmWarps, NT <= 12 ? 2 : 1) band_lu_mma_kernel(const double *__restrict__ Aent,
                                                                                   int64_t ent_bstride,
                                                                                   double *__restrict__ LU,
                                                                                   int64_t lu_bstride,
                                                                                   const BandDesc *__restrict__ desc,
-                                                                                  int nsp) {
+                                                                                  int nsp, const double *__restrict__ rhs,
+                                                                                  double *__restrict__ yout,
+                                                                                  const int32_t *__restrict__ perm_all,
+                                                                                  const int64_t *__restrict__ perm_off,
+                                                                                  const int64_t *__restrict__ vec_off,
+                                                                                  int64_t ndof) {
   extern __shared__ double smem[];
   const int bi = blockIdx.x / nsp, sp = blockIdx.x % nsp;
   const BandDesc d = desc[sp];
@@ -390,7 +425,16 @@ __global__ void __launch_bounds__(32 * kBmWarps, NT <= 12 ? 2 : 1) band_lu_mma_k
   A.ufr = A.lfr + NT * 64;
   A.cor = A.ufr + NT * 64;
   A.ebuf0 = A.cor + 2 * 72;
-  bm_body<NT>(A);
+  A.bs = A.ebuf0 + 4 * 8 * 8 * NT;
+  A.yout = nullptr;
+  if (FWD) {
+    const int32_t *perm = perm_all + perm_off[sp];
+    const double *bb = rhs + (int64_t)bi * ndof + vec_off[sp];
+    for (int i = threadIdx.x; i < d.n; i += blockDim.x) A.bs[i] = bb[perm[i]];
+    A.yout = yout + (int64_t)bi * ndof + vec_off[sp];
+    // (bm_body's prologue barrier orders these loads before the first use)
+  }
+  bm_body<NT, FWD>(A);
 }
 
 }  // namespace landau

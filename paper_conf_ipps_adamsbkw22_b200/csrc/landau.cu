@@ -144,6 +144,9 @@ struct landau_s {
   int64_t *d_perm_off = nullptr, *d_vec_off = nullptr;
   int64_t band_bstride = 0, band_cap = 0, band_nbatch = 0;
   double *d_band = nullptr;   // step-major LU factors [batch][band_bstride] (kernels_band.cuh)
+  double *d_yfwd = nullptr;   // forward-eliminated right-hand side of the fused factorisation [batch][ndof]
+  int64_t yfwd_cap = 0;
+  bool band_fwd_done = false; // the last factorisation eliminated the rhs and stored U only
   // host staging for landau_jacobian_host: full-batch device buffers, two copy streams
   double *d_vals_tmp = nullptr;
   int64_t vals_tmp_cap = 0;
@@ -1352,6 +1355,7 @@ void landau_destroy(landau_t h) {
   cudaFree(h->d_perm_off);
   cudaFree(h->d_vec_off);
   cudaFree(h->d_band);
+  cudaFree(h->d_yfwd);
   if (h->s_h2d) cudaStreamDestroy(h->s_h2d);
   if (h->s_d2h) cudaStreamDestroy(h->s_d2h);
   for (auto e : h->ev_h2d) cudaEventDestroy(e);
@@ -1753,8 +1757,11 @@ int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const d
 });
 }
 
-int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, double Ez, const double *J_csr_dev) {
-  return guarded(h, [&]() -> int {
+// The band factorisation; with rhs (the implicit step, DMMA kernel only) the kernel also eliminates rhs
+// forward into d_yfwd and writes only the U part of the factor (band_fwd_done: only the backward pass of
+// the solve remains, see band_solve_impl).  Returns LANDAU_EUNSUPPORTED (nothing launched) when rhs is
+// given and the DMMA kernel does not apply.
+int band_factor_impl(landau_t h, int64_t nbatch, double shift, double Ez, const double *J_csr_dev, const double *rhs) {
   if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
   if (!h || nbatch < 1 || !J_csr_dev) return fail(h, LANDAU_EINVAL, "band_factor: bad argument");
   int maxPp = 8, maxn = 0, maxent = 0;
@@ -1821,21 +1828,34 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
     const char *e = getenv("LANDAU_BAND_MMA");
     return !(e && atoi(e) == 0);
   }();
-#define BM(NT) (const void *)band_lu_mma_kernel<NT>
+#define BM(NT) (const void *)band_lu_mma_kernel<NT, false>
+#define BF(NT) (const void *)band_lu_mma_kernel<NT, true>
   static const void *const mma_kernels[18] = {nullptr, nullptr, nullptr, BM(3),  BM(4),  BM(5),  BM(6),  BM(7),  BM(8),
                                               BM(9),   BM(10),  BM(11),  BM(12), BM(13), BM(14), BM(15), BM(16), BM(17)};
+  static const void *const mma_kernels_fwd[18] = {nullptr, nullptr, nullptr, BF(3),  BF(4),  BF(5),  BF(6),
+                                                  BF(7),   BF(8),   BF(9),   BF(10), BF(11), BF(12), BF(13),
+                                                  BF(14),  BF(15),  BF(16),  BF(17)};
 #undef BM
+#undef BF
   const int mma_nt = maxPp / 8 + 1;
+  const bool mma_ok = band_mma && same_p && maxPp % 8 == 0 && mma_nt >= 3 && mma_nt <= 17 &&
+                      h->band_ent_max <= kBmE * 32 * kBmWarps;
+  if (rhs && (band_cw || !mma_ok)) return LANDAU_EUNSUPPORTED;
+  if (rhs && nbatch > h->yfwd_cap) {
+    cudaFree(h->d_yfwd);
+    h->d_yfwd = nullptr;
+    CU(cudaMalloc(&h->d_yfwd, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
+    h->yfwd_cap = nbatch;
+  }
   if (band_cw && same_p && maxPp <= 96 && maxPp % 8 == 0 && h->band_ent_max <= kBandE * 256) {
     // column-warp kernel with look-ahead: 8 warps of P / 8 columns (one window width per launch)
     kfn = cw_kernels[maxPp / 8 - 1];
     ksmem = sizeof(double) * (2 * kCwRing + 48) * maxPp;
     threads = 256;
-  } else if (band_mma && same_p && maxPp % 8 == 0 && mma_nt >= 3 && mma_nt <= 17 &&
-             h->band_ent_max <= kBmE * 32 * kBmWarps) {
+  } else if (mma_ok) {
     // blocked factorisation, DMMA trailing updates (kernels_band_mma.cuh): C4 2.0 ms vs 3.2 ms
-    kfn = mma_kernels[mma_nt];
-    ksmem = sizeof(double) * band_mma_smem_doubles(mma_nt);
+    kfn = rhs ? mma_kernels_fwd[mma_nt] : mma_kernels[mma_nt];
+    ksmem = sizeof(double) * (band_mma_smem_doubles(mma_nt) + (rhs ? maxn : 0));
     threads = 32 * kBmWarps;
   } else if (maxPp <= 88)   // 4 x 8 tiles, <= 242 threads; two CTAs per SM (128 registers) or one
     kfn = band_minb >= 2 ? (const void *)band_lu2_kernel<4, 8, 2> : (const void *)band_lu2_kernel<4, 8, 1>;
@@ -1850,22 +1870,34 @@ int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, d
     int64_t a3 = h->band_bstride;
     const BandDesc *a4 = h->d_band_desc;
     int a5 = h->S;
-    void *args[] = {&a0, &a1, &a2, &a3, &a4, &a5};
+    const double *a6 = rhs;
+    double *a7 = h->d_yfwd;
+    const int32_t *a8 = h->d_perm_all;
+    const int64_t *a9 = h->d_perm_off, *a10 = h->d_vec_off;
+    int64_t a11 = h->ndof;
+    void *args[] = {&a0, &a1, &a2, &a3, &a4, &a5, &a6, &a7, &a8, &a9, &a10, &a11};
+    // (the register-tile and column-warp kernels take the first six arguments)
     CU(cudaLaunchKernel(kfn, dim3(grid), dim3(threads), args, ksmem, h->stream));
   }
   h->launches++;
   h->tlaunch[LANDAU_T_FACTOR]++;
   KCHECK();
   h->band_nbatch = nbatch;
+  h->band_fwd_done = rhs != nullptr;
   return LANDAU_OK;
-});
 }
 
-int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev) {
-  return guarded(h, [&]() -> int {
+int landau_band_factor_field_batched(landau_t h, int64_t nbatch, double shift, double Ez, const double *J_csr_dev) {
+  return guarded(h, [&]() -> int { return band_factor_impl(h, nbatch, shift, Ez, J_csr_dev, nullptr); });
+}
+
+// yfwd: the fused factorisation's forward-eliminated rhs (backward pass only); else b_dev is solved fully
+int band_solve_impl(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev, const double *yfwd) {
   if (h && h->host_only) return fail(h, LANDAU_EUNSUPPORTED, "host-only handle");
-  if (!h || nbatch < 1 || !b_dev || !x_dev) return fail(h, LANDAU_EINVAL, "band_solve: bad argument");
+  if (!h || nbatch < 1 || (!b_dev && !yfwd) || !x_dev) return fail(h, LANDAU_EINVAL, "band_solve: bad argument");
   if (h->band_nbatch != nbatch) return fail(h, LANDAU_ESTATE, "band_solve: factor this batch first");
+  if (h->band_fwd_done != (yfwd != nullptr))
+    return fail(h, LANDAU_ESTATE, "band_solve: the last factorisation was the implicit step's fused one; factor again");
   Timer t(h, LANDAU_T_SOLVE);
   int maxn = 0, maxB = 0;
   for (auto &d : h->band_desc) maxn = std::max(maxn, d.n), maxB = std::max(maxB, d.B);
@@ -1875,12 +1907,15 @@ int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, d
   const int64_t warps = nbatch * h->S;
   band_solve_kernel<<<(unsigned)((warps + kWarps - 1) / kWarps), 32 * kWarps, smem, h->stream>>>(
       h->d_band, h->band_bstride, h->d_band_desc, h->d_perm_all, h->d_perm_off, h->d_vec_off, h->ndof, maxn, maxB,
-      b_dev, x_dev, h->S, (int)nbatch);
+      b_dev, x_dev, h->S, (int)nbatch, yfwd);
   h->launches++;
   h->tlaunch[LANDAU_T_SOLVE]++;
   KCHECK();
   return LANDAU_OK;
-});
+}
+
+int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev) {
+  return guarded(h, [&]() -> int { return band_solve_impl(h, nbatch, b_dev, x_dev, nullptr); });
 }
 
 int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
@@ -1943,8 +1978,23 @@ int landau_implicit_step_source_batched(landau_t h, int64_t nbatch, double dt, d
     // (M/dt + E_z (e/m) A_E - J(f^k)) f^{k+1} = M f_old / dt  by the band LU
     int rc = landau_set_state_batched(h, nbatch, f_new_dev);
     if (!rc) rc = dispatch_build(h, nbatch, h->d_Jwork, LANDAU_CSR);
-    if (!rc) rc = landau_band_factor_field_batched(h, nbatch, 1.0 / dt, Ez, h->d_Jwork);
-    if (!rc) rc = landau_band_solve_batched(h, nbatch, h->d_rhs, f_new_dev);
+    // the fused factorisation (rhs eliminated forward inside the DMMA kernel, U stored alone) where it
+    // applies (LANDAU_BAND_FUSED=0: factor + full solve)
+    static const bool fused = [] {
+      const char *e = getenv("LANDAU_BAND_FUSED");
+      return !(e && atoi(e) == 0);
+    }();
+    if (!rc) {
+      const int rf = fused ? band_factor_impl(h, nbatch, 1.0 / dt, Ez, h->d_Jwork, h->d_rhs) : LANDAU_EUNSUPPORTED;
+      if (rf == LANDAU_OK) {
+        rc = band_solve_impl(h, nbatch, nullptr, f_new_dev, h->d_yfwd);
+      } else if (rf == LANDAU_EUNSUPPORTED) {
+        rc = band_factor_impl(h, nbatch, 1.0 / dt, Ez, h->d_Jwork, nullptr);
+        if (!rc) rc = band_solve_impl(h, nbatch, h->d_rhs, f_new_dev, nullptr);
+      } else {
+        rc = rf;
+      }
+    }
     if (rc) return rc;
     delta_norm_kernel<<<(unsigned)nbatch, 256, 0, h->stream>>>(f_new_dev, h->d_f, h->ndof, h->d_norms);
     h->launches++;

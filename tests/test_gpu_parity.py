@@ -1249,3 +1249,51 @@ def test_jacobian3d_matches_oracle(ncell, order):
     torch.cuda.synchronize()
     assert torch.equal(J, J2)
     h.close()
+
+
+_STEP_CHILD = r'''
+import os, sys, numpy as np, torch
+sys.path.insert(0, os.getcwd())
+from paper_conf_ipps_adamsbkw22_b200 import inputs
+from paper_conf_ipps_adamsbkw22_b200 import landau as L
+path, nb = sys.argv[1], int(sys.argv[2])
+h = L.Landau.from_problem(inputs.config4_vertex(0), device=0)
+nodes = h.all_nodes()
+F = torch.tensor(np.stack([inputs.coefficients(inputs.config4_vertex(b), nodes) for b in range(0, 1024, 1024 // nb)]),
+                 device="cuda")
+Src = torch.tensor(np.stack([inputs.quench_source_shape(inputs.config4_vertex(b), nodes)
+                             for b in range(0, 1024, 1024 // nb)]), device="cuda")
+Fn = torch.empty_like(F)
+h.implicit_step_batched(0.002, F, Fn, Ez=0.1, max_iter=3, src=Src)
+state = "ok"
+try:   # the fused factorisation stored U only: the public solve must refuse it
+    h.band_solve_batched(F, torch.empty_like(F))
+    state = "solved"
+except Exception as e:
+    state = type(e).__name__ + ":" + str(e)[:80]
+np.savez(path, f=Fn.cpu().numpy(), state=np.array(state))
+'''
+
+
+def test_implicit_step_fused_forward_elimination():
+    """The implicit step's fused factorisation (the DMMA band kernel also eliminates the right-hand side
+    forward and stores U alone; the solve runs only the backward pass) gives the same iterates as the
+    separate factor + full solve (LANDAU_BAND_FUSED=0), up to rounding; after a fused factorisation the
+    public band solve refuses to run (LANDAU_ESTATE), since the L factor was not stored."""
+    import os
+    import subprocess
+    import sys
+    import tempfile
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = {}
+    with tempfile.TemporaryDirectory() as td:
+        for fused in ("1", "0"):
+            path = os.path.join(td, f"f{fused}.npz")
+            out = subprocess.run([sys.executable, "-c", _STEP_CHILD, path, "8"], capture_output=True, text=True,
+                                 timeout=600, cwd=root, env=dict(os.environ, LANDAU_BAND_FUSED=fused))
+            assert out.returncode == 0, out.stderr[-3000:]
+            res[fused] = dict(np.load(path))
+    a, b = res["1"]["f"], res["0"]["f"]
+    assert np.max(np.abs(a - b)) <= 1e-11 * np.max(np.abs(b))
+    assert "(-5)" in str(res["1"]["state"])   # LANDAU_ESTATE
+    assert str(res["0"]["state"]) == "solved"
