@@ -196,7 +196,8 @@ int landau_set_tensor_cache(landau_t h, int32_t enable);
  *   landau_band_info:      B and the RCM permutation perm[new] = old of one grid (host, may be NULL)
  *   landau_band_factor_batched: J_csr_dev = [nbatch][nnz_csr] (e.g. from landau_jacobian_batched)
  *   landau_band_solve_batched:  b_dev, x_dev = [nbatch][ndof] species-major (may alias); uses the
- *                          last factorisation (ESTATE before any, or when nbatch differs) */
+ *                          last factorisation (ESTATE before any, when nbatch differs, or after an
+ *                          implicit step, whose fused factorisation keeps only U -- factor again) */
 int landau_band_info(landau_t h, int32_t grid, int32_t *bandwidth, int32_t *perm);
 int landau_band_factor_batched(landau_t h, int64_t nbatch, double shift, const double *J_csr_dev);
 int landau_band_solve_batched(landau_t h, int64_t nbatch, const double *b_dev, double *x_dev);
@@ -220,7 +221,11 @@ int landau_advection(landau_t h, double Ez, double *values_dev, int32_t format);
  * ||f^{k+1} - f^k|| / ||f^{k+1}|| <= rtol (rtol > 0 reads the norms back once per iteration; rtol <= 0
  * runs exactly max_iter iterations with one read-back at the end).  iters (host, may be NULL): the
  * iterations run; dnorm (host, may be NULL): the largest relative change of the last iteration.
- * The handle's state afterwards is the last iterate f^{k} the final Jacobian was built about. */
+ * The handle's state afterwards is the last iterate f^{k} the final Jacobian was built about.
+ * Where the blocked (DMMA) band kernel applies, each iteration's factorisation also eliminates the
+ * right-hand side forward and stores only U (the solve then runs the backward pass alone); env
+ * LANDAU_BAND_FUSED=0 selects factor + full solve.  Either way the band factor held afterwards is the
+ * last iteration's. */
 int landau_implicit_step_batched(landau_t h, int64_t nbatch, double dt, double Ez, const double *f_old_dev,
                                  double *f_new_dev, int32_t max_iter, double rtol, int32_t *iters, double *dnorm);
 /* The same step with the source term S_a(t) of Eq. 1 / Eq. 4 (PAPER.md:1@6337, @8216; the thermal-quench
