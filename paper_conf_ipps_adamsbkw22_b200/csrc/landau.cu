@@ -1838,14 +1838,49 @@ int band_factor_impl(landau_t h, int64_t nbatch, double shift, double Ez, const 
 #undef BM
 #undef BF
   const int mma_nt = maxPp / 8 + 1;
-  const bool mma_ok = band_mma && same_p && maxPp % 8 == 0 && mma_nt >= 3 && mma_nt <= 17 &&
-                      h->band_ent_max <= kBmE * 32 * kBmWarps;
-  if (rhs && (band_cw || !mma_ok)) return LANDAU_EUNSUPPORTED;
+  // the DMMA kernel applies to every species block (window NT = P/8 + 1 tiles per side, 3..17); blocks
+  // of different bandwidth (separate grids, C3) are factored by one launch per species
+  bool mma_all = band_mma && h->band_ent_max <= kBmE * 32 * kBmWarps;
+  for (auto &d : h->band_desc) mma_all = mma_all && d.Pp % 8 == 0 && d.Pp / 8 + 1 >= 3 && d.Pp / 8 + 1 <= 17;
+  const bool mma_ok = mma_all && same_p;
+  if (rhs && (band_cw || !mma_all)) return LANDAU_EUNSUPPORTED;
   if (rhs && nbatch > h->yfwd_cap) {
     cudaFree(h->d_yfwd);
     h->d_yfwd = nullptr;
     CU(cudaMalloc(&h->d_yfwd, sizeof(double) * nbatch * std::max<int64_t>(h->ndof, 1)));
     h->yfwd_cap = nbatch;
+  }
+  static const bool per_species = [] {   // test knob: the per-species launches even for equal bands
+    const char *e = getenv("LANDAU_BAND_PER_SPECIES");
+    return e && atoi(e) != 0;
+  }();
+  if (mma_all && (!same_p || per_species) && !band_cw) {   // one DMMA launch per species block (its own window)
+    for (int a = 0; a < h->S; a++) {
+      const int nt = h->band_desc[a].Pp / 8 + 1;
+      const void *kf = rhs ? mma_kernels_fwd[nt] : mma_kernels[nt];
+      const size_t sm = sizeof(double) * (band_mma_smem_doubles(nt) + (rhs ? h->band_desc[a].n : 0));
+      if (sm > 200 * 1024) return fail(h, LANDAU_EUNSUPPORTED, "band factor: grid too large for one CTA");
+      if (sm > 48 * 1024) CU(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+      const double *a0 = h->d_Aent;
+      int64_t a1 = h->ent_bstride;
+      double *a2 = h->d_band;
+      int64_t a3 = h->band_bstride;
+      const BandDesc *a4 = h->d_band_desc + a;   // nsp = 1: this block only
+      int a5 = 1;
+      const double *a6 = rhs;
+      double *a7 = h->d_yfwd;
+      const int32_t *a8 = h->d_perm_all;
+      const int64_t *a9 = h->d_perm_off + a, *a10 = h->d_vec_off + a;
+      int64_t a11 = h->ndof;
+      void *args[] = {&a0, &a1, &a2, &a3, &a4, &a5, &a6, &a7, &a8, &a9, &a10, &a11};
+      CU(cudaLaunchKernel(kf, dim3((unsigned)nbatch), dim3(32 * kBmWarps), args, sm, h->stream));
+      h->launches++;
+      KCHECK();
+    }
+    h->tlaunch[LANDAU_T_FACTOR]++;
+    h->band_nbatch = nbatch;
+    h->band_fwd_done = rhs != nullptr;
+    return LANDAU_OK;
   }
   if (band_cw && same_p && maxPp <= 96 && maxPp % 8 == 0 && h->band_ent_max <= kBandE * 256) {
     // column-warp kernel with look-ahead: 8 warps of P / 8 columns (one window width per launch)

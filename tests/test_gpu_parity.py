@@ -1297,3 +1297,47 @@ def test_implicit_step_fused_forward_elimination():
     assert np.max(np.abs(a - b)) <= 1e-11 * np.max(np.abs(b))
     assert "(-5)" in str(res["1"]["state"])   # LANDAU_ESTATE
     assert str(res["0"]["state"]) == "solved"
+
+
+_C3_STEP_CHILD = r'''
+import os, sys, numpy as np, torch
+sys.path.insert(0, os.getcwd())
+from paper_conf_ipps_adamsbkw22_b200 import inputs
+from paper_conf_ipps_adamsbkw22_b200 import landau as L
+path = sys.argv[1]
+p = inputs.CONFIGS["C3"]()
+h = L.Landau.from_problem(p, device=0)
+f = torch.tensor(np.stack([inputs.coefficients(p, h.all_nodes())] * 3), device="cuda")
+fn = torch.empty_like(f)
+h.implicit_step_batched(0.01, f, fn, Ez=0.05, max_iter=2)
+J = torch.empty((3, h.nnz), dtype=torch.float64, device="cuda")
+h.set_state_batched(f)
+h.jacobian_batched(J)
+h.band_factor_batched(50.0, J)
+x = torch.empty_like(f)
+h.band_solve_batched(f, x)
+np.savez(path, fn=fn.cpu().numpy(), x=x.cpu().numpy())
+'''
+
+
+def test_band_per_species_launches_match():
+    """Species blocks on grids of different bandwidth are factored by one DMMA launch per species (each
+    with its own window size); forced on a C3 problem (LANDAU_BAND_PER_SPECIES=1: three grids, one
+    launch each) it gives the same implicit-step iterates and band solutions as the single launch over
+    all blocks, up to rounding."""
+    import os
+    import subprocess
+    import sys
+    import tempfile
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    res = {}
+    with tempfile.TemporaryDirectory() as td:
+        for ps in ("0", "1"):
+            path = os.path.join(td, f"p{ps}.npz")
+            out = subprocess.run([sys.executable, "-c", _C3_STEP_CHILD, path], capture_output=True, text=True,
+                                 timeout=600, cwd=root, env=dict(os.environ, LANDAU_BAND_PER_SPECIES=ps))
+            assert out.returncode == 0, out.stderr[-3000:]
+            res[ps] = dict(np.load(path))
+    for k in ("fn", "x"):
+        a, b = res["1"][k], res["0"][k]
+        assert np.max(np.abs(a - b)) <= 1e-12 * np.max(np.abs(b)), k
