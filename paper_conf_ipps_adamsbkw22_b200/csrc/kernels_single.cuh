@@ -18,6 +18,12 @@
 namespace landau {
 
 constexpr int kSbWarps = 8;   // 256 threads per CTA, one CTA per SM
+#ifndef LANDAU_SB_FOLD_REDUCE
+#define LANDAU_SB_FOLD_REDUCE 1
+#endif
+// a-2r folded into a-4: each element warp sums its points' group partials itself (same order as the
+// reduction phase, so bitwise the same G), which saves that phase and one grid barrier
+constexpr bool kSbFoldReduce = LANDAU_SB_FOLD_REDUCE != 0;
 
 struct SingleBuildArgs {
   // a-1
@@ -36,6 +42,7 @@ struct SingleBuildArgs {
   int nsplit;
   const double *rU, *zU;
   const int32_t *pu, *pm;
+  const int32_t *pinv;   // point -> ut (+ H for the mirror point pm[ut])
   double *G, *part;
   // a-4 element buffer, a-5 gather maps (one per grid) and output
   double *Cbuf;
@@ -216,7 +223,7 @@ __global__ void __launch_bounds__(32 * kSbWarps, 1) single_build_kernel(const Si
   // ---- a-2r: the groups' partials summed in group order (one thread per (b, component, point)) ----
   {
     const int64_t N = a.npts, Hp = a.T * 32, ngroups = (a.nsplit + kSbWarps - 1) / kSbWarps;
-    if (ngroups > 1 && !(LANDAU_SB_SKIP & 4)) {
+    if (ngroups > 1 && !(LANDAU_SB_SKIP & 4) && !kSbFoldReduce) {
       const int64_t total = (int64_t)a.nbatch * 10 * a.H;
       for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
         const int64_t b = k / (10 * a.H), c = (k / a.H) % 10, ut = k % a.H;
@@ -243,9 +250,23 @@ __global__ void __launch_bounds__(32 * kSbWarps, 1) single_build_kernel(const Si
       if (lane < NB) {
         const int64_t i = e * NB + lane;
         const double w = a.pw[i];
-        const double *Gb = a.G + b * 5 * N + i;
+        const int64_t Hp = a.T * 32, ngroups = (a.nsplit + kSbWarps - 1) / kSbWarps;
+        if (kSbFoldReduce && ngroups > 1) {   // a-2r here: the groups' partials of this point, in group order
+          const int32_t pv = a.pinv[i];
+          const bool mir = pv >= a.H;
+          const int64_t ut = mir ? pv - a.H : pv;
 #pragma unroll
-        for (int c = 0; c < 5; c++) u.el.A[wid][c][lane] = w * Gb[c * N];
+          for (int c = 0; c < 5; c++) {
+            const int cc = mir ? c + 5 : c;
+            double acc = 0.0;
+            for (int64_t g = 0; g < ngroups; g++) acc += __ldcg(a.part + ((b * ngroups + g) * 10 + cc) * Hp + ut);
+            u.el.A[wid][c][lane] = w * ((mir && (c == 1 || c == 4)) ? -acc : acc);
+          }
+        } else {
+          const double *Gb = a.G + b * 5 * N + i;
+#pragma unroll
+          for (int c = 0; c < 5; c++) u.el.A[wid][c][lane] = w * Gb[c * N];
+        }
       }
       __syncwarp();
       sf_cell<S>(u.el.A[wid], u.el.T[wid], lane, PLL, PLD, PDL, PDD, 2.0 / a.cell_h[e],

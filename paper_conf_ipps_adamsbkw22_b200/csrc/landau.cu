@@ -119,6 +119,7 @@ struct landau_s {
   int64_t vtx_cnt_cap = 0;
   double *d_rU = nullptr, *d_zU = nullptr;
   int32_t *d_pu = nullptr, *d_pm = nullptr;
+  int32_t *d_pinv = nullptr;   // point -> upper-half index (+ H for a mirror point): the fused build's a-4
   // slot-kernel item sets: [0] one i-tile per item (fine-grained: small batches), [1] runs of up to
   // LANDAU_MIR_RUN i-tiles per j-tile (fewer slots and stagings: large work, e.g. C5)
   struct MirSet {
@@ -986,6 +987,7 @@ int launch_single(landau_t h, int64_t nbatch, const InnerPlan &ip, double *out, 
     a.zU = h->d_zU;
     a.pu = h->d_pu;
     a.pm = h->d_pm;
+    a.pinv = h->d_pinv;
     a.G = h->d_G;
     a.part = h->d_part;
     a.Cbuf = h->d_C;
@@ -1370,6 +1372,7 @@ void landau_destroy(landau_t h) {
   cudaFree(h->d_rU);
   cudaFree(h->d_zU);
   cudaFree(h->d_pu);
+  cudaFree(h->d_pinv);
   cudaFree(h->d_pm);
   for (auto &ms : h->mset) {
     cudaFree(ms.items);
@@ -2372,8 +2375,14 @@ static int create_impl(landau_t &h, landau_t *out, const landau_mesh_t *mesh, co
       }
       h->mirror = true;
       h->H = H;
+      // inverse mirror map: point -> upper-half index ut, + H when the point is the mirror pm[ut]
+      std::vector<int32_t> pinv(P.npts, -1);
+      for (int64_t u = 0; u < H; u++) {
+        pinv[pu[u]] = (int32_t)u;
+        pinv[pm[u]] = (int32_t)(u + H);
+      }
       if ((rc = upload(h, &h->d_rU, rU)) || (rc = upload(h, &h->d_zU, zU)) || (rc = upload(h, &h->d_pu, pu)) ||
-          (rc = upload(h, &h->d_pm, pm)))
+          (rc = upload(h, &h->d_pm, pm)) || (rc = upload(h, &h->d_pinv, pinv)))
         return bail(rc);
       if (world > 1) {   // pair split: every rank targets every point, G summed by an all-reduce
         h->dist_pairs = true;
