@@ -89,7 +89,7 @@ __device__ __forceinline__ void bm_for_diags(F &&f) {
 // shared memory (doubles): panels [2 parities][2][NT][72], fragments of -L21 and U12 [2][NT][2][32],
 // factored corner (64) + pivot reciprocals (8) [2 parities], entering buffers [2 parities][2][8][8 NT]
 __host__ __device__ constexpr int band_mma_smem_doubles(int NT) {
-  return 4 * NT * kBmTS + 2 * NT * 64 + 2 * 72 + 4 * 8 * 8 * NT;
+  return 4 * NT * kBmTS + 2 * NT * 64 + 2 * 72 + 4 * 8 * 8 * NT + 64;
 }
 
 struct BmArgs {
@@ -99,6 +99,7 @@ struct BmArgs {
   const uint16_t *ent_pos;
   int n, Bp, P, W, npan;
   double *pan0, *lfr, *ufr, *cor, *ebuf0;
+  double *cin;        // the next corner tile handed from warp 0 to the corner warp (fragment order)
   double *bs;         // FWD: the right-hand side in RCM order (shared memory), eliminated in place
   double *yout;       // FWD: L^-1 b (RCM order) for the backward substitution
 };
@@ -141,7 +142,7 @@ __device__ __forceinline__ void bm_publish(double (&acc)[TPW][2], double *colp, 
 }
 template <int NT, int WID, int TPW>
 __device__ __forceinline__ void bm_update(double (&acc)[TPW][2], const double *lfr, const double *ufr, int lane,
-                                          double *cnext) {
+                                          double *cnext, double *cin) {
   bm_for_diags<NT, WID>([&](auto dc, auto mc) {
     constexpr int d = decltype(dc)::value, m0 = decltype(mc)::value;
     constexpr int len = NT - (d < 0 ? -d : d), I0 = d < 0 ? -d : 0, J0 = d > 0 ? d : 0;
@@ -149,7 +150,12 @@ __device__ __forceinline__ void bm_update(double (&acc)[TPW][2], const double *l
     if constexpr (d == 0) {   // look-ahead: update tile (1, 1) first and factor it -- the next corner
       dmma_8x8x4(acc[m0 + 1][0], acc[m0 + 1][1], lfr[64 + lane], ufr[64 + lane]);
       dmma_8x8x4(acc[m0 + 1][0], acc[m0 + 1][1], lfr[96 + lane], ufr[96 + lane]);
-      if (cnext) bm_corner_lu(acc[m0 + 1][0], acc[m0 + 1][1], cnext, lane);
+      if (cnext) {   // hand the updated tile to the corner warp, which factors it (bm_corner_warp)
+        cin[2 * lane] = acc[m0 + 1][0];
+        cin[2 * lane + 1] = acc[m0 + 1][1];
+        __threadfence_block();
+        asm volatile("bar.arrive 2, 64;" ::: "memory");
+      }
     }
 #pragma unroll
     for (int i = i0; i < len; i++) {
@@ -342,9 +348,14 @@ __device__ __forceinline__ void bm_body(const BmArgs &A) {
     // ---- C: rank-8 trailing update of the tiles with I, J >= 1 (all but the first of each diagonal)
     if (p >= 0) {
     double *cnext = p + 1 < A.npan ? A.cor + (par ^ 1) * 72 : nullptr;
-#define BM_UPD(w) bm_update<NT, w, TPW>(acc, A.lfr, A.ufr, lane, cnext)
+#define BM_UPD(w) bm_update<NT, w, TPW>(acc, A.lfr, A.ufr, lane, cnext, A.cin)
       BM_SWITCH(BM_UPD)
 #undef BM_UPD
+      if (cnext && warp == kBmWarps - 1) {   // the corner warp (one of the lightest): next panel's corner LU
+        asm volatile("bar.sync 2, 64;" ::: "memory");
+        double v0 = A.cin[2 * lane], v1 = A.cin[2 * lane + 1];
+        bm_corner_lu(v0, v1, cnext, lane);
+      }
       if (FWD && warp >= 1 && warp <= 3) {   // b(rows below the panel) -= L21 y
         const int r = 8 + tid - 32;
         if (r < Q && k + r < n) {
@@ -425,7 +436,8 @@ __global__ void __launch_bounds__(32 * kBmWarps, NT <= 12 ? 2 : 1) band_lu_mma_k
   A.ufr = A.lfr + NT * 64;
   A.cor = A.ufr + NT * 64;
   A.ebuf0 = A.cor + 2 * 72;
-  A.bs = A.ebuf0 + 4 * 8 * 8 * NT;
+  A.cin = A.ebuf0 + 4 * 8 * 8 * NT;
+  A.bs = A.cin + 64;
   A.yout = nullptr;
   if (FWD) {
     const int32_t *perm = perm_all + perm_off[sp];
